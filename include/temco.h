@@ -1,0 +1,175 @@
+/*
+ * temco.h -- C ABI of the B200-native TeMCO inference path.
+ *
+ * TeMCO (Song et al., ICPP '24; PAPER.md = /root/reference/PAPER.md, cited as
+ * P:L<line>) takes "an ordered tensor node list L in SSA form" (Alg. 1 input,
+ * P:L180) of a tensor-decomposed CNN and produces an optimized list whose
+ * inference uses only reduced tensors:
+ *   - skip connections carry the reduced tensor, the restore layers are copied
+ *     before the far uses (Alg. 1/2);
+ *   - lconv -> activation (-> pooling) -> fconv run as one fused kernel
+ *     (P:L265-311), extended through concatenations and adds by the layer
+ *     transformations of P:L321-333.
+ * The three calls the north star names are temco_plan_create (layer graph,
+ * decomposition ranks/factors, skip edges), temco_run (plan, input, output,
+ * stream) and temco_peak_internal_bytes (Eq. (3)/(4) accounting).
+ *
+ * Conventions
+ *  - Every function returns temco_status (0 = OK); no C++ exception crosses
+ *    the ABI.  temco_last_error() gives a thread-local message for the last
+ *    failure of the calling thread.
+ *  - Host arrays passed to temco_plan_create are BORROWED for the duration of
+ *    the call and copied; the caller may free them on return.
+ *  - A plan OWNS its device weights (BN-folded, packed, plan dtype), its
+ *    activation arena, TMA descriptors and (optionally) a captured CUDA graph.
+ *  - A plan is bound to the CUDA device current at create time; temco_run from
+ *    another current device returns TEMCO_ERR_DEVICE_MISMATCH.
+ *  - temco_run is stream-ordered and asynchronous: no host synchronisation, no
+ *    allocation.  A plan is NOT re-entrant (one run in flight per plan; the
+ *    arena is shared).  Launch errors surface at return, asynchronous faults at
+ *    the caller's next synchronisation.
+ *  - There is no CPU fallback: without a device every compute call fails with
+ *    TEMCO_ERR_NO_DEVICE (plans created with TEMCO_FLAG_NO_DEVICE support the
+ *    host-only queries: peak bytes and describe).
+ */
+#ifndef TEMCO_H
+#define TEMCO_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct temco_plan_s* temco_plan_t;
+/* identical to cudaStream_t (struct CUstream_st*); NULL = legacy default stream */
+typedef struct CUstream_st* temco_stream_t;
+
+typedef enum {
+  TEMCO_OK = 0,
+  TEMCO_ERR_INVALID_ARGUMENT = 1, /* NULL pointer, bad enum, non-positive size            */
+  TEMCO_ERR_INVALID_GRAPH = 2,    /* non-topological inputs, shape mismatch, skip edges   */
+  TEMCO_ERR_UNSUPPORTED = 3,      /* op / rank / layout outside the supported set         */
+  TEMCO_ERR_OUT_OF_MEMORY = 4,    /* device or host allocation failed                     */
+  TEMCO_ERR_CUDA = 5,             /* a CUDA runtime / driver call failed                  */
+  TEMCO_ERR_DEVICE_MISMATCH = 6,  /* current device differs from the plan's device        */
+  TEMCO_ERR_NO_DEVICE = 7         /* compute requested on a plan without a device         */
+} temco_status;
+
+/* operators of the ORIGINAL (undecomposed) layer graph */
+typedef enum {
+  TEMCO_OP_INPUT = 0,          /* graph input, NHWC [batch, height, width, channels]           */
+  TEMCO_OP_CONV2D = 1,         /* square kernel, stride, zero pad; groups == 1 unless undecomposed */
+  TEMCO_OP_BATCHNORM = 2,      /* inference BN: gamma*(x-mean)/sqrt(var+eps)+beta              */
+  TEMCO_OP_RELU = 3,
+  TEMCO_OP_SILU = 4,
+  TEMCO_OP_ADD = 5,            /* n-ary elementwise sum                                        */
+  TEMCO_OP_CONCAT = 6,         /* channel concatenation                                        */
+  TEMCO_OP_MAXPOOL = 7,        /* kernel, stride, pad (-inf padding)                           */
+  TEMCO_OP_AVGPOOL = 8,        /* kernel, stride, no padding                                   */
+  TEMCO_OP_GLOBAL_AVGPOOL = 9, /* mean over H, W                                               */
+  TEMCO_OP_LINEAR = 10         /* y = flatten_NCHW(x) W^T + b, W [out_channels, C*H*W]          */
+} temco_op;
+
+typedef struct {
+  int32_t op;                 /* temco_op                                                        */
+  int32_t n_inputs;
+  const int32_t* inputs;      /* indices of EARLIER layers (SSA, execution order)               */
+  int32_t out_channels;       /* conv / linear                                                   */
+  int32_t kernel, stride, pad, groups;   /* conv / pool                                          */
+  const float* weight;        /* conv OIHW (ignored when decomposed) / linear [out, in]; fp32    */
+  const float* bias;          /* [out_channels] or NULL                                          */
+  const float *bn_gamma, *bn_beta, *bn_mean, *bn_var;  /* [C] each, batchnorm only             */
+  float bn_eps;
+} temco_layer;
+
+typedef enum { TEMCO_DECOMP_TUCKER2 = 1, TEMCO_DECOMP_CP = 2 } temco_decomp_kind;
+
+/* decomposition of one conv layer (Eq. (2)); fp32, row-major:
+ *   Tucker-2: first [rank_in, C_in] (NULL iff rank_in == C_in: no fconv),
+ *             core  [rank_out, rank_in, K, K],
+ *             last  [C_out, rank_out] (NULL iff rank_out == C_out: no lconv)
+ *   CP      : rank_in == rank_out == R; first [R, C_in]; core = Kv [R, K];
+ *             core2 = Kh [R, K]; last [C_out, R]   (fconv -> dw Kx1 -> dw 1xK -> lconv)
+ * Any positive rank is accepted; the tcgen05 kernels (bf16 plans) need reduced
+ * ranks that are multiples of 8 (16-byte rows for TMA) and run every other
+ * group on the generic SIMT kernels. */
+typedef struct {
+  int32_t layer;
+  int32_t kind;               /* temco_decomp_kind */
+  int32_t rank_in, rank_out;
+  const float *first, *core, *core2, *last;
+} temco_decomp;
+
+/* declared skip edges: must be EXACTLY the input edges (src -> dst) with
+ * dst - src > 1 in layer order, else TEMCO_ERR_INVALID_GRAPH.  Alg. 1's own
+ * liveness decides what is optimized; the edges are a redundancy check. */
+typedef struct { int32_t src, dst; } temco_edge;
+
+enum { TEMCO_F32 = 0, TEMCO_BF16 = 1 };
+
+enum {
+  TEMCO_FLAG_NO_DEVICE = 1 << 0,       /* plan only: no uploads, no kernels              */
+  TEMCO_FLAG_NO_SKIPOPT = 1 << 1,      /* ablation: no skip connection optimization      */
+  TEMCO_FLAG_NO_FUSION = 1 << 2,       /* ablation: no activation-layer fusion           */
+  TEMCO_FLAG_CUDA_GRAPH = 1 << 3,      /* capture temco_run into a CUDA graph per (in,out,stream) */
+  TEMCO_FLAG_SIMT_ONLY = 1 << 4,       /* never select the tcgen05 kernels               */
+  TEMCO_FLAG_OVERHEAD_ALWAYS = 1 << 5, /* force Overhead() true  (tests)                 */
+  TEMCO_FLAG_OVERHEAD_NEVER = 1 << 6   /* force Overhead() false (tests)                 */
+};
+
+typedef struct {
+  int32_t batch, height, width, channels;  /* input NHWC                                    */
+  int32_t dtype;                           /* TEMCO_F32 | TEMCO_BF16: activations + weights */
+  int32_t distance_threshold;              /* Alg. 1 DISTANCE_THRESHOLD; <= 0 -> 1 */
+  int32_t flags;
+} temco_config;
+
+/* Build a plan: decomposition expansion, liveness, skip optimization
+ * (Alg. 1/2), DCE, fusion grouping, BN folding, weight packing, arena
+ * planning; then (unless TEMCO_FLAG_NO_DEVICE) upload to the current device. */
+temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers,
+                               const temco_decomp* decomps, int32_t n_decomps,
+                               const temco_edge* skip_edges, int32_t n_skip_edges,
+                               const temco_config* cfg, temco_plan_t* out_plan);
+
+/* Enqueue one inference on `stream`.  input: DEVICE pointer, NHWC contiguous,
+ * plan dtype.  output: DEVICE pointer, fp32, [batch, classes] for a
+ * linear/GAP output or NHWC [batch, H, W, C] for a feature-map output
+ * (temco_output_shape). */
+temco_status temco_run(temco_plan_t plan, const void* input, void* output, temco_stream_t stream);
+
+/* Same as temco_run with HOST buffers: the input is copied host->device into a
+ * plan-owned buffer, the run enqueued and the output copied device->host, all
+ * on `stream`; returns after the stream has synchronised.  Pinned host memory
+ * makes the copies asynchronous DMA. */
+temco_status temco_run_host(temco_plan_t plan, const void* host_input, void* host_output,
+                            temco_stream_t stream);
+
+/* Peak internal-tensor bytes (Eq. (3)/(4), reading R14): which = 0 -> the
+ * fused TeMCO schedule, 1 -> the unfused decomposed list L. */
+temco_status temco_peak_internal_bytes(temco_plan_t plan, int32_t which, int64_t* bytes);
+
+/* output dims: ndim = 2 ([N, K]) or 4 (NHWC) */
+temco_status temco_output_shape(temco_plan_t plan, int64_t dims[4], int32_t* ndim);
+
+/* JSON description: schedule (steps, members, inputs, bytes), chosen kernels,
+ * per-step algorithmic FLOPs / bytes, launches per run, arena size, peaks.
+ * Writes at most cap bytes (NUL-terminated); *needed = full length + 1. */
+temco_status temco_plan_describe(temco_plan_t plan, char* buf, size_t cap, size_t* needed);
+
+/* Enqueue one run with a CUDA event pair around every step (profiling; no
+ * CUDA graph) and, after synchronising, write per-step device milliseconds to
+ * step_ms[0 .. n_steps).  n_steps must equal the schedule length. */
+temco_status temco_run_profiled(temco_plan_t plan, const void* input, void* output,
+                                temco_stream_t stream, float* step_ms, int32_t n_steps);
+
+temco_status temco_plan_destroy(temco_plan_t plan);
+const char* temco_status_string(temco_status s);
+const char* temco_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TEMCO_H */

@@ -1,0 +1,671 @@
+// C ABI (include/temco.h): plan creation (planner + lowering + arena +
+// uploads), the stream-ordered executor and the host-side queries.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <map>
+#include <set>
+#include <sstream>
+#include <string>
+#include <vector>
+
+#include "kernels.h"
+#include "planner.h"
+#include "tc.h"
+
+using namespace temco;
+
+namespace {
+
+thread_local std::string g_last_error;
+
+temco_status set_err(temco_status s, const std::string& m) {
+  g_last_error = m;
+  return s;
+}
+
+#define CUDA_TRY(expr)                                                                          \
+  do {                                                                                          \
+    cudaError_t e_ = (expr);                                                                    \
+    if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
+  } while (0)
+
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC };
+
+struct StepExec {
+  int kind = K_NONE;
+  ConvDesc conv{};
+  EwDesc ew{};
+  LinearDesc lin{};
+  GroupDesc grp{};
+  TcChainDesc tc{};
+  std::string kernel;
+  int64_t flops = 0, io_bytes = 0;
+  int launches = 0;
+};
+
+}  // namespace
+
+struct temco_plan_s {
+  IR ir;
+  temco_config cfg{};
+  bool bf16 = false;
+  int flags = 0;
+  int device = -1;
+  bool has_device = false;
+
+  std::vector<StepExec> exec;
+  std::map<int, Loc> loc;
+  std::vector<float> params_h;
+  std::vector<GNode> gnodes_h;
+  std::vector<int32_t> gchild_h;
+  std::vector<uint16_t> tcw_h;     // bf16 weight pool of the tcgen05 kernels
+  float* params_d = nullptr;
+  GNode* gnodes_d = nullptr;
+  int32_t* gchild_d = nullptr;
+  uint16_t* tcw_d = nullptr;
+  char* arena_d = nullptr;
+  int64_t arena_bytes = 0;
+  int64_t in_bytes = 0, out_bytes = 0;
+  void* host_in_d = nullptr;
+  void* host_out_d = nullptr;
+  int max_expr_depth = 0;          // deepest fused-group expression (SIMT interpreter recursion)
+  int64_t out_dims[4] = {0, 0, 0, 0};
+  int out_ndim = 0;
+  // CUDA graph cache (TEMCO_FLAG_CUDA_GRAPH)
+  cudaGraphExec_t gexec = nullptr;
+  const void* g_in = nullptr;
+  void* g_out = nullptr;
+  cudaStream_t g_stream = nullptr;
+  std::string json;
+};
+
+namespace {
+
+int64_t push_params(temco_plan_s* P, const std::vector<float>& v) {
+  int64_t off = (int64_t)P->params_h.size();
+  // keep 16-byte alignment of every parameter block
+  P->params_h.insert(P->params_h.end(), v.begin(), v.end());
+  while (P->params_h.size() % 4) P->params_h.push_back(0.f);
+  return off;
+}
+
+int64_t push_params(temco_plan_s* P, const Buf& b) {
+  if (!b) return -1;
+  return push_params(P, *b);
+}
+
+void bn_scale_shift(const Node& n, std::vector<float>& scale, std::vector<float>& shift) {
+  scale.resize(n.C);
+  shift.resize(n.C);
+  for (int c = 0; c < n.C; ++c) {
+    double s = (double)(*n.bn_g)[c] / std::sqrt((double)(*n.bn_v)[c] + (double)n.eps);
+    scale[c] = (float)s;
+    shift[c] = (float)((double)(*n.bn_b)[c] - (double)(*n.bn_m)[c] * s);
+  }
+}
+
+// conv weight OIHW -> [K][kh][kw][C/groups]
+std::vector<float> repack_conv(const Node& n, int cin) {
+  const int cg = cin / n.groups;
+  std::vector<float> w((size_t)n.C * n.kh * n.kw * cg);
+  const std::vector<float>& s = *n.w;
+  for (int k = 0; k < n.C; ++k)
+    for (int c = 0; c < cg; ++c)
+      for (int a = 0; a < n.kh; ++a)
+        for (int b = 0; b < n.kw; ++b)
+          w[(((size_t)k * n.kh + a) * n.kw + b) * cg + c] = s[(((size_t)k * cg + c) * n.kh + a) * n.kw + b];
+  return w;
+}
+
+Loc tensor_loc(temco_plan_s* P, int id) { return P->loc.at(id); }
+
+// ---------------------------------------------------------------------------
+// lowering of one fused group into the SIMT interpreter's node table
+// ---------------------------------------------------------------------------
+struct GroupLowering {
+  temco_plan_s* P;
+  std::set<int> members;
+  std::map<int, int> made;
+  std::map<int, int> depth;   // expression depth of each lowered node (device recursion)
+
+  int node(int v) {
+    auto it = made.find(v);
+    if (it != made.end()) return it->second;
+    const IR& ir = P->ir;
+    const Node& n = ir.nodes[v];
+    GNode g{};
+    g.C = n.C; g.H = n.H; g.W = n.W;
+    g.w = g.b = -1;
+    std::vector<int> kids;
+    if (!members.count(v)) {
+      g.op = G_EXT;
+      g.t = tensor_loc(P, v);
+      g.tC = n.C; g.tH = n.H; g.tW = n.W;
+    } else if (n.role == ROLE_LCONV) {
+      const int r = ir.oin[v][0];
+      const Node& rn = ir.nodes[r];
+      g.op = G_LCONV;
+      g.R = rn.C;
+      g.t = tensor_loc(P, r);
+      g.tC = rn.C; g.tH = rn.H; g.tW = rn.W;
+      g.w = push_params(P, n.w);
+      g.b = push_params(P, n.b);
+    } else {
+      switch (n.op) {
+        case OP_BN: {
+          std::vector<float> sc, sh;
+          bn_scale_shift(n, sc, sh);
+          g.op = G_AFFINE;
+          g.w = push_params(P, sc);
+          g.b = push_params(P, sh);
+          break;
+        }
+        case OP_RELU: g.op = G_RELU; break;
+        case OP_SILU: g.op = G_SILU; break;
+        case OP_ADD: g.op = G_ADD; break;
+        case OP_CONCAT: g.op = G_CONCAT; break;
+        case OP_MAXPOOL: g.op = G_MAXPOOL; g.k = n.kh; g.s = n.sh; g.p = n.ph; break;
+        case OP_AVGPOOL: g.op = G_AVGPOOL; g.k = n.kh; g.s = n.sh; g.p = 0; break;
+        default: throw std::runtime_error("unexpected op inside a fused group");
+      }
+      for (int i : ir.oin[v]) kids.push_back(node(i));
+    }
+    int d = 1;
+    for (int k : kids) d = std::max(d, 1 + depth[k]);
+    g.nin = (int)kids.size();
+    g.child = (int)P->gchild_h.size();
+    P->gchild_h.insert(P->gchild_h.end(), kids.begin(), kids.end());
+    int id = (int)P->gnodes_h.size();
+    P->gnodes_h.push_back(g);
+    depth[id] = d;
+    P->max_expr_depth = std::max(P->max_expr_depth, d);
+    made[v] = id;
+    return id;
+  }
+};
+
+// ---------------------------------------------------------------------------
+// arena: greedy best-offset placement of the schedule's tensors by lifetime
+// ---------------------------------------------------------------------------
+int64_t plan_arena(temco_plan_s* P) {
+  const IR& ir = P->ir;
+  const int T = (int)ir.steps.size();
+  std::map<int, int> def, last;
+  for (int t = 0; t < T; ++t) {
+    def[ir.steps[t].out] = t;
+    if (!last.count(ir.steps[t].out)) last[ir.steps[t].out] = t;
+    for (int x : ir.steps[t].in) last[x] = t;
+  }
+  struct Item { int id; int64_t bytes; int a, b; int64_t off; };
+  std::vector<Item> items;
+  const int64_t elem = P->bf16 ? 2 : 4;
+  for (auto& kv : def) {
+    int id = kv.first;
+    if (id == ir.input || id == ir.output) continue;
+    const Node& n = ir.nodes[id];
+    int64_t bytes = (int64_t)ir.batch * n.C * n.H * n.W * elem;
+    bytes = (bytes + 1023) / 1024 * 1024;
+    items.push_back({id, bytes, kv.second, last[id], 0});
+  }
+  std::sort(items.begin(), items.end(), [](const Item& x, const Item& y) {
+    return x.bytes != y.bytes ? x.bytes > y.bytes : x.id < y.id;
+  });
+  std::vector<Item> placed;
+  int64_t total = 0;
+  for (Item& it : items) {
+    std::vector<std::pair<int64_t, int64_t>> busy;
+    for (const Item& q : placed)
+      if (!(q.b < it.a || it.b < q.a)) busy.push_back({q.off, q.off + q.bytes});
+    std::sort(busy.begin(), busy.end());
+    int64_t off = 0;
+    for (auto& r : busy) {
+      if (off + it.bytes <= r.first) break;
+      off = std::max(off, r.second);
+    }
+    it.off = off;
+    placed.push_back(it);
+    total = std::max(total, off + it.bytes);
+  }
+  const int32_t dt = P->bf16 ? DT_BF16 : DT_F32;
+  for (const Item& it : placed) P->loc[it.id] = Loc{W_ARENA, dt, it.off};
+  P->loc[ir.input] = Loc{W_INPUT, dt, 0};
+  P->loc[ir.output] = Loc{W_OUTPUT, DT_F32, 0};
+  return total;
+}
+
+int64_t tensor_bytes(const temco_plan_s* P, int id) {
+  const Node& n = P->ir.nodes[id];
+  int64_t el = (int64_t)P->ir.batch * n.C * n.H * n.W;
+  return el * (id == P->ir.output ? 4 : (P->bf16 ? 2 : 4));
+}
+
+void lower(temco_plan_s* P) {
+  IR& ir = P->ir;
+  const int N = ir.batch;
+  P->exec.assign(ir.steps.size(), StepExec());
+  for (size_t t = 0; t < ir.steps.size(); ++t) {
+    const Step& s = ir.steps[t];
+    StepExec& e = P->exec[t];
+    const Node& v = ir.nodes[s.out];
+    for (int m : s.members) e.flops += node_flops(ir, m);
+    for (int x : s.in) e.io_bytes += tensor_bytes(P, x);
+    if (v.op != OP_INPUT) e.io_bytes += tensor_bytes(P, s.out);
+    if (s.group) {
+      // try the tcgen05 chain kernel first (bf16 plans), else the interpreter
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+          tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tc)) {
+        e.kind = K_GROUP_TC;
+        e.kernel = "tc_chain";
+        e.launches = 1;
+        continue;
+      }
+      GroupLowering gl{P, std::set<int>(s.members.begin(), s.members.end()), {}};
+      GroupDesc& g = e.grp;
+      int tsrc;
+      if (v.role == ROLE_FCONV) {
+        g.root = ROOT_FCONV;
+        tsrc = ir.oin[s.out][0];
+        g.Nout = v.C;
+        if (v.C > 256) throw std::runtime_error("fused fconv with more than 256 outputs");
+        g.F = push_params(P, v.w);
+        g.Fb = push_params(P, v.b);
+        gl.members.erase(s.out);
+      } else if (v.op == OP_GAP) {
+        g.root = ROOT_GAP;
+        tsrc = ir.oin[s.out][0];
+        gl.members.erase(s.out);
+      } else {
+        g.root = ROOT_STORE;
+        tsrc = s.out;
+      }
+      const Node& tn = ir.nodes[tsrc];
+      g.tnode = gl.node(tsrc);
+      g.N = N; g.H = tn.H; g.W = tn.W; g.C = tn.C;
+      g.y = tensor_loc(P, s.out);
+      e.kind = K_GROUP_SIMT;
+      e.kernel = g.root == ROOT_GAP ? "simt_group_gap" : "simt_group";
+      e.launches = 1;
+      continue;
+    }
+    switch (v.op) {
+      case OP_INPUT:
+        e.kind = K_NONE;
+        e.kernel = "none";
+        break;
+      case OP_CONV: {
+        const Node& x = ir.nodes[ir.oin[s.out][0]];
+        ConvDesc& c = e.conv;
+        c.x = tensor_loc(P, x.id);
+        c.y = tensor_loc(P, s.out);
+        c.N = N; c.H = x.H; c.W = x.W; c.C = x.C;
+        c.Ho = v.H; c.Wo = v.W; c.K = v.C;
+        c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = v.groups;
+        c.w = push_params(P, repack_conv(v, x.C));
+        c.b = push_params(P, v.b);
+        e.kind = K_CONV;
+        e.kernel = v.groups > 1 ? "simt_dwconv" : "simt_conv";
+        e.launches = 1;
+        break;
+      }
+      case OP_LINEAR: {
+        const Node& x = ir.nodes[ir.oin[s.out][0]];
+        LinearDesc& l = e.lin;
+        l.x = tensor_loc(P, x.id);
+        l.y = tensor_loc(P, s.out);
+        l.N = N; l.K = x.C * x.H * x.W; l.O = v.C;
+        // permute columns from NCHW flattening (c, h, w) to our NHWC (h, w, c)
+        std::vector<float> w((size_t)l.O * l.K);
+        const std::vector<float>& src = *v.w;
+        for (int o = 0; o < l.O; ++o)
+          for (int c = 0; c < x.C; ++c)
+            for (int hw = 0; hw < x.H * x.W; ++hw)
+              w[(size_t)o * l.K + (size_t)hw * x.C + c] = src[(size_t)o * l.K + (size_t)c * x.H * x.W + hw];
+        l.w = push_params(P, w);
+        l.b = push_params(P, v.b);
+        l.relu = 0;
+        e.kind = K_LINEAR;
+        e.kernel = "simt_linear";
+        e.launches = 1;
+        break;
+      }
+      default: {
+        EwDesc& d = e.ew;
+        const Node& x = ir.nodes[ir.oin[s.out][0]];
+        d.y = tensor_loc(P, s.out);
+        d.N = N; d.H = x.H; d.W = x.W; d.C = v.C; d.Ho = v.H; d.Wo = v.W;
+        d.n_in = (int)ir.oin[s.out].size();
+        if (d.n_in > kMaxEwInputs) throw std::runtime_error("too many inputs for a standalone op");
+        for (int j = 0; j < d.n_in; ++j) {
+          d.x[j] = tensor_loc(P, ir.oin[s.out][j]);
+          d.xc[j] = ir.nodes[ir.oin[s.out][j]].C;
+        }
+        d.scale = d.shift = -1;
+        switch (v.op) {
+          case OP_BN: {
+            std::vector<float> sc, sh;
+            bn_scale_shift(v, sc, sh);
+            d.kind = EW_BN;
+            d.scale = push_params(P, sc);
+            d.shift = push_params(P, sh);
+            break;
+          }
+          case OP_RELU: d.kind = EW_RELU; break;
+          case OP_SILU: d.kind = EW_SILU; break;
+          case OP_ADD: d.kind = EW_ADD; break;
+          case OP_CONCAT: d.kind = EW_CONCAT; break;
+          case OP_MAXPOOL: d.kind = EW_MAXPOOL; d.k = v.kh; d.s = v.sh; d.p = v.ph; break;
+          case OP_AVGPOOL: d.kind = EW_AVGPOOL; d.k = v.kh; d.s = v.sh; d.p = 0; break;
+          case OP_GAP: d.kind = EW_GAP; break;
+          default: throw std::runtime_error("unexpected standalone op");
+        }
+        e.kind = K_EW;
+        e.kernel = std::string("simt_") + op_name(v.op);
+        e.launches = 1;
+      }
+    }
+  }
+}
+
+void json_ints(std::ostringstream& o, const std::vector<int>& v) {
+  o << "[";
+  for (size_t i = 0; i < v.size(); ++i) o << (i ? "," : "") << v[i];
+  o << "]";
+}
+
+std::string make_json(const temco_plan_s* P) {
+  const IR& ir = P->ir;
+  std::ostringstream o;
+  int launches = 0;
+  for (auto& e : P->exec) launches += e.launches;
+  o << "{\"peak_fused\":" << ir.peak_fused << ",\"peak_unfused\":" << ir.peak_unfused
+    << ",\"arena_bytes\":" << P->arena_bytes << ",\"n_L\":" << ir.nL << ",\"n_O\":" << ir.O.size()
+    << ",\"launches\":" << launches << ",\"dtype\":\"" << (P->bf16 ? "bf16" : "f32") << "\",\"decisions\":[";
+  for (size_t i = 0; i < ir.decisions.size(); ++i) {
+    const SkipDecision& d = ir.decisions[i];
+    o << (i ? "," : "") << "{\"node\":" << d.node << ",\"kind\":\""
+      << (d.kind == 0 ? "skip-optimized" : d.kind == 1 ? "skip-unreducible" : "skip-rejected") << "\",\"list\":";
+    json_ints(o, d.list);
+    o << "}";
+  }
+  o << "],\"O\":";
+  json_ints(o, ir.O);
+  o << ",\"steps\":[";
+  for (size_t t = 0; t < ir.steps.size(); ++t) {
+    const Step& s = ir.steps[t];
+    const Node& v = ir.nodes[s.out];
+    o << (t ? "," : "") << "{\"kind\":\"" << (s.group ? "group" : "op") << "\",\"out\":" << s.out << ",\"op\":\""
+      << op_name(v.op) << "\",\"role\":\"" << role_name(v.role) << "\",\"members\":";
+    json_ints(o, s.members);
+    o << ",\"inputs\":";
+    json_ints(o, s.in);
+    o << ",\"bytes\":" << ir.size(s.out);
+    if (!P->exec.empty()) {
+      const StepExec& e = P->exec[t];
+      o << ",\"kernel\":\"" << e.kernel << "\",\"flops\":" << e.flops << ",\"io_bytes\":" << e.io_bytes
+        << ",\"launches\":" << e.launches;
+      if (e.kind == K_GROUP_TC) o << ",\"tc_flops\":" << e.tc.alg_flops << ",\"tc_bytes\":" << e.tc.alg_bytes;
+    }
+    o << ",\"live\":" << ir.live_fused[t] << "}";
+  }
+  o << "],\"live_unfused\":[";
+  for (size_t t = 0; t < ir.live_unfused.size(); ++t) o << (t ? "," : "") << ir.live_unfused[t];
+  o << "]}";
+  return o.str();
+}
+
+template <class T>
+temco_status upload(T** dst, const std::vector<T>& src) {
+  if (src.empty()) return TEMCO_OK;
+  if (cudaMalloc(dst, src.size() * sizeof(T)) != cudaSuccess) return set_err(TEMCO_ERR_OUT_OF_MEMORY, "cudaMalloc");
+  CUDA_TRY(cudaMemcpy(*dst, src.data(), src.size() * sizeof(T), cudaMemcpyHostToDevice));
+  return TEMCO_OK;
+}
+
+void free_device(temco_plan_s* P) {
+  if (P->gexec) cudaGraphExecDestroy(P->gexec);
+  cudaFree(P->params_d);
+  cudaFree(P->gnodes_d);
+  cudaFree(P->gchild_d);
+  cudaFree(P->tcw_d);
+  cudaFree(P->arena_d);
+  cudaFree(P->host_in_d);
+  cudaFree(P->host_out_d);
+}
+
+RunPtrs run_ptrs(temco_plan_s* P, const void* in, void* out) {
+  return RunPtrs{P->arena_d, in, out, P->params_d};
+}
+
+temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st, cudaEvent_t* ev) {
+  RunPtrs rp = run_ptrs(P, in, out);
+  for (size_t t = 0; t < P->exec.size(); ++t) {
+    const StepExec& e = P->exec[t];
+    if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t], st));
+    switch (e.kind) {
+      case K_NONE: break;
+      case K_CONV: launch_conv(e.conv, rp, st); break;
+      case K_EW: launch_ew(e.ew, rp, st); break;
+      case K_LINEAR: launch_linear(e.lin, rp, st); break;
+      case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
+      case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
+    }
+    if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t + 1], st));
+  }
+  cudaError_t err = cudaGetLastError();
+  if (err != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string("kernel launch: ") + cudaGetErrorString(err));
+  return TEMCO_OK;
+}
+
+temco_status check_device(temco_plan_s* P) {
+  if (!P) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (!P->has_device) return set_err(TEMCO_ERR_NO_DEVICE, "plan was created without a device");
+  int dev = -1;
+  CUDA_TRY(cudaGetDevice(&dev));
+  if (dev != P->device) return set_err(TEMCO_ERR_DEVICE_MISMATCH, "current device differs from the plan's");
+  return TEMCO_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* temco_status_string(temco_status s) {
+  switch (s) {
+    case TEMCO_OK: return "ok";
+    case TEMCO_ERR_INVALID_ARGUMENT: return "invalid argument";
+    case TEMCO_ERR_INVALID_GRAPH: return "invalid graph";
+    case TEMCO_ERR_UNSUPPORTED: return "unsupported";
+    case TEMCO_ERR_OUT_OF_MEMORY: return "out of memory";
+    case TEMCO_ERR_CUDA: return "cuda error";
+    case TEMCO_ERR_DEVICE_MISMATCH: return "device mismatch";
+    case TEMCO_ERR_NO_DEVICE: return "no device";
+  }
+  return "unknown status";
+}
+
+const char* temco_last_error(void) { return g_last_error.c_str(); }
+
+temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, const temco_decomp* decomps,
+                               int32_t n_decomps, const temco_edge* skip_edges, int32_t n_skip_edges,
+                               const temco_config* cfg, temco_plan_t* out_plan) {
+  if (!cfg || !out_plan) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "cfg / out_plan is NULL");
+  *out_plan = nullptr;
+  if (cfg->dtype != TEMCO_F32 && cfg->dtype != TEMCO_BF16) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "bad dtype");
+  if ((cfg->flags & TEMCO_FLAG_OVERHEAD_ALWAYS) && (cfg->flags & TEMCO_FLAG_OVERHEAD_NEVER))
+    return set_err(TEMCO_ERR_INVALID_ARGUMENT, "contradictory overhead flags");
+  auto* P = new (std::nothrow) temco_plan_s();
+  if (!P) return set_err(TEMCO_ERR_OUT_OF_MEMORY, "host allocation");
+  P->cfg = *cfg;
+  P->bf16 = cfg->dtype == TEMCO_BF16;
+  P->flags = cfg->flags;
+  BuildOptions opt;
+  opt.distance_threshold = cfg->distance_threshold > 0 ? cfg->distance_threshold : 1;
+  opt.skip_opt = !(cfg->flags & TEMCO_FLAG_NO_SKIPOPT);
+  opt.fusion = !(cfg->flags & TEMCO_FLAG_NO_FUSION);
+  opt.overhead_policy = (cfg->flags & TEMCO_FLAG_OVERHEAD_ALWAYS) ? 1 : (cfg->flags & TEMCO_FLAG_OVERHEAD_NEVER) ? 2 : 0;
+  opt.bf16 = P->bf16;
+  std::string err;
+  temco_status st = build_ir(layers, n_layers, decomps, n_decomps, skip_edges, n_skip_edges, *cfg, opt, P->ir, err);
+  if (st != TEMCO_OK) {
+    delete P;
+    return set_err(st, err);
+  }
+  const Node& on = P->ir.nodes[P->ir.output];
+  if (on.H == 1 && on.W == 1 && (on.op == OP_LINEAR || on.op == OP_GAP)) {
+    P->out_ndim = 2;
+    P->out_dims[0] = cfg->batch;
+    P->out_dims[1] = on.C;
+  } else {
+    P->out_ndim = 4;
+    P->out_dims[0] = cfg->batch; P->out_dims[1] = on.H; P->out_dims[2] = on.W; P->out_dims[3] = on.C;
+  }
+  P->in_bytes = (int64_t)cfg->batch * cfg->height * cfg->width * cfg->channels * (P->bf16 ? 2 : 4);
+  P->out_bytes = (int64_t)cfg->batch * on.C * on.H * on.W * 4;
+  try {
+    P->arena_bytes = plan_arena(P);
+    lower(P);
+  } catch (const std::exception& ex) {
+    delete P;
+    return set_err(TEMCO_ERR_UNSUPPORTED, std::string("lowering: ") + ex.what());
+  }
+  P->json = make_json(P);
+  if (!(cfg->flags & TEMCO_FLAG_NO_DEVICE)) {
+    int dev = -1;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+      delete P;
+      return set_err(TEMCO_ERR_NO_DEVICE, "no CUDA device (use TEMCO_FLAG_NO_DEVICE for host-only plans)");
+    }
+    P->device = dev;
+    P->has_device = true;
+    // the SIMT group interpreter recurses once per expression level (~128 B
+    // frames, see -Xptxas -v); grow the per-thread stack when needed
+    size_t need = 1024 + (size_t)P->max_expr_depth * 192, cur = 0;
+    if (cudaDeviceGetLimit(&cur, cudaLimitStackSize) == cudaSuccess && cur < need &&
+        cudaDeviceSetLimit(cudaLimitStackSize, need) != cudaSuccess) {
+      delete P;
+      return set_err(TEMCO_ERR_CUDA, "cudaDeviceSetLimit(cudaLimitStackSize)");
+    }
+    temco_status s2 = TEMCO_OK;
+    if ((s2 = upload(&P->params_d, P->params_h)) != TEMCO_OK || (s2 = upload(&P->gnodes_d, P->gnodes_h)) != TEMCO_OK ||
+        (s2 = upload(&P->gchild_d, P->gchild_h)) != TEMCO_OK || (s2 = upload(&P->tcw_d, P->tcw_h)) != TEMCO_OK) {
+      free_device(P);
+      delete P;
+      return s2;
+    }
+    if (P->arena_bytes > 0 && cudaMalloc(&P->arena_d, P->arena_bytes) != cudaSuccess) {
+      free_device(P);
+      delete P;
+      return set_err(TEMCO_ERR_OUT_OF_MEMORY, "arena cudaMalloc");
+    }
+    std::string terr;
+    if (!tc_finalize(P->exec.size(), [&](size_t i) -> TcChainDesc* {
+          return P->exec[i].kind == K_GROUP_TC ? &P->exec[i].tc : nullptr;
+        }, P->arena_d, P->tcw_d, terr)) {
+      free_device(P);
+      delete P;
+      return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
+    }
+  }
+  // the host copies of large pools are no longer needed
+  *out_plan = P;
+  return TEMCO_OK;
+}
+
+temco_status temco_run(temco_plan_t P, const void* input, void* output, temco_stream_t stream) {
+  temco_status st = check_device(P);
+  if (st != TEMCO_OK) return st;
+  if (!input || !output) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "input / output is NULL");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if ((P->flags & TEMCO_FLAG_CUDA_GRAPH) && s != nullptr) {
+    if (!P->gexec || P->g_in != input || P->g_out != output || P->g_stream != s) {
+      if (P->gexec) cudaGraphExecDestroy(P->gexec);
+      P->gexec = nullptr;
+      cudaGraph_t graph;
+      CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
+      temco_status e = enqueue(P, input, output, s, nullptr);
+      cudaError_t ce = cudaStreamEndCapture(s, &graph);
+      if (e != TEMCO_OK) return e;
+      if (ce != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string("capture: ") + cudaGetErrorString(ce));
+      ce = cudaGraphInstantiate(&P->gexec, graph, 0);
+      cudaGraphDestroy(graph);
+      if (ce != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string("instantiate: ") + cudaGetErrorString(ce));
+      P->g_in = input;
+      P->g_out = output;
+      P->g_stream = s;
+    }
+    CUDA_TRY(cudaGraphLaunch(P->gexec, s));
+    return TEMCO_OK;
+  }
+  return enqueue(P, input, output, s, nullptr);
+}
+
+temco_status temco_run_host(temco_plan_t P, const void* host_input, void* host_output, temco_stream_t stream) {
+  temco_status st = check_device(P);
+  if (st != TEMCO_OK) return st;
+  if (!host_input || !host_output) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "host buffers are NULL");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (!P->host_in_d) {
+    if (cudaMalloc(&P->host_in_d, P->in_bytes) != cudaSuccess || cudaMalloc(&P->host_out_d, P->out_bytes) != cudaSuccess)
+      return set_err(TEMCO_ERR_OUT_OF_MEMORY, "staging buffers");
+  }
+  CUDA_TRY(cudaMemcpyAsync(P->host_in_d, host_input, P->in_bytes, cudaMemcpyHostToDevice, s));
+  st = temco_run(P, P->host_in_d, P->host_out_d, stream);
+  if (st != TEMCO_OK) return st;
+  CUDA_TRY(cudaMemcpyAsync(host_output, P->host_out_d, P->out_bytes, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  return TEMCO_OK;
+}
+
+temco_status temco_run_profiled(temco_plan_t P, const void* input, void* output, temco_stream_t stream,
+                                float* step_ms, int32_t n_steps) {
+  temco_status st = check_device(P);
+  if (st != TEMCO_OK) return st;
+  if (!input || !output || !step_ms || n_steps != (int32_t)P->exec.size())
+    return set_err(TEMCO_ERR_INVALID_ARGUMENT, "bad profiling arguments");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  std::vector<cudaEvent_t> ev(2 * P->exec.size());
+  for (auto& e : ev) CUDA_TRY(cudaEventCreate(&e));
+  st = enqueue(P, input, output, s, ev.data());
+  if (st == TEMCO_OK) {
+    CUDA_TRY(cudaStreamSynchronize(s));
+    for (size_t t = 0; t < P->exec.size(); ++t) cudaEventElapsedTime(&step_ms[t], ev[2 * t], ev[2 * t + 1]);
+  }
+  for (auto& e : ev) cudaEventDestroy(e);
+  return st;
+}
+
+temco_status temco_peak_internal_bytes(temco_plan_t P, int32_t which, int64_t* bytes) {
+  if (!P || !bytes || (which != 0 && which != 1)) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "bad arguments");
+  *bytes = which == 0 ? P->ir.peak_fused : P->ir.peak_unfused;
+  return TEMCO_OK;
+}
+
+temco_status temco_output_shape(temco_plan_t P, int64_t dims[4], int32_t* ndim) {
+  if (!P || !dims || !ndim) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "bad arguments");
+  for (int i = 0; i < 4; ++i) dims[i] = P->out_dims[i];
+  *ndim = P->out_ndim;
+  return TEMCO_OK;
+}
+
+temco_status temco_plan_describe(temco_plan_t P, char* buf, size_t cap, size_t* needed) {
+  if (!P) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "plan is NULL");
+  if (needed) *needed = P->json.size() + 1;
+  if (buf && cap > 0) {
+    size_t n = std::min(cap - 1, P->json.size());
+    memcpy(buf, P->json.data(), n);
+    buf[n] = 0;
+  }
+  return TEMCO_OK;
+}
+
+temco_status temco_plan_destroy(temco_plan_t P) {
+  if (!P) return TEMCO_OK;
+  if (P->has_device) free_device(P);
+  delete P;
+  return TEMCO_OK;
+}
+
+}  // extern "C"

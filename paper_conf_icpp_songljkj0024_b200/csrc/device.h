@@ -1,0 +1,94 @@
+// Plain-old-data descriptors shared by the host lowering (capi.cu) and the
+// device kernels (kernels_*.cu).  All activations are NHWC; every tensor is
+// addressed through a Loc so that a plan can be replayed on new input /
+// output pointers without touching its descriptors.
+#pragma once
+
+#include <cstdint>
+
+namespace temco {
+
+enum DType : int32_t { DT_F32 = 0, DT_BF16 = 1 };
+enum Where : int32_t { W_ARENA = 0, W_INPUT = 1, W_OUTPUT = 2 };
+
+struct Loc {
+  int32_t where = W_ARENA;   // arena / graph input / graph output
+  int32_t dtype = DT_F32;
+  int64_t off = 0;           // byte offset in the arena
+};
+
+struct RunPtrs {
+  char* arena;
+  const void* input;
+  void* output;
+  const float* params;       // fp32 parameter pool (SIMT kernels)
+};
+
+#ifdef __CUDACC__
+__host__ __device__ inline const void* loc_ptr(const Loc& l, const RunPtrs& p) {
+  return l.where == W_INPUT ? p.input : (l.where == W_OUTPUT ? (const void*)p.output : (const void*)(p.arena + l.off));
+}
+#endif
+
+// ---------------------------------------------------------------------------
+// standalone (non-fused) operators
+// ---------------------------------------------------------------------------
+struct ConvDesc {             // direct NHWC convolution (fconv on full tensors, cores, depthwise, plain)
+  Loc x, y;
+  int32_t N, H, W, C;         // input
+  int32_t Ho, Wo, K;          // output spatial, output channels
+  int32_t kh, kw, sh, sw, ph, pw, groups;
+  int64_t w;                  // params offset: [K][kh][kw][C/groups]
+  int64_t b;                  // params offset or -1
+};
+
+enum EwKind : int32_t { EW_BN, EW_RELU, EW_SILU, EW_ADD, EW_CONCAT, EW_MAXPOOL, EW_AVGPOOL, EW_GAP };
+
+constexpr int kMaxEwInputs = 64;
+struct EwDesc {               // elementwise / pooling / concat / GAP
+  int32_t kind;
+  int32_t n_in;
+  Loc x[kMaxEwInputs];
+  int32_t xc[kMaxEwInputs];   // channels of each input (concat)
+  Loc y;
+  int32_t N, H, W, C;         // input spatial + output channels
+  int32_t Ho, Wo;
+  int32_t k, s, p;
+  int64_t scale, shift;       // BN (params offsets)
+};
+
+struct LinearDesc {           // y[n, o] = b[o] + sum_k W[o, k] x[n, k], x flattened NHWC
+  Loc x, y;
+  int32_t N, K, O;
+  int64_t w, b;               // params offsets; W already permuted to NHWC order
+  int32_t relu;               // fused ReLU epilogue (a following standalone relu is folded in)
+};
+
+// ---------------------------------------------------------------------------
+// fused group, generic SIMT interpreter (all group shapes)
+// ---------------------------------------------------------------------------
+enum GOp : int32_t { G_LCONV, G_AFFINE, G_RELU, G_SILU, G_ADD, G_CONCAT, G_MAXPOOL, G_AVGPOOL, G_EXT };
+
+struct GNode {
+  int32_t op;
+  int32_t C, H, W;            // output per-image shape of this node
+  int32_t nin, child;         // children: children[child .. child + nin)
+  int32_t k, s, p;            // pooling
+  int32_t R;                  // G_LCONV: reduced channels
+  Loc t;                      // G_LCONV: reduced input; G_EXT: full tensor
+  int32_t tC, tH, tW;         // shape of t
+  int64_t w, b;               // G_LCONV weight [C][R] / bias; G_AFFINE scale / shift
+};
+
+enum RootKind : int32_t { ROOT_FCONV, ROOT_GAP, ROOT_STORE };
+
+struct GroupDesc {
+  int32_t root;               // RootKind
+  int32_t tnode;              // node index (global) whose value is the C-wide restored tensor t
+  int32_t N, H, W, C;         // t's shape (root resolution)
+  int32_t Nout;               // fconv output channels
+  int64_t F, Fb;              // fconv weight [Nout][C] / bias (-1)
+  Loc y;
+};
+
+}  // namespace temco

@@ -1,0 +1,16 @@
+// Launchers for the device kernels (kernels_simt.cu, kernels_tc.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "device.h"
+
+namespace temco {
+
+void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
+void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s);
+void launch_linear(const LinearDesc& d, const RunPtrs& p, cudaStream_t s);
+void launch_group_simt(const GroupDesc& d, const GNode* nodes, const int32_t* children, const RunPtrs& p,
+                       cudaStream_t s);
+
+}  // namespace temco

@@ -1,0 +1,142 @@
+"""GPU parity: temco_run (through the C ABI) vs the fp64 oracle.
+
+Bars (BASELINE.json north star): relative L2 <= 1e-4 in fp32 mode (SIMT
+kernels, no TF32) and <= 2e-2 in bf16 mode (bf16 storage, fp32 accumulation;
+the workloads hand both sides the same bf16-representable weights and input).
+Peak internal bytes must equal the oracle's exactly.  Full-size configs run in
+the launch configuration bench.py times; the oracle checks sampled images
+(images are independent, the kernels batch-invariant).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+def _plan_and_run(m, flags=0, x=None, stream=None):
+    from paper_conf_icpp_songljkj0024_b200 import Plan
+    p = Plan(m, flags=flags)
+    if x is None:
+        x = W.make_input(m)
+    xt = torch.from_numpy(x).cuda().to(torch.bfloat16 if m.dtype == "bf16" else torch.float32)
+    y = torch.full(p.output_shape(), float("nan"), dtype=torch.float32, device="cuda")
+    p.run(xt, y, stream)
+    torch.cuda.synchronize()
+    return p, y.cpu().numpy().astype(np.float64)
+
+
+def _rel(a, b):
+    return float(np.linalg.norm(a - b) / np.linalg.norm(b))
+
+
+SMALL = {
+    "c1": lambda dt: W.c1_basic_block(dtype=dt, batch=2),
+    "t1": lambda dt: W.t1_chain(dtype=dt, batch=2),
+    "t2_1": lambda dt: W.t2_stem_blocks(1, dtype=dt, batch=2),
+    "t2_3": lambda dt: W.t2_stem_blocks(3, dtype=dt, batch=3),
+    "t3": lambda dt: W.t3_mini_bottleneck(dtype=dt, batch=2),
+    "t4": lambda dt: W.t4_mini_densenet(dtype=dt, batch=2),
+    "resnet18_s": lambda dt: W.resnet18_cifar(batch=3, dtype=dt, height=16, width=16),
+    "resnet50_s": lambda dt: W.resnet50(batch=2, dtype=dt, height=64, width=64),
+    "vgg16_s": lambda dt: W.vgg16_cp(batch=2, dtype=dt, height=32, width=32),
+    "densenet121_s": lambda dt: W.densenet121(batch=2, dtype=dt, height=64, width=64),
+}
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+def test_fp32_mode(name):
+    m = SMALL[name]("f32")
+    x = W.make_input(m)
+    p, y = _plan_and_run(m, x=x)
+    o = oracle.plan(m)
+    ref = oracle.run_temco(o, x)
+    assert y.shape == ref.shape
+    assert np.isfinite(y).all()
+    assert _rel(y, ref) <= 1e-4, _rel(y, ref)
+    assert p.peak_internal_bytes(0) == o.peak_fused and p.peak_internal_bytes(1) == o.peak_unfused
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+def test_bf16_mode(name):
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_SIMT_ONLY
+    m = SMALL[name]("bf16")
+    x = W.make_input(m)
+    ref = oracle.run_temco(oracle.plan(m), x)
+    for flags in (0, FLAG_SIMT_ONLY):
+        p, y = _plan_and_run(m, flags=flags, x=x)
+        assert np.isfinite(y).all()
+        assert _rel(y, ref) <= 2e-2, (flags, _rel(y, ref))
+
+
+def test_ragged_batch_and_tiles():
+    """batch / pixel counts that leave ragged tails in every kernel's tiling."""
+    m = W.resnet18_cifar(batch=5, dtype="bf16", height=12, width=20)
+    x = W.make_input(m)
+    _, y = _plan_and_run(m, x=x)
+    ref = oracle.run_temco(oracle.plan(m), x)
+    assert _rel(y, ref) <= 2e-2
+
+
+FULL = {"resnet18_cifar": [0, 77, 127], "resnet50": [0, 255], "vgg16_cp": [0, 255], "densenet121": [0, 127]}
+
+
+@pytest.mark.parametrize("name", list(FULL))
+def test_full_config_sampled(name):
+    """Full BASELINE.json config in the bench launch configuration; sampled
+    images checked against the oracle one by one."""
+    m = W.build_config(name)
+    x = W.make_input(m)
+    p, y = _plan_and_run(m, x=x)
+    assert np.isfinite(y).all()
+    o = oracle.plan(m)
+    assert p.peak_internal_bytes(0) == o.peak_fused and p.peak_internal_bytes(1) == o.peak_unfused
+    for i in FULL[name]:
+        ref = oracle.run_temco(o, x[i:i + 1])
+        assert _rel(y[i:i + 1], ref) <= 2e-2, (i, _rel(y[i:i + 1], ref))
+
+
+def test_batch_invariance_and_shard_equivalence():
+    """A shard (images 2..5 run as their own batch) reproduces the same rows of
+    the full-batch run bit for bit: what the multi-GPU batch split relies on."""
+    m = W.resnet50(batch=8, dtype="bf16", height=64, width=64)
+    x = W.make_input(m)
+    _, y = _plan_and_run(m, x=x)
+    ms = W.resnet50(batch=4, dtype="bf16", height=64, width=64)
+    _, ys = _plan_and_run(ms, x=x[2:6])
+    assert np.array_equal(y[2:6], ys)
+
+
+def test_cuda_graph_host_run_and_profiled_agree():
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_CUDA_GRAPH, Plan
+    m = W.resnet18_cifar(batch=4, dtype="bf16")
+    x = W.make_input(m)
+    _, y0 = _plan_and_run(m, x=x)
+    p = Plan(m, flags=FLAG_CUDA_GRAPH)
+    xt = torch.from_numpy(x).cuda().to(torch.bfloat16)
+    y = torch.empty(p.output_shape(), device="cuda")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            p.run(xt, y, s)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy(), y0)
+    xh = torch.from_numpy(x).to(torch.bfloat16).pin_memory()
+    yh = torch.empty(p.output_shape()).pin_memory()
+    p.run_host(xh, yh, s)
+    assert np.array_equal(yh.numpy(), y0)
+    ms = p.run_profiled(xt, y, s)
+    assert len(ms) == len(p.describe()["steps"]) and all(t >= 0 for t in ms)
+    assert np.array_equal(y.cpu().numpy(), y0)
+
+
+def test_device_mismatch_and_errors():
+    from paper_conf_icpp_songljkj0024_b200 import Plan, TemcoError
+    p = Plan(W.c1_basic_block(dtype="f32"))
+    with pytest.raises(TemcoError) as e:
+        p.run(0, 0, 0)
+    assert e.value.status == 1
