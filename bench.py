@@ -1,0 +1,289 @@
+#!/usr/bin/env python
+"""TeMCO fused reduced-skip inference benchmark (driver contract).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config resnet50] [--impl reference]
+
+One step = one full forward pass (every schedule step of the TeMCO plan: core
+convs, fused restore->BN->add->ReLU->reduce groups, head) over one per-GPU batch
+of synthetic images already resident in HBM.  Under torchrun each rank runs its
+own contiguous shard of the global batch (weak scaling) and the fp32 logits are
+gathered with one NCCL all_gather per step (the only collective).
+Rank 0 prints ONE JSON line.
+
+`--impl reference` times the oracle (oracle/, fp64 numpy) as it stands on the
+host cores -- the reference arm of this tier -- on a bounded sample per step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+CONFIG_BATCH = {"resnet18_cifar": 128, "resnet50": 256, "vgg16_cp": 256, "densenet121": 128}
+CONFIG_TEXT = {
+    "resnet18_cifar": "ResNet-18 Tucker-2 decomposed, CIFAR-10 shape 32x32, batch 128",
+    "resnet50": "ResNet-50 Tucker-2 decomposed, ImageNet shape 224x224, batch 256 per GPU, bf16",
+    "vgg16_cp": "VGG-16 CP-decomposed convs, 224x224, batch 256 per GPU",
+    "densenet121": "DenseNet-121 Tucker-2 decomposed (concat skips), 224x224, batch 128 per GPU, 8-GPU batch shard",
+}
+METRIC = "images/sec"
+
+
+def _peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        d = json.load(open(path))
+        return d["hbm_gbs"], d["bf16_tflops"], d.get("bf16_tflops_sustained", d["bf16_tflops"]), "measured"
+    return 6650.0, 1590.0, 1400.0, "fallback"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+
+    def __init__(self, index):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("clocks.sm,clocks.max.sm,utilization.gpu,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(index), f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                       "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        self.p.wait()
+        rows = []
+        for line in open(self.f.name):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 7 and parts[0].isdigit():
+                rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return None
+        loaded = [r for r in rows if r[2].isdigit() and int(r[2]) > 0] or rows
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in loaded for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(int(r[0]) for r in loaded), "sm_max_mhz": int(rows[0][1]),
+                "reasons": reasons, "samples": len(loaded)}
+
+
+def _dist():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def reference_arm(args):
+    """Oracle (fp64 numpy) on the host cores: each step = a bounded sample."""
+    import oracle
+    ws, rank, _ = _dist()
+    if rank != 0:
+        return
+    from threadpoolctl import threadpool_info
+    m = W.build_config(args.config)
+    sample = {"resnet18_cifar": 8, "resnet50": 1, "vgg16_cp": 1, "densenet121": 1}[args.config]
+    pl = oracle.plan(m)
+    times = []
+    for step in range(args.warmup + args.steps):
+        x = W.make_input(m, start=step * sample, count=sample)
+        t0 = time.perf_counter()
+        oracle.run_temco(pl, x)
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(dt)
+    sec = sum(times) / len(times)
+    value = sample / sec
+    threads = max([t.get("num_threads", 1) for t in threadpool_info()] + [1])
+    line = {"metric": METRIC, "value": value, "unit": "images/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": sec * 1e3, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+            "config": {"workload": args.config, "description": CONFIG_TEXT[args.config],
+                       "sample_images_per_step": sample},
+            "cpu_baseline": {"value": value, "unit": "images/s", "cores": threads, "kind": "oracle",
+                             "sample": f"{sample} image(s) of {args.config} per step, TeMCO executor (fp64 numpy)"},
+            "e2e": {"value": value, "unit": "images/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(config):
+    """Oracle images/s on this host on ~10-30 s of CPU work (rank 0, N=1)."""
+    import oracle
+    from threadpoolctl import threadpool_info
+    m = W.build_config(config)
+    pl = oracle.plan(m)
+    sample = {"resnet18_cifar": 64, "resnet50": 8, "vgg16_cp": 8, "densenet121": 8}[config]
+    x = W.make_input(m, start=0, count=sample)
+    oracle.run_temco(pl, x[:1])                 # warm-up
+    t0 = time.perf_counter()
+    oracle.run_temco(pl, x)
+    dt = time.perf_counter() - t0
+    threads = max([t.get("num_threads", 1) for t in threadpool_info()] + [1])
+    return {"value": sample / dt, "unit": "images/s", "cores": threads, "kind": "oracle",
+            "sample": f"{sample} images of {config} through the oracle's TeMCO executor (fp64 numpy), {dt:.1f} s"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="resnet50", choices=list(CONFIG_BATCH))
+    ap.add_argument("--impl", default="temco", choices=["temco", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--simt-only", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    if args.impl == "reference":
+        return reference_arm(args)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_CUDA_GRAPH, FLAG_SIMT_ONLY, Plan
+
+    ws, rank, local = _dist()
+    torch.cuda.set_device(local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    B = CONFIG_BATCH[args.config]
+    m = W.build_config(args.config, batch=B)
+    flags = FLAG_CUDA_GRAPH | (FLAG_SIMT_ONLY if args.simt_only else 0)
+    plan = Plan(m, flags=flags)
+    desc = plan.describe()
+    out_shape = plan.output_shape()
+    x_host = W.make_input(m, start=rank * B, count=B)
+    tdt = torch.bfloat16 if m.dtype == "bf16" else torch.float32
+    x = torch.from_numpy(x_host).to(tdt).cuda()
+    y = torch.empty(out_shape, dtype=torch.float32, device="cuda")
+    gathered = torch.empty((ws,) + tuple(out_shape), dtype=torch.float32, device="cuda") if ws > 1 else None
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")      # > 126 MB L2
+    stream = torch.cuda.Stream()
+
+    def step():
+        plan.run(x, y, stream)
+        if ws > 1:
+            dist.all_gather_into_tensor(gathered, y)
+
+    with torch.cuda.stream(stream):
+        for _ in range(args.warmup):
+            step()
+    torch.cuda.synchronize()
+
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    clocks = Clocks(local)
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with torch.cuda.stream(stream):
+        for i in range(args.steps):
+            flush.fill_(i & 0xFF)                                            # L2 flush, outside the events
+            evs[i][0].record(stream)
+            step()
+            evs[i][1].record(stream)
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms = sum(a.elapsed_time(b) for a, b in evs)
+    if ws > 1:
+        t = torch.tensor([ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    ms_per_step = ms / args.steps
+    value = ws * B / (ms_per_step / 1e3)
+
+    # ---- end to end through the public API with host buffers -----------------
+    xh = torch.from_numpy(x_host).to(tdt).pin_memory()
+    yh = torch.empty(out_shape, dtype=torch.float32).pin_memory()
+    plan.run_host(xh, yh, stream)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    if ws > 1:
+        dist.barrier()
+    e0.record(stream)
+    for _ in range(args.steps):
+        plan.run_host(xh, yh, stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    e2e_ms = e0.elapsed_time(e1) / args.steps
+    if ws > 1:
+        t = torch.tensor([e2e_ms], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_ms = float(t.item())
+
+    # ---- roofline of the dominant kernel class (per-step CUDA events) --------
+    steps = desc["steps"]
+    prof = np.zeros(len(steps))
+    n_prof = max(3, min(args.steps, 10))
+    with torch.cuda.stream(stream):
+        for _ in range(n_prof):
+            flush.fill_(1)
+            prof += np.array(plan.run_profiled(x, y, stream))
+    prof /= n_prof
+    classes = {}
+    for s, t in zip(steps, prof):
+        k = s["kernel"]
+        if k == "none":
+            continue
+        c = classes.setdefault(k, {"ms": 0.0, "flops": 0, "bytes": 0, "launches": 0})
+        c["ms"] += float(t)
+        c["flops"] += s.get("tc_flops", s["flops"])
+        c["bytes"] += s.get("tc_bytes", s["io_bytes"])
+        c["launches"] += s["launches"]
+    hbm, tf_burst, tf_sust, src = _peaks()
+    dom = max(classes, key=lambda k: classes[k]["ms"])
+    c = classes[dom]
+    ai = c["flops"] / max(c["bytes"], 1)
+    if ai > tf_sust * 1e12 / (hbm * 1e9):
+        achieved, peak, unit, bound = c["flops"] / (c["ms"] * 1e-3) / 1e12, tf_sust, "TFLOP/s", "tensor"
+    else:
+        achieved, peak, unit, bound = c["bytes"] / (c["ms"] * 1e-3) / 1e9, hbm, "GB/s", "hbm"
+    total_ms = float(prof.sum())
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "images/s", "n_gpus": ws, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": m.dtype, "data": "synthetic",
+            "config": {"workload": args.config, "description": CONFIG_TEXT[args.config], "batch_per_gpu": B,
+                       "global_batch": ws * B, "image_hw": [m.height, m.width], "parallelism": f"dp{ws}",
+                       "l2": "flushed between timed steps (512 MiB write, outside the step events)",
+                       "peak_internal_bytes": plan.peak_internal_bytes(0),
+                       "peak_internal_bytes_unfused": plan.peak_internal_bytes(1),
+                       "internal_memory_reduction": 1 - plan.peak_internal_bytes(0) / plan.peak_internal_bytes(1),
+                       "cuda_graph": True, "kernels": "simt-only" if args.simt_only else "tcgen05+simt"},
+            "gpu_launches": desc["launches"] * args.steps,
+            "e2e": {"value": ws * B / (e2e_ms / 1e3), "unit": "images/s",
+                    "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
+                    "d2h_bytes_per_step": int(yh.numel() * yh.element_size())},
+            "roofline": {"bound": bound, "kernel": dom, "achieved": achieved, "peak": peak, "unit": unit,
+                         "frac": achieved / peak, "traffic": None, "peak_source": src,
+                         "launches_per_step": c["launches"], "share_of_step": c["ms"] / total_ms,
+                         "alg_flops_per_step": c["flops"], "alg_bytes_per_step": c["bytes"]},
+            "kernel_classes_ms": {k: round(v["ms"], 4) for k, v in sorted(classes.items(), key=lambda kv: -kv[1]["ms"])},
+            "clocks": clk,
+        }
+        if ws == 1 and not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline(args.config)
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
