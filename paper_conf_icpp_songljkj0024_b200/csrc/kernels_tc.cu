@@ -1,16 +1,668 @@
-// tcgen05 fused restore-chain -> BN -> add -> ReLU -> reduce kernel.
-// (first version: lowering disabled; every group runs on the SIMT interpreter)
+// tcgen05 fused restore-chain -> BN -> add -> ReLU -> reduce kernel (sm_100a).
+//
+// One fused group computes, per 128-pixel tile,
+//     t_l = act_l( sum_{j in l} r_j Lhat_j^T + b_l + t_{l-1} ),  out = t_D F^T
+// with the C-wide t never leaving the SM:
+//   GEMM1  TMA (r_j atom [128 x 64], Lhat_j atom [Cc x 64]) -> SMEM ring ->
+//          tcgen05.mma (M=128, N=Cc, K=16) -> TMEM accumulator (Cc fp32 columns)
+//   level epilogue: TMEM -> registers, + b_l, ReLU, -> TMEM (tcgen05.st) so the
+//          next level's MMAs accumulate on top of t_{l-1}; after the last level
+//          the bf16 tile P = t_D is written to SMEM in the SW128 K-major layout
+//   GEMM2  tcgen05.mma (A = P from SMEM, B = F atom via TMA) -> TMEM (Np columns),
+//          accumulated over the C chunks
+//   output epilogue: TMEM -> registers -> bf16 -> global.
+// Warp roles (192 threads, persistent over tiles): warps 0-3 epilogue (warp w
+// owns TMEM lanes 32w..32w+31 = pixel rows), warp 4 TMA producer, warp 5 MMA
+// issuer.  Two TMEM accumulators (chunks c, c+1) let the MMA of one chunk
+// overlap the epilogue of the other.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cmath>
+#include <set>
+
 #include "tc.h"
 
 namespace temco {
 
-bool tc_lower_chain(const IR&, const Step&, const std::map<int, Loc>&, std::vector<uint16_t>&, std::vector<float>&,
-                    TcChainDesc&) {
-  return false;
+// ===========================================================================
+// host: lowering of a fused group into a level chain
+// ===========================================================================
+namespace {
+
+struct PTerm {
+  int lconv;
+  std::vector<double> scale;   // per row of the lconv output
+  int c0;
+};
+
+struct PLevel {
+  std::vector<PTerm> terms;
+  std::vector<double> bias;
+  bool relu = false;
+};
+
+struct ChainParser {
+  const IR& ir;
+  std::set<int> members;
+  int C;
+  std::set<int> visited;
+  int H, W;
+
+  bool chain(int v, std::vector<PLevel>& out) {
+    if (!members.count(v)) return false;
+    visited.insert(v);
+    if (ir.nodes[v].op == OP_RELU) {
+      if (!pre(ir.oin[v][0], out)) return false;
+      out.back().relu = true;
+      return true;
+    }
+    return pre(v, out);
+  }
+
+  bool pre(int v, std::vector<PLevel>& out) {
+    PLevel L;
+    L.bias.assign(C, 0.0);
+    std::vector<PLevel> prev;
+    if (!contribute(v, nullptr, 0, L, prev)) return false;
+    if (L.terms.empty()) return false;
+    out = prev;
+    out.push_back(L);
+    return true;
+  }
+
+  bool contribute(int v, const std::vector<double>* sc, int c0, PLevel& L, std::vector<PLevel>& prev) {
+    if (!members.count(v)) return false;   // external full tensor: not on this kernel
+    visited.insert(v);
+    const Node& n = ir.nodes[v];
+    if (n.H != H || n.W != W) return false;
+    if (n.role == ROLE_LCONV) {
+      PTerm t;
+      t.lconv = v;
+      t.c0 = c0;
+      t.scale = sc ? *sc : std::vector<double>(n.C, 1.0);
+      if (n.b)
+        for (int c = 0; c < n.C; ++c) L.bias[c0 + c] += t.scale[c] * (*n.b)[c];
+      L.terms.push_back(std::move(t));
+      return true;
+    }
+    switch (n.op) {
+      case OP_BN: {
+        std::vector<double> s(n.C);
+        for (int c = 0; c < n.C; ++c) {
+          double k = (double)(*n.bn_g)[c] / std::sqrt((double)(*n.bn_v)[c] + (double)n.eps);
+          double sh = (double)(*n.bn_b)[c] - (double)(*n.bn_m)[c] * k;
+          double outer = sc ? (*sc)[c] : 1.0;
+          s[c] = outer * k;
+          L.bias[c0 + c] += outer * sh;
+        }
+        return contribute(ir.oin[v][0], &s, c0, L, prev);
+      }
+      case OP_ADD:
+        for (int x : ir.oin[v])
+          if (!contribute(x, sc, c0, L, prev)) return false;
+        return true;
+      case OP_CONCAT: {
+        int off = 0;
+        for (int x : ir.oin[v]) {
+          const int cx = ir.nodes[x].C;
+          std::vector<double> s2;
+          if (sc) s2.assign(sc->begin() + off, sc->begin() + off + cx);
+          if (!contribute(x, sc ? &s2 : nullptr, c0 + off, L, prev)) return false;
+          off += cx;
+        }
+        return true;
+      }
+      case OP_RELU: {
+        // a previous chain value t_{l-1}: unit scale, full width, at most one
+        if (sc || c0 != 0 || n.C != C || !prev.empty()) return false;
+        return chain(v, prev);
+      }
+      default:
+        return false;
+    }
+  }
+};
+
+uint16_t to_bf16(float f) {
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  u += 0x7FFF + ((u >> 16) & 1);
+  return (uint16_t)(u >> 16);
 }
 
-bool tc_finalize(size_t, const std::function<TcChainDesc*(size_t)>&, char*, uint16_t*, std::string&) { return true; }
+int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
+  while (pool.size() % 512) pool.push_back(0);   // 1024-byte aligned blocks (TMA base alignment)
+  int64_t off = (int64_t)pool.size();
+  for (float f : v) pool.push_back(to_bf16(f));
+  return off;
+}
 
-void launch_tc_chain(const TcChainDesc&, const uint16_t*, const RunPtrs&, cudaStream_t) {}
+int64_t push_f32(std::vector<float>& pool, const std::vector<double>& v) {
+  while (pool.size() % 4) pool.push_back(0.f);
+  int64_t off = (int64_t)pool.size();
+  for (double x : v) pool.push_back((float)x);
+  while (pool.size() % 4) pool.push_back(0.f);
+  return off;
+}
+
+}  // namespace
+
+bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
+                    std::vector<float>& params, TcChainDesc& d) {
+  const Node& root = ir.nodes[s.out];
+  if (root.role != ROLE_FCONV) return false;
+  const int tsrc = ir.oin[s.out][0];
+  const Node& tn = ir.nodes[tsrc];
+  const int C = tn.C, Nout = root.C;
+  if (Nout % 8 || Nout > 256) return false;
+  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
+  P.members.erase(s.out);
+  std::vector<PLevel> levels;
+  if (!P.chain(tsrc, levels)) return false;
+  if (P.visited != P.members) return false;          // every member must be part of the chain form
+  int nterms = 0;
+  for (auto& L : levels) nterms += (int)L.terms.size();
+  if ((int)levels.size() > kTcMaxLevels || nterms > kTcMaxTerms) return false;
+  // term inputs: bf16 reduced tensors in the arena, ranks % 8 == 0
+  for (auto& L : levels)
+    for (auto& t : L.terms) {
+      const int r = ir.oin[t.lconv][0];
+      const Loc& l = loc.at(r);
+      if (l.where != W_ARENA || l.dtype != DT_BF16 || ir.nodes[r].C % 8) return false;
+    }
+  const Loc& yl = loc.at(s.out);
+  if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
+
+  d = TcChainDesc();
+  d.C = C;
+  d.Cc = C <= 64 ? 64 : 128;
+  d.Cpad = (C + d.Cc - 1) / d.Cc * d.Cc;
+  d.nchunks = d.Cpad / d.Cc;
+  d.Nout = Nout;
+  d.Np = (Nout + 15) / 16 * 16;
+  d.npix = (int64_t)ir.batch * tn.H * tn.W;
+  d.ntiles = (int)((d.npix + 127) / 128);
+  d.y = yl;
+  d.n_levels = (int)levels.size();
+  int64_t flops_terms = 0, bytes_terms = 0;
+  int j = 0;
+  for (int l = 0; l < d.n_levels; ++l) {
+    const PLevel& L = levels[l];
+    d.relu[l] = L.relu ? 1 : 0;
+    std::vector<double> bias(d.Cpad, 0.0);
+    std::copy(L.bias.begin(), L.bias.end(), bias.begin());
+    d.bias[l] = push_f32(params, bias);
+    for (const PTerm& t : L.terms) {
+      const Node& lc = ir.nodes[t.lconv];
+      const int r = ir.oin[t.lconv][0];
+      const int R = ir.nodes[r].C;
+      TcTerm& T = d.term[j++];
+      T.r = loc.at(r);
+      T.R = R;
+      T.Rp = (R + 63) / 64 * 64;
+      T.c0 = t.c0;
+      T.C = lc.C;
+      std::vector<float> w((size_t)d.Cpad * T.Rp, 0.f);
+      for (int c = 0; c < lc.C; ++c)
+        for (int k = 0; k < R; ++k)
+          w[(size_t)(t.c0 + c) * T.Rp + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
+      T.w = push_bf16(tcw, w);
+      flops_terms += 2LL * lc.C * R;
+      bytes_terms += 2LL * R;
+    }
+    d.lvl_end[l] = j;
+  }
+  d.n_terms = j;
+  std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
+  for (int o = 0; o < Nout; ++o)
+    for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
+  d.F = push_bf16(tcw, f);
+  d.Fb = -1;
+  if (root.b) {
+    std::vector<double> fb(root.b->begin(), root.b->end());
+    d.Fb = push_f32(params, fb);
+  }
+  d.alg_flops = d.npix * (flops_terms + 2LL * Nout * C);
+  d.alg_bytes = d.npix * (bytes_terms + 2LL * Nout);
+  // shared memory: ring of (A 16 KB | B slot) stages + two P tiles + barriers
+  d.slot_b = std::max(d.Cc, d.Np) * 128;
+  const int pbytes = 128 * d.Cc * 2;
+  const int budget = 227 * 1024 - 1024 /*align*/ - 512 /*barriers*/ - 2 * pbytes;
+  d.stages = std::min(6, budget / (16384 + d.slot_b));
+  if (d.stages < 2) return false;
+  d.smem_bytes = 1024 + d.stages * (16384 + d.slot_b) + 2 * pbytes + 512;
+  const int cols = 2 * d.Cc + d.Np;
+  d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
+  return true;
+}
+
+bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char* arena, uint16_t* tcw,
+                 std::string& err) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  bool any = false;
+  for (size_t i = 0; i < n; ++i) any |= get(i) != nullptr;
+  if (!any) return true;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
+      err = "cuTensorMapEncodeTiled unavailable";
+      return false;
+    }
+    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  auto make = [&](unsigned char* dst, void* base, uint64_t inner, uint64_t outer, uint32_t box_outer) {
+    cuuint64_t dims[2] = {inner, outer};
+    cuuint64_t strides[1] = {inner * 2};
+    cuuint32_t box[2] = {64, box_outer};
+    cuuint32_t es[2] = {1, 1};
+    CUresult r = encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, base, dims, strides,
+                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+  };
+  for (size_t i = 0; i < n; ++i) {
+    TcChainDesc* d = get(i);
+    if (!d) continue;
+    for (int j = 0; j < d->n_terms; ++j) {
+      TcTerm& t = d->term[j];
+      if (!make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->npix, 128) ||
+          !make(t.wmap, tcw + t.w, (uint64_t)t.Rp, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+        err = "cuTensorMapEncodeTiled failed (term)";
+        return false;
+      }
+    }
+    if (!make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
+      err = "cuTensorMapEncodeTiled failed (F)";
+      return false;
+    }
+  }
+  return true;
+}
+
+// ===========================================================================
+// device
+// ===========================================================================
+namespace {
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void tma_load_2d(void* dst, const void* map, uint64_t* bar, int x, int y) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y)
+      : "memory");
+}
+
+// K-major, 128-byte swizzle UMMA shared-memory descriptor (8-row groups 1024 B apart)
+__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
+  return (uint64_t)((saddr & 0x3FFFF) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+
+// kind::f16 instruction descriptor: bf16 A/B, fp32 D, K-major A/B
+__host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+
+__device__ __forceinline__ void mma_bf16(uint32_t dtmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(dtmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
+}
+
+__device__ __forceinline__ void mma_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+#define TMEM_REGS32(v)                                                                                            \
+  "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),       \
+      "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]),        \
+      "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]),       \
+      "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
+      "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+      : TMEM_REGS32(v)
+      : "r"(taddr));
+}
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+      "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31, %32};" ::"r"(taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]), "r"(v[17]), "r"(v[18]),
+      "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]),
+      "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
+      : "memory");
+}
+
+__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8]) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "r"(taddr));
+}
+
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+__device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
+  return t.c0 < (c + 1) * Cc && t.c0 + t.C > c * Cc;
+}
+
+constexpr int kThreads = 192;
+constexpr int kSlotA = 16384;
+
+__global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  const int S = d.stages;
+  const int slot = kSlotA + d.slot_b;
+  const int Cc = d.Cc;
+  const int pbytes = 128 * Cc * 2;
+  uint8_t* ring = smem;
+  uint8_t* pbuf = ring + S * slot;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(pbuf + 2 * pbytes);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + S;
+  uint64_t* acc_full = bars + 2 * S;
+  uint64_t* acc_empty = acc_full + 2;
+  uint64_t* p_full = acc_empty + 2;
+  uint64_t* p_empty = p_full + 2;
+  uint64_t* out_full = p_empty + 2;
+  uint64_t* out_empty = out_full + 1;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(out_empty + 1);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&acc_full[b], 1);
+      mbar_init(&acc_empty[b], 128);
+      mbar_init(&p_full[b], 128);
+      mbar_init(&p_empty[b], 1);
+    }
+    mbar_init(out_full, 1);
+    mbar_init(out_empty, 128);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(d.tmem_cols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_slot;
+
+  if (warp == 4) {
+    // ------------------------------------------------------------ TMA producer
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      const uint32_t bytes_g1 = kSlotA + Cc * 128, bytes_g2 = d.Np * 128;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+        const int m0 = tile * 128;
+        for (int pc = 0; pc < d.nchunks; pc += 2) {
+          const int nb = min(2, d.nchunks - pc);
+          for (int l = 0; l < d.n_levels; ++l)
+            for (int bi = 0; bi < nb; ++bi) {
+              const int c = pc + bi;
+              for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
+                const TcTerm& t = d.term[j];
+                if (!term_hits(t, c, Cc)) continue;
+                for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                  mbar_wait(&empty[stage], phase ^ 1);
+                  mbar_expect_tx(&full[stage], bytes_g1);
+                  uint8_t* sa = ring + stage * slot;
+                  tma_load_2d(sa, t.tmap, &full[stage], ka * 64, m0);
+                  tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * 64, c * Cc);
+                  if (++stage == S) stage = 0, phase ^= 1;
+                }
+              }
+            }
+          for (int bi = 0; bi < nb; ++bi) {
+            const int c = pc + bi;
+            for (int a = 0; a < Cc / 64; ++a) {
+              mbar_wait(&empty[stage], phase ^ 1);
+              mbar_expect_tx(&full[stage], bytes_g2);
+              tma_load_2d(ring + stage * slot + kSlotA, d.fmap, &full[stage], c * Cc + a * 64, 0);
+              if (++stage == S) stage = 0, phase ^= 1;
+            }
+          }
+        }
+      }
+    }
+  } else if (warp == 5) {
+    // ------------------------------------------------------------ MMA issuer
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      uint32_t acc_use[2] = {0, 0}, p_use[2] = {0, 0}, tile_iter = 0;
+      const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
+      const uint32_t tout = tbase + 2 * Cc;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+        for (int pc = 0; pc < d.nchunks; pc += 2) {
+          const int nb = min(2, d.nchunks - pc);
+          for (int l = 0; l < d.n_levels; ++l)
+            for (int bi = 0; bi < nb; ++bi) {
+              const int c = pc + bi;
+              mbar_wait(&acc_empty[bi], (acc_use[bi] & 1) ^ 1);
+              tc_fence_after();
+              const uint32_t tacc = tbase + bi * Cc;
+              bool first = (l == 0);
+              for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
+                const TcTerm& t = d.term[j];
+                if (!term_hits(t, c, Cc)) continue;
+                for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                  mbar_wait(&full[stage], phase);
+                  tc_fence_after();
+                  const uint32_t sa = smem_u32(ring + stage * slot);
+                  const int nk = min(4, (t.R - ka * 64 + 15) / 16);
+                  for (int k = 0; k < nk; ++k) {
+                    mma_bf16(tacc, umma_desc(sa + 32 * k), umma_desc(sa + kSlotA + 32 * k), id1, first ? 0u : 1u);
+                    first = false;
+                  }
+                  mma_commit(&empty[stage]);
+                  if (++stage == S) stage = 0, phase ^= 1;
+                }
+              }
+              mma_commit(&acc_full[bi]);
+              ++acc_use[bi];
+            }
+          for (int bi = 0; bi < nb; ++bi) {
+            const int c = pc + bi;
+            mbar_wait(&p_full[bi], p_use[bi] & 1);
+            tc_fence_after();
+            if (c == 0) {
+              mbar_wait(out_empty, (tile_iter & 1) ^ 1);
+              tc_fence_after();
+            }
+            const uint32_t pa = smem_u32(pbuf + bi * pbytes);
+            for (int a = 0; a < Cc / 64; ++a) {
+              mbar_wait(&full[stage], phase);
+              tc_fence_after();
+              const uint32_t sb = smem_u32(ring + stage * slot + kSlotA);
+              for (int k = 0; k < 4; ++k)
+                mma_bf16(tout, umma_desc(pa + a * 16384 + 32 * k), umma_desc(sb + 32 * k), id2,
+                         (c > 0 || a > 0 || k > 0) ? 1u : 0u);
+              mma_commit(&empty[stage]);
+              if (++stage == S) stage = 0, phase ^= 1;
+            }
+            mma_commit(&p_empty[bi]);
+            ++p_use[bi];
+          }
+        }
+        mma_commit(out_full);
+        ++tile_iter;
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue (128 threads)
+    const int row = threadIdx.x;                       // pixel row in the tile == TMEM lane
+    const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+    uint32_t acc_use[2] = {0, 0}, p_use[2] = {0, 0}, tile_iter = 0;
+    __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+      const int64_t m = (int64_t)tile * 128 + row;
+      for (int pc = 0; pc < d.nchunks; pc += 2) {
+        const int nb = min(2, d.nchunks - pc);
+        for (int l = 0; l < d.n_levels; ++l) {
+          const bool last = l == d.n_levels - 1;
+          const bool relu = d.relu[l] != 0;
+          for (int bi = 0; bi < nb; ++bi) {
+            const int c = pc + bi;
+            mbar_wait(&acc_full[bi], acc_use[bi] & 1);
+            ++acc_use[bi];
+            tc_fence_after();
+            if (last) {
+              mbar_wait(&p_empty[bi], (p_use[bi] & 1) ^ 1);
+              ++p_use[bi];
+            }
+            const float* bias = p.params + d.bias[l] + (int64_t)c * Cc;
+            uint8_t* P = pbuf + bi * pbytes;
+            for (int g = 0; g < Cc / 32; ++g) {
+              const uint32_t ta = tbase + lane_off + bi * Cc + g * 32;
+              uint32_t v[32];
+              tmem_ld32(ta, v);
+              tmem_wait_ld();
+              float f[32];
+#pragma unroll
+              for (int i = 0; i < 32; ++i) {
+                float x = __uint_as_float(v[i]) + __ldg(bias + g * 32 + i);
+                f[i] = relu ? fmaxf(x, 0.f) : x;
+              }
+              if (!last) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = __float_as_uint(f[i]);
+                tmem_st32(ta, v);
+              } else {
+                const int col = g * 32;                     // within the chunk
+                uint8_t* atom = P + (col / 64) * 16384 + row * 128;
+                const int ch0 = (col % 64) / 8;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                  uint4 pk;
+                  pk.x = pack_bf16(f[8 * q + 0], f[8 * q + 1]);
+                  pk.y = pack_bf16(f[8 * q + 2], f[8 * q + 3]);
+                  pk.z = pack_bf16(f[8 * q + 4], f[8 * q + 5]);
+                  pk.w = pack_bf16(f[8 * q + 6], f[8 * q + 7]);
+                  *reinterpret_cast<uint4*>(atom + (((ch0 + q) ^ (row & 7)) * 16)) = pk;
+                }
+              }
+            }
+            if (!last) tmem_wait_st();
+            tc_fence_before();
+            mbar_arrive(&acc_empty[bi]);
+            if (last) {
+              asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+              mbar_arrive(&p_full[bi]);
+            }
+          }
+        }
+      }
+      // output epilogue
+      mbar_wait(out_full, tile_iter & 1);
+      ++tile_iter;
+      tc_fence_after();
+      for (int g = 0; g < d.Np / 8; ++g) {
+        uint32_t v[8];
+        tmem_ld8(tbase + lane_off + 2 * Cc + g * 8, v);
+        tmem_wait_ld();
+        if (m < d.npix && g * 8 < d.Nout) {
+          float f[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.Fb >= 0 ? __ldg(p.params + d.Fb + g * 8 + i) : 0.f);
+          uint4 pk;
+          pk.x = pack_bf16(f[0], f[1]);
+          pk.y = pack_bf16(f[2], f[3]);
+          pk.z = pack_bf16(f[4], f[5]);
+          pk.w = pack_bf16(f[6], f[7]);
+          *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) = pk;
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(out_empty);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase), "r"(d.tmem_cols));
+  }
+}
+
+}  // namespace
+
+void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  (void)tcw;
+  static bool configured = false;
+  if (!configured) {
+    cudaFuncSetAttribute(tc_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    configured = true;
+  }
+  int sms = 148;
+  static int dev_sms = 0;
+  if (!dev_sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  sms = dev_sms > 0 ? dev_sms : 148;
+  const int grid = std::min(d.ntiles, sms);
+  // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
+  tc_chain_kernel<<<grid, kThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+}
 
 }  // namespace temco

@@ -1,4 +1,12 @@
-// tcgen05 fused-group kernels (kernels_tc.cu): lowering + launch interface.
+// tcgen05 fused-group kernel (kernels_tc.cu): lowering + launch interface.
+//
+// Covers the groups whose restored tensor is a "level chain" (reading R12,
+// P:L305-317 + P:L321-333):
+//     t_1 = act_1( sum_{j in 1} Lhat_j r_j + b_1 )
+//     t_l = act_l( sum_{j in l} Lhat_j r_j + b_l + t_{l-1} )      l = 2..D
+// (Lhat = BN-folded lconv rows; a concat of lconvs is one level whose terms
+// write disjoint channel ranges, Fig. 9a) followed by the root fconv
+// out = F t_D.  All terms at the root resolution, bf16 ranks % 8 == 0.
 #pragma once
 
 #include <cuda_runtime.h>
@@ -18,28 +26,31 @@ constexpr int kTcMaxTerms = 16;    // reduced inputs (lconv leaves) per group
 constexpr int kTcMaxLevels = 16;
 
 struct TcTerm {
-  Loc r;                 // reduced input [N*H*W, R] bf16
-  int32_t R, Rp;         // rank, padded to a multiple of 64 (K atoms)
-  int32_t level;         // chain level this term accumulates into
-  int32_t c0, C;         // restored channel range it writes (concat members)
-  int64_t w;             // tc weight pool offset (elements): [C_total_rows][Rp] bf16, K-major
-  alignas(64) unsigned char tmap[128];   // CUtensorMap of r (filled by tc_finalize)
-  alignas(64) unsigned char wmap[128];   // CUtensorMap of the weight block
+  alignas(64) unsigned char tmap[128];   // CUtensorMap of r  [npix x R], box {64, 128}
+  alignas(64) unsigned char wmap[128];   // CUtensorMap of Lhat [Cpad x Rp], box {64, Cc}
+  Loc r;                 // reduced input [npix, R] bf16 (arena)
+  int32_t R, Rp;         // rank; padded to a multiple of 64 (one 128-byte K atom)
+  int32_t c0, C;         // restored channels this term writes (concat members)
+  int64_t w;             // tc weight pool offset (elements)
 };
 
 struct TcChainDesc {
-  int32_t n_terms, n_levels;
-  int32_t Ctot;          // restored width C
-  int32_t Nout, Np;      // fconv outputs and padded (multiple of 16)
-  int64_t npix;
-  int32_t relu[kTcMaxLevels];
-  int64_t bias[kTcMaxLevels];   // params offsets [C] fp32 (folded), -1 none
-  int64_t F;             // tc weight pool offset: [Np][Cpad] bf16
-  int32_t Cpad;          // C padded to a multiple of the chunk
-  Loc y;                 // output [npix, Nout] (plan dtype)
-  int64_t alg_flops, alg_bytes;
   TcTerm term[kTcMaxTerms];
-  alignas(64) unsigned char fmap[128];
+  alignas(64) unsigned char fmap[128];   // CUtensorMap of F [Np x Cpad], box {64, Np}
+  int32_t n_terms, n_levels;
+  int32_t lvl_end[kTcMaxLevels];         // terms [lvl_end[l-1], lvl_end[l]) accumulate into level l
+  int32_t relu[kTcMaxLevels];
+  int64_t bias[kTcMaxLevels];            // params offset: fp32 [Cpad] (folded BN shift + lconv biases)
+  int32_t C, Cpad, Cc, nchunks;          // restored width, padded, chunk width (64 | 128)
+  int32_t Nout, Np;                      // fconv outputs, padded to a multiple of 16
+  int64_t npix;
+  int32_t ntiles;
+  int64_t F;                             // tc weight pool offset of F
+  int64_t Fb;                            // params offset of the fconv bias or -1
+  Loc y;                                 // output [npix, Nout] bf16
+  int32_t stages, slot_b;                // smem ring depth, bytes of one B slot
+  int32_t smem_bytes, tmem_cols;
+  int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
 };
 
 bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
