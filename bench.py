@@ -242,8 +242,8 @@ def main():
             continue
         c = classes.setdefault(k, {"ms": 0.0, "flops": 0, "bytes": 0, "launches": 0})
         c["ms"] += float(t)
-        c["flops"] += s.get("tc_flops", s["flops"])
-        c["bytes"] += s.get("tc_bytes", s["io_bytes"])
+        c["flops"] += s.get("alg_flops", s["flops"])
+        c["bytes"] += s.get("alg_bytes", s["io_bytes"])
         c["launches"] += s["launches"]
     hbm, tf_burst, tf_sust, src = _peaks()
     dom = max(classes, key=lambda k: classes[k]["ms"])

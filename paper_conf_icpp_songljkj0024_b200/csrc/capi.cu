@@ -13,6 +13,7 @@
 
 #include "kernels.h"
 #include "planner.h"
+#include "conv_tc.h"
 #include "tc.h"
 
 using namespace temco;
@@ -32,7 +33,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC };
 
 struct StepExec {
   int kind = K_NONE;
@@ -41,6 +42,7 @@ struct StepExec {
   LinearDesc lin{};
   GroupDesc grp{};
   TcChainDesc tc{};
+  ConvTcDesc ctc{};
   std::string kernel;
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
@@ -296,6 +298,13 @@ void lower(temco_plan_s* P) {
         e.kernel = "none";
         break;
       case OP_CONV: {
+        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+            conv_tc_lower(ir, s.out, P->loc, P->tcw_h, P->params_h, e.ctc)) {
+          e.kind = K_CONV_TC;
+          e.kernel = "tc_conv";
+          e.launches = 1;
+          break;
+        }
         const Node& x = ir.nodes[ir.oin[s.out][0]];
         ConvDesc& c = e.conv;
         c.x = tensor_loc(P, x.id);
@@ -406,7 +415,8 @@ std::string make_json(const temco_plan_s* P) {
       const StepExec& e = P->exec[t];
       o << ",\"kernel\":\"" << e.kernel << "\",\"flops\":" << e.flops << ",\"io_bytes\":" << e.io_bytes
         << ",\"launches\":" << e.launches;
-      if (e.kind == K_GROUP_TC) o << ",\"tc_flops\":" << e.tc.alg_flops << ",\"tc_bytes\":" << e.tc.alg_bytes;
+      if (e.kind == K_GROUP_TC) o << ",\"alg_flops\":" << e.tc.alg_flops << ",\"alg_bytes\":" << e.tc.alg_bytes;
+      if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
     }
     o << ",\"live\":" << ir.live_fused[t] << "}";
   }
@@ -451,6 +461,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
       case K_LINEAR: launch_linear(e.lin, rp, st); break;
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
+      case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
     }
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t + 1], st));
   }
@@ -561,6 +572,12 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
       return set_err(TEMCO_ERR_OUT_OF_MEMORY, "arena cudaMalloc");
     }
     std::string terr;
+    for (auto& e : P->exec)
+      if (e.kind == K_CONV_TC && !conv_tc_finalize(e.ctc, P->tcw_d, terr)) {
+        free_device(P);
+        delete P;
+        return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
+      }
     if (!tc_finalize(P->exec.size(), [&](size_t i) -> TcChainDesc* {
           return P->exec[i].kind == K_GROUP_TC ? &P->exec[i].tc : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {

@@ -1,0 +1,302 @@
+// tcgen05 implicit-GEMM convolution (see conv_tc.h).
+//
+// Per 128-output-pixel tile: the im2col rows are gathered straight from the
+// NHWC input into the SW128 K-major SMEM layout (4 gather warps, 16-byte
+// cp.async with zero-fill for padding taps, completion signalled on an
+// mbarrier), the whole weight matrix stays resident in SMEM (one TMA load per
+// CTA), one thread issues tcgen05.mma (M=128, N=Np, K=16) into one of two TMEM
+// accumulators, and 4 epilogue warps drain TMEM -> bias -> bf16 -> global while
+// the next tile accumulates.  The small-rank convolutions are HBM-bound (AI ~
+// 25-40 flop/B); the tensor cores only have to keep up with the gather.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+
+#include "conv_tc.h"
+#include "tc_ptx.cuh"
+
+namespace temco {
+
+namespace {
+
+uint16_t f2bf(float f) {
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  u += 0x7FFF + ((u >> 16) & 1);
+  return (uint16_t)(u >> 16);
+}
+
+}  // namespace
+
+bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
+                   std::vector<float>& params, ConvTcDesc& d) {
+  const Node& v = ir.nodes[out];
+  if (v.op != OP_CONV || v.groups != 1) return false;
+  const Node& x = ir.nodes[ir.oin[out][0]];
+  const Loc& xl = loc.at(x.id);
+  const Loc& yl = loc.at(out);
+  if (xl.dtype != DT_BF16 || yl.dtype != DT_BF16 || yl.where != W_ARENA) return false;
+  if (v.C % 8 || v.C > 256) return false;
+  d = ConvTcDesc();
+  d.x = xl;
+  d.y = yl;
+  d.N = ir.batch; d.H = x.H; d.W = x.W; d.Cin = x.C;
+  d.Ho = v.H; d.Wo = v.W; d.kh = v.kh; d.kw = v.kw; d.sh = v.sh; d.sw = v.sw; d.ph = v.ph; d.pw = v.pw;
+  d.Nout = v.C;
+  d.Np = (v.C + 15) / 16 * 16;
+  d.vec = x.C % 8 == 0 ? 1 : 0;
+  d.K = v.kh * v.kw * x.C;
+  d.kchunks = (d.K + 7) / 8;
+  d.katoms = (d.K + 63) / 64;
+  d.npix = (int64_t)ir.batch * v.H * v.W;
+  d.ntiles = (int)((d.npix + 127) / 128);
+  const int wbytes = d.katoms * d.Np * 128;
+  if (wbytes > 112 * 1024) return false;
+  // weights [Np][katoms*64] bf16, k = (a*kw + b)*Cin + c
+  const int Kp = d.katoms * 64;
+  std::vector<uint16_t> w((size_t)d.Np * Kp, 0);
+  const std::vector<float>& src = *v.w;   // OIHW
+  for (int o = 0; o < v.C; ++o)
+    for (int c = 0; c < x.C; ++c)
+      for (int a = 0; a < v.kh; ++a)
+        for (int b = 0; b < v.kw; ++b)
+          w[(size_t)o * Kp + (a * v.kw + b) * x.C + c] = f2bf(src[(((size_t)o * x.C + c) * v.kh + a) * v.kw + b]);
+  while (tcw.size() % 512) tcw.push_back(0);
+  d.w = (int64_t)tcw.size();
+  tcw.insert(tcw.end(), w.begin(), w.end());
+  d.b = -1;
+  if (v.b) {
+    while (params.size() % 4) params.push_back(0.f);
+    d.b = (int64_t)params.size();
+    params.insert(params.end(), v.b->begin(), v.b->end());
+  }
+  d.stages = std::min(8, (220 * 1024 - wbytes) / 16384);
+  if (d.stages < 2) return false;
+  d.smem_bytes = 1024 + wbytes + d.stages * 16384 + 256;
+  const int cols = 2 * d.Np;
+  d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
+  d.alg_flops = 2 * d.npix * (int64_t)d.K * d.Nout;
+  d.alg_bytes = 2 * ((int64_t)d.N * d.H * d.W * d.Cin + d.npix * d.Nout);
+  return true;
+}
+
+bool conv_tc_finalize(ConvTcDesc& d, uint16_t* tcw, std::string& err) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
+      err = "cuTensorMapEncodeTiled unavailable";
+      return false;
+    }
+    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  const uint64_t Kp = (uint64_t)d.katoms * 64;
+  cuuint64_t dims[2] = {Kp, (cuuint64_t)d.Np};
+  cuuint64_t strides[1] = {Kp * 2};
+  cuuint32_t box[2] = {64, (cuuint32_t)d.Np};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = encode(reinterpret_cast<CUtensorMap*>(d.wmap), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, tcw + d.w, dims,
+                      strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    err = "cuTensorMapEncodeTiled failed (conv weights)";
+    return false;
+  }
+  return true;
+}
+
+namespace {
+
+using namespace ptx;
+
+constexpr int kConvThreads = 288;   // warps 0-3 epilogue, 4-7 gather, 8 MMA
+
+__global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_constant__ ConvTcDesc d, RunPtrs p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  const int S = d.stages;
+  const int wbytes = d.katoms * d.Np * 128;
+  uint8_t* wres = smem;
+  uint8_t* ring = smem + wbytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ring + S * 16384);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + S;
+  uint64_t* acc_full = bars + 2 * S;
+  uint64_t* acc_empty = acc_full + 2;
+  uint64_t* wbar = acc_empty + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wbar + 1);
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 128);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&acc_full[b], 1);
+      mbar_init(&acc_empty[b], 128);
+    }
+    mbar_init(wbar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(d.tmem_cols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_slot;
+  const int hw = d.Ho * d.Wo;
+
+  if (warp >= 4 && warp < 8) {
+    // ------------------------------------------------------------ im2col gather
+    const int g = threadIdx.x - 128;     // A row
+    const uint8_t* x = static_cast<const uint8_t*>(loc_ptr(d.x, p));
+    int stage = 0;
+    uint32_t phase = 0;
+    const int cpt = d.Cin / 8;           // 16-byte chunks per tap (vec path)
+    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+      const int64_t m = (int64_t)tile * 128 + g;
+      const bool mv = m < d.npix;
+      const int n = mv ? (int)(m / hw) : 0;
+      const int rem = mv ? (int)(m % hw) : 0;
+      const int hb = (rem / d.Wo) * d.sh - d.ph, wb = (rem % d.Wo) * d.sw - d.pw;
+      const int64_t img = (int64_t)n * d.H * d.W;
+      for (int kb = 0; kb < d.katoms; ++kb) {
+        mbar_wait(&empty[stage], phase ^ 1);
+        uint8_t* dst = ring + stage * 16384 + g * 128;
+        if (d.vec) {
+#pragma unroll
+          for (int q = 0; q < 8; ++q) {
+            const int kc = kb * 8 + q;
+            const uint8_t* src = x;
+            uint32_t bytes = 0;
+            if (mv && kc < d.kchunks) {
+              const int tap = kc / cpt, cc = kc - tap * cpt;
+              const int hi = hb + tap / d.kw, wi = wb + tap % d.kw;
+              if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W) {
+                src = x + ((img + (int64_t)hi * d.W + wi) * d.Cin + cc * 8) * 2;
+                bytes = 16;
+              }
+            }
+            cp_async16(dst + ((q ^ (g & 7)) * 16), src, bytes);
+          }
+          cp_async_arrive(&full[stage]);
+        } else {
+          const __nv_bfloat16* xb = reinterpret_cast<const __nv_bfloat16*>(x);
+#pragma unroll 1
+          for (int q = 0; q < 8; ++q) {
+            uint32_t pk[4];
+#pragma unroll
+            for (int e2 = 0; e2 < 4; ++e2) {
+              float f[2];
+#pragma unroll
+              for (int h = 0; h < 2; ++h) {
+                const int k = (kb * 8 + q) * 8 + e2 * 2 + h;
+                f[h] = 0.f;
+                if (mv && k < d.K) {
+                  const int tap = k / d.Cin, c = k - tap * d.Cin;
+                  const int hi = hb + tap / d.kw, wi = wb + tap % d.kw;
+                  if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W)
+                    f[h] = __bfloat162float(xb[(img + (int64_t)hi * d.W + wi) * d.Cin + c]);
+                }
+              }
+              pk[e2] = pack_bf16(f[0], f[1]);
+            }
+            *reinterpret_cast<uint4*>(dst + ((q ^ (g & 7)) * 16)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+          }
+          fence_proxy_async();
+          mbar_arrive(&full[stage]);
+        }
+        if (++stage == S) stage = 0, phase ^= 1;
+      }
+    }
+  } else if (warp == 8) {
+    // ------------------------------------------------------------ weights + MMA issuer
+    if (lane == 0) {
+      mbar_expect_tx(wbar, wbytes);
+      for (int kb = 0; kb < d.katoms; ++kb) tma_load_2d(wres + kb * d.Np * 128, d.wmap, wbar, kb * 64, 0);
+      mbar_wait(wbar, 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      const uint32_t id = idesc_bf16(128, d.Np);
+      int it = 0;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+        const int buf = it & 1;
+        mbar_wait(&acc_empty[buf], ((it >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t tacc = tbase + buf * d.Np;
+        for (int kb = 0; kb < d.katoms; ++kb) {
+          mbar_wait(&full[stage], phase);
+          fence_proxy_async();
+          tc_fence_after();
+          const uint32_t sa = smem_u32(ring + stage * 16384);
+          const uint32_t sb = smem_u32(wres + kb * d.Np * 128);
+          const int nk = min(4, (d.K - kb * 64 + 15) / 16);
+          for (int k = 0; k < nk; ++k)
+            mma_bf16(tacc, umma_desc(sa + 32 * k), umma_desc(sb + 32 * k), id, (kb | k) ? 1u : 0u);
+          mma_commit(&empty[stage]);
+          if (++stage == S) stage = 0, phase ^= 1;
+        }
+        mma_commit(&acc_full[buf]);
+      }
+    }
+  } else {
+    // ------------------------------------------------------------ epilogue
+    const int row = threadIdx.x;
+    const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+    __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+    int it = 0;
+    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+      const int buf = it & 1;
+      mbar_wait(&acc_full[buf], (it >> 1) & 1);
+      tc_fence_after();
+      const int64_t m = (int64_t)tile * 128 + row;
+      for (int g = 0; g < d.Np / 8; ++g) {
+        uint32_t v[8];
+        tmem_ld8(tbase + lane_off + buf * d.Np + g * 8, v);
+        tmem_wait_ld();
+        if (m < d.npix && g * 8 < d.Nout) {
+          float f[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.b >= 0 ? __ldg(p.params + d.b + g * 8 + i) : 0.f);
+          *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) =
+              make_uint4(pack_bf16(f[0], f[1]), pack_bf16(f[2], f[3]), pack_bf16(f[4], f[5]), pack_bf16(f[6], f[7]));
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[buf]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase), "r"(d.tmem_cols));
+  }
+}
+
+}  // namespace
+
+void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 0;
+  if (!configured) {
+    cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  // two CTAs per SM when TMEM (<= 256 columns each) and SMEM allow it
+  const bool two = d.tmem_cols <= 256 && d.smem_bytes <= 110 * 1024;
+  const int grid = std::min(d.ntiles, (sms > 0 ? sms : 148) * (two ? 2 : 1));
+  conv_tc_kernel<<<grid, kConvThreads, two ? d.smem_bytes : std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+}
+
+}  // namespace temco

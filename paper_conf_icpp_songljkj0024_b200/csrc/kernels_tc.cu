@@ -24,6 +24,7 @@
 #include <set>
 
 #include "tc.h"
+#include "tc_ptx.cuh"
 
 namespace temco {
 
@@ -153,15 +154,26 @@ int64_t push_f32(std::vector<float>& pool, const std::vector<double>& v) {
 bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                     std::vector<float>& params, TcChainDesc& d) {
   const Node& root = ir.nodes[s.out];
-  if (root.role != ROLE_FCONV) return false;
+  const bool gap = root.op == OP_GAP;
+  if (root.role != ROLE_FCONV && !gap) return false;
   const int tsrc = ir.oin[s.out][0];
   const Node& tn = ir.nodes[tsrc];
-  const int C = tn.C, Nout = root.C;
+  const int C = tn.C, Nout = gap ? 16 : root.C;
   if (Nout % 8 || Nout > 256) return false;
-  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
+  if (gap && tn.H * tn.W > 128) return false;
+  // pooled chain (Listing 1 with p >= 2): root fconv <- max/avg pool <- level chain
+  int pool = 0, pk = 1, ps = 1, pp = 0, csrc = tsrc;
+  if (!gap && (tn.op == OP_MAXPOOL || tn.op == OP_AVGPOOL) && s.members.size() > 2) {
+    pool = tn.op == OP_MAXPOOL ? 1 : 2;
+    pk = tn.kh; ps = tn.sh; pp = tn.ph;
+    csrc = ir.oin[tsrc][0];
+  }
+  const Node& cn = ir.nodes[csrc];
+  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, cn.H, cn.W};
   P.members.erase(s.out);
+  if (pool) P.members.erase(tsrc);
   std::vector<PLevel> levels;
-  if (!P.chain(tsrc, levels)) return false;
+  if (!P.chain(csrc, levels)) return false;
   if (P.visited != P.members) return false;          // every member must be part of the chain form
   int nterms = 0;
   for (auto& L : levels) nterms += (int)L.terms.size();
@@ -178,13 +190,27 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
 
   d = TcChainDesc();
   d.C = C;
-  d.Cc = C <= 64 ? 64 : 128;
+  d.Cc = (C <= 64 || pool) ? 64 : 128;
+  d.gather = pool ? 1 : 0;
+  d.pool = pool; d.pk = pk; d.ps = ps; d.pp = pp; d.taps = pk * pk;
+  d.Hin = cn.H; d.Win = cn.W; d.Ho = tn.H; d.Wo = tn.W;
   d.Cpad = (C + d.Cc - 1) / d.Cc * d.Cc;
   d.nchunks = d.Cpad / d.Cc;
   d.Nout = Nout;
   d.Np = (Nout + 15) / 16 * 16;
   d.npix = (int64_t)ir.batch * tn.H * tn.W;
-  d.ntiles = (int)((d.npix + 127) / 128);
+  d.nimg = ir.batch;
+  d.gap = gap ? 1 : 0;
+  d.hw = tn.H * tn.W;
+  if (gap) {
+    d.ipt = 128 / d.hw;
+    d.rows_per_tile = d.ipt * d.hw;
+    d.ntiles = (ir.batch + d.ipt - 1) / d.ipt;
+  } else {
+    d.ipt = 0;
+    d.rows_per_tile = 128;
+    d.ntiles = (int)((d.npix + 127) / 128);
+  }
   d.y = yl;
   d.n_levels = (int)levels.size();
   int64_t flops_terms = 0, bytes_terms = 0;
@@ -216,17 +242,24 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.lvl_end[l] = j;
   }
   d.n_terms = j;
-  std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
-  for (int o = 0; o < Nout; ++o)
-    for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
-  d.F = push_bf16(tcw, f);
   d.Fb = -1;
-  if (root.b) {
-    std::vector<double> fb(root.b->begin(), root.b->end());
-    d.Fb = push_f32(params, fb);
+  if (gap) {
+    d.F = 0;
+    d.alg_flops = d.npix * (flops_terms + C);
+    d.alg_bytes = d.npix * bytes_terms + 2LL * ir.batch * C;
+  } else {
+    std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
+    for (int o = 0; o < Nout; ++o)
+      for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
+    d.F = push_bf16(tcw, f);
+    if (root.b) {
+      std::vector<double> fb(root.b->begin(), root.b->end());
+      d.Fb = push_f32(params, fb);
+    }
+    const int64_t nin = (int64_t)ir.batch * cn.H * cn.W;   // chain evaluated once per input pixel
+    d.alg_flops = nin * flops_terms + d.npix * 2LL * Nout * C;
+    d.alg_bytes = nin * bytes_terms + d.npix * 2LL * Nout;
   }
-  d.alg_flops = d.npix * (flops_terms + 2LL * Nout * C);
-  d.alg_bytes = d.npix * (bytes_terms + 2LL * Nout);
   // shared memory: ring of (A 16 KB | B slot) stages + two P tiles + barriers
   d.slot_b = std::max(d.Cc, d.Np) * 128;
   const int pbytes = 128 * d.Cc * 2;
@@ -275,7 +308,7 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
         return false;
       }
     }
-    if (!make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
+    if (!d->gap && !make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
       err = "cuTensorMapEncodeTiled failed (F)";
       return false;
     }
@@ -287,117 +320,46 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
 // device
 // ===========================================================================
 namespace {
-
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
-}
-
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra WAIT_%=;\n"
-      "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-
-__device__ __forceinline__ void tma_load_2d(void* dst, const void* map, uint64_t* bar, int x, int y) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
-          smem_u32(dst)),
-      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y)
-      : "memory");
-}
-
-// K-major, 128-byte swizzle UMMA shared-memory descriptor (8-row groups 1024 B apart)
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
-  return (uint64_t)((saddr & 0x3FFFF) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
-         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
-}
-
-// kind::f16 instruction descriptor: bf16 A/B, fp32 D, K-major A/B
-__host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
-}
-
-__device__ __forceinline__ void mma_bf16(uint32_t dtmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "setp.ne.b32 p, %4, 0;\n"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
-      "}\n" ::"r"(dtmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
-}
-
-__device__ __forceinline__ void mma_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
-               : "memory");
-}
-
-__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-
-#define TMEM_REGS32(v)                                                                                            \
-  "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]), "=r"(v[8]),       \
-      "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15]), "=r"(v[16]),        \
-      "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]), "=r"(v[22]), "=r"(v[23]), "=r"(v[24]),       \
-      "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]), "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-
-__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
-      "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
-      : TMEM_REGS32(v)
-      : "r"(taddr));
-}
-
-__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&v)[32]) {
-  asm volatile(
-      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
-      "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31, %32};" ::"r"(taddr),
-      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
-      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]), "r"(v[17]), "r"(v[18]),
-      "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]),
-      "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
-      : "memory");
-}
-
-__device__ __forceinline__ void tmem_ld8(uint32_t taddr, uint32_t (&v)[8]) {
-  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
-               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
-               : "r"(taddr));
-}
-
-__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
-__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
-
-__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
-  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
-  return *reinterpret_cast<uint32_t*>(&h);
-}
+using namespace ptx;
 
 __device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
   return t.c0 < (c + 1) * Cc && t.c0 + t.C > c * Cc;
 }
 
-constexpr int kThreads = 192;
+constexpr int kThreads = 320;   // warps 0-3 epilogue, 4 TMA producer, 5 MMA, 6-9 gather (gather mode)
 constexpr int kSlotA = 16384;
+
+// The MMA work of one tile is a sequence of "units": chunk c of the restored
+// width (and, for a pooled chain, tap tau of the pooling window).  Units are
+// processed in pairs (two TMEM accumulators) -- consecutive chunks, or
+// consecutive taps of one chunk -- and every role walks the same order:
+//   for pair: for level l: for unit in pair: G1(unit, l) [+ epilogue E(unit, l)]
+//             then G2 for every chunk whose restored values are final.
+struct PairIter {
+  int c0, t0, nb;
+};
+
+__device__ __forceinline__ void unit_of(const TcChainDesc& d, const PairIter& it, int bi, int& c, int& tap) {
+  if (d.pool) {
+    c = it.c0;
+    tap = it.t0 + bi;
+  } else {
+    c = it.c0 + bi;
+    tap = 0;
+  }
+}
+
+#define FOR_PAIRS(d, it)                                                                            \
+  for (PairIter it{0, 0, 0}; it.c0 < (d).nchunks;                                                   \
+       (d).pool ? ((it.t0 += 2) >= (d).taps ? (it.t0 = 0, ++it.c0) : 0) : (it.c0 += 2))             \
+    if ((it.nb = (d).pool ? min(2, (d).taps - it.t0) : min(2, (d).nchunks - it.c0)), true)
+
+// chunks whose G2 follows this pair: non-pool -> c0 .. c0+nb-1; pool -> c0 after its last tap
+__device__ __forceinline__ int g2_count(const TcChainDesc& d, const PairIter& it) {
+  if (d.gap) return 0;
+  if (d.pool) return it.t0 + it.nb == d.taps ? 1 : 0;
+  return it.nb;
+}
 
 __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
@@ -422,7 +384,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
+      mbar_init(&full[s], d.gather ? 129 : 1);
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -450,35 +412,82 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      const uint32_t bytes_g1 = kSlotA + Cc * 128, bytes_g2 = d.Np * 128;
+      const uint32_t bytes_b = Cc * 128, bytes_a = d.gather ? 0 : kSlotA, bytes_f = d.Np * 128;
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        const int m0 = tile * 128;
-        for (int pc = 0; pc < d.nchunks; pc += 2) {
-          const int nb = min(2, d.nchunks - pc);
+        const int m0 = tile * d.rows_per_tile;
+        FOR_PAIRS(d, it) {
           for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < nb; ++bi) {
-              const int c = pc + bi;
+            for (int bi = 0; bi < it.nb; ++bi) {
+              int c, tap;
+              unit_of(d, it, bi, c, tap);
               for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
                 const TcTerm& t = d.term[j];
                 if (!term_hits(t, c, Cc)) continue;
                 for (int ka = 0; ka < t.Rp / 64; ++ka) {
                   mbar_wait(&empty[stage], phase ^ 1);
-                  mbar_expect_tx(&full[stage], bytes_g1);
+                  mbar_expect_tx(&full[stage], bytes_a + bytes_b);
                   uint8_t* sa = ring + stage * slot;
-                  tma_load_2d(sa, t.tmap, &full[stage], ka * 64, m0);
+                  if (!d.gather) tma_load_2d(sa, t.tmap, &full[stage], ka * 64, m0);
                   tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * 64, c * Cc);
                   if (++stage == S) stage = 0, phase ^= 1;
                 }
               }
             }
-          for (int bi = 0; bi < nb; ++bi) {
-            const int c = pc + bi;
+          for (int q = 0; q < g2_count(d, it); ++q) {
+            const int c = it.c0 + (d.pool ? 0 : q);
             for (int a = 0; a < Cc / 64; ++a) {
               mbar_wait(&empty[stage], phase ^ 1);
-              mbar_expect_tx(&full[stage], bytes_g2);
+              mbar_expect_tx(&full[stage], bytes_f);
               tma_load_2d(ring + stage * slot + kSlotA, d.fmap, &full[stage], c * Cc + a * 64, 0);
               if (++stage == S) stage = 0, phase ^= 1;
             }
+          }
+        }
+      }
+    }
+  } else if (warp >= 6) {
+    // ------------------------------------------------------------ gather producer (A rows)
+    if (d.gather) {
+      const int g = threadIdx.x - 192;
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+        const int64_t m = (int64_t)tile * d.rows_per_tile + g;
+        const bool mv = m < d.npix;
+        const int hw = d.Ho * d.Wo;
+        const int n = mv ? (int)(m / hw) : 0;
+        const int rem = mv ? (int)(m % hw) : 0;
+        const int ho = rem / d.Wo, wo = rem % d.Wo;
+        FOR_PAIRS(d, it) {
+          for (int l = 0; l < d.n_levels; ++l)
+            for (int bi = 0; bi < it.nb; ++bi) {
+              int c, tap;
+              unit_of(d, it, bi, c, tap);
+              const int hi = ho * d.ps - d.pp + tap / d.pk, wi = wo * d.ps - d.pp + tap % d.pk;
+              const bool valid = mv && hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
+              const int64_t pix = ((int64_t)n * d.Hin + hi) * d.Win + wi;
+              for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
+                const TcTerm& t = d.term[j];
+                if (!term_hits(t, c, Cc)) continue;
+                const uint8_t* rbase = reinterpret_cast<const uint8_t*>(p.arena + t.r.off);
+                for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                  mbar_wait(&empty[stage], phase ^ 1);
+                  uint8_t* dst = ring + stage * slot + g * 128;
+#pragma unroll
+                  for (int q = 0; q < 8; ++q) {
+                    const int k0 = ka * 64 + q * 8;
+                    const bool ok = valid && k0 < t.R;
+                    cp_async16(dst + ((q ^ (g & 7)) * 16), ok ? rbase + (pix * t.R + k0) * 2 : rbase, ok ? 16u : 0u);
+                  }
+                  cp_async_arrive(&full[stage]);
+                  if (++stage == S) stage = 0, phase ^= 1;
+                }
+              }
+            }
+          for (int q = 0; q < g2_count(d, it) * (Cc / 64); ++q) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            cp_async_arrive(&full[stage]);
+            if (++stage == S) stage = 0, phase ^= 1;
           }
         }
       }
@@ -492,11 +501,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
       const uint32_t tout = tbase + 2 * Cc;
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        for (int pc = 0; pc < d.nchunks; pc += 2) {
-          const int nb = min(2, d.nchunks - pc);
+        FOR_PAIRS(d, it) {
           for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < nb; ++bi) {
-              const int c = pc + bi;
+            for (int bi = 0; bi < it.nb; ++bi) {
+              int c, tap;
+              unit_of(d, it, bi, c, tap);
               mbar_wait(&acc_empty[bi], (acc_use[bi] & 1) ^ 1);
               tc_fence_after();
               const uint32_t tacc = tbase + bi * Cc;
@@ -506,6 +515,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 if (!term_hits(t, c, Cc)) continue;
                 for (int ka = 0; ka < t.Rp / 64; ++ka) {
                   mbar_wait(&full[stage], phase);
+                  if (d.gather) fence_proxy_async();
                   tc_fence_after();
                   const uint32_t sa = smem_u32(ring + stage * slot);
                   const int nk = min(4, (t.R - ka * 64 + 15) / 16);
@@ -520,15 +530,16 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               mma_commit(&acc_full[bi]);
               ++acc_use[bi];
             }
-          for (int bi = 0; bi < nb; ++bi) {
-            const int c = pc + bi;
-            mbar_wait(&p_full[bi], p_use[bi] & 1);
+          for (int q = 0; q < g2_count(d, it); ++q) {
+            const int c = it.c0 + (d.pool ? 0 : q);
+            const int pb = c & 1;
+            mbar_wait(&p_full[pb], p_use[pb] & 1);
             tc_fence_after();
             if (c == 0) {
               mbar_wait(out_empty, (tile_iter & 1) ^ 1);
               tc_fence_after();
             }
-            const uint32_t pa = smem_u32(pbuf + bi * pbytes);
+            const uint32_t pa = smem_u32(pbuf + pb * pbytes);
             for (int a = 0; a < Cc / 64; ++a) {
               mbar_wait(&full[stage], phase);
               tc_fence_after();
@@ -539,11 +550,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               mma_commit(&empty[stage]);
               if (++stage == S) stage = 0, phase ^= 1;
             }
-            mma_commit(&p_empty[bi]);
-            ++p_use[bi];
+            mma_commit(&p_empty[pb]);
+            ++p_use[pb];
           }
         }
-        mma_commit(out_full);
+        if (!d.gap) mma_commit(out_full);
         ++tile_iter;
       }
     }
@@ -553,64 +564,124 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
     uint32_t acc_use[2] = {0, 0}, p_use[2] = {0, 0}, tile_iter = 0;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+    float run[64];                                     // pooled values of the current chunk (pool mode, Cc = 64)
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-      const int64_t m = (int64_t)tile * 128 + row;
-      for (int pc = 0; pc < d.nchunks; pc += 2) {
-        const int nb = min(2, d.nchunks - pc);
+      const int64_t m = (int64_t)tile * d.rows_per_tile + row;
+      int ho = 0, wo = 0;
+      if (d.pool) {
+        const int rem = (int)(m % (d.Ho * d.Wo));
+        ho = rem / d.Wo;
+        wo = rem % d.Wo;
+      }
+      FOR_PAIRS(d, it) {
         for (int l = 0; l < d.n_levels; ++l) {
           const bool last = l == d.n_levels - 1;
           const bool relu = d.relu[l] != 0;
-          for (int bi = 0; bi < nb; ++bi) {
-            const int c = pc + bi;
+          for (int bi = 0; bi < it.nb; ++bi) {
+            int c, tap;
+            unit_of(d, it, bi, c, tap);
             mbar_wait(&acc_full[bi], acc_use[bi] & 1);
             ++acc_use[bi];
             tc_fence_after();
-            if (last) {
-              mbar_wait(&p_empty[bi], (p_use[bi] & 1) ^ 1);
-              ++p_use[bi];
+            const int pb = c & 1;
+            const bool writes_p = last && !d.gap && (!d.pool || tap == d.taps - 1);
+            if (writes_p) {
+              mbar_wait(&p_empty[pb], (p_use[pb] & 1) ^ 1);
+              ++p_use[pb];
             }
             const float* bias = p.params + d.bias[l] + (int64_t)c * Cc;
-            uint8_t* P = pbuf + bi * pbytes;
-            for (int g = 0; g < Cc / 32; ++g) {
-              const uint32_t ta = tbase + lane_off + bi * Cc + g * 32;
-              uint32_t v[32];
-              tmem_ld32(ta, v);
-              tmem_wait_ld();
-              float f[32];
+            uint8_t* P = pbuf + pb * pbytes;
+            if (d.pool && last) {
+              // pooled chain: fold this tap into the running max / sum (Cc == 64)
+              const int hi = ho * d.ps - d.pp + tap / d.pk, wi = wo * d.ps - d.pp + tap % d.pk;
+              const bool valid = hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
 #pragma unroll
-              for (int i = 0; i < 32; ++i) {
-                float x = __uint_as_float(v[i]) + __ldg(bias + g * 32 + i);
-                f[i] = relu ? fmaxf(x, 0.f) : x;
-              }
-              if (!last) {
+              for (int g = 0; g < 2; ++g) {
+                uint32_t v[32];
+                tmem_ld32(tbase + lane_off + bi * Cc + g * 32, v);
+                tmem_wait_ld();
 #pragma unroll
-                for (int i = 0; i < 32; ++i) v[i] = __float_as_uint(f[i]);
-                tmem_st32(ta, v);
-              } else {
-                const int col = g * 32;                     // within the chunk
-                uint8_t* atom = P + (col / 64) * 16384 + row * 128;
-                const int ch0 = (col % 64) / 8;
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                  uint4 pk;
-                  pk.x = pack_bf16(f[8 * q + 0], f[8 * q + 1]);
-                  pk.y = pack_bf16(f[8 * q + 2], f[8 * q + 3]);
-                  pk.z = pack_bf16(f[8 * q + 4], f[8 * q + 5]);
-                  pk.w = pack_bf16(f[8 * q + 6], f[8 * q + 7]);
-                  *reinterpret_cast<uint4*>(atom + (((ch0 + q) ^ (row & 7)) * 16)) = pk;
+                for (int i = 0; i < 32; ++i) {
+                  float x = __uint_as_float(v[i]) + __ldg(bias + g * 32 + i);
+                  x = relu ? fmaxf(x, 0.f) : x;
+                  float& r = run[g * 32 + i];
+                  if (d.pool == 1)
+                    r = tap == 0 ? (valid ? x : -INFINITY) : (valid ? fmaxf(r, x) : r);
+                  else
+                    r = tap == 0 ? x : r + x;
                 }
               }
+              if (writes_p) {
+                const float scale = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) {
+                  uint4 pk;
+                  pk.x = pack_bf16(run[8 * q + 0] * scale, run[8 * q + 1] * scale);
+                  pk.y = pack_bf16(run[8 * q + 2] * scale, run[8 * q + 3] * scale);
+                  pk.z = pack_bf16(run[8 * q + 4] * scale, run[8 * q + 5] * scale);
+                  pk.w = pack_bf16(run[8 * q + 6] * scale, run[8 * q + 7] * scale);
+                  *reinterpret_cast<uint4*>(P + row * 128 + ((q ^ (row & 7)) * 16)) = pk;
+                }
+              }
+            } else {
+              for (int g = 0; g < Cc / 32; ++g) {
+                const uint32_t ta = tbase + lane_off + bi * Cc + g * 32;
+                uint32_t v[32];
+                tmem_ld32(ta, v);
+                tmem_wait_ld();
+                float f[32];
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                  float x = __uint_as_float(v[i]) + __ldg(bias + g * 32 + i);
+                  f[i] = relu ? fmaxf(x, 0.f) : x;
+                }
+                if (!last) {
+#pragma unroll
+                  for (int i = 0; i < 32; ++i) v[i] = __float_as_uint(f[i]);
+                  tmem_st32(ta, v);
+                } else if (d.gap) {
+                  // GAP root: per-image column means of this 32-column group; tiles
+                  // hold whole images so the reduction order is fixed (deterministic)
+                  float* red = reinterpret_cast<float*>(pbuf);
+#pragma unroll
+                  for (int i = 0; i < 32; ++i) red[row * 32 + ((i + row) & 31)] = f[i];
+                  asm volatile("bar.sync 1, 128;" ::: "memory");
+                  for (int idx = row; idx < d.ipt * 32; idx += 128) {
+                    const int ii = idx / 32, col = idx % 32;
+                    const int n = tile * d.ipt + ii;
+                    float acc = 0.f;
+                    for (int r = ii * d.hw; r < (ii + 1) * d.hw; ++r) acc += red[r * 32 + ((col + r) & 31)];
+                    const int cg = c * Cc + g * 32 + col;
+                    if (n < d.nimg && cg < d.C) y[(int64_t)n * d.C + cg] = __float2bfloat16_rn(acc / (float)d.hw);
+                  }
+                  asm volatile("bar.sync 1, 128;" ::: "memory");
+                } else {
+                  const int col = g * 32;                     // within the chunk
+                  uint8_t* atom = P + (col / 64) * 16384 + row * 128;
+                  const int ch0 = (col % 64) / 8;
+#pragma unroll
+                  for (int q = 0; q < 4; ++q) {
+                    uint4 pk;
+                    pk.x = pack_bf16(f[8 * q + 0], f[8 * q + 1]);
+                    pk.y = pack_bf16(f[8 * q + 2], f[8 * q + 3]);
+                    pk.z = pack_bf16(f[8 * q + 4], f[8 * q + 5]);
+                    pk.w = pack_bf16(f[8 * q + 6], f[8 * q + 7]);
+                    *reinterpret_cast<uint4*>(atom + (((ch0 + q) ^ (row & 7)) * 16)) = pk;
+                  }
+                }
+              }
+              if (!last) tmem_wait_st();
             }
-            if (!last) tmem_wait_st();
             tc_fence_before();
             mbar_arrive(&acc_empty[bi]);
-            if (last) {
-              asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-              mbar_arrive(&p_full[bi]);
+            if (writes_p) {
+              fence_proxy_async();
+              mbar_arrive(&p_full[pb]);
             }
           }
         }
       }
+      if (d.gap) continue;
       // output epilogue
       mbar_wait(out_full, tile_iter & 1);
       ++tile_iter;
@@ -648,19 +719,15 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   (void)tcw;
   static bool configured = false;
+  static int sms = 0;
   if (!configured) {
     cudaFuncSetAttribute(tc_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    configured = true;
-  }
-  int sms = 148;
-  static int dev_sms = 0;
-  if (!dev_sms) {
     int dev = 0;
     cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
   }
-  sms = dev_sms > 0 ? dev_sms : 148;
-  const int grid = std::min(d.ntiles, sms);
+  const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
   // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
   tc_chain_kernel<<<grid, kThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }

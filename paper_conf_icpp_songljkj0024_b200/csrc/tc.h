@@ -45,6 +45,12 @@ struct TcChainDesc {
   int32_t Nout, Np;                      // fconv outputs, padded to a multiple of 16
   int64_t npix;
   int32_t ntiles;
+  int32_t rows_per_tile;                 // 128, or whole images for a GAP root
+  int32_t gap, hw, ipt;                  // GAP root: pixels per image, images per tile
+  int32_t nimg;
+  int32_t gather;                        // A rows gathered by 4 warps (cp.async) instead of TMA
+  int32_t pool, pk, ps, pp, taps;        // pooled chain: 0 none / 1 max / 2 avg, window, stride, pad
+  int32_t Hin, Win, Ho, Wo;              // chain resolution, root resolution
   int64_t F;                             // tc weight pool offset of F
   int64_t Fb;                            // params offset of the fconv bias or -1
   Loc y;                                 // output [npix, Nout] bf16
