@@ -112,7 +112,8 @@ namespace {
 
 using namespace ptx;
 
-constexpr int kConvThreads = 288;   // warps 0-3 epilogue, 4-7 gather, 8 MMA
+constexpr int kGatherWarps = 8;
+constexpr int kConvThreads = 32 * (5 + kGatherWarps);   // warps 0-3 epilogue, 4..11 gather, 12 MMA
 
 __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_constant__ ConvTcDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
@@ -132,7 +133,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 128);
+      mbar_init(&full[s], 32);
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -153,70 +154,97 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
   const uint32_t tbase = *tmem_slot;
   const int hw = d.Ho * d.Wo;
 
-  if (warp >= 4 && warp < 8) {
+  if (warp >= 4 && warp < 4 + kGatherWarps) {
     // ------------------------------------------------------------ im2col gather
-    const int g = threadIdx.x - 128;     // A row
+    // warp-per-stage: gather warp gw fills every kGatherWarps-th A stage (lane
+    // owns rows lane, lane+32, lane+64, lane+96), so kGatherWarps stages are in
+    // flight at once (each warp's cp.async batch completes in ~0.7-2 us).
+    const int gw = warp - 4;
     const uint8_t* x = static_cast<const uint8_t*>(loc_ptr(d.x, p));
-    int stage = 0;
-    uint32_t phase = 0;
+    const __nv_bfloat16* xb = reinterpret_cast<const __nv_bfloat16*>(x);
     const int cpt = d.Cin / 8;           // 16-byte chunks per tap (vec path)
+    const int kwc = d.kw * d.Cin;        // elements per kernel row (scalar path)
+    int64_t kseq = 0;                    // global A-stage counter
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-      const int64_t m = (int64_t)tile * 128 + g;
-      const bool mv = m < d.npix;
-      const int n = mv ? (int)(m / hw) : 0;
-      const int rem = mv ? (int)(m % hw) : 0;
-      const int hb = (rem / d.Wo) * d.sh - d.ph, wb = (rem % d.Wo) * d.sw - d.pw;
-      const int64_t img = (int64_t)n * d.H * d.W;
-      for (int kb = 0; kb < d.katoms; ++kb) {
+      int hb[4], wb[4];
+      int64_t img[4];
+      bool mv[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int64_t m = (int64_t)tile * 128 + lane + 32 * i;
+        mv[i] = m < d.npix;
+        const int n = mv[i] ? (int)(m / hw) : 0;
+        const int rem = mv[i] ? (int)(m % hw) : 0;
+        hb[i] = (rem / d.Wo) * d.sh - d.ph;
+        wb[i] = (rem % d.Wo) * d.sw - d.pw;
+        img[i] = (int64_t)n * d.H * d.W;
+      }
+      for (int kb = 0; kb < d.katoms; ++kb, ++kseq) {
+        if ((int)(kseq % kGatherWarps) != gw) continue;
+        const int stage = (int)(kseq % S);
+        const uint32_t phase = (uint32_t)((kseq / S) & 1);
         mbar_wait(&empty[stage], phase ^ 1);
-        uint8_t* dst = ring + stage * 16384 + g * 128;
         if (d.vec) {
 #pragma unroll
-          for (int q = 0; q < 8; ++q) {
-            const int kc = kb * 8 + q;
-            const uint8_t* src = x;
-            uint32_t bytes = 0;
-            if (mv && kc < d.kchunks) {
-              const int tap = kc / cpt, cc = kc - tap * cpt;
-              const int hi = hb + tap / d.kw, wi = wb + tap % d.kw;
-              if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W) {
-                src = x + ((img + (int64_t)hi * d.W + wi) * d.Cin + cc * 8) * 2;
-                bytes = 16;
+          for (int i = 0; i < 4; ++i) {
+            const int row = lane + 32 * i;
+            uint8_t* dst = ring + stage * 16384 + row * 128;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              const int kc = kb * 8 + q;
+              const uint8_t* src = x;
+              uint32_t bytes = 0;
+              if (mv[i] && kc < d.kchunks) {
+                const int tap = kc / cpt, cc = kc - tap * cpt;
+                const int hi = hb[i] + tap / d.kw, wi = wb[i] + tap % d.kw;
+                if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W) {
+                  src = x + ((img[i] + (int64_t)hi * d.W + wi) * d.Cin + cc * 8) * 2;
+                  bytes = 16;
+                }
               }
+              cp_async16(dst + ((q ^ (row & 7)) * 16), src, bytes);
             }
-            cp_async16(dst + ((q ^ (g & 7)) * 16), src, bytes);
           }
           cp_async_arrive(&full[stage]);
         } else {
-          const __nv_bfloat16* xb = reinterpret_cast<const __nv_bfloat16*>(x);
+          // small Cin (the 3-channel image): element gather with carried
+          // (a, b, c) counters -- k = (a * kw + b) * Cin + c, no divisions
 #pragma unroll 1
-          for (int q = 0; q < 8; ++q) {
-            uint32_t pk[4];
+          for (int i = 0; i < 4; ++i) {
+            const int row = lane + 32 * i;
+            uint8_t* dst = ring + stage * 16384 + row * 128;
+            int k = kb * 64;
+            int a = k / kwc, rr = k - a * kwc;
+            int b = rr / d.Cin, c = rr - b * d.Cin;
+#pragma unroll 1
+            for (int q = 0; q < 8; ++q) {
+              uint32_t pk[4];
 #pragma unroll
-            for (int e2 = 0; e2 < 4; ++e2) {
-              float f[2];
+              for (int e2 = 0; e2 < 4; ++e2) {
+                float f[2];
 #pragma unroll
-              for (int h = 0; h < 2; ++h) {
-                const int k = (kb * 8 + q) * 8 + e2 * 2 + h;
-                f[h] = 0.f;
-                if (mv && k < d.K) {
-                  const int tap = k / d.Cin, c = k - tap * d.Cin;
-                  const int hi = hb + tap / d.kw, wi = wb + tap % d.kw;
-                  if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W)
-                    f[h] = __bfloat162float(xb[(img + (int64_t)hi * d.W + wi) * d.Cin + c]);
+                for (int h = 0; h < 2; ++h) {
+                  f[h] = 0.f;
+                  const int hi = hb[i] + a, wi = wb[i] + b;
+                  if (mv[i] && k < d.K && hi >= 0 && hi < d.H && wi >= 0 && wi < d.W)
+                    f[h] = __bfloat162float(xb[(img[i] + (int64_t)hi * d.W + wi) * d.Cin + c]);
+                  ++k;
+                  if (++c == d.Cin) {
+                    c = 0;
+                    if (++b == d.kw) b = 0, ++a;
+                  }
                 }
+                pk[e2] = pack_bf16(f[0], f[1]);
               }
-              pk[e2] = pack_bf16(f[0], f[1]);
+              *reinterpret_cast<uint4*>(dst + ((q ^ (row & 7)) * 16)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
             }
-            *reinterpret_cast<uint4*>(dst + ((q ^ (g & 7)) * 16)) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
           }
           fence_proxy_async();
           mbar_arrive(&full[stage]);
         }
-        if (++stage == S) stage = 0, phase ^= 1;
       }
     }
-  } else if (warp == 8) {
+  } else if (warp == 4 + kGatherWarps) {
     // ------------------------------------------------------------ weights + MMA issuer
     if (lane == 0) {
       mbar_expect_tx(wbar, wbytes);
@@ -293,10 +321,8 @@ void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
-  // two CTAs per SM when TMEM (<= 256 columns each) and SMEM allow it
-  const bool two = d.tmem_cols <= 256 && d.smem_bytes <= 110 * 1024;
-  const int grid = std::min(d.ntiles, (sms > 0 ? sms : 148) * (two ? 2 : 1));
-  conv_tc_kernel<<<grid, kConvThreads, two ? d.smem_bytes : std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+  const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);   // persistent, one CTA per SM
+  conv_tc_kernel<<<grid, kConvThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }
 
 }  // namespace temco

@@ -384,7 +384,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], d.gather ? 129 : 1);
+      mbar_init(&full[s], d.gather ? 33 : 1);
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -447,47 +447,67 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
   } else if (warp >= 6) {
     // ------------------------------------------------------------ gather producer (A rows)
+    // warp-per-stage: gather warp gw fills every 4th stage of the ring (lane
+    // owns rows lane + 32 i), so 4 stages of cp.async are in flight at once
     if (d.gather) {
-      const int g = threadIdx.x - 192;
-      int stage = 0;
-      uint32_t phase = 0;
+      const int gw = warp - 6;
+      int64_t kseq = 0;
+      auto next = [&](int& stage, uint32_t& phase) {
+        stage = (int)(kseq % S);
+        phase = (uint32_t)((kseq / S) & 1);
+        return (int)((kseq++) & 3) == gw;
+      };
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        const int64_t m = (int64_t)tile * d.rows_per_tile + g;
-        const bool mv = m < d.npix;
+        int ho[4], wo[4], nn[4];
+        bool mv[4];
         const int hw = d.Ho * d.Wo;
-        const int n = mv ? (int)(m / hw) : 0;
-        const int rem = mv ? (int)(m % hw) : 0;
-        const int ho = rem / d.Wo, wo = rem % d.Wo;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int64_t m = (int64_t)tile * d.rows_per_tile + lane + 32 * i;
+          mv[i] = m < d.npix;
+          nn[i] = mv[i] ? (int)(m / hw) : 0;
+          const int rem = mv[i] ? (int)(m % hw) : 0;
+          ho[i] = rem / d.Wo;
+          wo[i] = rem % d.Wo;
+        }
         FOR_PAIRS(d, it) {
           for (int l = 0; l < d.n_levels; ++l)
             for (int bi = 0; bi < it.nb; ++bi) {
               int c, tap;
               unit_of(d, it, bi, c, tap);
-              const int hi = ho * d.ps - d.pp + tap / d.pk, wi = wo * d.ps - d.pp + tap % d.pk;
-              const bool valid = mv && hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
-              const int64_t pix = ((int64_t)n * d.Hin + hi) * d.Win + wi;
               for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
                 const TcTerm& t = d.term[j];
                 if (!term_hits(t, c, Cc)) continue;
                 const uint8_t* rbase = reinterpret_cast<const uint8_t*>(p.arena + t.r.off);
                 for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                  int stage;
+                  uint32_t phase;
+                  if (!next(stage, phase)) continue;
                   mbar_wait(&empty[stage], phase ^ 1);
-                  uint8_t* dst = ring + stage * slot + g * 128;
 #pragma unroll
-                  for (int q = 0; q < 8; ++q) {
-                    const int k0 = ka * 64 + q * 8;
-                    const bool ok = valid && k0 < t.R;
-                    cp_async16(dst + ((q ^ (g & 7)) * 16), ok ? rbase + (pix * t.R + k0) * 2 : rbase, ok ? 16u : 0u);
+                  for (int i = 0; i < 4; ++i) {
+                    const int row = lane + 32 * i;
+                    const int hi = ho[i] * d.ps - d.pp + tap / d.pk, wi = wo[i] * d.ps - d.pp + tap % d.pk;
+                    const bool valid = mv[i] && hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
+                    const int64_t pix = ((int64_t)nn[i] * d.Hin + hi) * d.Win + wi;
+                    uint8_t* dst = ring + stage * slot + row * 128;
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) {
+                      const int k0 = ka * 64 + q * 8;
+                      const bool ok = valid && k0 < t.R;
+                      cp_async16(dst + ((q ^ (row & 7)) * 16), ok ? rbase + (pix * t.R + k0) * 2 : rbase, ok ? 16u : 0u);
+                    }
                   }
                   cp_async_arrive(&full[stage]);
-                  if (++stage == S) stage = 0, phase ^= 1;
                 }
               }
             }
           for (int q = 0; q < g2_count(d, it) * (Cc / 64); ++q) {
+            int stage;
+            uint32_t phase;
+            if (!next(stage, phase)) continue;
             mbar_wait(&empty[stage], phase ^ 1);
             cp_async_arrive(&full[stage]);
-            if (++stage == S) stage = 0, phase ^= 1;
           }
         }
       }

@@ -12,7 +12,7 @@ import os
 
 import numpy as np
 
-_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libtemco.so")
+_LIB_PATH = os.environ.get("TEMCO_LIB") or os.path.join(os.path.dirname(os.path.abspath(__file__)), "libtemco.so")
 if not os.path.exists(_LIB_PATH):
     raise ImportError(f"{_LIB_PATH} is missing: build it with `python -m paper_conf_icpp_songljkj0024_b200.build` "
                       "(there is no CPU fallback)")
