@@ -116,7 +116,8 @@ enum {
   TEMCO_FLAG_CUDA_GRAPH = 1 << 3,      /* capture temco_run into a CUDA graph per (in,out,stream) */
   TEMCO_FLAG_SIMT_ONLY = 1 << 4,       /* never select the tcgen05 kernels               */
   TEMCO_FLAG_OVERHEAD_ALWAYS = 1 << 5, /* force Overhead() true  (tests)                 */
-  TEMCO_FLAG_OVERHEAD_NEVER = 1 << 6   /* force Overhead() false (tests)                 */
+  TEMCO_FLAG_OVERHEAD_NEVER = 1 << 6,  /* force Overhead() false (tests)                 */
+  TEMCO_FLAG_MMA_SMALL = 1 << 7        /* run groups with C <= 256 on the mma.sync kernel */
 };
 
 typedef struct {

@@ -14,6 +14,7 @@
 #include "kernels.h"
 #include "planner.h"
 #include "conv_tc.h"
+#include "mma_chain.h"
 #include "tc.h"
 
 using namespace temco;
@@ -33,7 +34,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA };
 
 struct StepExec {
   int kind = K_NONE;
@@ -43,6 +44,7 @@ struct StepExec {
   GroupDesc grp{};
   TcChainDesc tc{};
   ConvTcDesc ctc{};
+  MmaChainDesc mma{};
   std::string kernel;
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
@@ -256,7 +258,15 @@ void lower(temco_plan_s* P) {
     for (int x : s.in) e.io_bytes += tensor_bytes(P, x);
     if (v.op != OP_INPUT) e.io_bytes += tensor_bytes(P, s.out);
     if (s.group) {
-      // try the tcgen05 chain kernel first (bf16 plans), else the interpreter
+      // small restored widths: register-resident mma.sync kernel; larger ones:
+      // the tcgen05 chain kernel (bf16 plans); anything else: the interpreter
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && (P->flags & TEMCO_FLAG_MMA_SMALL) &&
+          ir.nodes[ir.oin[s.out][0]].C <= 256 && mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma)) {
+        e.kind = K_GROUP_MMA;
+        e.kernel = "mma_chain";
+        e.launches = 1;
+        continue;
+      }
       if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
           tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tc)) {
         e.kind = K_GROUP_TC;
@@ -417,6 +427,7 @@ std::string make_json(const temco_plan_s* P) {
         << ",\"launches\":" << e.launches;
       if (e.kind == K_GROUP_TC) o << ",\"alg_flops\":" << e.tc.alg_flops << ",\"alg_bytes\":" << e.tc.alg_bytes;
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
+      if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;
     }
     o << ",\"live\":" << ir.live_fused[t] << "}";
   }
@@ -462,6 +473,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
       case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
+      case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
     }
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t + 1], st));
   }

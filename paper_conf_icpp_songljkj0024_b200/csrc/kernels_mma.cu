@@ -1,0 +1,403 @@
+// Register-resident fused restore -> BN -> add -> ReLU -> [pool] -> reduce
+// kernel with mma.sync m16n8k16 (see mma_chain.h).
+//
+// Each warp owns 16 output pixels at a time.  Its reduced inputs are staged in
+// a per-warp SMEM double buffer with 16-byte cp.async (the next block / tap is
+// in flight while the current one computes), all weights (BN-folded Lhat,
+// F, level biases) are SMEM-resident for the whole persistent CTA.  For a
+// restored chunk of CH channels the accumulator fragments D[CH/8][4] hold the
+// 16 x CH restored tile in registers; bias / ReLU / max-pool run on them; then
+// they are re-packed to bf16 as the A operand of the reduce GEMM (the fp32
+// m16n8k16 C layout equals the bf16 A layout pairwise), accumulating out[16 x
+// Nout] in registers across chunks.  The C-wide tensor never leaves registers.
+#include <cuda_bf16.h>
+
+#include <algorithm>
+#include <cmath>
+
+#include "chain_parse.h"
+#include "mma_chain.h"
+
+namespace temco {
+
+namespace {
+using namespace chainp;
+
+uint16_t f2bf(float f) {
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  u += 0x7FFF + ((u >> 16) & 1);
+  return (uint16_t)(u >> 16);
+}
+
+}  // namespace
+
+bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
+                     MmaChainDesc& d) {
+  const Node& root = ir.nodes[s.out];
+  if (root.role != ROLE_FCONV) return false;
+  const int tsrc = ir.oin[s.out][0];
+  const Node& tn = ir.nodes[tsrc];
+  const int C = tn.C, Nout = root.C;
+  if (Nout % 8 || Nout > 128 || C % 16) return false;
+  int pool = 0, pk = 1, ps = 1, pp = 0, csrc = tsrc;
+  if ((tn.op == OP_MAXPOOL || tn.op == OP_AVGPOOL) && s.members.size() > 2) {
+    pool = tn.op == OP_MAXPOOL ? 1 : 2;
+    pk = tn.kh; ps = tn.sh; pp = tn.ph;
+    csrc = ir.oin[tsrc][0];
+  }
+  const Node& cn = ir.nodes[csrc];
+  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, cn.H, cn.W};
+  P.members.erase(s.out);
+  if (pool) P.members.erase(tsrc);
+  std::vector<PLevel> levels;
+  if (!P.chain(csrc, levels)) return false;
+  if (P.visited != P.members) return false;
+  int nterms = 0;
+  for (auto& L : levels) nterms += (int)L.terms.size();
+  if ((int)levels.size() > kMmaMaxLevels || nterms > kMmaMaxTerms) return false;
+  for (auto& L : levels)
+    for (auto& t : L.terms) {
+      const int r = ir.oin[t.lconv][0];
+      const Loc& l = loc.at(r);
+      if (l.where != W_ARENA || l.dtype != DT_BF16 || ir.nodes[r].C % 8 || ir.nodes[t.lconv].C % 8) return false;
+    }
+  const Loc& yl = loc.at(s.out);
+  if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
+  if (pool && C > 64) return false;             // running max lives in registers: one 64-wide chunk
+
+  d = MmaChainDesc();
+  d.C = C;
+  d.CH = C <= 64 ? 64 : 128;
+  d.Cpad = (C + d.CH - 1) / d.CH * d.CH;
+  d.nchunks = d.Cpad / d.CH;
+  d.Nout = Nout;
+  d.Np8 = Nout;
+  d.pool = pool; d.pk = pk; d.ps = ps; d.pp = pp; d.taps = pk * pk;
+  d.Hin = cn.H; d.Win = cn.W; d.Ho = tn.H; d.Wo = tn.W;
+  d.npix = (int64_t)ir.batch * tn.H * tn.W;
+  d.nblocks = (int)((d.npix + 15) / 16);
+  d.y = yl;
+  d.n_levels = (int)levels.size();
+  // blob: [Lhat_j rows (Rp + 8)] ... [F (Cpad + 8)] | fp32 biases
+  std::vector<uint16_t> blob;
+  std::vector<float> biases;
+  int j = 0, astride = 0;
+  int64_t fl_terms = 0, by_terms = 0;
+  for (int l = 0; l < d.n_levels; ++l) {
+    const PLevel& L = levels[l];
+    d.relu[l] = L.relu ? 1 : 0;
+    d.bias[l] = (int32_t)biases.size();
+    for (int c = 0; c < d.Cpad; ++c) biases.push_back(c < C ? (float)L.bias[c] : 0.f);
+    for (const PTerm& t : L.terms) {
+      const Node& lc = ir.nodes[t.lconv];
+      const int r = ir.oin[t.lconv][0];
+      const int R = ir.nodes[r].C;
+      MmaTerm& T = d.term[j++];
+      T.r = loc.at(r);
+      T.R = R;
+      T.Rp = (R + 15) / 16 * 16;
+      T.c0 = t.c0;
+      T.C = lc.C;
+      T.level = l;
+      T.w = (int32_t)blob.size();
+      const int rs = T.Rp + 8;
+      blob.resize(blob.size() + (size_t)lc.C * rs, 0);
+      for (int c = 0; c < lc.C; ++c)
+        for (int k = 0; k < R; ++k)
+          blob[T.w + (size_t)c * rs + k] = f2bf((float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]));
+      astride += rs;
+      fl_terms += 2LL * lc.C * R;
+      by_terms += 2LL * R;
+    }
+    d.lvl_end[l] = j;
+  }
+  d.n_terms = j;
+  if (((astride / 8) & 1) == 0) astride += 8;   // odd number of 16-byte chunks per row: conflict-free ldmatrix
+  d.a_stride = astride;
+  d.f = (int32_t)blob.size();
+  const int fs = d.Cpad + 8;
+  blob.resize(blob.size() + (size_t)d.Np8 * fs, 0);
+  for (int o = 0; o < Nout; ++o)
+    for (int c = 0; c < C; ++c) blob[d.f + (size_t)o * fs + c] = f2bf((*root.w)[(size_t)o * C + c]);
+  if (root.b) return false;                      // fconv factors carry no bias (O1)
+  while (blob.size() % 8) blob.push_back(0);
+  d.blob_bf16 = (int32_t)blob.size();
+  for (float b : biases) {
+    uint32_t u;
+    memcpy(&u, &b, 4);
+    blob.push_back((uint16_t)(u & 0xFFFF));
+    blob.push_back((uint16_t)(u >> 16));
+  }
+  while (blob.size() % 8) blob.push_back(0);
+  d.blob_bytes = (int32_t)blob.size() * 2;
+  const int stage_bytes = 8 * 2 * 16 * d.a_stride * 2;
+  d.smem_bytes = d.blob_bytes + stage_bytes + 256;
+  if (d.smem_bytes > 200 * 1024) return false;
+  while (tcw.size() % 512) tcw.push_back(0);
+  d.blob = (int64_t)tcw.size();
+  tcw.insert(tcw.end(), blob.begin(), blob.end());
+  const int64_t nin = (int64_t)ir.batch * cn.H * cn.W;
+  d.alg_flops = nin * fl_terms + d.npix * 2LL * Nout * C;
+  d.alg_bytes = nin * by_terms + d.npix * 2LL * Nout;
+  return true;
+}
+
+namespace {
+
+__device__ __forceinline__ uint32_t s_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+               : "r"(addr));
+}
+
+__device__ __forceinline__ void ldsm_x2(uint32_t addr, uint32_t& r0, uint32_t& r1) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0, %1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(addr));
+}
+
+__device__ __forceinline__ void mma16816(float (&c)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                         uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+      "{%0, %1, %2, %3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+
+__device__ __forceinline__ void cp16(uint32_t dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ uint32_t pk2(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+constexpr int kWarps = 8;
+
+// stage the A rows of unit u (a 16-pixel block, and for a pooled chain one tap)
+__device__ __forceinline__ void stage_unit(const MmaChainDesc& d, const RunPtrs& p, __nv_bfloat16* st, int64_t blk,
+                                           int tap, int lane) {
+  int off = 0;
+  for (int j = 0; j < d.n_terms; ++j) {
+    const MmaTerm& t = d.term[j];
+    const uint8_t* rb = reinterpret_cast<const uint8_t*>(p.arena + t.r.off);
+    const int cpr = t.Rp / 8;                     // 16-byte chunks per row (incl. K padding)
+    for (int c = lane; c < 16 * cpr; c += 32) {
+      const int row = c / cpr, q = c - row * cpr;
+      const int64_t m = blk * 16 + row;
+      int64_t pix = m;
+      bool ok = m < d.npix && q * 8 < t.R;
+      if (d.pool && ok) {
+        const int hw = d.Ho * d.Wo;
+        const int n = (int)(m / hw), rem = (int)(m % hw);
+        const int hi = (rem / d.Wo) * d.ps - d.pp + tap / d.pk, wi = (rem % d.Wo) * d.ps - d.pp + tap % d.pk;
+        ok = hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
+        pix = ((int64_t)n * d.Hin + hi) * d.Win + wi;
+      }
+      cp16(s_u32(st + row * d.a_stride + off + q * 8), ok ? rb + (pix * t.R + q * 8) * 2 : rb, ok ? 16u : 0u);
+    }
+    off += t.Rp + 8;
+  }
+}
+
+template <int CH, int NO, bool POOL>
+__global__ void __launch_bounds__(32 * kWarps, 1) mma_chain_kernel(const __grid_constant__ MmaChainDesc d, RunPtrs p,
+                                                                   const uint16_t* __restrict__ tcw) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int g = lane / 4, t4 = lane % 4;
+  // weights -> SMEM (once per persistent CTA)
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(tcw + d.blob);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  __syncthreads();
+  const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
+  const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
+  __nv_bfloat16* stage = reinterpret_cast<__nv_bfloat16*>(smem + d.blob_bytes) + (size_t)warp * 2 * 16 * d.a_stride;
+  const int units_per_blk = POOL ? d.taps : 1;
+  const int64_t gw = (int64_t)blockIdx.x * kWarps + warp, nw = (int64_t)gridDim.x * kWarps;
+  // ldmatrix lane addressing (A: 16 rows x 16 k; B: 8 rows x 16 k)
+  const int a_row = (lane & 7) + ((lane >> 3) & 1) * 8, a_col = (lane >> 4) * 8;
+  const int b_row = lane & 7, b_col = ((lane >> 3) & 1) * 8;
+
+  int64_t blk = gw;
+  int tap = 0;
+  int buf = 0;
+  if (blk < d.nblocks) stage_unit(d, p, stage, blk, 0, lane);
+  asm volatile("cp.async.commit_group;" ::: "memory");
+
+  float O[NO][4];
+  float run[POOL ? CH / 8 : 1][4];
+  while (blk < d.nblocks) {
+    // prefetch the next unit into the other buffer
+    int64_t nblk = blk;
+    int ntap = tap + 1;
+    if (ntap == units_per_blk) ntap = 0, nblk = blk + nw;
+    if (nblk < d.nblocks) stage_unit(d, p, stage + (buf ^ 1) * 16 * d.a_stride, nblk, ntap, lane);
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
+    __syncwarp();
+    const __nv_bfloat16* A = stage + buf * 16 * d.a_stride;
+
+    if (tap == 0) {
+#pragma unroll
+      for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
+    }
+    // validity of rows g, g+8 for this tap (pooled chains)
+    bool v0 = true, v1 = true;
+    if (POOL) {
+      const int hw = d.Ho * d.Wo;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int64_t m = blk * 16 + g + 8 * h;
+        const int rem = (int)(m % hw);
+        const int hi = (rem / d.Wo) * d.ps - d.pp + tap / d.pk, wi = (rem % d.Wo) * d.ps - d.pp + tap % d.pk;
+        const bool v = hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
+        (h ? v1 : v0) = v;
+      }
+    }
+    for (int ch = 0; ch < d.nchunks; ++ch) {
+      float D[CH / 8][4];
+      int toff = 0, j = 0;
+      for (int l = 0; l < d.n_levels; ++l) {
+        const float* bl = fb + d.bias[l] + ch * CH;
+#pragma unroll
+        for (int nb = 0; nb < CH / 8; ++nb) {
+          const float b0 = bl[nb * 8 + 2 * t4], b1 = bl[nb * 8 + 2 * t4 + 1];
+          if (l == 0) {
+            D[nb][0] = b0; D[nb][1] = b1; D[nb][2] = b0; D[nb][3] = b1;
+          } else {
+            D[nb][0] += b0; D[nb][1] += b1; D[nb][2] += b0; D[nb][3] += b1;
+          }
+        }
+        for (; j < d.lvl_end[l]; ++j) {
+          const MmaTerm& T = d.term[j];
+          const int lo = T.c0 - ch * CH, hi = lo + T.C;     // term's columns relative to the chunk
+          if (hi > 0 && lo < CH) {
+            const int rs = T.Rp + 8;
+            for (int ks = 0; ks < T.Rp / 16; ++ks) {
+              uint32_t a0, a1, a2, a3;
+              ldsm_x4(s_u32(A + a_row * d.a_stride + toff + ks * 16 + a_col), a0, a1, a2, a3);
+#pragma unroll
+              for (int nb = 0; nb < CH / 8; ++nb) {
+                if (nb * 8 >= lo && nb * 8 < hi) {
+                  uint32_t b0, b1;
+                  ldsm_x2(s_u32(blob + T.w + (nb * 8 - lo + b_row) * rs + ks * 16 + b_col), b0, b1);
+                  mma16816(D[nb], a0, a1, a2, a3, b0, b1);
+                }
+              }
+            }
+          }
+          toff += T.Rp + 8;
+        }
+        if (d.relu[l]) {
+#pragma unroll
+          for (int nb = 0; nb < CH / 8; ++nb)
+#pragma unroll
+            for (int i = 0; i < 4; ++i) D[nb][i] = fmaxf(D[nb][i], 0.f);
+        }
+      }
+      if (POOL) {
+        // running max / sum over taps (CH == C: single chunk)
+#pragma unroll
+        for (int nb = 0; nb < CH / 8; ++nb) {
+          if (d.pool == 1) {
+            const float n0 = v0 ? 0.f : -INFINITY, n1 = v1 ? 0.f : -INFINITY;
+            const float x0 = D[nb][0] + n0, x1 = D[nb][1] + n0, x2 = D[nb][2] + n1, x3 = D[nb][3] + n1;
+            if (tap == 0) {
+              run[nb][0] = x0; run[nb][1] = x1; run[nb][2] = x2; run[nb][3] = x3;
+            } else {
+              run[nb][0] = fmaxf(run[nb][0], x0); run[nb][1] = fmaxf(run[nb][1], x1);
+              run[nb][2] = fmaxf(run[nb][2], x2); run[nb][3] = fmaxf(run[nb][3], x3);
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) run[nb][i] = tap == 0 ? D[nb][i] : run[nb][i] + D[nb][i];
+          }
+        }
+        if (tap != d.taps - 1) continue;
+        const float sc = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
+#pragma unroll
+        for (int nb = 0; nb < CH / 8; ++nb)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) D[nb][i] = run[nb][i] * sc;
+      }
+      // reduce: out[16 x Nout] += P[16 x CH] F[:, chunk]^T, P re-packed from D
+      const int fs = d.Cpad + 8;
+#pragma unroll
+      for (int ks = 0; ks < CH / 16; ++ks) {
+        const uint32_t a0 = pk2(D[2 * ks][0], D[2 * ks][1]), a1 = pk2(D[2 * ks][2], D[2 * ks][3]);
+        const uint32_t a2 = pk2(D[2 * ks + 1][0], D[2 * ks + 1][1]), a3 = pk2(D[2 * ks + 1][2], D[2 * ks + 1][3]);
+#pragma unroll
+        for (int nb = 0; nb < NO; ++nb) {
+          if (nb * 8 < d.Nout) {
+            uint32_t b0, b1;
+            ldsm_x2(s_u32(blob + d.f + (nb * 8 + b_row) * fs + ch * CH + ks * 16 + b_col), b0, b1);
+            mma16816(O[nb], a0, a1, a2, a3, b0, b1);
+          }
+        }
+      }
+    }
+    if (!POOL || tap == d.taps - 1) {
+      __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+      const int64_t m0 = blk * 16 + g, m1 = m0 + 8;
+#pragma unroll
+      for (int nb = 0; nb < NO; ++nb) {
+        if (nb * 8 < d.Nout) {
+          const int col = nb * 8 + 2 * t4;
+          if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + m0 * d.Nout + col) = pk2(O[nb][0], O[nb][1]);
+          if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + m1 * d.Nout + col) = pk2(O[nb][2], O[nb][3]);
+        }
+      }
+    }
+    __syncwarp();
+    buf ^= 1;
+    tap = ntap;
+    blk = nblk;
+  }
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
+}
+
+template <int CH, int NO, bool POOL>
+void launch_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  if (!configured) {
+    cudaFuncSetAttribute(mma_chain_kernel<CH, NO, POOL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  const int per_sm = d.smem_bytes <= 100 * 1024 ? 2 : 1;
+  const int grid = (int)std::min<int64_t>((d.nblocks + kWarps - 1) / kWarps, (int64_t)sms * per_sm);
+  mma_chain_kernel<CH, NO, POOL><<<grid, 32 * kWarps, d.smem_bytes, s>>>(d, p, tcw);
+}
+
+}  // namespace
+
+void launch_mma_chain(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  const int no = d.Nout <= 32 ? 4 : d.Nout <= 64 ? 8 : 16;
+  if (d.pool) {
+    if (no == 4) launch_t<64, 4, true>(d, tcw, p, s);
+    else if (no == 8) launch_t<64, 8, true>(d, tcw, p, s);
+    else launch_t<64, 16, true>(d, tcw, p, s);
+    return;
+  }
+  if (d.CH == 64) {
+    if (no == 4) launch_t<64, 4, false>(d, tcw, p, s);
+    else if (no == 8) launch_t<64, 8, false>(d, tcw, p, s);
+    else launch_t<64, 16, false>(d, tcw, p, s);
+  } else {
+    if (no == 4) launch_t<128, 4, false>(d, tcw, p, s);
+    else if (no == 8) launch_t<128, 8, false>(d, tcw, p, s);
+    else launch_t<128, 16, false>(d, tcw, p, s);
+  }
+}
+
+}  // namespace temco

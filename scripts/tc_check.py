@@ -1,9 +1,9 @@
-"""Quick GPU check of the tcgen05 path vs the SIMT path and the oracle."""
-import sys, time, os
+"""Quick GPU check of the fused-group kernel paths vs the oracle."""
+import sys, os
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
 import workloads as W, oracle
-from paper_conf_icpp_songljkj0024_b200 import Plan, FLAG_SIMT_ONLY
+from paper_conf_icpp_songljkj0024_b200 import Plan, FLAG_SIMT_ONLY, FLAG_MMA_SMALL
 
 def run(m, flags, x):
     p = Plan(m, flags=flags)
@@ -20,8 +20,10 @@ for m in cases:
     x = W.make_input(m)
     ref = oracle.run_temco(oracle.plan(m), x)
     p, y = run(m, 0, x)
+    _, yt = run(m, FLAG_MMA_SMALL, x)
     _, ys = run(m, FLAG_SIMT_ONLY, x)
     kinds = {}
     for s in p.describe()["steps"]:
         kinds[s["kernel"]] = kinds.get(s["kernel"], 0) + 1
-    print(m.name, "tc vs oracle %.3e" % rel(y, ref), "simt vs oracle %.3e" % rel(ys, ref), "tc vs simt %.3e" % rel(y, ys), kinds, flush=True)
+    print(m.name, "default %.3e" % rel(y, ref), "mma-small %.3e" % rel(yt, ref), "simt %.3e" % rel(ys, ref),
+          "finite", bool(np.isfinite(y).all()), kinds, flush=True)
