@@ -585,7 +585,8 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
     }
     std::string terr;
     for (auto& e : P->exec)
-      if (e.kind == K_CONV_TC && !conv_tc_finalize(e.ctc, P->tcw_d, terr)) {
+      if (e.kind == K_CONV_TC && (!conv_tc_finalize(e.ctc, P->tcw_d, terr) ||
+                                   !conv_tc_finalize_x(e.ctc, P->arena_d + e.ctc.x.off, terr))) {
         free_device(P);
         delete P;
         return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);

@@ -19,6 +19,12 @@ namespace temco {
 
 struct ConvTcDesc {
   alignas(64) unsigned char wmap[128];   // CUtensorMap of W [Np x Kp], box {64, Np}
+  alignas(64) unsigned char xmap[128];   // TMA mode: 4D map of x [N, H, W, Cin], box {64, tw*s, th*s, tn}
+  // TMA mode (Cin % 8 == 0): output tiles are spatial boxes tn x th x tw (<= 128
+  // pixels); tap (a, b) of 64-channel atom kc is one tap-shifted, strided box
+  // load (hardware zero padding), K index = (tap * kpt + kc) * 64 + c
+  int32_t tma, s, kpt, taps;
+  int32_t tw, th, tn, nwb, nhb, nnb, mused;
   Loc x, y;
   int32_t N, H, W, Cin;
   int32_t Ho, Wo, kh, kw, sh, sw, ph, pw;
@@ -37,6 +43,7 @@ struct ConvTcDesc {
 bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                    std::vector<float>& params, ConvTcDesc& d);
 bool conv_tc_finalize(ConvTcDesc& d, uint16_t* tcw, std::string& err);
+bool conv_tc_finalize_x(ConvTcDesc& d, const void* x, std::string& err);   // TMA mode: input tensor map
 void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s);
 
 }  // namespace temco

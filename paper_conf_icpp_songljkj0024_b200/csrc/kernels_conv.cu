@@ -52,17 +52,38 @@ bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::ve
   d.katoms = (d.K + 63) / 64;
   d.npix = (int64_t)ir.batch * v.H * v.W;
   d.ntiles = (int)((d.npix + 127) / 128);
+  d.taps = v.kh * v.kw;
+  d.s = v.sh;
+  // TMA mode: 16-byte channel rows, square stride / padding, strided boxes <= 256
+  d.tma = (x.C % 8 == 0 && v.sh == v.sw && v.ph == v.pw && xl.where == W_ARENA) ? 1 : 0;
+  if (d.tma) {
+    d.kpt = (x.C + 63) / 64;
+    d.katoms = d.taps * d.kpt;
+    d.tw = std::min(v.W, 128);
+    d.th = std::min(v.H, 128 / d.tw);
+    d.tn = (d.th == v.H && d.tw == v.W) ? std::max(1, std::min(ir.batch, 128 / (v.H * v.W))) : 1;
+    d.nwb = (v.W + d.tw - 1) / d.tw;
+    d.nhb = (v.H + d.th - 1) / d.th;
+    d.nnb = (ir.batch + d.tn - 1) / d.tn;
+    d.mused = d.tw * d.th * d.tn;
+    d.ntiles = d.nnb * d.nhb * d.nwb;
+    if (d.tw * d.s > 256 || d.th * d.s > 256) d.tma = 0;
+  }
+  if (!d.tma) d.katoms = (d.K + 63) / 64;
   const int wbytes = d.katoms * d.Np * 128;
   if (wbytes > 112 * 1024) return false;
-  // weights [Np][katoms*64] bf16, k = (a*kw + b)*Cin + c
   const int Kp = d.katoms * 64;
   std::vector<uint16_t> w((size_t)d.Np * Kp, 0);
   const std::vector<float>& src = *v.w;   // OIHW
   for (int o = 0; o < v.C; ++o)
     for (int c = 0; c < x.C; ++c)
       for (int a = 0; a < v.kh; ++a)
-        for (int b = 0; b < v.kw; ++b)
-          w[(size_t)o * Kp + (a * v.kw + b) * x.C + c] = f2bf(src[(((size_t)o * x.C + c) * v.kh + a) * v.kw + b]);
+        for (int b = 0; b < v.kw; ++b) {
+          // TMA mode: k = (tap * kpt + c / 64) * 64 + c % 64; gather mode: k = tap * Cin + c
+          const int tap = a * v.kw + b;
+          const size_t k = d.tma ? (size_t)(tap * d.kpt) * 64 + c : (size_t)tap * x.C + c;
+          w[(size_t)o * Kp + k] = f2bf(src[(((size_t)o * x.C + c) * v.kh + a) * v.kw + b]);
+        }
   while (tcw.size() % 512) tcw.push_back(0);
   d.w = (int64_t)tcw.size();
   tcw.insert(tcw.end(), w.begin(), w.end());
@@ -103,6 +124,29 @@ bool conv_tc_finalize(ConvTcDesc& d, uint16_t* tcw, std::string& err) {
                       CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) {
     err = "cuTensorMapEncodeTiled failed (conv weights)";
+    return false;
+  }
+  return true;
+}
+
+bool conv_tc_finalize_x(ConvTcDesc& d, const void* x, std::string& err) {
+  if (!d.tma) return true;
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
+    err = "cuTensorMapEncodeTiled unavailable";
+    return false;
+  }
+  auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  cuuint64_t dims[4] = {(cuuint64_t)d.Cin, (cuuint64_t)d.W, (cuuint64_t)d.H, (cuuint64_t)d.N};
+  cuuint64_t strides[3] = {(cuuint64_t)d.Cin * 2, (cuuint64_t)d.W * d.Cin * 2, (cuuint64_t)d.H * d.W * d.Cin * 2};
+  cuuint32_t box[4] = {64, (cuuint32_t)(d.tw * d.s), (cuuint32_t)(d.th * d.s), (cuuint32_t)d.tn};
+  cuuint32_t es[4] = {1, (cuuint32_t)d.s, (cuuint32_t)d.s, 1};
+  CUresult r = encode(reinterpret_cast<CUtensorMap*>(d.xmap), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(x),
+                      dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    err = "cuTensorMapEncodeTiled failed (conv input)";
     return false;
   }
   return true;
@@ -309,6 +353,135 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
   }
 }
 
+
+// TMA mode: 6 warps -- 0-3 epilogue, 4 TMA producer (weights once, then one
+// tap-shifted strided box per (tap, 64-channel atom)), 5 MMA issuer.
+constexpr int kConvTmaThreads = 192;
+
+__global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __grid_constant__ ConvTcDesc d, RunPtrs p) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  const int S = d.stages;
+  const int wbytes = d.katoms * d.Np * 128;
+  uint8_t* wres = smem;
+  uint8_t* ring = smem + wbytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ring + S * 16384);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + S;
+  uint64_t* acc_full = bars + 2 * S;
+  uint64_t* acc_empty = acc_full + 2;
+  uint64_t* wbar = acc_empty + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wbar + 1);
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&acc_full[b], 1);
+      mbar_init(&acc_empty[b], 128);
+    }
+    mbar_init(wbar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(d.tmem_cols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tbase = *tmem_slot;
+  const int per_img = d.nhb * d.nwb;
+
+  if (warp == 4) {
+    if (lane == 0) {
+      mbar_expect_tx(wbar, wbytes);
+      for (int kb = 0; kb < d.katoms; ++kb) tma_load_2d(wres + kb * d.Np * 128, d.wmap, wbar, kb * 64, 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      const uint32_t bytes = 128u * d.tw * d.th * d.tn;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+        const int nb = tile / per_img, rem = tile % per_img;
+        const int n0 = nb * d.tn, h0 = (rem / d.nwb) * d.th, w0 = (rem % d.nwb) * d.tw;
+        for (int tap = 0; tap < d.taps; ++tap) {
+          const int a = tap / d.kw, b = tap % d.kw;
+          for (int kc = 0; kc < d.kpt; ++kc) {
+            mbar_wait(&empty[stage], phase ^ 1);
+            mbar_expect_tx(&full[stage], bytes);
+            tma_load_4d(ring + stage * 16384, d.xmap, &full[stage], kc * 64, w0 * d.s - d.pw + b, h0 * d.s - d.ph + a, n0);
+            if (++stage == S) stage = 0, phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 5) {
+    if (lane == 0) {
+      mbar_wait(wbar, 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      const uint32_t id = idesc_bf16(128, d.Np);
+      int it = 0;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+        const int buf = it & 1;
+        mbar_wait(&acc_empty[buf], ((it >> 1) & 1) ^ 1);
+        tc_fence_after();
+        const uint32_t tacc = tbase + buf * d.Np;
+        for (int tap = 0; tap < d.taps; ++tap)
+          for (int kc = 0; kc < d.kpt; ++kc) {
+            mbar_wait(&full[stage], phase);
+            tc_fence_after();
+            const uint32_t sa = smem_u32(ring + stage * 16384);
+            const uint32_t sb = smem_u32(wres + (tap * d.kpt + kc) * d.Np * 128);
+            const int nk = min(4, (d.Cin - kc * 64 + 15) / 16);
+            for (int k = 0; k < nk; ++k)
+              mma_bf16(tacc, umma_desc(sa + 32 * k), umma_desc(sb + 32 * k), id, (tap | kc | k) ? 1u : 0u);
+            mma_commit(&empty[stage]);
+            if (++stage == S) stage = 0, phase ^= 1;
+          }
+        mma_commit(&acc_full[buf]);
+      }
+    }
+  } else {
+    const int row = threadIdx.x;
+    const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
+    __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+    const int wi = row % d.tw, hi = (row / d.tw) % d.th, ni = row / (d.tw * d.th);
+    int it = 0;
+    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+      const int buf = it & 1;
+      const int nb = tile / per_img, rem = tile % per_img;
+      const int n = nb * d.tn + ni, ho = (rem / d.nwb) * d.th + hi, wo = (rem % d.nwb) * d.tw + wi;
+      const bool valid = row < d.mused && n < d.N && ho < d.Ho && wo < d.Wo;
+      const int64_t m = ((int64_t)n * d.Ho + ho) * d.Wo + wo;
+      mbar_wait(&acc_full[buf], (it >> 1) & 1);
+      tc_fence_after();
+      for (int g = 0; g < d.Np / 8; ++g) {
+        uint32_t v[8];
+        tmem_ld8(tbase + lane_off + buf * d.Np + g * 8, v);
+        tmem_wait_ld();
+        if (valid && g * 8 < d.Nout) {
+          float f[8];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.b >= 0 ? __ldg(p.params + d.b + g * 8 + i) : 0.f);
+          *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) =
+              make_uint4(pack_bf16(f[0], f[1]), pack_bf16(f[2], f[3]), pack_bf16(f[4], f[5]), pack_bf16(f[6], f[7]));
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[buf]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase), "r"(d.tmem_cols));
+  }
+}
+
 }  // namespace
 
 void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s) {
@@ -316,13 +489,17 @@ void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s) {
   static int sms = 0;
   if (!configured) {
     cudaFuncSetAttribute(conv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(conv_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
   const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);   // persistent, one CTA per SM
-  conv_tc_kernel<<<grid, kConvThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+  if (d.tma)
+    conv_tma_kernel<<<grid, kConvTmaThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+  else
+    conv_tc_kernel<<<grid, kConvThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }
 
 }  // namespace temco

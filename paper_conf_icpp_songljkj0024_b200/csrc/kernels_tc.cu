@@ -1,20 +1,23 @@
-// tcgen05 fused restore-chain -> BN -> add -> ReLU -> reduce kernel (sm_100a).
+// tcgen05 fused restore-chain -> BN -> add -> ReLU -> [pool] -> reduce kernel (sm_100a).
 //
 // One fused group computes, per 128-pixel tile,
 //     t_l = act_l( sum_{j in l} r_j Lhat_j^T + b_l + t_{l-1} ),  out = t_D F^T
 // with the C-wide t never leaving the SM:
-//   GEMM1  TMA (r_j atom [128 x 64], Lhat_j atom [Cc x 64]) -> SMEM ring ->
-//          tcgen05.mma (M=128, N=Cc, K=16) -> TMEM accumulator (Cc fp32 columns)
-//   level epilogue: TMEM -> registers, + b_l, ReLU, -> TMEM (tcgen05.st) so the
-//          next level's MMAs accumulate on top of t_{l-1}; after the last level
-//          the bf16 tile P = t_D is written to SMEM in the SW128 K-major layout
-//   GEMM2  tcgen05.mma (A = P from SMEM, B = F atom via TMA) -> TMEM (Np columns),
-//          accumulated over the C chunks
+//   GEMM1  r_j atoms [128 x 64] (TMA, or cp.async gather warps for pooled
+//          chains) and Lhat_j atoms [Cc x 64] (TMA) -> SMEM ring -> tcgen05.mma
+//          (M=128, N=Cc, K=16) -> TMEM accumulator; the level bias enters the
+//          same accumulator through the tensor core (constant SMEM ones tile x
+//          [b_hi, b_lo] columns), so the epilogue does no bias loads
+//   level epilogue (8 warps: lane quarter x column half): TMEM -> registers,
+//          ReLU, -> TMEM (tcgen05.st) so the next level accumulates on top of
+//          t_{l-1}; after the last level the bf16 tile P = t_D goes to SMEM in
+//          the SW128 K-major layout (or, pooled chains, into a running max / sum
+//          per tap; GAP roots reduce per image)
+//   GEMM2  tcgen05.mma (A = P from SMEM, B = F atom via TMA) -> TMEM (Np columns)
 //   output epilogue: TMEM -> registers -> bf16 -> global.
-// Warp roles (192 threads, persistent over tiles): warps 0-3 epilogue (warp w
-// owns TMEM lanes 32w..32w+31 = pixel rows), warp 4 TMA producer, warp 5 MMA
-// issuer.  Two TMEM accumulators (chunks c, c+1) let the MMA of one chunk
-// overlap the epilogue of the other.
+// Warp roles (448 threads, persistent over tiles): warps 0-7 epilogue, 8 TMA
+// producer, 9 MMA issuer, 10-13 gather (pooled chains).  Two TMEM accumulators
+// let the MMA of one unit overlap the epilogue of the other.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cudaTypedefs.h>
@@ -42,6 +45,13 @@ uint16_t to_bf16(float f) {
   return (uint16_t)(u >> 16);
 }
 
+float from_bf16(uint16_t h) {
+  uint32_t u = (uint32_t)h << 16;
+  float f;
+  memcpy(&f, &u, 4);
+  return f;
+}
+
 int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
   while (pool.size() % 512) pool.push_back(0);   // 1024-byte aligned blocks (TMA base alignment)
   int64_t off = (int64_t)pool.size();
@@ -49,18 +59,11 @@ int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
   return off;
 }
 
-int64_t push_f32(std::vector<float>& pool, const std::vector<double>& v) {
-  while (pool.size() % 4) pool.push_back(0.f);
-  int64_t off = (int64_t)pool.size();
-  for (double x : v) pool.push_back((float)x);
-  while (pool.size() % 4) pool.push_back(0.f);
-  return off;
-}
-
 }  // namespace
 
 bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                     std::vector<float>& params, TcChainDesc& d) {
+  (void)params;
   const Node& root = ir.nodes[s.out];
   const bool gap = root.op == OP_GAP;
   if (root.role != ROLE_FCONV && !gap) return false;
@@ -69,6 +72,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   const int C = tn.C, Nout = gap ? 16 : root.C;
   if (Nout % 8 || Nout > 256) return false;
   if (gap && tn.H * tn.W > 128) return false;
+  if (!gap && root.b) return false;              // fconv factors carry no bias (O1)
   // pooled chain (Listing 1 with p >= 2): root fconv <- max/avg pool <- level chain
   int pool = 0, pk = 1, ps = 1, pp = 0, csrc = tsrc;
   if (!gap && (tn.op == OP_MAXPOOL || tn.op == OP_AVGPOOL) && s.members.size() > 2) {
@@ -86,7 +90,6 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   int nterms = 0;
   for (auto& L : levels) nterms += (int)L.terms.size();
   if ((int)levels.size() > kTcMaxLevels || nterms > kTcMaxTerms) return false;
-  // term inputs: bf16 reduced tensors in the arena, ranks % 8 == 0
   for (auto& L : levels)
     for (auto& t : L.terms) {
       const int r = ir.oin[t.lconv][0];
@@ -99,7 +102,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d = TcChainDesc();
   d.C = C;
   d.Cc = (C <= 64 || pool) ? 64 : 128;
-  d.gather = pool ? 1 : 0;
+  d.gather = 0;
   d.pool = pool; d.pk = pk; d.ps = ps; d.pp = pp; d.taps = pk * pk;
   d.Hin = cn.H; d.Win = cn.W; d.Ho = tn.H; d.Wo = tn.W;
   d.Cpad = (C + d.Cc - 1) / d.Cc * d.Cc;
@@ -114,6 +117,18 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.ipt = 128 / d.hw;
     d.rows_per_tile = d.ipt * d.hw;
     d.ntiles = (ir.batch + d.ipt - 1) / d.ipt;
+  } else if (pool) {
+    d.ipt = 0;
+    d.rows_per_tile = 128;
+    d.tw = std::min(tn.W, 128);
+    d.th = std::min(tn.H, 128 / d.tw);
+    d.tn = (d.th == tn.H && d.tw == tn.W) ? std::max(1, std::min(ir.batch, 128 / (tn.H * tn.W))) : 1;
+    d.nwb = (tn.W + d.tw - 1) / d.tw;
+    d.nhb = (tn.H + d.th - 1) / d.th;
+    d.nnb = (ir.batch + d.tn - 1) / d.tn;
+    d.mused = d.tw * d.th * d.tn;
+    d.ntiles = d.nnb * d.nhb * d.nwb;
+    if (d.tw * ps > 256 || d.th * ps > 256) return false;
   } else {
     d.ipt = 0;
     d.rows_per_tile = 128;
@@ -126,9 +141,16 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
     d.relu[l] = L.relu ? 1 : 0;
-    std::vector<double> bias(d.Cpad, 0.0);
-    std::copy(L.bias.begin(), L.bias.end(), bias.begin());
-    d.bias[l] = push_f32(params, bias);
+    d.bias[l] = -1;
+    // bias as a rank-2 term: columns 0, 1 = bf16 hi / lo parts (error ~2^-16 |b|)
+    std::vector<float> bm((size_t)d.Cpad * 8, 0.f);
+    for (int c = 0; c < C; ++c) {
+      const float b = (float)L.bias[c];
+      const float hi = from_bf16(to_bf16(b));
+      bm[(size_t)c * 8 + 0] = hi;
+      bm[(size_t)c * 8 + 1] = b - hi;
+    }
+    d.boff[l] = push_bf16(tcw, bm);
     for (const PTerm& t : L.terms) {
       const Node& lc = ir.nodes[t.lconv];
       const int r = ir.oin[t.lconv][0];
@@ -137,12 +159,13 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
       T.r = loc.at(r);
       T.R = R;
       T.Rp = (R + 63) / 64 * 64;
+      T.Rw = (R + 7) / 8 * 8;
       T.c0 = t.c0;
       T.C = lc.C;
-      std::vector<float> w((size_t)d.Cpad * T.Rp, 0.f);
+      std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);
       for (int c = 0; c < lc.C; ++c)
         for (int k = 0; k < R; ++k)
-          w[(size_t)(t.c0 + c) * T.Rp + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
+          w[(size_t)(t.c0 + c) * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
       T.w = push_bf16(tcw, w);
       flops_terms += 2LL * lc.C * R;
       bytes_terms += 2LL * R;
@@ -160,21 +183,17 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     for (int o = 0; o < Nout; ++o)
       for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
     d.F = push_bf16(tcw, f);
-    if (root.b) {
-      std::vector<double> fb(root.b->begin(), root.b->end());
-      d.Fb = push_f32(params, fb);
-    }
     const int64_t nin = (int64_t)ir.batch * cn.H * cn.W;   // chain evaluated once per input pixel
     d.alg_flops = nin * flops_terms + d.npix * 2LL * Nout * C;
     d.alg_bytes = nin * bytes_terms + d.npix * 2LL * Nout;
   }
-  // shared memory: ring of (A 16 KB | B slot) stages + two P tiles + barriers
+  // shared memory: ring of (A 16 KB | B slot) stages + two P tiles + ones tile + barriers
   d.slot_b = std::max(d.Cc, d.Np) * 128;
   const int pbytes = 128 * d.Cc * 2;
-  const int budget = 227 * 1024 - 1024 /*align*/ - 512 /*barriers*/ - 2 * pbytes;
+  const int budget = 227 * 1024 - 1024 /*align*/ - 1024 /*barriers*/ - 2 * pbytes - 16384 /*ones*/;
   d.stages = std::min(6, budget / (16384 + d.slot_b));
   if (d.stages < 2) return false;
-  d.smem_bytes = 1024 + d.stages * (16384 + d.slot_b) + 2 * pbytes + 512;
+  d.smem_bytes = 1024 + d.stages * (16384 + d.slot_b) + 2 * pbytes + 16384 + 1024;
   const int cols = 2 * d.Cc + d.Np;
   d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
   return true;
@@ -205,17 +224,36 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
   };
+  auto make4 = [&](unsigned char* dst, void* base, const TcChainDesc* d, int R) {
+    cuuint64_t dims[4] = {(cuuint64_t)R, (cuuint64_t)d->Win, (cuuint64_t)d->Hin, (cuuint64_t)d->nimg};
+    cuuint64_t strides[3] = {(cuuint64_t)R * 2, (cuuint64_t)d->Win * R * 2, (cuuint64_t)d->Hin * d->Win * R * 2};
+    cuuint32_t box[4] = {64, (cuuint32_t)(d->tw * d->ps), (cuuint32_t)(d->th * d->ps), (cuuint32_t)d->tn};
+    cuuint32_t es[4] = {1, (cuuint32_t)d->ps, (cuuint32_t)d->ps, 1};
+    CUresult r = encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides,
+                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
+  };
   for (size_t i = 0; i < n; ++i) {
     TcChainDesc* d = get(i);
     if (!d) continue;
     for (int j = 0; j < d->n_terms; ++j) {
       TcTerm& t = d->term[j];
-      if (!make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->npix, 128) ||
-          !make(t.wmap, tcw + t.w, (uint64_t)t.Rp, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+      if (d->pool && !make4(t.tmap4, arena + t.r.off, d, t.R)) {
+        err = "cuTensorMapEncodeTiled failed (pooled term)";
+        return false;
+      }
+      if (!make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->nimg * d->Hin * d->Win, 128) ||
+          !make(t.wmap, tcw + t.w, (uint64_t)t.Rw, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
         err = "cuTensorMapEncodeTiled failed (term)";
         return false;
       }
     }
+    for (int l = 0; l < d->n_levels; ++l)
+      if (!make(d->bmap[l], tcw + d->boff[l], 8, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+        err = "cuTensorMapEncodeTiled failed (bias)";
+        return false;
+      }
     if (!d->gap && !make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
       err = "cuTensorMapEncodeTiled failed (F)";
       return false;
@@ -234,14 +272,16 @@ __device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
   return t.c0 < (c + 1) * Cc && t.c0 + t.C > c * Cc;
 }
 
-constexpr int kThreads = 320;   // warps 0-3 epilogue, 4 TMA producer, 5 MMA, 6-9 gather (gather mode)
+constexpr int kEpiWarps = 8;
+constexpr int kProdWarp = 8, kMmaWarp = 9, kGatherWarp0 = 10;
+constexpr int kThreads = 32 * 14;
 constexpr int kSlotA = 16384;
 
 // The MMA work of one tile is a sequence of "units": chunk c of the restored
 // width (and, for a pooled chain, tap tau of the pooling window).  Units are
 // processed in pairs (two TMEM accumulators) -- consecutive chunks, or
 // consecutive taps of one chunk -- and every role walks the same order:
-//   for pair: for level l: for unit in pair: G1(unit, l) [+ epilogue E(unit, l)]
+//   for pair: for level l: for unit in pair: [bias stage, term stages] + epilogue
 //             then G2 for every chunk whose restored values are final.
 struct PairIter {
   int c0, t0, nb;
@@ -262,7 +302,6 @@ __device__ __forceinline__ void unit_of(const TcChainDesc& d, const PairIter& it
        (d).pool ? ((it.t0 += 2) >= (d).taps ? (it.t0 = 0, ++it.c0) : 0) : (it.c0 += 2))             \
     if ((it.nb = (d).pool ? min(2, (d).taps - it.t0) : min(2, (d).nchunks - it.c0)), true)
 
-// chunks whose G2 follows this pair: non-pool -> c0 .. c0+nb-1; pool -> c0 after its last tap
 __device__ __forceinline__ int g2_count(const TcChainDesc& d, const PairIter& it) {
   if (d.gap) return 0;
   if (d.pool) return it.t0 + it.nb == d.taps ? 1 : 0;
@@ -278,7 +317,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   const int pbytes = 128 * Cc * 2;
   uint8_t* ring = smem;
   uint8_t* pbuf = ring + S * slot;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(pbuf + 2 * pbytes);
+  uint8_t* ones = pbuf + 2 * pbytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ones + 16384);
   uint64_t* full = bars;
   uint64_t* empty = bars + S;
   uint64_t* acc_full = bars + 2 * S;
@@ -290,6 +330,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(out_empty + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  // constant A operand of the bias MMA: K columns 0 and 1 = 1.0 (bf16), SW128 layout
+  for (int i = threadIdx.x; i < 16384 / 16; i += blockDim.x) {
+    const int row = i / 8, ch = i % 8;
+    uint4 v = make_uint4(0, 0, 0, 0);
+    if (ch == (row & 7)) v.x = 0x3F803F80u;          // logical chunk 0 of this row
+    reinterpret_cast<uint4*>(ones)[i] = v;
+  }
+  fence_proxy_async();
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], d.gather ? 33 : 1);
@@ -297,12 +345,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&acc_full[b], 1);
-      mbar_init(&acc_empty[b], 128);
-      mbar_init(&p_full[b], 128);
+      mbar_init(&acc_empty[b], 32 * kEpiWarps);
+      mbar_init(&p_full[b], 32 * kEpiWarps);
       mbar_init(&p_empty[b], 1);
     }
     mbar_init(out_full, 1);
-    mbar_init(out_empty, 128);
+    mbar_init(out_empty, 32 * kEpiWarps);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) {
@@ -315,19 +363,32 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
 
-  if (warp == 4) {
+  if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      const uint32_t bytes_b = Cc * 128, bytes_a = d.gather ? 0 : kSlotA, bytes_f = d.Np * 128;
+      const uint32_t bytes_b = Cc * 128, bytes_f = d.Np * 128;
+      const uint32_t bytes_a = d.gather ? 0 : d.pool ? 128u * d.tw * d.th * d.tn : (uint32_t)kSlotA;
+      const int per_img = d.nhb * d.nwb;
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
         const int m0 = tile * d.rows_per_tile;
+        int n0 = 0, h0 = 0, w0 = 0;
+        if (d.pool) {
+          const int nb = tile / per_img, rem = tile % per_img;
+          n0 = nb * d.tn;
+          h0 = (rem / d.nwb) * d.th;
+          w0 = (rem % d.nwb) * d.tw;
+        }
         FOR_PAIRS(d, it) {
           for (int l = 0; l < d.n_levels; ++l)
             for (int bi = 0; bi < it.nb; ++bi) {
               int c, tap;
               unit_of(d, it, bi, c, tap);
+              mbar_wait(&empty[stage], phase ^ 1);                 // bias stage
+              mbar_expect_tx(&full[stage], bytes_b);
+              tma_load_2d(ring + stage * slot + kSlotA, d.bmap[l], &full[stage], 0, c * Cc);
+              if (++stage == S) stage = 0, phase ^= 1;
               for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
                 const TcTerm& t = d.term[j];
                 if (!term_hits(t, c, Cc)) continue;
@@ -335,7 +396,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   mbar_wait(&empty[stage], phase ^ 1);
                   mbar_expect_tx(&full[stage], bytes_a + bytes_b);
                   uint8_t* sa = ring + stage * slot;
-                  if (!d.gather) tma_load_2d(sa, t.tmap, &full[stage], ka * 64, m0);
+                  if (d.pool)       // tap-shifted strided box of the chain-resolution input
+                    tma_load_4d(sa, t.tmap4, &full[stage], ka * 64, w0 * d.ps - d.pp + tap % d.pk,
+                                h0 * d.ps - d.pp + tap / d.pk, n0);
+                  else if (!d.gather)
+                    tma_load_2d(sa, t.tmap, &full[stage], ka * 64, m0);
                   tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * 64, c * Cc);
                   if (++stage == S) stage = 0, phase ^= 1;
                 }
@@ -353,12 +418,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
         }
       }
     }
-  } else if (warp >= 6) {
+  } else if (warp >= kGatherWarp0) {
     // ------------------------------------------------------------ gather producer (A rows)
     // warp-per-stage: gather warp gw fills every 4th stage of the ring (lane
     // owns rows lane + 32 i), so 4 stages of cp.async are in flight at once
     if (d.gather) {
-      const int gw = warp - 6;
+      const int gw = warp - kGatherWarp0;
       int64_t kseq = 0;
       auto next = [&](int& stage, uint32_t& phase) {
         stage = (int)(kseq % S);
@@ -383,6 +448,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
             for (int bi = 0; bi < it.nb; ++bi) {
               int c, tap;
               unit_of(d, it, bi, c, tap);
+              {
+                int stage;
+                uint32_t phase;
+                if (next(stage, phase)) {                          // bias stage: no A rows
+                  mbar_wait(&empty[stage], phase ^ 1);
+                  cp_async_arrive(&full[stage]);
+                }
+              }
               for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
                 const TcTerm& t = d.term[j];
                 if (!term_hits(t, c, Cc)) continue;
@@ -420,24 +493,32 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
         }
       }
     }
-  } else if (warp == 5) {
+  } else if (warp == kMmaWarp) {
     // ------------------------------------------------------------ MMA issuer
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      uint32_t acc_use[2] = {0, 0}, p_use[2] = {0, 0}, tile_iter = 0;
+      uint32_t acc_use0 = 0, acc_use1 = 0, p_use0 = 0, p_use1 = 0, tile_iter = 0;
       const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
       const uint32_t tout = tbase + 2 * Cc;
+      const uint32_t ones_addr = smem_u32(ones);
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
         FOR_PAIRS(d, it) {
           for (int l = 0; l < d.n_levels; ++l)
             for (int bi = 0; bi < it.nb; ++bi) {
               int c, tap;
               unit_of(d, it, bi, c, tap);
-              mbar_wait(&acc_empty[bi], (acc_use[bi] & 1) ^ 1);
+              uint32_t& use = bi ? acc_use1 : acc_use0;
+              mbar_wait(&acc_empty[bi], (use & 1) ^ 1);
               tc_fence_after();
               const uint32_t tacc = tbase + bi * Cc;
-              bool first = (l == 0);
+              // bias (initialises the accumulator at level 0)
+              mbar_wait(&full[stage], phase);
+              tc_fence_after();
+              mma_bf16(tacc, umma_desc(ones_addr), umma_desc(smem_u32(ring + stage * slot + kSlotA)), id1,
+                       l == 0 ? 0u : 1u);
+              mma_commit(&empty[stage]);
+              if (++stage == S) stage = 0, phase ^= 1;
               for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
                 const TcTerm& t = d.term[j];
                 if (!term_hits(t, c, Cc)) continue;
@@ -447,21 +528,20 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   tc_fence_after();
                   const uint32_t sa = smem_u32(ring + stage * slot);
                   const int nk = min(4, (t.R - ka * 64 + 15) / 16);
-                  for (int k = 0; k < nk; ++k) {
-                    mma_bf16(tacc, umma_desc(sa + 32 * k), umma_desc(sa + kSlotA + 32 * k), id1, first ? 0u : 1u);
-                    first = false;
-                  }
+                  for (int k = 0; k < nk; ++k)
+                    mma_bf16(tacc, umma_desc(sa + 32 * k), umma_desc(sa + kSlotA + 32 * k), id1, 1u);
                   mma_commit(&empty[stage]);
                   if (++stage == S) stage = 0, phase ^= 1;
                 }
               }
               mma_commit(&acc_full[bi]);
-              ++acc_use[bi];
+              ++use;
             }
           for (int q = 0; q < g2_count(d, it); ++q) {
             const int c = it.c0 + (d.pool ? 0 : q);
             const int pb = c & 1;
-            mbar_wait(&p_full[pb], p_use[pb] & 1);
+            uint32_t& puse = pb ? p_use1 : p_use0;
+            mbar_wait(&p_full[pb], puse & 1);
             tc_fence_after();
             if (c == 0) {
               mbar_wait(out_empty, (tile_iter & 1) ^ 1);
@@ -479,7 +559,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               if (++stage == S) stage = 0, phase ^= 1;
             }
             mma_commit(&p_empty[pb]);
-            ++p_use[pb];
+            ++puse;
           }
         }
         if (!d.gap) mma_commit(out_full);
@@ -487,19 +567,30 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       }
     }
   } else {
-    // ------------------------------------------------------------ epilogue (128 threads)
-    const int row = threadIdx.x;                       // pixel row in the tile == TMEM lane
-    const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
-    uint32_t acc_use[2] = {0, 0}, p_use[2] = {0, 0}, tile_iter = 0;
+    // ------------------------------------------------------------ epilogue (8 warps)
+    // warp w: TMEM lane quarter q = w % 4 (pixel rows 32q..32q+31), column half h = w / 4
+    const int q = warp & 3, h = warp >> 2;
+    const int row = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    const int half = Cc / 2;                          // columns per warp (32 or 64)
+    const int c_lo = h * half;
+    uint32_t acc_use0 = 0, acc_use1 = 0, p_use0 = 0, p_use1 = 0, tile_iter = 0;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
-    float run[64];                                     // pooled values of the current chunk (pool mode, Cc = 64)
+    float run[32];                                    // pooled values (pool mode, Cc = 64 -> 32 per warp)
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-      const int64_t m = (int64_t)tile * d.rows_per_tile + row;
+      int64_t m = (int64_t)tile * d.rows_per_tile + row;
+      bool mvalid = m < d.npix;
       int ho = 0, wo = 0;
       if (d.pool) {
-        const int rem = (int)(m % (d.Ho * d.Wo));
-        ho = rem / d.Wo;
-        wo = rem % d.Wo;
+        // spatial tile: row -> (image, output row, output column)
+        const int per_img = d.nhb * d.nwb;
+        const int nb = tile / per_img, rem = tile % per_img;
+        const int ni = row / (d.tw * d.th), hi = (row / d.tw) % d.th, wi = row % d.tw;
+        const int n = nb * d.tn + ni;
+        ho = (rem / d.nwb) * d.th + hi;
+        wo = (rem % d.nwb) * d.tw + wi;
+        mvalid = row < d.mused && n < d.nimg && ho < d.Ho && wo < d.Wo;
+        m = ((int64_t)n * d.Ho + ho) * d.Wo + wo;
       }
       FOR_PAIRS(d, it) {
         for (int l = 0; l < d.n_levels; ++l) {
@@ -508,97 +599,113 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           for (int bi = 0; bi < it.nb; ++bi) {
             int c, tap;
             unit_of(d, it, bi, c, tap);
-            mbar_wait(&acc_full[bi], acc_use[bi] & 1);
-            ++acc_use[bi];
+            uint32_t& use = bi ? acc_use1 : acc_use0;
+            mbar_wait(&acc_full[bi], use & 1);
+            ++use;
             tc_fence_after();
             const int pb = c & 1;
             const bool writes_p = last && !d.gap && (!d.pool || tap == d.taps - 1);
             if (writes_p) {
-              mbar_wait(&p_empty[pb], (p_use[pb] & 1) ^ 1);
-              ++p_use[pb];
+              uint32_t& puse = pb ? p_use1 : p_use0;
+              mbar_wait(&p_empty[pb], (puse & 1) ^ 1);
+              ++puse;
             }
-            const float* bias = p.params + d.bias[l] + (int64_t)c * Cc;
+            const uint32_t ta = tbase + lane_off + bi * Cc + c_lo;
             uint8_t* P = pbuf + pb * pbytes;
-            if (d.pool && last) {
-              // pooled chain: fold this tap into the running max / sum (Cc == 64)
+            if (!last) {
+              // t_l = relu(acc) back into TMEM for the next level's MMAs
+              uint32_t v[2][32];
+              tmem_ld32(ta, v[0]);
+              if (half == 64) tmem_ld32(ta + 32, v[1]);
+              tmem_wait_ld();
+              if (relu) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[0][i] = __float_as_uint(fmaxf(__uint_as_float(v[0][i]), 0.f));
+                if (half == 64)
+#pragma unroll
+                  for (int i = 0; i < 32; ++i) v[1][i] = __float_as_uint(fmaxf(__uint_as_float(v[1][i]), 0.f));
+              }
+              tmem_st32(ta, v[0]);
+              if (half == 64) tmem_st32(ta + 32, v[1]);
+              tmem_wait_st();
+            } else if (d.pool) {
+              // pooled chain: fold this tap into the running max / sum (half == 32)
               const int hi = ho * d.ps - d.pp + tap / d.pk, wi = wo * d.ps - d.pp + tap % d.pk;
               const bool valid = hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
+              uint32_t v[32];
+              tmem_ld32(ta, v);
+              tmem_wait_ld();
 #pragma unroll
-              for (int g = 0; g < 2; ++g) {
-                uint32_t v[32];
-                tmem_ld32(tbase + lane_off + bi * Cc + g * 32, v);
-                tmem_wait_ld();
-#pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                  float x = __uint_as_float(v[i]) + __ldg(bias + g * 32 + i);
-                  x = relu ? fmaxf(x, 0.f) : x;
-                  float& r = run[g * 32 + i];
-                  if (d.pool == 1)
-                    r = tap == 0 ? (valid ? x : -INFINITY) : (valid ? fmaxf(r, x) : r);
-                  else
-                    r = tap == 0 ? x : r + x;
-                }
+              for (int i = 0; i < 32; ++i) {
+                float x = __uint_as_float(v[i]);
+                x = relu ? fmaxf(x, 0.f) : x;
+                if (d.pool == 1)
+                  run[i] = tap == 0 ? (valid ? x : -INFINITY) : (valid ? fmaxf(run[i], x) : run[i]);
+                else
+                  run[i] = tap == 0 ? x : run[i] + x;
               }
               if (writes_p) {
-                const float scale = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
+                const float sc = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
+                const int ch0 = c_lo / 8;
 #pragma unroll
-                for (int q = 0; q < 8; ++q) {
+                for (int qq = 0; qq < 4; ++qq) {
                   uint4 pk;
-                  pk.x = pack_bf16(run[8 * q + 0] * scale, run[8 * q + 1] * scale);
-                  pk.y = pack_bf16(run[8 * q + 2] * scale, run[8 * q + 3] * scale);
-                  pk.z = pack_bf16(run[8 * q + 4] * scale, run[8 * q + 5] * scale);
-                  pk.w = pack_bf16(run[8 * q + 6] * scale, run[8 * q + 7] * scale);
-                  *reinterpret_cast<uint4*>(P + row * 128 + ((q ^ (row & 7)) * 16)) = pk;
+                  pk.x = pack_bf16(run[8 * qq + 0] * sc, run[8 * qq + 1] * sc);
+                  pk.y = pack_bf16(run[8 * qq + 2] * sc, run[8 * qq + 3] * sc);
+                  pk.z = pack_bf16(run[8 * qq + 4] * sc, run[8 * qq + 5] * sc);
+                  pk.w = pack_bf16(run[8 * qq + 6] * sc, run[8 * qq + 7] * sc);
+                  *reinterpret_cast<uint4*>(P + row * 128 + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
                 }
               }
-            } else {
-              for (int g = 0; g < Cc / 32; ++g) {
-                const uint32_t ta = tbase + lane_off + bi * Cc + g * 32;
+            } else if (d.gap) {
+              // GAP root: per-image column means; tiles hold whole images so the
+              // summation order is fixed (deterministic, batch-invariant)
+              float* red = reinterpret_cast<float*>(pbuf + h * pbytes);
+              for (int g = 0; g < half / 32; ++g) {
                 uint32_t v[32];
-                tmem_ld32(ta, v);
+                tmem_ld32(ta + g * 32, v);
                 tmem_wait_ld();
-                float f[32];
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
-                  float x = __uint_as_float(v[i]) + __ldg(bias + g * 32 + i);
-                  f[i] = relu ? fmaxf(x, 0.f) : x;
+                  const float x = relu ? fmaxf(__uint_as_float(v[i]), 0.f) : __uint_as_float(v[i]);
+                  red[row * 32 + ((i + row) & 31)] = x;
                 }
-                if (!last) {
+                asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
+                for (int idx = row; idx < d.ipt * 32; idx += 128) {
+                  const int ii = idx / 32, col = idx % 32;
+                  const int n = tile * d.ipt + ii;
+                  float acc = 0.f;
+                  for (int r = ii * d.hw; r < (ii + 1) * d.hw; ++r) acc += red[r * 32 + ((col + r) & 31)];
+                  const int cg = c * Cc + c_lo + g * 32 + col;
+                  if (n < d.nimg && cg < d.C) y[(int64_t)n * d.C + cg] = __float2bfloat16_rn(acc / (float)d.hw);
+                }
+                asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
+              }
+            } else {
+              // last level: P = bf16 relu(acc) -> SMEM (SW128 K-major atoms of 64 columns)
+              for (int g = 0; g < half / 32; ++g) {
+                uint32_t v[32];
+                tmem_ld32(ta + g * 32, v);
+                tmem_wait_ld();
+                const int col = c_lo + g * 32;
+                uint8_t* atom = P + (col / 64) * 16384 + row * 128;
+                const int ch0 = (col % 64) / 8;
 #pragma unroll
-                  for (int i = 0; i < 32; ++i) v[i] = __float_as_uint(f[i]);
-                  tmem_st32(ta, v);
-                } else if (d.gap) {
-                  // GAP root: per-image column means of this 32-column group; tiles
-                  // hold whole images so the reduction order is fixed (deterministic)
-                  float* red = reinterpret_cast<float*>(pbuf);
+                for (int qq = 0; qq < 4; ++qq) {
+                  float f[8];
 #pragma unroll
-                  for (int i = 0; i < 32; ++i) red[row * 32 + ((i + row) & 31)] = f[i];
-                  asm volatile("bar.sync 1, 128;" ::: "memory");
-                  for (int idx = row; idx < d.ipt * 32; idx += 128) {
-                    const int ii = idx / 32, col = idx % 32;
-                    const int n = tile * d.ipt + ii;
-                    float acc = 0.f;
-                    for (int r = ii * d.hw; r < (ii + 1) * d.hw; ++r) acc += red[r * 32 + ((col + r) & 31)];
-                    const int cg = c * Cc + g * 32 + col;
-                    if (n < d.nimg && cg < d.C) y[(int64_t)n * d.C + cg] = __float2bfloat16_rn(acc / (float)d.hw);
+                  for (int i = 0; i < 8; ++i) {
+                    const float x = __uint_as_float(v[8 * qq + i]);
+                    f[i] = relu ? fmaxf(x, 0.f) : x;
                   }
-                  asm volatile("bar.sync 1, 128;" ::: "memory");
-                } else {
-                  const int col = g * 32;                     // within the chunk
-                  uint8_t* atom = P + (col / 64) * 16384 + row * 128;
-                  const int ch0 = (col % 64) / 8;
-#pragma unroll
-                  for (int q = 0; q < 4; ++q) {
-                    uint4 pk;
-                    pk.x = pack_bf16(f[8 * q + 0], f[8 * q + 1]);
-                    pk.y = pack_bf16(f[8 * q + 2], f[8 * q + 3]);
-                    pk.z = pack_bf16(f[8 * q + 4], f[8 * q + 5]);
-                    pk.w = pack_bf16(f[8 * q + 6], f[8 * q + 7]);
-                    *reinterpret_cast<uint4*>(atom + (((ch0 + q) ^ (row & 7)) * 16)) = pk;
-                  }
+                  uint4 pk;
+                  pk.x = pack_bf16(f[0], f[1]);
+                  pk.y = pack_bf16(f[2], f[3]);
+                  pk.z = pack_bf16(f[4], f[5]);
+                  pk.w = pack_bf16(f[6], f[7]);
+                  *reinterpret_cast<uint4*>(atom + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
                 }
               }
-              if (!last) tmem_wait_st();
             }
             tc_fence_before();
             mbar_arrive(&acc_empty[bi]);
@@ -610,23 +717,21 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
         }
       }
       if (d.gap) continue;
-      // output epilogue
+      // output epilogue: column groups of 8 split between the two warp halves
       mbar_wait(out_full, tile_iter & 1);
       ++tile_iter;
       tc_fence_after();
-      for (int g = 0; g < d.Np / 8; ++g) {
+      const int ng = d.Np / 8, gh = (ng + 1) / 2;
+      for (int g = h * gh; g < min(ng, (h + 1) * gh); ++g) {
         uint32_t v[8];
         tmem_ld8(tbase + lane_off + 2 * Cc + g * 8, v);
         tmem_wait_ld();
-        if (m < d.npix && g * 8 < d.Nout) {
-          float f[8];
-#pragma unroll
-          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.Fb >= 0 ? __ldg(p.params + d.Fb + g * 8 + i) : 0.f);
+        if (mvalid && g * 8 < d.Nout) {
           uint4 pk;
-          pk.x = pack_bf16(f[0], f[1]);
-          pk.y = pack_bf16(f[2], f[3]);
-          pk.z = pack_bf16(f[4], f[5]);
-          pk.w = pack_bf16(f[6], f[7]);
+          pk.x = pack_bf16(__uint_as_float(v[0]), __uint_as_float(v[1]));
+          pk.y = pack_bf16(__uint_as_float(v[2]), __uint_as_float(v[3]));
+          pk.z = pack_bf16(__uint_as_float(v[4]), __uint_as_float(v[5]));
+          pk.w = pack_bf16(__uint_as_float(v[6]), __uint_as_float(v[7]));
           *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) = pk;
         }
       }

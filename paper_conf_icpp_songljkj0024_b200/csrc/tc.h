@@ -27,9 +27,11 @@ constexpr int kTcMaxLevels = 16;
 
 struct TcTerm {
   alignas(64) unsigned char tmap[128];   // CUtensorMap of r  [npix x R], box {64, 128}
-  alignas(64) unsigned char wmap[128];   // CUtensorMap of Lhat [Cpad x Rp], box {64, Cc}
+  alignas(64) unsigned char wmap[128];   // CUtensorMap of Lhat [Cpad x Rw], box {64, Cc}
+  alignas(64) unsigned char tmap4[128];  // pooled chains: 4D map of r [N, Hin, Win, R], strided tap boxes
   Loc r;                 // reduced input [npix, R] bf16 (arena)
   int32_t R, Rp;         // rank; padded to a multiple of 64 (one 128-byte K atom)
+  int32_t Rw;            // row length of the packed weights (R rounded to 8; TMA zero-fills to Rp)
   int32_t c0, C;         // restored channels this term writes (concat members)
   int64_t w;             // tc weight pool offset (elements)
 };
@@ -37,6 +39,10 @@ struct TcTerm {
 struct TcChainDesc {
   TcTerm term[kTcMaxTerms];
   alignas(64) unsigned char fmap[128];   // CUtensorMap of F [Np x Cpad], box {64, Np}
+  // level biases enter the accumulator through the tensor core: a constant
+  // SMEM "ones" A tile (K columns 0, 1 = 1) times B = [b_hi, b_lo] per channel
+  alignas(64) unsigned char bmap[kTcMaxLevels][128];   // CUtensorMap of [Cpad x 8] bf16, box {64, Cc}
+  int64_t boff[kTcMaxLevels];            // tc weight pool offsets of the bias matrices
   int32_t n_terms, n_levels;
   int32_t lvl_end[kTcMaxLevels];         // terms [lvl_end[l-1], lvl_end[l]) accumulate into level l
   int32_t relu[kTcMaxLevels];
@@ -51,6 +57,9 @@ struct TcChainDesc {
   int32_t gather;                        // A rows gathered by 4 warps (cp.async) instead of TMA
   int32_t pool, pk, ps, pp, taps;        // pooled chain: 0 none / 1 max / 2 avg, window, stride, pad
   int32_t Hin, Win, Ho, Wo;              // chain resolution, root resolution
+  // pooled chains: output tiles are spatial boxes tn x th x tw (<= 128 pixels),
+  // tap (dh, dw) of a term is one strided 4D TMA box (zero-filled outside)
+  int32_t tw, th, tn, nwb, nhb, nnb, mused;
   int64_t F;                             // tc weight pool offset of F
   int64_t Fb;                            // params offset of the fconv bias or -1
   Loc y;                                 // output [npix, Nout] bf16
