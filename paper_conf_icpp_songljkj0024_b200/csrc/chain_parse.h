@@ -3,6 +3,16 @@
 //   t_l = act_l( sum_{j in l} diag(scale_j) L_j r_j + b_l + t_{l-1} )
 // BN layers fold into per-row scales and the level bias, adds merge terms
 // (P:L333), concats place terms at channel offsets (Fig. 9a).
+//
+// Pooled members (Listing 1 with p >= 2) inside a level:
+//  * avgpool over a *linear* member (e.g. DenseNet's transition output
+//    avgpool(lconv(r))) is linear, avgpool(L r + b) = L avgpool(r) + b, so its
+//    terms become "tap-accumulate" terms (k*k tap-shifted reads of r summed
+//    into the same accumulator, weights / k^2);
+//  * any other pool (max, or over a ReLU) becomes a PMember evaluated per tap:
+//    pool_tap( act(sum scale L r + b) ), then the level's own bias (the post-BN
+//    shift) and activation.  A BN after a max-pool folds through it only for
+//    positive scales (max(s x) = s max(x), s > 0); otherwise the parse fails.
 #pragma once
 
 #include <cmath>
@@ -18,12 +28,24 @@ struct PTerm {
   int lconv;
   std::vector<double> scale;   // per row of the lconv output
   int c0;
+  int tk = 1, ts = 1, tp = 0;  // tap-accumulate (folded avg pool): k x k window, stride, pad
+};
+
+struct PMember {               // pooled non-linear member (per-tap epilogue)
+  int c0 = 0, C = 0;
+  int kind = 1;                // 1 max, 2 avg
+  int k = 1, s = 1, p = 0;
+  int Hin = 0, Win = 0;
+  std::vector<PTerm> terms;
+  std::vector<double> bias;    // member bias (size C), scaled
+  bool relu = false;
 };
 
 struct PLevel {
   std::vector<PTerm> terms;
   std::vector<double> bias;
   bool relu = false;
+  std::vector<PMember> pm;
 };
 
 struct ChainParser {
@@ -49,10 +71,46 @@ struct ChainParser {
     L.bias.assign(C, 0.0);
     std::vector<PLevel> prev;
     if (!contribute(v, nullptr, 0, L, prev)) return false;
-    if (L.terms.empty()) return false;
+    if (L.terms.empty() && L.pm.empty()) return false;
     out = prev;
     out.push_back(L);
     return true;
+  }
+
+  // linear sub-expression (lconv / bn / add) at resolution (h, w): terms + bias
+  bool linear(int v, const std::vector<double>* sc, int c0, int h, int w, std::vector<PTerm>& terms,
+              std::vector<double>& bias, int bias_off) {
+    if (!members.count(v)) return false;
+    visited.insert(v);
+    const Node& n = ir.nodes[v];
+    if (n.H != h || n.W != w) return false;
+    if (n.role == ROLE_LCONV) {
+      PTerm t;
+      t.lconv = v;
+      t.c0 = c0;
+      t.scale = sc ? *sc : std::vector<double>(n.C, 1.0);
+      if (n.b)
+        for (int c = 0; c < n.C; ++c) bias[bias_off + c] += t.scale[c] * (*n.b)[c];
+      terms.push_back(std::move(t));
+      return true;
+    }
+    if (n.op == OP_BN) {
+      std::vector<double> s(n.C);
+      for (int c = 0; c < n.C; ++c) {
+        double k = (double)(*n.bn_g)[c] / std::sqrt((double)(*n.bn_v)[c] + (double)n.eps);
+        double sh = (double)(*n.bn_b)[c] - (double)(*n.bn_m)[c] * k;
+        double outer = sc ? (*sc)[c] : 1.0;
+        s[c] = outer * k;
+        bias[bias_off + c] += outer * sh;
+      }
+      return linear(ir.oin[v][0], &s, c0, h, w, terms, bias, bias_off);
+    }
+    if (n.op == OP_ADD) {
+      for (int x : ir.oin[v])
+        if (!linear(x, sc, c0, h, w, terms, bias, bias_off)) return false;
+      return true;
+    }
+    return false;
   }
 
   bool contribute(int v, const std::vector<double>* sc, int c0, PLevel& L, std::vector<PLevel>& prev) {
@@ -102,12 +160,60 @@ struct ChainParser {
         if (sc || c0 != 0 || n.C != C || !prev.empty()) return false;
         return chain(v, prev);
       }
+      case OP_MAXPOOL:
+      case OP_AVGPOOL: {
+        const int u = ir.oin[v][0];
+        const Node& un = ir.nodes[u];
+        // avg pool over a linear member: tap-accumulate terms (weights / k^2)
+        if (n.op == OP_AVGPOOL && ir.nodes[u].op != OP_RELU) {
+          std::vector<PTerm> terms;
+          std::vector<double> bias(n.C, 0.0);
+          std::set<int> saved = visited;
+          if (linear(u, sc, c0, un.H, un.W, terms, bias, 0)) {
+            const double inv = 1.0 / (n.kh * n.kw);
+            for (PTerm& t : terms) {
+              for (double& x : t.scale) x *= inv;
+              t.tk = n.kh;
+              t.ts = n.sh;
+              t.tp = 0;
+              L.terms.push_back(t);
+            }
+            for (int c = 0; c < n.C; ++c) L.bias[c0 + c] += bias[c];
+            visited.insert(v);
+            return true;
+          }
+          visited = saved;
+        }
+        // non-linear pooled member: act(sum scale L r + b) per tap, then pool
+        if (sc)
+          for (double x : *sc)
+            if (!(x > 0.0)) return false;
+        PMember m;
+        m.c0 = c0;
+        m.C = n.C;
+        m.kind = n.op == OP_MAXPOOL ? 1 : 2;
+        m.k = n.kh;
+        m.s = n.sh;
+        m.p = n.ph;
+        m.Hin = un.H;
+        m.Win = un.W;
+        m.bias.assign(n.C, 0.0);
+        int lin = u;
+        if (un.op == OP_RELU) {
+          if (!members.count(u)) return false;
+          visited.insert(u);
+          m.relu = true;
+          lin = ir.oin[u][0];
+        }
+        if (!linear(lin, sc, c0, un.H, un.W, m.terms, m.bias, 0)) return false;
+        L.pm.push_back(std::move(m));
+        return true;
+      }
       default:
         return false;
     }
   }
 };
-
 
 }  // namespace chainp
 }  // namespace temco

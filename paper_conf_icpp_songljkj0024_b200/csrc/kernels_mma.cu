@@ -54,7 +54,12 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
   if (!P.chain(csrc, levels)) return false;
   if (P.visited != P.members) return false;
   int nterms = 0;
-  for (auto& L : levels) nterms += (int)L.terms.size();
+  for (auto& L : levels) {
+    nterms += (int)L.terms.size();
+    if (!L.pm.empty()) return false;                 // pooled concat members: tcgen05 / generic paths
+    for (auto& t : L.terms)
+      if (t.tk > 1) return false;
+  }
   if ((int)levels.size() > kMmaMaxLevels || nterms > kMmaMaxTerms) return false;
   for (auto& L : levels)
     for (auto& t : L.terms) {

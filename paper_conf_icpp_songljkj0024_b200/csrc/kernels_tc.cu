@@ -1,23 +1,24 @@
-// tcgen05 fused restore-chain -> BN -> add -> ReLU -> [pool] -> reduce kernel (sm_100a).
+// tcgen05 fused restore-chain -> BN -> add/concat -> ReLU -> [pool] -> reduce kernel (sm_100a).
 //
-// One fused group computes, per 128-pixel tile,
+// One fused group computes, per output tile,
 //     t_l = act_l( sum_{j in l} r_j Lhat_j^T + b_l + t_{l-1} ),  out = t_D F^T
 // with the C-wide t never leaving the SM:
-//   GEMM1  r_j atoms [128 x 64] (TMA, or cp.async gather warps for pooled
-//          chains) and Lhat_j atoms [Cc x 64] (TMA) -> SMEM ring -> tcgen05.mma
-//          (M=128, N=Cc, K=16) -> TMEM accumulator; the level bias enters the
-//          same accumulator through the tensor core (constant SMEM ones tile x
-//          [b_hi, b_lo] columns), so the epilogue does no bias loads
-//   level epilogue (8 warps: lane quarter x column half): TMEM -> registers,
+//   GEMM1  r_j atoms [rows x 64] (2D TMA of 128 consecutive pixels, or 4D TMA of
+//          a tap-shifted, strided spatial box) and Lhat_j atoms [Cc x 64] (TMA)
+//          -> SMEM ring -> tcgen05.mma (M=128, N=Cc, K=16) -> TMEM accumulator;
+//          the level bias enters the same accumulator through the tensor core
+//          (constant SMEM ones tile x [b_hi, b_lo] columns)
+//   level epilogue (8 warps: TMEM lane quarter x column half): TMEM -> regs,
 //          ReLU, -> TMEM (tcgen05.st) so the next level accumulates on top of
 //          t_{l-1}; after the last level the bf16 tile P = t_D goes to SMEM in
-//          the SW128 K-major layout (or, pooled chains, into a running max / sum
-//          per tap; GAP roots reduce per image)
+//          the SW128 K-major layout.  Pooled-member chunks keep one TMEM region
+//          per tap and fold max / sum in registers; GAP roots reduce per image.
 //   GEMM2  tcgen05.mma (A = P from SMEM, B = F atom via TMA) -> TMEM (Np columns)
 //   output epilogue: TMEM -> registers -> bf16 -> global.
-// Warp roles (448 threads, persistent over tiles): warps 0-7 epilogue, 8 TMA
-// producer, 9 MMA issuer, 10-13 gather (pooled chains).  Two TMEM accumulators
-// let the MMA of one unit overlap the epilogue of the other.
+// Warp roles (320 threads, persistent over tiles): warps 0-7 epilogue, 8 TMA
+// producer, 9 MMA issuer.  Units (a chunk, or a tap group of a pooled chunk)
+// alternate between two TMEM buffers so one unit's MMAs overlap the previous
+// unit's epilogue.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cudaTypedefs.h>
@@ -33,7 +34,7 @@
 namespace temco {
 
 // ===========================================================================
-// host: lowering of a fused group into a level chain
+// host: lowering
 // ===========================================================================
 namespace {
 using namespace chainp;
@@ -59,52 +60,70 @@ int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
   return off;
 }
 
+// bias as a rank-2 term: columns 0, 1 = bf16 hi / lo parts (error ~2^-16 |b|)
+int64_t push_bias(std::vector<uint16_t>& pool, const std::vector<double>& b, int c0, int Cpad) {
+  std::vector<float> bm((size_t)Cpad * 8, 0.f);
+  for (size_t c = 0; c < b.size(); ++c) {
+    const float x = (float)b[c];
+    const float hi = from_bf16(to_bf16(x));
+    bm[(size_t)(c0 + c) * 8 + 0] = hi;
+    bm[(size_t)(c0 + c) * 8 + 1] = x - hi;
+  }
+  return push_bf16(pool, bm);
+}
+
 }  // namespace
 
 bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                     std::vector<float>& params, TcChainDesc& d) {
-  (void)params;
   const Node& root = ir.nodes[s.out];
   const bool gap = root.op == OP_GAP;
   if (root.role != ROLE_FCONV && !gap) return false;
+  if (!gap && root.b) return false;              // fconv factors carry no bias (O1)
   const int tsrc = ir.oin[s.out][0];
   const Node& tn = ir.nodes[tsrc];
   const int C = tn.C, Nout = gap ? 16 : root.C;
   if (Nout % 8 || Nout > 256) return false;
   if (gap && tn.H * tn.W > 128) return false;
-  if (!gap && root.b) return false;              // fconv factors carry no bias (O1)
-  // pooled chain (Listing 1 with p >= 2): root fconv <- max/avg pool <- level chain
-  int pool = 0, pk = 1, ps = 1, pp = 0, csrc = tsrc;
-  if (!gap && (tn.op == OP_MAXPOOL || tn.op == OP_AVGPOOL) && s.members.size() > 2) {
-    pool = tn.op == OP_MAXPOOL ? 1 : 2;
-    pk = tn.kh; ps = tn.sh; pp = tn.ph;
-    csrc = ir.oin[tsrc][0];
-  }
-  const Node& cn = ir.nodes[csrc];
-  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, cn.H, cn.W};
+  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
   P.members.erase(s.out);
-  if (pool) P.members.erase(tsrc);
   std::vector<PLevel> levels;
-  if (!P.chain(csrc, levels)) return false;
+  if (!P.chain(tsrc, levels)) return false;
   if (P.visited != P.members) return false;          // every member must be part of the chain form
+  // pooled members / tap-accumulate terms: single level, member in the leading channels
+  bool taps_any = false;
+  for (auto& L : levels)
+    for (auto& t : L.terms) taps_any |= t.tk > 1;
+  const PMember* pm = nullptr;
+  for (auto& L : levels) {
+    if (L.pm.size() > 1) return false;
+    if (!L.pm.empty()) pm = &L.pm[0];
+  }
+  const bool mixed = pm || taps_any;
+  if (mixed && levels.size() != 1) return false;
+  if (pm && (pm->c0 != 0 || pm->C % 64)) return false;
+  if (pm && gap) return false;                       // GAP over a max-pooled member: generic path
   int nterms = 0;
   for (auto& L : levels) nterms += (int)L.terms.size();
+  if (pm) nterms += (int)pm->terms.size();
   if ((int)levels.size() > kTcMaxLevels || nterms > kTcMaxTerms) return false;
+  auto term_ok = [&](const PTerm& t) {
+    const int r = ir.oin[t.lconv][0];
+    const Loc& l = loc.at(r);
+    return l.where == W_ARENA && l.dtype == DT_BF16 && ir.nodes[r].C % 8 == 0;
+  };
   for (auto& L : levels)
-    for (auto& t : L.terms) {
-      const int r = ir.oin[t.lconv][0];
-      const Loc& l = loc.at(r);
-      if (l.where != W_ARENA || l.dtype != DT_BF16 || ir.nodes[r].C % 8) return false;
-    }
+    for (auto& t : L.terms)
+      if (!term_ok(t)) return false;
+  if (pm)
+    for (auto& t : pm->terms)
+      if (!term_ok(t)) return false;
   const Loc& yl = loc.at(s.out);
   if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
 
   d = TcChainDesc();
   d.C = C;
-  d.Cc = (C <= 64 || pool) ? 64 : 128;
-  d.gather = 0;
-  d.pool = pool; d.pk = pk; d.ps = ps; d.pp = pp; d.taps = pk * pk;
-  d.Hin = cn.H; d.Win = cn.W; d.Ho = tn.H; d.Wo = tn.W;
+  d.Cc = (C <= 64 || mixed) ? 64 : 128;
   d.Cpad = (C + d.Cc - 1) / d.Cc * d.Cc;
   d.nchunks = d.Cpad / d.Cc;
   d.Nout = Nout;
@@ -113,13 +132,11 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d.nimg = ir.batch;
   d.gap = gap ? 1 : 0;
   d.hw = tn.H * tn.W;
-  if (gap) {
-    d.ipt = 128 / d.hw;
-    d.rows_per_tile = d.ipt * d.hw;
-    d.ntiles = (ir.batch + d.ipt - 1) / d.ipt;
-  } else if (pool) {
-    d.ipt = 0;
-    d.rows_per_tile = 128;
+  d.Ho = tn.H;
+  d.Wo = tn.W;
+  d.spatial = mixed ? 1 : 0;
+  d.post = -1;
+  if (d.spatial) {
     d.tw = std::min(tn.W, 128);
     d.th = std::min(tn.H, 128 / d.tw);
     d.tn = (d.th == tn.H && d.tw == tn.W) ? std::max(1, std::min(ir.batch, 128 / (tn.H * tn.W))) : 1;
@@ -128,65 +145,118 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.nnb = (ir.batch + d.tn - 1) / d.tn;
     d.mused = d.tw * d.th * d.tn;
     d.ntiles = d.nnb * d.nhb * d.nwb;
-    if (d.tw * ps > 256 || d.th * ps > 256) return false;
+    d.rows_per_tile = 128;
+    if (gap) {
+      if (d.th != tn.H || d.tw != tn.W) return false;    // GAP needs whole images per tile
+      d.ipt = d.tn;
+    }
+  } else if (gap) {
+    d.ipt = 128 / d.hw;
+    d.rows_per_tile = d.ipt * d.hw;
+    d.ntiles = (ir.batch + d.ipt - 1) / d.ipt;
   } else {
-    d.ipt = 0;
     d.rows_per_tile = 128;
     d.ntiles = (int)((d.npix + 127) / 128);
   }
   d.y = yl;
   d.n_levels = (int)levels.size();
-  int64_t flops_terms = 0, bytes_terms = 0;
+  int64_t flops = 0, bytes = 0;
   int j = 0;
+  auto add_term = [&](const PTerm& t) -> bool {
+    const Node& lc = ir.nodes[t.lconv];
+    const int r = ir.oin[t.lconv][0];
+    const Node& rn = ir.nodes[r];
+    const int R = rn.C;
+    TcTerm& T = d.term[j++];
+    T.r = loc.at(r);
+    T.R = R;
+    T.Rp = (R + 63) / 64 * 64;
+    T.Rw = (R + 7) / 8 * 8;
+    T.c0 = t.c0;
+    T.C = lc.C;
+    T.Hin = rn.H;
+    T.Win = rn.W;
+    T.tk = t.tk;
+    T.ts = t.ts;
+    T.tp = t.tp;
+    std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);
+    for (int c = 0; c < lc.C; ++c)
+      for (int k = 0; k < R; ++k)
+        w[(size_t)(t.c0 + c) * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
+    T.w = push_bf16(tcw, w);
+    const int64_t in_pix = (int64_t)ir.batch * rn.H * rn.W;
+    flops += in_pix * 2LL * lc.C * R;
+    bytes += in_pix * 2LL * R;
+    if (d.spatial && (d.tw * T.ts > 256 || d.th * T.ts > 256)) return false;
+    return true;
+  };
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
     d.relu[l] = L.relu ? 1 : 0;
-    d.bias[l] = -1;
-    // bias as a rank-2 term: columns 0, 1 = bf16 hi / lo parts (error ~2^-16 |b|)
-    std::vector<float> bm((size_t)d.Cpad * 8, 0.f);
-    for (int c = 0; c < C; ++c) {
-      const float b = (float)L.bias[c];
-      const float hi = from_bf16(to_bf16(b));
-      bm[(size_t)c * 8 + 0] = hi;
-      bm[(size_t)c * 8 + 1] = b - hi;
+    // pooled-member channels take no level bias through the MMA: their level bias
+    // (the post-BN shift) is added after pooling, in the epilogue
+    std::vector<double> lb = L.bias;
+    if (pm && l == 0) {
+      std::vector<double> post(d.Cc * (pm->C / d.Cc), 0.0);
+      for (int c = 0; c < pm->C; ++c) {
+        post[c] = lb[c];
+        lb[c] = 0.0;
+      }
+      while (params.size() % 4) params.push_back(0.f);
+      d.post = (int64_t)params.size();
+      for (double x : post) params.push_back((float)x);
     }
-    d.boff[l] = push_bf16(tcw, bm);
-    for (const PTerm& t : L.terms) {
-      const Node& lc = ir.nodes[t.lconv];
-      const int r = ir.oin[t.lconv][0];
-      const int R = ir.nodes[r].C;
-      TcTerm& T = d.term[j++];
-      T.r = loc.at(r);
-      T.R = R;
-      T.Rp = (R + 63) / 64 * 64;
-      T.Rw = (R + 7) / 8 * 8;
-      T.c0 = t.c0;
-      T.C = lc.C;
-      std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);
-      for (int c = 0; c < lc.C; ++c)
-        for (int k = 0; k < R; ++k)
-          w[(size_t)(t.c0 + c) * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
-      T.w = push_bf16(tcw, w);
-      flops_terms += 2LL * lc.C * R;
-      bytes_terms += 2LL * R;
-    }
+    d.boff[l] = push_bias(tcw, lb, 0, d.Cpad);
+    for (const PTerm& t : L.terms)
+      if (!add_term(t)) return false;
     d.lvl_end[l] = j;
   }
   d.n_terms = j;
+  if (pm) {
+    d.npc = pm->C / d.Cc;
+    d.mpool = pm->kind;
+    d.mk = pm->k;
+    d.ms = pm->s;
+    d.mp = pm->p;
+    d.mtaps = pm->k * pm->k;
+    d.mrelu = pm->relu ? 1 : 0;
+    d.mHin = pm->Hin;
+    d.mWin = pm->Win;
+    d.mt0 = j;
+    for (const PTerm& t : pm->terms) {
+      PTerm u = t;
+      u.tk = 1;
+      u.ts = pm->s;
+      if (!add_term(u)) return false;
+    }
+    d.mt1 = j;
+    // the member is evaluated once per tap: count its work at the taps actually run
+    d.boffm = push_bias(tcw, pm->bias, 0, d.Cpad);
+    if (d.tw * d.ms > 256 || d.th * d.ms > 256) return false;
+  }
+  d.F = 0;
   d.Fb = -1;
   if (gap) {
-    d.F = 0;
-    d.alg_flops = d.npix * (flops_terms + C);
-    d.alg_bytes = d.npix * bytes_terms + 2LL * ir.batch * C;
+    d.alg_flops = flops + d.npix * C;
+    d.alg_bytes = bytes + 2LL * ir.batch * C;
   } else {
     std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
     for (int o = 0; o < Nout; ++o)
       for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
     d.F = push_bf16(tcw, f);
-    const int64_t nin = (int64_t)ir.batch * cn.H * cn.W;   // chain evaluated once per input pixel
-    d.alg_flops = nin * flops_terms + d.npix * 2LL * Nout * C;
-    d.alg_bytes = nin * bytes_terms + d.npix * 2LL * Nout;
+    d.alg_flops = flops + d.npix * 2LL * Nout * C;
+    d.alg_bytes = bytes + d.npix * 2LL * Nout;
   }
+  // pooled member: as many taps per unit as two unit buffers + the output allow
+  d.tpu = 1;
+  d.ntg = 1;
+  if (pm) {
+    int t = d.mtaps;
+    while (t > 1 && 2 * t * d.Cc + d.Np > 512) --t;
+    d.ntg = (d.mtaps + t - 1) / t;
+    d.tpu = (d.mtaps + d.ntg - 1) / d.ntg;
+  }
+  d.ubuf = d.tpu * d.Cc;
   // shared memory: ring of (A 16 KB | B slot) stages + two P tiles + ones tile + barriers
   d.slot_b = std::max(d.Cc, d.Np) * 128;
   const int pbytes = 128 * d.Cc * 2;
@@ -194,9 +264,9 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d.stages = std::min(6, budget / (16384 + d.slot_b));
   if (d.stages < 2) return false;
   d.smem_bytes = 1024 + d.stages * (16384 + d.slot_b) + 2 * pbytes + 16384 + 1024;
-  const int cols = 2 * d.Cc + d.Np;
+  const int cols = 2 * d.ubuf + d.Np;
   d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
-  return true;
+  return cols <= 512;
 }
 
 bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char* arena, uint16_t* tcw,
@@ -224,11 +294,11 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
   };
-  auto make4 = [&](unsigned char* dst, void* base, const TcChainDesc* d, int R) {
-    cuuint64_t dims[4] = {(cuuint64_t)R, (cuuint64_t)d->Win, (cuuint64_t)d->Hin, (cuuint64_t)d->nimg};
-    cuuint64_t strides[3] = {(cuuint64_t)R * 2, (cuuint64_t)d->Win * R * 2, (cuuint64_t)d->Hin * d->Win * R * 2};
-    cuuint32_t box[4] = {64, (cuuint32_t)(d->tw * d->ps), (cuuint32_t)(d->th * d->ps), (cuuint32_t)d->tn};
-    cuuint32_t es[4] = {1, (cuuint32_t)d->ps, (cuuint32_t)d->ps, 1};
+  auto make4 = [&](unsigned char* dst, void* base, const TcChainDesc* d, const TcTerm& t) {
+    cuuint64_t dims[4] = {(cuuint64_t)t.R, (cuuint64_t)t.Win, (cuuint64_t)t.Hin, (cuuint64_t)d->nimg};
+    cuuint64_t strides[3] = {(cuuint64_t)t.R * 2, (cuuint64_t)t.Win * t.R * 2, (cuuint64_t)t.Hin * t.Win * t.R * 2};
+    cuuint32_t box[4] = {64, (cuuint32_t)(d->tw * t.ts), (cuuint32_t)(d->th * t.ts), (cuuint32_t)d->tn};
+    cuuint32_t es[4] = {1, (cuuint32_t)t.ts, (cuuint32_t)t.ts, 1};
     CUresult r = encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides,
                         box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
@@ -237,14 +307,15 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
   for (size_t i = 0; i < n; ++i) {
     TcChainDesc* d = get(i);
     if (!d) continue;
-    for (int j = 0; j < d->n_terms; ++j) {
+    const int nt = d->npc ? d->mt1 : d->n_terms;
+    for (int j = 0; j < nt; ++j) {
       TcTerm& t = d->term[j];
-      if (d->pool && !make4(t.tmap4, arena + t.r.off, d, t.R)) {
-        err = "cuTensorMapEncodeTiled failed (pooled term)";
-        return false;
-      }
-      if (!make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->nimg * d->Hin * d->Win, 128) ||
-          !make(t.wmap, tcw + t.w, (uint64_t)t.Rw, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+      bool ok = make(t.wmap, tcw + t.w, (uint64_t)t.Rw, (uint64_t)d->Cpad, (uint32_t)d->Cc);
+      if (d->spatial)
+        ok = ok && make4(t.tmap4, arena + t.r.off, d, t);
+      else
+        ok = ok && make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->nimg * t.Hin * t.Win, 128);
+      if (!ok) {
         err = "cuTensorMapEncodeTiled failed (term)";
         return false;
       }
@@ -254,6 +325,10 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
         err = "cuTensorMapEncodeTiled failed (bias)";
         return false;
       }
+    if (d->npc && !make(d->bmapm, tcw + d->boffm, 8, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+      err = "cuTensorMapEncodeTiled failed (member bias)";
+      return false;
+    }
     if (!d->gap && !make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
       err = "cuTensorMapEncodeTiled failed (F)";
       return false;
@@ -273,39 +348,52 @@ __device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
 }
 
 constexpr int kEpiWarps = 8;
-constexpr int kProdWarp = 8, kMmaWarp = 9, kGatherWarp0 = 10;
-constexpr int kThreads = 32 * 14;
+constexpr int kProdWarp = 8, kMmaWarp = 9;
+constexpr int kThreads = 32 * 10;
 constexpr int kSlotA = 16384;
 
-// The MMA work of one tile is a sequence of "units": chunk c of the restored
-// width (and, for a pooled chain, tap tau of the pooling window).  Units are
-// processed in pairs (two TMEM accumulators) -- consecutive chunks, or
-// consecutive taps of one chunk -- and every role walks the same order:
-//   for pair: for level l: for unit in pair: [bias stage, term stages] + epilogue
-//             then G2 for every chunk whose restored values are final.
-struct PairIter {
-  int c0, t0, nb;
+// Units of one tile: pooled chunks c < npc contribute ntg tap-group units each,
+// every other chunk one unit.  Units are processed in pairs (TMEM buffers 0, 1);
+// all roles walk the same order: for pair: for level: for unit in pair.
+struct Unit {
+  int c, tg, nt;      // chunk, tap group, taps in the unit (1 for plain chunks)
+  bool pooled, last;  // pooled-member chunk; last unit of its chunk
 };
 
-__device__ __forceinline__ void unit_of(const TcChainDesc& d, const PairIter& it, int bi, int& c, int& tap) {
-  if (d.pool) {
-    c = it.c0;
-    tap = it.t0 + bi;
+__device__ __forceinline__ int units_per_tile(const TcChainDesc& d) { return d.npc * d.ntg + d.nchunks - d.npc; }
+
+__device__ __forceinline__ Unit unit_at(const TcChainDesc& d, int u) {
+  Unit x;
+  if (u < d.npc * d.ntg) {
+    x.c = u / d.ntg;
+    x.tg = u % d.ntg;
+    x.nt = min(d.tpu, d.mtaps - x.tg * d.tpu);
+    x.pooled = true;
+    x.last = x.tg == d.ntg - 1;
   } else {
-    c = it.c0 + bi;
-    tap = 0;
+    x.c = d.npc + (u - d.npc * d.ntg);
+    x.tg = 0;
+    x.nt = 1;
+    x.pooled = false;
+    x.last = true;
   }
+  return x;
 }
 
-#define FOR_PAIRS(d, it)                                                                            \
-  for (PairIter it{0, 0, 0}; it.c0 < (d).nchunks;                                                   \
-       (d).pool ? ((it.t0 += 2) >= (d).taps ? (it.t0 = 0, ++it.c0) : 0) : (it.c0 += 2))             \
-    if ((it.nb = (d).pool ? min(2, (d).taps - it.t0) : min(2, (d).nchunks - it.c0)), true)
+struct TileGeo {
+  int m0, n0, h0, w0;
+};
 
-__device__ __forceinline__ int g2_count(const TcChainDesc& d, const PairIter& it) {
-  if (d.gap) return 0;
-  if (d.pool) return it.t0 + it.nb == d.taps ? 1 : 0;
-  return it.nb;
+__device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
+  TileGeo g{tile * d.rows_per_tile, 0, 0, 0};
+  if (d.spatial) {
+    const int per_img = d.nhb * d.nwb;
+    const int nb = tile / per_img, rem = tile % per_img;
+    g.n0 = nb * d.tn;
+    g.h0 = (rem / d.nwb) * d.th;
+    g.w0 = (rem % d.nwb) * d.tw;
+  }
+  return g;
 }
 
 __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
@@ -340,7 +428,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   fence_proxy_async();
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], d.gather ? 33 : 1);
+      mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -362,6 +450,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+  const int U = units_per_tile(d);
 
   if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer
@@ -369,127 +458,57 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       int stage = 0;
       uint32_t phase = 0;
       const uint32_t bytes_b = Cc * 128, bytes_f = d.Np * 128;
-      const uint32_t bytes_a = d.gather ? 0 : d.pool ? 128u * d.tw * d.th * d.tn : (uint32_t)kSlotA;
-      const int per_img = d.nhb * d.nwb;
-      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        const int m0 = tile * d.rows_per_tile;
-        int n0 = 0, h0 = 0, w0 = 0;
-        if (d.pool) {
-          const int nb = tile / per_img, rem = tile % per_img;
-          n0 = nb * d.tn;
-          h0 = (rem / d.nwb) * d.th;
-          w0 = (rem % d.nwb) * d.tw;
-        }
-        FOR_PAIRS(d, it) {
-          for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < it.nb; ++bi) {
-              int c, tap;
-              unit_of(d, it, bi, c, tap);
-              mbar_wait(&empty[stage], phase ^ 1);                 // bias stage
-              mbar_expect_tx(&full[stage], bytes_b);
-              tma_load_2d(ring + stage * slot + kSlotA, d.bmap[l], &full[stage], 0, c * Cc);
-              if (++stage == S) stage = 0, phase ^= 1;
-              for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
-                const TcTerm& t = d.term[j];
-                if (!term_hits(t, c, Cc)) continue;
-                for (int ka = 0; ka < t.Rp / 64; ++ka) {
-                  mbar_wait(&empty[stage], phase ^ 1);
-                  mbar_expect_tx(&full[stage], bytes_a + bytes_b);
-                  uint8_t* sa = ring + stage * slot;
-                  if (d.pool)       // tap-shifted strided box of the chain-resolution input
-                    tma_load_4d(sa, t.tmap4, &full[stage], ka * 64, w0 * d.ps - d.pp + tap % d.pk,
-                                h0 * d.ps - d.pp + tap / d.pk, n0);
-                  else if (!d.gather)
-                    tma_load_2d(sa, t.tmap, &full[stage], ka * 64, m0);
-                  tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * 64, c * Cc);
-                  if (++stage == S) stage = 0, phase ^= 1;
-                }
-              }
-            }
-          for (int q = 0; q < g2_count(d, it); ++q) {
-            const int c = it.c0 + (d.pool ? 0 : q);
-            for (int a = 0; a < Cc / 64; ++a) {
-              mbar_wait(&empty[stage], phase ^ 1);
-              mbar_expect_tx(&full[stage], bytes_f);
-              tma_load_2d(ring + stage * slot + kSlotA, d.fmap, &full[stage], c * Cc + a * 64, 0);
-              if (++stage == S) stage = 0, phase ^= 1;
-            }
-          }
-        }
-      }
-    }
-  } else if (warp >= kGatherWarp0) {
-    // ------------------------------------------------------------ gather producer (A rows)
-    // warp-per-stage: gather warp gw fills every 4th stage of the ring (lane
-    // owns rows lane + 32 i), so 4 stages of cp.async are in flight at once
-    if (d.gather) {
-      const int gw = warp - kGatherWarp0;
-      int64_t kseq = 0;
-      auto next = [&](int& stage, uint32_t& phase) {
-        stage = (int)(kseq % S);
-        phase = (uint32_t)((kseq / S) & 1);
-        return (int)((kseq++) & 3) == gw;
+      const uint32_t bytes_a = d.spatial ? 128u * d.tw * d.th * d.tn : (uint32_t)kSlotA;
+      auto load_b = [&](const void* map, int x, int y) {
+        mbar_wait(&empty[stage], phase ^ 1);
+        mbar_expect_tx(&full[stage], bytes_b);
+        tma_load_2d(ring + stage * slot + kSlotA, map, &full[stage], x, y);
+        if (++stage == S) stage = 0, phase ^= 1;
       };
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        int ho[4], wo[4], nn[4];
-        bool mv[4];
-        const int hw = d.Ho * d.Wo;
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int64_t m = (int64_t)tile * d.rows_per_tile + lane + 32 * i;
-          mv[i] = m < d.npix;
-          nn[i] = mv[i] ? (int)(m / hw) : 0;
-          const int rem = mv[i] ? (int)(m % hw) : 0;
-          ho[i] = rem / d.Wo;
-          wo[i] = rem % d.Wo;
-        }
-        FOR_PAIRS(d, it) {
+        const TileGeo gg = tile_geo(d, tile);
+        for (int u0 = 0; u0 < U; u0 += 2) {
+          const int nb = min(2, U - u0);
           for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < it.nb; ++bi) {
-              int c, tap;
-              unit_of(d, it, bi, c, tap);
-              {
-                int stage;
-                uint32_t phase;
-                if (next(stage, phase)) {                          // bias stage: no A rows
-                  mbar_wait(&empty[stage], phase ^ 1);
-                  cp_async_arrive(&full[stage]);
-                }
-              }
-              for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
-                const TcTerm& t = d.term[j];
-                if (!term_hits(t, c, Cc)) continue;
-                const uint8_t* rbase = reinterpret_cast<const uint8_t*>(p.arena + t.r.off);
-                for (int ka = 0; ka < t.Rp / 64; ++ka) {
-                  int stage;
-                  uint32_t phase;
-                  if (!next(stage, phase)) continue;
-                  mbar_wait(&empty[stage], phase ^ 1);
-#pragma unroll
-                  for (int i = 0; i < 4; ++i) {
-                    const int row = lane + 32 * i;
-                    const int hi = ho[i] * d.ps - d.pp + tap / d.pk, wi = wo[i] * d.ps - d.pp + tap % d.pk;
-                    const bool valid = mv[i] && hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
-                    const int64_t pix = ((int64_t)nn[i] * d.Hin + hi) * d.Win + wi;
-                    uint8_t* dst = ring + stage * slot + row * 128;
-#pragma unroll
-                    for (int q = 0; q < 8; ++q) {
-                      const int k0 = ka * 64 + q * 8;
-                      const bool ok = valid && k0 < t.R;
-                      cp_async16(dst + ((q ^ (row & 7)) * 16), ok ? rbase + (pix * t.R + k0) * 2 : rbase, ok ? 16u : 0u);
+            for (int bi = 0; bi < nb; ++bi) {
+              const Unit un = unit_at(d, u0 + bi);
+              load_b(un.pooled ? d.bmapm : d.bmap[l], 0, un.c * Cc);             // bias stage
+              const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
+              const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
+              for (int r = 0; r < un.nt; ++r)
+                for (int j = j0; j < j1; ++j) {
+                  const TcTerm& t = d.term[j];
+                  if (!un.pooled && !term_hits(t, un.c, Cc)) continue;
+                  const int ntap = un.pooled ? 1 : t.tk * t.tk;
+                  for (int q = 0; q < ntap; ++q) {
+                    const int tap = un.pooled ? un.tg * d.tpu + r : q;
+                    const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
+                    for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                      mbar_wait(&empty[stage], phase ^ 1);
+                      mbar_expect_tx(&full[stage], bytes_a + bytes_b);
+                      uint8_t* sa = ring + stage * slot;
+                      if (d.spatial)      // (tap-shifted) strided box of the term's input
+                        tma_load_4d(sa, t.tmap4, &full[stage], ka * 64, gg.w0 * t.ts - pad + tap % kk,
+                                    gg.h0 * t.ts - pad + tap / kk, gg.n0);
+                      else
+                        tma_load_2d(sa, t.tmap, &full[stage], ka * 64, gg.m0);
+                      tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * 64, un.c * Cc);
+                      if (++stage == S) stage = 0, phase ^= 1;
                     }
                   }
-                  cp_async_arrive(&full[stage]);
                 }
+            }
+          if (!d.gap)
+            for (int bi = 0; bi < nb; ++bi) {
+              const Unit un = unit_at(d, u0 + bi);
+              if (!un.last) continue;
+              for (int a = 0; a < Cc / 64; ++a) {
+                mbar_wait(&empty[stage], phase ^ 1);
+                mbar_expect_tx(&full[stage], bytes_f);
+                tma_load_2d(ring + stage * slot + kSlotA, d.fmap, &full[stage], un.c * Cc + a * 64, 0);
+                if (++stage == S) stage = 0, phase ^= 1;
               }
             }
-          for (int q = 0; q < g2_count(d, it) * (Cc / 64); ++q) {
-            int stage;
-            uint32_t phase;
-            if (!next(stage, phase)) continue;
-            mbar_wait(&empty[stage], phase ^ 1);
-            cp_async_arrive(&full[stage]);
-          }
         }
       }
     }
@@ -500,73 +519,80 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       uint32_t phase = 0;
       uint32_t acc_use0 = 0, acc_use1 = 0, p_use0 = 0, p_use1 = 0, tile_iter = 0;
       const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
-      const uint32_t tout = tbase + 2 * Cc;
+      const uint32_t tout = tbase + 2 * d.ubuf;
       const uint32_t ones_addr = smem_u32(ones);
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        FOR_PAIRS(d, it) {
+        for (int u0 = 0; u0 < U; u0 += 2) {
+          const int nb = min(2, U - u0);
           for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < it.nb; ++bi) {
-              int c, tap;
-              unit_of(d, it, bi, c, tap);
+            for (int bi = 0; bi < nb; ++bi) {
+              const Unit un = unit_at(d, u0 + bi);
               uint32_t& use = bi ? acc_use1 : acc_use0;
               mbar_wait(&acc_empty[bi], (use & 1) ^ 1);
               tc_fence_after();
-              const uint32_t tacc = tbase + bi * Cc;
-              // bias (initialises the accumulator at level 0)
+              const uint32_t tacc = tbase + bi * d.ubuf;
+              // bias (initialises every tap region of the accumulator at level 0)
               mbar_wait(&full[stage], phase);
               tc_fence_after();
-              mma_bf16(tacc, umma_desc(ones_addr), umma_desc(smem_u32(ring + stage * slot + kSlotA)), id1,
-                       l == 0 ? 0u : 1u);
+              for (int r = 0; r < un.nt; ++r)
+                mma_bf16(tacc + r * Cc, umma_desc(ones_addr), umma_desc(smem_u32(ring + stage * slot + kSlotA)), id1,
+                         l == 0 ? 0u : 1u);
               mma_commit(&empty[stage]);
               if (++stage == S) stage = 0, phase ^= 1;
-              for (int j = l ? d.lvl_end[l - 1] : 0; j < d.lvl_end[l]; ++j) {
-                const TcTerm& t = d.term[j];
-                if (!term_hits(t, c, Cc)) continue;
-                for (int ka = 0; ka < t.Rp / 64; ++ka) {
-                  mbar_wait(&full[stage], phase);
-                  if (d.gather) fence_proxy_async();
-                  tc_fence_after();
-                  const uint32_t sa = smem_u32(ring + stage * slot);
-                  const int nk = min(4, (t.R - ka * 64 + 15) / 16);
-                  for (int k = 0; k < nk; ++k)
-                    mma_bf16(tacc, umma_desc(sa + 32 * k), umma_desc(sa + kSlotA + 32 * k), id1, 1u);
-                  mma_commit(&empty[stage]);
-                  if (++stage == S) stage = 0, phase ^= 1;
+              const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
+              const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
+              for (int r = 0; r < un.nt; ++r)
+                for (int j = j0; j < j1; ++j) {
+                  const TcTerm& t = d.term[j];
+                  if (!un.pooled && !term_hits(t, un.c, Cc)) continue;
+                  const int ntap = un.pooled ? 1 : t.tk * t.tk;
+                  for (int q = 0; q < ntap; ++q)
+                    for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                      mbar_wait(&full[stage], phase);
+                      tc_fence_after();
+                      const uint32_t sa = smem_u32(ring + stage * slot);
+                      const int nk = min(4, (t.R - ka * 64 + 15) / 16);
+                      for (int k = 0; k < nk; ++k)
+                        mma_bf16(tacc + r * Cc, umma_desc(sa + 32 * k), umma_desc(sa + kSlotA + 32 * k), id1, 1u);
+                      mma_commit(&empty[stage]);
+                      if (++stage == S) stage = 0, phase ^= 1;
+                    }
                 }
-              }
               mma_commit(&acc_full[bi]);
               ++use;
             }
-          for (int q = 0; q < g2_count(d, it); ++q) {
-            const int c = it.c0 + (d.pool ? 0 : q);
-            const int pb = c & 1;
-            uint32_t& puse = pb ? p_use1 : p_use0;
-            mbar_wait(&p_full[pb], puse & 1);
-            tc_fence_after();
-            if (c == 0) {
-              mbar_wait(out_empty, (tile_iter & 1) ^ 1);
+          if (!d.gap)
+            for (int bi = 0; bi < nb; ++bi) {
+              const Unit un = unit_at(d, u0 + bi);
+              if (!un.last) continue;
+              const int pb = un.c & 1;
+              uint32_t& puse = pb ? p_use1 : p_use0;
+              mbar_wait(&p_full[pb], puse & 1);
               tc_fence_after();
+              if (un.c == 0) {
+                mbar_wait(out_empty, (tile_iter & 1) ^ 1);
+                tc_fence_after();
+              }
+              const uint32_t pa = smem_u32(pbuf + pb * pbytes);
+              for (int a = 0; a < Cc / 64; ++a) {
+                mbar_wait(&full[stage], phase);
+                tc_fence_after();
+                const uint32_t sb = smem_u32(ring + stage * slot + kSlotA);
+                for (int k = 0; k < 4; ++k)
+                  mma_bf16(tout, umma_desc(pa + a * 16384 + 32 * k), umma_desc(sb + 32 * k), id2,
+                           (un.c > 0 || a > 0 || k > 0) ? 1u : 0u);
+                mma_commit(&empty[stage]);
+                if (++stage == S) stage = 0, phase ^= 1;
+              }
+              mma_commit(&p_empty[pb]);
+              ++puse;
             }
-            const uint32_t pa = smem_u32(pbuf + pb * pbytes);
-            for (int a = 0; a < Cc / 64; ++a) {
-              mbar_wait(&full[stage], phase);
-              tc_fence_after();
-              const uint32_t sb = smem_u32(ring + stage * slot + kSlotA);
-              for (int k = 0; k < 4; ++k)
-                mma_bf16(tout, umma_desc(pa + a * 16384 + 32 * k), umma_desc(sb + 32 * k), id2,
-                         (c > 0 || a > 0 || k > 0) ? 1u : 0u);
-              mma_commit(&empty[stage]);
-              if (++stage == S) stage = 0, phase ^= 1;
-            }
-            mma_commit(&p_empty[pb]);
-            ++puse;
-          }
         }
         if (!d.gap) mma_commit(out_full);
         ++tile_iter;
       }
     }
-  } else {
+  } else if (warp < kEpiWarps) {
     // ------------------------------------------------------------ epilogue (8 warps)
     // warp w: TMEM lane quarter q = w % 4 (pixel rows 32q..32q+31), column half h = w / 4
     const int q = warp & 3, h = warp >> 2;
@@ -576,43 +602,85 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     const int c_lo = h * half;
     uint32_t acc_use0 = 0, acc_use1 = 0, p_use0 = 0, p_use1 = 0, tile_iter = 0;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
-    float run[32];                                    // pooled values (pool mode, Cc = 64 -> 32 per warp)
+    float run[32];                                    // pooled member (Cc = 64 -> 32 columns per warp)
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
       int64_t m = (int64_t)tile * d.rows_per_tile + row;
       bool mvalid = m < d.npix;
       int ho = 0, wo = 0;
-      if (d.pool) {
+      if (d.spatial) {
         // spatial tile: row -> (image, output row, output column)
-        const int per_img = d.nhb * d.nwb;
-        const int nb = tile / per_img, rem = tile % per_img;
+        const TileGeo gg = tile_geo(d, tile);
         const int ni = row / (d.tw * d.th), hi = (row / d.tw) % d.th, wi = row % d.tw;
-        const int n = nb * d.tn + ni;
-        ho = (rem / d.nwb) * d.th + hi;
-        wo = (rem % d.nwb) * d.tw + wi;
+        const int n = gg.n0 + ni;
+        ho = gg.h0 + hi;
+        wo = gg.w0 + wi;
         mvalid = row < d.mused && n < d.nimg && ho < d.Ho && wo < d.Wo;
         m = ((int64_t)n * d.Ho + ho) * d.Wo + wo;
       }
-      FOR_PAIRS(d, it) {
+      for (int u0 = 0; u0 < U; u0 += 2) {
+        const int nb = min(2, U - u0);
         for (int l = 0; l < d.n_levels; ++l) {
           const bool last = l == d.n_levels - 1;
           const bool relu = d.relu[l] != 0;
-          for (int bi = 0; bi < it.nb; ++bi) {
-            int c, tap;
-            unit_of(d, it, bi, c, tap);
+          for (int bi = 0; bi < nb; ++bi) {
+            const Unit un = unit_at(d, u0 + bi);
             uint32_t& use = bi ? acc_use1 : acc_use0;
             mbar_wait(&acc_full[bi], use & 1);
             ++use;
             tc_fence_after();
-            const int pb = c & 1;
-            const bool writes_p = last && !d.gap && (!d.pool || tap == d.taps - 1);
+            const int pb = un.c & 1;
+            const bool writes_p = last && !d.gap && un.last;
             if (writes_p) {
               uint32_t& puse = pb ? p_use1 : p_use0;
               mbar_wait(&p_empty[pb], (puse & 1) ^ 1);
               ++puse;
             }
-            const uint32_t ta = tbase + lane_off + bi * Cc + c_lo;
+            const uint32_t ta = tbase + lane_off + bi * d.ubuf + c_lo;
             uint8_t* P = pbuf + pb * pbytes;
-            if (!last) {
+            if (un.pooled) {
+              // pooled member: fold the unit's taps into the running max / sum (half == 32)
+              for (int r = 0; r < un.nt; ++r) {
+                const int tap = un.tg * d.tpu + r;
+                const int hi = ho * d.ms - d.mp + tap / d.mk, wi = wo * d.ms - d.mp + tap % d.mk;
+                const bool valid = hi >= 0 && hi < d.mHin && wi >= 0 && wi < d.mWin;
+                uint32_t v[32];
+                tmem_ld32(ta + r * Cc, v);
+                tmem_wait_ld();
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                  float x = __uint_as_float(v[i]);
+                  x = d.mrelu ? fmaxf(x, 0.f) : x;
+                  if (d.mpool == 1)
+                    run[i] = tap == 0 ? (valid ? x : -INFINITY) : (valid ? fmaxf(run[i], x) : run[i]);
+                  else
+                    run[i] = tap == 0 ? x : run[i] + x;
+                }
+              }
+              if (un.last) {
+                // pooled value, + post-pool shift (BN after the pool), level activation
+                const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
+                const float* post = d.post >= 0 ? p.params + d.post + un.c * Cc + c_lo : nullptr;
+#pragma unroll
+                for (int i = 0; i < 32; ++i) {
+                  float x = run[i] * sc + (post ? __ldg(post + i) : 0.f);
+                  run[i] = relu ? fmaxf(x, 0.f) : x;
+                }
+                if (d.gap) {
+                  // not reached: GAP with a pooled member is not lowered here
+                } else {
+                  const int ch0 = c_lo / 8;
+#pragma unroll
+                  for (int qq = 0; qq < 4; ++qq) {
+                    uint4 pk;
+                    pk.x = pack_bf16(run[8 * qq + 0], run[8 * qq + 1]);
+                    pk.y = pack_bf16(run[8 * qq + 2], run[8 * qq + 3]);
+                    pk.z = pack_bf16(run[8 * qq + 4], run[8 * qq + 5]);
+                    pk.w = pack_bf16(run[8 * qq + 6], run[8 * qq + 7]);
+                    *reinterpret_cast<uint4*>(P + row * 128 + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
+                  }
+                }
+              }
+            } else if (!last) {
               // t_l = relu(acc) back into TMEM for the next level's MMAs
               uint32_t v[2][32];
               tmem_ld32(ta, v[0]);
@@ -628,35 +696,6 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               tmem_st32(ta, v[0]);
               if (half == 64) tmem_st32(ta + 32, v[1]);
               tmem_wait_st();
-            } else if (d.pool) {
-              // pooled chain: fold this tap into the running max / sum (half == 32)
-              const int hi = ho * d.ps - d.pp + tap / d.pk, wi = wo * d.ps - d.pp + tap % d.pk;
-              const bool valid = hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
-              uint32_t v[32];
-              tmem_ld32(ta, v);
-              tmem_wait_ld();
-#pragma unroll
-              for (int i = 0; i < 32; ++i) {
-                float x = __uint_as_float(v[i]);
-                x = relu ? fmaxf(x, 0.f) : x;
-                if (d.pool == 1)
-                  run[i] = tap == 0 ? (valid ? x : -INFINITY) : (valid ? fmaxf(run[i], x) : run[i]);
-                else
-                  run[i] = tap == 0 ? x : run[i] + x;
-              }
-              if (writes_p) {
-                const float sc = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
-                const int ch0 = c_lo / 8;
-#pragma unroll
-                for (int qq = 0; qq < 4; ++qq) {
-                  uint4 pk;
-                  pk.x = pack_bf16(run[8 * qq + 0] * sc, run[8 * qq + 1] * sc);
-                  pk.y = pack_bf16(run[8 * qq + 2] * sc, run[8 * qq + 3] * sc);
-                  pk.z = pack_bf16(run[8 * qq + 4] * sc, run[8 * qq + 5] * sc);
-                  pk.w = pack_bf16(run[8 * qq + 6] * sc, run[8 * qq + 7] * sc);
-                  *reinterpret_cast<uint4*>(P + row * 128 + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
-                }
-              }
             } else if (d.gap) {
               // GAP root: per-image column means; tiles hold whole images so the
               // summation order is fixed (deterministic, batch-invariant)
@@ -676,7 +715,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   const int n = tile * d.ipt + ii;
                   float acc = 0.f;
                   for (int r = ii * d.hw; r < (ii + 1) * d.hw; ++r) acc += red[r * 32 + ((col + r) & 31)];
-                  const int cg = c * Cc + c_lo + g * 32 + col;
+                  const int cg = un.c * Cc + c_lo + g * 32 + col;
                   if (n < d.nimg && cg < d.C) y[(int64_t)n * d.C + cg] = __float2bfloat16_rn(acc / (float)d.hw);
                 }
                 asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
@@ -724,7 +763,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       const int ng = d.Np / 8, gh = (ng + 1) / 2;
       for (int g = h * gh; g < min(ng, (h + 1) * gh); ++g) {
         uint32_t v[8];
-        tmem_ld8(tbase + lane_off + 2 * Cc + g * 8, v);
+        tmem_ld8(tbase + lane_off + 2 * d.ubuf + g * 8, v);
         tmem_wait_ld();
         if (mvalid && g * 8 < d.Nout) {
           uint4 pk;
