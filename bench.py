@@ -128,7 +128,7 @@ def cpu_baseline(config):
     from threadpoolctl import threadpool_info
     m = W.build_config(config)
     pl = oracle.plan(m)
-    sample = {"resnet18_cifar": 64, "resnet50": 8, "vgg16_cp": 8, "densenet121": 8}[config]
+    sample = {"resnet18_cifar": 256, "resnet50": 24, "vgg16_cp": 24, "densenet121": 24}[config]
     x = W.make_input(m, start=0, count=sample)
     oracle.run_temco(pl, x[:1])                 # warm-up
     t0 = time.perf_counter()
@@ -156,6 +156,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_icpp_songljkj0024_b200 import FLAG_CUDA_GRAPH, FLAG_SIMT_ONLY, Plan
+    from paper_conf_icpp_songljkj0024_b200.shard import gather_logits, shard_range
 
     ws, rank, local = _dist()
     torch.cuda.set_device(local)
@@ -167,7 +168,8 @@ def main():
     plan = Plan(m, flags=flags)
     desc = plan.describe()
     out_shape = plan.output_shape()
-    x_host = W.make_input(m, start=rank * B, count=B)
+    start, stop = shard_range(rank, ws, B)
+    x_host = W.make_input(m, start=start, count=stop - start)
     tdt = torch.bfloat16 if m.dtype == "bf16" else torch.float32
     x = torch.from_numpy(x_host).to(tdt).cuda()
     y = torch.empty(out_shape, dtype=torch.float32, device="cuda")
@@ -178,7 +180,7 @@ def main():
     def step():
         plan.run(x, y, stream)
         if ws > 1:
-            dist.all_gather_into_tensor(gathered, y)
+            gather_logits(y, ws, gathered)
 
     with torch.cuda.stream(stream):
         for _ in range(args.warmup):

@@ -170,7 +170,8 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     TcTerm& T = d.term[j++];
     T.r = loc.at(r);
     T.R = R;
-    T.Rp = (R + 63) / 64 * 64;
+    T.aw = R <= 16 ? 16 : R <= 32 ? 32 : 64;      // box width ~ rank: no mostly-OOB boxes
+    T.Rp = (R + T.aw - 1) / T.aw * T.aw;
     T.Rw = (R + 7) / 8 * 8;
     T.c0 = t.c0;
     T.C = lc.C;
@@ -257,13 +258,21 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.tpu = (d.mtaps + d.ntg - 1) / d.ntg;
   }
   d.ubuf = d.tpu * d.Cc;
-  // shared memory: ring of (A 16 KB | B slot) stages + two P tiles + ones tile + barriers
-  d.slot_b = std::max(d.Cc, d.Np) * 128;
+  // shared memory: ring of (A | B) stages sized by the widest K atom of the group
+  // (small ranks -> small stages -> a deep ring), two P tiles, ones tile, barriers
+  int awmax = 16;
+  const int nall = pm ? d.mt1 : d.n_terms;
+  for (int i = 0; i < nall; ++i) awmax = std::max(awmax, d.term[i].aw);
+  d.slot_a = 128 * awmax * 2;
+  int sb = std::max(d.Cc * awmax * 2, d.Cc * 32);
+  if (!gap) sb = std::max(sb, d.Np * 128);
+  d.slot_b = (sb + 1023) / 1024 * 1024;
   const int pbytes = 128 * d.Cc * 2;
-  const int budget = 227 * 1024 - 1024 /*align*/ - 1024 /*barriers*/ - 2 * pbytes - 16384 /*ones*/;
-  d.stages = std::min(6, budget / (16384 + d.slot_b));
+  const int runbytes = pm ? 32768 : 0;     // pooled member: running max / sum slab (after the barriers)
+  const int budget = 227 * 1024 - 1024 /*align*/ - 2048 /*barriers*/ - runbytes - 2 * pbytes - 4096 /*ones*/;
+  d.stages = std::min(24, budget / (d.slot_a + d.slot_b));
   if (d.stages < 2) return false;
-  d.smem_bytes = 1024 + d.stages * (16384 + d.slot_b) + 2 * pbytes + 16384 + 1024;
+  d.smem_bytes = 1024 + d.stages * (d.slot_a + d.slot_b) + 2 * pbytes + 4096 + 2048 + runbytes;
   const int cols = 2 * d.ubuf + d.Np;
   d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
   return cols <= 512;
@@ -284,23 +293,26 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
     }
     encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
   }
-  auto make = [&](unsigned char* dst, void* base, uint64_t inner, uint64_t outer, uint32_t box_outer) {
+  auto swz = [](int aw) {
+    return aw == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : aw == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+  };
+  auto make = [&](unsigned char* dst, void* base, uint64_t inner, uint64_t outer, uint32_t box_outer, int aw = 64) {
     cuuint64_t dims[2] = {inner, outer};
     cuuint64_t strides[1] = {inner * 2};
-    cuuint32_t box[2] = {64, box_outer};
+    cuuint32_t box[2] = {(cuuint32_t)aw, box_outer};
     cuuint32_t es[2] = {1, 1};
     CUresult r = encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, base, dims, strides,
-                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz(aw),
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
   };
   auto make4 = [&](unsigned char* dst, void* base, const TcChainDesc* d, const TcTerm& t) {
     cuuint64_t dims[4] = {(cuuint64_t)t.R, (cuuint64_t)t.Win, (cuuint64_t)t.Hin, (cuuint64_t)d->nimg};
     cuuint64_t strides[3] = {(cuuint64_t)t.R * 2, (cuuint64_t)t.Win * t.R * 2, (cuuint64_t)t.Hin * t.Win * t.R * 2};
-    cuuint32_t box[4] = {64, (cuuint32_t)(d->tw * t.ts), (cuuint32_t)(d->th * t.ts), (cuuint32_t)d->tn};
+    cuuint32_t box[4] = {(cuuint32_t)t.aw, (cuuint32_t)(d->tw * t.ts), (cuuint32_t)(d->th * t.ts), (cuuint32_t)d->tn};
     cuuint32_t es[4] = {1, (cuuint32_t)t.ts, (cuuint32_t)t.ts, 1};
     CUresult r = encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, base, dims, strides,
-                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz(t.aw),
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     return r == CUDA_SUCCESS;
   };
@@ -310,22 +322,22 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
     const int nt = d->npc ? d->mt1 : d->n_terms;
     for (int j = 0; j < nt; ++j) {
       TcTerm& t = d->term[j];
-      bool ok = make(t.wmap, tcw + t.w, (uint64_t)t.Rw, (uint64_t)d->Cpad, (uint32_t)d->Cc);
+      bool ok = make(t.wmap, tcw + t.w, (uint64_t)t.Rw, (uint64_t)d->Cpad, (uint32_t)d->Cc, t.aw);
       if (d->spatial)
         ok = ok && make4(t.tmap4, arena + t.r.off, d, t);
       else
-        ok = ok && make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->nimg * t.Hin * t.Win, 128);
+        ok = ok && make(t.tmap, arena + t.r.off, (uint64_t)t.R, (uint64_t)d->nimg * t.Hin * t.Win, 128, t.aw);
       if (!ok) {
         err = "cuTensorMapEncodeTiled failed (term)";
         return false;
       }
     }
     for (int l = 0; l < d->n_levels; ++l)
-      if (!make(d->bmap[l], tcw + d->boff[l], 8, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+      if (!make(d->bmap[l], tcw + d->boff[l], 8, (uint64_t)d->Cpad, (uint32_t)d->Cc, 16)) {
         err = "cuTensorMapEncodeTiled failed (bias)";
         return false;
       }
-    if (d->npc && !make(d->bmapm, tcw + d->boffm, 8, (uint64_t)d->Cpad, (uint32_t)d->Cc)) {
+    if (d->npc && !make(d->bmapm, tcw + d->boffm, 8, (uint64_t)d->Cpad, (uint32_t)d->Cc, 16)) {
       err = "cuTensorMapEncodeTiled failed (member bias)";
       return false;
     }
@@ -350,7 +362,6 @@ __device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
 constexpr int kEpiWarps = 8;
 constexpr int kProdWarp = 8, kMmaWarp = 9;
 constexpr int kThreads = 32 * 10;
-constexpr int kSlotA = 16384;
 
 // Units of one tile: pooled chunks c < npc contribute ntg tap-group units each,
 // every other chunk one unit.  Units are processed in pairs (TMEM buffers 0, 1);
@@ -400,13 +411,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   const int S = d.stages;
+  const int kSlotA = d.slot_a;
   const int slot = kSlotA + d.slot_b;
   const int Cc = d.Cc;
   const int pbytes = 128 * Cc * 2;
   uint8_t* ring = smem;
   uint8_t* pbuf = ring + S * slot;
   uint8_t* ones = pbuf + 2 * pbytes;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(ones + 16384);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ones + 4096);
   uint64_t* full = bars;
   uint64_t* empty = bars + S;
   uint64_t* acc_full = bars + 2 * S;
@@ -418,11 +430,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(out_empty + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  // constant A operand of the bias MMA: K columns 0 and 1 = 1.0 (bf16), SW128 layout
-  for (int i = threadIdx.x; i < 16384 / 16; i += blockDim.x) {
-    const int row = i / 8, ch = i % 8;
+  // constant A operand of the bias MMA: K columns 0 and 1 = 1.0 (bf16), one SW32 atom
+  for (int i = threadIdx.x; i < 128 * 2; i += blockDim.x) {
+    const int row = i / 2, ch = i % 2;
     uint4 v = make_uint4(0, 0, 0, 0);
-    if (ch == (row & 7)) v.x = 0x3F803F80u;          // logical chunk 0 of this row
+    if (ch == swz_chunk(row, 0, 16)) v.x = 0x3F803F80u;   // logical chunk 0 of this row
     reinterpret_cast<uint4*>(ones)[i] = v;
   }
   fence_proxy_async();
@@ -457,11 +469,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      const uint32_t bytes_b = Cc * 128, bytes_f = d.Np * 128;
-      const uint32_t bytes_a = d.spatial ? 128u * d.tw * d.th * d.tn : (uint32_t)kSlotA;
-      auto load_b = [&](const void* map, int x, int y) {
+      const uint32_t bytes_f = d.Np * 128;
+      const uint32_t rows_a = d.spatial ? (uint32_t)(d.tw * d.th * d.tn) : 128u;
+      auto load_b = [&](const void* map, int x, int y) {           // bias: [Cc x 16] SW32 box
         mbar_wait(&empty[stage], phase ^ 1);
-        mbar_expect_tx(&full[stage], bytes_b);
+        mbar_expect_tx(&full[stage], Cc * 32);
         tma_load_2d(ring + stage * slot + kSlotA, map, &full[stage], x, y);
         if (++stage == S) stage = 0, phase ^= 1;
       };
@@ -483,16 +495,16 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   for (int q = 0; q < ntap; ++q) {
                     const int tap = un.pooled ? un.tg * d.tpu + r : q;
                     const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
-                    for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                    for (int ka = 0; ka < t.Rp / t.aw; ++ka) {
                       mbar_wait(&empty[stage], phase ^ 1);
-                      mbar_expect_tx(&full[stage], bytes_a + bytes_b);
+                      mbar_expect_tx(&full[stage], (rows_a + Cc) * t.aw * 2);
                       uint8_t* sa = ring + stage * slot;
                       if (d.spatial)      // (tap-shifted) strided box of the term's input
-                        tma_load_4d(sa, t.tmap4, &full[stage], ka * 64, gg.w0 * t.ts - pad + tap % kk,
+                        tma_load_4d(sa, t.tmap4, &full[stage], ka * t.aw, gg.w0 * t.ts - pad + tap % kk,
                                     gg.h0 * t.ts - pad + tap / kk, gg.n0);
                       else
-                        tma_load_2d(sa, t.tmap, &full[stage], ka * 64, gg.m0);
-                      tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * 64, un.c * Cc);
+                        tma_load_2d(sa, t.tmap, &full[stage], ka * t.aw, gg.m0);
+                      tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * t.aw, un.c * Cc);
                       if (++stage == S) stage = 0, phase ^= 1;
                     }
                   }
@@ -517,7 +529,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      uint32_t acc_use0 = 0, acc_use1 = 0, p_use0 = 0, p_use1 = 0, tile_iter = 0;
+      uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
       const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
       const uint32_t tout = tbase + 2 * d.ubuf;
       const uint32_t ones_addr = smem_u32(ones);
@@ -527,15 +539,15 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           for (int l = 0; l < d.n_levels; ++l)
             for (int bi = 0; bi < nb; ++bi) {
               const Unit un = unit_at(d, u0 + bi);
-              uint32_t& use = bi ? acc_use1 : acc_use0;
-              mbar_wait(&acc_empty[bi], (use & 1) ^ 1);
+              const uint32_t abit = 1u << bi;
+              mbar_wait(&acc_empty[bi], ((acc_par & abit) ? 1u : 0u) ^ 1u);
               tc_fence_after();
               const uint32_t tacc = tbase + bi * d.ubuf;
               // bias (initialises every tap region of the accumulator at level 0)
               mbar_wait(&full[stage], phase);
               tc_fence_after();
               for (int r = 0; r < un.nt; ++r)
-                mma_bf16(tacc + r * Cc, umma_desc(ones_addr), umma_desc(smem_u32(ring + stage * slot + kSlotA)), id1,
+                mma_bf16(tacc + r * Cc, umma_desc_k(ones_addr, 16), umma_desc_k(smem_u32(ring + stage * slot + kSlotA), 16), id1,
                          l == 0 ? 0u : 1u);
               mma_commit(&empty[stage]);
               if (++stage == S) stage = 0, phase ^= 1;
@@ -547,27 +559,28 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   if (!un.pooled && !term_hits(t, un.c, Cc)) continue;
                   const int ntap = un.pooled ? 1 : t.tk * t.tk;
                   for (int q = 0; q < ntap; ++q)
-                    for (int ka = 0; ka < t.Rp / 64; ++ka) {
+                    for (int ka = 0; ka < t.Rp / t.aw; ++ka) {
                       mbar_wait(&full[stage], phase);
                       tc_fence_after();
                       const uint32_t sa = smem_u32(ring + stage * slot);
-                      const int nk = min(4, (t.R - ka * 64 + 15) / 16);
+                      const int nk = min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
                       for (int k = 0; k < nk; ++k)
-                        mma_bf16(tacc + r * Cc, umma_desc(sa + 32 * k), umma_desc(sa + kSlotA + 32 * k), id1, 1u);
+                        mma_bf16(tacc + r * Cc, umma_desc_k(sa + 32 * k, t.aw), umma_desc_k(sa + kSlotA + 32 * k, t.aw),
+                                 id1, 1u);
                       mma_commit(&empty[stage]);
                       if (++stage == S) stage = 0, phase ^= 1;
                     }
                 }
               mma_commit(&acc_full[bi]);
-              ++use;
+              acc_par ^= abit;
             }
           if (!d.gap)
             for (int bi = 0; bi < nb; ++bi) {
               const Unit un = unit_at(d, u0 + bi);
               if (!un.last) continue;
               const int pb = un.c & 1;
-              uint32_t& puse = pb ? p_use1 : p_use0;
-              mbar_wait(&p_full[pb], puse & 1);
+              const uint32_t pbit = 1u << pb;
+              mbar_wait(&p_full[pb], (p_par & pbit) ? 1u : 0u);
               tc_fence_after();
               if (un.c == 0) {
                 mbar_wait(out_empty, (tile_iter & 1) ^ 1);
@@ -585,7 +598,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 if (++stage == S) stage = 0, phase ^= 1;
               }
               mma_commit(&p_empty[pb]);
-              ++puse;
+              p_par ^= pbit;
             }
         }
         if (!d.gap) mma_commit(out_full);
@@ -600,9 +613,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     const int half = Cc / 2;                          // columns per warp (32 or 64)
     const int c_lo = h * half;
-    uint32_t acc_use0 = 0, acc_use1 = 0, p_use0 = 0, p_use1 = 0, tile_iter = 0;
+    uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
-    float run[32];                                    // pooled member (Cc = 64 -> 32 columns per warp)
+    float* runbuf = reinterpret_cast<float*>(bars + 64);   // pooled member running max / sum (32 KB)
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
       int64_t m = (int64_t)tile * d.rows_per_tile + row;
       bool mvalid = m < d.npix;
@@ -624,21 +637,23 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           const bool relu = d.relu[l] != 0;
           for (int bi = 0; bi < nb; ++bi) {
             const Unit un = unit_at(d, u0 + bi);
-            uint32_t& use = bi ? acc_use1 : acc_use0;
-            mbar_wait(&acc_full[bi], use & 1);
-            ++use;
+            const uint32_t abit = 1u << bi;
+            mbar_wait(&acc_full[bi], (acc_par & abit) ? 1u : 0u);
+            acc_par ^= abit;
             tc_fence_after();
             const int pb = un.c & 1;
             const bool writes_p = last && !d.gap && un.last;
             if (writes_p) {
-              uint32_t& puse = pb ? p_use1 : p_use0;
-              mbar_wait(&p_empty[pb], (puse & 1) ^ 1);
-              ++puse;
+              const uint32_t pbit = 1u << pb;
+              mbar_wait(&p_empty[pb], ((p_par & pbit) ? 1u : 0u) ^ 1u);
+              p_par ^= pbit;
             }
             const uint32_t ta = tbase + lane_off + bi * d.ubuf + c_lo;
             uint8_t* P = pbuf + pb * pbytes;
             if (un.pooled) {
-              // pooled member: fold the unit's taps into the running max / sum (half == 32)
+              // pooled member: fold the unit's taps into the running max / sum (half == 32),
+              // kept in a conflict-free SMEM slab (element i of thread t at run[i * 256 + t])
+              float* run = runbuf + threadIdx.x;
               for (int r = 0; r < un.nt; ++r) {
                 const int tap = un.tg * d.tpu + r;
                 const int hi = ho * d.ms - d.mp + tap / d.mk, wi = wo * d.ms - d.mp + tap % d.mk;
@@ -646,55 +661,66 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 uint32_t v[32];
                 tmem_ld32(ta + r * Cc, v);
                 tmem_wait_ld();
+                const bool first = tap == 0;
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
                   float x = __uint_as_float(v[i]);
                   x = d.mrelu ? fmaxf(x, 0.f) : x;
+                  float cur = first ? (d.mpool == 1 ? -INFINITY : 0.f) : run[i * 256];
                   if (d.mpool == 1)
-                    run[i] = tap == 0 ? (valid ? x : -INFINITY) : (valid ? fmaxf(run[i], x) : run[i]);
+                    cur = valid ? fmaxf(cur, x) : cur;
                   else
-                    run[i] = tap == 0 ? x : run[i] + x;
+                    cur += x;
+                  run[i * 256] = cur;
                 }
               }
               if (un.last) {
                 // pooled value, + post-pool shift (BN after the pool), level activation
                 const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
                 const float* post = d.post >= 0 ? p.params + d.post + un.c * Cc + c_lo : nullptr;
+                const int ch0 = c_lo / 8;
 #pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                  float x = run[i] * sc + (post ? __ldg(post + i) : 0.f);
-                  run[i] = relu ? fmaxf(x, 0.f) : x;
-                }
-                if (d.gap) {
-                  // not reached: GAP with a pooled member is not lowered here
-                } else {
-                  const int ch0 = c_lo / 8;
+                for (int qq = 0; qq < 4; ++qq) {
+                  float f[8];
 #pragma unroll
-                  for (int qq = 0; qq < 4; ++qq) {
-                    uint4 pk;
-                    pk.x = pack_bf16(run[8 * qq + 0], run[8 * qq + 1]);
-                    pk.y = pack_bf16(run[8 * qq + 2], run[8 * qq + 3]);
-                    pk.z = pack_bf16(run[8 * qq + 4], run[8 * qq + 5]);
-                    pk.w = pack_bf16(run[8 * qq + 6], run[8 * qq + 7]);
-                    *reinterpret_cast<uint4*>(P + row * 128 + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
+                  for (int i = 0; i < 8; ++i) {
+                    const float x = run[(8 * qq + i) * 256] * sc + (post ? __ldg(post + 8 * qq + i) : 0.f);
+                    f[i] = relu ? fmaxf(x, 0.f) : x;
                   }
+                  uint4 pk;
+                  pk.x = pack_bf16(f[0], f[1]);
+                  pk.y = pack_bf16(f[2], f[3]);
+                  pk.z = pack_bf16(f[4], f[5]);
+                  pk.w = pack_bf16(f[6], f[7]);
+                  *reinterpret_cast<uint4*>(P + row * 128 + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
                 }
               }
             } else if (!last) {
               // t_l = relu(acc) back into TMEM for the next level's MMAs
-              uint32_t v[2][32];
-              tmem_ld32(ta, v[0]);
-              if (half == 64) tmem_ld32(ta + 32, v[1]);
-              tmem_wait_ld();
-              if (relu) {
+              if (half == 64) {
+                uint32_t a[32], b[32];
+                tmem_ld32(ta, a);
+                tmem_ld32(ta + 32, b);
+                tmem_wait_ld();
+                if (relu) {
 #pragma unroll
-                for (int i = 0; i < 32; ++i) v[0][i] = __float_as_uint(fmaxf(__uint_as_float(v[0][i]), 0.f));
-                if (half == 64)
+                  for (int i = 0; i < 32; ++i) {
+                    a[i] = __float_as_uint(fmaxf(__uint_as_float(a[i]), 0.f));
+                    b[i] = __float_as_uint(fmaxf(__uint_as_float(b[i]), 0.f));
+                  }
+                }
+                tmem_st32(ta, a);
+                tmem_st32(ta + 32, b);
+              } else {
+                uint32_t a[32];
+                tmem_ld32(ta, a);
+                tmem_wait_ld();
+                if (relu) {
 #pragma unroll
-                  for (int i = 0; i < 32; ++i) v[1][i] = __float_as_uint(fmaxf(__uint_as_float(v[1][i]), 0.f));
+                  for (int i = 0; i < 32; ++i) a[i] = __float_as_uint(fmaxf(__uint_as_float(a[i]), 0.f));
+                }
+                tmem_st32(ta, a);
               }
-              tmem_st32(ta, v[0]);
-              if (half == 64) tmem_st32(ta + 32, v[1]);
               tmem_wait_st();
             } else if (d.gap) {
               // GAP root: per-image column means; tiles hold whole images so the

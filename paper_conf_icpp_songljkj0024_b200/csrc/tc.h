@@ -32,7 +32,8 @@ struct TcTerm {
   alignas(64) unsigned char wmap[128];   // Lhat [Cpad x Rw], box {64, Cc}
   alignas(64) unsigned char tmap4[128];  // spatial tiles: 4D map of r [N, Hin, Win, R], box {64, tw*ts, th*ts, tn}
   Loc r;                 // reduced input [N, Hin, Win, R] bf16 (arena)
-  int32_t R, Rp;         // rank; padded to a multiple of 64 (one 128-byte K atom)
+  int32_t R, Rp;         // rank; padded to a multiple of the K atom
+  int32_t aw;            // K atom width in elements (16 / 32 / 64 -> SW32 / SW64 / SW128 boxes)
   int32_t Rw;            // row length of the packed weights (R rounded to 8; TMA zero-fills to Rp)
   int32_t c0, C;         // restored channels this term writes (concat members)
   int32_t Hin, Win;      // resolution of r
@@ -70,7 +71,7 @@ struct TcChainDesc {
   int64_t F;                             // tc weight pool offset of F
   int64_t Fb;                            // unused (fconv factors carry no bias)
   Loc y;                                 // output [npix, Nout] bf16, or [N, C] for GAP
-  int32_t stages, slot_b;                // smem ring depth, bytes of one B slot
+  int32_t stages, slot_a, slot_b;        // smem ring depth, bytes of one A / B slot
   int32_t smem_bytes, tmem_cols;
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
 };

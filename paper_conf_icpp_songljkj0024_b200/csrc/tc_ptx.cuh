@@ -50,6 +50,21 @@ __device__ __forceinline__ uint64_t umma_desc(uint32_t saddr) {
          ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
 
+// K-major descriptor for a K atom of `aw` bf16 elements per row (16, 32 or 64):
+// swizzle = row bytes (SW32 / SW64 / SW128), 8-row groups 8 * row bytes apart.
+// The atom base must be aligned to 8 * row bytes.
+__device__ __forceinline__ uint64_t umma_desc_k(uint32_t saddr, int aw) {
+  const uint64_t layout = aw == 64 ? 2 : aw == 32 ? 4 : 6;
+  const uint64_t sbo = (uint64_t)(16 * aw) >> 4;
+  return (uint64_t)((saddr & 0x3FFFF) >> 4) | ((uint64_t)1 << 16) | (sbo << 32) | ((uint64_t)1 << 46) |
+         (layout << 61);
+}
+
+// physical 16-byte chunk of logical chunk k in row r of a K atom with `aw` elements
+__host__ __device__ __forceinline__ int swz_chunk(int r, int k, int aw) {
+  return aw == 64 ? (k ^ (r & 7)) : aw == 32 ? (k ^ ((r >> 1) & 3)) : (k ^ ((r >> 2) & 1));
+}
+
 // kind::f16 instruction descriptor: bf16 A/B, fp32 D, K-major A/B
 __host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
   return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
