@@ -9,8 +9,12 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-BUILD = os.path.join(ROOT, "build", "temco")
-LIB = os.path.join(PKG, "libtemco.so")
+# experiment variants: TEMCO_VARIANT=name TEMCO_EXTRA_FLAGS="-DTEMCO_TRACE" builds
+# build/exp/libtemco_<name>.so (select it at run time with TEMCO_LIB)
+VARIANT = os.environ.get("TEMCO_VARIANT", "")
+EXTRA = os.environ.get("TEMCO_EXTRA_FLAGS", "").split()
+BUILD = os.path.join(ROOT, "build", "temco" + ("_" + VARIANT if VARIANT else ""))
+LIB = os.path.join(ROOT, "build", "exp", f"libtemco_{VARIANT}.so") if VARIANT else os.path.join(PKG, "libtemco.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 SOURCES = ["planner.cpp", "capi.cu", "kernels_simt.cu", "kernels_tc.cu", "kernels_conv.cu", "kernels_mma.cu"]
@@ -36,7 +40,7 @@ def _compile(src, verbose):
     o = os.path.join(BUILD, src + ".o")
     if not _stale(o, [s] + _headers()):
         return o
-    cmd = [NVCC] + GENCODE + COMMON + ["-c", s, "-o", o]
+    cmd = [NVCC] + GENCODE + COMMON + EXTRA + ["-c", s, "-o", o]
     if src.endswith(".cu"):
         cmd += ["-Xptxas", "-v"] if verbose else []
     if verbose:
@@ -51,6 +55,7 @@ def _compile(src, verbose):
 
 def build(verbose: bool = False) -> str:
     os.makedirs(BUILD, exist_ok=True)
+    os.makedirs(os.path.dirname(LIB), exist_ok=True)
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), SOURCES))
     if _stale(LIB, objs):

@@ -308,7 +308,7 @@ void lower(temco_plan_s* P) {
         e.kernel = "none";
         break;
       case OP_CONV: {
-        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && ir.nodes[ir.oin[s.out][0]].C % 8 == 0 &&
             conv_tc_lower(ir, s.out, P->loc, P->tcw_h, P->params_h, e.ctc)) {
           e.kind = K_CONV_TC;
           e.kernel = "tc_conv";
@@ -325,7 +325,7 @@ void lower(temco_plan_s* P) {
         c.w = push_params(P, repack_conv(v, x.C));
         c.b = push_params(P, v.b);
         e.kind = K_CONV;
-        e.kernel = v.groups > 1 ? "simt_dwconv" : "simt_conv";
+        e.kernel = v.groups > 1 ? "simt_dwconv" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
         e.launches = 1;
         break;
       }
@@ -425,7 +425,11 @@ std::string make_json(const temco_plan_s* P) {
       const StepExec& e = P->exec[t];
       o << ",\"kernel\":\"" << e.kernel << "\",\"flops\":" << e.flops << ",\"io_bytes\":" << e.io_bytes
         << ",\"launches\":" << e.launches;
-      if (e.kind == K_GROUP_TC) o << ",\"alg_flops\":" << e.tc.alg_flops << ",\"alg_bytes\":" << e.tc.alg_bytes;
+      if (e.kind == K_GROUP_TC)
+        o << ",\"alg_flops\":" << e.tc.alg_flops << ",\"alg_bytes\":" << e.tc.alg_bytes << ",\"tc\":{\"n_prod\":"
+          << e.tc.n_prod << ",\"n_mma\":" << e.tc.n_mma << ",\"units\":" << e.tc.units << ",\"stages\":" << e.tc.stages
+          << ",\"resident\":" << e.tc.resident << ",\"pipelined\":" << (e.tc.mma_head > 0) << ",\"ntiles\":"
+          << e.tc.ntiles << ",\"Cc\":" << e.tc.Cc << ",\"levels\":" << e.tc.n_levels << "}";
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;
     }
@@ -467,7 +471,12 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t], st));
     switch (e.kind) {
       case K_NONE: break;
-      case K_CONV: launch_conv(e.conv, rp, st); break;
+      case K_CONV:
+        if (conv_small_ok(e.conv))
+          launch_conv_small(e.conv, rp, st);
+        else
+          launch_conv(e.conv, rp, st);
+        break;
       case K_EW: launch_ew(e.ew, rp, st); break;
       case K_LINEAR: launch_linear(e.lin, rp, st); break;
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;

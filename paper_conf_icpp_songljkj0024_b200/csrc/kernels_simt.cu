@@ -32,6 +32,96 @@ inline int grid_for(int64_t total, int block) {
 }
 
 // ---------------------------------------------------------------------------
+// small-Cin direct convolution (the stem core on the 3-channel image, CP first
+// factors on it): a 16 x 32 output tile per CTA, its input footprint staged in
+// SMEM as fp32, each thread two output rows x 8 output channels (weights are
+// warp-broadcast SMEM reads shared by the two pixels).  gridDim.z = K / 8.
+// ---------------------------------------------------------------------------
+constexpr int kSmTH = 16, kSmTW = 32, kSmKC = 8;
+
+__global__ void __launch_bounds__(256) conv_small_kernel(ConvDesc d, RunPtrs p, int tiles_w, int tiles_h) {
+  extern __shared__ float sm[];
+  const int Cin = d.C;
+  const int ir = (kSmTH - 1) * d.sh + d.kh, ic = (kSmTW - 1) * d.sw + d.kw;
+  const int taps = d.kh * d.kw;
+  float* xs = sm;                                   // [ir][ic][Cin]
+  float* ws = sm + (ir * ic * Cin + 3) / 4 * 4;     // [tap][c][8], 16-byte aligned
+  const int tile = blockIdx.x;
+  const int n = tile / (tiles_w * tiles_h);
+  const int h0 = (tile / tiles_w) % tiles_h * kSmTH, w0 = tile % tiles_w * kSmTW;
+  const int k0 = blockIdx.y * kSmKC;
+  const void* x = loc_ptr(d.x, p);
+  // stage the input footprint (zero padding outside the image)
+  const int hi0 = h0 * d.sh - d.ph, wi0 = w0 * d.sw - d.pw;
+  const int rowlen = ic * Cin;
+  for (int i = threadIdx.x; i < ir * rowlen; i += blockDim.x) {
+    const int r = i / rowlen, e = i % rowlen;
+    const int hi = hi0 + r, wi = wi0 + e / Cin, c = e % Cin;
+    float v = 0.f;
+    if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W)
+      v = ldv(x, (((int64_t)n * d.H + hi) * d.W + wi) * Cin + c, d.x.dtype);
+    xs[i] = v;
+  }
+  for (int i = threadIdx.x; i < taps * Cin * kSmKC; i += blockDim.x) {
+    const int j = i % kSmKC, tc = i / kSmKC;
+    const int k = k0 + j;
+    ws[i] = k < d.K ? p.params[d.w + (int64_t)k * taps * Cin + tc] : 0.f;
+  }
+  __syncthreads();
+  const int tx = threadIdx.x % kSmTW, ty = threadIdx.x / kSmTW;   // rows ty and ty + 8
+  float acc0[kSmKC], acc1[kSmKC];
+#pragma unroll
+  for (int j = 0; j < kSmKC; ++j) {
+    const float b = (d.b >= 0 && k0 + j < d.K) ? p.params[d.b + k0 + j] : 0.f;
+    acc0[j] = b;
+    acc1[j] = b;
+  }
+  const int r8 = 8 * d.sh * rowlen;
+  for (int a = 0; a < d.kh; ++a)
+    for (int bb = 0; bb < d.kw; ++bb) {
+      const float* xp = xs + (ty * d.sh + a) * rowlen + (tx * d.sw + bb) * Cin;
+      const float* wp = ws + (a * d.kw + bb) * Cin * kSmKC;
+      for (int c = 0; c < Cin; ++c) {
+        const float x0 = xp[c], x1 = xp[r8 + c];
+        const float4 wa = reinterpret_cast<const float4*>(wp + c * kSmKC)[0];
+        const float4 wb = reinterpret_cast<const float4*>(wp + c * kSmKC)[1];
+        const float w8[8] = {wa.x, wa.y, wa.z, wa.w, wb.x, wb.y, wb.z, wb.w};
+#pragma unroll
+        for (int j = 0; j < kSmKC; ++j) {
+          acc0[j] = fmaf(w8[j], x0, acc0[j]);
+          acc1[j] = fmaf(w8[j], x1, acc1[j]);
+        }
+      }
+    }
+  void* y = const_cast<void*>(loc_ptr(d.y, p));
+  const int wo = w0 + tx;
+#pragma unroll
+  for (int s = 0; s < 2; ++s) {
+    const int ho = h0 + ty + 8 * s;
+    if (ho >= d.Ho || wo >= d.Wo) continue;
+    const float* acc = s ? acc1 : acc0;
+    const int64_t base = (((int64_t)n * d.Ho + ho) * d.Wo + wo) * d.K + k0;
+    if (d.y.dtype == DT_BF16 && k0 + kSmKC <= d.K && d.K % 8 == 0) {
+      uint4 pk;
+      __nv_bfloat162 h01 = __floats2bfloat162_rn(acc[0], acc[1]), h23 = __floats2bfloat162_rn(acc[2], acc[3]);
+      __nv_bfloat162 h45 = __floats2bfloat162_rn(acc[4], acc[5]), h67 = __floats2bfloat162_rn(acc[6], acc[7]);
+      pk.x = *reinterpret_cast<uint32_t*>(&h01);
+      pk.y = *reinterpret_cast<uint32_t*>(&h23);
+      pk.z = *reinterpret_cast<uint32_t*>(&h45);
+      pk.w = *reinterpret_cast<uint32_t*>(&h67);
+      *reinterpret_cast<uint4*>(reinterpret_cast<__nv_bfloat16*>(y) + base) = pk;
+    } else {
+      for (int j = 0; j < kSmKC && k0 + j < d.K; ++j) stv(y, base + j, acc[j], d.y.dtype);
+    }
+  }
+}
+
+int conv_small_smem(const ConvDesc& d) {
+  const int ir = (kSmTH - 1) * d.sh + d.kh, ic = (kSmTW - 1) * d.sw + d.kw;
+  return ((ir * ic * d.C + 3) / 4 * 4 + d.kh * d.kw * d.C * kSmKC) * 4;
+}
+
+// ---------------------------------------------------------------------------
 // direct NHWC convolution: one thread per output element, output channel
 // fastest so a warp shares its input pixels (broadcast loads)
 // ---------------------------------------------------------------------------
@@ -326,6 +416,21 @@ __global__ void group_gap_kernel(GroupDesc d, GCtx g) {
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.K;
   conv_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
+}
+
+bool conv_small_ok(const ConvDesc& d) {
+  return d.groups == 1 && d.C <= 8 && d.K <= 64 && d.sh == d.sw && d.sh <= 4 && conv_small_smem(d) <= 96 * 1024;
+}
+
+void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  if (!configured) {
+    cudaFuncSetAttribute(conv_small_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
+    configured = true;
+  }
+  const int tw = (d.Wo + kSmTW - 1) / kSmTW, th = (d.Ho + kSmTH - 1) / kSmTH;
+  dim3 grid((unsigned)(d.N * tw * th), (unsigned)((d.K + kSmKC - 1) / kSmKC));
+  conv_small_kernel<<<grid, 256, conv_small_smem(d), s>>>(d, p, tw, th);
 }
 
 void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s) {

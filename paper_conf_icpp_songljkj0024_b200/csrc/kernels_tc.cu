@@ -72,6 +72,184 @@ int64_t push_bias(std::vector<uint16_t>& pool, const std::vector<double>& b, int
   return push_bf16(pool, bm);
 }
 
+// Per-tile producer / MMA programs.  Unit order (all roles): for each pair of
+// units: for each level: for each unit of the pair: [bias, terms x taps x K
+// atoms]; then the fconv atoms of the pair's finished chunks.  TMEM buffer of
+// unit u of a tile = (units before the tile + u) & 1.
+void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
+  std::vector<TcProdOp> P;
+  std::vector<TcMmaOp> M;
+  const int Cc = d.Cc;
+  const int U = d.npc * d.ntg + d.nchunks - d.npc;
+  d.units = U;
+  const bool res = d.resident != 0;
+  const int rows_a = d.spatial ? d.tw * d.th * d.tn : 128;
+  const int pbytes = 128 * Cc * 2;
+  auto moff = [&](const unsigned char* m) {
+    return (uint16_t)((reinterpret_cast<const char*>(m) - reinterpret_cast<const char*>(&d)) / 64);
+  };
+  struct HUnit {
+    int c, tg, nt;
+    bool pooled, last;
+  };
+  auto unit_at = [&](int u) {
+    HUnit x;
+    if (u < d.npc * d.ntg) {
+      x.c = u / d.ntg;
+      x.tg = u % d.ntg;
+      x.nt = std::min(d.tpu, d.mtaps - x.tg * d.tpu);
+      x.pooled = true;
+      x.last = x.tg == d.ntg - 1;
+    } else {
+      x.c = d.npc + (u - d.npc * d.ntg);
+      x.tg = 0;
+      x.nt = 1;
+      x.pooled = false;
+      x.last = true;
+    }
+    return x;
+  };
+  for (int u0 = 0; u0 < U; u0 += 2) {
+    const int nb = std::min(2, U - u0);
+    for (int l = 0; l < d.n_levels; ++l)
+      for (int bi = 0; bi < nb; ++bi) {
+        const int u = u0 + bi;
+        const HUnit un = unit_at(u);
+        // bias: initialises (level 0) every tap region of the accumulator
+        if (!res) {
+          TcProdOp o{};
+          o.kind = PK_B;
+          o.bmap = moff(un.pooled ? d.bmapm : d.bmap[l]);
+          o.bx = 0;
+          o.by = (int16_t)(un.c * Cc);
+          o.bytes = (uint16_t)(Cc * 32);
+          P.push_back(o);
+        }
+        for (int r = 0; r < un.nt; ++r) {
+          TcMmaOp m{};
+          m.flags = MF_ONES | (l == 0 ? MF_ZERO : 0) | (r == 0 ? MF_ACC_WAIT : 0);
+          if (res) {
+            m.flags |= MF_BRES;
+            m.boff = (uint32_t)((un.pooled ? d.bresm : d.bres[l]) + un.c * Cc * 32);
+          } else {
+            m.flags |= MF_SB | (r == 0 ? MF_SW : 0) | (r == un.nt - 1 ? MF_SD : 0);
+          }
+          m.unit = (uint8_t)u;
+          m.nk = 1;
+          m.la = 16;
+          m.lb = 16;
+          m.tcol = (uint16_t)(r * Cc);
+          M.push_back(m);
+        }
+        const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
+        const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
+        for (int r = 0; r < un.nt; ++r)
+          for (int j = j0; j < j1; ++j) {
+            const TcTerm& t = d.term[j];
+            if (!un.pooled && !(t.c0 < (un.c + 1) * Cc && t.c0 + t.C > un.c * Cc)) continue;
+            const int ntap = un.pooled ? 1 : t.tk * t.tk;
+            const int katoms = t.Rp / t.aw;
+            for (int q = 0; q < ntap; ++q) {
+              const int tap = un.pooled ? un.tg * d.tpu + r : q;
+              const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
+              for (int ka = 0; ka < katoms; ++ka) {
+                TcProdOp o{};
+                o.kind = d.spatial ? PK_A4D : PK_A2D;
+                o.ts = (uint8_t)t.ts;
+                o.amap = moff(d.spatial ? t.tmap4 : t.tmap);
+                o.ac = (int16_t)(ka * t.aw);
+                o.dx = (int16_t)(tap % kk - pad);
+                o.dy = (int16_t)(tap / kk - pad);
+                o.bytes = (uint16_t)((rows_a + (res ? 0 : Cc)) * t.aw * 2);
+                if (!res) {
+                  o.kind |= PK_B;
+                  o.bmap = moff(t.wmap);
+                  o.bx = (int16_t)(ka * t.aw);
+                  o.by = (int16_t)(un.c * Cc);
+                }
+                P.push_back(o);
+                TcMmaOp m{};
+                m.flags = MF_SW | MF_SA | MF_SD | (res ? MF_BRES : MF_SB);
+                m.unit = (uint8_t)u;
+                m.nk = (uint8_t)std::min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
+                m.la = (uint8_t)t.aw;
+                m.lb = (uint8_t)t.aw;
+                m.tcol = (uint16_t)(r * Cc);
+                if (res) m.boff = (uint32_t)(t.wres + ((un.c - t.cfirst) * katoms + ka) * Cc * t.aw * 2);
+                M.push_back(m);
+              }
+            }
+          }
+        M.back().flags |= MF_ACC_COMMIT;
+      }
+    if (!d.gap)
+      for (int bi = 0; bi < nb; ++bi) {
+        const HUnit un = unit_at(u0 + bi);
+        if (!un.last) continue;
+        const int pb = un.c & 1;
+        const int na = Cc / 64;
+        for (int a = 0; a < na; ++a) {
+          if (!res) {
+            TcProdOp o{};
+            o.kind = PK_B;
+            o.bmap = moff(d.fmap);
+            o.bx = (int16_t)(un.c * Cc + a * 64);
+            o.by = 0;
+            o.bytes = (uint16_t)(d.Np * 128);
+            P.push_back(o);
+          }
+          TcMmaOp m{};
+          m.flags = MF_F | (a == 0 ? MF_P_WAIT : 0) | (a == 0 && un.c == 0 ? MF_OUT_WAIT | MF_ZERO : 0) |
+                    (a == na - 1 ? MF_P_COMMIT : 0) | (res ? MF_BRES : MF_SW | MF_SB | MF_SD);
+          m.unit = (uint8_t)pb;
+          m.nk = 4;
+          m.la = 64;
+          m.lb = 64;
+          m.aoff = (uint32_t)(pb * pbytes + a * 16384);
+          if (res) m.boff = (uint32_t)(d.fres + (un.c * na + a) * d.Np * 128);
+          M.push_back(m);
+        }
+      }
+  }
+  if (!d.gap) M.back().flags |= MF_OUT_COMMIT;
+  d.n_prod = (int32_t)P.size();
+  d.n_mma = (int32_t)M.size();
+  // programs live in SMEM (after the pooled slab) when they fit next to the ring
+  const int pbytes_prog = (int)(P.size() * sizeof(TcProdOp) + M.size() * sizeof(TcMmaOp));
+  d.prog_smem = 0;
+  const char* exp_env = getenv("TEMCO_TC_EXP");   // experiment switches (bit 0: programs in global memory)
+  const int exp_bits = exp_env ? atoi(exp_env) : 0;
+  if (pbytes_prog <= 32768 && !(exp_bits & 1)) {
+    const int need = (pbytes_prog + 127) / 128 * 128;
+    while (d.stages > 2 && d.smem_bytes + need > 227 * 1024)
+      d.stages--, d.smem_bytes -= d.slot_a + d.slot_b;
+    if (d.smem_bytes + need <= 227 * 1024) {
+      d.prog_smem = need;
+      d.smem_bytes += need;
+    }
+  }
+  // pipelined MMA order (unit ops of tile t+1 before the fconv ops of tile t):
+  // needs resident weights (the ring then carries only unit stages, consumed in
+  // the same order) and a program of the form [unit ops][fconv ops]
+  d.mma_head = 0;
+  // and every TMEM buffer the head of tile t+1 waits for must be released by the
+  // epilogue before it waits for tile t's output: one level, <= 2 units per tile
+  if (res && !d.gap && d.n_levels == 1 && U <= 2) {
+    int h = 0;
+    while (h < (int)M.size() && !(M[h].flags & MF_F)) ++h;
+    bool tail_f = true;
+    for (size_t i = h; i < M.size(); ++i) tail_f &= (M[i].flags & MF_F) != 0;
+    if (tail_f && h > 0 && h < (int)M.size()) d.mma_head = h;
+  }
+  while (tcw.size() % 512) tcw.push_back(0);
+  d.prog_off = (int64_t)tcw.size();
+  const size_t nbytes = P.size() * sizeof(TcProdOp) + M.size() * sizeof(TcMmaOp);
+  tcw.resize(tcw.size() + (nbytes + 1) / 2);
+  char* dst = reinterpret_cast<char*>(tcw.data() + d.prog_off);
+  memcpy(dst, P.data(), P.size() * sizeof(TcProdOp));
+  memcpy(dst + P.size() * sizeof(TcProdOp), M.data(), M.size() * sizeof(TcMmaOp));
+}
+
 }  // namespace
 
 bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
@@ -180,6 +358,8 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     T.tk = t.tk;
     T.ts = t.ts;
     T.tp = t.tp;
+    T.cfirst = t.c0 / d.Cc;
+    T.nhit = (t.c0 + lc.C - 1) / d.Cc - T.cfirst + 1;
     std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);
     for (int c = 0; c < lc.C; ++c)
       for (int k = 0; k < R; ++k)
@@ -270,12 +450,38 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   const int pbytes = 128 * d.Cc * 2;
   const int runbytes = pm ? 32768 : 0;     // pooled member: running max / sum slab (after the barriers)
   const int budget = 227 * 1024 - 1024 /*align*/ - 2048 /*barriers*/ - runbytes - 2 * pbytes - 4096 /*ones*/;
-  d.stages = std::min(24, budget / (d.slot_a + d.slot_b));
+  // resident weights: every B box (term atoms of the chunks a term reaches, level
+  // and member biases, F atoms) once per CTA, if that leaves a ring of >= 6 A slots
+  int64_t woff = 0;
+  for (int i = 0; i < nall; ++i) {
+    TcTerm& T = d.term[i];
+    T.wres = (int32_t)woff;
+    woff += (int64_t)T.nhit * (T.Rp / T.aw) * d.Cc * T.aw * 2;
+  }
+  for (int l = 0; l < d.n_levels; ++l) {
+    d.bres[l] = (int32_t)woff;
+    woff += (int64_t)d.nchunks * d.Cc * 32;
+  }
+  d.bresm = (int32_t)woff;
+  woff += (int64_t)d.npc * d.Cc * 32;
+  d.fres = (int32_t)woff;
+  if (!gap) woff += (int64_t)(d.Cpad / 64) * d.Np * 128;
+  d.resident = woff + 6LL * d.slot_a <= budget ? 1 : 0;
+  if (d.resident) {
+    d.wres_bytes = (int32_t)woff;
+    d.slot_b = 0;
+    d.stages = std::min<int64_t>(24, (budget - woff) / d.slot_a);
+  } else {
+    d.wres_bytes = 0;
+    d.stages = std::min(24, budget / (d.slot_a + d.slot_b));
+  }
   if (d.stages < 2) return false;
-  d.smem_bytes = 1024 + d.stages * (d.slot_a + d.slot_b) + 2 * pbytes + 4096 + 2048 + runbytes;
+  d.smem_bytes = 1024 + d.wres_bytes + d.stages * (d.slot_a + d.slot_b) + 2 * pbytes + 4096 + 2048 + runbytes;
   const int cols = 2 * d.ubuf + d.Np;
   d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
-  return cols <= 512;
+  if (cols > 512) return false;
+  build_programs(d, tcw);
+  return true;
 }
 
 bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char* arena, uint16_t* tcw,
@@ -319,6 +525,8 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
   for (size_t i = 0; i < n; ++i) {
     TcChainDesc* d = get(i);
     if (!d) continue;
+    d->prod = reinterpret_cast<const TcProdOp*>(tcw + d->prog_off);
+    d->mma = reinterpret_cast<const TcMmaOp*>(reinterpret_cast<const char*>(d->prod) + d->n_prod * sizeof(TcProdOp));
     const int nt = d->npc ? d->mt1 : d->n_terms;
     for (int j = 0; j < nt; ++j) {
       TcTerm& t = d->term[j];
@@ -358,6 +566,34 @@ using namespace ptx;
 __device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
   return t.c0 < (c + 1) * Cc && t.c0 + t.C > c * Cc;
 }
+
+#ifdef TEMCO_TRACE
+// experiment builds only: %globaltimer stamps of CTA 0's pipeline events
+constexpr int kTraceRows = 12;
+__device__ unsigned long long g_trace[kTraceRows][512];
+__device__ int g_dbg;   // 1: TMA-only run (MMA / epilogue roles idle; output garbage)
+__device__ __forceinline__ void trace_stamp(int row, int& n) {
+  if (blockIdx.x == 0 && n < 512) {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    g_trace[row][n] = t;
+  }
+  ++n;
+}
+#ifdef TEMCO_NOSTAMP
+#define TRACE(row, n) ((void)0)
+#else
+#define TRACE(row, n) trace_stamp(row, n)
+#endif
+// cycle accounting of CTA 0's MMA issuer: waits by kind, op loads, total
+__device__ unsigned long long g_prof[16];
+#define PROF_T0() (_pt0 = clock64())
+#define PROF_ADD(var) (var += clock64() - _pt0)
+#else
+#define TRACE(row, n) ((void)0)
+#define PROF_T0() ((void)0)
+#define PROF_ADD(var) ((void)0)
+#endif
 
 constexpr int kEpiWarps = 8;
 constexpr int kProdWarp = 8, kMmaWarp = 9;
@@ -415,7 +651,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   const int slot = kSlotA + d.slot_b;
   const int Cc = d.Cc;
   const int pbytes = 128 * Cc * 2;
-  uint8_t* ring = smem;
+  uint8_t* wres = smem;                    // resident weights (d.resident), else empty
+  uint8_t* ring = smem + d.wres_bytes;
   uint8_t* pbuf = ring + S * slot;
   uint8_t* ones = pbuf + 2 * pbytes;
   uint64_t* bars = reinterpret_cast<uint64_t*>(ones + 4096);
@@ -427,7 +664,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   uint64_t* p_empty = p_full + 2;
   uint64_t* out_full = p_empty + 2;
   uint64_t* out_empty = out_full + 1;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(out_empty + 1);
+  uint64_t* wbar = out_empty + 1;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wbar + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   // constant A operand of the bias MMA: K columns 0 and 1 = 1.0 (bf16), one SW32 atom
@@ -451,7 +689,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
     mbar_init(out_full, 1);
     mbar_init(out_empty, 32 * kEpiWarps);
+    mbar_init(wbar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  // per-tile programs -> SMEM
+  const TcProdOp* prod = d.prod;
+  const TcMmaOp* mprog = d.mma;
+  if (d.prog_smem) {
+    uint8_t* ps = reinterpret_cast<uint8_t*>(bars) + 2048 + (d.npc ? 32768 : 0);
+    const int n16 = (d.n_prod * (int)sizeof(TcProdOp) + d.n_mma * (int)sizeof(TcMmaOp)) / 16;
+    const uint4* src = reinterpret_cast<const uint4*>(d.prod);
+    for (int i = threadIdx.x; i < n16; i += blockDim.x) reinterpret_cast<uint4*>(ps)[i] = src[i];
+    prod = reinterpret_cast<const TcProdOp*>(ps);
+    mprog = reinterpret_cast<const TcMmaOp*>(ps + d.n_prod * sizeof(TcProdOp));
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
@@ -469,143 +719,188 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      const uint32_t bytes_f = d.Np * 128;
-      const uint32_t rows_a = d.spatial ? (uint32_t)(d.tw * d.th * d.tn) : 128u;
-      auto load_b = [&](const void* map, int x, int y) {           // bias: [Cc x 16] SW32 box
-        mbar_wait(&empty[stage], phase ^ 1);
-        mbar_expect_tx(&full[stage], Cc * 32);
-        tma_load_2d(ring + stage * slot + kSlotA, map, &full[stage], x, y);
-        if (++stage == S) stage = 0, phase ^= 1;
-      };
+      [[maybe_unused]] int n0 = 0, n1 = 0;
+      const char* dbase = reinterpret_cast<const char*>(&d);
+      if (d.resident) {
+        // every B box once: term atoms, level / member biases, F atoms
+        mbar_expect_tx(wbar, d.wres_bytes);
+        const int nall = d.npc ? d.mt1 : d.n_terms;
+        for (int j = 0; j < nall; ++j) {
+          const TcTerm& t = d.term[j];
+          const int ka_n = t.Rp / t.aw, bb = Cc * t.aw * 2;
+          for (int c = 0; c < t.nhit; ++c)
+            for (int ka = 0; ka < ka_n; ++ka)
+              tma_load_2d(wres + t.wres + (c * ka_n + ka) * bb, t.wmap, wbar, ka * t.aw, (t.cfirst + c) * Cc);
+        }
+        for (int l = 0; l < d.n_levels; ++l)
+          for (int c = 0; c < d.nchunks; ++c) tma_load_2d(wres + d.bres[l] + c * Cc * 32, d.bmap[l], wbar, 0, c * Cc);
+        for (int c = 0; c < d.npc; ++c) tma_load_2d(wres + d.bresm + c * Cc * 32, d.bmapm, wbar, 0, c * Cc);
+        if (!d.gap)
+          for (int a = 0; a < d.Cpad / 64; ++a) tma_load_2d(wres + d.fres + a * d.Np * 128, d.fmap, wbar, a * 64, 0);
+      }
+      const int np = d.n_prod;
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
         const TileGeo gg = tile_geo(d, tile);
-        for (int u0 = 0; u0 < U; u0 += 2) {
-          const int nb = min(2, U - u0);
-          for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < nb; ++bi) {
-              const Unit un = unit_at(d, u0 + bi);
-              load_b(un.pooled ? d.bmapm : d.bmap[l], 0, un.c * Cc);             // bias stage
-              const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
-              const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
-              for (int r = 0; r < un.nt; ++r)
-                for (int j = j0; j < j1; ++j) {
-                  const TcTerm& t = d.term[j];
-                  if (!un.pooled && !term_hits(t, un.c, Cc)) continue;
-                  const int ntap = un.pooled ? 1 : t.tk * t.tk;
-                  for (int q = 0; q < ntap; ++q) {
-                    const int tap = un.pooled ? un.tg * d.tpu + r : q;
-                    const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
-                    for (int ka = 0; ka < t.Rp / t.aw; ++ka) {
-                      mbar_wait(&empty[stage], phase ^ 1);
-                      mbar_expect_tx(&full[stage], (rows_a + Cc) * t.aw * 2);
-                      uint8_t* sa = ring + stage * slot;
-                      if (d.spatial)      // (tap-shifted) strided box of the term's input
-                        tma_load_4d(sa, t.tmap4, &full[stage], ka * t.aw, gg.w0 * t.ts - pad + tap % kk,
-                                    gg.h0 * t.ts - pad + tap / kk, gg.n0);
-                      else
-                        tma_load_2d(sa, t.tmap, &full[stage], ka * t.aw, gg.m0);
-                      tma_load_2d(sa + kSlotA, t.wmap, &full[stage], ka * t.aw, un.c * Cc);
-                      if (++stage == S) stage = 0, phase ^= 1;
-                    }
-                  }
-                }
-            }
-          if (!d.gap)
-            for (int bi = 0; bi < nb; ++bi) {
-              const Unit un = unit_at(d, u0 + bi);
-              if (!un.last) continue;
-              for (int a = 0; a < Cc / 64; ++a) {
-                mbar_wait(&empty[stage], phase ^ 1);
-                mbar_expect_tx(&full[stage], bytes_f);
-                tma_load_2d(ring + stage * slot + kSlotA, d.fmap, &full[stage], un.c * Cc + a * 64, 0);
-                if (++stage == S) stage = 0, phase ^= 1;
-              }
-            }
+        for (int i = 0; i < np; ++i) {
+          const TcProdOp o = prod[i];
+#ifdef TEMCO_TRACE
+          if (g_dbg) {   // TMA-only experiment: the producer recycles its own stages
+            if (n0 >= S) mbar_wait(&full[stage], phase ^ 1);
+          } else
+#endif
+          mbar_wait(&empty[stage], phase ^ 1);
+          TRACE(0, n0);
+          mbar_expect_tx(&full[stage], o.bytes);
+          uint8_t* sa = ring + stage * slot;
+          if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
+            tma_load_4d(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.w0 * o.ts + o.dx, gg.h0 * o.ts + o.dy, gg.n0);
+          else if (o.kind & PK_A2D)
+            tma_load_2d(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.m0);
+          if (o.kind & PK_B) tma_load_2d(sa + kSlotA, dbase + o.bmap * 64, &full[stage], o.bx, o.by);
+          TRACE(1, n1);
+          if (++stage == S) stage = 0, phase ^= 1;
         }
       }
+#ifdef TEMCO_TRACE
+      if (g_dbg)
+        for (int k = 0; k < S && k < n0; ++k) {
+          const int i = n0 - 1 - k;
+          mbar_wait(&full[i % S], (i / S) & 1);
+        }
+#endif
     }
   } else if (warp == kMmaWarp) {
+#ifdef TEMCO_TRACE
+    if (g_dbg) goto done;
+#endif
     // ------------------------------------------------------------ MMA issuer
-    if (lane == 0) {
+    {   // whole warp (uniform control flow); elect.sync picks the issuing lane
       int stage = 0;
       uint32_t phase = 0;
       uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
+      [[maybe_unused]] int n2 = 0, n3 = 0, n8 = 0, n9 = 0, n10 = 0, n11 = 0;
       const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
       const uint32_t tout = tbase + 2 * d.ubuf;
       const uint32_t ones_addr = smem_u32(ones);
-      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        for (int u0 = 0; u0 < U; u0 += 2) {
-          const int nb = min(2, U - u0);
-          for (int l = 0; l < d.n_levels; ++l)
-            for (int bi = 0; bi < nb; ++bi) {
-              const Unit un = unit_at(d, u0 + bi);
-              const uint32_t abit = 1u << bi;
-              mbar_wait(&acc_empty[bi], ((acc_par & abit) ? 1u : 0u) ^ 1u);
-              tc_fence_after();
-              const uint32_t tacc = tbase + bi * d.ubuf;
-              // bias (initialises every tap region of the accumulator at level 0)
-              mbar_wait(&full[stage], phase);
-              tc_fence_after();
-              for (int r = 0; r < un.nt; ++r)
-                mma_bf16(tacc + r * Cc, umma_desc_k(ones_addr, 16), umma_desc_k(smem_u32(ring + stage * slot + kSlotA), 16), id1,
-                         l == 0 ? 0u : 1u);
-              mma_commit(&empty[stage]);
-              if (++stage == S) stage = 0, phase ^= 1;
-              const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
-              const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
-              for (int r = 0; r < un.nt; ++r)
-                for (int j = j0; j < j1; ++j) {
-                  const TcTerm& t = d.term[j];
-                  if (!un.pooled && !term_hits(t, un.c, Cc)) continue;
-                  const int ntap = un.pooled ? 1 : t.tk * t.tk;
-                  for (int q = 0; q < ntap; ++q)
-                    for (int ka = 0; ka < t.Rp / t.aw; ++ka) {
-                      mbar_wait(&full[stage], phase);
-                      tc_fence_after();
-                      const uint32_t sa = smem_u32(ring + stage * slot);
-                      const int nk = min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
-                      for (int k = 0; k < nk; ++k)
-                        mma_bf16(tacc + r * Cc, umma_desc_k(sa + 32 * k, t.aw), umma_desc_k(sa + kSlotA + 32 * k, t.aw),
-                                 id1, 1u);
-                      mma_commit(&empty[stage]);
-                      if (++stage == S) stage = 0, phase ^= 1;
-                    }
-                }
-              mma_commit(&acc_full[bi]);
-              acc_par ^= abit;
-            }
-          if (!d.gap)
-            for (int bi = 0; bi < nb; ++bi) {
-              const Unit un = unit_at(d, u0 + bi);
-              if (!un.last) continue;
-              const int pb = un.c & 1;
-              const uint32_t pbit = 1u << pb;
-              mbar_wait(&p_full[pb], (p_par & pbit) ? 1u : 0u);
-              tc_fence_after();
-              if (un.c == 0) {
-                mbar_wait(out_empty, (tile_iter & 1) ^ 1);
-                tc_fence_after();
-              }
-              const uint32_t pa = smem_u32(pbuf + pb * pbytes);
-              for (int a = 0; a < Cc / 64; ++a) {
-                mbar_wait(&full[stage], phase);
-                tc_fence_after();
-                const uint32_t sb = smem_u32(ring + stage * slot + kSlotA);
-                for (int k = 0; k < 4; ++k)
-                  mma_bf16(tout, umma_desc(pa + a * 16384 + 32 * k), umma_desc(sb + 32 * k), id2,
-                           (un.c > 0 || a > 0 || k > 0) ? 1u : 0u);
-                mma_commit(&empty[stage]);
-                if (++stage == S) stage = 0, phase ^= 1;
-              }
-              mma_commit(&p_empty[pb]);
-              p_par ^= pbit;
-            }
+      const uint32_t wres_addr = smem_u32(wres);
+      const uint32_t ring_addr = smem_u32(ring);
+      const uint32_t pbuf_addr = smem_u32(pbuf);
+      if (d.resident) mbar_wait(wbar, 0);
+      const int nm = d.n_mma;
+#ifdef TEMCO_TRACE
+      long long pc_acc = 0, pc_p = 0, pc_out = 0, pc_full = 0, pc_issue = 0, pc_n = 0, pc_dec = 0, pc_com = 0;
+      const long long pc_start = clock64();
+#endif
+      auto exec = [&](const TcMmaOp o, int gu, uint32_t tile_iter) {
+#ifdef TEMCO_TRACE
+          long long _pt0 = 0;
+#endif
+          const uint32_t f = o.flags;
+          const int bs = (gu + o.unit) & 1;
+          if (f & MF_ACC_WAIT) {
+            PROF_T0();
+            mbar_wait(&acc_empty[bs], ((acc_par >> bs) & 1u) ^ 1u);
+            PROF_ADD(pc_acc);
+            TRACE(8, n8);
+            tc_fence_after();
+          }
+          if (f & MF_P_WAIT) {
+            TRACE(9, n9);
+            PROF_T0();
+            mbar_wait(&p_full[o.unit], (p_par >> o.unit) & 1u);
+            PROF_ADD(pc_p);
+            TRACE(10, n10);
+            tc_fence_after();
+          }
+          if (f & MF_OUT_WAIT) {
+            PROF_T0();
+            mbar_wait(out_empty, (tile_iter & 1) ^ 1);
+            PROF_ADD(pc_out);
+            tc_fence_after();
+          }
+          if (f & MF_SW) {
+            PROF_T0();
+            mbar_wait(&full[stage], phase);
+            PROF_ADD(pc_full);
+            TRACE(2, n2);
+            tc_fence_after();
+          }
+          PROF_T0();
+          const uint32_t st = ring_addr + stage * slot;
+          const uint32_t a = (f & MF_ONES) ? ones_addr : (f & MF_F) ? pbuf_addr + o.aoff : st;
+          const uint32_t b = (f & MF_BRES) ? wres_addr + o.boff : st + kSlotA;
+          const uint64_t ad = umma_desc_k(a, o.la), bd = umma_desc_k(b, o.lb);
+          const uint32_t dt = (f & MF_F) ? tout : tbase + bs * d.ubuf + o.tcol;
+          const uint32_t id = (f & MF_F) ? id2 : id1;
+          const uint32_t acc0 = (f & MF_ZERO) ? 0u : 1u;
+          PROF_ADD(pc_dec);
+          {
+          PROF_T0();
+          for (int k = 0; k < o.nk; ++k) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, id, k ? 1u : acc0);
+          PROF_ADD(pc_issue);
+#ifdef TEMCO_TRACE
+          pc_n += o.nk;
+#endif
+          }
+          PROF_T0();
+          if (f & MF_SD) {
+            mma_commit_w(&empty[stage]);
+            if (++stage == S) stage = 0, phase ^= 1;
+          }
+          if (f & MF_ACC_COMMIT) {
+            mma_commit_w(&acc_full[bs]);
+            TRACE(3, n3);
+            acc_par ^= 1u << bs;
+          }
+          if (f & MF_P_COMMIT) {
+            mma_commit_w(&p_empty[o.unit]);
+            p_par ^= 1u << o.unit;
+          }
+          if (f & MF_OUT_COMMIT) {
+            mma_commit_w(out_full);
+            TRACE(11, n11);
+          }
+          PROF_ADD(pc_com);
+      };
+      if (d.mma_head > 0) {
+        // software pipeline over tiles: the unit ops of tile t+1 go ahead of the
+        // fconv ops of tile t (which wait for the epilogue's P tile of t)
+        const int nh = d.mma_head;
+        int t = blockIdx.x, gu = 0;
+        for (int i = 0; i < nh && t < d.ntiles; ++i) exec(mprog[i], gu, tile_iter);
+        for (; t < d.ntiles; t += gridDim.x) {
+          if (t + (int)gridDim.x < d.ntiles)
+            for (int i = 0; i < nh; ++i) exec(mprog[i], gu + d.units, tile_iter + 1);
+          for (int i = nh; i < nm; ++i) exec(mprog[i], gu, tile_iter);
+          gu += d.units;
+          ++tile_iter;
         }
-        if (!d.gap) mma_commit(out_full);
-        ++tile_iter;
+      } else {
+        int gu = 0;   // units issued so far (TMEM buffer parity)
+        for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+          for (int i = 0; i < nm; ++i) exec(mprog[i], gu, tile_iter);
+          gu += d.units;
+          ++tile_iter;
+        }
       }
+#ifdef TEMCO_TRACE
+      if (blockIdx.x == 0 && lane == 0) {
+        g_prof[0] = clock64() - pc_start;
+        g_prof[1] = pc_acc;
+        g_prof[2] = pc_p;
+        g_prof[3] = pc_out;
+        g_prof[4] = pc_full;
+        g_prof[5] = pc_issue;
+        g_prof[6] = pc_n;
+        g_prof[7] = pc_dec;
+        g_prof[8] = pc_com;
+      }
+#endif
     }
   } else if (warp < kEpiWarps) {
+#ifdef TEMCO_TRACE
+    if (g_dbg) goto done;
+#endif
     // ------------------------------------------------------------ epilogue (8 warps)
     // warp w: TMEM lane quarter q = w % 4 (pixel rows 32q..32q+31), column half h = w / 4
     const int q = warp & 3, h = warp >> 2;
@@ -614,8 +909,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     const int half = Cc / 2;                          // columns per warp (32 or 64)
     const int c_lo = h * half;
     uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
+    [[maybe_unused]] int n4 = 0, n5 = 0, n6 = 0, n7 = 0;
+    const bool tr = threadIdx.x == 0;
+    (void)tr;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
     float* runbuf = reinterpret_cast<float*>(bars + 64);   // pooled member running max / sum (32 KB)
+    int gu = 0;   // units consumed so far (TMEM buffer parity)
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
       int64_t m = (int64_t)tile * d.rows_per_tile + row;
       bool mvalid = m < d.npix;
@@ -630,15 +929,17 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
         mvalid = row < d.mused && n < d.nimg && ho < d.Ho && wo < d.Wo;
         m = ((int64_t)n * d.Ho + ho) * d.Wo + wo;
       }
-      for (int u0 = 0; u0 < U; u0 += 2) {
+      for (int u0 = 0; u0 < U; gu += min(2, U - u0), u0 += 2) {
         const int nb = min(2, U - u0);
         for (int l = 0; l < d.n_levels; ++l) {
           const bool last = l == d.n_levels - 1;
           const bool relu = d.relu[l] != 0;
           for (int bi = 0; bi < nb; ++bi) {
             const Unit un = unit_at(d, u0 + bi);
-            const uint32_t abit = 1u << bi;
-            mbar_wait(&acc_full[bi], (acc_par & abit) ? 1u : 0u);
+            const int bs = (gu + bi) & 1;
+            const uint32_t abit = 1u << bs;
+            mbar_wait(&acc_full[bs], (acc_par & abit) ? 1u : 0u);
+            if (tr) TRACE(4, n4);
             acc_par ^= abit;
             tc_fence_after();
             const int pb = un.c & 1;
@@ -648,7 +949,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               mbar_wait(&p_empty[pb], ((p_par & pbit) ? 1u : 0u) ^ 1u);
               p_par ^= pbit;
             }
-            const uint32_t ta = tbase + lane_off + bi * d.ubuf + c_lo;
+            const uint32_t ta = tbase + lane_off + bs * d.ubuf + c_lo;
             uint8_t* P = pbuf + pb * pbytes;
             if (un.pooled) {
               // pooled member: fold the unit's taps into the running max / sum (half == 32),
@@ -773,7 +1074,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               }
             }
             tc_fence_before();
-            mbar_arrive(&acc_empty[bi]);
+            if (tr) TRACE(5, n5);
+            mbar_arrive(&acc_empty[bs]);
             if (writes_p) {
               fence_proxy_async();
               mbar_arrive(&p_full[pb]);
@@ -783,7 +1085,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       }
       if (d.gap) continue;
       // output epilogue: column groups of 8 split between the two warp halves
+      if (tr) TRACE(6, n6);
       mbar_wait(out_full, tile_iter & 1);
+      if (tr) TRACE(7, n7);
       ++tile_iter;
       tc_fence_after();
       const int ng = d.Np / 8, gh = (ng + 1) / 2;
@@ -804,6 +1108,9 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       mbar_arrive(out_empty);
     }
   }
+#ifdef TEMCO_TRACE
+done:
+#endif
   tc_fence_before();
   __syncthreads();
   if (warp == 0) {
@@ -813,6 +1120,17 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 }
 
 }  // namespace
+
+#ifdef TEMCO_TRACE
+extern "C" void temco_debug_prof(long long* out) { cudaMemcpyFromSymbol(out, g_prof, sizeof(g_prof)); }
+extern "C" void temco_debug_set(int dbg) { cudaMemcpyToSymbol(g_dbg, &dbg, sizeof(int)); }
+extern "C" void temco_debug_trace(long long* out) {
+  cudaMemcpyFromSymbol(out, g_trace, sizeof(g_trace));
+  void* p = nullptr;
+  cudaGetSymbolAddress(&p, g_trace);
+  cudaMemset(p, 0, sizeof(g_trace));
+}
+#endif
 
 void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   (void)tcw;

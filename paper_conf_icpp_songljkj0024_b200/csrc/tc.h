@@ -39,7 +39,48 @@ struct TcTerm {
   int32_t Hin, Win;      // resolution of r
   int32_t tk, ts, tp;    // tap-accumulate window (1 = plain term)
   int64_t w;             // tc weight pool offset (elements)
+  int32_t cfirst, nhit;  // chunks [cfirst, cfirst + nhit) receive this term
+  int32_t wres;          // resident mode: byte offset of [nhit][Rp/aw] boxes (Cc x aw) in the weight region
 };
+
+// Per-tile programs (host-generated, identical for every tile of a group): the
+// producer and MMA roles replay flat op lists instead of re-deriving the unit /
+// level / term / tap / K-atom loop nest per stage (a single issuing thread is
+// latency-bound on that scalar code).
+enum : uint8_t { PK_A4D = 1, PK_A2D = 2, PK_B = 4 };
+struct TcProdOp {                 // one ring stage
+  uint8_t kind, ts;               // PK_*; tile-base stride of a 4D A box
+  uint16_t amap, bmap;            // byte offsets / 64 of the CUtensorMaps inside TcChainDesc
+  int16_t ac, dx, dy;             // A coords: channel; tap offsets (4D: w0*ts+dx, h0*ts+dy)
+  int16_t bx, by;                 // B coords
+  uint16_t bytes;                 // expect_tx
+  uint16_t pad[7];
+};
+static_assert(sizeof(TcProdOp) == 32, "TcProdOp layout");
+enum : uint16_t {
+  MF_ACC_WAIT = 1,      // wait acc_empty[bs] first
+  MF_P_WAIT = 2,        // wait p_full[unit]
+  MF_OUT_WAIT = 4,      // wait out_empty
+  MF_SW = 8,            // wait full[stage]
+  MF_SA = 16,           // A operand = current stage slot A
+  MF_SB = 32,           // B operand = current stage slot B
+  MF_SD = 64,           // commit empty[stage] + advance after
+  MF_ONES = 128,        // A = constant ones tile (bias MMA)
+  MF_F = 256,           // fconv MMA: A = P[unit] + aoff, D = output region, N = Np
+  MF_ZERO = 512,        // first MMA of the accumulator (k == 0 does not accumulate)
+  MF_ACC_COMMIT = 1024, // commit acc_full[bs] after
+  MF_P_COMMIT = 2048,   // commit p_empty[unit] after
+  MF_OUT_COMMIT = 4096, // commit out_full after
+  MF_BRES = 8192,       // B = resident weights + boff
+};
+struct TcMmaOp {
+  uint16_t flags;
+  uint8_t unit, nk;               // unit index in the tile (TMEM buffer parity) or P buffer; K=16 steps
+  uint8_t la, lb;                 // K-atom widths (layouts) of A and B
+  uint16_t tcol;                  // TMEM column offset inside the unit buffer
+  uint32_t aoff, boff;
+};
+static_assert(sizeof(TcMmaOp) == 16, "TcMmaOp layout");
 
 struct TcChainDesc {
   TcTerm term[kTcMaxTerms];
@@ -71,6 +112,18 @@ struct TcChainDesc {
   int64_t F;                             // tc weight pool offset of F
   int64_t Fb;                            // unused (fconv factors carry no bias)
   Loc y;                                 // output [npix, Nout] bf16, or [N, C] for GAP
+  // resident weights (every B operand fits in SMEM): loaded once per CTA, the
+  // ring then carries only A tiles.  Avoids all 148 SMs re-reading the same
+  // few weight lines through TMA every stage (L2 same-line contention).
+  int32_t resident, wres_bytes;
+  int32_t bres[kTcMaxLevels], bresm;     // bias boxes: [nchunks] x (Cc x 16), byte offsets
+  int32_t fres;                          // F boxes: [Cpad / 64] x (Np x 64)
+  int64_t prog_off;                      // tc weight pool offset (elements) of [prod ops][mma ops]
+  int32_t n_prod, n_mma, units;          // ops per tile; units per tile
+  int32_t mma_head;                      // > 0: pipelined MMA order, unit ops = mma[0, mma_head)
+  int32_t prog_smem;                     // > 0: programs copied to SMEM at kernel start (bytes reserved)
+  const TcProdOp* prod;                  // device pointers (tc_finalize)
+  const TcMmaOp* mma;
   int32_t stages, slot_a, slot_b;        // smem ring depth, bytes of one A / B slot
   int32_t smem_bytes, tmem_cols;
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
