@@ -256,6 +256,12 @@ def main():
     else:
         achieved, peak, unit, bound = c["bytes"] / (c["ms"] * 1e-3) / 1e9, hbm, "GB/s", "hbm"
     total_ms = float(prof.sum())
+    # DRAM traffic of the dominant class from the committed ncu capture of this
+    # config (scripts/launch_summary.py --json), bytes per step like `achieved`
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    if os.path.exists(tpath):
+        traffic = json.load(open(tpath)).get(dom)
 
     if rank == 0:
         line = {
@@ -274,7 +280,9 @@ def main():
                     "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
                     "d2h_bytes_per_step": int(yh.numel() * yh.element_size())},
             "roofline": {"bound": bound, "kernel": dom, "achieved": achieved, "peak": peak, "unit": unit,
-                         "frac": achieved / peak, "traffic": None, "peak_source": src,
+                         "frac": achieved / peak, "traffic": traffic,
+                         "traffic_note": "DRAM read+write bytes per step of the class (ncu, cold L2), from "
+                                         "profiles/traffic_<config>.json", "peak_source": src,
                          "launches_per_step": c["launches"], "share_of_step": c["ms"] / total_ms,
                          "alg_flops_per_step": c["flops"], "alg_bytes_per_step": c["bytes"]},
             "kernel_classes_ms": {k: round(v["ms"], 4) for k, v in sorted(classes.items(), key=lambda kv: -kv[1]["ms"])},
