@@ -428,7 +428,7 @@ std::string make_json(const temco_plan_s* P) {
       if (e.kind == K_GROUP_TC)
         o << ",\"alg_flops\":" << e.tc.alg_flops << ",\"alg_bytes\":" << e.tc.alg_bytes << ",\"tc\":{\"n_prod\":"
           << e.tc.n_prod << ",\"n_mma\":" << e.tc.n_mma << ",\"units\":" << e.tc.units << ",\"stages\":" << e.tc.stages
-          << ",\"resident\":" << e.tc.resident << ",\"pipelined\":" << (e.tc.mma_head > 0) << ",\"ntiles\":"
+          << ",\"resident\":" << e.tc.resident << ",\"smem\":" << e.tc.smem_bytes << ",\"tmem\":" << e.tc.tmem_cols << ",\"pipelined\":" << (e.tc.mma_head > 0) << ",\"ntiles\":"
           << e.tc.ntiles << ",\"Cc\":" << e.tc.Cc << ",\"levels\":" << e.tc.n_levels << "}";
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;

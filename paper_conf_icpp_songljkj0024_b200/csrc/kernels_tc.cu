@@ -60,6 +60,14 @@ int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
   return off;
 }
 
+// fp32 vector padded with zeros to n entries, 16-byte aligned in the params pool
+int64_t push_f32(std::vector<float>& params, const std::vector<double>& v, int n) {
+  while (params.size() % 4) params.push_back(0.f);
+  const int64_t off = (int64_t)params.size();
+  for (int i = 0; i < n; ++i) params.push_back(i < (int)v.size() ? (float)v[i] : 0.f);
+  return off;
+}
+
 // bias as a rank-2 term: columns 0, 1 = bf16 hi / lo parts (error ~2^-16 |b|)
 int64_t push_bias(std::vector<uint16_t>& pool, const std::vector<double>& b, int c0, int Cpad) {
   std::vector<float> bm((size_t)Cpad * 8, 0.f);
@@ -115,32 +123,10 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
       for (int bi = 0; bi < nb; ++bi) {
         const int u = u0 + bi;
         const HUnit un = unit_at(u);
-        // bias: initialises (level 0) every tap region of the accumulator
-        if (!res) {
-          TcProdOp o{};
-          o.kind = PK_B;
-          o.bmap = moff(un.pooled ? d.bmapm : d.bmap[l]);
-          o.bx = 0;
-          o.by = (int16_t)(un.c * Cc);
-          o.bytes = (uint16_t)(Cc * 32);
-          P.push_back(o);
-        }
-        for (int r = 0; r < un.nt; ++r) {
-          TcMmaOp m{};
-          m.flags = MF_ONES | (l == 0 ? MF_ZERO : 0) | (r == 0 ? MF_ACC_WAIT : 0);
-          if (res) {
-            m.flags |= MF_BRES;
-            m.boff = (uint32_t)((un.pooled ? d.bresm : d.bres[l]) + un.c * Cc * 32);
-          } else {
-            m.flags |= MF_SB | (r == 0 ? MF_SW : 0) | (r == un.nt - 1 ? MF_SD : 0);
-          }
-          m.unit = (uint8_t)u;
-          m.nk = 1;
-          m.la = 16;
-          m.lb = 16;
-          m.tcol = (uint16_t)(r * Cc);
-          M.push_back(m);
-        }
+        // level biases are added by the epilogue: the first MMA into each tap region
+        // at level 0 overwrites (MF_ZERO); a region no term reaches gets a zero-init MMA
+        const size_t m_first = M.size();
+        std::vector<char> region_done(un.nt, 0);
         const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
         const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
         for (int r = 0; r < un.nt; ++r)
@@ -170,6 +156,8 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
                 P.push_back(o);
                 TcMmaOp m{};
                 m.flags = MF_SW | MF_SA | MF_SD | (res ? MF_BRES : MF_SB);
+                if (l == 0 && !region_done[r]) m.flags |= MF_ZERO;
+                region_done[r] = 1;
                 m.unit = (uint8_t)u;
                 m.nk = (uint8_t)std::min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
                 m.la = (uint8_t)t.aw;
@@ -180,6 +168,18 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
               }
             }
           }
+        for (int r = 0; r < un.nt; ++r)
+          if (l == 0 && !region_done[r]) {   // zero-init: ones tile x zero tile
+            TcMmaOp m{};
+            m.flags = MF_ONES | MF_BZERO | MF_ZERO;
+            m.unit = (uint8_t)u;
+            m.nk = 1;
+            m.la = 16;
+            m.lb = 16;
+            m.tcol = (uint16_t)(r * Cc);
+            M.push_back(m);
+          }
+        M[m_first].flags |= MF_ACC_WAIT;
         M.back().flags |= MF_ACC_COMMIT;
       }
     if (!d.gap)
@@ -215,7 +215,7 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
   d.n_prod = (int32_t)P.size();
   d.n_mma = (int32_t)M.size();
   // programs live in SMEM (after the pooled slab) when they fit next to the ring
-  const int pbytes_prog = (int)(P.size() * sizeof(TcProdOp) + M.size() * sizeof(TcMmaOp));
+  const int pbytes_prog = (int)(P.size() * sizeof(TcProdOp) + M.size() * sizeof(TcMmaOpD));
   d.prog_smem = 0;
   const char* exp_env = getenv("TEMCO_TC_EXP");   // experiment switches (bit 0: programs in global memory)
   const int exp_bits = exp_env ? atoi(exp_env) : 0;
@@ -242,12 +242,40 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
     if (tail_f && h > 0 && h < (int)M.size()) d.mma_head = h;
   }
   while (tcw.size() % 512) tcw.push_back(0);
+  // device MMA ops: descriptors relative to the aligned SMEM base (final layout)
+  const int slot = d.slot_a + d.slot_b;
+  const uint32_t ring_off = (uint32_t)d.wres_bytes;
+  const uint32_t pbuf_off = ring_off + (uint32_t)(d.stages * slot);
+  const uint32_t ones_off = pbuf_off + 2u * (uint32_t)pbytes;
+  auto dtmpl = [](uint32_t off, int aw) {
+    const uint64_t layout = aw == 64 ? 2 : aw == 32 ? 4 : 6;
+    return (uint64_t)(off >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(16 * aw >> 4) << 32) | ((uint64_t)1 << 46) |
+           (layout << 61);
+  };
+  auto idesc = [](int M_, int N_) {
+    return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N_ >> 3) << 17) | ((uint32_t)(M_ >> 4) << 24);
+  };
+  std::vector<TcMmaOpD> MD(M.size());
+  for (size_t i = 0; i < M.size(); ++i) {
+    const TcMmaOp& m = M[i];
+    TcMmaOpD& o = MD[i];
+    const bool isF = m.flags & MF_F;
+    const uint32_t aoff = (m.flags & MF_ONES) ? ones_off : isF ? pbuf_off + m.aoff : ring_off;
+    const uint32_t boff = (m.flags & MF_BZERO) ? ones_off + 4096u : (m.flags & MF_BRES) ? m.boff : ring_off + (uint32_t)d.slot_a;
+    o.adesc = dtmpl(aoff, m.la);
+    o.bdesc = dtmpl(boff, m.lb);
+    o.idesc = isF ? idesc(128, d.Np) : idesc(128, Cc);
+    o.tmem = isF ? (uint32_t)(2 * d.ubuf) : m.tcol;
+    o.flags = m.flags;
+    o.unit = m.unit;
+    o.nk = m.nk;
+  }
   d.prog_off = (int64_t)tcw.size();
-  const size_t nbytes = P.size() * sizeof(TcProdOp) + M.size() * sizeof(TcMmaOp);
+  const size_t nbytes = P.size() * sizeof(TcProdOp) + MD.size() * sizeof(TcMmaOpD);
   tcw.resize(tcw.size() + (nbytes + 1) / 2);
   char* dst = reinterpret_cast<char*>(tcw.data() + d.prog_off);
   memcpy(dst, P.data(), P.size() * sizeof(TcProdOp));
-  memcpy(dst + P.size() * sizeof(TcProdOp), M.data(), M.size() * sizeof(TcMmaOp));
+  memcpy(dst + P.size() * sizeof(TcProdOp), MD.data(), MD.size() * sizeof(TcMmaOpD));
 }
 
 }  // namespace
@@ -388,6 +416,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
       for (double x : post) params.push_back((float)x);
     }
     d.boff[l] = push_bias(tcw, lb, 0, d.Cpad);
+    d.lbias[l] = push_f32(params, lb, d.Cpad);
     for (const PTerm& t : L.terms)
       if (!add_term(t)) return false;
     d.lvl_end[l] = j;
@@ -413,6 +442,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.mt1 = j;
     // the member is evaluated once per tap: count its work at the taps actually run
     d.boffm = push_bias(tcw, pm->bias, 0, d.Cpad);
+    d.mbias = push_f32(params, pm->bias, d.Cpad);
     if (d.tw * d.ms > 256 || d.th * d.ms > 256) return false;
   }
   d.F = 0;
@@ -449,7 +479,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d.slot_b = (sb + 1023) / 1024 * 1024;
   const int pbytes = 128 * d.Cc * 2;
   const int runbytes = pm ? 32768 : 0;     // pooled member: running max / sum slab (after the barriers)
-  const int budget = 227 * 1024 - 1024 /*align*/ - 2048 /*barriers*/ - runbytes - 2 * pbytes - 4096 /*ones*/;
+  const int budget = 227 * 1024 - 1024 /*align*/ - 2048 /*barriers*/ - runbytes - 2 * pbytes - 8192 /*ones, zeros*/;
   // resident weights: every B box (term atoms of the chunks a term reaches, level
   // and member biases, F atoms) once per CTA, if that leaves a ring of >= 6 A slots
   int64_t woff = 0;
@@ -458,12 +488,6 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     T.wres = (int32_t)woff;
     woff += (int64_t)T.nhit * (T.Rp / T.aw) * d.Cc * T.aw * 2;
   }
-  for (int l = 0; l < d.n_levels; ++l) {
-    d.bres[l] = (int32_t)woff;
-    woff += (int64_t)d.nchunks * d.Cc * 32;
-  }
-  d.bresm = (int32_t)woff;
-  woff += (int64_t)d.npc * d.Cc * 32;
   d.fres = (int32_t)woff;
   if (!gap) woff += (int64_t)(d.Cpad / 64) * d.Np * 128;
   d.resident = woff + 6LL * d.slot_a <= budget ? 1 : 0;
@@ -476,7 +500,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.stages = std::min(24, budget / (d.slot_a + d.slot_b));
   }
   if (d.stages < 2) return false;
-  d.smem_bytes = 1024 + d.wres_bytes + d.stages * (d.slot_a + d.slot_b) + 2 * pbytes + 4096 + 2048 + runbytes;
+  d.smem_bytes = 1024 + d.wres_bytes + d.stages * (d.slot_a + d.slot_b) + 2 * pbytes + 8192 + 2048 + runbytes;
   const int cols = 2 * d.ubuf + d.Np;
   d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
   if (cols > 512) return false;
@@ -526,7 +550,7 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
     TcChainDesc* d = get(i);
     if (!d) continue;
     d->prod = reinterpret_cast<const TcProdOp*>(tcw + d->prog_off);
-    d->mma = reinterpret_cast<const TcMmaOp*>(reinterpret_cast<const char*>(d->prod) + d->n_prod * sizeof(TcProdOp));
+    d->mma = reinterpret_cast<const TcMmaOpD*>(reinterpret_cast<const char*>(d->prod) + d->n_prod * sizeof(TcProdOp));
     const int nt = d->npc ? d->mt1 : d->n_terms;
     for (int j = 0; j < nt; ++j) {
       TcTerm& t = d->term[j];
@@ -595,6 +619,19 @@ __device__ unsigned long long g_prof[16];
 #define PROF_ADD(var) ((void)0)
 #endif
 
+// 32 consecutive fp32 values (16-byte aligned) -> registers
+__device__ __forceinline__ void load_bias32(const float* src, float (&b)[32]) {
+  const float4* s4 = reinterpret_cast<const float4*>(src);
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const float4 v = __ldg(s4 + i);
+    b[4 * i] = v.x;
+    b[4 * i + 1] = v.y;
+    b[4 * i + 2] = v.z;
+    b[4 * i + 3] = v.w;
+  }
+}
+
 constexpr int kEpiWarps = 8;
 constexpr int kProdWarp = 8, kMmaWarp = 9;
 constexpr int kThreads = 32 * 10;
@@ -655,7 +692,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   uint8_t* ring = smem + d.wres_bytes;
   uint8_t* pbuf = ring + S * slot;
   uint8_t* ones = pbuf + 2 * pbytes;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(ones + 4096);
+  uint8_t* zeros = ones + 4096;            // zero B tile (zero-init MMA of a region no term reaches)
+  uint64_t* bars = reinterpret_cast<uint64_t*>(zeros + 4096);
   uint64_t* full = bars;
   uint64_t* empty = bars + S;
   uint64_t* acc_full = bars + 2 * S;
@@ -675,6 +713,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     if (ch == swz_chunk(row, 0, 16)) v.x = 0x3F803F80u;   // logical chunk 0 of this row
     reinterpret_cast<uint4*>(ones)[i] = v;
   }
+  for (int i = threadIdx.x; i < 4096 / 16; i += blockDim.x) reinterpret_cast<uint4*>(zeros)[i] = make_uint4(0, 0, 0, 0);
   fence_proxy_async();
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
@@ -694,14 +733,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   }
   // per-tile programs -> SMEM
   const TcProdOp* prod = d.prod;
-  const TcMmaOp* mprog = d.mma;
+  const TcMmaOpD* mprog = d.mma;
   if (d.prog_smem) {
     uint8_t* ps = reinterpret_cast<uint8_t*>(bars) + 2048 + (d.npc ? 32768 : 0);
-    const int n16 = (d.n_prod * (int)sizeof(TcProdOp) + d.n_mma * (int)sizeof(TcMmaOp)) / 16;
+    const int n16 = (d.n_prod * (int)sizeof(TcProdOp) + d.n_mma * (int)sizeof(TcMmaOpD)) / 16;
     const uint4* src = reinterpret_cast<const uint4*>(d.prod);
     for (int i = threadIdx.x; i < n16; i += blockDim.x) reinterpret_cast<uint4*>(ps)[i] = src[i];
     prod = reinterpret_cast<const TcProdOp*>(ps);
-    mprog = reinterpret_cast<const TcMmaOp*>(ps + d.n_prod * sizeof(TcProdOp));
+    mprog = reinterpret_cast<const TcMmaOpD*>(ps + d.n_prod * sizeof(TcProdOp));
   }
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
@@ -716,12 +755,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 
   if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer
-    if (lane == 0) {
+    {   // whole warp; one elected lane issues (the resident preload runs in lane 0)
       int stage = 0;
       uint32_t phase = 0;
       [[maybe_unused]] int n0 = 0, n1 = 0;
       const char* dbase = reinterpret_cast<const char*>(&d);
-      if (d.resident) {
+      if (d.resident && lane == 0) {
         // every B box once: term atoms, level / member biases, F atoms
         mbar_expect_tx(wbar, d.wres_bytes);
         const int nall = d.npc ? d.mt1 : d.n_terms;
@@ -732,37 +771,35 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
             for (int ka = 0; ka < ka_n; ++ka)
               tma_load_2d(wres + t.wres + (c * ka_n + ka) * bb, t.wmap, wbar, ka * t.aw, (t.cfirst + c) * Cc);
         }
-        for (int l = 0; l < d.n_levels; ++l)
-          for (int c = 0; c < d.nchunks; ++c) tma_load_2d(wres + d.bres[l] + c * Cc * 32, d.bmap[l], wbar, 0, c * Cc);
-        for (int c = 0; c < d.npc; ++c) tma_load_2d(wres + d.bresm + c * Cc * 32, d.bmapm, wbar, 0, c * Cc);
         if (!d.gap)
           for (int a = 0; a < d.Cpad / 64; ++a) tma_load_2d(wres + d.fres + a * d.Np * 128, d.fmap, wbar, a * 64, 0);
       }
+      __syncwarp();
       const int np = d.n_prod;
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
         const TileGeo gg = tile_geo(d, tile);
         for (int i = 0; i < np; ++i) {
           const TcProdOp o = prod[i];
 #ifdef TEMCO_TRACE
-          if (g_dbg) {   // TMA-only experiment: the producer recycles its own stages
+          if (g_dbg & 1) {   // TMA-only experiment: the producer recycles its own stages
             if (n0 >= S) mbar_wait(&full[stage], phase ^ 1);
           } else
 #endif
           mbar_wait(&empty[stage], phase ^ 1);
           TRACE(0, n0);
-          mbar_expect_tx(&full[stage], o.bytes);
+          mbar_expect_tx_w(&full[stage], o.bytes);
           uint8_t* sa = ring + stage * slot;
           if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
-            tma_load_4d(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.w0 * o.ts + o.dx, gg.h0 * o.ts + o.dy, gg.n0);
+            tma_load_4d_w(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.w0 * o.ts + o.dx, gg.h0 * o.ts + o.dy, gg.n0);
           else if (o.kind & PK_A2D)
-            tma_load_2d(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.m0);
-          if (o.kind & PK_B) tma_load_2d(sa + kSlotA, dbase + o.bmap * 64, &full[stage], o.bx, o.by);
+            tma_load_2d_w(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.m0);
+          if (o.kind & PK_B) tma_load_2d_w(sa + kSlotA, dbase + o.bmap * 64, &full[stage], o.bx, o.by);
           TRACE(1, n1);
           if (++stage == S) stage = 0, phase ^= 1;
         }
       }
 #ifdef TEMCO_TRACE
-      if (g_dbg)
+      if ((g_dbg & 1) && lane == 0)
         for (int k = 0; k < S && k < n0; ++k) {
           const int i = n0 - 1 - k;
           mbar_wait(&full[i % S], (i / S) & 1);
@@ -771,7 +808,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
   } else if (warp == kMmaWarp) {
 #ifdef TEMCO_TRACE
-    if (g_dbg) goto done;
+    if (g_dbg & 1) goto done;
 #endif
     // ------------------------------------------------------------ MMA issuer
     {   // whole warp (uniform control flow); elect.sync picks the issuing lane
@@ -779,19 +816,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       uint32_t phase = 0;
       uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
       [[maybe_unused]] int n2 = 0, n3 = 0, n8 = 0, n9 = 0, n10 = 0, n11 = 0;
-      const uint32_t id1 = idesc_bf16(128, Cc), id2 = idesc_bf16(128, d.Np);
-      const uint32_t tout = tbase + 2 * d.ubuf;
-      const uint32_t ones_addr = smem_u32(ones);
-      const uint32_t wres_addr = smem_u32(wres);
-      const uint32_t ring_addr = smem_u32(ring);
-      const uint32_t pbuf_addr = smem_u32(pbuf);
       if (d.resident) mbar_wait(wbar, 0);
       const int nm = d.n_mma;
 #ifdef TEMCO_TRACE
       long long pc_acc = 0, pc_p = 0, pc_out = 0, pc_full = 0, pc_issue = 0, pc_n = 0, pc_dec = 0, pc_com = 0;
       const long long pc_start = clock64();
 #endif
-      auto exec = [&](const TcMmaOp o, int gu, uint32_t tile_iter) {
+      const uint64_t base16 = smem_u32(smem) >> 4;
+      auto exec = [&](const TcMmaOpD& o, int gu, uint32_t tile_iter) {
 #ifdef TEMCO_TRACE
           long long _pt0 = 0;
 #endif
@@ -826,17 +858,16 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
             tc_fence_after();
           }
           PROF_T0();
-          const uint32_t st = ring_addr + stage * slot;
-          const uint32_t a = (f & MF_ONES) ? ones_addr : (f & MF_F) ? pbuf_addr + o.aoff : st;
-          const uint32_t b = (f & MF_BRES) ? wres_addr + o.boff : st + kSlotA;
-          const uint64_t ad = umma_desc_k(a, o.la), bd = umma_desc_k(b, o.lb);
-          const uint32_t dt = (f & MF_F) ? tout : tbase + bs * d.ubuf + o.tcol;
-          const uint32_t id = (f & MF_F) ? id2 : id1;
+          const uint64_t st16 = (uint64_t)((stage * slot) >> 4);
+          const uint64_t ad = o.adesc + base16 + ((f & MF_SA) ? st16 : 0);
+          const uint64_t bd = o.bdesc + base16 + ((f & MF_SB) ? st16 : 0);
+          const uint32_t dt = tbase + o.tmem + ((f & MF_F) ? 0u : (uint32_t)(bs * d.ubuf));
           const uint32_t acc0 = (f & MF_ZERO) ? 0u : 1u;
           PROF_ADD(pc_dec);
           {
           PROF_T0();
-          for (int k = 0; k < o.nk; ++k) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, id, k ? 1u : acc0);
+          mma_bf16_w(dt, ad, bd, o.idesc, acc0);
+          for (int k = 1; k < o.nk; ++k) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, o.idesc, 1u);
           PROF_ADD(pc_issue);
 #ifdef TEMCO_TRACE
           pc_n += o.nk;
@@ -899,7 +930,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
   } else if (warp < kEpiWarps) {
 #ifdef TEMCO_TRACE
-    if (g_dbg) goto done;
+    if (g_dbg & 1) goto done;
 #endif
     // ------------------------------------------------------------ epilogue (8 warps)
     // warp w: TMEM lane quarter q = w % 4 (pixel rows 32q..32q+31), column half h = w / 4
@@ -951,10 +982,22 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
             }
             const uint32_t ta = tbase + lane_off + bs * d.ubuf + c_lo;
             uint8_t* P = pbuf + pb * pbytes;
+            // level / member bias (fp32, added here rather than through the tensor core)
+            const float* bsrc = p.params + (un.pooled ? d.mbias : d.lbias[l]) + un.c * Cc + c_lo;
+#ifdef TEMCO_TRACE
+            if (g_dbg & 2) {   // experiment: epilogue does no TMEM / SMEM work
+            } else
+#endif
             if (un.pooled) {
-              // pooled member: fold the unit's taps into the running max / sum (half == 32),
-              // kept in a conflict-free SMEM slab (element i of thread t at run[i * 256 + t])
+              // pooled member: fold the unit's taps into the running max / sum (half == 32);
+              // registers within the unit, a conflict-free SMEM slab across units
+              // (element i of thread t at run[i * 256 + t])
               float* run = runbuf + threadIdx.x;
+              float cur[32];
+              const float4* b4 = reinterpret_cast<const float4*>(bsrc);
+              const bool fresh = un.tg == 0;
+#pragma unroll
+              for (int i = 0; i < 32; ++i) cur[i] = fresh ? (d.mpool == 1 ? -INFINITY : 0.f) : run[i * 256];
               for (int r = 0; r < un.nt; ++r) {
                 const int tap = un.tg * d.tpu + r;
                 const int hi = ho * d.ms - d.mp + tap / d.mk, wi = wo * d.ms - d.mp + tap % d.mk;
@@ -962,30 +1005,39 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 uint32_t v[32];
                 tmem_ld32(ta + r * Cc, v);
                 tmem_wait_ld();
-                const bool first = tap == 0;
 #pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                  float x = __uint_as_float(v[i]);
-                  x = d.mrelu ? fmaxf(x, 0.f) : x;
-                  float cur = first ? (d.mpool == 1 ? -INFINITY : 0.f) : run[i * 256];
-                  if (d.mpool == 1)
-                    cur = valid ? fmaxf(cur, x) : cur;
-                  else
-                    cur += x;
-                  run[i * 256] = cur;
+                for (int i4 = 0; i4 < 8; ++i4) {
+                  const float4 bb = __ldg(b4 + i4);
+                  const float bq[4] = {bb.x, bb.y, bb.z, bb.w};
+#pragma unroll
+                  for (int k = 0; k < 4; ++k) {
+                    const int i = 4 * i4 + k;
+                    float x = __uint_as_float(v[i]) + bq[k];
+                    x = d.mrelu ? fmaxf(x, 0.f) : x;
+                    if (d.mpool == 1)
+                      cur[i] = valid ? fmaxf(cur[i], x) : cur[i];
+                    else
+                      cur[i] += x;
+                  }
                 }
               }
-              if (un.last) {
+              if (!un.last) {
+#pragma unroll
+                for (int i = 0; i < 32; ++i) run[i * 256] = cur[i];
+              } else {
                 // pooled value, + post-pool shift (BN after the pool), level activation
                 const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
-                const float* post = d.post >= 0 ? p.params + d.post + un.c * Cc + c_lo : nullptr;
+                const float4* pv4 = reinterpret_cast<const float4*>(p.params + (d.post >= 0 ? d.post : d.mbias) + un.c * Cc + c_lo);
+                const float pscale = d.post >= 0 ? 1.f : 0.f;
                 const int ch0 = c_lo / 8;
 #pragma unroll
                 for (int qq = 0; qq < 4; ++qq) {
                   float f[8];
+                  const float4 pa = __ldg(pv4 + 2 * qq), pb2 = __ldg(pv4 + 2 * qq + 1);
+                  const float pq[8] = {pa.x, pa.y, pa.z, pa.w, pb2.x, pb2.y, pb2.z, pb2.w};
 #pragma unroll
                   for (int i = 0; i < 8; ++i) {
-                    const float x = run[(8 * qq + i) * 256] * sc + (post ? __ldg(post + 8 * qq + i) : 0.f);
+                    const float x = cur[8 * qq + i] * sc + pscale * pq[i];
                     f[i] = relu ? fmaxf(x, 0.f) : x;
                   }
                   uint4 pk;
@@ -997,30 +1049,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 }
               }
             } else if (!last) {
-              // t_l = relu(acc) back into TMEM for the next level's MMAs
-              if (half == 64) {
-                uint32_t a[32], b[32];
-                tmem_ld32(ta, a);
-                tmem_ld32(ta + 32, b);
-                tmem_wait_ld();
-                if (relu) {
-#pragma unroll
-                  for (int i = 0; i < 32; ++i) {
-                    a[i] = __float_as_uint(fmaxf(__uint_as_float(a[i]), 0.f));
-                    b[i] = __float_as_uint(fmaxf(__uint_as_float(b[i]), 0.f));
-                  }
-                }
-                tmem_st32(ta, a);
-                tmem_st32(ta + 32, b);
-              } else {
+              // t_l = relu(acc + b_l) back into TMEM for the next level's MMAs
+              for (int g = 0; g < half / 32; ++g) {
                 uint32_t a[32];
-                tmem_ld32(ta, a);
+                float bv[32];
+                load_bias32(bsrc + g * 32, bv);
+                tmem_ld32(ta + g * 32, a);
                 tmem_wait_ld();
-                if (relu) {
 #pragma unroll
-                  for (int i = 0; i < 32; ++i) a[i] = __float_as_uint(fmaxf(__uint_as_float(a[i]), 0.f));
+                for (int i = 0; i < 32; ++i) {
+                  const float x = __uint_as_float(a[i]) + bv[i];
+                  a[i] = __float_as_uint(relu ? fmaxf(x, 0.f) : x);
                 }
-                tmem_st32(ta, a);
+                tmem_st32(ta + g * 32, a);
               }
               tmem_wait_st();
             } else if (d.gap) {
@@ -1029,11 +1070,14 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               float* red = reinterpret_cast<float*>(pbuf + h * pbytes);
               for (int g = 0; g < half / 32; ++g) {
                 uint32_t v[32];
+                float bv[32];
+                load_bias32(bsrc + g * 32, bv);
                 tmem_ld32(ta + g * 32, v);
                 tmem_wait_ld();
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
-                  const float x = relu ? fmaxf(__uint_as_float(v[i]), 0.f) : __uint_as_float(v[i]);
+                  const float x0 = __uint_as_float(v[i]) + bv[i];
+                  const float x = relu ? fmaxf(x0, 0.f) : x0;
                   red[row * 32 + ((i + row) & 31)] = x;
                 }
                 asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
@@ -1048,9 +1092,11 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
               }
             } else {
-              // last level: P = bf16 relu(acc) -> SMEM (SW128 K-major atoms of 64 columns)
+              // last level: P = bf16 relu(acc + b) -> SMEM (SW128 K-major atoms of 64 columns)
               for (int g = 0; g < half / 32; ++g) {
                 uint32_t v[32];
+                float bv[32];
+                load_bias32(bsrc + g * 32, bv);
                 tmem_ld32(ta + g * 32, v);
                 tmem_wait_ld();
                 const int col = c_lo + g * 32;
@@ -1061,7 +1107,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   float f[8];
 #pragma unroll
                   for (int i = 0; i < 8; ++i) {
-                    const float x = __uint_as_float(v[8 * qq + i]);
+                    const float x = __uint_as_float(v[8 * qq + i]) + bv[8 * qq + i];
                     f[i] = relu ? fmaxf(x, 0.f) : x;
                   }
                   uint4 pk;
@@ -1091,7 +1137,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       ++tile_iter;
       tc_fence_after();
       const int ng = d.Np / 8, gh = (ng + 1) / 2;
-      for (int g = h * gh; g < min(ng, (h + 1) * gh); ++g) {
+#ifdef TEMCO_TRACE
+      const int gend = (g_dbg & 2) ? 0 : min(ng, (h + 1) * gh);
+#else
+      const int gend = min(ng, (h + 1) * gh);
+#endif
+      for (int g = h * gh; g < gend; ++g) {
         uint32_t v[8];
         tmem_ld8(tbase + lane_off + 2 * d.ubuf + g * 8, v);
         tmem_wait_ld();
@@ -1131,6 +1182,18 @@ extern "C" void temco_debug_trace(long long* out) {
   cudaMemset(p, 0, sizeof(g_trace));
 }
 #endif
+
+// diagnostics: registers, max threads per block, static / max dynamic SMEM of the chain kernel
+extern "C" int temco_debug_tc_attrs(int* out) {
+  cudaFuncAttributes a;
+  const cudaError_t e = cudaFuncGetAttributes(&a, tc_chain_kernel);
+  out[0] = a.numRegs;
+  out[1] = a.maxThreadsPerBlock;
+  out[2] = (int)a.sharedSizeBytes;
+  out[3] = a.maxDynamicSharedSizeBytes;
+  out[4] = (int)a.localSizeBytes;
+  return (int)e;
+}
 
 void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   (void)tcw;

@@ -72,6 +72,7 @@ enum : uint16_t {
   MF_P_COMMIT = 2048,   // commit p_empty[unit] after
   MF_OUT_COMMIT = 4096, // commit out_full after
   MF_BRES = 8192,       // B = resident weights + boff
+  MF_BZERO = 16384,     // B = zero tile (with MF_ONES | MF_ZERO: zero-initialise the region)
 };
 struct TcMmaOp {
   uint16_t flags;
@@ -81,6 +82,17 @@ struct TcMmaOp {
   uint32_t aoff, boff;
 };
 static_assert(sizeof(TcMmaOp) == 16, "TcMmaOp layout");
+// device form: UMMA descriptors precomputed on the host relative to the
+// 1024-aligned SMEM base (start-address field = offset >> 4); the issuer only
+// adds (base >> 4) and, for ring operands, (stage * slot) >> 4
+struct TcMmaOpD {
+  uint64_t adesc, bdesc;
+  uint32_t idesc, tmem;           // instruction descriptor; TMEM column (unit ops: + buffer * ubuf)
+  uint16_t flags;
+  uint8_t unit, nk;
+  uint32_t pad;
+};
+static_assert(sizeof(TcMmaOpD) == 32, "TcMmaOpD layout");
 
 struct TcChainDesc {
   TcTerm term[kTcMaxTerms];
@@ -91,6 +103,7 @@ struct TcChainDesc {
   alignas(64) unsigned char bmapm[128];                 // pooled member bias
   int64_t boff[kTcMaxLevels];            // tc weight pool offsets of the bias matrices
   int64_t boffm;
+  int64_t lbias[kTcMaxLevels], mbias;    // fp32 params offsets of the level / member biases (epilogue adds)
   int32_t n_terms, n_levels;             // outer (level) terms: [0, n_terms)
   int32_t lvl_end[kTcMaxLevels];         // terms [lvl_end[l-1], lvl_end[l]) accumulate into level l
   int32_t relu[kTcMaxLevels];
@@ -123,7 +136,7 @@ struct TcChainDesc {
   int32_t mma_head;                      // > 0: pipelined MMA order, unit ops = mma[0, mma_head)
   int32_t prog_smem;                     // > 0: programs copied to SMEM at kernel start (bytes reserved)
   const TcProdOp* prod;                  // device pointers (tc_finalize)
-  const TcMmaOp* mma;
+  const TcMmaOpD* mma;
   int32_t stages, slot_a, slot_b;        // smem ring depth, bytes of one A / B slot
   int32_t smem_bytes, tmem_cols;
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
