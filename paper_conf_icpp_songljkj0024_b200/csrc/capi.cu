@@ -16,6 +16,7 @@
 #include "conv_tc.h"
 #include "mma_chain.h"
 #include "tc.h"
+#include "tc_wide.h"
 
 using namespace temco;
 
@@ -34,7 +35,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW };
 
 struct StepExec {
   int kind = K_NONE;
@@ -43,6 +44,7 @@ struct StepExec {
   LinearDesc lin{};
   GroupDesc grp{};
   TcChainDesc tc{};
+  wide::TcChainDesc tcw{};
   ConvTcDesc ctc{};
   MmaChainDesc mma{};
   std::string kernel;
@@ -274,6 +276,14 @@ void lower(temco_plan_s* P) {
         e.launches = 1;
         continue;
       }
+      // groups whose per-tile reduced inputs exceed shared memory: TMEM-resident levels
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+          wide::tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tcw)) {
+        e.kind = K_GROUP_TCW;
+        e.kernel = "tc_chain";
+        e.launches = 1;
+        continue;
+      }
       GroupLowering gl{P, std::set<int>(s.members.begin(), s.members.end()), {}};
       GroupDesc& g = e.grp;
       int tsrc;
@@ -428,8 +438,13 @@ std::string make_json(const temco_plan_s* P) {
       if (e.kind == K_GROUP_TC)
         o << ",\"alg_flops\":" << e.tc.alg_flops << ",\"alg_bytes\":" << e.tc.alg_bytes << ",\"tc\":{\"n_prod\":"
           << e.tc.n_prod << ",\"n_mma\":" << e.tc.n_mma << ",\"units\":" << e.tc.units << ",\"stages\":" << e.tc.stages
-          << ",\"resident\":" << e.tc.resident << ",\"smem\":" << e.tc.smem_bytes << ",\"tmem\":" << e.tc.tmem_cols << ",\"pipelined\":" << (e.tc.mma_head > 0) << ",\"ntiles\":"
+          << ",\"resident\":" << e.tc.resident << ",\"smem\":" << e.tc.smem_bytes << ",\"tmem\":" << e.tc.tmem_cols << ",\"fres\":" << e.tc.fres << ",\"slots\":" << e.tc.ns << ",\"ntiles\":"
           << e.tc.ntiles << ",\"Cc\":" << e.tc.Cc << ",\"levels\":" << e.tc.n_levels << "}";
+      if (e.kind == K_GROUP_TCW)
+        o << ",\"alg_flops\":" << e.tcw.alg_flops << ",\"alg_bytes\":" << e.tcw.alg_bytes << ",\"tc\":{\"variant\":\"wide\",\"n_prod\":"
+          << e.tcw.n_prod << ",\"n_mma\":" << e.tcw.n_mma << ",\"units\":" << e.tcw.units << ",\"stages\":" << e.tcw.stages
+          << ",\"resident\":" << e.tcw.resident << ",\"smem\":" << e.tcw.smem_bytes << ",\"tmem\":" << e.tcw.tmem_cols
+          << ",\"ntiles\":" << e.tcw.ntiles << ",\"Cc\":" << e.tcw.Cc << ",\"levels\":" << e.tcw.n_levels << "}";
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;
     }
@@ -481,6 +496,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
       case K_LINEAR: launch_linear(e.lin, rp, st); break;
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
+      case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
       case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
       case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
     }
@@ -602,6 +618,13 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
       }
     if (!tc_finalize(P->exec.size(), [&](size_t i) -> TcChainDesc* {
           return P->exec[i].kind == K_GROUP_TC ? &P->exec[i].tc : nullptr;
+        }, P->arena_d, P->tcw_d, terr)) {
+      free_device(P);
+      delete P;
+      return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
+    }
+    if (!wide::tc_finalize(P->exec.size(), [&](size_t i) -> wide::TcChainDesc* {
+          return P->exec[i].kind == K_GROUP_TCW ? &P->exec[i].tcw : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {
       free_device(P);
       delete P;

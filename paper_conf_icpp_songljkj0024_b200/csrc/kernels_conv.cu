@@ -182,7 +182,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&acc_full[b], 1);
-      mbar_init(&acc_empty[b], 128);
+      mbar_init(&acc_empty[b], 4);
     }
     mbar_init(wbar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -342,7 +342,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
         }
       }
       tc_fence_before();
-      mbar_arrive(&acc_empty[buf]);
+      warp_arrive(&acc_empty[buf]);
     }
   }
   tc_fence_before();
@@ -380,7 +380,7 @@ __global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __gr
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&acc_full[b], 1);
-      mbar_init(&acc_empty[b], 128);
+      mbar_init(&acc_empty[b], 4);
     }
     mbar_init(wbar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -471,7 +471,7 @@ __global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __gr
         }
       }
       tc_fence_before();
-      mbar_arrive(&acc_empty[buf]);
+      warp_arrive(&acc_empty[buf]);
     }
   }
   tc_fence_before();

@@ -1,24 +1,26 @@
 // tcgen05 fused restore-chain -> BN -> add/concat -> ReLU -> [pool] -> reduce kernel (sm_100a).
 //
-// One fused group computes, per output tile,
+// One fused group computes, per output tile of 128 pixels,
 //     t_l = act_l( sum_{j in l} r_j Lhat_j^T + b_l + t_{l-1} ),  out = t_D F^T
-// with the C-wide t never leaving the SM:
-//   GEMM1  r_j atoms [rows x 64] (2D TMA of 128 consecutive pixels, or 4D TMA of
-//          a tap-shifted, strided spatial box) and Lhat_j atoms [Cc x 64] (TMA)
-//          -> SMEM ring -> tcgen05.mma (M=128, N=Cc, K=16) -> TMEM accumulator;
-//          the level bias enters the same accumulator through the tensor core
-//          (constant SMEM ones tile x [b_hi, b_lo] columns)
-//   level epilogue (8 warps: TMEM lane quarter x column half): TMEM -> regs,
-//          ReLU, -> TMEM (tcgen05.st) so the next level accumulates on top of
-//          t_{l-1}; after the last level the bf16 tile P = t_D goes to SMEM in
-//          the SW128 K-major layout.  Pooled-member chunks keep one TMEM region
-//          per tap and fold max / sum in registers; GAP roots reduce per image.
-//   GEMM2  tcgen05.mma (A = P from SMEM, B = F atom via TMA) -> TMEM (Np columns)
-//   output epilogue: TMEM -> registers -> bf16 -> global.
-// Warp roles (320 threads, persistent over tiles): warps 0-7 epilogue, 8 TMA
-// producer, 9 MMA issuer.  Units (a chunk, or a tap group of a pooled chunk)
-// alternate between two TMEM buffers so one unit's MMAs overlap the previous
-// unit's epilogue.
+// with the C-wide t never leaving the SM.  The restored width is cut into units
+// of 64 channels; a unit's levels are evaluated back to back:
+//   GEMM1  r_j atoms [rows x aw] (2D TMA of 128 consecutive pixels, or 4D TMA of
+//          a tap-shifted, strided spatial box) x Lhat_j atoms [64 x aw] (TMA,
+//          SMEM-resident when they fit) -> tcgen05.mma (M=128, N=64) into a
+//          fresh TMEM accumulator slot per (unit, level); slots form a ring, so
+//          the MMA issuer runs ahead of the epilogue by several unit-levels.
+//   level epilogue: TMEM -> registers, + b_l + t_{l-1} (t lives in registers:
+//          no tcgen05.st round trip), ReLU; the slot is released as soon as it
+//          has been read.  After the last level the bf16 tile P = t_D goes to
+//          SMEM in the SW128 K-major layout.  Pooled-member units keep one TMEM
+//          region per tap and fold max / sum in registers; GAP roots reduce per
+//          image.
+//   GEMM2  tcgen05.mma (A = P, B = F atom) accumulates out over the units in
+//          a TMEM output buffer; the output epilogue stores bf16 rows.
+// Warp roles (640 threads, persistent over tiles): warps 0-15 epilogue in two
+// teams of 8 that take alternate tiles (one team's TMEM-load latency hides
+// behind the other's arithmetic); warp 16 TMA producer (A / B ring), 17 GEMM1
+// issuer, 18 GEMM2 issuer, 19 F-ring producer (and TMEM allocation).
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cudaTypedefs.h>
@@ -46,13 +48,6 @@ uint16_t to_bf16(float f) {
   return (uint16_t)(u >> 16);
 }
 
-float from_bf16(uint16_t h) {
-  uint32_t u = (uint32_t)h << 16;
-  float f;
-  memcpy(&f, &u, 4);
-  return f;
-}
-
 int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
   while (pool.size() % 512) pool.push_back(0);   // 1024-byte aligned blocks (TMA base alignment)
   int64_t off = (int64_t)pool.size();
@@ -68,185 +63,132 @@ int64_t push_f32(std::vector<float>& params, const std::vector<double>& v, int n
   return off;
 }
 
-// bias as a rank-2 term: columns 0, 1 = bf16 hi / lo parts (error ~2^-16 |b|)
-int64_t push_bias(std::vector<uint16_t>& pool, const std::vector<double>& b, int c0, int Cpad) {
-  std::vector<float> bm((size_t)Cpad * 8, 0.f);
-  for (size_t c = 0; c < b.size(); ++c) {
-    const float x = (float)b[c];
-    const float hi = from_bf16(to_bf16(x));
-    bm[(size_t)(c0 + c) * 8 + 0] = hi;
-    bm[(size_t)(c0 + c) * 8 + 1] = x - hi;
+struct HUnit {
+  int c, tg, nt;
+  bool pooled, last;
+};
+
+HUnit unit_of(const TcChainDesc& d, int u) {
+  HUnit x;
+  if (u < d.npc * d.ntg) {
+    x.c = u / d.ntg;
+    x.tg = u % d.ntg;
+    x.nt = std::min(d.tpu, d.mtaps - x.tg * d.tpu);
+    x.pooled = true;
+    x.last = x.tg == d.ntg - 1;
+  } else {
+    x.c = d.npc + (u - d.npc * d.ntg);
+    x.tg = 0;
+    x.nt = 1;
+    x.pooled = false;
+    x.last = true;
   }
-  return push_bf16(pool, bm);
+  return x;
 }
 
-// Per-tile producer / MMA programs.  Unit order (all roles): for each pair of
-// units: for each level: for each unit of the pair: [bias, terms x taps x K
-// atoms]; then the fconv atoms of the pair's finished chunks.  TMEM buffer of
-// unit u of a tile = (units before the tile + u) & 1.
+// Per-tile producer / MMA programs.  Producer: every distinct A atom of the
+// tile (term x tap x K atom) once into the tile's A buffer, then (B streamed)
+// one ring stage per MMA op.  MMA order: for each unit: for each of its levels
+// (pooled units: one): [terms x taps x K atoms] into one accumulator slot.
 void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
-  std::vector<TcProdOp> P;
+  std::vector<TcProdOp> P, PB;
   std::vector<TcMmaOp> M;
   const int Cc = d.Cc;
   const int U = d.npc * d.ntg + d.nchunks - d.npc;
   d.units = U;
   const bool res = d.resident != 0;
   const int rows_a = d.spatial ? d.tw * d.th * d.tn : 128;
-  const int pbytes = 128 * Cc * 2;
   auto moff = [&](const unsigned char* m) {
     return (uint16_t)((reinterpret_cast<const char*>(m) - reinterpret_cast<const char*>(&d)) / 64);
   };
-  struct HUnit {
-    int c, tg, nt;
-    bool pooled, last;
+  std::map<std::tuple<int, int, int>, uint32_t> atom;   // (term, tap, K atom) -> offset in the A buffer
+  uint32_t aoff = 0;
+  int atx = 0;
+  auto atom_of = [&](int j, int tap, int ka, int kk, int pad) {
+    const auto key = std::make_tuple(j, tap, ka);
+    auto it = atom.find(key);
+    if (it != atom.end()) return it->second;
+    const TcTerm& t = d.term[j];
+    TcProdOp o{};
+    o.kind = d.spatial ? PK_A4D : PK_A2D;
+    o.ts = (uint8_t)t.ts;
+    o.amap = moff(d.spatial ? t.tmap4 : t.tmap);
+    o.ac = (int16_t)(ka * t.aw);
+    o.dx = (int16_t)(tap % kk - pad);
+    o.dy = (int16_t)(tap / kk - pad);
+    o.bytes = (uint16_t)(rows_a * t.aw * 2);
+    o.dst = aoff;
+    P.push_back(o);
+    atx += rows_a * t.aw * 2;
+    const uint32_t off = aoff;
+    aoff += (uint32_t)((rows_a * t.aw * 2 + 1023) / 1024 * 1024);
+    atom[key] = off;
+    return off;
   };
-  auto unit_at = [&](int u) {
-    HUnit x;
-    if (u < d.npc * d.ntg) {
-      x.c = u / d.ntg;
-      x.tg = u % d.ntg;
-      x.nt = std::min(d.tpu, d.mtaps - x.tg * d.tpu);
-      x.pooled = true;
-      x.last = x.tg == d.ntg - 1;
-    } else {
-      x.c = d.npc + (u - d.npc * d.ntg);
-      x.tg = 0;
-      x.nt = 1;
-      x.pooled = false;
-      x.last = true;
-    }
-    return x;
-  };
-  for (int u0 = 0; u0 < U; u0 += 2) {
-    const int nb = std::min(2, U - u0);
-    for (int l = 0; l < d.n_levels; ++l)
-      for (int bi = 0; bi < nb; ++bi) {
-        const int u = u0 + bi;
-        const HUnit un = unit_at(u);
-        // level biases are added by the epilogue: the first MMA into each tap region
-        // at level 0 overwrites (MF_ZERO); a region no term reaches gets a zero-init MMA
-        const size_t m_first = M.size();
-        std::vector<char> region_done(un.nt, 0);
-        const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
-        const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
-        for (int r = 0; r < un.nt; ++r)
-          for (int j = j0; j < j1; ++j) {
-            const TcTerm& t = d.term[j];
-            if (!un.pooled && !(t.c0 < (un.c + 1) * Cc && t.c0 + t.C > un.c * Cc)) continue;
-            const int ntap = un.pooled ? 1 : t.tk * t.tk;
-            const int katoms = t.Rp / t.aw;
-            for (int q = 0; q < ntap; ++q) {
-              const int tap = un.pooled ? un.tg * d.tpu + r : q;
-              const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
-              for (int ka = 0; ka < katoms; ++ka) {
+  int spt = 0;
+  for (int u = 0; u < U; ++u) {
+    const HUnit un = unit_of(d, u);
+    const int nl = un.pooled ? 1 : d.n_levels;
+    for (int l = 0; l < nl; ++l) {
+      ++spt;
+      const size_t m_first = M.size();
+      std::vector<char> region_done(un.nt, 0);
+      const int j0 = un.pooled ? d.mt0 : (l ? d.lvl_end[l - 1] : 0);
+      const int j1 = un.pooled ? d.mt1 : d.lvl_end[l];
+      for (int r = 0; r < un.nt; ++r)
+        for (int j = j0; j < j1; ++j) {
+          const TcTerm& t = d.term[j];
+          if (!un.pooled && !(t.c0 < (un.c + 1) * Cc && t.c0 + t.C > un.c * Cc)) continue;
+          const int ntap = un.pooled ? 1 : t.tk * t.tk;
+          const int katoms = t.Rp / t.aw;
+          for (int q = 0; q < ntap; ++q) {
+            const int tap = un.pooled ? un.tg * d.tpu + r : q;
+            const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
+            for (int ka = 0; ka < katoms; ++ka) {
+              TcMmaOp m{};
+              m.aoff = atom_of(j, tap, ka, kk, pad);
+              m.flags = MF_AT | (res ? MF_BRES : MF_SW | MF_SB | MF_SD);
+              if (!res) {
                 TcProdOp o{};
-                o.kind = d.spatial ? PK_A4D : PK_A2D;
-                o.ts = (uint8_t)t.ts;
-                o.amap = moff(d.spatial ? t.tmap4 : t.tmap);
-                o.ac = (int16_t)(ka * t.aw);
-                o.dx = (int16_t)(tap % kk - pad);
-                o.dy = (int16_t)(tap / kk - pad);
-                o.bytes = (uint16_t)((rows_a + (res ? 0 : Cc)) * t.aw * 2);
-                if (!res) {
-                  o.kind |= PK_B;
-                  o.bmap = moff(t.wmap);
-                  o.bx = (int16_t)(ka * t.aw);
-                  o.by = (int16_t)(un.c * Cc);
-                }
-                P.push_back(o);
-                TcMmaOp m{};
-                m.flags = MF_SW | MF_SA | MF_SD | (res ? MF_BRES : MF_SB);
-                if (l == 0 && !region_done[r]) m.flags |= MF_ZERO;
-                region_done[r] = 1;
-                m.unit = (uint8_t)u;
-                m.nk = (uint8_t)std::min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
-                m.la = (uint8_t)t.aw;
-                m.lb = (uint8_t)t.aw;
-                m.tcol = (uint16_t)(r * Cc);
-                if (res) m.boff = (uint32_t)(t.wres + ((un.c - t.cfirst) * katoms + ka) * Cc * t.aw * 2);
-                M.push_back(m);
+                o.kind = PK_B;
+                o.bmap = moff(t.wmap);
+                o.bx = (int16_t)(ka * t.aw);
+                o.by = (int16_t)(un.c * Cc);
+                o.bytes = (uint16_t)(Cc * t.aw * 2);
+                PB.push_back(o);
               }
+              if (!region_done[r]) m.flags |= MF_ZERO;
+              region_done[r] = 1;
+              m.nk = (uint8_t)std::min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
+              m.la = (uint8_t)t.aw;
+              m.lb = (uint8_t)t.aw;
+              m.tcol = (uint16_t)(r * Cc);
+              if (res) m.boff = (uint32_t)(t.wres + ((un.c - t.cfirst) * katoms + ka) * Cc * t.aw * 2);
+              M.push_back(m);
             }
           }
-        for (int r = 0; r < un.nt; ++r)
-          if (l == 0 && !region_done[r]) {   // zero-init: ones tile x zero tile
-            TcMmaOp m{};
-            m.flags = MF_ONES | MF_BZERO | MF_ZERO;
-            m.unit = (uint8_t)u;
-            m.nk = 1;
-            m.la = 16;
-            m.lb = 16;
-            m.tcol = (uint16_t)(r * Cc);
-            M.push_back(m);
-          }
-        M[m_first].flags |= MF_ACC_WAIT;
-        M.back().flags |= MF_ACC_COMMIT;
-      }
-    if (!d.gap)
-      for (int bi = 0; bi < nb; ++bi) {
-        const HUnit un = unit_at(u0 + bi);
-        if (!un.last) continue;
-        const int pb = un.c & 1;
-        const int na = Cc / 64;
-        for (int a = 0; a < na; ++a) {
-          if (!res) {
-            TcProdOp o{};
-            o.kind = PK_B;
-            o.bmap = moff(d.fmap);
-            o.bx = (int16_t)(un.c * Cc + a * 64);
-            o.by = 0;
-            o.bytes = (uint16_t)(d.Np * 128);
-            P.push_back(o);
-          }
+        }
+      for (int r = 0; r < un.nt; ++r)
+        if (!region_done[r]) {   // zero-init: ones tile x zero tile
           TcMmaOp m{};
-          m.flags = MF_F | (a == 0 ? MF_P_WAIT : 0) | (a == 0 && un.c == 0 ? MF_OUT_WAIT | MF_ZERO : 0) |
-                    (a == na - 1 ? MF_P_COMMIT : 0) | (res ? MF_BRES : MF_SW | MF_SB | MF_SD);
-          m.unit = (uint8_t)pb;
-          m.nk = 4;
-          m.la = 64;
-          m.lb = 64;
-          m.aoff = (uint32_t)(pb * pbytes + a * 16384);
-          if (res) m.boff = (uint32_t)(d.fres + (un.c * na + a) * d.Np * 128);
+          m.flags = MF_ONES | MF_BZERO | MF_ZERO;
+          m.nk = 1;
+          m.la = 16;
+          m.lb = 16;
+          m.tcol = (uint16_t)(r * Cc);
           M.push_back(m);
         }
-      }
-  }
-  if (!d.gap) M.back().flags |= MF_OUT_COMMIT;
-  d.n_prod = (int32_t)P.size();
-  d.n_mma = (int32_t)M.size();
-  // programs live in SMEM (after the pooled slab) when they fit next to the ring
-  const int pbytes_prog = (int)(P.size() * sizeof(TcProdOp) + M.size() * sizeof(TcMmaOpD));
-  d.prog_smem = 0;
-  const char* exp_env = getenv("TEMCO_TC_EXP");   // experiment switches (bit 0: programs in global memory)
-  const int exp_bits = exp_env ? atoi(exp_env) : 0;
-  if (pbytes_prog <= 32768 && !(exp_bits & 1)) {
-    const int need = (pbytes_prog + 127) / 128 * 128;
-    while (d.stages > 2 && d.smem_bytes + need > 227 * 1024)
-      d.stages--, d.smem_bytes -= d.slot_a + d.slot_b;
-    if (d.smem_bytes + need <= 227 * 1024) {
-      d.prog_smem = need;
-      d.smem_bytes += need;
+      M[m_first].flags |= MF_ACC_WAIT;
+      M.back().flags |= MF_ACC_COMMIT;
     }
   }
-  // pipelined MMA order (unit ops of tile t+1 before the fconv ops of tile t):
-  // needs resident weights (the ring then carries only unit stages, consumed in
-  // the same order) and a program of the form [unit ops][fconv ops]
-  d.mma_head = 0;
-  // and every TMEM buffer the head of tile t+1 waits for must be released by the
-  // epilogue before it waits for tile t's output: one level, <= 2 units per tile
-  if (res && !d.gap && d.n_levels == 1 && U <= 2) {
-    int h = 0;
-    while (h < (int)M.size() && !(M[h].flags & MF_F)) ++h;
-    bool tail_f = true;
-    for (size_t i = h; i < M.size(); ++i) tail_f &= (M[i].flags & MF_F) != 0;
-    if (tail_f && h > 0 && h < (int)M.size()) d.mma_head = h;
-  }
+  d.n_aload = (int32_t)P.size();
+  d.a_tx = atx;
+  for (const TcProdOp& o : PB) P.push_back(o);
+  d.spt = spt;
+  d.n_prod = (int32_t)P.size();
+  d.n_mma = (int32_t)M.size();
   while (tcw.size() % 512) tcw.push_back(0);
-  // device MMA ops: descriptors relative to the aligned SMEM base (final layout)
-  const int slot = d.slot_a + d.slot_b;
-  const uint32_t ring_off = (uint32_t)d.wres_bytes;
-  const uint32_t pbuf_off = ring_off + (uint32_t)(d.stages * slot);
-  const uint32_t ones_off = pbuf_off + 2u * (uint32_t)pbytes;
   auto dtmpl = [](uint32_t off, int aw) {
     const uint64_t layout = aw == 64 ? 2 : aw == 32 ? 4 : 6;
     return (uint64_t)(off >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(16 * aw >> 4) << 32) | ((uint64_t)1 << 46) |
@@ -259,15 +201,15 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
   for (size_t i = 0; i < M.size(); ++i) {
     const TcMmaOp& m = M[i];
     TcMmaOpD& o = MD[i];
-    const bool isF = m.flags & MF_F;
-    const uint32_t aoff = (m.flags & MF_ONES) ? ones_off : isF ? pbuf_off + m.aoff : ring_off;
-    const uint32_t boff = (m.flags & MF_BZERO) ? ones_off + 4096u : (m.flags & MF_BRES) ? m.boff : ring_off + (uint32_t)d.slot_a;
+    const uint32_t aoff = (m.flags & MF_ONES) ? (uint32_t)d.off_ones : (uint32_t)d.off_abuf + m.aoff;
+    const uint32_t boff = (m.flags & MF_BZERO) ? (uint32_t)d.off_zeros
+                          : (m.flags & MF_BRES) ? m.boff
+                                                : (uint32_t)d.off_ring;
     o.adesc = dtmpl(aoff, m.la);
     o.bdesc = dtmpl(boff, m.lb);
-    o.idesc = isF ? idesc(128, d.Np) : idesc(128, Cc);
-    o.tmem = isF ? (uint32_t)(2 * d.ubuf) : m.tcol;
+    o.idesc = idesc(128, Cc);
+    o.tmem = m.tcol;
     o.flags = m.flags;
-    o.unit = m.unit;
     o.nk = m.nk;
   }
   d.prog_off = (int64_t)tcw.size();
@@ -307,7 +249,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   }
   const bool mixed = pm || taps_any;
   if (mixed && levels.size() != 1) return false;
-  if (pm && (pm->c0 != 0 || pm->C % 64)) return false;
+  if (pm && (pm->c0 != 0 || pm->C % kTcCc)) return false;
   if (pm && gap) return false;                       // GAP over a max-pooled member: generic path
   int nterms = 0;
   for (auto& L : levels) nterms += (int)L.terms.size();
@@ -329,7 +271,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
 
   d = TcChainDesc();
   d.C = C;
-  d.Cc = (C <= 64 || mixed) ? 64 : 128;
+  d.Cc = kTcCc;
   d.Cpad = (C + d.Cc - 1) / d.Cc * d.Cc;
   d.nchunks = d.Cpad / d.Cc;
   d.Nout = Nout;
@@ -402,8 +344,8 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
     d.relu[l] = L.relu ? 1 : 0;
-    // pooled-member channels take no level bias through the MMA: their level bias
-    // (the post-BN shift) is added after pooling, in the epilogue
+    // pooled-member channels take no level bias before the pool: their level
+    // bias (the post-BN shift) is added after pooling, in the epilogue
     std::vector<double> lb = L.bias;
     if (pm && l == 0) {
       std::vector<double> post(d.Cc * (pm->C / d.Cc), 0.0);
@@ -415,7 +357,6 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
       d.post = (int64_t)params.size();
       for (double x : post) params.push_back((float)x);
     }
-    d.boff[l] = push_bias(tcw, lb, 0, d.Cpad);
     d.lbias[l] = push_f32(params, lb, d.Cpad);
     for (const PTerm& t : L.terms)
       if (!add_term(t)) return false;
@@ -440,13 +381,10 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
       if (!add_term(u)) return false;
     }
     d.mt1 = j;
-    // the member is evaluated once per tap: count its work at the taps actually run
-    d.boffm = push_bias(tcw, pm->bias, 0, d.Cpad);
     d.mbias = push_f32(params, pm->bias, d.Cpad);
     if (d.tw * d.ms > 256 || d.th * d.ms > 256) return false;
   }
   d.F = 0;
-  d.Fb = -1;
   if (gap) {
     d.alg_flops = flops + d.npix * C;
     d.alg_bytes = bytes + 2LL * ir.batch * C;
@@ -458,53 +396,110 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.alg_flops = flops + d.npix * 2LL * Nout * C;
     d.alg_bytes = bytes + d.npix * 2LL * Nout;
   }
-  // pooled member: as many taps per unit as two unit buffers + the output allow
+  // TMEM: accumulator slots (ubuf columns: one region per tap of a pooled unit)
+  // and one or two output buffers of Np columns
+  const int npcols = gap ? 0 : d.Np;
+  d.no = gap ? 0 : (512 - 2 * npcols >= 4 * d.Cc ? 2 : 1);
+  const int avail = 512 - d.no * npcols;
   d.tpu = 1;
   d.ntg = 1;
   if (pm) {
-    int t = d.mtaps;
-    while (t > 1 && 2 * t * d.Cc + d.Np > 512) --t;
+    int t = std::max(1, std::min(d.mtaps, avail / (4 * d.Cc)));
     d.ntg = (d.mtaps + t - 1) / t;
     d.tpu = (d.mtaps + d.ntg - 1) / d.ntg;
   }
   d.ubuf = d.tpu * d.Cc;
-  // shared memory: ring of (A | B) stages sized by the widest K atom of the group
-  // (small ranks -> small stages -> a deep ring), two P tiles, ones tile, barriers
+  d.ns = std::min(8, avail / d.ubuf) & ~1;     // even: each epilogue team owns half the slots
+  if (d.ns < 2) return false;
+  d.out_col = d.ns * d.ubuf;
+  d.tmem_cols = 512;
+  // shared memory: [resident weights][A buffers][B ring][F ring][4 P buffers][ones][zeros][barriers][programs]
+  const int rows_a = d.spatial ? d.tw * d.th * d.tn : 128;
   int awmax = 16;
+  int64_t abytes = 0;
   const int nall = pm ? d.mt1 : d.n_terms;
-  for (int i = 0; i < nall; ++i) awmax = std::max(awmax, d.term[i].aw);
-  d.slot_a = 128 * awmax * 2;
-  int sb = std::max(d.Cc * awmax * 2, d.Cc * 32);
-  if (!gap) sb = std::max(sb, d.Np * 128);
-  d.slot_b = (sb + 1023) / 1024 * 1024;
-  const int pbytes = 128 * d.Cc * 2;
-  const int runbytes = pm ? 32768 : 0;     // pooled member: running max / sum slab (after the barriers)
-  const int budget = 227 * 1024 - 1024 /*align*/ - 2048 /*barriers*/ - runbytes - 2 * pbytes - 8192 /*ones, zeros*/;
-  // resident weights: every B box (term atoms of the chunks a term reaches, level
-  // and member biases, F atoms) once per CTA, if that leaves a ring of >= 6 A slots
-  int64_t woff = 0;
+  for (int i = 0; i < nall; ++i) {
+    const TcTerm& T = d.term[i];
+    awmax = std::max(awmax, T.aw);
+    const int ntap = i >= d.n_terms ? d.mtaps : T.tk * T.tk;
+    abytes += (int64_t)ntap * (T.Rp / T.aw) * ((rows_a * T.aw * 2 + 1023) / 1024 * 1024);
+  }
+  d.atr = 1;
+  d.abytes = (int32_t)abytes;
+  d.slot_a = 0;
+  const int slot_b_stream = (d.Cc * awmax * 2 + 1023) / 1024 * 1024;
+  const int fixed = 1024 /*align*/ + 4 * 16384 /*P*/ + 8192 /*ones, zeros*/ + 1024 /*barriers*/;
+  const int64_t budget = 227 * 1024 - fixed;
+  int64_t wb = 0;
   for (int i = 0; i < nall; ++i) {
     TcTerm& T = d.term[i];
-    T.wres = (int32_t)woff;
-    woff += (int64_t)T.nhit * (T.Rp / T.aw) * d.Cc * T.aw * 2;
+    T.wres = (int32_t)wb;
+    wb += (int64_t)T.nhit * (T.Rp / T.aw) * d.Cc * T.aw * 2;
   }
-  d.fres = (int32_t)woff;
-  if (!gap) woff += (int64_t)(d.Cpad / 64) * d.Np * 128;
-  d.resident = woff + 6LL * d.slot_a <= budget ? 1 : 0;
-  if (d.resident) {
-    d.wres_bytes = (int32_t)woff;
-    d.slot_b = 0;
-    d.stages = std::min<int64_t>(24, (budget - woff) / d.slot_a);
-  } else {
-    d.wres_bytes = 0;
-    d.stages = std::min(24, budget / (d.slot_a + d.slot_b));
+  const int64_t wf = gap ? 0 : (int64_t)d.nchunks * d.Np * 128;
+  d.fslot = gap ? 0 : (d.Np * 128 + 1023) / 1024 * 1024;
+  // first arrangement that fits: two A buffers before one, resident B before
+  // resident F; a streamed B needs >= 4 ring stages
+  struct Opt { int nab; bool b, f; };
+  const Opt opts[8] = {{2, true, true}, {2, true, false}, {2, false, true}, {2, false, false},
+                       {1, true, true}, {1, true, false}, {1, false, true}, {1, false, false}};
+  bool found = false;
+  for (const Opt& o : opts) {
+    if (gap && o.f) continue;
+    const int64_t wres = (o.b ? wb : 0) + (o.f ? wf : 0);
+    const int64_t wres_al = (wres + 1023) / 1024 * 1024;
+    const int fst = (gap || o.f) ? 0 : 3;
+    const int64_t left = budget - wres_al - o.nab * abytes - (int64_t)fst * d.fslot;
+    if (left < (o.b ? 0 : 4LL * slot_b_stream)) continue;
+    d.nabuf = o.nab;
+    d.resident = o.b ? 1 : 0;
+    d.fres = o.f ? 1 : 0;
+    d.wres_bytes = (int32_t)wres_al;
+    d.fbase = (int32_t)(o.b ? wb : 0);
+    d.fstages = fst;
+    d.slot_b = o.b ? 0 : slot_b_stream;
+    d.stages = o.b ? 0 : (int)std::min<int64_t>(24, left / slot_b_stream);
+    found = true;
+    break;
   }
-  if (d.stages < 2) return false;
-  d.smem_bytes = 1024 + d.wres_bytes + d.stages * (d.slot_a + d.slot_b) + 2 * pbytes + 8192 + 2048 + runbytes;
-  const int cols = 2 * d.ubuf + d.Np;
-  d.tmem_cols = cols <= 32 ? 32 : cols <= 64 ? 64 : cols <= 128 ? 128 : cols <= 256 ? 256 : 512;
-  if (cols > 512) return false;
+  // kernel choice (measured on B200): this kernel's 64-channel
+  // units issue N=64 MMAs (about half the per-instruction tensor rate of N=128)
+  // but keep many small tiles in flight; the wide kernel (N=128, levels
+  // accumulated in TMEM) wins for multi-level chains and K >= 128 per unit
+  int kmax = 0;
+  for (int c = 0; c < d.nchunks; ++c) {
+    int k = 0;
+    for (int i = 0; i < d.n_terms; ++i) {
+      const TcTerm& T = d.term[i];
+      if (T.c0 < (c + 1) * d.Cc && T.c0 + T.C > c * d.Cc) k += T.Rp * T.tk * T.tk;
+    }
+    kmax = std::max(kmax, k);
+  }
+  bool taps = false;
+  for (int i = 0; i < d.n_terms; ++i) taps |= d.term[i].tk > 1;
+  const bool prefer_wide = !pm && (d.n_levels >= 2 || (kmax >= 128 && !taps));
+  if (getenv("TEMCO_TC_V2") == nullptr && prefer_wide) return false;
+  if (!found || getenv("TEMCO_TC_WIDE")) return false;   // -> the wide (TMEM-level) kernel
+  d.exp = getenv("TEMCO_TC_EXP") ? atoi(getenv("TEMCO_TC_EXP")) : 0;
+  if (getenv("TEMCO_TC_TRACE_OUT") && atoi(getenv("TEMCO_TC_TRACE_OUT")) == s.out) d.exp |= 4;
+  d.off_abuf = d.wres_bytes;
+  d.off_ring = d.off_abuf + d.nabuf * d.abytes;
+  d.off_fring = d.off_ring + d.stages * d.slot_b;
+  d.off_p = d.off_fring + d.fstages * d.fslot;
+  d.off_ones = d.off_p + 4 * 16384;
+  d.off_zeros = d.off_ones + 4096;
+  d.off_bars = d.off_zeros + 4096;
+  d.off_prog = d.off_bars + 1024;
+  d.smem_bytes = 1024 + d.off_prog;
   build_programs(d, tcw);
+  // programs live in SMEM when they fit
+  const int pbytes_prog = d.n_prod * (int)sizeof(TcProdOp) + d.n_mma * (int)sizeof(TcMmaOpD);
+  const int need = (pbytes_prog + 127) / 128 * 128;
+  d.prog_smem = 0;
+  if (d.smem_bytes + need <= 227 * 1024) {
+    d.prog_smem = need;
+    d.smem_bytes += need;
+  }
   return true;
 }
 
@@ -564,15 +559,6 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
         return false;
       }
     }
-    for (int l = 0; l < d->n_levels; ++l)
-      if (!make(d->bmap[l], tcw + d->boff[l], 8, (uint64_t)d->Cpad, (uint32_t)d->Cc, 16)) {
-        err = "cuTensorMapEncodeTiled failed (bias)";
-        return false;
-      }
-    if (d->npc && !make(d->bmapm, tcw + d->boffm, 8, (uint64_t)d->Cpad, (uint32_t)d->Cc, 16)) {
-      err = "cuTensorMapEncodeTiled failed (member bias)";
-      return false;
-    }
     if (!d->gap && !make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
       err = "cuTensorMapEncodeTiled failed (F)";
       return false;
@@ -587,64 +573,16 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
 namespace {
 using namespace ptx;
 
-__device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
-  return t.c0 < (c + 1) * Cc && t.c0 + t.C > c * Cc;
-}
+constexpr int kTeamWarps = 8;
+constexpr int kEpiWarps = 2 * kTeamWarps;
+constexpr int kProdWarp = 16, kMmaWarp = 17, kG2Warp = 18, kFWarp = 19;
+constexpr int kThreads = 32 * 20;
+constexpr int kTeamArrivals = kTeamWarps;   // one elected arrive per epilogue warp
 
-#ifdef TEMCO_TRACE
-// experiment builds only: %globaltimer stamps of CTA 0's pipeline events
-constexpr int kTraceRows = 12;
-__device__ unsigned long long g_trace[kTraceRows][512];
-__device__ int g_dbg;   // 1: TMA-only run (MMA / epilogue roles idle; output garbage)
-__device__ __forceinline__ void trace_stamp(int row, int& n) {
-  if (blockIdx.x == 0 && n < 512) {
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    g_trace[row][n] = t;
-  }
-  ++n;
-}
-#ifdef TEMCO_NOSTAMP
-#define TRACE(row, n) ((void)0)
-#else
-#define TRACE(row, n) trace_stamp(row, n)
-#endif
-// cycle accounting of CTA 0's MMA issuer: waits by kind, op loads, total
-__device__ unsigned long long g_prof[16];
-#define PROF_T0() (_pt0 = clock64())
-#define PROF_ADD(var) (var += clock64() - _pt0)
-#else
-#define TRACE(row, n) ((void)0)
-#define PROF_T0() ((void)0)
-#define PROF_ADD(var) ((void)0)
-#endif
-
-// 32 consecutive fp32 values (16-byte aligned) -> registers
-__device__ __forceinline__ void load_bias32(const float* src, float (&b)[32]) {
-  const float4* s4 = reinterpret_cast<const float4*>(src);
-#pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    const float4 v = __ldg(s4 + i);
-    b[4 * i] = v.x;
-    b[4 * i + 1] = v.y;
-    b[4 * i + 2] = v.z;
-    b[4 * i + 3] = v.w;
-  }
-}
-
-constexpr int kEpiWarps = 8;
-constexpr int kProdWarp = 8, kMmaWarp = 9;
-constexpr int kThreads = 32 * 10;
-
-// Units of one tile: pooled chunks c < npc contribute ntg tap-group units each,
-// every other chunk one unit.  Units are processed in pairs (TMEM buffers 0, 1);
-// all roles walk the same order: for pair: for level: for unit in pair.
 struct Unit {
   int c, tg, nt;      // chunk, tap group, taps in the unit (1 for plain chunks)
   bool pooled, last;  // pooled-member chunk; last unit of its chunk
 };
-
-__device__ __forceinline__ int units_per_tile(const TcChainDesc& d) { return d.npc * d.ntg + d.nchunks - d.npc; }
 
 __device__ __forceinline__ Unit unit_at(const TcChainDesc& d, int u) {
   Unit x;
@@ -668,6 +606,27 @@ struct TileGeo {
   int m0, n0, h0, w0;
 };
 
+#ifdef TEMCO_TRACE
+// experiment builds only: %globaltimer stamps of CTA 0's pipeline events for the
+// group lowered with TEMCO_TC_TRACE_OUT=<its output id> (exp bit 4)
+constexpr int kTraceRows = 12;
+__device__ unsigned long long g_trace[kTraceRows][512];
+// per-row event counters live in registers of the stamping thread (tn[row])
+#define TRACE(row)                                                              \
+  do {                                                                          \
+    if ((d.exp & 4) && blockIdx.x == 0 && (threadIdx.x & 31) == 0) {            \
+      const int n_ = tn[row]++;                                                 \
+      if (n_ < 512) {                                                           \
+        unsigned long long t_;                                                  \
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_));                 \
+        g_trace[row][n_] = t_;                                                  \
+      }                                                                         \
+    }                                                                           \
+  } while (0)
+#else
+#define TRACE(row) ((void)0)
+#endif
+
 __device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
   TileGeo g{tile * d.rows_per_tile, 0, 0, 0};
   if (d.spatial) {
@@ -680,37 +639,50 @@ __device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
   return g;
 }
 
+// ring position: stage / parity advance
+struct Ring {
+  int s;
+  uint32_t ph;
+  __device__ __forceinline__ void next(int n) {
+    if (++s == n) s = 0, ph ^= 1u;
+  }
+};
+
 __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   const int S = d.stages;
-  const int kSlotA = d.slot_a;
-  const int slot = kSlotA + d.slot_b;
-  const int Cc = d.Cc;
-  const int pbytes = 128 * Cc * 2;
-  uint8_t* wres = smem;                    // resident weights (d.resident), else empty
-  uint8_t* ring = smem + d.wres_bytes;
-  uint8_t* pbuf = ring + S * slot;
-  uint8_t* ones = pbuf + 2 * pbytes;
-  uint8_t* zeros = ones + 4096;            // zero B tile (zero-init MMA of a region no term reaches)
-  uint64_t* bars = reinterpret_cast<uint64_t*>(zeros + 4096);
-  uint64_t* full = bars;
-  uint64_t* empty = bars + S;
-  uint64_t* acc_full = bars + 2 * S;
-  uint64_t* acc_empty = acc_full + 2;
-  uint64_t* p_full = acc_empty + 2;
-  uint64_t* p_empty = p_full + 2;
-  uint64_t* out_full = p_empty + 2;
-  uint64_t* out_empty = out_full + 1;
-  uint64_t* wbar = out_empty + 1;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wbar + 1);
+  const int slot = d.slot_a + d.slot_b;
+  const int NS = d.ns;
+  uint8_t* wres = smem;
+  uint8_t* abuf = smem + d.off_abuf;
+  uint8_t* ring = smem + d.off_ring;
+  uint8_t* fring = smem + d.off_fring;
+  uint8_t* pbuf = smem + d.off_p;
+  uint8_t* ones = smem + d.off_ones;
+  uint8_t* zeros = smem + d.off_zeros;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + d.off_bars);
+  uint64_t* full = bars;                  // [S]
+  uint64_t* empty = full + S;             // [S]
+  uint64_t* ffull = empty + S;            // [fstages]
+  uint64_t* fempty = ffull + 4;           // [fstages]
+  uint64_t* acc_full = fempty + 4;        // [NS]
+  uint64_t* acc_empty = acc_full + 8;     // [NS]
+  uint64_t* p_full = acc_empty + 8;       // [4] (team * 2 + chunk parity)
+  uint64_t* p_empty = p_full + 4;         // [4]
+  uint64_t* out_full = p_empty + 4;       // [2]
+  uint64_t* out_empty = out_full + 2;     // [2]
+  uint64_t* wbar = out_empty + 2;
+  uint64_t* a_full = wbar + 1;            // [2] A buffers
+  uint64_t* a_empty = a_full + 2;         // [2]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(a_empty + 2);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  // constant A operand of the bias MMA: K columns 0 and 1 = 1.0 (bf16), one SW32 atom
+  // constant A operand of the zero-init MMA: K column 0 = 1.0 (bf16), one SW32 atom
   for (int i = threadIdx.x; i < 128 * 2; i += blockDim.x) {
     const int row = i / 2, ch = i % 2;
     uint4 v = make_uint4(0, 0, 0, 0);
-    if (ch == swz_chunk(row, 0, 16)) v.x = 0x3F803F80u;   // logical chunk 0 of this row
+    if (ch == swz_chunk(row, 0, 16)) v.x = 0x00003F80u;
     reinterpret_cast<uint4*>(ones)[i] = v;
   }
   for (int i = threadIdx.x; i < 4096 / 16; i += blockDim.x) reinterpret_cast<uint4*>(zeros)[i] = make_uint4(0, 0, 0, 0);
@@ -720,29 +692,39 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       mbar_init(&full[s], 1);
       mbar_init(&empty[s], 1);
     }
-    for (int b = 0; b < 2; ++b) {
-      mbar_init(&acc_full[b], 1);
-      mbar_init(&acc_empty[b], 32 * kEpiWarps);
-      mbar_init(&p_full[b], 32 * kEpiWarps);
-      mbar_init(&p_empty[b], 1);
+    for (int s = 0; s < 4; ++s) {
+      mbar_init(&ffull[s], 1);
+      mbar_init(&fempty[s], 1);
+      mbar_init(&p_full[s], kTeamArrivals);
+      mbar_init(&p_empty[s], 1);
     }
-    mbar_init(out_full, 1);
-    mbar_init(out_empty, 32 * kEpiWarps);
+    for (int s = 0; s < 8; ++s) {
+      mbar_init(&acc_full[s], 1);
+      mbar_init(&acc_empty[s], kTeamArrivals);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&out_full[b], 1);
+      mbar_init(&out_empty[b], kTeamArrivals);
+    }
     mbar_init(wbar, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&a_full[b], 1);
+      mbar_init(&a_empty[b], 1);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   // per-tile programs -> SMEM
   const TcProdOp* prod = d.prod;
   const TcMmaOpD* mprog = d.mma;
   if (d.prog_smem) {
-    uint8_t* ps = reinterpret_cast<uint8_t*>(bars) + 2048 + (d.npc ? 32768 : 0);
+    uint8_t* ps = smem + d.off_prog;
     const int n16 = (d.n_prod * (int)sizeof(TcProdOp) + d.n_mma * (int)sizeof(TcMmaOpD)) / 16;
     const uint4* src = reinterpret_cast<const uint4*>(d.prod);
     for (int i = threadIdx.x; i < n16; i += blockDim.x) reinterpret_cast<uint4*>(ps)[i] = src[i];
     prod = reinterpret_cast<const TcProdOp*>(ps);
     mprog = reinterpret_cast<const TcMmaOpD*>(ps + d.n_prod * sizeof(TcProdOp));
   }
-  if (warp == 0) {
+  if (warp == kFWarp) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(d.tmem_cols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -751,202 +733,199 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
-  const int U = units_per_tile(d);
+  const int U = d.units;
+#ifdef TEMCO_TRACE
+  int tn[kTraceRows] = {0};
+#endif
+  const bool has_w = d.resident || d.fres;
 
+  // register rebalancing inside the CTA's launch allocation (640 x 96): the role
+  // warpgroup (warps 16-19) drops to 40, the four epilogue warpgroups rise to
+  // 104 (128*40 + 512*104 <= 640*96); each branch is dominated by its setmaxnreg
+  if (warp >= kEpiWarps) {
+  asm volatile("setmaxnreg.dec.sync.aligned.u32 40;");
   if (warp == kProdWarp) {
-    // ------------------------------------------------------------ TMA producer
-    {   // whole warp; one elected lane issues (the resident preload runs in lane 0)
-      int stage = 0;
-      uint32_t phase = 0;
-      [[maybe_unused]] int n0 = 0, n1 = 0;
-      const char* dbase = reinterpret_cast<const char*>(&d);
-      if (d.resident && lane == 0) {
-        // every B box once: term atoms, level / member biases, F atoms
-        mbar_expect_tx(wbar, d.wres_bytes);
+    // ------------------------------------------------------------ TMA producer (A / B ring)
+    const char* dbase = reinterpret_cast<const char*>(&d);
+    if (has_w && lane == 0) {
+      // every resident box once: term atoms of the chunks a term reaches, F atoms
+      mbar_expect_tx(wbar, (uint32_t)((d.resident ? d.fbase : 0) + (d.fres ? d.nchunks * d.Np * 128 : 0)));
+      if (d.resident) {
         const int nall = d.npc ? d.mt1 : d.n_terms;
         for (int j = 0; j < nall; ++j) {
           const TcTerm& t = d.term[j];
-          const int ka_n = t.Rp / t.aw, bb = Cc * t.aw * 2;
+          const int ka_n = t.Rp / t.aw, bb = d.Cc * t.aw * 2;
           for (int c = 0; c < t.nhit; ++c)
             for (int ka = 0; ka < ka_n; ++ka)
-              tma_load_2d(wres + t.wres + (c * ka_n + ka) * bb, t.wmap, wbar, ka * t.aw, (t.cfirst + c) * Cc);
-        }
-        if (!d.gap)
-          for (int a = 0; a < d.Cpad / 64; ++a) tma_load_2d(wres + d.fres + a * d.Np * 128, d.fmap, wbar, a * 64, 0);
-      }
-      __syncwarp();
-      const int np = d.n_prod;
-      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-        const TileGeo gg = tile_geo(d, tile);
-        for (int i = 0; i < np; ++i) {
-          const TcProdOp o = prod[i];
-#ifdef TEMCO_TRACE
-          if (g_dbg & 1) {   // TMA-only experiment: the producer recycles its own stages
-            if (n0 >= S) mbar_wait(&full[stage], phase ^ 1);
-          } else
-#endif
-          mbar_wait(&empty[stage], phase ^ 1);
-          TRACE(0, n0);
-          mbar_expect_tx_w(&full[stage], o.bytes);
-          uint8_t* sa = ring + stage * slot;
-          if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
-            tma_load_4d_w(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.w0 * o.ts + o.dx, gg.h0 * o.ts + o.dy, gg.n0);
-          else if (o.kind & PK_A2D)
-            tma_load_2d_w(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.m0);
-          if (o.kind & PK_B) tma_load_2d_w(sa + kSlotA, dbase + o.bmap * 64, &full[stage], o.bx, o.by);
-          TRACE(1, n1);
-          if (++stage == S) stage = 0, phase ^= 1;
+              tma_load_2d(wres + t.wres + (c * ka_n + ka) * bb, t.wmap, wbar, ka * t.aw, (t.cfirst + c) * d.Cc);
         }
       }
-#ifdef TEMCO_TRACE
-      if ((g_dbg & 1) && lane == 0)
-        for (int k = 0; k < S && k < n0; ++k) {
-          const int i = n0 - 1 - k;
-          mbar_wait(&full[i % S], (i / S) & 1);
+      if (d.fres)
+        for (int c = 0; c < d.nchunks; ++c) tma_load_2d(wres + d.fbase + c * d.Np * 128, d.fmap, wbar, c * 64, 0);
+    }
+    __syncwarp();
+    Ring r{0, 0};
+    const int np = d.n_prod, na = d.n_aload;
+    int it = 0;
+    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+      const TileGeo gg = tile_geo(d, tile);
+      // the tile's reduced-input atoms, once, into A buffer ab
+      const int ab = d.nabuf == 2 ? (it & 1) : 0;
+      const int use = d.nabuf == 2 ? (it >> 1) : it;
+      mbar_wait(&a_empty[ab], ((uint32_t)use & 1u) ^ 1u);
+      mbar_expect_tx_w(&a_full[ab], (uint32_t)d.a_tx);
+      uint8_t* ba = abuf + ab * d.abytes;
+      for (int i = 0; i < na; ++i) {
+        const TcProdOp o = prod[i];
+        if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
+          tma_load_4d_w(ba + o.dst, dbase + o.amap * 64, &a_full[ab], o.ac, gg.w0 * o.ts + o.dx, gg.h0 * o.ts + o.dy,
+                        gg.n0);
+        else
+          tma_load_2d_w(ba + o.dst, dbase + o.amap * 64, &a_full[ab], o.ac, gg.m0);
+      }
+      TRACE(0);
+      // streamed weights: one ring stage per MMA op
+      for (int i = na; i < np; ++i) {
+        const TcProdOp o = prod[i];
+        mbar_wait(&empty[r.s], r.ph ^ 1);
+        mbar_expect_tx_w(&full[r.s], o.bytes);
+        tma_load_2d_w(ring + r.s * slot, dbase + o.bmap * 64, &full[r.s], o.bx, o.by);
+        r.next(S);
+      }
+    }
+  } else if (warp == kFWarp) {
+    // ------------------------------------------------------------ F ring producer (F not resident)
+    if (!d.gap && !d.fres) {
+      Ring r{0, 0};
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x)
+        for (int c = 0; c < d.nchunks; ++c) {
+          mbar_wait(&fempty[r.s], r.ph ^ 1);
+          mbar_expect_tx_w(&ffull[r.s], (uint32_t)(d.Np * 128));
+          tma_load_2d_w(fring + r.s * d.fslot, d.fmap, &ffull[r.s], c * 64, 0);
+          r.next(d.fstages);
         }
-#endif
     }
   } else if (warp == kMmaWarp) {
-#ifdef TEMCO_TRACE
-    if (g_dbg & 1) goto done;
-#endif
-    // ------------------------------------------------------------ MMA issuer
-    {   // whole warp (uniform control flow); elect.sync picks the issuing lane
-      int stage = 0;
-      uint32_t phase = 0;
-      uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
-      [[maybe_unused]] int n2 = 0, n3 = 0, n8 = 0, n9 = 0, n10 = 0, n11 = 0;
-      if (d.resident) mbar_wait(wbar, 0);
-      const int nm = d.n_mma;
-#ifdef TEMCO_TRACE
-      long long pc_acc = 0, pc_p = 0, pc_out = 0, pc_full = 0, pc_issue = 0, pc_n = 0, pc_dec = 0, pc_com = 0;
-      const long long pc_start = clock64();
-#endif
-      const uint64_t base16 = smem_u32(smem) >> 4;
-      auto exec = [&](const TcMmaOpD& o, int gu, uint32_t tile_iter) {
-#ifdef TEMCO_TRACE
-          long long _pt0 = 0;
-#endif
-          const uint32_t f = o.flags;
-          const int bs = (gu + o.unit) & 1;
-          if (f & MF_ACC_WAIT) {
-            PROF_T0();
-            mbar_wait(&acc_empty[bs], ((acc_par >> bs) & 1u) ^ 1u);
-            PROF_ADD(pc_acc);
-            TRACE(8, n8);
-            tc_fence_after();
-          }
-          if (f & MF_P_WAIT) {
-            TRACE(9, n9);
-            PROF_T0();
-            mbar_wait(&p_full[o.unit], (p_par >> o.unit) & 1u);
-            PROF_ADD(pc_p);
-            TRACE(10, n10);
-            tc_fence_after();
-          }
-          if (f & MF_OUT_WAIT) {
-            PROF_T0();
-            mbar_wait(out_empty, (tile_iter & 1) ^ 1);
-            PROF_ADD(pc_out);
-            tc_fence_after();
-          }
-          if (f & MF_SW) {
-            PROF_T0();
-            mbar_wait(&full[stage], phase);
-            PROF_ADD(pc_full);
-            TRACE(2, n2);
-            tc_fence_after();
-          }
-          PROF_T0();
-          const uint64_t st16 = (uint64_t)((stage * slot) >> 4);
-          const uint64_t ad = o.adesc + base16 + ((f & MF_SA) ? st16 : 0);
-          const uint64_t bd = o.bdesc + base16 + ((f & MF_SB) ? st16 : 0);
-          const uint32_t dt = tbase + o.tmem + ((f & MF_F) ? 0u : (uint32_t)(bs * d.ubuf));
-          const uint32_t acc0 = (f & MF_ZERO) ? 0u : 1u;
-          PROF_ADD(pc_dec);
-          {
-          PROF_T0();
-          mma_bf16_w(dt, ad, bd, o.idesc, acc0);
+    // ------------------------------------------------------------ GEMM1 issuer
+    if (has_w) mbar_wait(wbar, 0);
+    Ring st{0, 0};
+    Ring slr[2] = {{0, 0}, {0, 0}};      // per-team accumulator sub-rings
+    const int NST = NS / 2;
+    int it = 0;
+    const int nm = d.n_mma;
+    const uint64_t base16 = smem_u32(smem) >> 4;
+    const uint32_t ub = (uint32_t)d.ubuf;
+    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+      Ring& sl = slr[it & 1];
+      const int sbase = (it & 1) * NST;
+      const int ab = d.nabuf == 2 ? (it & 1) : 0;
+      const int use = d.nabuf == 2 ? (it >> 1) : it;
+      mbar_wait(&a_full[ab], (uint32_t)use & 1u);
+      TRACE(1);
+      tc_fence_after();
+      const uint64_t ab16 = (uint64_t)((ab * d.abytes) >> 4);
+      for (int i = 0; i < nm; ++i) {
+        const TcMmaOpD o = mprog[i];
+        const uint32_t f = o.flags;
+        if (f & MF_ACC_WAIT) {
+          mbar_wait(&acc_empty[sbase + sl.s], sl.ph ^ 1);
+          TRACE(2);
+          tc_fence_after();
+        }
+        if (f & MF_SW) {
+          mbar_wait(&full[st.s], st.ph);
+          tc_fence_after();
+        }
+        const uint64_t st16 = (uint64_t)((st.s * slot) >> 4);
+        const uint64_t ad = o.adesc + base16 + ((f & MF_AT) ? ab16 : 0);
+        const uint64_t bd = o.bdesc + base16 + ((f & MF_SB) ? st16 : 0);
+        const uint32_t dt = tbase + (uint32_t)(sbase + sl.s) * ub + o.tmem;
+        if (!(d.exp & 2)) {
+          mma_bf16_w(dt, ad, bd, o.idesc, (f & MF_ZERO) ? 0u : 1u);
           for (int k = 1; k < o.nk; ++k) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, o.idesc, 1u);
-          PROF_ADD(pc_issue);
-#ifdef TEMCO_TRACE
-          pc_n += o.nk;
-#endif
-          }
-          PROF_T0();
-          if (f & MF_SD) {
-            mma_commit_w(&empty[stage]);
-            if (++stage == S) stage = 0, phase ^= 1;
-          }
-          if (f & MF_ACC_COMMIT) {
-            mma_commit_w(&acc_full[bs]);
-            TRACE(3, n3);
-            acc_par ^= 1u << bs;
-          }
-          if (f & MF_P_COMMIT) {
-            mma_commit_w(&p_empty[o.unit]);
-            p_par ^= 1u << o.unit;
-          }
-          if (f & MF_OUT_COMMIT) {
-            mma_commit_w(out_full);
-            TRACE(11, n11);
-          }
-          PROF_ADD(pc_com);
-      };
-      if (d.mma_head > 0) {
-        // software pipeline over tiles: the unit ops of tile t+1 go ahead of the
-        // fconv ops of tile t (which wait for the epilogue's P tile of t)
-        const int nh = d.mma_head;
-        int t = blockIdx.x, gu = 0;
-        for (int i = 0; i < nh && t < d.ntiles; ++i) exec(mprog[i], gu, tile_iter);
-        for (; t < d.ntiles; t += gridDim.x) {
-          if (t + (int)gridDim.x < d.ntiles)
-            for (int i = 0; i < nh; ++i) exec(mprog[i], gu + d.units, tile_iter + 1);
-          for (int i = nh; i < nm; ++i) exec(mprog[i], gu, tile_iter);
-          gu += d.units;
-          ++tile_iter;
         }
-      } else {
-        int gu = 0;   // units issued so far (TMEM buffer parity)
-        for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
-          for (int i = 0; i < nm; ++i) exec(mprog[i], gu, tile_iter);
-          gu += d.units;
-          ++tile_iter;
+        if (f & MF_SD) {
+          mma_commit_w(&empty[st.s]);
+          st.next(S);
+        }
+        if (f & MF_ACC_COMMIT) {
+          mma_commit_w(&acc_full[sbase + sl.s]);
+          TRACE(3);
+          sl.next(NST);
         }
       }
-#ifdef TEMCO_TRACE
-      if (blockIdx.x == 0 && lane == 0) {
-        g_prof[0] = clock64() - pc_start;
-        g_prof[1] = pc_acc;
-        g_prof[2] = pc_p;
-        g_prof[3] = pc_out;
-        g_prof[4] = pc_full;
-        g_prof[5] = pc_issue;
-        g_prof[6] = pc_n;
-        g_prof[7] = pc_dec;
-        g_prof[8] = pc_com;
-      }
-#endif
+      mma_commit_w(&a_empty[ab]);   // the tile's A buffer is free once its MMAs complete
     }
-  } else if (warp < kEpiWarps) {
-#ifdef TEMCO_TRACE
-    if (g_dbg & 1) goto done;
-#endif
-    // ------------------------------------------------------------ epilogue (8 warps)
-    // warp w: TMEM lane quarter q = w % 4 (pixel rows 32q..32q+31), column half h = w / 4
-    const int q = warp & 3, h = warp >> 2;
+  } else if (warp == kG2Warp) {
+    // ------------------------------------------------------------ GEMM2 issuer: out += P_c F_c^T
+    if (!d.gap) {
+      if (d.fres) mbar_wait(wbar, 0);
+      Ring fr{0, 0};
+      uint32_t pph = 0;                 // phase bits of the 4 P buffers
+      const uint32_t idesc2 = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(d.Np >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+      const uint64_t pdesc0 = umma_desc(smem_u32(pbuf));
+      int it = 0;
+      for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
+        const int team = it & 1;
+        // output buffer: one per team (no == 2) or shared (no == 1); out_full /
+        // out_empty barriers are per team so every wait has a single in-order party
+        const int ob = d.no == 2 ? team : 0;
+        if (d.no == 2) {
+          mbar_wait(&out_empty[team], (((uint32_t)it >> 1) & 1u) ^ 1u);
+        } else if (it > 0) {
+          mbar_wait(&out_empty[(it - 1) & 1], ((uint32_t)(it - 1) >> 1) & 1u);
+        }
+        TRACE(11);
+        tc_fence_after();
+        const uint32_t dt = tbase + (uint32_t)(d.out_col + ob * d.Np);
+        int cp = 0;                     // chunk index among the tile's finished chunks
+        for (int u = 0; u < U; ++u) {
+          const Unit un = unit_at(d, u);
+          if (!un.last) continue;
+          const int pb = team * 2 + (cp & 1);
+          mbar_wait(&p_full[pb], (pph >> pb) & 1u);
+          TRACE(7);
+          pph ^= 1u << pb;
+          tc_fence_after();
+          uint64_t bdesc;
+          if (d.fres) {
+            bdesc = umma_desc(smem_u32(wres + d.fbase + un.c * d.Np * 128));
+          } else {
+            mbar_wait(&ffull[fr.s], fr.ph);
+            tc_fence_after();
+            bdesc = umma_desc(smem_u32(fring + fr.s * d.fslot));
+          }
+          const uint64_t adesc = pdesc0 + (uint64_t)((pb * 16384) >> 4);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) mma_bf16_w(dt, adesc + 2 * k, bdesc + 2 * k, idesc2, (cp | k) ? 1u : 0u);
+          mma_commit_w(&p_empty[pb]);
+          TRACE(8);
+          if (!d.fres) {
+            mma_commit_w(&fempty[fr.s]);
+            fr.next(d.fstages);
+          }
+          ++cp;
+        }
+        mma_commit_w(&out_full[team]);
+      }
+    }
+  }
+  } else {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 104;");
+    // ------------------------------------------------------------ epilogue teams
+    // team k takes the CTA's tiles k, k+2, ...; warp tw of a team: TMEM lane
+    // quarter q = warp % 4 (pixel rows 32q..32q+31), column half h (32 of the unit's 64)
+    const int team = warp / kTeamWarps, tw = warp % kTeamWarps;
+    const int q = warp & 3, h = tw >> 2;
     const int row = q * 32 + lane;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
-    const int half = Cc / 2;                          // columns per warp (32 or 64)
-    const int c_lo = h * half;
-    uint32_t acc_par = 0, p_par = 0, tile_iter = 0;   // phase parity bits per buffer (registers only)
-    [[maybe_unused]] int n4 = 0, n5 = 0, n6 = 0, n7 = 0;
-    const bool tr = threadIdx.x == 0;
-    (void)tr;
+    const int c_lo = h * 32;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
-    float* runbuf = reinterpret_cast<float*>(bars + 64);   // pooled member running max / sum (32 KB)
-    int gu = 0;   // units consumed so far (TMEM buffer parity)
-    for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x) {
+    uint32_t pph = 0;
+    int it = team;
+    const int NST = NS / 2, sbase = team * NST;
+    Ring sl{0, 0};                        // this team's accumulator sub-ring
+    for (int tile = blockIdx.x + team * gridDim.x; tile < d.ntiles; tile += 2 * gridDim.x, it += 2) {
       int64_t m = (int64_t)tile * d.rows_per_tile + row;
       bool mvalid = m < d.npix;
       int ho = 0, wo = 0;
@@ -960,211 +939,195 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
         mvalid = row < d.mused && n < d.nimg && ho < d.Ho && wo < d.Wo;
         m = ((int64_t)n * d.Ho + ho) * d.Wo + wo;
       }
-      for (int u0 = 0; u0 < U; gu += min(2, U - u0), u0 += 2) {
-        const int nb = min(2, U - u0);
-        for (int l = 0; l < d.n_levels; ++l) {
-          const bool last = l == d.n_levels - 1;
-          const bool relu = d.relu[l] != 0;
-          for (int bi = 0; bi < nb; ++bi) {
-            const Unit un = unit_at(d, u0 + bi);
-            const int bs = (gu + bi) & 1;
-            const uint32_t abit = 1u << bs;
-            mbar_wait(&acc_full[bs], (acc_par & abit) ? 1u : 0u);
-            if (tr) TRACE(4, n4);
-            acc_par ^= abit;
-            tc_fence_after();
-            const int pb = un.c & 1;
-            const bool writes_p = last && !d.gap && un.last;
-            if (writes_p) {
-              const uint32_t pbit = 1u << pb;
-              mbar_wait(&p_empty[pb], ((p_par & pbit) ? 1u : 0u) ^ 1u);
-              p_par ^= pbit;
-            }
-            const uint32_t ta = tbase + lane_off + bs * d.ubuf + c_lo;
-            uint8_t* P = pbuf + pb * pbytes;
-            // level / member bias (fp32, added here rather than through the tensor core)
-            const float* bsrc = p.params + (un.pooled ? d.mbias : d.lbias[l]) + un.c * Cc + c_lo;
-#ifdef TEMCO_TRACE
-            if (g_dbg & 2) {   // experiment: epilogue does no TMEM / SMEM work
-            } else
-#endif
-            if (un.pooled) {
-              // pooled member: fold the unit's taps into the running max / sum (half == 32);
-              // registers within the unit, a conflict-free SMEM slab across units
-              // (element i of thread t at run[i * 256 + t])
-              float* run = runbuf + threadIdx.x;
-              float cur[32];
-              const float4* b4 = reinterpret_cast<const float4*>(bsrc);
-              const bool fresh = un.tg == 0;
+      // accumulator slot of this tile's first unit-level
+      float t[32];   // running level value t_l (pooled units: running max / sum over taps)
+      int cp = 0;
+      for (int u = 0; u < U; ++u) {
+        const Unit un = unit_at(d, u);
+        const int col0 = un.c * d.Cc + c_lo;           // first restored channel of this thread
+        const int nl = un.pooled ? 1 : d.n_levels;
+        for (int l = 0; l < nl; ++l) {
+          const bool last = un.last && l == nl - 1;
+          mbar_wait(&acc_full[sbase + sl.s], sl.ph);
+          if (warp == 0) TRACE(4);
+          if (warp == kTeamWarps) TRACE(10);
+          tc_fence_after();
+          const uint32_t ta = tbase + lane_off + (uint32_t)((sbase + sl.s) * d.ubuf + c_lo);
+          if (un.pooled) {
+            // pooled member: fold this unit's taps (max of the raw accumulators, or
+            // sum of act(acc + b)) into the running value
+            if (un.tg == 0) {
 #pragma unroll
-              for (int i = 0; i < 32; ++i) cur[i] = fresh ? (d.mpool == 1 ? -INFINITY : 0.f) : run[i * 256];
-              for (int r = 0; r < un.nt; ++r) {
-                const int tap = un.tg * d.tpu + r;
-                const int hi = ho * d.ms - d.mp + tap / d.mk, wi = wo * d.ms - d.mp + tap % d.mk;
-                const bool valid = hi >= 0 && hi < d.mHin && wi >= 0 && wi < d.mWin;
-                uint32_t v[32];
-                tmem_ld32(ta + r * Cc, v);
-                tmem_wait_ld();
+              for (int i = 0; i < 32; ++i) t[i] = d.mpool == 1 ? -INFINITY : 0.f;
+            }
+            const float4* b4 = reinterpret_cast<const float4*>(p.params + d.mbias + col0);
+            for (int r = 0; r < un.nt; ++r) {
+              const int tap = un.tg * d.tpu + r;
+              const int hi = ho * d.ms - d.mp + tap / d.mk, wi = wo * d.ms - d.mp + tap % d.mk;
+              const bool valid = hi >= 0 && hi < d.mHin && wi >= 0 && wi < d.mWin;
+              uint32_t v[32];
+              tmem_ld32(ta + r * d.Cc, v);
+              tmem_wait_ld();
+              if (d.mpool == 1) {
+                if (valid) {
+#pragma unroll
+                  for (int i = 0; i < 32; ++i) t[i] = fmaxf(t[i], __uint_as_float(v[i]));
+                }
+              } else {
 #pragma unroll
                 for (int i4 = 0; i4 < 8; ++i4) {
                   const float4 bb = __ldg(b4 + i4);
                   const float bq[4] = {bb.x, bb.y, bb.z, bb.w};
 #pragma unroll
                   for (int k = 0; k < 4; ++k) {
-                    const int i = 4 * i4 + k;
-                    float x = __uint_as_float(v[i]) + bq[k];
-                    x = d.mrelu ? fmaxf(x, 0.f) : x;
-                    if (d.mpool == 1)
-                      cur[i] = valid ? fmaxf(cur[i], x) : cur[i];
-                    else
-                      cur[i] += x;
+                    const float z = __uint_as_float(v[4 * i4 + k]) + bq[k];
+                    t[4 * i4 + k] += d.mrelu ? fmaxf(z, 0.f) : z;
                   }
-                }
-              }
-              if (!un.last) {
-#pragma unroll
-                for (int i = 0; i < 32; ++i) run[i * 256] = cur[i];
-              } else {
-                // pooled value, + post-pool shift (BN after the pool), level activation
-                const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
-                const float4* pv4 = reinterpret_cast<const float4*>(p.params + (d.post >= 0 ? d.post : d.mbias) + un.c * Cc + c_lo);
-                const float pscale = d.post >= 0 ? 1.f : 0.f;
-                const int ch0 = c_lo / 8;
-#pragma unroll
-                for (int qq = 0; qq < 4; ++qq) {
-                  float f[8];
-                  const float4 pa = __ldg(pv4 + 2 * qq), pb2 = __ldg(pv4 + 2 * qq + 1);
-                  const float pq[8] = {pa.x, pa.y, pa.z, pa.w, pb2.x, pb2.y, pb2.z, pb2.w};
-#pragma unroll
-                  for (int i = 0; i < 8; ++i) {
-                    const float x = cur[8 * qq + i] * sc + pscale * pq[i];
-                    f[i] = relu ? fmaxf(x, 0.f) : x;
-                  }
-                  uint4 pk;
-                  pk.x = pack_bf16(f[0], f[1]);
-                  pk.y = pack_bf16(f[2], f[3]);
-                  pk.z = pack_bf16(f[4], f[5]);
-                  pk.w = pack_bf16(f[6], f[7]);
-                  *reinterpret_cast<uint4*>(P + row * 128 + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
-                }
-              }
-            } else if (!last) {
-              // t_l = relu(acc + b_l) back into TMEM for the next level's MMAs
-              for (int g = 0; g < half / 32; ++g) {
-                uint32_t a[32];
-                float bv[32];
-                load_bias32(bsrc + g * 32, bv);
-                tmem_ld32(ta + g * 32, a);
-                tmem_wait_ld();
-#pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                  const float x = __uint_as_float(a[i]) + bv[i];
-                  a[i] = __float_as_uint(relu ? fmaxf(x, 0.f) : x);
-                }
-                tmem_st32(ta + g * 32, a);
-              }
-              tmem_wait_st();
-            } else if (d.gap) {
-              // GAP root: per-image column means; tiles hold whole images so the
-              // summation order is fixed (deterministic, batch-invariant)
-              float* red = reinterpret_cast<float*>(pbuf + h * pbytes);
-              for (int g = 0; g < half / 32; ++g) {
-                uint32_t v[32];
-                float bv[32];
-                load_bias32(bsrc + g * 32, bv);
-                tmem_ld32(ta + g * 32, v);
-                tmem_wait_ld();
-#pragma unroll
-                for (int i = 0; i < 32; ++i) {
-                  const float x0 = __uint_as_float(v[i]) + bv[i];
-                  const float x = relu ? fmaxf(x0, 0.f) : x0;
-                  red[row * 32 + ((i + row) & 31)] = x;
-                }
-                asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
-                for (int idx = row; idx < d.ipt * 32; idx += 128) {
-                  const int ii = idx / 32, col = idx % 32;
-                  const int n = tile * d.ipt + ii;
-                  float acc = 0.f;
-                  for (int r = ii * d.hw; r < (ii + 1) * d.hw; ++r) acc += red[r * 32 + ((col + r) & 31)];
-                  const int cg = un.c * Cc + c_lo + g * 32 + col;
-                  if (n < d.nimg && cg < d.C) y[(int64_t)n * d.C + cg] = __float2bfloat16_rn(acc / (float)d.hw);
-                }
-                asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
-              }
-            } else {
-              // last level: P = bf16 relu(acc + b) -> SMEM (SW128 K-major atoms of 64 columns)
-              for (int g = 0; g < half / 32; ++g) {
-                uint32_t v[32];
-                float bv[32];
-                load_bias32(bsrc + g * 32, bv);
-                tmem_ld32(ta + g * 32, v);
-                tmem_wait_ld();
-                const int col = c_lo + g * 32;
-                uint8_t* atom = P + (col / 64) * 16384 + row * 128;
-                const int ch0 = (col % 64) / 8;
-#pragma unroll
-                for (int qq = 0; qq < 4; ++qq) {
-                  float f[8];
-#pragma unroll
-                  for (int i = 0; i < 8; ++i) {
-                    const float x = __uint_as_float(v[8 * qq + i]) + bv[8 * qq + i];
-                    f[i] = relu ? fmaxf(x, 0.f) : x;
-                  }
-                  uint4 pk;
-                  pk.x = pack_bf16(f[0], f[1]);
-                  pk.y = pack_bf16(f[2], f[3]);
-                  pk.z = pack_bf16(f[4], f[5]);
-                  pk.w = pack_bf16(f[6], f[7]);
-                  *reinterpret_cast<uint4*>(atom + (((ch0 + qq) ^ (row & 7)) * 16)) = pk;
                 }
               }
             }
             tc_fence_before();
-            if (tr) TRACE(5, n5);
-            mbar_arrive(&acc_empty[bs]);
-            if (writes_p) {
-              fence_proxy_async();
-              mbar_arrive(&p_full[pb]);
+            warp_arrive(&acc_empty[sbase + sl.s]);
+            sl.next(NST);
+            if (!un.last) continue;
+            // pooled value (+ member bias, act, for max), + post-pool shift -> t
+            const float4* p4 = reinterpret_cast<const float4*>(p.params + (d.post >= 0 ? d.post : d.mbias) + col0);
+            const float pscale = d.post >= 0 ? 1.f : 0.f;
+            const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
+#pragma unroll
+            for (int i4 = 0; i4 < 8; ++i4) {
+              const float4 bb = __ldg(b4 + i4), pp = __ldg(p4 + i4);
+              const float bq[4] = {bb.x, bb.y, bb.z, bb.w}, pq[4] = {pp.x, pp.y, pp.z, pp.w};
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                const int i = 4 * i4 + k;
+                float z = t[i] * sc;
+                if (d.mpool == 1) {
+                  z += bq[k];
+                  z = d.mrelu ? fmaxf(z, 0.f) : z;
+                }
+                t[i] = z + pscale * pq[k];
+              }
+            }
+          } else if (d.exp & 1) {
+            warp_arrive(&acc_empty[sbase + sl.s]);
+            sl.next(NST);
+          } else {
+            uint32_t v[32];
+            tmem_ld32(ta, v);
+            const float4* b4 = reinterpret_cast<const float4*>(p.params + d.lbias[l] + col0);
+            tmem_wait_ld();
+            tc_fence_before();
+            warp_arrive(&acc_empty[sbase + sl.s]);
+            if (warp == 0) TRACE(5);
+            sl.next(NST);
+#pragma unroll
+            for (int i4 = 0; i4 < 8; ++i4) {
+              const float4 bb = __ldg(b4 + i4);
+              const float bq[4] = {bb.x, bb.y, bb.z, bb.w};
+#pragma unroll
+              for (int k = 0; k < 4; ++k) {
+                const int i = 4 * i4 + k;
+                const float z = __uint_as_float(v[i]) + bq[k];
+                t[i] = l == 0 ? z : z + t[i];
+              }
             }
           }
+          const bool relu = d.relu[un.pooled ? 0 : l] != 0;
+          if (!last) {
+            if (relu) {
+#pragma unroll
+              for (int i = 0; i < 32; ++i) t[i] = fmaxf(t[i], 0.f);
+            }
+            continue;
+          }
+          if (d.gap) {
+            // GAP root: per-image column means; tiles hold whole images so the
+            // summation order is fixed (deterministic, batch-invariant)
+            float* red = reinterpret_cast<float*>(pbuf + (team * 2 + h) * 16384);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) red[row * 32 + ((i + row) & 31)] = relu ? fmaxf(t[i], 0.f) : t[i];
+            const int bar_id = 1 + team * 2 + h;
+            asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
+            for (int idx = row; idx < d.ipt * 32; idx += 128) {
+              const int ii = idx / 32, col = idx % 32;
+              const int n = tile * d.ipt + ii;
+              float acc = 0.f;
+              for (int rr = ii * d.hw; rr < (ii + 1) * d.hw; ++rr) acc += red[rr * 32 + ((col + rr) & 31)];
+              const int cg = col0 + col;
+              if (n < d.nimg && cg < d.C) y[(int64_t)n * d.C + cg] = __float2bfloat16_rn(acc / (float)d.hw);
+            }
+            asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
+            continue;
+          }
+          // last level: P = bf16 act(x) -> SMEM (one SW128 K-major atom per 64-channel unit)
+          const int pb = team * 2 + (cp & 1);
+          mbar_wait(&p_empty[pb], ((pph >> pb) & 1u) ^ 1u);
+          pph ^= 1u << pb;
+          uint8_t* prow = pbuf + pb * 16384 + row * 128;
+#pragma unroll
+          for (int qq = 0; qq < 4; ++qq) {
+            uint4 pk;
+            if (relu) {
+              pk.x = pack_bf16_relu(t[8 * qq + 0], t[8 * qq + 1]);
+              pk.y = pack_bf16_relu(t[8 * qq + 2], t[8 * qq + 3]);
+              pk.z = pack_bf16_relu(t[8 * qq + 4], t[8 * qq + 5]);
+              pk.w = pack_bf16_relu(t[8 * qq + 6], t[8 * qq + 7]);
+            } else {
+              pk.x = pack_bf16(t[8 * qq + 0], t[8 * qq + 1]);
+              pk.y = pack_bf16(t[8 * qq + 2], t[8 * qq + 3]);
+              pk.z = pack_bf16(t[8 * qq + 4], t[8 * qq + 5]);
+              pk.w = pack_bf16(t[8 * qq + 6], t[8 * qq + 7]);
+            }
+            const int ch = h * 4 + qq;
+            *reinterpret_cast<uint4*>(prow + ((ch ^ (row & 7)) * 16)) = pk;
+          }
+          fence_proxy_async();
+          warp_arrive(&p_full[pb]);
+          if (warp == 0) TRACE(6);
+          ++cp;
         }
       }
       if (d.gap) continue;
-      // output epilogue: column groups of 8 split between the two warp halves
-      if (tr) TRACE(6, n6);
-      mbar_wait(out_full, tile_iter & 1);
-      if (tr) TRACE(7, n7);
-      ++tile_iter;
+      // output epilogue: column groups of 8 split between the two column halves
+      const int ob = d.no == 2 ? team : 0;
+      mbar_wait(&out_full[team], (uint32_t)(it >> 1) & 1u);
+      if (warp == 0) TRACE(9);
       tc_fence_after();
       const int ng = d.Np / 8, gh = (ng + 1) / 2;
-#ifdef TEMCO_TRACE
-      const int gend = (g_dbg & 2) ? 0 : min(ng, (h + 1) * gh);
-#else
       const int gend = min(ng, (h + 1) * gh);
-#endif
-      for (int g = h * gh; g < gend; ++g) {
-        uint32_t v[8];
-        tmem_ld8(tbase + lane_off + 2 * d.ubuf + g * 8, v);
+      const uint32_t to = tbase + lane_off + (uint32_t)(d.out_col + ob * d.Np);
+      __nv_bfloat16* yrow = y + m * d.Nout;
+      const int gvalid = mvalid ? min(gend, d.Nout / 8) : 0;
+      for (int g0 = h * gh; g0 < gend; g0 += 2) {
+        uint32_t v0[8], v1[8];
+        tmem_ld8(to + g0 * 8, v0);
+        if (g0 + 1 < gend) tmem_ld8(to + (g0 + 1) * 8, v1);
         tmem_wait_ld();
-        if (mvalid && g * 8 < d.Nout) {
+        if (g0 < gvalid) {
           uint4 pk;
-          pk.x = pack_bf16(__uint_as_float(v[0]), __uint_as_float(v[1]));
-          pk.y = pack_bf16(__uint_as_float(v[2]), __uint_as_float(v[3]));
-          pk.z = pack_bf16(__uint_as_float(v[4]), __uint_as_float(v[5]));
-          pk.w = pack_bf16(__uint_as_float(v[6]), __uint_as_float(v[7]));
-          *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) = pk;
+          pk.x = pack_bf16(__uint_as_float(v0[0]), __uint_as_float(v0[1]));
+          pk.y = pack_bf16(__uint_as_float(v0[2]), __uint_as_float(v0[3]));
+          pk.z = pack_bf16(__uint_as_float(v0[4]), __uint_as_float(v0[5]));
+          pk.w = pack_bf16(__uint_as_float(v0[6]), __uint_as_float(v0[7]));
+          *reinterpret_cast<uint4*>(yrow + g0 * 8) = pk;
+        }
+        if (g0 + 1 < gvalid) {
+          uint4 pk;
+          pk.x = pack_bf16(__uint_as_float(v1[0]), __uint_as_float(v1[1]));
+          pk.y = pack_bf16(__uint_as_float(v1[2]), __uint_as_float(v1[3]));
+          pk.z = pack_bf16(__uint_as_float(v1[4]), __uint_as_float(v1[5]));
+          pk.w = pack_bf16(__uint_as_float(v1[6]), __uint_as_float(v1[7]));
+          *reinterpret_cast<uint4*>(yrow + (g0 + 1) * 8) = pk;
         }
       }
       tc_fence_before();
-      mbar_arrive(out_empty);
+      warp_arrive(&out_empty[team]);
     }
   }
-#ifdef TEMCO_TRACE
-done:
-#endif
   tc_fence_before();
   __syncthreads();
-  if (warp == 0) {
+  if (warp == kFWarp) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tbase), "r"(d.tmem_cols));
   }
@@ -1173,8 +1136,6 @@ done:
 }  // namespace
 
 #ifdef TEMCO_TRACE
-extern "C" void temco_debug_prof(long long* out) { cudaMemcpyFromSymbol(out, g_prof, sizeof(g_prof)); }
-extern "C" void temco_debug_set(int dbg) { cudaMemcpyToSymbol(g_dbg, &dbg, sizeof(int)); }
 extern "C" void temco_debug_trace(long long* out) {
   cudaMemcpyFromSymbol(out, g_trace, sizeof(g_trace));
   void* p = nullptr;
@@ -1207,7 +1168,7 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
     configured = true;
   }
   const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
-  // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
+  // >= 114 KB of shared memory keeps one CTA per SM (each owns all 512 TMEM columns)
   tc_chain_kernel<<<grid, kThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }
 

@@ -1,4 +1,6 @@
-// tcgen05 fused-group kernel (kernels_tc.cu): lowering + launch interface.
+// tcgen05 fused-group kernel, wide-group variant (kernels_tc_wide.cu): lowering + launch interface.
+// Used for groups whose per-tile reduced inputs do not fit in shared memory
+// (the level accumulates in TMEM over 128-channel units; see kernels_tc_wide.cu).
 //
 // Covers the groups whose restored tensor parses into a "level chain"
 // (chain_parse.h; reading R12, P:L305-317 + P:L321-333):
@@ -23,15 +25,15 @@
 #include "planner.h"
 
 namespace temco {
+namespace wide {
 
 constexpr int kTcMaxTerms = 40;    // reduced inputs (lconv leaves) per group, incl. pooled-member terms
 constexpr int kTcMaxLevels = 16;
-constexpr int kTcCc = 64;          // restored channels per unit (MMA N of GEMM1, one TMEM slot)
 
 struct TcTerm {
-  alignas(64) unsigned char tmap[128];   // 2D map of r [npix x R], box {aw, 128} (consecutive tiles)
-  alignas(64) unsigned char wmap[128];   // Lhat [Cpad x Rw], box {aw, Cc}
-  alignas(64) unsigned char tmap4[128];  // spatial tiles: 4D map of r [N, Hin, Win, R], box {aw, tw*ts, th*ts, tn}
+  alignas(64) unsigned char tmap[128];   // 2D map of r [npix x R], box {64, 128} (consecutive tiles)
+  alignas(64) unsigned char wmap[128];   // Lhat [Cpad x Rw], box {64, Cc}
+  alignas(64) unsigned char tmap4[128];  // spatial tiles: 4D map of r [N, Hin, Win, R], box {64, tw*ts, th*ts, tn}
   Loc r;                 // reduced input [N, Hin, Win, R] bf16 (arena)
   int32_t R, Rp;         // rank; padded to a multiple of the K atom
   int32_t aw;            // K atom width in elements (16 / 32 / 64 -> SW32 / SW64 / SW128 boxes)
@@ -46,7 +48,8 @@ struct TcTerm {
 
 // Per-tile programs (host-generated, identical for every tile of a group): the
 // producer and MMA roles replay flat op lists instead of re-deriving the unit /
-// level / term / tap / K-atom loop nest per stage.
+// level / term / tap / K-atom loop nest per stage (a single issuing thread is
+// latency-bound on that scalar code).
 enum : uint8_t { PK_A4D = 1, PK_A2D = 2, PK_B = 4 };
 struct TcProdOp {                 // one ring stage
   uint8_t kind, ts;               // PK_*; tile-base stride of a 4D A box
@@ -54,40 +57,42 @@ struct TcProdOp {                 // one ring stage
   int16_t ac, dx, dy;             // A coords: channel; tap offsets (4D: w0*ts+dx, h0*ts+dy)
   int16_t bx, by;                 // B coords
   uint16_t bytes;                 // expect_tx
-  uint16_t pad0;
-  uint32_t dst;                   // A-tile mode: byte offset of the atom in the tile's A buffer
-  uint16_t pad[4];
+  uint16_t pad[7];
 };
 static_assert(sizeof(TcProdOp) == 32, "TcProdOp layout");
 enum : uint16_t {
-  MF_ACC_WAIT = 1,      // first op of an accumulator slot: wait acc_empty[slot]
-  MF_AT = 2,            // A operand = atom of the tile-resident A buffer (+ buffer offset)
+  MF_ACC_WAIT = 1,      // wait acc_empty[bs] first
+  MF_P_WAIT = 2,        // wait p_full[unit]
+  MF_OUT_WAIT = 4,      // wait out_empty
   MF_SW = 8,            // wait full[stage]
   MF_SA = 16,           // A operand = current stage slot A
   MF_SB = 32,           // B operand = current stage slot B
   MF_SD = 64,           // commit empty[stage] + advance after
-  MF_ONES = 128,        // A = constant ones tile (zero-init MMA)
-  MF_ZERO = 512,        // first MMA into a TMEM region (k == 0 does not accumulate)
-  MF_ACC_COMMIT = 1024, // last op of the slot: commit acc_full[slot], advance the slot
+  MF_ONES = 128,        // A = constant ones tile (bias MMA)
+  MF_F = 256,           // fconv MMA: A = P[unit] + aoff, D = output region, N = Np
+  MF_ZERO = 512,        // first MMA of the accumulator (k == 0 does not accumulate)
+  MF_ACC_COMMIT = 1024, // commit acc_full[bs] after
+  MF_P_COMMIT = 2048,   // commit p_empty[unit] after
+  MF_OUT_COMMIT = 4096, // commit out_full after
   MF_BRES = 8192,       // B = resident weights + boff
   MF_BZERO = 16384,     // B = zero tile (with MF_ONES | MF_ZERO: zero-initialise the region)
 };
 struct TcMmaOp {
   uint16_t flags;
-  uint8_t nk;                     // K=16 steps
+  uint8_t unit, nk;               // unit index in the tile (TMEM buffer parity) or P buffer; K=16 steps
   uint8_t la, lb;                 // K-atom widths (layouts) of A and B
-  uint16_t tcol;                  // TMEM column offset inside the slot (tap region)
-  uint32_t boff;
-  uint32_t aoff;                  // A-tile mode: atom offset in the A buffer
+  uint16_t tcol;                  // TMEM column offset inside the unit buffer
+  uint32_t aoff, boff;
 };
+static_assert(sizeof(TcMmaOp) == 16, "TcMmaOp layout");
 // device form: UMMA descriptors precomputed on the host relative to the
 // 1024-aligned SMEM base (start-address field = offset >> 4); the issuer only
 // adds (base >> 4) and, for ring operands, (stage * slot) >> 4
 struct TcMmaOpD {
   uint64_t adesc, bdesc;
-  uint32_t idesc, tmem;           // instruction descriptor; TMEM column inside the slot
+  uint32_t idesc, tmem;           // instruction descriptor; TMEM column (unit ops: + buffer * ubuf)
   uint16_t flags;
-  uint8_t nk, pad0;
+  uint8_t unit, nk;
   uint32_t pad;
 };
 static_assert(sizeof(TcMmaOpD) == 32, "TcMmaOpD layout");
@@ -95,11 +100,17 @@ static_assert(sizeof(TcMmaOpD) == 32, "TcMmaOpD layout");
 struct TcChainDesc {
   TcTerm term[kTcMaxTerms];
   alignas(64) unsigned char fmap[128];   // F [Np x Cpad], box {64, Np}
+  // level biases enter the accumulator through the tensor core: a constant
+  // SMEM "ones" A tile (K columns 0, 1 = 1) times B = [b_hi, b_lo] per channel
+  alignas(64) unsigned char bmap[kTcMaxLevels][128];   // [Cpad x 8] bf16, box {64, Cc}
+  alignas(64) unsigned char bmapm[128];                 // pooled member bias
+  int64_t boff[kTcMaxLevels];            // tc weight pool offsets of the bias matrices
+  int64_t boffm;
   int64_t lbias[kTcMaxLevels], mbias;    // fp32 params offsets of the level / member biases (epilogue adds)
   int32_t n_terms, n_levels;             // outer (level) terms: [0, n_terms)
   int32_t lvl_end[kTcMaxLevels];         // terms [lvl_end[l-1], lvl_end[l]) accumulate into level l
   int32_t relu[kTcMaxLevels];
-  int32_t C, Cpad, Cc, nchunks;          // restored width, padded, unit width (kTcCc)
+  int32_t C, Cpad, Cc, nchunks;          // restored width, padded, chunk width (64 | 128)
   int32_t Nout, Np;                      // fconv outputs, padded to a multiple of 16
   int64_t npix;                          // root-resolution pixels
   int32_t ntiles;
@@ -112,30 +123,24 @@ struct TcChainDesc {
   // pooled member in channel chunks [0, npc): per-tap MMA regions (tpu taps per
   // unit, ntg tap groups), then pool, + post-shift (params, fp32 [npc*Cc]), act
   int32_t npc, mpool, mk, ms, mp, mtaps, mrelu, mt0, mt1, mHin, mWin;
-  int32_t tpu, ntg, ubuf;                // ubuf = TMEM columns of one accumulator slot (tpu * Cc)
+  int32_t tpu, ntg, ubuf;                // ubuf = TMEM columns of one unit buffer
   int64_t post;                          // params offset of the post-pool shift, -1 none
   int64_t F;                             // tc weight pool offset of F
+  int64_t Fb;                            // unused (fconv factors carry no bias)
   Loc y;                                 // output [npix, Nout] bf16, or [N, C] for GAP
-  // accumulator slots (TMEM ring, one per unit-level) and output buffers
-  int32_t ns, no, out_col, spt;          // slots; output buffers (Np columns each) from column out_col; slots / tile
-  // resident weights: B boxes (every term atom of the chunks it reaches) and/or
-  // F atoms loaded once per CTA; otherwise streamed (B with A through the ring,
-  // F through its own ring)
-  int32_t resident, fres, wres_bytes;
-  int32_t fbase;                         // F atoms: [nchunks] x (Np x 64) at this byte offset (resident)
-  int32_t fstages, fslot;                // F ring (not resident)
+  // resident weights (every B operand fits in SMEM): loaded once per CTA, the
+  // ring then carries only A tiles.  Avoids all 148 SMs re-reading the same
+  // few weight lines through TMA every stage (L2 same-line contention).
+  int32_t resident, wres_bytes;
+  int32_t bres[kTcMaxLevels], bresm;     // bias boxes: [nchunks] x (Cc x 16), byte offsets
+  int32_t fres;                          // F boxes: [Cpad / 64] x (Np x 64)
   int64_t prog_off;                      // tc weight pool offset (elements) of [prod ops][mma ops]
   int32_t n_prod, n_mma, units;          // ops per tile; units per tile
+  int32_t mma_head;                      // > 0: pipelined MMA order, unit ops = mma[0, mma_head)
   int32_t prog_smem;                     // > 0: programs copied to SMEM at kernel start (bytes reserved)
   const TcProdOp* prod;                  // device pointers (tc_finalize)
   const TcMmaOpD* mma;
   int32_t stages, slot_a, slot_b;        // smem ring depth, bytes of one A / B slot
-  // A-tile mode: every reduced-input atom of a tile is loaded once into one of
-  // nabuf A buffers (abytes each) and read by all units' MMAs
-  int32_t atr, n_aload, nabuf, abytes, a_tx;
-  int32_t exp;                           // experiment bits (TEMCO_TC_EXP): 1 epilogue skips TMEM work, 2 no MMAs
-  // SMEM layout (byte offsets from the 1024-aligned base)
-  int32_t off_abuf, off_ring, off_fring, off_p, off_ones, off_zeros, off_bars, off_prog;
   int32_t smem_bytes, tmem_cols;
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
 };
@@ -146,4 +151,5 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
                  std::string& err);
 void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s);
 
+}  // namespace wide
 }  // namespace temco
