@@ -318,7 +318,18 @@ void lower(temco_plan_s* P) {
         e.kernel = "none";
         break;
       case OP_CONV: {
-        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && ir.nodes[ir.oin[s.out][0]].C % 8 == 0 &&
+        const bool rank_conv = [&] {   // reduced-rank core conv: the memory-bound SIMT kernel
+          if (!P->bf16 || getenv("TEMCO_CONV_TC")) return false;
+          const Node& x = ir.nodes[ir.oin[s.out][0]];
+          ConvDesc c{};
+          c.x = tensor_loc(P, x.id);
+          c.y = tensor_loc(P, s.out);
+          c.N = N; c.H = x.H; c.W = x.W; c.C = x.C;
+          c.Ho = v.H; c.Wo = v.W; c.K = v.C;
+          c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = v.groups;
+          return conv_rank_ok(c);
+        }();
+        if (!rank_conv && P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && ir.nodes[ir.oin[s.out][0]].C % 8 == 0 &&
             conv_tc_lower(ir, s.out, P->loc, P->tcw_h, P->params_h, e.ctc)) {
           e.kind = K_CONV_TC;
           e.kernel = "tc_conv";
@@ -335,7 +346,7 @@ void lower(temco_plan_s* P) {
         c.w = push_params(P, repack_conv(v, x.C));
         c.b = push_params(P, v.b);
         e.kind = K_CONV;
-        e.kernel = v.groups > 1 ? "simt_dwconv" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
+        e.kernel = v.groups > 1 ? "simt_dwconv" : conv_rank_ok(c) ? "simt_conv_rank" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
         e.launches = 1;
         break;
       }
@@ -487,7 +498,9 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
     switch (e.kind) {
       case K_NONE: break;
       case K_CONV:
-        if (conv_small_ok(e.conv))
+        if (conv_rank_ok(e.conv))
+          launch_conv_rank(e.conv, rp, st);
+        else if (conv_small_ok(e.conv))
           launch_conv_small(e.conv, rp, st);
         else
           launch_conv(e.conv, rp, st);

@@ -10,6 +10,8 @@ namespace temco {
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_small_ok(const ConvDesc& d);   // small-Cin direct conv applies (stem on the image)
 void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
+bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)
+void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_linear(const LinearDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_group_simt(const GroupDesc& d, const GNode* nodes, const int32_t* children, const RunPtrs& p,

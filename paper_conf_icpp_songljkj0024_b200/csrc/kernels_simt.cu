@@ -122,6 +122,116 @@ int conv_small_smem(const ConvDesc& d) {
 }
 
 // ---------------------------------------------------------------------------
+// reduced-rank core convolution (Tucker core K x K on R_in -> R_out channels,
+// the 1x1 cores, CP pointwise factors): memory-bound work (AI < 150 flop/B at
+// R <= 64), so a direct SIMT kernel with coalesced 16-byte staging beats an
+// implicit GEMM whose tiles are dominated by tensor-core issue latency.
+// CTA: a box of ni images x th rows x tw columns of output pixels (one pixel
+// per thread), kc output channels (gridDim.y = K / kc).  The input footprint
+// is staged in SMEM as bf16 (16-byte row segments), the weights as fp32
+// [tap][cin][kc] (warp-broadcast float4 reads); fp32 accumulation.
+// ---------------------------------------------------------------------------
+struct RankTile {
+  int ni, th, tw, kc, fr, fc;   // images, rows, cols per tile; output channels per CTA; footprint rows / cols
+  int tiles_w, tiles_h, tiles_n;
+  int smem;
+};
+
+__host__ __device__ inline RankTile rank_tile(const ConvDesc& d) {
+  RankTile t;
+  t.tw = d.Wo <= 32 ? d.Wo : (d.Wo + (d.Wo + 31) / 32 - 1) / ((d.Wo + 31) / 32);
+  t.th = 256 / t.tw < d.Ho ? 256 / t.tw : d.Ho;
+  t.ni = (t.th == d.Ho) ? (256 / (t.tw * t.th) < d.N ? 256 / (t.tw * t.th) : d.N) : 1;
+  if (t.ni < 1) t.ni = 1;
+  t.kc = d.K <= 16 ? d.K : 16;
+  t.fr = (t.th - 1) * d.sh + d.kh;
+  t.fc = (t.tw - 1) * d.sw + d.kw;
+  t.tiles_w = (d.Wo + t.tw - 1) / t.tw;
+  t.tiles_h = (d.Ho + t.th - 1) / t.th;
+  t.tiles_n = (d.N + t.ni - 1) / t.ni;
+  t.smem = t.ni * t.fr * t.fc * d.C * 2 + d.kh * d.kw * d.C * t.kc * 4;
+  return t;
+}
+
+template <int KC>
+__global__ void __launch_bounds__(256) conv_rank_kernel(ConvDesc d, RankTile t, RunPtrs p) {
+  extern __shared__ __align__(16) unsigned char smr[];
+  const int Cin = d.C;
+  const int taps = d.kh * d.kw;
+  float* ws = reinterpret_cast<float*>(smr);                                   // [tap][cin][KC]
+  __nv_bfloat16* xs = reinterpret_cast<__nv_bfloat16*>(smr + taps * Cin * KC * 4);   // [img][fr][fc][cin]
+  const int tile = blockIdx.x;
+  const int tw_i = tile % t.tiles_w, th_i = (tile / t.tiles_w) % t.tiles_h, tn_i = tile / (t.tiles_w * t.tiles_h);
+  const int n0 = tn_i * t.ni, h0 = th_i * t.th, w0 = tw_i * t.tw;
+  const int k0 = blockIdx.y * KC;
+  // weights [k][tap][cin] (params) -> [tap][cin][k] (SMEM, fp32)
+  for (int i = threadIdx.x; i < taps * Cin * KC; i += blockDim.x) {
+    const int k = i % KC, tc = i / KC;
+    ws[i] = p.params[d.w + (int64_t)(k0 + k) * taps * Cin + tc];
+  }
+  // input footprint, 16-byte vectors (Cin % 8 == 0), zero padding
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
+  const int hi0 = h0 * d.sh - d.ph, wi0 = w0 * d.sw - d.pw;
+  const int cv = Cin / 8;
+  const int nvec = t.ni * t.fr * t.fc * cv;
+  for (int i = threadIdx.x; i < nvec; i += blockDim.x) {
+    const int c8 = i % cv, pix = i / cv;
+    const int col = pix % t.fc, row = (pix / t.fc) % t.fr, img = pix / (t.fc * t.fr);
+    const int n = n0 + img, hi = hi0 + row, wi = wi0 + col;
+    uint4 v = make_uint4(0, 0, 0, 0);
+    if (n < d.N && hi >= 0 && hi < d.H && wi >= 0 && wi < d.W)
+      v = __ldg(reinterpret_cast<const uint4*>(x + (((int64_t)n * d.H + hi) * d.W + wi) * Cin) + c8);
+    reinterpret_cast<uint4*>(xs)[i] = v;
+  }
+  __syncthreads();
+  const int px = threadIdx.x;
+  const int img = px / (t.th * t.tw), r = (px / t.tw) % t.th, c = px % t.tw;
+  const int n = n0 + img, ho = h0 + r, wo = w0 + c;
+  if (img >= t.ni || n >= d.N || ho >= d.Ho || wo >= d.Wo) return;
+  float acc[KC];
+#pragma unroll
+  for (int k = 0; k < KC; ++k) acc[k] = d.b >= 0 ? p.params[d.b + k0 + k] : 0.f;
+  const __nv_bfloat16* xi = xs + ((size_t)img * t.fr * t.fc) * Cin;
+  for (int a = 0; a < d.kh; ++a)
+    for (int bb = 0; bb < d.kw; ++bb) {
+      const __nv_bfloat16* xp = xi + ((size_t)(r * d.sh + a) * t.fc + (c * d.sw + bb)) * Cin;
+      const float* wp = ws + (a * d.kw + bb) * Cin * KC;
+      for (int c8 = 0; c8 < cv; ++c8) {
+        const uint4 u = reinterpret_cast<const uint4*>(xp)[c8];
+        const uint32_t uw[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const float xv = __uint_as_float(j & 1 ? (uw[j / 2] & 0xFFFF0000u) : (uw[j / 2] << 16));
+          const float4* w4 = reinterpret_cast<const float4*>(wp + (c8 * 8 + j) * KC);
+#pragma unroll
+          for (int k4 = 0; k4 < KC / 4; ++k4) {
+            const float4 w = w4[k4];
+            acc[4 * k4 + 0] = fmaf(xv, w.x, acc[4 * k4 + 0]);
+            acc[4 * k4 + 1] = fmaf(xv, w.y, acc[4 * k4 + 1]);
+            acc[4 * k4 + 2] = fmaf(xv, w.z, acc[4 * k4 + 2]);
+            acc[4 * k4 + 3] = fmaf(xv, w.w, acc[4 * k4 + 3]);
+          }
+        }
+      }
+    }
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+  __nv_bfloat16* yp = y + (((int64_t)n * d.Ho + ho) * d.Wo + wo) * d.K + k0;
+#pragma unroll
+  for (int k8 = 0; k8 < KC / 8; ++k8) {
+    uint4 pk;
+    __nv_bfloat162 h0v = __floats2bfloat162_rn(acc[8 * k8 + 0], acc[8 * k8 + 1]);
+    __nv_bfloat162 h1v = __floats2bfloat162_rn(acc[8 * k8 + 2], acc[8 * k8 + 3]);
+    __nv_bfloat162 h2v = __floats2bfloat162_rn(acc[8 * k8 + 4], acc[8 * k8 + 5]);
+    __nv_bfloat162 h3v = __floats2bfloat162_rn(acc[8 * k8 + 6], acc[8 * k8 + 7]);
+    pk.x = *reinterpret_cast<uint32_t*>(&h0v);
+    pk.y = *reinterpret_cast<uint32_t*>(&h1v);
+    pk.z = *reinterpret_cast<uint32_t*>(&h2v);
+    pk.w = *reinterpret_cast<uint32_t*>(&h3v);
+    reinterpret_cast<uint4*>(yp)[k8] = pk;
+  }
+}
+
+// ---------------------------------------------------------------------------
 // direct NHWC convolution: one thread per output element, output channel
 // fastest so a warp shares its input pixels (broadcast loads)
 // ---------------------------------------------------------------------------
@@ -416,6 +526,29 @@ __global__ void group_gap_kernel(GroupDesc d, GCtx g) {
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.K;
   conv_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
+}
+
+bool conv_rank_ok(const ConvDesc& d) {
+  if (d.groups != 1 || d.x.dtype != DT_BF16 || d.y.dtype != DT_BF16) return false;
+  // measured on B200 against the tcgen05 implicit GEMM (kernels_conv.cu): the
+  // direct kernel wins while one 8-channel output group covers the layer
+  if (d.C % 8 || d.C > 64 || d.K != 8) return false;
+  return rank_tile(d).smem <= 160 * 1024;
+}
+
+void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  if (!configured) {
+    cudaFuncSetAttribute(conv_rank_kernel<8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024);
+    cudaFuncSetAttribute(conv_rank_kernel<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024);
+    configured = true;
+  }
+  const RankTile t = rank_tile(d);
+  dim3 grid((unsigned)(t.tiles_n * t.tiles_h * t.tiles_w), (unsigned)(d.K / t.kc));
+  if (t.kc == 8)
+    conv_rank_kernel<8><<<grid, 256, t.smem, s>>>(d, t, p);
+  else
+    conv_rank_kernel<16><<<grid, 256, t.smem, s>>>(d, t, p);
 }
 
 bool conv_small_ok(const ConvDesc& d) {
