@@ -59,7 +59,7 @@ def build(verbose: bool = False) -> str:
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose), SOURCES))
     if _stale(LIB, objs):
-        cmd = [NVCC] + GENCODE + ["-shared", "-o", LIB] + objs
+        cmd = [NVCC] + GENCODE + ["-shared", "-o", LIB] + objs + ["-L/usr/local/cuda/lib64", "-lcublas"]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")

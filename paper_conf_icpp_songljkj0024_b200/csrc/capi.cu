@@ -18,6 +18,8 @@
 #include "tc.h"
 #include "tc_wide.h"
 
+#include <cublas_v2.h>
+
 using namespace temco;
 
 namespace {
@@ -73,6 +75,9 @@ struct temco_plan_s {
   int32_t* gchild_d = nullptr;
   uint16_t* tcw_d = nullptr;
   char* arena_d = nullptr;
+  cublasHandle_t blas = nullptr;   // plain library GEMMs (the classifier head)
+  float* lin_ws_d = nullptr;       // fp32 GEMM result before the bias / ReLU / cast epilogue
+  int64_t lin_ws_elems = 0;
   int64_t arena_bytes = 0;
   int64_t in_bytes = 0, out_bytes = 0;
   void* host_in_d = nullptr;
@@ -345,8 +350,16 @@ void lower(temco_plan_s* P) {
         c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = v.groups;
         c.w = push_params(P, repack_conv(v, x.C));
         c.b = push_params(P, v.b);
+        c.w2 = -1;
+        if (v.groups == x.C && v.C == x.C) {   // depthwise: [tap][C] copy for the vectorised kernel
+          std::vector<float> w2((size_t)v.kh * v.kw * v.C);
+          const std::vector<float>& src = *v.w;
+          for (int k = 0; k < v.C; ++k)
+            for (int t = 0; t < v.kh * v.kw; ++t) w2[(size_t)t * v.C + k] = src[(size_t)k * v.kh * v.kw + t];
+          c.w2 = push_params(P, w2);
+        }
         e.kind = K_CONV;
-        e.kernel = v.groups > 1 ? "simt_dwconv" : conv_rank_ok(c) ? "simt_conv_rank" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
+        e.kernel = v.groups > 1 ? (dwconv_vec_ok(c) ? "simt_dwconv_vec" : "simt_dwconv") : conv_rank_ok(c) ? "simt_conv_rank" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
         e.launches = 1;
         break;
       }
@@ -366,8 +379,24 @@ void lower(temco_plan_s* P) {
         l.w = push_params(P, w);
         l.b = push_params(P, v.b);
         l.relu = 0;
+        l.wb = -1;
+        l.blas = 0;
         e.kind = K_LINEAR;
         e.kernel = "simt_linear";
+        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && l.x.dtype == DT_BF16) {
+          // bf16 plans: the head is a plain GEMM -> cuBLAS (bf16 operands, fp32 accumulate)
+          while (P->tcw_h.size() % 512) P->tcw_h.push_back(0);
+          l.wb = (int64_t)P->tcw_h.size();
+          for (float f : w) {
+            uint32_t u;
+            memcpy(&u, &f, 4);
+            u += 0x7FFF + ((u >> 16) & 1);
+            P->tcw_h.push_back((uint16_t)(u >> 16));
+          }
+          l.blas = 1;
+          P->lin_ws_elems = std::max<int64_t>(P->lin_ws_elems, (int64_t)l.N * l.O);
+          e.kernel = "blas_linear";
+        }
         e.launches = 1;
         break;
       }
@@ -484,6 +513,8 @@ void free_device(temco_plan_s* P) {
   cudaFree(P->arena_d);
   cudaFree(P->host_in_d);
   cudaFree(P->host_out_d);
+  cudaFree(P->lin_ws_d);
+  if (P->blas) cublasDestroy(P->blas);
 }
 
 RunPtrs run_ptrs(temco_plan_s* P, const void* in, void* out) {
@@ -498,7 +529,9 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
     switch (e.kind) {
       case K_NONE: break;
       case K_CONV:
-        if (conv_rank_ok(e.conv))
+        if (dwconv_vec_ok(e.conv))
+          launch_dwconv_vec(e.conv, rp, st);
+        else if (conv_rank_ok(e.conv))
           launch_conv_rank(e.conv, rp, st);
         else if (conv_small_ok(e.conv))
           launch_conv_small(e.conv, rp, st);
@@ -506,7 +539,21 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
           launch_conv(e.conv, rp, st);
         break;
       case K_EW: launch_ew(e.ew, rp, st); break;
-      case K_LINEAR: launch_linear(e.lin, rp, st); break;
+      case K_LINEAR:
+        if (e.lin.blas) {
+          // y = W x: column-major C[O x N] = W^T[O x K] * x[K x N] (W row-major [O][K], x row-major [N][K])
+          const float one = 1.f, zero = 0.f;
+          const void* xin = loc_ptr(e.lin.x, rp);
+          if (cublasSetStream(P->blas, st) != CUBLAS_STATUS_SUCCESS ||
+              cublasGemmEx(P->blas, CUBLAS_OP_T, CUBLAS_OP_N, e.lin.O, e.lin.N, e.lin.K, &one, P->tcw_d + e.lin.wb,
+                           CUDA_R_16BF, e.lin.K, xin, CUDA_R_16BF, e.lin.K, &zero, P->lin_ws_d, CUDA_R_32F, e.lin.O,
+                           CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT) != CUBLAS_STATUS_SUCCESS)
+            return set_err(TEMCO_ERR_CUDA, "cublasGemmEx (classifier head)");
+          launch_linear_epilogue(e.lin, P->lin_ws_d, rp, st);
+        } else {
+          launch_linear(e.lin, rp, st);
+        }
+        break;
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
       case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
@@ -620,6 +667,18 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
       free_device(P);
       delete P;
       return set_err(TEMCO_ERR_OUT_OF_MEMORY, "arena cudaMalloc");
+    }
+    if (P->lin_ws_elems > 0) {
+      if (cudaMalloc(&P->lin_ws_d, P->lin_ws_elems * sizeof(float)) != cudaSuccess) {
+        free_device(P);
+        delete P;
+        return set_err(TEMCO_ERR_OUT_OF_MEMORY, "GEMM workspace cudaMalloc");
+      }
+      if (cublasCreate(&P->blas) != CUBLAS_STATUS_SUCCESS) {
+        free_device(P);
+        delete P;
+        return set_err(TEMCO_ERR_CUDA, "cublasCreate");
+      }
     }
     std::string terr;
     for (auto& e : P->exec)

@@ -40,6 +40,7 @@ struct ConvDesc {             // direct NHWC convolution (fconv on full tensors,
   int32_t kh, kw, sh, sw, ph, pw, groups;
   int64_t w;                  // params offset: [K][kh][kw][C/groups]
   int64_t b;                  // params offset or -1
+  int64_t w2;                 // depthwise: params offset of the weights in [kh][kw][C] order, -1 none
 };
 
 enum EwKind : int32_t { EW_BN, EW_RELU, EW_SILU, EW_ADD, EW_CONCAT, EW_MAXPOOL, EW_AVGPOOL, EW_GAP };
@@ -62,6 +63,8 @@ struct LinearDesc {           // y[n, o] = b[o] + sum_k W[o, k] x[n, k], x flatt
   int32_t N, K, O;
   int64_t w, b;               // params offsets; W already permuted to NHWC order
   int32_t relu;               // fused ReLU epilogue (a following standalone relu is folded in)
+  int64_t wb;                 // bf16 plans: tc weight pool offset of the bf16 copy of W (cuBLAS GEMM), -1 none
+  int32_t blas;               // 1: y = epilogue(cublasGemmEx(W, x)) (plain library GEMM, fp32 accumulate)
 };
 
 // ---------------------------------------------------------------------------

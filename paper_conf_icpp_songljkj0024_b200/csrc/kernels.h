@@ -10,10 +10,14 @@ namespace temco {
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_small_ok(const ConvDesc& d);   // small-Cin direct conv applies (stem on the image)
 void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
+bool dwconv_vec_ok(const ConvDesc& d);   // depthwise bf16, C % 8 == 0: vectorised kernel
+void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)
 void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_linear(const LinearDesc& d, const RunPtrs& p, cudaStream_t s);
+// bias + ReLU + cast of the fp32 GEMM result ws [N x O] into y
+void launch_linear_epilogue(const LinearDesc& d, const float* ws, const RunPtrs& p, cudaStream_t s);
 void launch_group_simt(const GroupDesc& d, const GNode* nodes, const int32_t* children, const RunPtrs& p,
                        cudaStream_t s);
 

@@ -232,6 +232,58 @@ __global__ void __launch_bounds__(256) conv_rank_kernel(ConvDesc d, RankTile t, 
 }
 
 // ---------------------------------------------------------------------------
+// depthwise (CP factor) convolution, bf16 NHWC: memory-bound, so one thread
+// per (output pixel, 8-channel group) with 16-byte vector loads / stores --
+// consecutive threads cover consecutive 16-byte chunks of a pixel row (fully
+// coalesced), the kh x kw taps of neighbouring threads hit L1 / L2.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) dwconv_vec_kernel(ConvDesc d, RunPtrs p) {
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const int cg = d.C / 8;
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * cg;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int g = (int)(i % cg);
+    const int64_t pix = i / cg;
+    const int wo = (int)(pix % d.Wo);
+    const int64_t t = pix / d.Wo;
+    const int ho = (int)(t % d.Ho);
+    const int n = (int)(t / d.Ho);
+    float acc[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[j] = d.b >= 0 ? __ldg(p.params + d.b + g * 8 + j) : 0.f;
+    for (int a = 0; a < d.kh; ++a) {
+      const int hi = ho * d.sh - d.ph + a;
+      if (hi < 0 || hi >= d.H) continue;
+      for (int b = 0; b < d.kw; ++b) {
+        const int wi = wo * d.sw - d.pw + b;
+        if (wi < 0 || wi >= d.W) continue;
+        const uint4 u = __ldg(reinterpret_cast<const uint4*>(x + (((int64_t)n * d.H + hi) * d.W + wi) * d.C) + g);
+        const uint32_t uw[4] = {u.x, u.y, u.z, u.w};
+        const int tap = a * d.kw + b;
+        // weights in [tap][C] order (d.w2): two float4 per tap and 8-channel group
+        const float4* w4 = reinterpret_cast<const float4*>(p.params + d.w2 + (int64_t)tap * d.C + g * 8);
+        const float4 wa = __ldg(w4), wb = __ldg(w4 + 1);
+        const float wv[8] = {wa.x, wa.y, wa.z, wa.w, wb.x, wb.y, wb.z, wb.w};
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const float xv = __uint_as_float(j & 1 ? (uw[j / 2] & 0xFFFF0000u) : (uw[j / 2] << 16));
+          acc[j] = fmaf(xv, wv[j], acc[j]);
+        }
+      }
+    }
+    uint4 pk;
+    __nv_bfloat162 h0v = __floats2bfloat162_rn(acc[0], acc[1]), h1v = __floats2bfloat162_rn(acc[2], acc[3]);
+    __nv_bfloat162 h2v = __floats2bfloat162_rn(acc[4], acc[5]), h3v = __floats2bfloat162_rn(acc[6], acc[7]);
+    pk.x = *reinterpret_cast<uint32_t*>(&h0v);
+    pk.y = *reinterpret_cast<uint32_t*>(&h1v);
+    pk.z = *reinterpret_cast<uint32_t*>(&h2v);
+    pk.w = *reinterpret_cast<uint32_t*>(&h3v);
+    reinterpret_cast<uint4*>(y + pix * d.C)[g] = pk;
+  }
+}
+
+// ---------------------------------------------------------------------------
 // direct NHWC convolution: one thread per output element, output channel
 // fastest so a warp shares its input pixels (broadcast loads)
 // ---------------------------------------------------------------------------
@@ -526,6 +578,33 @@ __global__ void group_gap_kernel(GroupDesc d, GCtx g) {
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.K;
   conv_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
+}
+
+__global__ void linear_epilogue_kernel(LinearDesc d, const float* ws, RunPtrs p) {
+  void* y = const_cast<void*>(loc_ptr(d.y, p));
+  const int64_t total = (int64_t)d.N * d.O;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int o = (int)(i % d.O);
+    float v = ws[i] + (d.b >= 0 ? p.params[d.b + o] : 0.f);
+    if (d.relu) v = fmaxf(v, 0.f);
+    stv(y, i, v, d.y.dtype);
+  }
+}
+
+void launch_linear_epilogue(const LinearDesc& d, const float* ws, const RunPtrs& p, cudaStream_t s) {
+  const int64_t total = (int64_t)d.N * d.O;
+  linear_epilogue_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, ws, p);
+}
+
+bool dwconv_vec_ok(const ConvDesc& d) {
+  return d.groups == d.C && d.K == d.C && d.C % 8 == 0 && d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.w2 >= 0;
+}
+
+void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * (d.C / 8);
+  int64_t g = (total + 255) / 256;
+  if (g > 148LL * 64) g = 148LL * 64;
+  dwconv_vec_kernel<<<(unsigned)g, 256, 0, s>>>(d, p);
 }
 
 bool conv_rank_ok(const ConvDesc& d) {

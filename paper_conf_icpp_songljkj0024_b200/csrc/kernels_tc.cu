@@ -226,15 +226,18 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
                     std::vector<float>& params, TcChainDesc& d) {
   const Node& root = ir.nodes[s.out];
   const bool gap = root.op == OP_GAP;
-  if (root.role != ROLE_FCONV && !gap) return false;
-  if (!gap && root.b) return false;              // fconv factors carry no bias (O1)
-  const int tsrc = ir.oin[s.out][0];
+  // store root: the group's value itself is the output (e.g. VGG's last pooled
+  // block feeding the classifier), written as bf16 NHWC without a fconv
+  const bool store = !gap && root.role != ROLE_FCONV;
+  if (!store && !gap && root.b) return false;    // fconv factors carry no bias (O1)
+  const int tsrc = store ? s.out : ir.oin[s.out][0];
   const Node& tn = ir.nodes[tsrc];
-  const int C = tn.C, Nout = gap ? 16 : root.C;
+  const int C = tn.C, Nout = (gap || store) ? 16 : root.C;
   if (Nout % 8 || Nout > 256) return false;
   if (gap && tn.H * tn.W > 128) return false;
+  if (store && C % kTcCc) return false;
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
-  P.members.erase(s.out);
+  if (!store) P.members.erase(s.out);
   std::vector<PLevel> levels;
   if (!P.chain(tsrc, levels)) return false;
   if (P.visited != P.members) return false;          // every member must be part of the chain form
@@ -251,6 +254,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   if (mixed && levels.size() != 1) return false;
   if (pm && (pm->c0 != 0 || pm->C % kTcCc)) return false;
   if (pm && gap) return false;                       // GAP over a max-pooled member: generic path
+  const bool nogemm2 = gap || store;
   int nterms = 0;
   for (auto& L : levels) nterms += (int)L.terms.size();
   if (pm) nterms += (int)pm->terms.size();
@@ -385,9 +389,13 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     if (d.tw * d.ms > 256 || d.th * d.ms > 256) return false;
   }
   d.F = 0;
+  d.store = store ? 1 : 0;
   if (gap) {
     d.alg_flops = flops + d.npix * C;
     d.alg_bytes = bytes + 2LL * ir.batch * C;
+  } else if (store) {
+    d.alg_flops = flops;
+    d.alg_bytes = bytes + d.npix * 2LL * C;
   } else {
     std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
     for (int o = 0; o < Nout; ++o)
@@ -398,8 +406,8 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   }
   // TMEM: accumulator slots (ubuf columns: one region per tap of a pooled unit)
   // and one or two output buffers of Np columns
-  const int npcols = gap ? 0 : d.Np;
-  d.no = gap ? 0 : (512 - 2 * npcols >= 4 * d.Cc ? 2 : 1);
+  const int npcols = nogemm2 ? 0 : d.Np;
+  d.no = nogemm2 ? 0 : (512 - 2 * npcols >= 4 * d.Cc ? 2 : 1);
   const int avail = 512 - d.no * npcols;
   d.tpu = 1;
   d.ntg = 1;
@@ -436,8 +444,8 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     T.wres = (int32_t)wb;
     wb += (int64_t)T.nhit * (T.Rp / T.aw) * d.Cc * T.aw * 2;
   }
-  const int64_t wf = gap ? 0 : (int64_t)d.nchunks * d.Np * 128;
-  d.fslot = gap ? 0 : (d.Np * 128 + 1023) / 1024 * 1024;
+  const int64_t wf = nogemm2 ? 0 : (int64_t)d.nchunks * d.Np * 128;
+  d.fslot = nogemm2 ? 0 : (d.Np * 128 + 1023) / 1024 * 1024;
   // first arrangement that fits: two A buffers before one, resident B before
   // resident F; a streamed B needs >= 4 ring stages
   struct Opt { int nab; bool b, f; };
@@ -445,10 +453,10 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
                        {1, true, true}, {1, true, false}, {1, false, true}, {1, false, false}};
   bool found = false;
   for (const Opt& o : opts) {
-    if (gap && o.f) continue;
+    if (nogemm2 && o.f) continue;
     const int64_t wres = (o.b ? wb : 0) + (o.f ? wf : 0);
     const int64_t wres_al = (wres + 1023) / 1024 * 1024;
-    const int fst = (gap || o.f) ? 0 : 3;
+    const int fst = (nogemm2 || o.f) ? 0 : 3;
     const int64_t left = budget - wres_al - o.nab * abytes - (int64_t)fst * d.fslot;
     if (left < (o.b ? 0 : 4LL * slot_b_stream)) continue;
     d.nabuf = o.nab;
@@ -559,7 +567,7 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
         return false;
       }
     }
-    if (!d->gap && !make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
+    if (!d->gap && !d->store && !make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)d->Np)) {
       err = "cuTensorMapEncodeTiled failed (F)";
       return false;
     }
@@ -795,7 +803,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
   } else if (warp == kFWarp) {
     // ------------------------------------------------------------ F ring producer (F not resident)
-    if (!d.gap && !d.fres) {
+    if (!d.gap && !d.store && !d.fres) {
       Ring r{0, 0};
       for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x)
         for (int c = 0; c < d.nchunks; ++c) {
@@ -858,7 +866,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
     }
   } else if (warp == kG2Warp) {
     // ------------------------------------------------------------ GEMM2 issuer: out += P_c F_c^T
-    if (!d.gap) {
+    if (!d.gap && !d.store) {
       if (d.fres) mbar_wait(wbar, 0);
       Ring fr{0, 0};
       uint32_t pph = 0;                 // phase bits of the 4 P buffers
@@ -1060,6 +1068,22 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
             asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
             continue;
           }
+          if (d.store) {
+            // store root: the restored value itself, bf16 NHWC [npix, C]
+            if (mvalid) {
+              uint4* dst = reinterpret_cast<uint4*>(y + m * d.C + col0);
+#pragma unroll
+              for (int qq = 0; qq < 4; ++qq) {
+                uint4 pk;
+                pk.x = relu ? pack_bf16_relu(t[8 * qq + 0], t[8 * qq + 1]) : pack_bf16(t[8 * qq + 0], t[8 * qq + 1]);
+                pk.y = relu ? pack_bf16_relu(t[8 * qq + 2], t[8 * qq + 3]) : pack_bf16(t[8 * qq + 2], t[8 * qq + 3]);
+                pk.z = relu ? pack_bf16_relu(t[8 * qq + 4], t[8 * qq + 5]) : pack_bf16(t[8 * qq + 4], t[8 * qq + 5]);
+                pk.w = relu ? pack_bf16_relu(t[8 * qq + 6], t[8 * qq + 7]) : pack_bf16(t[8 * qq + 6], t[8 * qq + 7]);
+                dst[qq] = pk;
+              }
+            }
+            continue;
+          }
           // last level: P = bf16 act(x) -> SMEM (one SW128 K-major atom per 64-channel unit)
           const int pb = team * 2 + (cp & 1);
           mbar_wait(&p_empty[pb], ((pph >> pb) & 1u) ^ 1u);
@@ -1088,7 +1112,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           ++cp;
         }
       }
-      if (d.gap) continue;
+      if (d.gap || d.store) continue;
       // output epilogue: column groups of 8 split between the two column halves
       const int ob = d.no == 2 ? team : 0;
       mbar_wait(&out_full[team], (uint32_t)(it >> 1) & 1u);

@@ -105,6 +105,7 @@ struct TcChainDesc {
   int32_t ntiles;
   int32_t rows_per_tile;                 // consecutive tiles: 128, or whole images for a GAP root
   int32_t gap, hw, ipt;                  // GAP root: pixels per image, images per tile
+  int32_t store;                         // store root: write t_D (bf16 [npix, C]) instead of a fconv
   int32_t nimg;
   int32_t Ho, Wo;                        // root resolution
   // spatial tiles (any tap-shifted read): tn x th x tw output pixels (<= 128)
@@ -115,7 +116,7 @@ struct TcChainDesc {
   int32_t tpu, ntg, ubuf;                // ubuf = TMEM columns of one accumulator slot (tpu * Cc)
   int64_t post;                          // params offset of the post-pool shift, -1 none
   int64_t F;                             // tc weight pool offset of F
-  Loc y;                                 // output [npix, Nout] bf16, or [N, C] for GAP
+  Loc y;                                 // output [npix, Nout] bf16, [N, C] for GAP, [npix, C] for store
   // accumulator slots (TMEM ring, one per unit-level) and output buffers
   int32_t ns, no, out_col, spt;          // slots; output buffers (Np columns each) from column out_col; slots / tile
   // resident weights: B boxes (every term atom of the chunks it reaches) and/or
