@@ -52,6 +52,7 @@ struct StepExec {
   std::string kernel;
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
+  bool stem = false;   // K_CONV on the tensor-core small-Cin kernel (kernels_stem.cu)
 };
 
 }  // namespace
@@ -267,10 +268,11 @@ void lower(temco_plan_s* P) {
     if (s.group) {
       // small restored widths: register-resident mma.sync kernel; larger ones:
       // the tcgen05 chain kernel (bf16 plans); anything else: the interpreter
-      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && (P->flags & TEMCO_FLAG_MMA_SMALL) &&
-          ir.nodes[ir.oin[s.out][0]].C <= 256 && mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma)) {
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
+          mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma) &&
+          ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
         e.kind = K_GROUP_MMA;
-        e.kernel = "mma_chain";
+        e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
         e.launches = 1;
         continue;
       }
@@ -359,7 +361,8 @@ void lower(temco_plan_s* P) {
           c.w2 = push_params(P, w2);
         }
         e.kind = K_CONV;
-        e.kernel = v.groups > 1 ? (dwconv_vec_ok(c) ? "simt_dwconv_vec" : "simt_dwconv") : conv_rank_ok(c) ? "simt_conv_rank" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
+        e.stem = !(P->flags & TEMCO_FLAG_SIMT_ONLY) && !dwconv_vec_ok(c) && !conv_rank_ok(c) && conv_stem_ok(c);
+        e.kernel = e.stem ? "mma_conv_stem" : v.groups > 1 ? (dwconv_vec_ok(c) ? "simt_dwconv_vec" : "simt_dwconv") : conv_rank_ok(c) ? "simt_conv_rank" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
         e.launches = 1;
         break;
       }
@@ -529,7 +532,9 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
     switch (e.kind) {
       case K_NONE: break;
       case K_CONV:
-        if (dwconv_vec_ok(e.conv))
+        if (e.stem)
+          launch_conv_stem(e.conv, rp, st);
+        else if (dwconv_vec_ok(e.conv))
           launch_dwconv_vec(e.conv, rp, st);
         else if (conv_rank_ok(e.conv))
           launch_conv_rank(e.conv, rp, st);

@@ -10,6 +10,8 @@ namespace temco {
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_small_ok(const ConvDesc& d);   // small-Cin direct conv applies (stem on the image)
 void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
+bool conv_stem_ok(const ConvDesc& d);    // bf16 small-Cin conv on tensor cores (mma.sync, kernels_stem.cu)
+void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool dwconv_vec_ok(const ConvDesc& d);   // depthwise bf16, C % 8 == 0: vectorised kernel
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)

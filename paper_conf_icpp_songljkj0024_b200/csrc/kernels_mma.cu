@@ -136,9 +136,13 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
   }
   while (blob.size() % 8) blob.push_back(0);
   d.blob_bytes = (int32_t)blob.size() * 2;
-  const int stage_bytes = 8 * 2 * 16 * d.a_stride * 2;
-  d.smem_bytes = d.blob_bytes + stage_bytes + 256;
-  if (d.smem_bytes > 200 * 1024) return false;
+  // per-warp prefetch ring: as deep as 8 units within ~200 KB (16 warps for
+  // 64-wide chunks, 8 for 128-wide ones, whose fragments need > 128 registers)
+  const int unit_bytes = 16 * d.a_stride * 2;
+  d.warps = d.CH == 64 ? 16 : 8;
+  d.nbuf = std::min(8, (200 * 1024 - d.blob_bytes - 256) / (d.warps * unit_bytes));
+  if (d.nbuf < 2) return false;
+  d.smem_bytes = d.blob_bytes + d.warps * d.nbuf * unit_bytes + 256;
   while (tcw.size() % 512) tcw.push_back(0);
   d.blob = (int64_t)tcw.size();
   tcw.insert(tcw.end(), blob.begin(), blob.end());
@@ -180,7 +184,19 @@ __device__ __forceinline__ uint32_t pk2(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
-constexpr int kWarps = 8;
+
+// cp.async.wait_group takes an immediate: dispatch the ring depth
+__device__ __forceinline__ void cp_async_wait_dyn(int n) {
+  switch (n) {
+    case 1: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
+    case 2: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
+    case 3: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
+    case 4: asm volatile("cp.async.wait_group 4;" ::: "memory"); break;
+    case 5: asm volatile("cp.async.wait_group 5;" ::: "memory"); break;
+    case 6: asm volatile("cp.async.wait_group 6;" ::: "memory"); break;
+    default: asm volatile("cp.async.wait_group 7;" ::: "memory"); break;
+  }
+}
 
 // stage the A rows of unit u (a 16-pixel block, and for a pooled chain one tap)
 __device__ __forceinline__ void stage_unit(const MmaChainDesc& d, const RunPtrs& p, __nv_bfloat16* st, int64_t blk,
@@ -208,7 +224,7 @@ __device__ __forceinline__ void stage_unit(const MmaChainDesc& d, const RunPtrs&
   }
 }
 
-template <int CH, int NO, bool POOL>
+template <int CH, int NO, bool POOL, int kWarps>
 __global__ void __launch_bounds__(32 * kWarps, 1) mma_chain_kernel(const __grid_constant__ MmaChainDesc d, RunPtrs p,
                                                                    const uint16_t* __restrict__ tcw) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -223,31 +239,45 @@ __global__ void __launch_bounds__(32 * kWarps, 1) mma_chain_kernel(const __grid_
   __syncthreads();
   const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
   const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
-  __nv_bfloat16* stage = reinterpret_cast<__nv_bfloat16*>(smem + d.blob_bytes) + (size_t)warp * 2 * 16 * d.a_stride;
+  __nv_bfloat16* stage = reinterpret_cast<__nv_bfloat16*>(smem + d.blob_bytes) + (size_t)warp * d.nbuf * 16 * d.a_stride;
   const int units_per_blk = POOL ? d.taps : 1;
   const int64_t gw = (int64_t)blockIdx.x * kWarps + warp, nw = (int64_t)gridDim.x * kWarps;
   // ldmatrix lane addressing (A: 16 rows x 16 k; B: 8 rows x 16 k)
   const int a_row = (lane & 7) + ((lane >> 3) & 1) * 8, a_col = (lane >> 4) * 8;
   const int b_row = lane & 7, b_col = ((lane >> 3) & 1) * 8;
 
+  // NB-deep per-warp prefetch ring over the warp's unit sequence (block, tap):
+  // these groups are HBM-bound with a few hundred bytes per unit, so many units
+  // must be in flight per warp to cover the memory latency (Little's law)
+  const int NB = d.nbuf;
+  const int ustride = 16 * d.a_stride;
+  int64_t pblk = gw;
+  int ptap = 0;
+  auto advance = [&](int64_t& b, int& t) {
+    if (++t == units_per_blk) t = 0, b += nw;
+  };
+  for (int k = 0; k < NB - 1; ++k) {
+    if (pblk < d.nblocks) stage_unit(d, p, stage + k * ustride, pblk, ptap, lane);
+    asm volatile("cp.async.commit_group;" ::: "memory");
+    advance(pblk, ptap);
+  }
   int64_t blk = gw;
   int tap = 0;
-  int buf = 0;
-  if (blk < d.nblocks) stage_unit(d, p, stage, blk, 0, lane);
-  asm volatile("cp.async.commit_group;" ::: "memory");
+  int buf = 0, pbuf = NB - 1;
 
   float O[NO][4];
   float run[POOL ? CH / 8 : 1][4];
   while (blk < d.nblocks) {
-    // prefetch the next unit into the other buffer
-    int64_t nblk = blk;
-    int ntap = tap + 1;
-    if (ntap == units_per_blk) ntap = 0, nblk = blk + nw;
-    if (nblk < d.nblocks) stage_unit(d, p, stage + (buf ^ 1) * 16 * d.a_stride, nblk, ntap, lane);
+    if (pblk < d.nblocks) stage_unit(d, p, stage + pbuf * ustride, pblk, ptap, lane);
     asm volatile("cp.async.commit_group;" ::: "memory");
-    asm volatile("cp.async.wait_group 1;" ::: "memory");
+    advance(pblk, ptap);
+    if (++pbuf == NB) pbuf = 0;
+    cp_async_wait_dyn(NB - 1);
     __syncwarp();
-    const __nv_bfloat16* A = stage + buf * 16 * d.a_stride;
+    const __nv_bfloat16* A = stage + buf * ustride;
+    int64_t nblk = blk;
+    int ntap = tap;
+    advance(nblk, ntap);
 
     if (tap == 0) {
 #pragma unroll
@@ -361,7 +391,7 @@ __global__ void __launch_bounds__(32 * kWarps, 1) mma_chain_kernel(const __grid_
       }
     }
     __syncwarp();
-    buf ^= 1;
+    if (++buf == NB) buf = 0;
     tap = ntap;
     blk = nblk;
   }
@@ -373,20 +403,173 @@ void launch_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cuda
   static bool configured = false;
   static int sms = 148;
   if (!configured) {
-    cudaFuncSetAttribute(mma_chain_kernel<CH, NO, POOL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(mma_chain_kernel<CH, NO, POOL, (CH == 64 ? 16 : 8)>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
-  const int per_sm = d.smem_bytes <= 100 * 1024 ? 2 : 1;
-  const int grid = (int)std::min<int64_t>((d.nblocks + kWarps - 1) / kWarps, (int64_t)sms * per_sm);
-  mma_chain_kernel<CH, NO, POOL><<<grid, 32 * kWarps, d.smem_bytes, s>>>(d, p, tcw);
+  const int per_sm = 1;   // 16 warps x ~100 registers: one persistent CTA per SM
+  const int grid = (int)std::min<int64_t>((d.nblocks + d.warps - 1) / d.warps, (int64_t)sms * per_sm);
+  mma_chain_kernel<CH, NO, POOL, (CH == 64 ? 16 : 8)><<<grid, 32 * d.warps, d.smem_bytes, s>>>(d, p, tcw);
+}
+
+
+// ---------------------------------------------------------------------------
+// Lean variant for the commonest HBM-bound shape: one level, one reduced input
+// (lconv -> BN -> [ReLU] -> fconv; VGG's per-conv groups, ResNet's in-block
+// groups), rank <= 32, C % 64 == 0, Nout <= 32.  Straight-line templated code:
+// the A fragments come straight from global memory into registers (two 32-bit
+// loads per row pair and k-step; the next block's are in flight while the
+// current one computes), the weights are ldmatrix'd from SMEM, the restored
+// 16 x 64 chunk lives in 32 accumulator registers and is re-packed in place
+// as the A operand of the reduce GEMM.  ~100 instructions per 16 pixels.
+// ---------------------------------------------------------------------------
+constexpr int kLeanWarps = 16;
+
+template <int KS>
+__device__ __forceinline__ void lean_load_a(uint32_t (&a)[KS][4], const uint32_t* __restrict__ r, int64_t blk,
+                                            int64_t npix, int R, int g, int t4) {
+  const int64_t m0 = blk * 16 + g, m1 = m0 + 8;
+  const bool v0 = m0 < npix, v1 = m1 < npix;
+  const int rw = R / 2;   // 32-bit words per row
+#pragma unroll
+  for (int ks = 0; ks < KS; ++ks) {
+    const int k0 = ks * 16 + 2 * t4, k1 = k0 + 8;
+    a[ks][0] = (v0 && k0 < R) ? __ldg(r + m0 * rw + k0 / 2) : 0u;
+    a[ks][1] = (v1 && k0 < R) ? __ldg(r + m1 * rw + k0 / 2) : 0u;
+    a[ks][2] = (v0 && k1 < R) ? __ldg(r + m0 * rw + k1 / 2) : 0u;
+    a[ks][3] = (v1 && k1 < R) ? __ldg(r + m1 * rw + k1 / 2) : 0u;
+  }
+}
+
+template <int KS, int NO>
+__global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __grid_constant__ MmaChainDesc d,
+                                                                      RunPtrs p, const uint16_t* __restrict__ tcw) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int g = lane / 4, t4 = lane % 4;
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(tcw + d.blob);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  __syncthreads();
+  const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
+  const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2) + d.bias[0];
+  const MmaTerm& T = d.term[0];
+  const uint32_t* r = reinterpret_cast<const uint32_t*>(p.arena + T.r.off);
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+  const int rs = T.Rp + 8, fs = d.Cpad + 8;
+  const bool relu = d.relu[0] != 0;
+  // ldmatrix.x4 lane addressing: matrix q = lane / 8 -> (n-tile + q / 2, k half q % 2)
+  const int lq = lane >> 3, lr = lane & 7;
+  const uint32_t wbase = s_u32(blob + T.w + ((lq >> 1) * 8 + lr) * rs + (lq & 1) * 8);
+  const uint32_t fbase = s_u32(blob + d.f + lr * fs + lq * 8);
+  const int64_t nw = (int64_t)gridDim.x * kLeanWarps;
+  int64_t blk = (int64_t)blockIdx.x * kLeanWarps + warp;
+  // three blocks of A fragments in registers: the one being computed and the
+  // next two in flight (each block is only ~100 instructions of work)
+  uint32_t a[KS][4], an[KS][4], ann[KS][4];
+  if (blk < d.nblocks) lean_load_a<KS>(a, r, blk, d.npix, T.R, g, t4);
+  if (blk + nw < d.nblocks) lean_load_a<KS>(an, r, blk + nw, d.npix, T.R, g, t4);
+  for (; blk < d.nblocks; blk += nw) {
+    if (blk + 2 * nw < d.nblocks) lean_load_a<KS>(ann, r, blk + 2 * nw, d.npix, T.R, g, t4);
+    float O[NO][4];
+#pragma unroll
+    for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
+#pragma unroll 1
+    for (int c0 = 0; c0 < d.Cpad; c0 += 64) {
+      float D[8][4];
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt) {
+        const float2 b = *reinterpret_cast<const float2*>(fb + c0 + nt * 8 + 2 * t4);
+        D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+      }
+#pragma unroll
+      for (int ks = 0; ks < KS; ++ks)
+#pragma unroll
+        for (int np = 0; np < 4; ++np) {
+          uint32_t b0, b1, b2, b3;
+          ldsm_x4(wbase + (uint32_t)(((c0 + np * 16) * rs + ks * 16) * 2), b0, b1, b2, b3);
+          mma16816(D[2 * np], a[ks][0], a[ks][1], a[ks][2], a[ks][3], b0, b1);
+          mma16816(D[2 * np + 1], a[ks][0], a[ks][1], a[ks][2], a[ks][3], b2, b3);
+        }
+      if (relu) {
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+      }
+      // reduce: O += P F^T over this chunk (4 k-steps of 16 restored channels)
+#pragma unroll
+      for (int kp = 0; kp < 2; ++kp) {
+        uint32_t pa[2][4];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int ks = 2 * kp + h;
+          pa[h][0] = pk2(D[2 * ks][0], D[2 * ks][1]);
+          pa[h][1] = pk2(D[2 * ks][2], D[2 * ks][3]);
+          pa[h][2] = pk2(D[2 * ks + 1][0], D[2 * ks + 1][1]);
+          pa[h][3] = pk2(D[2 * ks + 1][2], D[2 * ks + 1][3]);
+        }
+#pragma unroll
+        for (int nb = 0; nb < NO; ++nb) {
+          uint32_t f0, f1, f2, f3;
+          ldsm_x4(fbase + (uint32_t)((nb * 8 * fs + c0 + kp * 32) * 2), f0, f1, f2, f3);
+          mma16816(O[nb], pa[0][0], pa[0][1], pa[0][2], pa[0][3], f0, f1);
+          mma16816(O[nb], pa[1][0], pa[1][1], pa[1][2], pa[1][3], f2, f3);
+        }
+      }
+    }
+    const int64_t m0 = blk * 16 + g, m1 = m0 + 8;
+#pragma unroll
+    for (int nb = 0; nb < NO; ++nb) {
+      const int col = nb * 8 + 2 * t4;
+      if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + m0 * d.Nout + col) = pk2(O[nb][0], O[nb][1]);
+      if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + m1 * d.Nout + col) = pk2(O[nb][2], O[nb][3]);
+    }
+#pragma unroll
+    for (int ks = 0; ks < KS; ++ks)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        a[ks][i] = an[ks][i];
+        an[ks][i] = ann[ks][i];
+      }
+  }
+}
+
+template <int KS, int NO>
+void launch_lean_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  if (!configured) {
+    cudaFuncSetAttribute(mma_lean_kernel<KS, NO>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  const int grid = (int)std::min<int64_t>((d.nblocks + kLeanWarps - 1) / kLeanWarps, (int64_t)sms);
+  mma_lean_kernel<KS, NO><<<grid, 32 * kLeanWarps, d.blob_bytes, s>>>(d, p, tcw);
 }
 
 }  // namespace
 
+bool mma_lean_ok(const MmaChainDesc& d) {
+  return !d.pool && d.n_levels == 1 && d.n_terms == 1 && d.term[0].c0 == 0 && d.term[0].C == d.C &&
+         d.C % 64 == 0 && d.Cpad == d.C && d.term[0].Rp <= 32 && d.Nout <= 32 && d.blob_bytes <= 200 * 1024;
+}
+
 void launch_mma_chain(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  if (mma_lean_ok(d)) {
+    const int ks = d.term[0].Rp / 16, no = (d.Nout + 7) / 8;
+#define TEMCO_LEAN_CASE(k, n) \
+    if (ks == k && no == n) return launch_lean_t<k, n>(d, tcw, p, s);
+    TEMCO_LEAN_CASE(1, 1) TEMCO_LEAN_CASE(1, 2) TEMCO_LEAN_CASE(1, 3) TEMCO_LEAN_CASE(1, 4)
+    TEMCO_LEAN_CASE(2, 1) TEMCO_LEAN_CASE(2, 2) TEMCO_LEAN_CASE(2, 3) TEMCO_LEAN_CASE(2, 4)
+#undef TEMCO_LEAN_CASE
+  }
   const int no = d.Nout <= 32 ? 4 : d.Nout <= 64 ? 8 : 16;
   if (d.pool) {
     if (no == 4) launch_t<64, 4, true>(d, tcw, p, s);

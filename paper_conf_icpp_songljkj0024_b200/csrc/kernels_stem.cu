@@ -1,0 +1,243 @@
+// Small-Cin direct convolution on tensor cores (bf16 mode): the Tucker stem core
+// on the 3-channel image (7x7 s2 for ResNet-50 / DenseNet-121, 3x3 s1 for the
+// CIFAR ResNet-18) and VGG's first CP factor (1x1, 3 -> 8).
+//
+// A full-rank image mode is not decomposed (R17), so this conv reads the raw
+// image: K = kh*kw*Cin is tiny (<= ~200) and the output has 8..64 channels.
+// It is HBM-bound (AI ~ 10-20 flop/B), so the design goal is to read the image
+// once with no im2col materialisation:
+//   * a CTA stages the input footprint of a 16 x 32 output tile in SMEM as bf16,
+//     pixel stride Cp = Cin rounded up to even (zero channel padding), so each
+//     kernel row (kw pixels x Cp channels) is a contiguous run of SMEM;
+//   * the implicit-GEMM A fragments of mma.sync.m16n8k16 (row = output pixel,
+//     column = (kernel row, pixel-in-row, channel)) are single 32-bit LDS from
+//     that footprint (pairs never straddle a kernel row because Cp is even);
+//     K is padded to k-steps of 16 with zero weights;
+//   * the B fragments (weights, bf16) are register-resident for the whole CTA;
+//   * fp32 accumulation, bf16 NHWC output written straight from the fragments
+//     (four lanes cover one pixel's 16-byte channel group: coalesced rows).
+#include <cuda_bf16.h>
+
+#include <algorithm>
+
+#include "kernels.h"
+
+namespace temco {
+
+namespace {
+
+constexpr int kStTH = 16, kStTW = 32;   // output tile (rows x cols); 8 warps x 4 m-tiles of 16 pixels
+constexpr int kStThreads = 256;
+
+constexpr int kStCPT = 6;   // footprint chunks (16 B of an image row) per thread and tile
+
+struct StemGeo {
+  int Cp, rowK, KS, NT;   // padded channels, elements per kernel row, k-steps, n-tiles
+  int PR, PC, rowlen;     // footprint rows / pixels, elements per footprint row
+  int ncr;                // 16-byte image-row chunks covering one footprint row
+  int cmagic;             // (j * cmagic) >> 17 == j / Cin for j < 2048
+  int buf;                // 32-bit words of one footprint buffer (incl. slack)
+  int smem;               // bytes (two buffers)
+};
+
+StemGeo stem_geo(const ConvDesc& d) {
+  StemGeo g;
+  g.Cp = (d.C + 1) / 2 * 2;
+  g.rowK = d.kw * g.Cp;
+  g.KS = (d.kh * g.rowK + 15) / 16;
+  g.NT = d.K / 8;
+  g.PR = (kStTH - 1) * d.sh + d.kh;
+  g.PC = (kStTW - 1) * d.sw + d.kw;
+  g.rowlen = g.PC * g.Cp;
+  g.ncr = (g.PC * d.C + 7) / 8 + 1;
+  g.cmagic = ((1 << 17) + d.C - 1) / d.C;
+  // + slack: padded k columns past the last kernel row read (finite) footprint data
+  g.buf = (g.PR * g.rowlen + 64) / 2;
+  g.smem = g.buf * 4 * 2;
+  return g;
+}
+
+__device__ __forceinline__ void mma_bf16_16816(float* c, const uint32_t* a, uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+      "{%0,%1,%2,%3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+__device__ __forceinline__ uint32_t pack2(float lo, float hi) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(lo, hi);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+template <int KS, int NT>
+__global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, StemGeo g, RunPtrs p, int tiles_w,
+                                                               int tiles_h) {
+  extern __shared__ __align__(16) __nv_bfloat16 xs[];   // two footprint buffers of g.buf elements
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int gq = lane >> 2, tq = lane & 3;
+  // ---- per-thread k-pair offsets into a pixel's footprint window and the B fragments
+  const float* wf = p.params + d.w;   // fp32 [K][kh][kw][Cin]
+  int off[KS][2];
+  uint32_t bfr[NT][KS][2];
+#pragma unroll
+  for (int ks = 0; ks < KS; ++ks)
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int k = ks * 16 + 2 * tq + 8 * h;           // even: the pair (k, k+1) shares its kernel row
+      const int kr = k / g.rowK, j = k - kr * g.rowK;
+      off[ks][h] = kr < d.kh ? kr * g.rowlen + j : 0;
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt) {
+        const int o = nt * 8 + gq;
+        float w2[2];
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int jj = j + e, px = jj / g.Cp, c = jj - px * g.Cp;
+          w2[e] = (kr < d.kh && c < d.C) ? wf[(((int64_t)o * d.kh + kr) * d.kw + px) * d.C + c] : 0.f;
+        }
+        bfr[nt][ks][h] = pack2(w2[0], w2[1]);
+      }
+    }
+  float bias[NT][2];
+#pragma unroll
+  for (int nt = 0; nt < NT; ++nt)
+#pragma unroll
+    for (int e = 0; e < 2; ++e) bias[nt][e] = d.b >= 0 ? p.params[d.b + nt * 8 + 2 * tq + e] : 0.f;
+  // both buffers start zeroed: the pad channels and the slack are never written again
+  for (int i = threadIdx.x; i < g.buf; i += kStThreads) reinterpret_cast<uint32_t*>(xs)[i] = 0u;
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const uint4* x4 = reinterpret_cast<const uint4*>(loc_ptr(d.x, p));
+  const int rowC = d.W * d.C;            // image row in elements (% 8 == 0)
+  const int fl = g.PC * d.C;             // footprint row in elements
+  const int ntiles = d.N * tiles_w * tiles_h;
+  // footprint of a tile as 16-byte chunks of image rows, kStCPT chunks per thread in registers
+  uint4 v[kStCPT];
+  auto load = [&](int tile) {
+    const int n = tile / (tiles_w * tiles_h);
+    const int h0 = (tile / tiles_w) % tiles_h * kStTH, w0 = tile % tiles_w * kStTW;
+    const int hi0 = h0 * d.sh - d.ph, e0 = (w0 * d.sw - d.pw) * d.C;
+    const int a0 = e0 >= 0 ? e0 / 8 : -((7 - e0) / 8);
+#pragma unroll
+    for (int q = 0; q < kStCPT; ++q) {
+      const int i = threadIdx.x + q * kStThreads;
+      const int r = i / g.ncr, ch = a0 + (i - r * g.ncr);
+      const int hi = hi0 + r;
+      const bool ok = i < g.PR * g.ncr && hi >= 0 && hi < d.H && ch >= 0 && ch * 8 < rowC;
+      v[q] = ok ? __ldg(x4 + (((int64_t)n * d.H + hi) * rowC) / 8 + ch) : make_uint4(0, 0, 0, 0);
+    }
+  };
+  auto store = [&](int tile, __nv_bfloat16* buf) {
+    const int h0 = (tile / tiles_w) % tiles_h * kStTH, w0 = tile % tiles_w * kStTW;
+    (void)h0;
+    const int e0 = (w0 * d.sw - d.pw) * d.C;
+    const int a0 = e0 >= 0 ? e0 / 8 : -((7 - e0) / 8);
+#pragma unroll
+    for (int q = 0; q < kStCPT; ++q) {
+      const int i = threadIdx.x + q * kStThreads;
+      if (i >= g.PR * g.ncr) break;
+      const int r = i / g.ncr;
+      const int j0 = (a0 + (i - r * g.ncr)) * 8 - e0;   // footprint-row position of the chunk's element 0
+      const uint32_t w[4] = {v[q].x, v[q].y, v[q].z, v[q].w};
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        const int j = j0 + e;
+        if (j >= 0 && j < fl) {
+          const int px = (j * g.cmagic) >> 17, c = j - px * d.C;
+          reinterpret_cast<unsigned short*>(buf)[r * g.rowlen + px * g.Cp + c] =
+              (unsigned short)(w[e >> 1] >> ((e & 1) * 16));
+        }
+      }
+    }
+  };
+  int tile = blockIdx.x;
+  if (tile < ntiles) load(tile);
+  int b = 0;
+  for (; tile < ntiles; tile += gridDim.x, b ^= 1) {
+    __nv_bfloat16* buf = xs + b * g.buf * 2;
+    store(tile, buf);
+    __syncthreads();
+    const int n = tile / (tiles_w * tiles_h);
+    const int h0 = (tile / tiles_w) % tiles_h * kStTH, w0 = tile % tiles_w * kStTW;
+    if (tile + (int)gridDim.x < ntiles) load(tile + gridDim.x);   // in flight during the MMAs
+    const uint32_t* xw = reinterpret_cast<const uint32_t*>(buf);
+    // ---- 4 m-tiles per warp: output row (warp * 2 + mt / 2), 16 columns (mt & 1)
+#pragma unroll 1
+    for (int mt = 0; mt < 4; ++mt) {
+      const int orow = warp * 2 + (mt >> 1), ocol = (mt & 1) * 16;
+      const int b0 = (orow * d.sh) * g.rowlen + ((ocol + gq) * d.sw) * g.Cp;     // pixel rows gq, gq + 8
+      const int b1 = b0 + 8 * d.sw * g.Cp;
+      float acc[NT][4];
+#pragma unroll
+      for (int nt = 0; nt < NT; ++nt) {
+        acc[nt][0] = acc[nt][2] = bias[nt][0];
+        acc[nt][1] = acc[nt][3] = bias[nt][1];
+      }
+#pragma unroll
+      for (int ks = 0; ks < KS; ++ks) {
+        uint32_t a[4];
+        a[0] = xw[(b0 + off[ks][0]) >> 1];
+        a[1] = xw[(b1 + off[ks][0]) >> 1];
+        a[2] = xw[(b0 + off[ks][1]) >> 1];
+        a[3] = xw[(b1 + off[ks][1]) >> 1];
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt) mma_bf16_16816(acc[nt], a, bfr[nt][ks][0], bfr[nt][ks][1]);
+      }
+      const int oy = h0 + orow;
+      if (oy >= d.Ho) continue;
+#pragma unroll
+      for (int hf = 0; hf < 2; ++hf) {
+        const int ox = w0 + ocol + gq + 8 * hf;
+        if (ox >= d.Wo) continue;
+        __nv_bfloat16* yp = y + (((int64_t)n * d.Ho + oy) * d.Wo + ox) * d.K + 2 * tq;
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt)
+          *reinterpret_cast<uint32_t*>(yp + nt * 8) = pack2(acc[nt][2 * hf], acc[nt][2 * hf + 1]);
+      }
+    }
+  }
+}
+
+template <int KS, int NT>
+void launch_stem_t(const ConvDesc& d, const StemGeo& g, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  if (!configured) {
+    cudaFuncSetAttribute(conv_stem_kernel<KS, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, conv_stem_kernel<KS, NT>, kStThreads, g.smem);
+  const int tw = (d.Wo + kStTW - 1) / kStTW, th = (d.Ho + kStTH - 1) / kStTH;
+  const int ntiles = d.N * tw * th;
+  const int grid = std::min(ntiles, sms * std::max(per_sm, 1));
+  conv_stem_kernel<KS, NT><<<(unsigned)grid, kStThreads, g.smem, s>>>(d, g, p, tw, th);
+}
+
+}  // namespace
+
+bool conv_stem_ok(const ConvDesc& d) {
+  if (d.x.dtype != DT_BF16 || d.y.dtype != DT_BF16 || d.groups != 1 || d.C > 8 || d.K % 8 || d.sh != d.sw) return false;
+  const StemGeo g = stem_geo(d);
+  const bool shape = (g.NT == 1 || g.NT == 2) && (g.KS == 1 || g.KS == 3 || g.KS == 13);
+  return shape && g.smem <= 96 * 1024 && (d.W * d.C) % 8 == 0 && g.PR * g.ncr <= kStCPT * kStThreads &&
+         g.PC * d.C < 2048;
+}
+
+void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
+  const StemGeo g = stem_geo(d);
+#define TEMCO_STEM_CASE(ks, nt) \
+  if (g.KS == ks && g.NT == nt) return launch_stem_t<ks, nt>(d, g, p, s);
+  TEMCO_STEM_CASE(1, 1)
+  TEMCO_STEM_CASE(3, 1)
+  TEMCO_STEM_CASE(13, 1)
+  TEMCO_STEM_CASE(1, 2)
+  TEMCO_STEM_CASE(3, 2)
+  TEMCO_STEM_CASE(13, 2)
+#undef TEMCO_STEM_CASE
+}
+
+}  // namespace temco

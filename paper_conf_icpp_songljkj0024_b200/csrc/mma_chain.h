@@ -46,12 +46,14 @@ struct MmaChainDesc {
   int32_t blob_bf16;                // bf16 elements of the blob (biases follow as fp32)
   int32_t blob_bytes;
   int32_t a_stride;                 // per-warp A staging: elements per pixel row (sum of Rp + 8 per term)
+  int32_t nbuf, warps;              // per-warp prefetch ring depth (units); warps per CTA
   int32_t smem_bytes;
   int64_t alg_flops, alg_bytes;
 };
 
 bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                      MmaChainDesc& d);
+bool mma_lean_ok(const MmaChainDesc& d);   // the lean single-term kernel applies
 void launch_mma_chain(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s);
 
 }  // namespace temco

@@ -6,7 +6,7 @@ import workloads as W
 from paper_conf_icpp_songljkj0024_b200 import Plan
 cfg = sys.argv[1] if len(sys.argv) > 1 else "resnet50"
 m = W.build_config(cfg)
-p = Plan(m)
+p = Plan(m, flags=int(os.environ.get("TEMCO_PLAN_FLAGS", "0")))
 d = p.describe()
 x = torch.from_numpy(W.make_input(m)).cuda().to(torch.bfloat16)
 y = torch.empty(p.output_shape(), device="cuda")
