@@ -69,7 +69,6 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
     }
   const Loc& yl = loc.at(s.out);
   if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
-  if (pool && C > 64) return false;             // running max lives in registers: one 64-wide chunk
 
   d = MmaChainDesc();
   d.C = C;
@@ -149,6 +148,9 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
   const int64_t nin = (int64_t)ir.batch * cn.H * cn.W;
   d.alg_flops = nin * fl_terms + d.npix * 2LL * Nout * C;
   d.alg_bytes = nin * by_terms + d.npix * 2LL * Nout;
+  // the generic kernel keeps a pooled chain's running max in registers (one
+  // 64-wide chunk); the lean kernel walks chunks as units
+  if (pool && C > 64 && !mma_lean_ok(d)) return false;
   return true;
 }
 
@@ -427,20 +429,63 @@ void launch_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cuda
 // ---------------------------------------------------------------------------
 constexpr int kLeanWarps = 16;
 
+// unit = (16-pixel output block, 64-channel chunk, pool tap); a warp walks its
+// blocks' units in that order, with the A fragments of the next two units in
+// flight.  Pooled groups gather the tap-shifted input rows (zero rows, masked
+// to -inf for a max pool, outside the image).
+struct LeanCursor {
+  int64_t blk;
+  int ch, tap;
+  int hi0[2], wi0[2], nrow[2];   // pooled: per fragment row, the tap window origin and n * Hin
+};
+
+// (re)compute the per-row pool window origins when a cursor enters a new block
+__device__ __forceinline__ void lean_set_block(const MmaChainDesc& d, LeanCursor& u, int g) {
+  if (!d.pool) return;
+  const int hw = d.Ho * d.Wo;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const int m = (int)(u.blk * 16) + g + 8 * h;
+    const int n = m / hw, rem = m - n * hw;
+    const int ho = rem / d.Wo, wo = rem - ho * d.Wo;
+    u.hi0[h] = ho * d.ps - d.pp;
+    u.wi0[h] = wo * d.ps - d.pp;
+    u.nrow[h] = n * d.Hin;
+  }
+}
+
 template <int KS>
-__device__ __forceinline__ void lean_load_a(uint32_t (&a)[KS][4], const uint32_t* __restrict__ r, int64_t blk,
-                                            int64_t npix, int R, int g, int t4) {
-  const int64_t m0 = blk * 16 + g, m1 = m0 + 8;
-  const bool v0 = m0 < npix, v1 = m1 < npix;
+__device__ __forceinline__ void lean_load_a(uint32_t (&a)[KS][4], const MmaChainDesc& d, const uint32_t* __restrict__ r,
+                                            const LeanCursor& u, int R, int g, int t4) {
+  const int64_t m0 = u.blk * 16 + g, m1 = m0 + 8;
+  int64_t p0 = m0, p1 = m1;
+  bool v0 = m0 < d.npix, v1 = m1 < d.npix;
+  if (d.pool) {
+    const int ty = u.tap / d.pk, tx = u.tap - ty * d.pk;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int hi = u.hi0[h] + ty, wi = u.wi0[h] + tx;
+      const bool v = (h ? v1 : v0) && hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
+      const int64_t pix = (int64_t)(u.nrow[h] + hi) * d.Win + wi;
+      if (h) v1 = v, p1 = pix; else v0 = v, p0 = pix;
+    }
+  }
   const int rw = R / 2;   // 32-bit words per row
 #pragma unroll
   for (int ks = 0; ks < KS; ++ks) {
     const int k0 = ks * 16 + 2 * t4, k1 = k0 + 8;
-    a[ks][0] = (v0 && k0 < R) ? __ldg(r + m0 * rw + k0 / 2) : 0u;
-    a[ks][1] = (v1 && k0 < R) ? __ldg(r + m1 * rw + k0 / 2) : 0u;
-    a[ks][2] = (v0 && k1 < R) ? __ldg(r + m0 * rw + k1 / 2) : 0u;
-    a[ks][3] = (v1 && k1 < R) ? __ldg(r + m1 * rw + k1 / 2) : 0u;
+    a[ks][0] = (v0 && k0 < R) ? __ldg(r + p0 * rw + k0 / 2) : 0u;
+    a[ks][1] = (v1 && k0 < R) ? __ldg(r + p1 * rw + k0 / 2) : 0u;
+    a[ks][2] = (v0 && k1 < R) ? __ldg(r + p0 * rw + k1 / 2) : 0u;
+    a[ks][3] = (v1 && k1 < R) ? __ldg(r + p1 * rw + k1 / 2) : 0u;
   }
+}
+
+// is fragment row h's tap inside the image (max-pool masking)
+__device__ __forceinline__ bool lean_tap_valid(const MmaChainDesc& d, const LeanCursor& u, int h) {
+  const int ty = u.tap / d.pk, tx = u.tap - ty * d.pk;
+  const int hi = u.hi0[h] + ty, wi = u.wi0[h] + tx;
+  return hi >= 0 && hi < d.Hin && wi >= 0 && wi < d.Win;
 }
 
 template <int KS, int NO>
@@ -462,45 +507,88 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
   const int rs = T.Rp + 8, fs = d.Cpad + 8;
   const bool relu = d.relu[0] != 0;
+  const int taps = d.pool ? d.taps : 1;
+  const int nch = d.Cpad / 64;
   // ldmatrix.x4 lane addressing: matrix q = lane / 8 -> (n-tile + q / 2, k half q % 2)
   const int lq = lane >> 3, lr = lane & 7;
   const uint32_t wbase = s_u32(blob + T.w + ((lq >> 1) * 8 + lr) * rs + (lq & 1) * 8);
   const uint32_t fbase = s_u32(blob + d.f + lr * fs + lq * 8);
   const int64_t nw = (int64_t)gridDim.x * kLeanWarps;
-  int64_t blk = (int64_t)blockIdx.x * kLeanWarps + warp;
-  // three blocks of A fragments in registers: the one being computed and the
-  // next two in flight (each block is only ~100 instructions of work)
+  auto advance = [&](LeanCursor& u) {
+    if (++u.tap == taps) {
+      u.tap = 0;
+      if (++u.ch == nch) {
+        u.ch = 0;
+        u.blk += nw;
+        if (u.blk < d.nblocks) lean_set_block(d, u, g);
+      }
+    }
+  };
+  LeanCursor cur{};
+  cur.blk = (int64_t)blockIdx.x * kLeanWarps + warp;
+  if (cur.blk < d.nblocks) lean_set_block(d, cur, g);
+  LeanCursor pf = cur;
   uint32_t a[KS][4], an[KS][4], ann[KS][4];
-  if (blk < d.nblocks) lean_load_a<KS>(a, r, blk, d.npix, T.R, g, t4);
-  if (blk + nw < d.nblocks) lean_load_a<KS>(an, r, blk + nw, d.npix, T.R, g, t4);
-  for (; blk < d.nblocks; blk += nw) {
-    if (blk + 2 * nw < d.nblocks) lean_load_a<KS>(ann, r, blk + 2 * nw, d.npix, T.R, g, t4);
-    float O[NO][4];
+  if (pf.blk < d.nblocks) lean_load_a<KS>(a, d, r, pf, T.R, g, t4);
+  advance(pf);
+  if (pf.blk < d.nblocks) lean_load_a<KS>(an, d, r, pf, T.R, g, t4);
+  advance(pf);
+  float O[NO][4];
+  float run[8][4];
+  const float sc = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
+  for (; cur.blk < d.nblocks; advance(cur)) {
+    if (pf.blk < d.nblocks) lean_load_a<KS>(ann, d, r, pf, T.R, g, t4);
+    advance(pf);
+    const int c0 = cur.ch * 64;
+    if (cur.ch == 0 && cur.tap == 0) {
 #pragma unroll
-    for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
-#pragma unroll 1
-    for (int c0 = 0; c0 < d.Cpad; c0 += 64) {
-      float D[8][4];
+      for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
+    }
+    float D[8][4];
 #pragma unroll
-      for (int nt = 0; nt < 8; ++nt) {
-        const float2 b = *reinterpret_cast<const float2*>(fb + c0 + nt * 8 + 2 * t4);
-        D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+    for (int nt = 0; nt < 8; ++nt) {
+      const float2 b = *reinterpret_cast<const float2*>(fb + c0 + nt * 8 + 2 * t4);
+      D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+    }
+#pragma unroll
+    for (int ks = 0; ks < KS; ++ks)
+#pragma unroll
+      for (int np = 0; np < 4; ++np) {
+        uint32_t b0, b1, b2, b3;
+        ldsm_x4(wbase + (uint32_t)(((c0 + np * 16) * rs + ks * 16) * 2), b0, b1, b2, b3);
+        mma16816(D[2 * np], a[ks][0], a[ks][1], a[ks][2], a[ks][3], b0, b1);
+        mma16816(D[2 * np + 1], a[ks][0], a[ks][1], a[ks][2], a[ks][3], b2, b3);
+      }
+    if (relu) {
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+    }
+    bool last = true;
+    if (d.pool) {
+      // fold this tap into the running max / sum (max: taps outside the image excluded)
+      float n0 = 0.f, n1 = 0.f;
+      if (d.pool == 1) {
+        n0 = lean_tap_valid(d, cur, 0) ? 0.f : -INFINITY;
+        n1 = lean_tap_valid(d, cur, 1) ? 0.f : -INFINITY;
       }
 #pragma unroll
-      for (int ks = 0; ks < KS; ++ks)
+      for (int nt = 0; nt < 8; ++nt) {
+        const float x[4] = {D[nt][0] + n0, D[nt][1] + n0, D[nt][2] + n1, D[nt][3] + n1};
 #pragma unroll
-        for (int np = 0; np < 4; ++np) {
-          uint32_t b0, b1, b2, b3;
-          ldsm_x4(wbase + (uint32_t)(((c0 + np * 16) * rs + ks * 16) * 2), b0, b1, b2, b3);
-          mma16816(D[2 * np], a[ks][0], a[ks][1], a[ks][2], a[ks][3], b0, b1);
-          mma16816(D[2 * np + 1], a[ks][0], a[ks][1], a[ks][2], a[ks][3], b2, b3);
-        }
-      if (relu) {
+        for (int i = 0; i < 4; ++i)
+          run[nt][i] = cur.tap == 0 ? x[i] : d.pool == 1 ? fmaxf(run[nt][i], x[i]) : run[nt][i] + x[i];
+      }
+      last = cur.tap == taps - 1;
+      if (last) {
 #pragma unroll
         for (int nt = 0; nt < 8; ++nt)
 #pragma unroll
-          for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+          for (int i = 0; i < 4; ++i) D[nt][i] = run[nt][i] * sc;
       }
+    }
+    if (last) {
       // reduce: O += P F^T over this chunk (4 k-steps of 16 restored channels)
 #pragma unroll
       for (int kp = 0; kp < 2; ++kp) {
@@ -521,13 +609,15 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
           mma16816(O[nb], pa[1][0], pa[1][1], pa[1][2], pa[1][3], f2, f3);
         }
       }
-    }
-    const int64_t m0 = blk * 16 + g, m1 = m0 + 8;
+      if (cur.ch == nch - 1) {
+        const int64_t m0 = cur.blk * 16 + g, m1 = m0 + 8;
 #pragma unroll
-    for (int nb = 0; nb < NO; ++nb) {
-      const int col = nb * 8 + 2 * t4;
-      if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + m0 * d.Nout + col) = pk2(O[nb][0], O[nb][1]);
-      if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + m1 * d.Nout + col) = pk2(O[nb][2], O[nb][3]);
+        for (int nb = 0; nb < NO; ++nb) {
+          const int col = nb * 8 + 2 * t4;
+          if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + m0 * d.Nout + col) = pk2(O[nb][0], O[nb][1]);
+          if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + m1 * d.Nout + col) = pk2(O[nb][2], O[nb][3]);
+        }
+      }
     }
 #pragma unroll
     for (int ks = 0; ks < KS; ++ks)
@@ -557,7 +647,7 @@ void launch_lean_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p,
 }  // namespace
 
 bool mma_lean_ok(const MmaChainDesc& d) {
-  return !d.pool && d.n_levels == 1 && d.n_terms == 1 && d.term[0].c0 == 0 && d.term[0].C == d.C &&
+  return (d.pool != 2 || d.pp == 0) && d.n_levels == 1 && d.n_terms == 1 && d.term[0].c0 == 0 && d.term[0].C == d.C &&
          d.C % 64 == 0 && d.Cpad == d.C && d.term[0].Rp <= 32 && d.Nout <= 32 && d.blob_bytes <= 200 * 1024;
 }
 
