@@ -37,7 +37,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK };
 
 struct StepExec {
   int kind = K_NONE;
@@ -49,6 +49,7 @@ struct StepExec {
   wide::TcChainDesc tcw{};
   ConvTcDesc ctc{};
   MmaChainDesc mma{};
+  RankConvDesc rk{};
   std::string kernel;
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
@@ -325,6 +326,26 @@ void lower(temco_plan_s* P) {
         e.kernel = "none";
         break;
       case OP_CONV: {
+        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && !getenv("TEMCO_NO_RKMMA") && v.groups == 1) {
+          const Node& x = ir.nodes[ir.oin[s.out][0]];
+          ConvDesc c{};
+          c.x = tensor_loc(P, x.id);
+          c.y = tensor_loc(P, s.out);
+          c.N = N; c.H = x.H; c.W = x.W; c.C = x.C;
+          c.Ho = v.H; c.Wo = v.W; c.K = v.C;
+          c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = v.groups;
+          c.b = v.b ? push_params(P, v.b) : -1;
+          // 3x3 cores on 8 channels: the direct SIMT kernel measured faster (kernels_simt.cu)
+          if (c.C <= 64 && c.K <= 64 && !(c.C == 8 && c.K == 8 && c.kh * c.kw > 1)) {
+            const std::vector<float> w = repack_conv(v, x.C);
+            if (conv_rank_mma_lower(c, w.data(), P->tcw_h, e.rk)) {
+              e.kind = K_CONV_RK;
+              e.kernel = "mma_conv_rank";
+              e.launches = 1;
+              break;
+            }
+          }
+        }
         const bool rank_conv = [&] {   // reduced-rank core conv: the memory-bound SIMT kernel
           if (!P->bf16 || getenv("TEMCO_CONV_TC")) return false;
           const Node& x = ir.nodes[ir.oin[s.out][0]];
@@ -489,6 +510,7 @@ std::string make_json(const temco_plan_s* P) {
           << ",\"resident\":" << e.tcw.resident << ",\"smem\":" << e.tcw.smem_bytes << ",\"tmem\":" << e.tcw.tmem_cols
           << ",\"ntiles\":" << e.tcw.ntiles << ",\"Cc\":" << e.tcw.Cc << ",\"levels\":" << e.tcw.n_levels << "}";
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
+      if (e.kind == K_CONV_RK) o << ",\"alg_flops\":" << e.rk.alg_flops << ",\"alg_bytes\":" << e.rk.alg_bytes;
       if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;
     }
     o << ",\"live\":" << ir.live_fused[t] << "}";
@@ -563,6 +585,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
       case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
       case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
+      case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
       case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
     }
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t + 1], st));

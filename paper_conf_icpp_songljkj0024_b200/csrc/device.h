@@ -43,6 +43,20 @@ struct ConvDesc {             // direct NHWC convolution (fconv on full tensors,
   int64_t w2;                 // depthwise: params offset of the weights in [kh][kw][C] order, -1 none
 };
 
+struct RankConvDesc {          // reduced-rank conv on tensor cores (kernels_rank.cu), bf16
+  Loc x, y;
+  int32_t N, H, W, C, Ho, Wo, K;
+  int32_t kh, kw, sh, sw, ph, pw;
+  int32_t npix, nblocks;      // output pixels, 16-pixel blocks
+  int32_t KS, NT;             // k-steps of 16 input channels, n-tiles of 8 output channels
+  int32_t pair;               // Cin == 8: a k-step of 16 covers two taps
+  int32_t wstride;            // bf16 elements per weight row in SMEM
+  int64_t wblob;              // tc weight pool offset: [tap][K][wstride] bf16
+  int32_t blob_bytes;
+  int64_t b;                  // params offset of an fp32 bias, or -1
+  int64_t alg_flops, alg_bytes;
+};
+
 enum EwKind : int32_t { EW_BN, EW_RELU, EW_SILU, EW_ADD, EW_CONCAT, EW_MAXPOOL, EW_AVGPOOL, EW_GAP };
 
 constexpr int kMaxEwInputs = 64;

@@ -3,6 +3,8 @@
 
 #include <cuda_runtime.h>
 
+#include <vector>
+
 #include "device.h"
 
 namespace temco {
@@ -12,6 +14,9 @@ bool conv_small_ok(const ConvDesc& d);   // small-Cin direct conv applies (stem 
 void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_stem_ok(const ConvDesc& d);    // bf16 small-Cin conv on tensor cores (mma.sync, kernels_stem.cu)
 void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
+// reduced-rank conv (Cin, K % 8 == 0, Cin <= 64, K <= 64) on tensor cores; w = fp32 [K][kh][kw][Cin]
+bool conv_rank_mma_lower(const ConvDesc& c, const float* w, std::vector<uint16_t>& tcw, RankConvDesc& d);
+void launch_conv_rank_mma(const RankConvDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s);
 bool dwconv_vec_ok(const ConvDesc& d);   // depthwise bf16, C % 8 == 0: vectorised kernel
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)

@@ -614,7 +614,8 @@ __device__ __forceinline__ void trace_stamp(int row, int& n) {
 #define TRACE(row, n) trace_stamp(row, n)
 #endif
 // cycle accounting of CTA 0's MMA issuer: waits by kind, op loads, total
-__device__ unsigned long long g_prof[16];
+__device__ unsigned long long g_prof[64][16];   // per wide-kernel launch (launch order)
+__device__ int g_prof_n;
 #define PROF_T0() (_pt0 = clock64())
 #define PROF_ADD(var) (var += clock64() - _pt0)
 #else
@@ -920,15 +921,19 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       }
 #ifdef TEMCO_TRACE
       if (blockIdx.x == 0 && lane == 0) {
-        g_prof[0] = clock64() - pc_start;
-        g_prof[1] = pc_acc;
-        g_prof[2] = pc_p;
-        g_prof[3] = pc_out;
-        g_prof[4] = pc_full;
-        g_prof[5] = pc_issue;
-        g_prof[6] = pc_n;
-        g_prof[7] = pc_dec;
-        g_prof[8] = pc_com;
+        const int li = atomicAdd(&g_prof_n, 1) & 63;
+        g_prof[li][0] = clock64() - pc_start;
+        g_prof[li][1] = pc_acc;
+        g_prof[li][2] = pc_p;
+        g_prof[li][3] = pc_out;
+        g_prof[li][4] = pc_full;
+        g_prof[li][5] = pc_issue;
+        g_prof[li][6] = pc_n;
+        g_prof[li][7] = pc_dec;
+        g_prof[li][8] = pc_com;
+        g_prof[li][9] = d.ntiles;
+        g_prof[li][10] = d.units;
+        g_prof[li][11] = d.stages;
       }
 #endif
     }
@@ -1194,3 +1199,16 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
 
 }  // namespace wide
 }  // namespace temco
+
+#ifdef TEMCO_TRACE
+// experiment builds: CTA 0 MMA-issuer cycle accounting of each wide-kernel launch since the last call
+extern "C" int temco_debug_wide_prof(unsigned long long* out) {
+  int n = 0;
+  cudaMemcpyFromSymbol(&n, temco::wide::g_prof_n, sizeof(int));
+  cudaMemcpyFromSymbol(out, temco::wide::g_prof, sizeof(unsigned long long) * 64 * 16);
+  const int z = 0;
+  cudaMemcpyToSymbol(temco::wide::g_prof_n, &z, sizeof(int));
+  return n;
+}
+extern "C" void temco_debug_wide_dbg(int v) { cudaMemcpyToSymbol(temco::wide::g_dbg, &v, sizeof(int)); }
+#endif
