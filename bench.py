@@ -256,6 +256,25 @@ def main():
     else:
         achieved, peak, unit, bound = c["bytes"] / (c["ms"] * 1e-3) / 1e9, hbm, "GB/s", "hbm"
     total_ms = float(prof.sum())
+    # every class against its own bound, and the fused-group family (SURVEY 8(a)
+    # row a6: tc_chain + mma_lean + mma_chain) as a time-weighted roofline
+    # fraction over its launches: sum_i max(F_i / P_tc, B_i / P_hbm) / sum_i t_i
+    by_class = {}
+    for k, v in classes.items():
+        a_i = v["flops"] / max(v["bytes"], 1)
+        tb = a_i > tf_sust * 1e12 / (hbm * 1e9)
+        ach = v["flops"] / (v["ms"] * 1e-3) / 1e12 if tb else v["bytes"] / (v["ms"] * 1e-3) / 1e9
+        by_class[k] = {"bound": "tensor" if tb else "hbm", "achieved": round(ach, 1),
+                       "unit": "TFLOP/s" if tb else "GB/s", "frac": round(ach / (tf_sust if tb else hbm), 4),
+                       "ms": round(v["ms"], 4)}
+    ideal = actual = 0.0
+    for s, t in zip(steps, prof):
+        if s["kernel"] in ("tc_chain", "mma_lean", "mma_chain") and t > 0:
+            ideal += max(s.get("alg_flops", s["flops"]) / (tf_sust * 1e12), s.get("alg_bytes", s["io_bytes"]) / (hbm * 1e9))
+            actual += float(t) * 1e-3
+    fused = {"kernels": ["tc_chain", "mma_lean", "mma_chain"], "roofline_ms": round(ideal * 1e3, 4),
+             "measured_ms": round(actual * 1e3, 4), "frac": round(ideal / actual, 4) if actual else None,
+             "note": "per launch max(alg FLOP / sustained bf16 peak, alg bytes / HBM peak), summed, / measured"}
     # DRAM traffic of the dominant class from the committed ncu capture of this
     # config (scripts/launch_summary.py --json), bytes per step like `achieved`
     traffic = None
@@ -286,6 +305,8 @@ def main():
                          "launches_per_step": c["launches"], "share_of_step": c["ms"] / total_ms,
                          "alg_flops_per_step": c["flops"], "alg_bytes_per_step": c["bytes"]},
             "kernel_classes_ms": {k: round(v["ms"], 4) for k, v in sorted(classes.items(), key=lambda kv: -kv[1]["ms"])},
+            "roofline_by_class": by_class,
+            "fused_group_roofline": fused,
             "clocks": clk,
         }
         if ws == 1 and not args.no_cpu_baseline:

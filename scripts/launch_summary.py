@@ -12,7 +12,8 @@ import collections, csv, io, json, sys
 CLASS = {"tc_chain_kernel": "tc_chain", "conv_tc_kernel": "tc_conv", "conv_tma_kernel": "tc_conv",
          "conv_small_kernel": "simt_conv_small", "conv_stem_kernel": "mma_conv_stem", "linear_kernel": "simt_linear", "conv_kernel": "simt_conv",
          "ew_kernel": "simt_ew", "group_simt_kernel": "simt_group", "group_gap_kernel": "simt_group_gap",
-         "mma_chain_kernel": "mma_chain"}
+         "mma_chain_kernel": "mma_chain", "mma_lean_kernel": "mma_lean", "conv_rank_mma_kernel": "mma_conv_rank",
+         "conv_rank_kernel": "simt_conv_rank", "dwconv_vec_kernel": "simt_dwconv_vec", "linear_epilogue_kernel": "blas_linear"}
 
 path, n = sys.argv[1], int(sys.argv[2])
 lines = open(path).read().splitlines()
@@ -27,7 +28,8 @@ for r in rows:
     except ValueError:
         pass
 def short(name):
-    return name.split("(")[0].split("::")[-1]
+    n = name.split("(")[0].split("::")[-1]
+    return n.split("<")[0].split(" ")[-1]
 
 
 ids = [i for i in sorted(launch) if short(launch[i]["name"]) in CLASS][:n]   # our kernels only
