@@ -5,6 +5,7 @@
 // kernels_tc.cu replace the hot fused groups in bf16 mode.
 #include <cuda_bf16.h>
 
+#include <algorithm>
 #include <cfloat>
 
 #include "kernels.h"
@@ -237,32 +238,183 @@ __global__ void __launch_bounds__(256) conv_rank_kernel(ConvDesc d, RankTile t, 
 // consecutive threads cover consecutive 16-byte chunks of a pixel row (fully
 // coalesced), the kh x kw taps of neighbouring threads hit L1 / L2.
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) dwconv_vec_kernel(ConvDesc d, RunPtrs p) {
+// vertical 3x1 CP factor (stride 1): a thread walks a strip of kColRows output
+// rows of one (column, 8-channel group) with a sliding window -- the strip's
+// kColRows + 2 input rows are loaded once, all in flight together
+constexpr int kColRows = 8;
+__global__ void __launch_bounds__(256) dwconv_col_kernel(ConvDesc d, RunPtrs p) {
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
   const int cg = d.C / 8;
-  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * cg;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int g = (int)(i % cg);
-    const int64_t pix = i / cg;
-    const int wo = (int)(pix % d.Wo);
-    const int64_t t = pix / d.Wo;
-    const int ho = (int)(t % d.Ho);
-    const int n = (int)(t / d.Ho);
+  const int per_row = d.Wo * cg;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= per_row) return;
+  const int wo = idx / cg, g = idx - wo * cg;
+  const int spi = (d.Ho + kColRows - 1) / kColRows;     // strips per image
+  float w[3][8], bias[8];
+#pragma unroll
+  for (int t = 0; t < 3; ++t) {
+    const float4* w4 = reinterpret_cast<const float4*>(p.params + d.w2 + t * d.C + g * 8);
+    const float4 wa = __ldg(w4), wb = __ldg(w4 + 1);
+    w[t][0] = wa.x; w[t][1] = wa.y; w[t][2] = wa.z; w[t][3] = wa.w;
+    w[t][4] = wb.x; w[t][5] = wb.y; w[t][6] = wb.z; w[t][7] = wb.w;
+  }
+#pragma unroll
+  for (int j = 0; j < 8; ++j) bias[j] = d.b >= 0 ? __ldg(p.params + d.b + g * 8 + j) : 0.f;
+  for (int st = blockIdx.y; st < d.N * spi; st += gridDim.y) {
+    const int n = st / spi, h0 = (st - n * spi) * kColRows;
+    uint4 v[kColRows + 2];
+#pragma unroll
+    for (int r = 0; r < kColRows + 2; ++r) {
+      const int hi = h0 - d.ph + r;
+      v[r] = make_uint4(0, 0, 0, 0);
+      if (hi >= 0 && hi < d.H && h0 + r - 2 < d.Ho)
+        v[r] = __ldg(reinterpret_cast<const uint4*>(x + (((int64_t)n * d.H + hi) * d.W + wo) * d.C) + g);
+    }
+#pragma unroll
+    for (int r = 0; r < kColRows; ++r) {
+      if (h0 + r >= d.Ho) break;
+      float acc[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) acc[j] = bias[j];
+#pragma unroll
+      for (int t = 0; t < 3; ++t) {
+        const uint32_t uw[4] = {v[r + t].x, v[r + t].y, v[r + t].z, v[r + t].w};
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const float xv = __uint_as_float(j & 1 ? (uw[j / 2] & 0xFFFF0000u) : (uw[j / 2] << 16));
+          acc[j] = fmaf(xv, w[t][j], acc[j]);
+        }
+      }
+      uint4 pk;
+      __nv_bfloat162 h0v = __floats2bfloat162_rn(acc[0], acc[1]), h1v = __floats2bfloat162_rn(acc[2], acc[3]);
+      __nv_bfloat162 h2v = __floats2bfloat162_rn(acc[4], acc[5]), h3v = __floats2bfloat162_rn(acc[6], acc[7]);
+      pk.x = *reinterpret_cast<uint32_t*>(&h0v);
+      pk.y = *reinterpret_cast<uint32_t*>(&h1v);
+      pk.z = *reinterpret_cast<uint32_t*>(&h2v);
+      pk.w = *reinterpret_cast<uint32_t*>(&h3v);
+      reinterpret_cast<uint4*>(y + (((int64_t)n * d.Ho + h0 + r) * d.Wo + wo) * d.C)[g] = pk;
+    }
+  }
+}
+
+// horizontal 1x3 CP factor (stride 1): one 16-byte load per thread; the left /
+// right neighbours come from the lanes cg away (warp shuffles), only lanes whose
+// neighbour lies outside the warp load it themselves
+__global__ void __launch_bounds__(256) dwconv_row_kernel(ConvDesc d, RunPtrs p) {
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const int cg = d.C / 8;
+  const int per_row = d.Wo * cg;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  const int lane = threadIdx.x & 31;
+  const bool act = idx < per_row;
+  const int wo = act ? idx / cg : 0, g = act ? idx - wo * cg : 0;
+  float w[3][8], bias[8];
+#pragma unroll
+  for (int t = 0; t < 3; ++t) {
+    const float4* w4 = reinterpret_cast<const float4*>(p.params + d.w2 + t * d.C + g * 8);
+    const float4 wa = __ldg(w4), wb = __ldg(w4 + 1);
+    w[t][0] = wa.x; w[t][1] = wa.y; w[t][2] = wa.z; w[t][3] = wa.w;
+    w[t][4] = wb.x; w[t][5] = wb.y; w[t][6] = wb.z; w[t][7] = wb.w;
+  }
+#pragma unroll
+  for (int j = 0; j < 8; ++j) bias[j] = d.b >= 0 ? __ldg(p.params + d.b + g * 8 + j) : 0.f;
+  constexpr int kRU = 4;   // rows per iteration: their loads in flight together
+  const int rows = d.N * d.Ho;
+  for (int row0 = blockIdx.y * kRU; row0 < rows; row0 += gridDim.y * kRU) {
+  uint4 cr[kRU];
+#pragma unroll
+  for (int q = 0; q < kRU; ++q)
+    cr[q] = (act && row0 + q < rows)
+                ? __ldg(reinterpret_cast<const uint4*>(x + (int64_t)(row0 + q) * d.W * d.C) + g + (int64_t)wo * cg)
+                : make_uint4(0, 0, 0, 0);
+#pragma unroll
+  for (int q = 0; q < kRU; ++q) {
+    const int row = row0 + q;
+    const uint4* xr = reinterpret_cast<const uint4*>(x + (int64_t)row * d.W * d.C) + g;   // Ho == H, stride 1
+    const uint4 z = make_uint4(0, 0, 0, 0);
+    const uint4 c = cr[q];
+    uint4 v[3];
+    v[1] = c;
+#pragma unroll
+    for (int side = 0; side < 2; ++side) {
+      const int wi = wo - d.pw + 2 * side;      // left (side 0) / right (side 1) neighbour column
+      uint4 s4;
+      s4.x = side ? __shfl_down_sync(0xffffffffu, c.x, cg) : __shfl_up_sync(0xffffffffu, c.x, cg);
+      s4.y = side ? __shfl_down_sync(0xffffffffu, c.y, cg) : __shfl_up_sync(0xffffffffu, c.y, cg);
+      s4.z = side ? __shfl_down_sync(0xffffffffu, c.z, cg) : __shfl_up_sync(0xffffffffu, c.z, cg);
+      s4.w = side ? __shfl_down_sync(0xffffffffu, c.w, cg) : __shfl_up_sync(0xffffffffu, c.w, cg);
+      const bool inwarp = side ? lane + cg < 32 && idx + cg < per_row : lane >= cg;
+      if (!(wi >= 0 && wi < d.W))
+        s4 = z;
+      else if (!inwarp && act && row < rows)
+        s4 = __ldg(xr + (int64_t)wi * cg);
+      v[2 * side] = s4;
+    }
+    if (!act || row >= rows) continue;
+    float acc[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[j] = bias[j];
+#pragma unroll
+    for (int t = 0; t < 3; ++t) {
+      const uint32_t uw[4] = {v[t].x, v[t].y, v[t].z, v[t].w};
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const float xv = __uint_as_float(j & 1 ? (uw[j / 2] & 0xFFFF0000u) : (uw[j / 2] << 16));
+        acc[j] = fmaf(xv, w[t][j], acc[j]);
+      }
+    }
+    uint4 pk;
+    __nv_bfloat162 h0v = __floats2bfloat162_rn(acc[0], acc[1]), h1v = __floats2bfloat162_rn(acc[2], acc[3]);
+    __nv_bfloat162 h2v = __floats2bfloat162_rn(acc[4], acc[5]), h3v = __floats2bfloat162_rn(acc[6], acc[7]);
+    pk.x = *reinterpret_cast<uint32_t*>(&h0v);
+    pk.y = *reinterpret_cast<uint32_t*>(&h1v);
+    pk.z = *reinterpret_cast<uint32_t*>(&h2v);
+    pk.w = *reinterpret_cast<uint32_t*>(&h3v);
+    reinterpret_cast<uint4*>(y + ((int64_t)row * d.Wo + wo) * d.C)[g] = pk;
+  }
+  }
+}
+
+template <int KH, int KW>   // 0, 0: runtime kernel size (<= 9 taps)
+__global__ void __launch_bounds__(256) dwconv_vec_kernel(ConvDesc d, RunPtrs p) {
+  // grid: x = chunks of (output column, 8-channel group) of one output row, y = output rows (n, ho):
+  // 32-bit index math only (the 64-bit div/mod chain dominated the previous flat-index version)
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const int cg = d.C / 8;
+  const int per_row = d.Wo * cg;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= per_row) return;
+  const int wo = idx / cg, g = idx - wo * cg;
+  for (int row = blockIdx.y; row < d.N * d.Ho; row += gridDim.y) {
+    const int n = row / d.Ho, ho = row - n * d.Ho;
+    // all taps' 16-byte loads in flight before any arithmetic (the CP factors are
+    // 3x1 / 1x3: one load in flight per thread capped this kernel at ~2 TB/s)
+    constexpr int kMaxTaps = KH > 0 ? KH * KW : 9;
+    const int kw = KH > 0 ? KW : d.kw;
+    uint4 v[kMaxTaps];
+    const int taps = KH > 0 ? KH * KW : d.kh * d.kw;
+#pragma unroll
+    for (int t = 0; t < kMaxTaps; ++t) {
+      v[t] = make_uint4(0, 0, 0, 0);
+      if (t < taps) {
+        const int a = t / kw, b = t - a * kw;
+        const int hi = ho * d.sh - d.ph + a, wi = wo * d.sw - d.pw + b;
+        if (hi >= 0 && hi < d.H && wi >= 0 && wi < d.W)
+          v[t] = __ldg(reinterpret_cast<const uint4*>(x + (((int64_t)n * d.H + hi) * d.W + wi) * d.C) + g);
+      }
+    }
     float acc[8];
 #pragma unroll
     for (int j = 0; j < 8; ++j) acc[j] = d.b >= 0 ? __ldg(p.params + d.b + g * 8 + j) : 0.f;
-    for (int a = 0; a < d.kh; ++a) {
-      const int hi = ho * d.sh - d.ph + a;
-      if (hi < 0 || hi >= d.H) continue;
-      for (int b = 0; b < d.kw; ++b) {
-        const int wi = wo * d.sw - d.pw + b;
-        if (wi < 0 || wi >= d.W) continue;
-        const uint4 u = __ldg(reinterpret_cast<const uint4*>(x + (((int64_t)n * d.H + hi) * d.W + wi) * d.C) + g);
-        const uint32_t uw[4] = {u.x, u.y, u.z, u.w};
-        const int tap = a * d.kw + b;
+#pragma unroll
+    for (int t = 0; t < kMaxTaps; ++t) {
+      if (t < taps) {
+        const uint32_t uw[4] = {v[t].x, v[t].y, v[t].z, v[t].w};
         // weights in [tap][C] order (d.w2): two float4 per tap and 8-channel group
-        const float4* w4 = reinterpret_cast<const float4*>(p.params + d.w2 + (int64_t)tap * d.C + g * 8);
+        const float4* w4 = reinterpret_cast<const float4*>(p.params + d.w2 + t * d.C + g * 8);
         const float4 wa = __ldg(w4), wb = __ldg(w4 + 1);
         const float wv[8] = {wa.x, wa.y, wa.z, wa.w, wb.x, wb.y, wb.z, wb.w};
 #pragma unroll
@@ -279,7 +431,7 @@ __global__ void __launch_bounds__(256) dwconv_vec_kernel(ConvDesc d, RunPtrs p) 
     pk.y = *reinterpret_cast<uint32_t*>(&h1v);
     pk.z = *reinterpret_cast<uint32_t*>(&h2v);
     pk.w = *reinterpret_cast<uint32_t*>(&h3v);
-    reinterpret_cast<uint4*>(y + pix * d.C)[g] = pk;
+    reinterpret_cast<uint4*>(y + ((int64_t)row * d.Wo + wo) * d.C)[g] = pk;
   }
 }
 
@@ -597,14 +749,29 @@ void launch_linear_epilogue(const LinearDesc& d, const float* ws, const RunPtrs&
 }
 
 bool dwconv_vec_ok(const ConvDesc& d) {
-  return d.groups == d.C && d.K == d.C && d.C % 8 == 0 && d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.w2 >= 0;
+  return d.groups == d.C && d.K == d.C && d.C % 8 == 0 && d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.w2 >= 0 &&
+         d.kh * d.kw <= 9;
 }
 
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
-  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * (d.C / 8);
-  int64_t g = (total + 255) / 256;
-  if (g > 148LL * 64) g = 148LL * 64;
-  dwconv_vec_kernel<<<(unsigned)g, 256, 0, s>>>(d, p);
+  const int per_row = d.Wo * (d.C / 8);
+  const int rows = d.N * d.Ho;
+  // rows per block: a persistent-ish y grid (8 blocks per SM per x chunk) instead of one
+  // tiny block per output row
+  const int xb = (per_row + 255) / 256;
+  dim3 grid((unsigned)xb, (unsigned)std::min(rows, std::max(1, 148 * 8 / xb)));
+  if (d.kh == 3 && d.kw == 1 && d.sh == 1 && d.sw == 1 && d.pw == 0 && d.Ho == d.H + 2 * d.ph - 2) {
+    const int strips = d.N * ((d.Ho + kColRows - 1) / kColRows);
+    dwconv_col_kernel<<<dim3((unsigned)xb, (unsigned)std::min(strips, std::max(1, 148 * 8 / xb))), 256, 0, s>>>(d, p);
+  } else if (d.kh == 3 && d.kw == 1)
+    dwconv_vec_kernel<3, 1><<<grid, 256, 0, s>>>(d, p);
+  else if (d.kh == 1 && d.kw == 3 && d.sh == 1 && d.sw == 1 && d.ph == 0 && d.pw == 1 && d.Wo == d.W &&
+           d.Ho == d.H && d.C / 8 <= 16) {
+    dwconv_row_kernel<<<dim3((unsigned)xb, (unsigned)std::min((rows + 3) / 4, std::max(1, 148 * 8 / xb))), 256, 0, s>>>(d, p);
+  } else if (d.kh == 1 && d.kw == 3)
+    dwconv_vec_kernel<1, 3><<<grid, 256, 0, s>>>(d, p);
+  else
+    dwconv_vec_kernel<0, 0><<<grid, 256, 0, s>>>(d, p);
 }
 
 bool conv_rank_ok(const ConvDesc& d) {

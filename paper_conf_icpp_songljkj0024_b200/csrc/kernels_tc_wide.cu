@@ -828,7 +828,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
       const long long pc_start = clock64();
 #endif
       const uint64_t base16 = smem_u32(smem) >> 4;
-      auto exec = [&](const TcMmaOpD& o, int gu, uint32_t tile_iter) {
+      auto exec = [&](const TcMmaOpD o, int gu, uint32_t tile_iter) {   // by value: one LDS.128 pair, then registers
 #ifdef TEMCO_TRACE
           long long _pt0 = 0;
 #endif
@@ -871,8 +871,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           PROF_ADD(pc_dec);
           {
           PROF_T0();
-          mma_bf16_w(dt, ad, bd, o.idesc, acc0);
-          for (int k = 1; k < o.nk; ++k) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, o.idesc, 1u);
+          // K=16 steps of the op (nk <= 4), unrolled: descriptors advance by 32 bytes (>> 4 = 2)
+          const uint32_t idesc = o.idesc, nk = o.nk;
+          mma_bf16_w(dt, ad, bd, idesc, acc0);
+#pragma unroll
+          for (uint32_t k = 1; k < 4; ++k)
+            if (k < nk) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, idesc, 1u);
           PROF_ADD(pc_issue);
 #ifdef TEMCO_TRACE
           pc_n += o.nk;
