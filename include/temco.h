@@ -117,7 +117,9 @@ enum {
   TEMCO_FLAG_SIMT_ONLY = 1 << 4,       /* never select the tcgen05 kernels               */
   TEMCO_FLAG_OVERHEAD_ALWAYS = 1 << 5, /* force Overhead() true  (tests)                 */
   TEMCO_FLAG_OVERHEAD_NEVER = 1 << 6,  /* force Overhead() false (tests)                 */
-  TEMCO_FLAG_MMA_SMALL = 1 << 7        /* run groups with C <= 256 on the mma.sync kernel */
+  TEMCO_FLAG_MMA_SMALL = 1 << 7,       /* run groups with C <= 256 on the mma.sync kernel */
+  TEMCO_FLAG_MMA_CAT = 1 << 8          /* single-level concat groups on the mma.sync concat
+                                          kernel (kernels_cat.cu; measured slower than tcgen05) */
 };
 
 typedef struct {

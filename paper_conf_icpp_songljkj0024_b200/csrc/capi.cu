@@ -37,7 +37,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT };
 
 struct StepExec {
   int kind = K_NONE;
@@ -50,6 +50,7 @@ struct StepExec {
   ConvTcDesc ctc{};
   MmaChainDesc mma{};
   RankConvDesc rk{};
+  CatDesc cat{};
   std::string kernel;
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
@@ -274,6 +275,15 @@ void lower(temco_plan_s* P) {
           ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
         e.kind = K_GROUP_MMA;
         e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
+        e.launches = 1;
+        continue;
+      }
+      // single-level concats (DenseNet's layer groups, incl. pooled / avg-pooled members) on
+      // mma.sync: opt-in, measured 1.4-2.5x slower than the tcgen05 chain kernel on B200
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && (P->flags & TEMCO_FLAG_MMA_CAT) &&
+          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+        e.kind = K_GROUP_CAT;
+        e.kernel = "mma_cat";
         e.launches = 1;
         continue;
       }
@@ -511,6 +521,7 @@ std::string make_json(const temco_plan_s* P) {
           << ",\"ntiles\":" << e.tcw.ntiles << ",\"Cc\":" << e.tcw.Cc << ",\"levels\":" << e.tcw.n_levels << "}";
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_CONV_RK) o << ",\"alg_flops\":" << e.rk.alg_flops << ",\"alg_bytes\":" << e.rk.alg_bytes;
+      if (e.kind == K_GROUP_CAT) o << ",\"alg_flops\":" << e.cat.alg_flops << ",\"alg_bytes\":" << e.cat.alg_bytes;
       if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;
     }
     o << ",\"live\":" << ir.live_fused[t] << "}";
@@ -586,6 +597,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
       case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
       case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
       case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
+      case K_GROUP_CAT: launch_mma_cat(e.cat, P->tcw_d, rp, st); break;
       case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
     }
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t + 1], st));

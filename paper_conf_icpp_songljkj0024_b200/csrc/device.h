@@ -57,6 +57,38 @@ struct RankConvDesc {          // reduced-rank conv on tensor cores (kernels_ran
   int64_t alg_flops, alg_bytes;
 };
 
+// single-level concat group on mma.sync (kernels_cat.cu)
+constexpr int kCatMaxTerms = 40, kCatMaxUnits = 160, kCatMaxChunks = 32;
+enum : int8_t { CU_FIRST = 1, CU_LAST = 2, CU_POOLED = 4, CU_TAP_FIRST = 8, CU_TAP_LAST = 16 };
+struct CatTerm {
+  Loc r;                      // reduced input [N, Hin, Win, R] bf16 (arena)
+  int32_t R, ks, c0, C;       // rank, k-steps of 16, restored channel range
+  int32_t Hin, Win;
+  int32_t kind;               // 0 level term (tk > 1: folded avg pool), 1 pooled-member term
+  int32_t tk, ts, tp;         // tap window (term or pool), stride, pad
+  int32_t rs, w;              // SMEM row stride (elements), weight offset [C][rs] in the blob
+};
+struct CatUnit {              // one (64-channel chunk, term, tap) step of a 16-pixel block
+  int16_t term, chunk;        // term -1: a chunk no term reaches
+  int8_t tap, flags, nt0, nt1;   // n-tiles [nt0, nt1) of the chunk the term writes
+  int32_t woff;               // weight row of n-tile nt0 in the blob (elements)
+};
+struct CatDesc {
+  CatTerm term[kCatMaxTerms];
+  CatUnit unit[kCatMaxUnits];
+  int32_t n_terms, n_plain, n_units;
+  int32_t C, nchunks, Nout, NO;
+  int32_t H, W, npix, nblocks;
+  int32_t relu;               // level activation
+  int32_t pool, pk, ps, pp, mrelu, pc0, pc1;   // pooled member: kind, window, act, chunk range
+  int32_t f, fs;              // F [Nout][fs] offset (elements)
+  int32_t lbias, mbias;       // fp32 offsets (floats) after the bf16 part
+  int32_t blob_bf16, blob_bytes;
+  int64_t blob;               // tc weight pool offset
+  Loc y;
+  int64_t alg_flops, alg_bytes;
+};
+
 enum EwKind : int32_t { EW_BN, EW_RELU, EW_SILU, EW_ADD, EW_CONCAT, EW_MAXPOOL, EW_AVGPOOL, EW_GAP };
 
 constexpr int kMaxEwInputs = 64;

@@ -5,7 +5,10 @@
 
 #include <vector>
 
+#include <map>
+
 #include "device.h"
+#include "planner.h"
 
 namespace temco {
 
@@ -17,6 +20,10 @@ void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 // reduced-rank conv (Cin, K % 8 == 0, Cin <= 64, K <= 64) on tensor cores; w = fp32 [K][kh][kw][Cin]
 bool conv_rank_mma_lower(const ConvDesc& c, const float* w, std::vector<uint16_t>& tcw, RankConvDesc& d);
 void launch_conv_rank_mma(const RankConvDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s);
+// single-level concat group (kernels_cat.cu); false if the group is not of that form
+bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
+                   CatDesc& d);
+void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s);
 bool dwconv_vec_ok(const ConvDesc& d);   // depthwise bf16, C % 8 == 0: vectorised kernel
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)

@@ -1,0 +1,507 @@
+// Register-resident fused kernel for single-level concat groups on mma.sync
+// (bf16 mode): DenseNet's per-layer groups
+//     fconv( ReLU( BN( concat[ pool(stem restore) | avgpool(transition lconv) | lconv_1 | ... ] ) ) )
+// (Fig. 9a: concat -> fconv as one block-diagonal restore into the
+// same accumulator; P:L305-317 for the pooled member), SURVEY 8(a) row a6.
+//
+// The group is parsed into one level (chain_parse.h): plain terms (lconv rows,
+// BN-folded), tap-accumulate terms (avgpool over a linear member, weights / k^2)
+// and at most one max/avg-pooled non-linear member (evaluated per tap, then
+// pooled, then the post-BN shift).  The host flattens the work of one 16-pixel
+// output block into a unit list, identical for every block:
+//     for each 64-channel chunk: for each (term, tap) reaching it: one unit
+// and the kernel walks (block, unit) with the A fragments (the term's reduced
+// input rows at the tap, gathered straight from global memory into registers)
+// of the next two units in flight.  The restored 16 x 64 chunk lives in 32
+// accumulator registers; after its last unit it gets the level ReLU and is
+// re-packed in place as the A operand of the reduce GEMM (out += P F^T).
+// Everything is HBM-bound: bytes per pixel = sum of the reduced inputs + out.
+#include <cuda_bf16.h>
+
+#include <algorithm>
+#include <cmath>
+#include <set>
+
+#include "chain_parse.h"
+#include "kernels.h"
+
+namespace temco {
+
+namespace {
+using namespace chainp;
+
+uint16_t f2bf(float f) {
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  u += 0x7FFF + ((u >> 16) & 1);
+  return (uint16_t)(u >> 16);
+}
+
+}  // namespace
+
+bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
+                   CatDesc& d) {
+  const Node& root = ir.nodes[s.out];
+  if (root.role != ROLE_FCONV || root.b) return false;
+  const int tsrc = ir.oin[s.out][0];
+  const Node& tn = ir.nodes[tsrc];
+  const int C = tn.C, Nout = root.C;
+  if (Nout % 8 || Nout > 64 || C % 64 || C > 64 * kCatMaxChunks) return false;
+  ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
+  P.members.erase(s.out);
+  std::vector<PLevel> levels;
+  if (!P.chain(tsrc, levels)) return false;
+  if (P.visited != P.members || levels.size() != 1) return false;
+  const PLevel& L = levels[0];
+  if (L.pm.size() > 1) return false;
+  const PMember* pm = L.pm.empty() ? nullptr : &L.pm[0];
+  if (pm && (pm->c0 % 64 || pm->C % 64 || (pm->kind == 2 && pm->p != 0))) return false;
+
+  d = CatDesc();
+  d.C = C;
+  d.nchunks = C / 64;
+  d.Nout = Nout;
+  d.NO = Nout / 8;
+  d.H = tn.H;
+  d.W = tn.W;
+  d.npix = ir.batch * tn.H * tn.W;
+  if ((int64_t)ir.batch * tn.H * tn.W >= (1LL << 31) - 16) return false;
+  d.nblocks = (d.npix + 15) / 16;
+  d.relu = L.relu ? 1 : 0;
+  const Loc& yl = loc.at(s.out);
+  if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
+  d.y = yl;
+
+  std::vector<uint16_t> blob;
+  std::vector<float> fbias;
+  int64_t flops = 0, bytes = 0;
+  // terms: plain / tap-accumulate (level), then the pooled member's
+  auto add_term = [&](const PTerm& t, int kind) -> bool {
+    if (d.n_terms == kCatMaxTerms) return false;
+    const Node& lc = ir.nodes[t.lconv];
+    const int r = ir.oin[t.lconv][0];
+    const Node& rn = ir.nodes[r];
+    const Loc& rl = loc.at(r);
+    if (rl.where != W_ARENA || rl.dtype != DT_BF16 || rn.C % 8 || rn.C > 64 || lc.C % 8 || t.c0 % 8) return false;
+    CatTerm& T = d.term[d.n_terms++];
+    T.r = rl;
+    T.R = rn.C;
+    T.ks = (rn.C + 15) / 16;
+    T.c0 = t.c0;
+    T.C = lc.C;
+    T.Hin = rn.H;
+    T.Win = rn.W;
+    T.kind = kind;
+    if (kind == 0) {
+      T.tk = t.tk;
+      T.ts = t.ts;
+      T.tp = t.tp;
+    } else {
+      T.tk = pm->k;
+      T.ts = pm->s;
+      T.tp = pm->p;
+    }
+    T.rs = T.ks * 16 + 8;
+    while (blob.size() % 8) blob.push_back(0);
+    T.w = (int32_t)blob.size();
+    blob.resize(blob.size() + (size_t)lc.C * T.rs, 0);
+    for (int c = 0; c < lc.C; ++c)
+      for (int k = 0; k < T.R; ++k)
+        blob[T.w + (size_t)c * T.rs + k] = f2bf((float)(t.scale[c] * (*lc.w)[(size_t)c * T.R + k]));
+    const int64_t in_pix = (int64_t)ir.batch * rn.H * rn.W;
+    flops += in_pix * 2LL * lc.C * T.R;
+    bytes += in_pix * 2LL * T.R;
+    return true;
+  };
+  for (const PTerm& t : L.terms)
+    if (!add_term(t, 0)) return false;
+  d.n_plain = d.n_terms;
+  if (pm)
+    for (const PTerm& t : pm->terms)
+      if (!add_term(t, 1)) return false;
+  // F [Nout][C + 8]
+  while (blob.size() % 8) blob.push_back(0);
+  d.f = (int32_t)blob.size();
+  d.fs = C + 8;
+  blob.resize(blob.size() + (size_t)Nout * d.fs, 0);
+  for (int o = 0; o < Nout; ++o)
+    for (int c = 0; c < C; ++c) blob[d.f + (size_t)o * d.fs + c] = f2bf((*root.w)[(size_t)o * C + c]);
+  while (blob.size() % 8) blob.push_back(0);
+  d.blob_bf16 = (int32_t)blob.size();
+  // fp32: level bias [C] (pooled channels: the post-pool shift), member bias [C] (0 elsewhere)
+  d.lbias = 0;
+  d.mbias = C;
+  fbias.assign(2 * C, 0.f);
+  for (int c = 0; c < C; ++c) fbias[c] = (float)L.bias[c];
+  if (pm) {
+    for (int c = 0; c < pm->C; ++c) fbias[C + pm->c0 + c] = (float)pm->bias[c];
+    d.pool = pm->kind;
+    d.pk = pm->k;
+    d.ps = pm->s;
+    d.pp = pm->p;
+    d.mrelu = pm->relu ? 1 : 0;
+    d.pc0 = pm->c0 / 64;
+    d.pc1 = (pm->c0 + pm->C) / 64;
+  }
+  for (float b : fbias) {
+    uint32_t u;
+    memcpy(&u, &b, 4);
+    blob.push_back((uint16_t)(u & 0xFFFF));
+    blob.push_back((uint16_t)(u >> 16));
+  }
+  while (blob.size() % 8) blob.push_back(0);
+  d.blob_bytes = (int32_t)blob.size() * 2;
+  if (d.blob_bytes > 200 * 1024) return false;
+  // unit list of one block
+  std::vector<CatUnit> U;
+  for (int ch = 0; ch < d.nchunks; ++ch) {
+    const bool pooled = pm && ch >= d.pc0 && ch < d.pc1;
+    const size_t first = U.size();
+    auto hits = [&](const CatTerm& T, int& lo, int& hi) {
+      lo = std::max(T.c0, ch * 64);
+      hi = std::min(T.c0 + T.C, ch * 64 + 64);
+      return lo < hi;
+    };
+    if (pooled) {
+      const int taps = pm->k * pm->k;
+      for (int tap = 0; tap < taps; ++tap) {
+        const size_t tf = U.size();
+        for (int j = d.n_plain; j < d.n_terms; ++j) {
+          int lo, hi;
+          if (!hits(d.term[j], lo, hi)) continue;
+          CatUnit u{};
+          u.term = (int16_t)j;
+          u.tap = (int8_t)tap;
+          u.chunk = (int16_t)ch;
+          u.nt0 = (int8_t)((lo - ch * 64) / 8);
+          u.nt1 = (int8_t)((hi - ch * 64) / 8);
+          u.woff = d.term[j].w + (lo - d.term[j].c0) * d.term[j].rs;
+          U.push_back(u);
+        }
+        if (U.size() == tf) return false;
+        U[tf].flags |= CU_TAP_FIRST;
+        U.back().flags |= CU_TAP_LAST;
+      }
+    } else {
+      for (int j = 0; j < d.n_plain; ++j) {
+        int lo, hi;
+        if (!hits(d.term[j], lo, hi)) continue;
+        for (int tap = 0; tap < d.term[j].tk * d.term[j].tk; ++tap) {
+          CatUnit u{};
+          u.term = (int16_t)j;
+          u.tap = (int8_t)tap;
+          u.chunk = (int16_t)ch;
+          u.nt0 = (int8_t)((lo - ch * 64) / 8);
+          u.nt1 = (int8_t)((hi - ch * 64) / 8);
+          u.woff = d.term[j].w + (lo - d.term[j].c0) * d.term[j].rs;
+          U.push_back(u);
+        }
+      }
+      if (U.size() == first) {   // a chunk no term reaches (zero restore): one empty unit
+        CatUnit u{};
+        u.term = -1;
+        u.chunk = (int16_t)ch;
+        U.push_back(u);
+      }
+    }
+    U[first].flags |= CU_FIRST;
+    U.back().flags |= CU_LAST;
+    if (pooled) U[first].flags |= CU_POOLED, U.back().flags |= CU_POOLED;
+    for (size_t i = first; i < U.size(); ++i)
+      if (pooled) U[i].flags |= CU_POOLED;
+  }
+  if ((int)U.size() > kCatMaxUnits) return false;
+  d.n_units = (int)U.size();
+  for (int i = 0; i < d.n_units; ++i) d.unit[i] = U[i];
+  while (tcw.size() % 512) tcw.push_back(0);
+  d.blob = (int64_t)tcw.size();
+  tcw.insert(tcw.end(), blob.begin(), blob.end());
+  d.alg_flops = flops + (int64_t)d.npix * 2LL * Nout * C;
+  d.alg_bytes = bytes + (int64_t)d.npix * 2LL * Nout;
+  return true;
+}
+
+namespace {
+
+constexpr int kCatWarps = 16;
+
+__device__ __forceinline__ uint32_t s_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3)
+               : "r"(addr));
+}
+
+__device__ __forceinline__ void ldsm_x2(uint32_t addr, uint32_t& r0, uint32_t& r1) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0, %1}, [%2];" : "=r"(r0), "=r"(r1) : "r"(addr));
+}
+
+__device__ __forceinline__ void mma16816(float (&c)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+      "{%0, %1, %2, %3};"
+      : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+__device__ __forceinline__ uint32_t pk2(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+// output-pixel coordinates of the two fragment rows of a block
+struct CatRows {
+  int n[2], ho[2], wo[2];
+  bool ok[2];
+};
+
+__device__ __forceinline__ CatRows cat_rows(const CatDesc& d, int blk, int g) {
+  CatRows r;
+  const int hw = d.H * d.W;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const int m = blk * 16 + g + 8 * h;
+    r.ok[h] = m < d.npix;
+    r.n[h] = m / hw;
+    const int rem = m - r.n[h] * hw;
+    r.ho[h] = rem / d.W;
+    r.wo[h] = rem - r.ho[h] * d.W;
+  }
+  return r;
+}
+
+// A fragments of one unit (term, tap) for the block's rows; also the rows'
+// tap validity (max-pool masking)
+template <int KSM>
+__device__ __forceinline__ void cat_load(uint32_t (&a)[KSM][4], bool (&valid)[2], const CatDesc& d, const RunPtrs& p,
+                                         const CatUnit& u, const CatRows& rw, int t4) {
+  if (u.term < 0) {
+#pragma unroll
+    for (int ks = 0; ks < KSM; ++ks) a[ks][0] = a[ks][1] = a[ks][2] = a[ks][3] = 0u;
+    valid[0] = valid[1] = false;
+    return;
+  }
+  const CatTerm& T = d.term[u.term];
+  const uint32_t* x = reinterpret_cast<const uint32_t*>(p.arena + T.r.off);
+  const int ty = u.tap / T.tk, tx = u.tap - ty * T.tk;
+  int64_t off[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const int hi = rw.ho[h] * T.ts - T.tp + ty, wi = rw.wo[h] * T.ts - T.tp + tx;
+    valid[h] = rw.ok[h] && hi >= 0 && hi < T.Hin && wi >= 0 && wi < T.Win;
+    off[h] = ((int64_t)(rw.n[h] * T.Hin + hi) * T.Win + wi) * (T.R / 2);
+  }
+#pragma unroll
+  for (int ks = 0; ks < KSM; ++ks) {
+    const int k0 = ks * 16 + 2 * t4, k1 = k0 + 8;
+    a[ks][0] = (valid[0] && k0 < T.R) ? __ldg(x + off[0] + k0 / 2) : 0u;
+    a[ks][1] = (valid[1] && k0 < T.R) ? __ldg(x + off[1] + k0 / 2) : 0u;
+    a[ks][2] = (valid[0] && k1 < T.R) ? __ldg(x + off[0] + k1 / 2) : 0u;
+    a[ks][3] = (valid[1] && k1 < T.R) ? __ldg(x + off[1] + k1 / 2) : 0u;
+  }
+}
+
+template <int NO, int KSM, bool POOL>
+__global__ void __launch_bounds__(32 * kCatWarps, 1) mma_cat_kernel(const __grid_constant__ CatDesc d, RunPtrs p,
+                                                                     const uint16_t* __restrict__ tcw) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int g = lane / 4, t4 = lane % 4;
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(tcw + d.blob);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  __syncthreads();
+  const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
+  const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+  const int lq = lane >> 3, lr = lane & 7;
+  const uint32_t sbase = s_u32(blob);
+  const int nw = gridDim.x * kCatWarps;
+  const int NU = d.n_units;
+  // prefetch cursor: (block, unit) two units ahead of the compute cursor
+  int pblk = blockIdx.x * kCatWarps + warp, pu = 0;
+  CatRows prow = cat_rows(d, pblk, g);
+  uint32_t a[KSM][4], an[KSM][4], ann[KSM][4];
+  bool va[2], van[2], vann[2];
+  auto pf_next = [&](uint32_t (&dst)[KSM][4], bool (&v)[2]) {
+    if (pblk < d.nblocks) cat_load<KSM>(dst, v, d, p, d.unit[pu], prow, t4);
+    if (++pu == NU) {
+      pu = 0;
+      pblk += nw;
+      prow = cat_rows(d, pblk, g);
+    }
+  };
+  pf_next(a, va);
+  pf_next(an, van);
+  float O[NO][4];
+  float D[8][4], run[POOL ? 8 : 1][4];
+  for (int blk = blockIdx.x * kCatWarps + warp; blk < d.nblocks; blk += nw) {
+#pragma unroll
+    for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
+    for (int ui = 0; ui < NU; ++ui) {
+      pf_next(ann, vann);
+      const CatUnit u = d.unit[ui];
+      const int c0 = u.chunk * 64;
+      const bool pooled = POOL && (u.flags & CU_POOLED) != 0;
+      if ((u.flags & CU_FIRST) && !pooled) {
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt) {
+          const float2 b = *reinterpret_cast<const float2*>(fb + d.lbias + c0 + nt * 8 + 2 * t4);
+          D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+        }
+      }
+      if (pooled && (u.flags & CU_TAP_FIRST)) {
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt) {
+          const float2 b = *reinterpret_cast<const float2*>(fb + d.mbias + c0 + nt * 8 + 2 * t4);
+          D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+        }
+      }
+      if (u.term >= 0) {
+        const int nks = d.term[u.term].ks, rs = d.term[u.term].rs;
+        // lane address of ldmatrix: rows (n-tile base + lr), k half lq & 1; x4 covers two n-tiles
+        const uint32_t wb = sbase + (uint32_t)((u.woff + ((lq >> 1) * 8 + lr) * rs + (lq & 1) * 8) * 2);
+        const uint32_t wb2 = sbase + (uint32_t)((u.woff + lr * rs + (lq & 1) * 8) * 2);
+#pragma unroll
+        for (int ks = 0; ks < KSM; ++ks) {
+          if (ks < nks) {
+#pragma unroll
+            for (int nt = 0; nt < 8; nt += 2) {
+              if (nt >= u.nt0 && nt < u.nt1) {
+                const uint32_t roff = (uint32_t)(((nt - u.nt0) * 8 * rs + ks * 16) * 2);
+                if (nt + 1 < u.nt1) {
+                  uint32_t b0, b1, b2, b3;
+                  ldsm_x4(wb + roff, b0, b1, b2, b3);
+                  mma16816(D[nt], a[ks], b0, b1);
+                  mma16816(D[nt + 1], a[ks], b2, b3);
+                } else {
+                  uint32_t b0, b1;
+                  ldsm_x2(wb2 + roff, b0, b1);
+                  mma16816(D[nt], a[ks], b0, b1);
+                }
+              } else if (nt + 1 >= u.nt0 && nt + 1 < u.nt1) {   // odd start: tile nt + 1 alone
+                uint32_t b0, b1;
+                ldsm_x2(wb2 + (uint32_t)(((nt + 1 - u.nt0) * 8 * rs + ks * 16) * 2), b0, b1);
+                mma16816(D[nt + 1], a[ks], b0, b1);
+              }
+            }
+          }
+        }
+      }
+      if constexpr (POOL) if (pooled && (u.flags & CU_TAP_LAST)) {
+        // member activation, max / sum over the pooling window (max: taps outside excluded)
+        const int tap = u.tap;
+        const float n0 = (d.pool == 1 && !va[0]) ? -INFINITY : 0.f;
+        const float n1 = (d.pool == 1 && !va[1]) ? -INFINITY : 0.f;
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            float z = d.mrelu ? fmaxf(D[nt][i], 0.f) : D[nt][i];
+            z += i < 2 ? n0 : n1;
+            run[nt][i] = tap == 0 ? z : d.pool == 1 ? fmaxf(run[nt][i], z) : run[nt][i] + z;
+          }
+      }
+      if (u.flags & CU_LAST) {
+        if constexpr (POOL) if (pooled) {
+          const float sc = d.pool == 2 ? 1.f / (float)(d.pk * d.pk) : 1.f;
+#pragma unroll
+          for (int nt = 0; nt < 8; ++nt) {
+            const float2 b = *reinterpret_cast<const float2*>(fb + d.lbias + c0 + nt * 8 + 2 * t4);
+            D[nt][0] = run[nt][0] * sc + b.x;
+            D[nt][1] = run[nt][1] * sc + b.y;
+            D[nt][2] = run[nt][2] * sc + b.x;
+            D[nt][3] = run[nt][3] * sc + b.y;
+          }
+        }
+        if (d.relu) {
+#pragma unroll
+          for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+            for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+        }
+        // reduce: O += P F^T over this chunk
+#pragma unroll
+        for (int kp = 0; kp < 2; ++kp) {
+          uint32_t pa[2][4];
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int ks = 2 * kp + h;
+            pa[h][0] = pk2(D[2 * ks][0], D[2 * ks][1]);
+            pa[h][1] = pk2(D[2 * ks][2], D[2 * ks][3]);
+            pa[h][2] = pk2(D[2 * ks + 1][0], D[2 * ks + 1][1]);
+            pa[h][3] = pk2(D[2 * ks + 1][2], D[2 * ks + 1][3]);
+          }
+#pragma unroll
+          for (int nb = 0; nb < NO; ++nb) {
+            if (nb >= d.NO) break;   // NO is the template bound (even), d.NO the real n-tile count
+            uint32_t f0, f1, f2, f3;
+            ldsm_x4(sbase + (uint32_t)((d.f + (nb * 8 + lr) * d.fs + c0 + kp * 32 + lq * 8) * 2), f0, f1, f2, f3);
+            mma16816(O[nb], pa[0], f0, f1);
+            mma16816(O[nb], pa[1], f2, f3);
+          }
+        }
+      }
+#pragma unroll
+      for (int ks = 0; ks < KSM; ++ks)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          a[ks][i] = an[ks][i];
+          an[ks][i] = ann[ks][i];
+        }
+      va[0] = van[0]; va[1] = van[1];
+      van[0] = vann[0]; van[1] = vann[1];
+    }
+    const int m0 = blk * 16 + g, m1 = m0 + 8;
+#pragma unroll
+    for (int nb = 0; nb < NO; ++nb) {
+      if (nb >= d.NO) break;
+      const int col = nb * 8 + 2 * t4;
+      if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + (int64_t)m0 * d.Nout + col) = pk2(O[nb][0], O[nb][1]);
+      if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + (int64_t)m1 * d.Nout + col) = pk2(O[nb][2], O[nb][3]);
+    }
+  }
+}
+
+template <int NO, int KSM, bool POOL>
+void launch_cat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  if (!configured) {
+    cudaFuncSetAttribute(mma_cat_kernel<NO, KSM, POOL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mma_cat_kernel<NO, KSM, POOL>, 32 * kCatWarps, d.blob_bytes);
+  const int grid = std::min((d.nblocks + kCatWarps - 1) / kCatWarps, sms * std::max(per_sm, 1));
+  mma_cat_kernel<NO, KSM, POOL><<<grid, 32 * kCatWarps, d.blob_bytes, s>>>(d, p, tcw);
+}
+
+template <int KSM, bool POOL>
+void launch_cat_no(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  switch ((d.NO + 1) / 2) {
+    case 1: return launch_cat_t<2, KSM, POOL>(d, tcw, p, s);
+    case 2: return launch_cat_t<4, KSM, POOL>(d, tcw, p, s);
+    case 3: return launch_cat_t<6, KSM, POOL>(d, tcw, p, s);
+    default: return launch_cat_t<8, KSM, POOL>(d, tcw, p, s);
+  }
+}
+
+}  // namespace
+
+void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  int ksm = 1;
+  for (int j = 0; j < d.n_terms; ++j) ksm = std::max(ksm, d.term[j].ks);
+  const bool pool = d.pool != 0;
+  if (ksm == 1) return pool ? launch_cat_no<1, true>(d, tcw, p, s) : launch_cat_no<1, false>(d, tcw, p, s);
+  if (ksm == 2) return pool ? launch_cat_no<2, true>(d, tcw, p, s) : launch_cat_no<2, false>(d, tcw, p, s);
+  return pool ? launch_cat_no<4, true>(d, tcw, p, s) : launch_cat_no<4, false>(d, tcw, p, s);
+}
+
+}  // namespace temco

@@ -29,6 +29,7 @@ FLAG_SIMT_ONLY = 1 << 4
 FLAG_OVERHEAD_ALWAYS = 1 << 5
 FLAG_OVERHEAD_NEVER = 1 << 6
 FLAG_MMA_SMALL = 1 << 7
+FLAG_MMA_CAT = 1 << 8
 
 EXPORTS = ["temco_plan_create", "temco_run", "temco_run_host", "temco_peak_internal_bytes", "temco_output_shape",
            "temco_plan_describe", "temco_run_profiled", "temco_plan_destroy", "temco_status_string",

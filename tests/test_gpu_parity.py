@@ -63,11 +63,11 @@ def test_fp32_mode(name):
 
 @pytest.mark.parametrize("name", list(SMALL))
 def test_bf16_mode(name):
-    from paper_conf_icpp_songljkj0024_b200 import FLAG_MMA_SMALL, FLAG_SIMT_ONLY
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_MMA_CAT, FLAG_MMA_SMALL, FLAG_SIMT_ONLY
     m = SMALL[name]("bf16")
     x = W.make_input(m)
     ref = oracle.run_temco(oracle.plan(m), x)
-    for flags in (0, FLAG_SIMT_ONLY, FLAG_MMA_SMALL):
+    for flags in (0, FLAG_SIMT_ONLY, FLAG_MMA_SMALL, FLAG_MMA_CAT):
         p, y = _plan_and_run(m, flags=flags, x=x)
         assert np.isfinite(y).all()
         assert _rel(y, ref) <= 2e-2, (flags, _rel(y, ref))

@@ -1,0 +1,35 @@
+"""The small parity cases of test_gpu_parity.py exercise every kernel family the
+full-size bench configs launch (host-only: plans with TEMCO_FLAG_NO_DEVICE pick
+the same kernels as device plans)."""
+import collections
+
+import workloads as W
+
+
+def _kernels(m, flags=0):
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_NO_DEVICE, Plan
+    p = Plan(m, flags=FLAG_NO_DEVICE | flags)
+    return collections.Counter(s["kernel"] for s in p.describe()["steps"])
+
+
+def test_small_cases_cover_the_full_configs():
+    small = collections.Counter()
+    for m in (W.resnet18_cifar(batch=3, dtype="bf16", height=16, width=16),
+              W.resnet50(batch=2, dtype="bf16", height=64, width=64),
+              W.vgg16_cp(batch=2, dtype="bf16", height=32, width=32),
+              W.densenet121(batch=2, dtype="bf16", height=64, width=64)):
+        small.update(_kernels(m))
+    full = collections.Counter()
+    for name in ("resnet18_cifar", "resnet50", "vgg16_cp", "densenet121"):
+        full.update(_kernels(W.build_config(name)))
+    assert set(full) <= set(small), set(full) - set(small)
+    # the tensor-core families are all on the bench path
+    for k in ("tc_chain", "mma_lean", "mma_conv_rank", "mma_conv_stem", "tc_conv"):
+        assert full[k] > 0, k
+
+
+def test_opt_in_concat_kernel_is_selected_by_its_flag():
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_MMA_CAT
+    m = W.densenet121(batch=2, dtype="bf16", height=64, width=64)
+    assert _kernels(m)["mma_cat"] == 0
+    assert _kernels(m, FLAG_MMA_CAT)["mma_cat"] > 0
