@@ -629,6 +629,162 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
   }
 }
 
+// 64-channel, rank <= 16 groups (VGG's block-1/2 groups, ResNet's stage-1 in-block
+// groups, the stem-restore copies): every operand but A is register-resident
+// for the whole kernel -- restore weights (16 regs), fconv weights, biases --
+// and the bias enters through the MMA's C operand (D = A B + bias), so a
+// 16-pixel block costs ~12 MMAs + ReLU / re-pack, about a third of the
+// instructions of the generic lean path.
+
+__device__ __forceinline__ void mma16816c(float (&dd)[4], uint32_t a0, uint32_t a1, uint32_t a2, uint32_t a3,
+                                          uint32_t b0, uint32_t b1, float c0, float c1) {
+  asm volatile(
+      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0, %1, %2, %3}, {%4, %5, %6, %7}, {%8, %9}, "
+      "{%10, %11, %10, %11};"
+      : "=f"(dd[0]), "=f"(dd[1]), "=f"(dd[2]), "=f"(dd[3])
+      : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1), "f"(c0), "f"(c1));
+}
+
+template <int NO, bool POOL, int kL64Warps = POOL ? 8 : 16>   // pooled: run[] needs > 128 registers
+__global__ void __launch_bounds__(32 * kL64Warps, 1) mma_lean64_kernel(const __grid_constant__ MmaChainDesc d,
+                                                                       RunPtrs p, const uint16_t* __restrict__ tcw) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int g = lane / 4, t4 = lane % 4;
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(tcw + d.blob);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  __syncthreads();
+  const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
+  const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2) + d.bias[0];
+  const MmaTerm& T = d.term[0];
+  const uint32_t* r = reinterpret_cast<const uint32_t*>(p.arena + T.r.off);
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+  const int rs = T.Rp + 8, fs = d.Cpad + 8;
+  const int lq = lane >> 3, lr = lane & 7;
+  // register-resident operands: restore B fragments, fconv B fragments, biases
+  uint32_t wb[8][2], fw[NO][4][2];
+  float bias[8][2];
+#pragma unroll
+  for (int np = 0; np < 4; ++np)
+    ldsm_x4(s_u32(blob + T.w + (np * 16 + (lq >> 1) * 8 + lr) * rs + (lq & 1) * 8), wb[2 * np][0], wb[2 * np][1],
+            wb[2 * np + 1][0], wb[2 * np + 1][1]);
+#pragma unroll
+  for (int nb = 0; nb < NO; ++nb)
+#pragma unroll
+    for (int kp = 0; kp < 2; ++kp)
+      ldsm_x4(s_u32(blob + d.f + (nb * 8 + lr) * fs + kp * 32 + lq * 8), fw[nb][2 * kp][0], fw[nb][2 * kp][1],
+              fw[nb][2 * kp + 1][0], fw[nb][2 * kp + 1][1]);
+#pragma unroll
+  for (int nt = 0; nt < 8; ++nt) {
+    const float2 b = *reinterpret_cast<const float2*>(fb + nt * 8 + 2 * t4);
+    bias[nt][0] = b.x;
+    bias[nt][1] = b.y;
+  }
+  const bool relu = d.relu[0] != 0;
+  const int taps = POOL ? d.taps : 1;
+  const int64_t nw = (int64_t)gridDim.x * kL64Warps;
+  auto advance = [&](LeanCursor& u) {
+    if (++u.tap == taps) {
+      u.tap = 0;
+      u.blk += nw;
+      if (u.blk < d.nblocks) lean_set_block(d, u, g);
+    }
+  };
+  LeanCursor cur{};
+  cur.blk = (int64_t)blockIdx.x * kL64Warps + warp;
+  if (cur.blk < d.nblocks) lean_set_block(d, cur, g);
+  LeanCursor pf = cur;
+  uint32_t a[1][4], an[1][4], ann[1][4];
+  if (pf.blk < d.nblocks) lean_load_a<1>(a, d, r, pf, T.R, g, t4);
+  advance(pf);
+  if (pf.blk < d.nblocks) lean_load_a<1>(an, d, r, pf, T.R, g, t4);
+  advance(pf);
+  float run[POOL ? 8 : 1][4];
+  const float sc = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
+  for (; cur.blk < d.nblocks; advance(cur)) {
+    if (pf.blk < d.nblocks) lean_load_a<1>(ann, d, r, pf, T.R, g, t4);
+    advance(pf);
+    float D[8][4];
+#pragma unroll
+    for (int nt = 0; nt < 8; ++nt)
+      mma16816c(D[nt], a[0][0], a[0][1], a[0][2], a[0][3], wb[nt][0], wb[nt][1], bias[nt][0], bias[nt][1]);
+    if (relu) {
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+    }
+    bool last = true;
+    if constexpr (POOL) {
+      float n0 = 0.f, n1 = 0.f;
+      if (d.pool == 1) {
+        n0 = lean_tap_valid(d, cur, 0) ? 0.f : -INFINITY;
+        n1 = lean_tap_valid(d, cur, 1) ? 0.f : -INFINITY;
+      }
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt) {
+        const float x[4] = {D[nt][0] + n0, D[nt][1] + n0, D[nt][2] + n1, D[nt][3] + n1};
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          run[nt][i] = cur.tap == 0 ? x[i] : d.pool == 1 ? fmaxf(run[nt][i], x[i]) : run[nt][i] + x[i];
+      }
+      last = cur.tap == taps - 1;
+      if (last) {
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) D[nt][i] = run[nt][i] * sc;
+      }
+    }
+    if (last) {
+      float O[NO][4];
+#pragma unroll
+      for (int ks = 0; ks < 4; ++ks) {
+        const uint32_t p0 = pk2(D[2 * ks][0], D[2 * ks][1]), p1 = pk2(D[2 * ks][2], D[2 * ks][3]);
+        const uint32_t p2 = pk2(D[2 * ks + 1][0], D[2 * ks + 1][1]), p3 = pk2(D[2 * ks + 1][2], D[2 * ks + 1][3]);
+#pragma unroll
+        for (int nb = 0; nb < NO; ++nb) {
+          if (ks == 0)
+            mma16816c(O[nb], p0, p1, p2, p3, fw[nb][0][0], fw[nb][0][1], 0.f, 0.f);
+          else
+            mma16816(O[nb], p0, p1, p2, p3, fw[nb][ks][0], fw[nb][ks][1]);
+        }
+      }
+      const int64_t m0 = cur.blk * 16 + g, m1 = m0 + 8;
+#pragma unroll
+      for (int nb = 0; nb < NO; ++nb) {
+        const int col = nb * 8 + 2 * t4;
+        if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + m0 * d.Nout + col) = pk2(O[nb][0], O[nb][1]);
+        if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + m1 * d.Nout + col) = pk2(O[nb][2], O[nb][3]);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      a[0][i] = an[0][i];
+      an[0][i] = ann[0][i];
+    }
+  }
+}
+
+template <int NO, bool POOL>
+void launch_lean64_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  if (!configured) {
+    cudaFuncSetAttribute(mma_lean64_kernel<NO, POOL>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  constexpr int kW = POOL ? 8 : 16;
+  const int grid = (int)std::min<int64_t>((d.nblocks + kW - 1) / kW, (int64_t)sms);
+  mma_lean64_kernel<NO, POOL><<<grid, 32 * kW, d.blob_bytes, s>>>(d, p, tcw);
+}
+
 template <int KS, int NO>
 void launch_lean_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   static bool configured = false;
@@ -652,6 +808,12 @@ bool mma_lean_ok(const MmaChainDesc& d) {
 }
 
 void launch_mma_chain(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  // register-resident 64-channel variant; pooled groups stay on the generic lean path
+  // (their running max needs > 128 registers: 8 warps per SM measured slower)
+  if (mma_lean_ok(d) && d.Cpad == 64 && d.term[0].Rp == 16 && d.Nout <= 16 && !d.pool) {
+    if (d.Nout <= 8) return launch_lean64_t<1, false>(d, tcw, p, s);
+    return launch_lean64_t<2, false>(d, tcw, p, s);
+  }
   if (mma_lean_ok(d)) {
     const int ks = d.term[0].Rp / 16, no = (d.Nout + 7) / 8;
 #define TEMCO_LEAN_CASE(k, n) \
