@@ -211,15 +211,22 @@ def main():
     value = ws * B / (ms_per_step / 1e3)
 
     # ---- end to end through the public API with host buffers -----------------
+    # temco_run_host_async: every step copies its input host->device (pinned,
+    # on the plan's copy stream, overlapping the previous step's compute), runs,
+    # and copies the logits back; the region ends after the last D2H completes
     xh = torch.from_numpy(x_host).to(tdt).pin_memory()
     yh = torch.empty(out_shape, dtype=torch.float32).pin_memory()
     plan.run_host(xh, yh, stream)
+    plan.run_host_async(xh, yh, stream)
+    torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     if ws > 1:
         dist.barrier()
     e0.record(stream)
     for _ in range(args.steps):
-        plan.run_host(xh, yh, stream)
+        plan.run_host_async(xh, yh, stream)
+        if ws > 1:
+            gather_logits(y, ws, gathered)
     e1.record(stream)
     torch.cuda.synchronize()
     e2e_ms = e0.elapsed_time(e1) / args.steps
@@ -295,7 +302,7 @@ def main():
                        "internal_memory_reduction": 1 - plan.peak_internal_bytes(0) / plan.peak_internal_bytes(1),
                        "cuda_graph": True, "kernels": "simt-only" if args.simt_only else "tcgen05+simt"},
             "gpu_launches": desc["launches"] * args.steps,
-            "e2e": {"value": ws * B / (e2e_ms / 1e3), "unit": "images/s",
+            "e2e": {"value": ws * B / (e2e_ms / 1e3), "unit": "images/s", "api": "temco_run_host_async (pipelined H2D)",
                     "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),
                     "d2h_bytes_per_step": int(yh.numel() * yh.element_size())},
             "roofline": {"bound": bound, "kernel": dom, "achieved": achieved, "peak": peak, "unit": unit,

@@ -150,6 +150,17 @@ temco_status temco_run(temco_plan_t plan, const void* input, void* output, temco
 temco_status temco_run_host(temco_plan_t plan, const void* host_input, void* host_output,
                             temco_stream_t stream);
 
+/* Asynchronous, pipelined variant of temco_run_host for a stream of batches:
+ * the host->device copy of this call's input runs on a plan-owned copy stream
+ * into one of two plan-owned staging buffers (alternating per call), so it
+ * overlaps the previous call's compute; the run and the device->host copy of
+ * the output are enqueued on `stream`.  Returns without synchronising: the
+ * caller synchronises `stream` before reading host_output or reusing
+ * host_input (pinned memory required for the overlap).  Consecutive calls on
+ * one plan must use the same stream (the arena is shared; runs serialise). */
+temco_status temco_run_host_async(temco_plan_t plan, const void* host_input, void* host_output,
+                                  temco_stream_t stream);
+
 /* Peak internal-tensor bytes (Eq. (3)/(4), reading R14): which = 0 -> the
  * fused TeMCO schedule, 1 -> the unfused decomposed list L. */
 temco_status temco_peak_internal_bytes(temco_plan_t plan, int32_t which, int64_t* bytes);

@@ -85,6 +85,12 @@ struct temco_plan_s {
   int64_t in_bytes = 0, out_bytes = 0;
   void* host_in_d = nullptr;
   void* host_out_d = nullptr;
+  // temco_run_host_async: double-buffered staging, copy stream, per-buffer events
+  void* async_in_d[2] = {nullptr, nullptr};
+  void* async_out_d[2] = {nullptr, nullptr};
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_in_ready[2] = {nullptr, nullptr}, ev_buf_free[2] = {nullptr, nullptr};
+  int async_flip = 0;
   int max_expr_depth = 0;          // deepest fused-group expression (SIMT interpreter recursion)
   int64_t out_dims[4] = {0, 0, 0, 0};
   int out_ndim = 0;
@@ -549,6 +555,13 @@ void free_device(temco_plan_s* P) {
   cudaFree(P->arena_d);
   cudaFree(P->host_in_d);
   cudaFree(P->host_out_d);
+  for (int b = 0; b < 2; ++b) {
+    cudaFree(P->async_in_d[b]);
+    cudaFree(P->async_out_d[b]);
+    if (P->ev_in_ready[b]) cudaEventDestroy(P->ev_in_ready[b]);
+    if (P->ev_buf_free[b]) cudaEventDestroy(P->ev_buf_free[b]);
+  }
+  if (P->copy_stream) cudaStreamDestroy(P->copy_stream);
   cudaFree(P->lin_ws_d);
   if (P->blas) cublasDestroy(P->blas);
 }
@@ -790,6 +803,37 @@ temco_status temco_run_host(temco_plan_t P, const void* host_input, void* host_o
   if (st != TEMCO_OK) return st;
   CUDA_TRY(cudaMemcpyAsync(host_output, P->host_out_d, P->out_bytes, cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaStreamSynchronize(s));
+  return TEMCO_OK;
+}
+
+temco_status temco_run_host_async(temco_plan_t P, const void* host_input, void* host_output,
+                                  temco_stream_t stream) {
+  temco_status st = check_device(P);
+  if (st != TEMCO_OK) return st;
+  if (!host_input || !host_output) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "host buffers are NULL");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (!P->copy_stream) {
+    for (int b = 0; b < 2; ++b)
+      if (cudaMalloc(&P->async_in_d[b], P->in_bytes) != cudaSuccess ||
+          cudaMalloc(&P->async_out_d[b], P->out_bytes) != cudaSuccess)
+        return set_err(TEMCO_ERR_OUT_OF_MEMORY, "async staging buffers");
+    CUDA_TRY(cudaStreamCreateWithFlags(&P->copy_stream, cudaStreamNonBlocking));
+    for (int b = 0; b < 2; ++b) {
+      CUDA_TRY(cudaEventCreateWithFlags(&P->ev_in_ready[b], cudaEventDisableTiming));
+      CUDA_TRY(cudaEventCreateWithFlags(&P->ev_buf_free[b], cudaEventDisableTiming));
+    }
+  }
+  const int b = P->async_flip;
+  P->async_flip ^= 1;
+  // staging buffer b is free once the run that read it (two calls ago) is done
+  CUDA_TRY(cudaStreamWaitEvent(P->copy_stream, P->ev_buf_free[b], 0));
+  CUDA_TRY(cudaMemcpyAsync(P->async_in_d[b], host_input, P->in_bytes, cudaMemcpyHostToDevice, P->copy_stream));
+  CUDA_TRY(cudaEventRecord(P->ev_in_ready[b], P->copy_stream));
+  CUDA_TRY(cudaStreamWaitEvent(s, P->ev_in_ready[b], 0));
+  st = temco_run(P, P->async_in_d[b], P->async_out_d[b], stream);
+  if (st != TEMCO_OK) return st;
+  CUDA_TRY(cudaEventRecord(P->ev_buf_free[b], s));
+  CUDA_TRY(cudaMemcpyAsync(host_output, P->async_out_d[b], P->out_bytes, cudaMemcpyDeviceToHost, s));
   return TEMCO_OK;
 }
 

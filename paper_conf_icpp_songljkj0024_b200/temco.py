@@ -31,7 +31,7 @@ FLAG_OVERHEAD_NEVER = 1 << 6
 FLAG_MMA_SMALL = 1 << 7
 FLAG_MMA_CAT = 1 << 8
 
-EXPORTS = ["temco_plan_create", "temco_run", "temco_run_host", "temco_peak_internal_bytes", "temco_output_shape",
+EXPORTS = ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_peak_internal_bytes", "temco_output_shape",
            "temco_plan_describe", "temco_run_profiled", "temco_plan_destroy", "temco_status_string",
            "temco_last_error"]
 
@@ -63,6 +63,7 @@ _lib.temco_plan_create.argtypes = [C.POINTER(_Layer), C.c_int32, C.POINTER(_Deco
                                    C.c_int32, C.POINTER(_Config), C.POINTER(C.c_void_p)]
 _lib.temco_run.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
 _lib.temco_run_host.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
+_lib.temco_run_host_async.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
 _lib.temco_run_profiled.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, _fp, C.c_int32]
 _lib.temco_peak_internal_bytes.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_int64)]
 _lib.temco_output_shape.argtypes = [C.c_void_p, C.POINTER(C.c_int64), C.POINTER(C.c_int32)]
@@ -71,7 +72,7 @@ _lib.temco_plan_destroy.argtypes = [C.c_void_p]
 _lib.temco_status_string.argtypes = [C.c_int]
 _lib.temco_status_string.restype = C.c_char_p
 _lib.temco_last_error.restype = C.c_char_p
-for _f in ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_profiled", "temco_peak_internal_bytes",
+for _f in ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_run_profiled", "temco_peak_internal_bytes",
            "temco_output_shape", "temco_plan_describe", "temco_plan_destroy"]:
     getattr(_lib, _f).restype = C.c_int
 
@@ -194,6 +195,14 @@ class Plan:
         yp = y_host.data_ptr() if hasattr(y_host, "data_ptr") else y_host.ctypes.data
         _check(_lib.temco_run_host(self._h, C.c_void_p(xp), C.c_void_p(yp), _stream_handle(stream)),
                "temco_run_host")
+
+    def run_host_async(self, x_host, y_host, stream=None):
+        """Pipelined host-buffer run (temco_run_host_async): returns before the
+        work completes; synchronise `stream` before reading y_host."""
+        xp = x_host.data_ptr() if hasattr(x_host, "data_ptr") else x_host.ctypes.data
+        yp = y_host.data_ptr() if hasattr(y_host, "data_ptr") else y_host.ctypes.data
+        _check(_lib.temco_run_host_async(self._h, C.c_void_p(xp), C.c_void_p(yp), _stream_handle(stream)),
+               "temco_run_host_async")
 
     def run_profiled(self, x, y, stream=None):
         n = len(self.describe()["steps"])

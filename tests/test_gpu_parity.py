@@ -140,3 +140,22 @@ def test_device_mismatch_and_errors():
     with pytest.raises(TemcoError) as e:
         p.run(0, 0, 0)
     assert e.value.status == 1
+
+
+def test_run_host_async_pipeline_matches_device_run():
+    """temco_run_host_async: consecutive calls alternate staging buffers and
+    overlap the next input copy with the current run; every output equals the
+    device-buffer run of the same input."""
+    from paper_conf_icpp_songljkj0024_b200 import Plan
+    m = W.resnet18_cifar(batch=4, dtype="bf16")
+    xs = [W.make_input(m, start=4 * k, count=4) for k in range(3)]
+    p = Plan(m)
+    refs = [_plan_and_run(m, x=x)[1] for x in xs]
+    s = torch.cuda.Stream()
+    xh = [torch.from_numpy(x).to(torch.bfloat16).pin_memory() for x in xs]
+    yh = [torch.empty(p.output_shape()).pin_memory() for _ in xs]
+    for k in range(3):
+        p.run_host_async(xh[k], yh[k], s)
+    s.synchronize()
+    for k in range(3):
+        assert np.array_equal(yh[k].numpy(), refs[k])
