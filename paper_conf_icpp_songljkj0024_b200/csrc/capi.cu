@@ -352,7 +352,8 @@ void lower(temco_plan_s* P) {
           c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = v.groups;
           c.b = v.b ? push_params(P, v.b) : -1;
           // 3x3 cores on 8 channels: the direct SIMT kernel measured faster (kernels_simt.cu)
-          if (c.C <= 64 && c.K <= 64 && !(c.C == 8 && c.K == 8 && c.kh * c.kw > 1)) {
+          // (wider outputs stay on the tcgen05 implicit GEMM: measured faster for K > 64)
+          if (c.C <= 256 && c.K <= 64 && !(c.C == 8 && c.K == 8 && c.kh * c.kw > 1)) {
             const std::vector<float> w = repack_conv(v, x.C);
             if (conv_rank_mma_lower(c, w.data(), P->tcw_h, e.rk)) {
               e.kind = K_CONV_RK;

@@ -48,7 +48,7 @@ __device__ __forceinline__ uint32_t pk2(float a, float b) {
 }
 
 struct RkCursor {
-  int blk, tap;
+  int blk, tap, kc, nc;          // block, tap, 64-channel input chunk, 64-channel output chunk
   int hi0[2], wi0[2], nrow[2];   // per fragment row: window origin, n * H
   bool ok[2];                    // output row exists
 };
@@ -105,7 +105,7 @@ __device__ __forceinline__ void rk_load(uint32_t (&a)[KS][4], const RankConvDesc
   }
 #pragma unroll
   for (int ks = 0; ks < KS; ++ks) {
-    const int k0 = ks * 16 + 2 * t4, k1 = k0 + 8;
+    const int k0 = u.kc * 64 + ks * 16 + 2 * t4, k1 = k0 + 8;
     a[ks][0] = (v[0] && k0 < d.C) ? __ldg(x + p[0] + k0 / 2) : 0u;
     a[ks][1] = (v[1] && k0 < d.C) ? __ldg(x + p[1] + k0 / 2) : 0u;
     a[ks][2] = (v[0] && k1 < d.C) ? __ldg(x + p[0] + k1 / 2) : 0u;
@@ -113,7 +113,7 @@ __device__ __forceinline__ void rk_load(uint32_t (&a)[KS][4], const RankConvDesc
   }
 }
 
-template <int KS, int NT>
+template <int KS, int NT, bool KCH>   // KCH: Cin > 64, walk 64-channel input chunks
 __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const __grid_constant__ RankConvDesc d,
                                                                          RunPtrs p, const uint16_t* __restrict__ tcw) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -135,12 +135,14 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
   const uint32_t wbase4 = s_u32(wb + ((lq >> 1) * 8 + lr) * ws + (lq & 1) * 8);
   const uint32_t wbase2 = s_u32(wb + lr * ws + (lq & 1) * 8);
   const int nw = gridDim.x * kRkWarps;
+  // unit order per block: output chunk, tap, input chunk
   auto advance = [&](RkCursor& u) {
-    if (++u.tap == taps) {
-      u.tap = 0;
-      u.blk += nw;
-      if (u.blk < d.nblocks) rk_set_block(d, u, g);
-    }
+    if (KCH && ++u.kc < d.nkc) return;
+    u.kc = 0;
+    if (++u.tap < taps) return;
+    u.tap = 0;
+    u.blk += nw;
+    if (u.blk < d.nblocks) rk_set_block(d, u, g);
   };
   RkCursor cur{};
   cur.blk = blockIdx.x * kRkWarps + warp;
@@ -155,11 +157,12 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
   for (; cur.blk < d.nblocks; advance(cur)) {
     if (pf.blk < d.nblocks) rk_load<KS>(ann, d, x, pf, t4);
     advance(pf);
-    if (cur.tap == 0) {
+    constexpr int ntc = NT;                            // K <= 64: one output chunk
+    if (cur.tap == 0 && cur.kc == 0) {
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt) {
         float b0 = 0.f, b1 = 0.f;
-        if (d.b >= 0) {
+        if (d.b >= 0 && nt < ntc) {
           b0 = p.params[d.b + nt * 8 + 2 * t4];
           b1 = p.params[d.b + nt * 8 + 2 * t4 + 1];
         }
@@ -167,23 +170,30 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
         acc[nt][1] = acc[nt][3] = b1;
       }
     }
-    const uint32_t tw = (uint32_t)(cur.tap * d.K * ws * 2);
+    const uint32_t tw = (uint32_t)((cur.tap * d.K * ws + (KCH ? cur.kc * 64 : 0)) * 2);
 #pragma unroll
     for (int ks = 0; ks < KS; ++ks) {
+      if (KCH && cur.kc * 64 + ks * 16 >= d.C) break;      // the last input chunk may be short
 #pragma unroll
       for (int np = 0; np < NT / 2; ++np) {
-        uint32_t b0, b1, b2, b3;
-        ldsm_x4(wbase4 + tw + (uint32_t)((np * 16 * ws + ks * 16) * 2), b0, b1, b2, b3);
-        mma16816(acc[2 * np], a[ks], b0, b1);
-        mma16816(acc[2 * np + 1], a[ks], b2, b3);
+        if (2 * np + 1 < ntc) {
+          uint32_t b0, b1, b2, b3;
+          ldsm_x4(wbase4 + tw + (uint32_t)((np * 16 * ws + ks * 16) * 2), b0, b1, b2, b3);
+          mma16816(acc[2 * np], a[ks], b0, b1);
+          mma16816(acc[2 * np + 1], a[ks], b2, b3);
+        } else if (2 * np < ntc) {
+          uint32_t b0, b1;
+          ldsm_x2(wbase2 + tw + (uint32_t)((2 * np * 8 * ws + ks * 16) * 2), b0, b1);
+          mma16816(acc[2 * np], a[ks], b0, b1);
+        }
       }
-      if (NT & 1) {
+      if ((NT & 1) && NT - 1 < ntc) {
         uint32_t b0, b1;
         ldsm_x2(wbase2 + tw + (uint32_t)(((NT - 1) * 8 * ws + ks * 16) * 2), b0, b1);
         mma16816(acc[NT - 1], a[ks], b0, b1);
       }
     }
-    if (cur.tap == taps - 1) {
+    if (cur.tap == taps - 1 && (!KCH || cur.kc == d.nkc - 1)) {
       const int m0 = cur.blk * 16 + g, m1 = m0 + 8;
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt) {
@@ -202,19 +212,19 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
   }
 }
 
-template <int KS, int NT>
+template <int KS, int NT, bool KCH>
 void launch_rk_t(const RankConvDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   static bool configured = false;
   static int sms = 148;
   if (!configured) {
-    cudaFuncSetAttribute(conv_rank_mma_kernel<KS, NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(conv_rank_mma_kernel<KS, NT, KCH>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
   const int grid = std::min((d.nblocks + kRkWarps - 1) / kRkWarps, sms);
-  conv_rank_mma_kernel<KS, NT><<<grid, 32 * kRkWarps, d.blob_bytes, s>>>(d, p, tcw);
+  conv_rank_mma_kernel<KS, NT, KCH><<<grid, 32 * kRkWarps, d.blob_bytes, s>>>(d, p, tcw);
 }
 
 uint16_t f2bf(float f) {
@@ -228,8 +238,10 @@ uint16_t f2bf(float f) {
 
 bool conv_rank_mma_lower(const ConvDesc& c, const float* w_khkwc, std::vector<uint16_t>& tcw, RankConvDesc& d) {
   if (c.groups != 1 || c.x.dtype != DT_BF16 || c.y.dtype != DT_BF16 || c.C % 8 || c.K % 8) return false;
-  const int KS = (c.C + 15) / 16, NT = c.K / 8;
-  if (KS > 4 || NT > 8 || (int64_t)c.N * c.Ho * c.Wo >= (1LL << 31) - 16) return false;
+  // up to 64 input / output channels per unit; wider convs walk 64-channel chunks
+  const int nkc = (c.C + 63) / 64, nnc = (c.K + 63) / 64;
+  const int KS = nkc > 1 ? 4 : (c.C + 15) / 16, NT = c.K / 8;
+  if (nkc * 64 > 256 || nnc > 1 || (int64_t)c.N * c.Ho * c.Wo >= (1LL << 31) - 16) return false;
   d = RankConvDesc();
   d.x = c.x;
   d.y = c.y;
@@ -241,11 +253,13 @@ bool conv_rank_mma_lower(const ConvDesc& c, const float* w_khkwc, std::vector<ui
   d.nblocks = (d.npix + 15) / 16;
   d.KS = KS;
   d.NT = NT;
+  d.nkc = nkc;
+  d.nnc = nnc;
   // weights [tap][K][KS*16 + 8] bf16 (row stride an odd number of 16-byte chunks:
   // conflict-free ldmatrix), zero K padding
-  d.wstride = KS * 16 + 8;
+  d.wstride = (nkc > 1 ? nkc * 64 : KS * 16) + 8;
   const int taps = c.kh * c.kw;
-  d.pair = (c.C == 8 && taps > 1) ? 1 : 0;
+  d.pair = (c.C == 8 && taps > 1 && nkc == 1) ? 1 : 0;
   const int units = d.pair ? (taps + 1) / 2 : taps;
   std::vector<uint16_t> blob((size_t)units * c.K * d.wstride, 0);
   for (int t = 0; t < taps; ++t) {
@@ -267,7 +281,8 @@ bool conv_rank_mma_lower(const ConvDesc& c, const float* w_khkwc, std::vector<ui
 
 void launch_conv_rank_mma(const RankConvDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
 #define TEMCO_RK_CASE(ks, nt) \
-  if (d.KS == ks && d.NT == nt) return launch_rk_t<ks, nt>(d, tcw, p, s);
+  if (d.nkc == 1 && d.KS == ks && d.NT == nt) return launch_rk_t<ks, nt, false>(d, tcw, p, s); \
+  if (d.nkc > 1 && ks == 4 && d.NT == nt) return launch_rk_t<4, nt, true>(d, tcw, p, s);
 #define TEMCO_RK_ROW(ks) \
   TEMCO_RK_CASE(ks, 1) TEMCO_RK_CASE(ks, 2) TEMCO_RK_CASE(ks, 3) TEMCO_RK_CASE(ks, 4) \
   TEMCO_RK_CASE(ks, 5) TEMCO_RK_CASE(ks, 6) TEMCO_RK_CASE(ks, 7) TEMCO_RK_CASE(ks, 8)
