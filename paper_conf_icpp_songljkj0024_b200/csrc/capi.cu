@@ -274,22 +274,28 @@ void lower(temco_plan_s* P) {
     for (int x : s.in) e.io_bytes += tensor_bytes(P, x);
     if (v.op != OP_INPUT) e.io_bytes += tensor_bytes(P, s.out);
     if (s.group) {
-      // small restored widths: register-resident mma.sync kernel; larger ones:
-      // the tcgen05 chain kernel (bf16 plans); anything else: the interpreter
-      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
+      // groups with a 3x3/s2 max-pooled 64-channel member (the stem restore copies):
+      // restore-once mma.sync kernel; single-input groups: the lean mma.sync kernels;
+      // opt-in (TEMCO_FLAG_MMA_CAT, measured slower than tcgen05): the generic mma.sync
+      // concat kernel; else tcgen05, else the interpreter
+      const bool mma_ok = P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY);
+      if (mma_ok) {
+        std::vector<uint16_t> scratch;
+        CatDesc cd;
+        if (mma_cat_lower(ir, s, P->loc, scratch, cd) &&
+            ((mma_poolcat_ok(cd) && !getenv("TEMCO_NO_POOLCAT")) || (P->flags & TEMCO_FLAG_MMA_CAT)) &&
+            mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+          e.kind = K_GROUP_CAT;
+          e.kernel = mma_poolcat_ok(e.cat) ? "mma_poolcat" : "mma_cat";
+          e.launches = 1;
+          continue;
+        }
+      }
+      if (mma_ok && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
           mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma) &&
           ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
         e.kind = K_GROUP_MMA;
         e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
-        e.launches = 1;
-        continue;
-      }
-      // single-level concats (DenseNet's layer groups, incl. pooled / avg-pooled members) on
-      // mma.sync: opt-in, measured 1.4-2.5x slower than the tcgen05 chain kernel on B200
-      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && (P->flags & TEMCO_FLAG_MMA_CAT) &&
-          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
-        e.kind = K_GROUP_CAT;
-        e.kernel = "mma_cat";
         e.launches = 1;
         continue;
       }

@@ -19,6 +19,8 @@
 #include <cuda_bf16.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cmath>
 #include <set>
 
@@ -46,7 +48,8 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
   const int tsrc = ir.oin[s.out][0];
   const Node& tn = ir.nodes[tsrc];
   const int C = tn.C, Nout = root.C;
-  if (Nout % 8 || Nout > 64 || C % 64 || C > 64 * kCatMaxChunks) return false;
+  if (Nout % 8 || Nout > 64 || C % 8 || C > 64 * kCatMaxChunks) return false;
+  const int Cpad = (C + 63) / 64 * 64;   // a short last chunk: zero weights / bias / F columns
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
   P.members.erase(s.out);
   std::vector<PLevel> levels;
@@ -59,7 +62,7 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
 
   d = CatDesc();
   d.C = C;
-  d.nchunks = C / 64;
+  d.nchunks = Cpad / 64;
   d.Nout = Nout;
   d.NO = Nout / 8;
   d.H = tn.H;
@@ -122,7 +125,7 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
   // F [Nout][C + 8]
   while (blob.size() % 8) blob.push_back(0);
   d.f = (int32_t)blob.size();
-  d.fs = C + 8;
+  d.fs = Cpad + 8;
   blob.resize(blob.size() + (size_t)Nout * d.fs, 0);
   for (int o = 0; o < Nout; ++o)
     for (int c = 0; c < C; ++c) blob[d.f + (size_t)o * d.fs + c] = f2bf((*root.w)[(size_t)o * C + c]);
@@ -130,11 +133,11 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
   d.blob_bf16 = (int32_t)blob.size();
   // fp32: level bias [C] (pooled channels: the post-pool shift), member bias [C] (0 elsewhere)
   d.lbias = 0;
-  d.mbias = C;
-  fbias.assign(2 * C, 0.f);
+  d.mbias = Cpad;
+  fbias.assign(2 * Cpad, 0.f);
   for (int c = 0; c < C; ++c) fbias[c] = (float)L.bias[c];
   if (pm) {
-    for (int c = 0; c < pm->C; ++c) fbias[C + pm->c0 + c] = (float)pm->bias[c];
+    for (int c = 0; c < pm->C; ++c) fbias[Cpad + pm->c0 + c] = (float)pm->bias[c];
     d.pool = pm->kind;
     d.pk = pm->k;
     d.ps = pm->s;
@@ -483,6 +486,245 @@ void launch_cat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaS
   mma_cat_kernel<NO, KSM, POOL><<<grid, 32 * kCatWarps, d.blob_bytes, s>>>(d, p, tcw);
 }
 
+// ---------------------------------------------------------------------------
+// Pooled-concat groups whose pooled member is a 3x3 / stride-2 max pool over a
+// rank <= 16 restore of 64 channels (the stem restore copies: ResNet-50's
+// stem -> maxpool -> layer1 groups, DenseNet-121's block-1 layer groups).
+// Restore-once: a CTA owns an 8 x 16 output tile; phase 1 restores every pixel
+// of its (2*8+1) x (2*16+1) input footprint once (act(Lhat r + b), bf16, -inf
+// outside the image) into SMEM -- 2.25 restores per output instead of the 9 of
+// a per-tap evaluation; phase 2 max-pools each output's 3 x 3 window straight
+// into the bf16x2 A fragments of the reduce GEMM, adds the post-pool shift and
+// the level ReLU, then the plain concat terms (other 64-channel chunks) are
+// restored from global memory per output block as in the generic kernel.
+// ---------------------------------------------------------------------------
+constexpr int kPcTH = 8, kPcTW = 16, kPcWarps = 8, kPcStride = 34;   // words per footprint pixel (64 bf16 ch + pad: conflict-free pooling reads)
+
+template <int NO>
+__global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __grid_constant__ CatDesc d, RunPtrs p,
+                                                                    const uint16_t* __restrict__ tcw, int tiles_w,
+                                                                    int tiles_h) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int g = lane / 4, t4 = lane % 4;
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(tcw + d.blob);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  __syncthreads();
+  const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
+  const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
+  uint32_t* fp = reinterpret_cast<uint32_t*>(smem + (d.blob_bytes + 15) / 16 * 16);   // footprint [PR*PC][kPcStride]
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+  const int lq = lane >> 3, lr = lane & 7;
+  const uint32_t sbase = s_u32(blob);
+  const CatTerm& M = d.term[d.n_plain];                 // the pooled member's (single) term
+  const int PR = (kPcTH - 1) * 2 + 3, PC = (kPcTW - 1) * 2 + 3;
+  // member restore fragments and bias (registers for the whole kernel)
+  uint32_t wm[8][2];
+  float mb[8][2];
+#pragma unroll
+  for (int np = 0; np < 4; ++np)
+    ldsm_x4(sbase + (uint32_t)((M.w + (np * 16 + (lq >> 1) * 8 + lr) * M.rs + (lq & 1) * 8) * 2), wm[2 * np][0],
+            wm[2 * np][1], wm[2 * np + 1][0], wm[2 * np + 1][1]);
+#pragma unroll
+  for (int nt = 0; nt < 8; ++nt) {
+    const float2 b = *reinterpret_cast<const float2*>(fb + d.mbias + nt * 8 + 2 * t4);
+    mb[nt][0] = b.x;
+    mb[nt][1] = b.y;
+  }
+  const uint32_t* rm = reinterpret_cast<const uint32_t*>(p.arena + M.r.off);
+  const int ntiles = d.npix / (d.H * d.W) * tiles_w * tiles_h;
+  for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int n = tile / (tiles_w * tiles_h);
+    const int oh0 = (tile / tiles_w) % tiles_h * kPcTH, ow0 = tile % tiles_w * kPcTW;
+    const int ih0 = oh0 * 2 - 1, iw0 = ow0 * 2 - 1;
+    // ---- phase 1: restore the footprint once; all of the warp's loads first (in flight together)
+    constexpr int kMaxB = 5;   // footprint blocks per warp: ceil(17 * 33 / 16 / 8)
+    uint32_t a[kMaxB][4];
+    bool v[kMaxB][2];
+#pragma unroll
+    for (int q = 0; q < kMaxB; ++q) {
+      const int fb16 = warp + q * kPcWarps;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int px = fb16 * 16 + g + 8 * h;
+        const int fr = px / PC, fc = px - fr * PC;
+        const int ih = ih0 + fr, iw = iw0 + fc;
+        v[q][h] = px < PR * PC && ih >= 0 && ih < M.Hin && iw >= 0 && iw < M.Win;
+        const int64_t off = ((int64_t)(n * M.Hin + ih) * M.Win + iw) * (M.R / 2);
+        a[q][h] = (v[q][h] && 2 * t4 < M.R) ? __ldg(rm + off + t4) : 0u;
+        a[q][2 + h] = (v[q][h] && 2 * t4 + 8 < M.R) ? __ldg(rm + off + t4 + 4) : 0u;
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < kMaxB; ++q) {
+      const int fb16 = warp + q * kPcWarps;
+      if (fb16 * 16 >= PR * PC) break;
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt) {
+        float D[4] = {mb[nt][0], mb[nt][1], mb[nt][0], mb[nt][1]};
+        mma16816(D, a[q], wm[nt][0], wm[nt][1]);
+        if (d.mrelu) {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) D[i] = fmaxf(D[i], 0.f);
+        }
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int px = fb16 * 16 + g + 8 * h;
+          if (px < PR * PC)
+            fp[px * kPcStride + nt * 4 + t4] = v[q][h] ? pk2(D[2 * h], D[2 * h + 1]) : 0xFF80FF80u;   // -inf pair
+        }
+      }
+    }
+    __syncthreads();
+    // ---- phase 2: one 16-pixel output row per warp
+    if (warp < kPcTH) {
+      const int oh = oh0 + warp;
+      float O[NO][4];
+#pragma unroll
+      for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
+      CatRows rw;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        rw.n[h] = n;
+        rw.ho[h] = oh;
+        rw.wo[h] = ow0 + g + 8 * h;
+        rw.ok[h] = oh < d.H && rw.wo[h] < d.W;
+      }
+      // chunk 0: the pooled member -> P fragments (bf16x2 max over the 3 x 3 window)
+#pragma unroll
+      for (int ks = 0; ks < 4; ++ks) {
+        uint32_t pa[4];
+#pragma unroll
+        for (int r4 = 0; r4 < 4; ++r4) {
+          const int h = r4 & 1, chw = ks * 8 + t4 + (r4 >> 1) * 4;   // word of channels 16ks + 2t4 (+8)
+          const int fc0 = 2 * (g + 8 * h), fr0 = 2 * warp;
+          __nv_bfloat162 m = __halves2bfloat162(__float2bfloat16_rn(-INFINITY), __float2bfloat16_rn(-INFINITY));
+#pragma unroll
+          for (int ty = 0; ty < 3; ++ty)
+#pragma unroll
+            for (int tx = 0; tx < 3; ++tx) {
+              const uint32_t w = fp[((fr0 + ty) * PC + fc0 + tx) * kPcStride + chw];
+              m = __hmax2(m, *reinterpret_cast<const __nv_bfloat162*>(&w));
+            }
+          // + post-pool shift (the level bias of these channels), level ReLU
+          const int ch = ks * 16 + (r4 >> 1) * 8 + 2 * t4;
+          float lo = __low2float(m) + fb[d.lbias + ch], hi = __high2float(m) + fb[d.lbias + ch + 1];
+          if (d.relu) lo = fmaxf(lo, 0.f), hi = fmaxf(hi, 0.f);
+          pa[r4 == 0 ? 0 : r4 == 1 ? 1 : r4 == 2 ? 2 : 3] = pk2(lo, hi);
+        }
+#pragma unroll
+        for (int nb = 0; nb < NO; ++nb) {
+          if (nb >= d.NO) break;
+          uint32_t f0, f1;
+          ldsm_x2(sbase + (uint32_t)((d.f + (nb * 8 + lr) * d.fs + ks * 16 + (lq & 1) * 8) * 2), f0, f1);
+          mma16816(O[nb], pa, f0, f1);
+        }
+      }
+      // other chunks: plain concat terms, restored per output block
+      for (int ch = 1; ch < d.nchunks; ++ch) {
+        float D[8][4];
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt) {
+          const float2 b = *reinterpret_cast<const float2*>(fb + d.lbias + ch * 64 + nt * 8 + 2 * t4);
+          D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+        }
+        for (int ui = 0; ui < d.n_units; ++ui) {
+          const CatUnit u = d.unit[ui];
+          if (u.chunk != ch || u.term < 0) continue;
+          uint32_t a[1][4];
+          bool va[2];
+          cat_load<1>(a, va, d, p, u, rw, t4);
+          const int rs = d.term[u.term].rs;
+          const uint32_t wb = sbase + (uint32_t)((u.woff + ((lq >> 1) * 8 + lr) * rs + (lq & 1) * 8) * 2);
+          const uint32_t wb2 = sbase + (uint32_t)((u.woff + lr * rs + (lq & 1) * 8) * 2);
+#pragma unroll
+          for (int nt = 0; nt < 8; nt += 2) {
+            if (nt >= u.nt0 && nt < u.nt1) {
+              const uint32_t roff = (uint32_t)(((nt - u.nt0) * 8 * rs) * 2);
+              if (nt + 1 < u.nt1) {
+                uint32_t b0, b1, b2, b3;
+                ldsm_x4(wb + roff, b0, b1, b2, b3);
+                mma16816(D[nt], a[0], b0, b1);
+                mma16816(D[nt + 1], a[0], b2, b3);
+              } else {
+                uint32_t b0, b1;
+                ldsm_x2(wb2 + roff, b0, b1);
+                mma16816(D[nt], a[0], b0, b1);
+              }
+            } else if (nt + 1 >= u.nt0 && nt + 1 < u.nt1) {
+              uint32_t b0, b1;
+              ldsm_x2(wb2 + (uint32_t)(((nt + 1 - u.nt0) * 8 * rs) * 2), b0, b1);
+              mma16816(D[nt + 1], a[0], b0, b1);
+            }
+          }
+        }
+        if (d.relu) {
+#pragma unroll
+          for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+            for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+        }
+#pragma unroll
+        for (int kp = 0; kp < 2; ++kp) {
+          uint32_t pa[2][4];
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int ks = 2 * kp + h;
+            pa[h][0] = pk2(D[2 * ks][0], D[2 * ks][1]);
+            pa[h][1] = pk2(D[2 * ks][2], D[2 * ks][3]);
+            pa[h][2] = pk2(D[2 * ks + 1][0], D[2 * ks + 1][1]);
+            pa[h][3] = pk2(D[2 * ks + 1][2], D[2 * ks + 1][3]);
+          }
+#pragma unroll
+          for (int nb = 0; nb < NO; ++nb) {
+            if (nb >= d.NO) break;
+            uint32_t f0, f1, f2, f3;
+            ldsm_x4(sbase + (uint32_t)((d.f + (nb * 8 + lr) * d.fs + ch * 64 + kp * 32 + lq * 8) * 2), f0, f1, f2,
+                    f3);
+            mma16816(O[nb], pa[0], f0, f1);
+            mma16816(O[nb], pa[1], f2, f3);
+          }
+        }
+      }
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        if (!rw.ok[h]) continue;
+        const int64_t m = ((int64_t)n * d.H + oh) * d.W + rw.wo[h];
+#pragma unroll
+        for (int nb = 0; nb < NO; ++nb) {
+          if (nb >= d.NO) break;
+          *reinterpret_cast<uint32_t*>(y + m * d.Nout + nb * 8 + 2 * t4) = pk2(O[nb][2 * h], O[nb][2 * h + 1]);
+        }
+      }
+    }
+    __syncthreads();   // the footprint buffer is rewritten by the next tile
+  }
+}
+
+template <int NO>
+void launch_poolcat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  const int PR = (kPcTH - 1) * 2 + 3, PC = (kPcTW - 1) * 2 + 3;
+  const int smem = (d.blob_bytes + 15) / 16 * 16 + PR * PC * kPcStride * 4;
+  if (!configured) {
+    cudaFuncSetAttribute(mma_poolcat_kernel<NO>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mma_poolcat_kernel<NO>, 32 * kPcWarps, smem);
+  const int tw = (d.W + kPcTW - 1) / kPcTW, th = (d.H + kPcTH - 1) / kPcTH;
+  const int ntiles = d.npix / (d.H * d.W) * tw * th;
+  const int grid = std::min(ntiles, sms * std::max(per_sm, 1));
+  mma_poolcat_kernel<NO><<<grid, 32 * kPcWarps, smem, s>>>(d, p, tcw, tw, th);
+}
+
 template <int KSM, bool POOL>
 void launch_cat_no(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   switch ((d.NO + 1) / 2) {
@@ -495,7 +737,25 @@ void launch_cat_no(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cuda
 
 }  // namespace
 
+bool mma_poolcat_ok(const CatDesc& d) {
+  if (getenv("TEMCO_DEBUG_CAT"))
+    fprintf(stderr, "poolcat? pool %d k %d s %d p %d pc %d-%d NO %d terms %d/%d R %d blob %d\n", d.pool, d.pk, d.ps,
+            d.pp, d.pc0, d.pc1, d.NO, d.n_plain, d.n_terms, d.n_terms > d.n_plain ? d.term[d.n_plain].R : -1,
+            d.blob_bytes);
+  if (d.pool != 1 || d.pk != 3 || d.ps != 2 || d.pp != 1 || d.pc0 != 0 || d.pc1 != 1 || d.NO > 4) return false;
+  if (d.n_terms != d.n_plain + 1 || d.term[d.n_plain].R > 16) return false;
+  for (int j = 0; j < d.n_plain; ++j)
+    if (d.term[j].tk != 1 || d.term[j].R > 16) return false;
+  const int PR = (kPcTH - 1) * 2 + 3, PC = (kPcTW - 1) * 2 + 3;
+  return (d.blob_bytes + 15) / 16 * 16 + PR * PC * kPcStride * 4 <= 227 * 1024;
+}
+
 void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  if (mma_poolcat_ok(d)) {
+    if (d.NO == 1) return launch_poolcat_t<1>(d, tcw, p, s);
+    if (d.NO == 2) return launch_poolcat_t<2>(d, tcw, p, s);
+    return launch_poolcat_t<4>(d, tcw, p, s);   // 3 or 4 n-tiles (bounded by d.NO inside)
+  }
   int ksm = 1;
   for (int j = 0; j < d.n_terms; ++j) ksm = std::max(ksm, d.term[j].ks);
   const bool pool = d.pool != 0;
