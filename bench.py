@@ -265,7 +265,7 @@ def main():
     total_ms = float(prof.sum())
     # every class against its own bound, and the fused-group family (SURVEY 8(a)
     # row a6: tc_chain + mma_lean + mma_chain) as a time-weighted roofline
-    # fraction over its launches: sum_i max(F_i / P_tc, B_i / P_hbm) / sum_i t_i
+    # fraction over its launches (+ mma_poolcat / mma_cat): sum_i max(F_i / P_tc, B_i / P_hbm) / sum_i t_i
     by_class = {}
     for k, v in classes.items():
         a_i = v["flops"] / max(v["bytes"], 1)
@@ -276,10 +276,10 @@ def main():
                        "ms": round(v["ms"], 4)}
     ideal = actual = 0.0
     for s, t in zip(steps, prof):
-        if s["kernel"] in ("tc_chain", "mma_lean", "mma_chain") and t > 0:
+        if s["kernel"] in ("tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat") and t > 0:
             ideal += max(s.get("alg_flops", s["flops"]) / (tf_sust * 1e12), s.get("alg_bytes", s["io_bytes"]) / (hbm * 1e9))
             actual += float(t) * 1e-3
-    fused = {"kernels": ["tc_chain", "mma_lean", "mma_chain"], "roofline_ms": round(ideal * 1e3, 4),
+    fused = {"kernels": ["tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat"], "roofline_ms": round(ideal * 1e3, 4),
              "measured_ms": round(actual * 1e3, 4), "frac": round(ideal / actual, 4) if actual else None,
              "note": "per launch max(alg FLOP / sustained bf16 peak, alg bytes / HBM peak), summed, / measured"}
     # DRAM traffic of the dominant class from the committed ncu capture of this
