@@ -500,7 +500,7 @@ void launch_cat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaS
 // ---------------------------------------------------------------------------
 constexpr int kPcTH = 8, kPcTW = 16, kPcWarps = 8, kPcStride = 34;   // words per footprint pixel (64 bf16 ch + pad: conflict-free pooling reads)
 
-template <int NO>
+template <int NO, int PK, int PS, int PP>   // pool window / stride / pad: (3, 2, 1) or (2, 2, 0)
 __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __grid_constant__ CatDesc d, RunPtrs p,
                                                                     const uint16_t* __restrict__ tcw, int tiles_w,
                                                                     int tiles_h) {
@@ -520,7 +520,7 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
   const int lq = lane >> 3, lr = lane & 7;
   const uint32_t sbase = s_u32(blob);
   const CatTerm& M = d.term[d.n_plain];                 // the pooled member's (single) term
-  const int PR = (kPcTH - 1) * 2 + 3, PC = (kPcTW - 1) * 2 + 3;
+  const int PR = (kPcTH - 1) * PS + PK, PC = (kPcTW - 1) * PS + PK;
   // member restore fragments and bias (registers for the whole kernel)
   uint32_t wm[8][2];
   float mb[8][2];
@@ -539,7 +539,7 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
   for (int tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
     const int n = tile / (tiles_w * tiles_h);
     const int oh0 = (tile / tiles_w) % tiles_h * kPcTH, ow0 = tile % tiles_w * kPcTW;
-    const int ih0 = oh0 * 2 - 1, iw0 = ow0 * 2 - 1;
+    const int ih0 = oh0 * PS - PP, iw0 = ow0 * PS - PP;
     // ---- phase 1: restore the footprint once; all of the warp's loads first (in flight together)
     constexpr int kMaxB = 5;   // footprint blocks per warp: ceil(17 * 33 / 16 / 8)
     uint32_t a[kMaxB][4];
@@ -600,12 +600,12 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
 #pragma unroll
         for (int r4 = 0; r4 < 4; ++r4) {
           const int h = r4 & 1, chw = ks * 8 + t4 + (r4 >> 1) * 4;   // word of channels 16ks + 2t4 (+8)
-          const int fc0 = 2 * (g + 8 * h), fr0 = 2 * warp;
+          const int fc0 = PS * (g + 8 * h), fr0 = PS * warp;
           __nv_bfloat162 m = __halves2bfloat162(__float2bfloat16_rn(-INFINITY), __float2bfloat16_rn(-INFINITY));
 #pragma unroll
-          for (int ty = 0; ty < 3; ++ty)
+          for (int ty = 0; ty < PK; ++ty)
 #pragma unroll
-            for (int tx = 0; tx < 3; ++tx) {
+            for (int tx = 0; tx < PK; ++tx) {
               const uint32_t w = fp[((fr0 + ty) * PC + fc0 + tx) * kPcStride + chw];
               m = __hmax2(m, *reinterpret_cast<const __nv_bfloat162*>(&w));
             }
@@ -704,25 +704,25 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
   }
 }
 
-template <int NO>
+template <int NO, int PK, int PS, int PP>
 void launch_poolcat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   static bool configured = false;
   static int sms = 148;
-  const int PR = (kPcTH - 1) * 2 + 3, PC = (kPcTW - 1) * 2 + 3;
+  const int PR = (kPcTH - 1) * PS + PK, PC = (kPcTW - 1) * PS + PK;
   const int smem = (d.blob_bytes + 15) / 16 * 16 + PR * PC * kPcStride * 4;
   if (!configured) {
-    cudaFuncSetAttribute(mma_poolcat_kernel<NO>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(mma_poolcat_kernel<NO, PK, PS, PP>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
   int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mma_poolcat_kernel<NO>, 32 * kPcWarps, smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, mma_poolcat_kernel<NO, PK, PS, PP>, 32 * kPcWarps, smem);
   const int tw = (d.W + kPcTW - 1) / kPcTW, th = (d.H + kPcTH - 1) / kPcTH;
   const int ntiles = d.npix / (d.H * d.W) * tw * th;
   const int grid = std::min(ntiles, sms * std::max(per_sm, 1));
-  mma_poolcat_kernel<NO><<<grid, 32 * kPcWarps, smem, s>>>(d, p, tcw, tw, th);
+  mma_poolcat_kernel<NO, PK, PS, PP><<<grid, 32 * kPcWarps, smem, s>>>(d, p, tcw, tw, th);
 }
 
 template <int KSM, bool POOL>
@@ -742,19 +742,25 @@ bool mma_poolcat_ok(const CatDesc& d) {
     fprintf(stderr, "poolcat? pool %d k %d s %d p %d pc %d-%d NO %d terms %d/%d R %d blob %d\n", d.pool, d.pk, d.ps,
             d.pp, d.pc0, d.pc1, d.NO, d.n_plain, d.n_terms, d.n_terms > d.n_plain ? d.term[d.n_plain].R : -1,
             d.blob_bytes);
-  if (d.pool != 1 || d.pk != 3 || d.ps != 2 || d.pp != 1 || d.pc0 != 0 || d.pc1 != 1 || d.NO > 4) return false;
+  const bool win = (d.pk == 3 && d.ps == 2 && d.pp == 1) || (d.pk == 2 && d.ps == 2 && d.pp == 0);
+  if (d.pool != 1 || !win || d.pc0 != 0 || d.pc1 != 1 || d.NO > 4) return false;
   if (d.n_terms != d.n_plain + 1 || d.term[d.n_plain].R > 16) return false;
   for (int j = 0; j < d.n_plain; ++j)
     if (d.term[j].tk != 1 || d.term[j].R > 16) return false;
-  const int PR = (kPcTH - 1) * 2 + 3, PC = (kPcTW - 1) * 2 + 3;
+  const int PR = (kPcTH - 1) * d.ps + d.pk, PC = (kPcTW - 1) * d.ps + d.pk;
   return (d.blob_bytes + 15) / 16 * 16 + PR * PC * kPcStride * 4 <= 227 * 1024;
 }
 
 void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   if (mma_poolcat_ok(d)) {
-    if (d.NO == 1) return launch_poolcat_t<1>(d, tcw, p, s);
-    if (d.NO == 2) return launch_poolcat_t<2>(d, tcw, p, s);
-    return launch_poolcat_t<4>(d, tcw, p, s);   // 3 or 4 n-tiles (bounded by d.NO inside)
+    if (d.pk == 2) {   // VGG's 2x2 / stride-2 pools
+      if (d.NO == 1) return launch_poolcat_t<1, 2, 2, 0>(d, tcw, p, s);
+      if (d.NO == 2) return launch_poolcat_t<2, 2, 2, 0>(d, tcw, p, s);
+      return launch_poolcat_t<4, 2, 2, 0>(d, tcw, p, s);
+    }
+    if (d.NO == 1) return launch_poolcat_t<1, 3, 2, 1>(d, tcw, p, s);
+    if (d.NO == 2) return launch_poolcat_t<2, 3, 2, 1>(d, tcw, p, s);
+    return launch_poolcat_t<4, 3, 2, 1>(d, tcw, p, s);   // 3 or 4 n-tiles (bounded by d.NO inside)
   }
   int ksm = 1;
   for (int j = 0; j < d.n_terms; ++j) ksm = std::max(ksm, d.term[j].ks);

@@ -1,5 +1,5 @@
 timeout 600 python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1
-for c in resnet50 densenet121; do
+for c in vgg16_cp; do
 for v in "" "TEMCO_NO_POOLCAT=1"; do
   echo "=== $c $v"; env $v python scripts/step_profile.py $c 400
 done; done > gpurun_out/exp_pc.log 2>&1
