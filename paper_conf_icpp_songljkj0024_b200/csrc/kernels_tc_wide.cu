@@ -1196,7 +1196,8 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
-  const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
+  int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
+  if (getenv("TEMCO_TC_GRID")) grid = std::min(grid, atoi(getenv("TEMCO_TC_GRID")));   // experiments
   // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
   tc_chain_kernel<<<grid, kThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }
