@@ -1,3 +1,5 @@
-for v in "" "TEMCO_TC_GRID=74" "TEMCO_TC_GRID=37"; do
-  echo "=== resnet50 $v"; env $v python scripts/step_profile.py resnet50 400 | grep "tc_chain\|total"
-done > gpurun_out/exp_grid.log 2>&1
+timeout 600 python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1
+for c in resnet50 densenet121; do
+for v in "" "TEMCO_WIDE_NB2=1"; do
+  echo "=== $c $v"; env $v python scripts/step_profile.py $c 400 | grep "tc_chain\|total"
+done; done > gpurun_out/exp_nb.log 2>&1
