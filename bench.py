@@ -223,10 +223,13 @@ def main():
     if ws > 1:
         dist.barrier()
     e0.record(stream)
-    for _ in range(args.steps):
-        plan.run_host_async(xh, yh, stream)
-        if ws > 1:
-            gather_logits(y, ws, gathered)
+    with torch.cuda.stream(stream):
+        for _ in range(args.steps):
+            plan.run_host_async(xh, yh, stream)
+            if ws > 1:
+                # this step's logits (host) back on the device for the NCCL gather, stream-ordered
+                y.copy_(yh, non_blocking=True)
+                gather_logits(y, ws, gathered)
     e1.record(stream)
     torch.cuda.synchronize()
     e2e_ms = e0.elapsed_time(e1) / args.steps
