@@ -573,6 +573,15 @@ void free_device(temco_plan_s* P) {
   if (P->blas) cublasDestroy(P->blas);
 }
 
+}  // namespace
+
+bool temco::pdl_enabled() {
+  static const bool on = getenv("TEMCO_NO_PDL") == nullptr;
+  return on;
+}
+
+namespace {
+
 RunPtrs run_ptrs(temco_plan_s* P, const void* in, void* out) {
   return RunPtrs{P->arena_d, in, out, P->params_d};
 }

@@ -513,6 +513,8 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
     for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   __syncthreads();
+  pdl_wait();
+  pdl_trigger_early();
   const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
   const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
   uint32_t* fp = reinterpret_cast<uint32_t*>(smem + (d.blob_bytes + 15) / 16 * 16);   // footprint [PR*PC][kPcStride]
@@ -722,7 +724,7 @@ void launch_poolcat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, c
   const int tw = (d.W + kPcTW - 1) / kPcTW, th = (d.H + kPcTH - 1) / kPcTH;
   const int ntiles = d.npix / (d.H * d.W) * tw * th;
   const int grid = std::min(ntiles, sms * std::max(per_sm, 1));
-  mma_poolcat_kernel<NO, PK, PS, PP><<<grid, 32 * kPcWarps, smem, s>>>(d, p, tcw, tw, th);
+  launch_pdl(mma_poolcat_kernel<NO, PK, PS, PP>, dim3(grid), dim3(32 * kPcWarps), smem, s, d, p, tcw, tw, th);
 }
 
 template <int KSM, bool POOL>

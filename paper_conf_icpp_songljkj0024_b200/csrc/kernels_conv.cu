@@ -394,6 +394,8 @@ __global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __gr
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+  pdl_wait();
+  pdl_trigger_early();
   const int per_img = d.nhb * d.nwb;
 
   if (warp == 4) {
@@ -497,7 +499,7 @@ void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s) {
   }
   const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);   // persistent, one CTA per SM
   if (d.tma)
-    conv_tma_kernel<<<grid, kConvTmaThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+    launch_pdl(conv_tma_kernel, dim3(grid), dim3(kConvTmaThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
   else
     conv_tc_kernel<<<grid, kConvThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }

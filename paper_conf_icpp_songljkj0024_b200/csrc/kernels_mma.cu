@@ -500,6 +500,8 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
     for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   __syncthreads();
+  pdl_wait();
+  pdl_trigger_early();
   const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
   const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2) + d.bias[0];
   const MmaTerm& T = d.term[0];
@@ -657,6 +659,8 @@ __global__ void __launch_bounds__(32 * kL64Warps, 1) mma_lean64_kernel(const __g
     for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   __syncthreads();
+  pdl_wait();
+  pdl_trigger_early();
   const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
   const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2) + d.bias[0];
   const MmaTerm& T = d.term[0];
@@ -782,7 +786,7 @@ void launch_lean64_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& 
   }
   constexpr int kW = POOL ? 8 : 16;
   const int grid = (int)std::min<int64_t>((d.nblocks + kW - 1) / kW, (int64_t)sms);
-  mma_lean64_kernel<NO, POOL><<<grid, 32 * kW, d.blob_bytes, s>>>(d, p, tcw);
+  launch_pdl(mma_lean64_kernel<NO, POOL>, dim3(grid), dim3(32 * kW), d.blob_bytes, s, d, p, tcw);
 }
 
 template <int KS, int NO>
@@ -797,7 +801,7 @@ void launch_lean_t(const MmaChainDesc& d, const uint16_t* tcw, const RunPtrs& p,
     configured = true;
   }
   const int grid = (int)std::min<int64_t>((d.nblocks + kLeanWarps - 1) / kLeanWarps, (int64_t)sms);
-  mma_lean_kernel<KS, NO><<<grid, 32 * kLeanWarps, d.blob_bytes, s>>>(d, p, tcw);
+  launch_pdl(mma_lean_kernel<KS, NO>, dim3(grid), dim3(32 * kLeanWarps), d.blob_bytes, s, d, p, tcw);
 }
 
 }  // namespace

@@ -125,6 +125,8 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
     for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
   }
   __syncthreads();
+  pdl_wait();
+  pdl_trigger_early();
   const __nv_bfloat16* wb = reinterpret_cast<const __nv_bfloat16*>(smem);
   const uint32_t* x = reinterpret_cast<const uint32_t*>(loc_ptr(d.x, p));
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
@@ -224,7 +226,7 @@ void launch_rk_t(const RankConvDesc& d, const uint16_t* tcw, const RunPtrs& p, c
     configured = true;
   }
   const int grid = std::min((d.nblocks + kRkWarps - 1) / kRkWarps, sms);
-  conv_rank_mma_kernel<KS, NT, KCH><<<grid, 32 * kRkWarps, d.blob_bytes, s>>>(d, p, tcw);
+  launch_pdl(conv_rank_mma_kernel<KS, NT, KCH>, dim3(grid), dim3(32 * kRkWarps), d.blob_bytes, s, d, p, tcw);
 }
 
 uint16_t f2bf(float f) {

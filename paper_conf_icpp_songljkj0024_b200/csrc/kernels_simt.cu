@@ -156,6 +156,8 @@ __host__ __device__ inline RankTile rank_tile(const ConvDesc& d) {
 
 template <int KC>
 __global__ void __launch_bounds__(256) conv_rank_kernel(ConvDesc d, RankTile t, RunPtrs p) {
+  pdl_wait();
+  pdl_trigger_early();
   extern __shared__ __align__(16) unsigned char smr[];
   const int Cin = d.C;
   const int taps = d.kh * d.kw;
@@ -261,6 +263,8 @@ __global__ void __launch_bounds__(256) dwconv_col_kernel(ConvDesc d, RunPtrs p) 
   }
 #pragma unroll
   for (int j = 0; j < 8; ++j) bias[j] = d.b >= 0 ? __ldg(p.params + d.b + g * 8 + j) : 0.f;
+  pdl_wait();
+  pdl_trigger_early();
   for (int st = blockIdx.y; st < d.N * spi; st += gridDim.y) {
     const int n = st / spi, h0 = (st - n * spi) * kColRows;
     uint4 v[kColRows + 2];
@@ -320,6 +324,8 @@ __global__ void __launch_bounds__(256) dwconv_row_kernel(ConvDesc d, RunPtrs p) 
   }
 #pragma unroll
   for (int j = 0; j < 8; ++j) bias[j] = d.b >= 0 ? __ldg(p.params + d.b + g * 8 + j) : 0.f;
+  pdl_wait();
+  pdl_trigger_early();
   constexpr int kRU = 4;   // rows per iteration: their loads in flight together
   const int rows = d.N * d.Ho;
   for (int row0 = blockIdx.y * kRU; row0 < rows; row0 += gridDim.y * kRU) {
@@ -379,6 +385,8 @@ __global__ void __launch_bounds__(256) dwconv_row_kernel(ConvDesc d, RunPtrs p) 
 
 template <int KH, int KW>   // 0, 0: runtime kernel size (<= 9 taps)
 __global__ void __launch_bounds__(256) dwconv_vec_kernel(ConvDesc d, RunPtrs p) {
+  pdl_wait();
+  pdl_trigger_early();
   // grid: x = chunks of (output column, 8-channel group) of one output row, y = output rows (n, ho):
   // 32-bit index math only (the 64-bit div/mod chain dominated the previous flat-index version)
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
@@ -762,16 +770,16 @@ void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   dim3 grid((unsigned)xb, (unsigned)std::min(rows, std::max(1, 148 * 8 / xb)));
   if (d.kh == 3 && d.kw == 1 && d.sh == 1 && d.sw == 1 && d.pw == 0 && d.Ho == d.H + 2 * d.ph - 2) {
     const int strips = d.N * ((d.Ho + kColRows - 1) / kColRows);
-    dwconv_col_kernel<<<dim3((unsigned)xb, (unsigned)std::min(strips, std::max(1, 148 * 8 / xb))), 256, 0, s>>>(d, p);
+    launch_pdl(dwconv_col_kernel, dim3((unsigned)xb, (unsigned)std::min(strips, std::max(1, 148 * 8 / xb))), dim3(256), 0, s, d, p);
   } else if (d.kh == 3 && d.kw == 1)
-    dwconv_vec_kernel<3, 1><<<grid, 256, 0, s>>>(d, p);
+    launch_pdl(dwconv_vec_kernel<3, 1>, grid, dim3(256), 0, s, d, p);
   else if (d.kh == 1 && d.kw == 3 && d.sh == 1 && d.sw == 1 && d.ph == 0 && d.pw == 1 && d.Wo == d.W &&
            d.Ho == d.H && d.C / 8 <= 16) {
-    dwconv_row_kernel<<<dim3((unsigned)xb, (unsigned)std::min((rows + 3) / 4, std::max(1, 148 * 8 / xb))), 256, 0, s>>>(d, p);
+    launch_pdl(dwconv_row_kernel, dim3((unsigned)xb, (unsigned)std::min((rows + 3) / 4, std::max(1, 148 * 8 / xb))), dim3(256), 0, s, d, p);
   } else if (d.kh == 1 && d.kw == 3)
-    dwconv_vec_kernel<1, 3><<<grid, 256, 0, s>>>(d, p);
+    launch_pdl(dwconv_vec_kernel<1, 3>, grid, dim3(256), 0, s, d, p);
   else
-    dwconv_vec_kernel<0, 0><<<grid, 256, 0, s>>>(d, p);
+    launch_pdl(dwconv_vec_kernel<0, 0>, grid, dim3(256), 0, s, d, p);
 }
 
 bool conv_rank_ok(const ConvDesc& d) {
@@ -792,9 +800,9 @@ void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   const RankTile t = rank_tile(d);
   dim3 grid((unsigned)(t.tiles_n * t.tiles_h * t.tiles_w), (unsigned)(d.K / t.kc));
   if (t.kc == 8)
-    conv_rank_kernel<8><<<grid, 256, t.smem, s>>>(d, t, p);
+    launch_pdl(conv_rank_kernel<8>, grid, dim3(256), t.smem, s, d, t, p);
   else
-    conv_rank_kernel<16><<<grid, 256, t.smem, s>>>(d, t, p);
+    launch_pdl(conv_rank_kernel<16>, grid, dim3(256), t.smem, s, d, t, p);
 }
 
 bool conv_small_ok(const ConvDesc& d) {

@@ -151,6 +151,8 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
     }
   };
   int tile = blockIdx.x;
+  pdl_wait();
+  pdl_trigger_early();
   if (tile < ntiles) load(tile);
   int b = 0;
   for (; tile < ntiles; tile += gridDim.x, b ^= 1) {
@@ -214,7 +216,7 @@ void launch_stem_t(const ConvDesc& d, const StemGeo& g, const RunPtrs& p, cudaSt
   const int tw = (d.Wo + kStTW - 1) / kStTW, th = (d.Ho + kStTH - 1) / kStTH;
   const int ntiles = d.N * tw * th;
   const int grid = std::min(ntiles, sms * std::max(per_sm, 1));
-  conv_stem_kernel<KS, NT><<<(unsigned)grid, kStThreads, g.smem, s>>>(d, g, p, tw, th);
+  launch_pdl(conv_stem_kernel<KS, NT>, dim3((unsigned)grid), dim3(kStThreads), g.smem, s, d, g, p, tw, th);
 }
 
 }  // namespace

@@ -741,6 +741,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   __syncthreads();
   tc_fence_after();
   const uint32_t tbase = *tmem_slot;
+  pdl_wait();
+  pdl_trigger_early();
   const int U = d.units;
 #ifdef TEMCO_TRACE
   int tn[kTraceRows] = {0};
@@ -1193,7 +1195,7 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   }
   const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
   // >= 114 KB of shared memory keeps one CTA per SM (each owns all 512 TMEM columns)
-  tc_chain_kernel<<<grid, kThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+  launch_pdl(tc_chain_kernel, dim3(grid), dim3(kThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }
 
 }  // namespace temco
