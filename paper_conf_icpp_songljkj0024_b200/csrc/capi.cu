@@ -279,23 +279,28 @@ void lower(temco_plan_s* P) {
       // opt-in (TEMCO_FLAG_MMA_CAT, measured slower than tcgen05): the generic mma.sync
       // concat kernel; else tcgen05, else the interpreter
       const bool mma_ok = P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY);
-      if (mma_ok) {
-        std::vector<uint16_t> scratch;
-        CatDesc cd;
-        if (mma_cat_lower(ir, s, P->loc, scratch, cd) &&
-            ((mma_poolcat_ok(cd) && !getenv("TEMCO_NO_POOLCAT")) || (P->flags & TEMCO_FLAG_MMA_CAT)) &&
-            mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
-          e.kind = K_GROUP_CAT;
-          e.kernel = mma_poolcat_ok(e.cat) ? "mma_poolcat" : "mma_cat";
-          e.launches = 1;
-          continue;
-        }
+      std::vector<uint16_t> scratch;
+      CatDesc cd;
+      const bool cat_form = mma_ok && mma_cat_lower(ir, s, P->loc, scratch, cd);
+      if (cat_form && mma_poolcat_ok(cd) && !getenv("TEMCO_NO_POOLCAT") &&
+          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+        e.kind = K_GROUP_CAT;
+        e.kernel = "mma_poolcat";
+        e.launches = 1;
+        continue;
       }
       if (mma_ok && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
           mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma) &&
           ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
         e.kind = K_GROUP_MMA;
         e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
+        e.launches = 1;
+        continue;
+      }
+      if (cat_form && ((mma_catp_ok(cd) && !getenv("TEMCO_NO_CATP")) || (P->flags & TEMCO_FLAG_MMA_CAT)) &&
+          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+        e.kind = K_GROUP_CAT;
+        e.kernel = mma_catp_ok(e.cat) ? "mma_catp" : "mma_cat";
         e.launches = 1;
         continue;
       }

@@ -111,6 +111,7 @@ struct CatDesc {
   CatTerm term[kCatMaxTerms];
   CatUnit unit[kCatMaxUnits];
   int32_t n_terms, n_plain, n_units;
+  int16_t chunk_u0[kCatMaxChunks + 1];   // units of chunk c: [chunk_u0[c], chunk_u0[c + 1])
   int32_t C, nchunks, Nout, NO;
   int32_t H, W, npix, nblocks;
   int32_t relu;               // level activation

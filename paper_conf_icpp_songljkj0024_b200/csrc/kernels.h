@@ -24,7 +24,8 @@ void launch_conv_rank_mma(const RankConvDesc& d, const uint16_t* tcw, const RunP
 bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                    CatDesc& d);
 void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s);
-bool mma_poolcat_ok(const CatDesc& d);   // restore-once 3x3/s2 max-pooled member (launch_mma_cat dispatches)
+bool mma_poolcat_ok(const CatDesc& d);
+bool mma_catp_ok(const CatDesc& d);      // chunk-parallel concat kernel applies (launch_mma_cat dispatches)   // restore-once 3x3/s2 max-pooled member (launch_mma_cat dispatches)
 bool dwconv_vec_ok(const ConvDesc& d);   // depthwise bf16, C % 8 == 0: vectorised kernel
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)

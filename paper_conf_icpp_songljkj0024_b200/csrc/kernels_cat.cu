@@ -215,6 +215,10 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
   }
   if ((int)U.size() > kCatMaxUnits) return false;
   d.n_units = (int)U.size();
+  for (int c = 0, i = 0; c <= d.nchunks; ++c) {
+    while (i < d.n_units && U[i].chunk < c) ++i;
+    d.chunk_u0[c] = (int16_t)i;
+  }
   for (int i = 0; i < d.n_units; ++i) d.unit[i] = U[i];
   while (tcw.size() % 512) tcw.push_back(0);
   d.blob = (int64_t)tcw.size();
@@ -727,6 +731,168 @@ void launch_poolcat_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, c
   launch_pdl(mma_poolcat_kernel<NO, PK, PS, PP>, dim3(grid), dim3(32 * kPcWarps), smem, s, d, p, tcw, tw, th);
 }
 
+// ---------------------------------------------------------------------------
+// Chunk-parallel concat kernel for single-level concat groups without a pooled
+// member on few pixels (DenseNet-121 blocks 2-4: 25k-100k pixels, C up to 1024 in
+// 64-channel chunks of one or two lconv terms each).  The per-block work of the
+// generic concat kernel is a long serial chain of (term, tap) units; here each
+// warp owns ONE (16-pixel block, 64-channel chunk) pair -- its units' loads all
+// in flight together, restore, ReLU, and the chunk's partial reduce GEMM -- and
+// the CTA sums the chunks' partial outputs through SMEM (fixed order:
+// deterministic, batch-invariant).
+// ---------------------------------------------------------------------------
+constexpr int kCpWarps = 16;
+
+template <int NO, int KSM>
+__global__ void __launch_bounds__(32 * kCpWarps, 1) mma_catp_kernel(const __grid_constant__ CatDesc d, RunPtrs p,
+                                                                    const uint16_t* __restrict__ tcw) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int g = lane / 4, t4 = lane % 4;
+  {
+    const uint4* src = reinterpret_cast<const uint4*>(tcw + d.blob);
+    uint4* dst = reinterpret_cast<uint4*>(smem);
+    for (int i = threadIdx.x; i < d.blob_bytes / 16; i += blockDim.x) dst[i] = __ldg(src + i);
+  }
+  __syncthreads();
+  pdl_wait();
+  pdl_trigger_early();
+  const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
+  const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
+  float* red = reinterpret_cast<float*>(smem + (d.blob_bytes + 15) / 16 * 16);   // [warp][16][Nout]
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+  const int lq = lane >> 3, lr = lane & 7;
+  const uint32_t sbase = s_u32(blob);
+  const int nch = d.nchunks, bpi = kCpWarps / nch;    // blocks per iteration
+  const int wb = warp / nch, ch = warp - wb * nch;
+  const bool active = wb < bpi;
+  const int u0 = d.chunk_u0[ch], u1 = d.chunk_u0[ch + 1];
+  for (int it = blockIdx.x; it * bpi < d.nblocks; it += gridDim.x) {
+    const int blk = it * bpi + wb;
+    if (active && blk < d.nblocks) {
+      const CatRows rw = cat_rows(d, blk, g);
+      float D[8][4];
+#pragma unroll
+      for (int nt = 0; nt < 8; ++nt) {
+        const float2 b = *reinterpret_cast<const float2*>(fb + d.lbias + ch * 64 + nt * 8 + 2 * t4);
+        D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
+      }
+      // units in batches of 4: their loads in flight together
+      for (int ub = u0; ub < u1; ub += 4) {
+        uint32_t a[4][KSM][4];
+        bool va[2];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (ub + q < u1) cat_load<KSM>(a[q], va, d, p, d.unit[ub + q], rw, t4);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          if (ub + q >= u1) break;
+          const CatUnit u = d.unit[ub + q];
+          if (u.term < 0) continue;
+          const int nks = d.term[u.term].ks, rs = d.term[u.term].rs;
+          const uint32_t wb4 = sbase + (uint32_t)((u.woff + ((lq >> 1) * 8 + lr) * rs + (lq & 1) * 8) * 2);
+          const uint32_t wb2 = sbase + (uint32_t)((u.woff + lr * rs + (lq & 1) * 8) * 2);
+#pragma unroll
+          for (int ks = 0; ks < KSM; ++ks) {
+            if (ks >= nks) break;
+#pragma unroll
+            for (int nt = 0; nt < 8; nt += 2) {
+              if (nt >= u.nt0 && nt < u.nt1) {
+                const uint32_t roff = (uint32_t)(((nt - u.nt0) * 8 * rs + ks * 16) * 2);
+                if (nt + 1 < u.nt1) {
+                  uint32_t b0, b1, b2, b3;
+                  ldsm_x4(wb4 + roff, b0, b1, b2, b3);
+                  mma16816(D[nt], a[q][ks], b0, b1);
+                  mma16816(D[nt + 1], a[q][ks], b2, b3);
+                } else {
+                  uint32_t b0, b1;
+                  ldsm_x2(wb2 + roff, b0, b1);
+                  mma16816(D[nt], a[q][ks], b0, b1);
+                }
+              } else if (nt + 1 >= u.nt0 && nt + 1 < u.nt1) {
+                uint32_t b0, b1;
+                ldsm_x2(wb2 + (uint32_t)(((nt + 1 - u.nt0) * 8 * rs + ks * 16) * 2), b0, b1);
+                mma16816(D[nt + 1], a[q][ks], b0, b1);
+              }
+            }
+          }
+        }
+      }
+      if (d.relu) {
+#pragma unroll
+        for (int nt = 0; nt < 8; ++nt)
+#pragma unroll
+          for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+      }
+      float O[NO][4];
+#pragma unroll
+      for (int i = 0; i < NO; ++i) O[i][0] = O[i][1] = O[i][2] = O[i][3] = 0.f;
+#pragma unroll
+      for (int kp = 0; kp < 2; ++kp) {
+        uint32_t pa[2][4];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int ks = 2 * kp + h;
+          pa[h][0] = pk2(D[2 * ks][0], D[2 * ks][1]);
+          pa[h][1] = pk2(D[2 * ks][2], D[2 * ks][3]);
+          pa[h][2] = pk2(D[2 * ks + 1][0], D[2 * ks + 1][1]);
+          pa[h][3] = pk2(D[2 * ks + 1][2], D[2 * ks + 1][3]);
+        }
+#pragma unroll
+        for (int nb = 0; nb < NO; ++nb) {
+          if (nb >= d.NO) break;
+          uint32_t f0, f1, f2, f3;
+          ldsm_x4(sbase + (uint32_t)((d.f + (nb * 8 + lr) * d.fs + ch * 64 + kp * 32 + lq * 8) * 2), f0, f1, f2, f3);
+          mma16816(O[nb], pa[0], f0, f1);
+          mma16816(O[nb], pa[1], f2, f3);
+        }
+      }
+      float* rwp = red + (size_t)warp * 16 * d.Nout;
+#pragma unroll
+      for (int nb = 0; nb < NO; ++nb) {
+        if (nb >= d.NO) break;
+        const int col = nb * 8 + 2 * t4;
+        *reinterpret_cast<float2*>(rwp + g * d.Nout + col) = make_float2(O[nb][0], O[nb][1]);
+        *reinterpret_cast<float2*>(rwp + (g + 8) * d.Nout + col) = make_float2(O[nb][2], O[nb][3]);
+      }
+    }
+    __syncthreads();
+    // sum the chunks' partials (chunk order fixed) and store bf16 pairs
+    const int per_blk = 16 * d.Nout / 2;
+    for (int i = threadIdx.x; i < bpi * per_blk; i += blockDim.x) {
+      const int b = i / per_blk, e = (i - b * per_blk) * 2;
+      const int blk = it * bpi + b;
+      const int m = blk * 16 + e / d.Nout;
+      if (blk >= d.nblocks || m >= d.npix) continue;
+      float s0 = 0.f, s1 = 0.f;
+      for (int c = 0; c < nch; ++c) {
+        const float2 v = *reinterpret_cast<const float2*>(red + (size_t)(b * nch + c) * 16 * d.Nout + e);
+        s0 += v.x;
+        s1 += v.y;
+      }
+      *reinterpret_cast<uint32_t*>(y + (int64_t)m * d.Nout + e % d.Nout) = pk2(s0, s1);
+    }
+    __syncthreads();
+  }
+}
+
+template <int NO, int KSM>
+void launch_catp_t(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  static bool configured = false;
+  static int sms = 148;
+  const int smem = (d.blob_bytes + 15) / 16 * 16 + kCpWarps * 16 * d.Nout * 4;
+  if (!configured) {
+    cudaFuncSetAttribute(mma_catp_kernel<NO, KSM>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    configured = true;
+  }
+  const int bpi = kCpWarps / d.nchunks;
+  const int grid = std::min((d.nblocks + bpi - 1) / bpi, sms);
+  launch_pdl(mma_catp_kernel<NO, KSM>, dim3(grid), dim3(32 * kCpWarps), smem, s, d, p, tcw);
+}
+
 template <int KSM, bool POOL>
 void launch_cat_no(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   switch ((d.NO + 1) / 2) {
@@ -738,6 +904,15 @@ void launch_cat_no(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cuda
 }
 
 }  // namespace
+
+bool mma_catp_ok(const CatDesc& d) {
+  // measured (B200): wins only where the tcgen05 kernel's 128-pixel tiles leave most SMs idle
+  // (ResNet-18c stages 3-4: 16-64 tiles); 1.5-2x slower than tcgen05 on DenseNet's blocks 2-4
+  if (d.pool != 0 || d.nchunks > 8 || d.npix >= 74 * 128) return false;
+  for (int j = 0; j < d.n_terms; ++j)
+    if (d.term[j].ks > 4) return false;
+  return (d.blob_bytes + 15) / 16 * 16 + kCpWarps * 16 * d.Nout * 4 <= 227 * 1024;
+}
 
 bool mma_poolcat_ok(const CatDesc& d) {
   if (getenv("TEMCO_DEBUG_CAT"))
@@ -754,6 +929,15 @@ bool mma_poolcat_ok(const CatDesc& d) {
 }
 
 void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  if (mma_catp_ok(d)) {
+    int ksm = 1;
+    for (int j = 0; j < d.n_terms; ++j) ksm = std::max(ksm, d.term[j].ks);
+    const int no2 = (d.NO + 1) / 2;
+#define TEMCO_CATP(n, k) if ((no2 * 2 <= n) && ksm <= k) return launch_catp_t<n, k>(d, tcw, p, s);
+    TEMCO_CATP(2, 1) TEMCO_CATP(2, 2) TEMCO_CATP(2, 4) TEMCO_CATP(4, 1) TEMCO_CATP(4, 2) TEMCO_CATP(4, 4)
+    TEMCO_CATP(8, 1) TEMCO_CATP(8, 2) TEMCO_CATP(8, 4)
+#undef TEMCO_CATP
+  }
   if (mma_poolcat_ok(d)) {
     if (d.pk == 2) {   // VGG's 2x2 / stride-2 pools
       if (d.NO == 1) return launch_poolcat_t<1, 2, 2, 0>(d, tcw, p, s);
