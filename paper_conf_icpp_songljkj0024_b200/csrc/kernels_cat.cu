@@ -915,10 +915,6 @@ bool mma_catp_ok(const CatDesc& d) {
 }
 
 bool mma_poolcat_ok(const CatDesc& d) {
-  if (getenv("TEMCO_DEBUG_CAT"))
-    fprintf(stderr, "poolcat? pool %d k %d s %d p %d pc %d-%d NO %d terms %d/%d R %d blob %d\n", d.pool, d.pk, d.ps,
-            d.pp, d.pc0, d.pc1, d.NO, d.n_plain, d.n_terms, d.n_terms > d.n_plain ? d.term[d.n_plain].R : -1,
-            d.blob_bytes);
   const bool win = (d.pk == 3 && d.ps == 2 && d.pp == 1) || (d.pk == 2 && d.ps == 2 && d.pp == 0);
   if (d.pool != 1 || !win || d.pc0 != 0 || d.pc1 != 1 || d.NO > 4) return false;
   if (d.n_terms != d.n_plain + 1 || d.term[d.n_plain].R > 16) return false;

@@ -1199,7 +1199,8 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
     configured = true;
   }
   int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
-  if (getenv("TEMCO_TC_GRID")) grid = std::min(grid, atoi(getenv("TEMCO_TC_GRID")));   // experiments
+  static const int grid_cap = getenv("TEMCO_TC_GRID") ? atoi(getenv("TEMCO_TC_GRID")) : 0;   // experiments
+  if (grid_cap > 0) grid = std::min(grid, grid_cap);
   // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
   launch_pdl(tc_chain_kernel, dim3(grid), dim3(kThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }
