@@ -137,6 +137,59 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
   const uint32_t wbase4 = s_u32(wb + ((lq >> 1) * 8 + lr) * ws + (lq & 1) * 8);
   const uint32_t wbase2 = s_u32(wb + lr * ws + (lq & 1) * 8);
   const int nw = gridDim.x * kRkWarps;
+  if constexpr (KS == 1 && !KCH) {
+    if (d.nblocks <= 2 * nw && taps <= 9) {
+      // few blocks per warp (small feature maps: launch / latency bound): every tap's
+      // A fragments of the block in flight at once instead of two units ahead
+      for (int blk = blockIdx.x * kRkWarps + warp; blk < d.nblocks; blk += nw) {
+        RkCursor u{};
+        u.blk = blk;
+        rk_set_block(d, u, g);
+        uint32_t at[9][1][4];
+#pragma unroll
+        for (int t = 0; t < 9; ++t) {
+          u.tap = t;
+          if (t < taps) rk_load<1>(at[t], d, x, u, t4);
+        }
+        float acc[NT][4];
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt) {
+          float b0 = 0.f, b1 = 0.f;
+          if (d.b >= 0) {
+            b0 = p.params[d.b + nt * 8 + 2 * t4];
+            b1 = p.params[d.b + nt * 8 + 2 * t4 + 1];
+          }
+          acc[nt][0] = acc[nt][2] = b0;
+          acc[nt][1] = acc[nt][3] = b1;
+        }
+#pragma unroll
+        for (int t = 0; t < 9; ++t) {
+          if (t >= taps) break;
+          const uint32_t tw = (uint32_t)(t * d.K * ws * 2);
+#pragma unroll
+          for (int np = 0; np < NT / 2; ++np) {
+            uint32_t b0, b1, b2, b3;
+            ldsm_x4(wbase4 + tw + (uint32_t)(np * 16 * ws * 2), b0, b1, b2, b3);
+            mma16816(acc[2 * np], at[t][0], b0, b1);
+            mma16816(acc[2 * np + 1], at[t][0], b2, b3);
+          }
+          if (NT & 1) {
+            uint32_t b0, b1;
+            ldsm_x2(wbase2 + tw + (uint32_t)((NT - 1) * 8 * ws * 2), b0, b1);
+            mma16816(acc[NT - 1], at[t][0], b0, b1);
+          }
+        }
+        const int m0 = blk * 16 + g, m1 = m0 + 8;
+#pragma unroll
+        for (int nt = 0; nt < NT; ++nt) {
+          const int col = nt * 8 + 2 * t4;
+          if (m0 < d.npix) *reinterpret_cast<uint32_t*>(y + (int64_t)m0 * d.K + col) = pk2(acc[nt][0], acc[nt][1]);
+          if (m1 < d.npix) *reinterpret_cast<uint32_t*>(y + (int64_t)m1 * d.K + col) = pk2(acc[nt][2], acc[nt][3]);
+        }
+      }
+      return;
+    }
+  }
   // unit order per block: output chunk, tap, input chunk
   auto advance = [&](RkCursor& u) {
     if (KCH && ++u.kc < d.nkc) return;
