@@ -219,6 +219,38 @@ void launch_stem_t(const ConvDesc& d, const StemGeo& g, const RunPtrs& p, cudaSt
   launch_pdl(conv_stem_kernel<KS, NT>, dim3((unsigned)grid), dim3(kStThreads), g.smem, s, d, g, p, tw, th);
 }
 
+// 1x1 stride-1 conv on the image (VGG's first CP factor, 3 -> 8): a pure per-pixel
+// map, HBM-bound on the 6-byte pixel read + 16-byte write -- one thread per pixel,
+// weights in registers, fp32 FMAs, one 16-byte store
+template <int CIN>
+__global__ void __launch_bounds__(256) conv_pw_small_kernel(ConvDesc d, RunPtrs p) {
+  float w[8][CIN], b[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+#pragma unroll
+    for (int c = 0; c < CIN; ++c) w[k][c] = p.params[d.w + k * CIN + c];
+    b[k] = d.b >= 0 ? p.params[d.b + k] : 0.f;
+  }
+  pdl_wait();
+  pdl_trigger_early();
+  const unsigned short* x = reinterpret_cast<const unsigned short*>(loc_ptr(d.x, p));
+  uint4* y = reinterpret_cast<uint4*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const int64_t npix = (int64_t)d.N * d.H * d.W;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < npix; i += (int64_t)gridDim.x * blockDim.x) {
+    float xv[CIN];
+#pragma unroll
+    for (int c = 0; c < CIN; ++c) xv[c] = __uint_as_float((uint32_t)__ldg(x + i * CIN + c) << 16);
+    float o[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      o[k] = b[k];
+#pragma unroll
+      for (int c = 0; c < CIN; ++c) o[k] = fmaf(w[k][c], xv[c], o[k]);
+    }
+    y[i] = make_uint4(pack2(o[0], o[1]), pack2(o[2], o[3]), pack2(o[4], o[5]), pack2(o[6], o[7]));
+  }
+}
+
 }  // namespace
 
 bool conv_stem_ok(const ConvDesc& d) {
@@ -230,6 +262,12 @@ bool conv_stem_ok(const ConvDesc& d) {
 }
 
 void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
+  if (d.kh == 1 && d.kw == 1 && d.sh == 1 && d.ph == 0 && d.pw == 0 && d.C == 3 && d.K == 8) {
+    const int64_t npix = (int64_t)d.N * d.H * d.W;
+    const int grid = (int)std::min<int64_t>((npix + 255) / 256, 148LL * 16);
+    launch_pdl(conv_pw_small_kernel<3>, dim3(grid), dim3(256), 0, s, d, p);
+    return;
+  }
   const StemGeo g = stem_geo(d);
 #define TEMCO_STEM_CASE(ks, nt) \
   if (g.KS == ks && g.NT == nt) return launch_stem_t<ks, nt>(d, g, p, s);
