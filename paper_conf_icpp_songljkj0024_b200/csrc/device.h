@@ -84,6 +84,7 @@ struct RankConvDesc {          // reduced-rank conv on tensor cores (kernels_ran
   int32_t KS, NT;             // k-steps of 16 input channels, n-tiles of 8 output channels
   int32_t pair;               // Cin == 8: a k-step of 16 covers two taps
   int32_t nkc, nnc;           // 64-channel input / output chunks (wide convs)
+  int32_t all_taps;           // single-k-step convs: load every tap of a block at once
   int32_t wstride;            // bf16 elements per weight row in SMEM
   int64_t wblob;              // tc weight pool offset: [tap][K][wstride] bf16
   int32_t blob_bytes;
