@@ -139,18 +139,18 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
   const uint32_t wbase4 = s_u32(wb + ((lq >> 1) * 8 + lr) * ws + (lq & 1) * 8);
   const uint32_t wbase2 = s_u32(wb + lr * ws + (lq & 1) * 8);
   const int nw = gridDim.x * kRkWarps;
-  if constexpr (KS == 1 && !KCH) {
+  if constexpr (KS <= 2 && !KCH) {
     if ((d.nblocks <= 2 * nw || all_taps_mode(d)) && taps <= 9) {
       // every tap's A fragments of the block in flight at once (instead of two units ahead)
       for (int blk = blockIdx.x * kRkWarps + warp; blk < d.nblocks; blk += nw) {
         RkCursor u{};
         u.blk = blk;
         rk_set_block(d, u, g);
-        uint32_t at[9][1][4];
+        uint32_t at[9][KS][4];
 #pragma unroll
         for (int t = 0; t < 9; ++t) {
           u.tap = t;
-          if (t < taps) rk_load<1>(at[t], d, x, u, t4);
+          if (t < taps) rk_load<KS>(at[t], d, x, u, t4);
         }
         float acc[NT][4];
 #pragma unroll
@@ -168,16 +168,19 @@ __global__ void __launch_bounds__(32 * kRkWarps, 1) conv_rank_mma_kernel(const _
           if (t >= taps) break;
           const uint32_t tw = (uint32_t)(t * d.K * ws * 2);
 #pragma unroll
-          for (int np = 0; np < NT / 2; ++np) {
-            uint32_t b0, b1, b2, b3;
-            ldsm_x4(wbase4 + tw + (uint32_t)(np * 16 * ws * 2), b0, b1, b2, b3);
-            mma16816(acc[2 * np], at[t][0], b0, b1);
-            mma16816(acc[2 * np + 1], at[t][0], b2, b3);
-          }
-          if (NT & 1) {
-            uint32_t b0, b1;
-            ldsm_x2(wbase2 + tw + (uint32_t)((NT - 1) * 8 * ws * 2), b0, b1);
-            mma16816(acc[NT - 1], at[t][0], b0, b1);
+          for (int ks = 0; ks < KS; ++ks) {
+#pragma unroll
+            for (int np = 0; np < NT / 2; ++np) {
+              uint32_t b0, b1, b2, b3;
+              ldsm_x4(wbase4 + tw + (uint32_t)((np * 16 * ws + ks * 16) * 2), b0, b1, b2, b3);
+              mma16816(acc[2 * np], at[t][ks], b0, b1);
+              mma16816(acc[2 * np + 1], at[t][ks], b2, b3);
+            }
+            if (NT & 1) {
+              uint32_t b0, b1;
+              ldsm_x2(wbase2 + tw + (uint32_t)(((NT - 1) * 8 * ws + ks * 16) * 2), b0, b1);
+              mma16816(acc[NT - 1], at[t][ks], b0, b1);
+            }
           }
         }
         const int m0 = blk * 16 + g, m1 = m0 + 8;
