@@ -50,9 +50,39 @@ def _peaks():
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+    """SM clock and throttle reasons sampled DURING the timed region (B200_PROFILING.md clocks
+    line): an NVML sampler thread every 2 ms (short steps end before nvidia-smi's 100 ms loop
+    takes a sample); nvidia-smi -lms 100 as the fallback when NVML is unavailable."""
+
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4))
 
     def __init__(self, index):
+        self.rows, self.p, self.t = [], None, None
+        try:
+            import threading
+
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            self.stop_ev = threading.Event()
+
+            def run():
+                while not self.stop_ev.is_set():
+                    try:
+                        self.rows.append((pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM),
+                                          pynvml.nvmlDeviceGetUtilizationRates(h).gpu,
+                                          pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)))
+                    except Exception:
+                        pass
+                    self.stop_ev.wait(0.002)
+
+            self.t = threading.Thread(target=run, daemon=True)
+            self.t.start()
+            return
+        except Exception:
+            self.t = None
         self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
         q = ("clocks.sm,clocks.max.sm,utilization.gpu,clocks_event_reasons.hw_slowdown,"
              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
@@ -64,6 +94,15 @@ class Clocks:
             self.p = None
 
     def stop(self):
+        if self.t is not None:
+            self.stop_ev.set()
+            self.t.join()
+            if not self.rows:
+                return None
+            loaded = [r for r in self.rows if r[1] > 0] or self.rows
+            reasons = sorted({n for r in loaded for n, bit in self.REASONS if r[2] & bit})
+            return {"sm_mhz": statistics.median(r[0] for r in loaded), "sm_max_mhz": self.max_mhz,
+                    "reasons": reasons, "samples": len(loaded), "source": "nvml"}
         if self.p is None:
             return None
         self.p.terminate()
@@ -80,7 +119,7 @@ class Clocks:
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in loaded for i in range(4) if r[3 + i].lower() == "active"})
         return {"sm_mhz": statistics.median(int(r[0]) for r in loaded), "sm_max_mhz": int(rows[0][1]),
-                "reasons": reasons, "samples": len(loaded)}
+                "reasons": reasons, "samples": len(loaded), "source": "nvidia-smi"}
 
 
 def _dist():
@@ -279,10 +318,10 @@ def main():
                        "ms": round(v["ms"], 4)}
     ideal = actual = 0.0
     for s, t in zip(steps, prof):
-        if s["kernel"] in ("tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat") and t > 0:
+        if s["kernel"] in ("tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat", "mma_catp") and t > 0:
             ideal += max(s.get("alg_flops", s["flops"]) / (tf_sust * 1e12), s.get("alg_bytes", s["io_bytes"]) / (hbm * 1e9))
             actual += float(t) * 1e-3
-    fused = {"kernels": ["tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat"], "roofline_ms": round(ideal * 1e3, 4),
+    fused = {"kernels": ["tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat", "mma_catp"], "roofline_ms": round(ideal * 1e3, 4),
              "measured_ms": round(actual * 1e3, 4), "frac": round(ideal / actual, 4) if actual else None,
              "note": "per launch max(alg FLOP / sustained bf16 peak, alg bytes / HBM peak), summed, / measured"}
     # DRAM traffic of the dominant class from the committed ncu capture of this
