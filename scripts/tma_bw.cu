@@ -86,18 +86,19 @@ int main() {
     cuuint32_t es[2] = {1, 1};
     encode(&map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, buf, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    for (int stages : {2, 4, 8, 12}) {
+    for (int nsm : {sms, sms / 2, sms / 4, 16})
+    for (int stages : {4, 8}) {
       const int iters = 4000;
-      stream_kernel<<<sms, 32, stages * 16384 + 1024>>>(map, buf, mode, stages, 100, rows, cyc);
-      stream_kernel<<<sms, 32, stages * 16384 + 1024>>>(map, buf, mode, stages, iters, rows, cyc);
+      stream_kernel<<<nsm, 32, stages * 16384 + 1024>>>(map, buf, mode, stages, 100, rows, cyc);
+      stream_kernel<<<nsm, 32, stages * 16384 + 1024>>>(map, buf, mode, stages, iters, rows, cyc);
       cudaDeviceSynchronize();
       unsigned long long h[256];
-      cudaMemcpy(h, cyc, sms * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
+      cudaMemcpy(h, cyc, nsm * sizeof(unsigned long long), cudaMemcpyDeviceToHost);
       double avg = 0;
-      for (int i = 0; i < sms; ++i) avg += (double)h[i] / sms;
+      for (int i = 0; i < nsm; ++i) avg += (double)h[i] / nsm;
       const double bpc = 16384.0 * iters / avg;
-      printf("%s stages %2d: %6.1f B/cycle/SM  (%5.0f cycles per 16 KB stage, ~%.1f TB/s over %d SMs at 1.965 GHz)\n",
-             names[mode], stages, bpc, avg / iters, bpc * sms * 1.965e9 / 1e12, sms);
+      printf("%s SMs %3d stages %2d: %6.1f B/cycle/SM  (%5.0f cycles per 16 KB stage, ~%.1f TB/s aggregate at 1.965 GHz)\n",
+             names[mode], nsm, stages, bpc, avg / iters, bpc * nsm * 1.965e9 / 1e12);
     }
   }
   printf("%s\n", cudaGetErrorString(cudaGetLastError()));
