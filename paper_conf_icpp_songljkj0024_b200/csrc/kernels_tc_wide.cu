@@ -142,7 +142,10 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
             for (int q = 0; q < ntap; ++q) {
               const int tap = un.pooled ? un.tg * d.tpu + r : q;
               const int kk = un.pooled ? d.mk : t.tk, pad = un.pooled ? d.mp : t.tp;
-              for (int ka = 0; ka < katoms; ++ka) {
+              const int step = d.k2 ? 2 : 1;   // K atoms per ring stage
+              for (int ka = 0; ka < katoms; ka += step) {
+                const int n2 = std::min(step, katoms - ka);
+                auto nk_of = [&](int a) { return std::min(t.aw / 16, (t.R - a * t.aw + 15) / 16); };
                 TcProdOp o{};
                 o.kind = d.spatial ? PK_A4D : PK_A2D;
                 o.ts = (uint8_t)t.ts;
@@ -150,7 +153,9 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
                 o.ac = (int16_t)(ka * t.aw);
                 o.dx = (int16_t)(tap % kk - pad);
                 o.dy = (int16_t)(tap / kk - pad);
-                o.bytes = (uint16_t)((rows_a + (res ? 0 : Cc)) * t.aw * 2);
+                o.bytes = (uint32_t)(n2 * (rows_a + (res ? 0 : Cc)) * t.aw * 2);
+                o.n2 = (uint8_t)n2;
+                o.aw = (uint8_t)t.aw;
                 if (!res) {
                   o.kind |= PK_B;
                   o.bmap = moff(t.wmap);
@@ -163,7 +168,12 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
                 if (l == 0 && !region_done[r]) m.flags |= MF_ZERO;
                 region_done[r] = 1;
                 m.unit = (uint8_t)u;
-                m.nk = (uint8_t)std::min(t.aw / 16, (t.R - ka * t.aw + 15) / 16);
+                m.nk = (uint8_t)(nk_of(ka) + (n2 == 2 ? nk_of(ka + 1) : 0));
+                if (n2 == 2) {
+                  m.nk1 = (uint8_t)nk_of(ka);
+                  m.a2 = (uint16_t)((rows_a * t.aw * 2) >> 4);
+                  m.b2 = (uint16_t)((Cc * t.aw * 2) >> 4);
+                }
                 m.la = (uint8_t)t.aw;
                 m.lb = (uint8_t)t.aw;
                 m.tcol = (uint16_t)(r * Cc);
@@ -199,7 +209,8 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
             o.bmap = moff(d.fmap);
             o.bx = (int16_t)(un.c * Cc + a * 64);
             o.by = 0;
-            o.bytes = (uint16_t)(d.Np * 128);
+            o.bytes = (uint32_t)(d.Np * 128);
+            o.n2 = 1;
             P.push_back(o);
           }
           TcMmaOp m{};
@@ -269,10 +280,12 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
     o.adesc = dtmpl(aoff, m.la);
     o.bdesc = dtmpl(boff, m.lb);
     o.idesc = isF ? idesc(128, d.Np) : idesc(128, Cc);
-    o.tmem = isF ? (uint32_t)(2 * d.ubuf) : m.tcol;
+    o.tmem = (isF ? (uint32_t)(2 * d.ubuf) : m.tcol) | ((uint32_t)m.nk1 << 24);
     o.flags = m.flags;
     o.unit = m.unit;
     o.nk = m.nk;
+    o.a2 = m.a2;
+    o.b2 = m.b2;
   }
   d.prog_off = (int64_t)tcw.size();
   const size_t nbytes = P.size() * sizeof(TcProdOp) + MD.size() * sizeof(TcMmaOpD);
@@ -477,8 +490,15 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   int awmax = 16;
   const int nall = pm ? d.mt1 : d.n_terms;
   for (int i = 0; i < nall; ++i) awmax = std::max(awmax, d.term[i].aw);
-  d.slot_a = 128 * awmax * 2;
-  int sb = std::max(d.Cc * awmax * 2, d.Cc * 32);
+  // two K atoms per ring stage when some term spans several atoms (ranks > 64: ResNet-50
+  // stages 3-4): half the stages / commits / handshakes per MMA, measured -13..-26 % on those
+  // groups (and +1-2 % on single-atom groups, which keep one atom per stage)
+  int max_atoms = 1;
+  for (int i = 0; i < (pm ? d.mt1 : d.n_terms); ++i) max_atoms = std::max(max_atoms, d.term[i].Rp / d.term[i].aw);
+  d.k2 = (!pm && max_atoms >= 2 && !getenv("TEMCO_WIDE_NOK2")) ? 1 : 0;
+  const int rows_a_l = d.spatial ? d.tw * d.th * d.tn : 128;
+  d.slot_a = (d.k2 ? 2 : 1) * std::max(128, rows_a_l) * awmax * 2;
+  int sb = std::max((d.k2 ? 2 : 1) * d.Cc * awmax * 2, d.Cc * 32);
   if (!gap) sb = std::max(sb, d.Np * 128);
   d.slot_b = (sb + 1023) / 1024 * 1024;
   const int pbytes = 128 * d.Cc * 2;
@@ -760,6 +780,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
   pdl_trigger_early();
   const int U = units_per_tile(d);
 
+  const int rows_atom = d.spatial ? d.tw * d.th * d.tn : 128;   // rows of one A box
   if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer
     {   // whole warp; one elected lane issues (the resident preload runs in lane 0)
@@ -796,11 +817,15 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           TRACE(0, n0);
           mbar_expect_tx_w(&full[stage], o.bytes);
           uint8_t* sa = ring + stage * slot;
-          if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
-            tma_load_4d_w(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.w0 * o.ts + o.dx, gg.h0 * o.ts + o.dy, gg.n0);
-          else if (o.kind & PK_A2D)
-            tma_load_2d_w(sa, dbase + o.amap * 64, &full[stage], o.ac, gg.m0);
-          if (o.kind & PK_B) tma_load_2d_w(sa + kSlotA, dbase + o.bmap * 64, &full[stage], o.bx, o.by);
+          for (int a = 0; a < (int)o.n2; ++a) {   // one or two K atoms per stage
+            const int aoffb = a * rows_atom * o.aw * 2, boffb = a * Cc * o.aw * 2, ka = a * o.aw;
+            if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
+              tma_load_4d_w(sa + aoffb, dbase + o.amap * 64, &full[stage], o.ac + ka, gg.w0 * o.ts + o.dx,
+                            gg.h0 * o.ts + o.dy, gg.n0);
+            else if (o.kind & PK_A2D)
+              tma_load_2d_w(sa + aoffb, dbase + o.amap * 64, &full[stage], o.ac + ka, gg.m0);
+            if (o.kind & PK_B) tma_load_2d_w(sa + kSlotA + boffb, dbase + o.bmap * 64, &full[stage], o.bx + ka, o.by);
+          }
           TRACE(1, n1);
           if (++stage == S) stage = 0, phase ^= 1;
         }
@@ -868,7 +893,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           const uint64_t st16 = (uint64_t)((stage * slot) >> 4);
           const uint64_t ad = o.adesc + base16 + ((f & MF_SA) ? st16 : 0);
           const uint64_t bd = o.bdesc + base16 + ((f & MF_SB) ? st16 : 0);
-          const uint32_t dt = tbase + o.tmem + ((f & MF_F) ? 0u : (uint32_t)(bs * d.ubuf));
+          const uint32_t dt = tbase + (o.tmem & 0xFFFFu) + ((f & MF_F) ? 0u : (uint32_t)(bs * d.ubuf));
+          const uint32_t nk1 = (o.tmem >> 24) ? (o.tmem >> 24) : 8u;   // steps in the stage's first atom
           const uint32_t acc0 = (f & MF_ZERO) ? 0u : 1u;
           PROF_ADD(pc_dec);
           {
@@ -877,8 +903,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           const uint32_t idesc = o.idesc, nk = o.nk;
           mma_bf16_w(dt, ad, bd, idesc, acc0);
 #pragma unroll
-          for (uint32_t k = 1; k < 4; ++k)
-            if (k < nk) mma_bf16_w(dt, ad + 2 * k, bd + 2 * k, idesc, 1u);
+          for (uint32_t k = 1; k < 8; ++k)
+            if (k < nk) {
+              const bool second = k >= nk1;   // second atom of a two-atom stage
+              const uint32_t kk = second ? k - nk1 : k;
+              mma_bf16_w(dt, ad + (second ? o.a2 : 0) + 2 * kk, bd + (second ? o.b2 : 0) + 2 * kk, idesc, 1u);
+            }
           PROF_ADD(pc_issue);
 #ifdef TEMCO_TRACE
           pc_n += o.nk;

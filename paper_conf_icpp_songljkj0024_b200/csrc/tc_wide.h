@@ -56,8 +56,9 @@ struct TcProdOp {                 // one ring stage
   uint16_t amap, bmap;            // byte offsets / 64 of the CUtensorMaps inside TcChainDesc
   int16_t ac, dx, dy;             // A coords: channel; tap offsets (4D: w0*ts+dx, h0*ts+dy)
   int16_t bx, by;                 // B coords
-  uint16_t bytes;                 // expect_tx
-  uint16_t pad[7];
+  uint32_t bytes;                 // expect_tx
+  uint8_t n2, aw;                 // K atoms in the stage (1 or 2), atom width (elements)
+  uint16_t pad[5];
 };
 static_assert(sizeof(TcProdOp) == 32, "TcProdOp layout");
 enum : uint16_t {
@@ -83,17 +84,19 @@ struct TcMmaOp {
   uint8_t la, lb;                 // K-atom widths (layouts) of A and B
   uint16_t tcol;                  // TMEM column offset inside the unit buffer
   uint32_t aoff, boff;
+  uint8_t nk1;                    // two-atom stage: K=16 steps of the first atom (0: one atom)
+  uint16_t a2, b2;                // descriptor deltas (>> 4) of the second atom
 };
-static_assert(sizeof(TcMmaOp) == 16, "TcMmaOp layout");
 // device form: UMMA descriptors precomputed on the host relative to the
 // 1024-aligned SMEM base (start-address field = offset >> 4); the issuer only
 // adds (base >> 4) and, for ring operands, (stage * slot) >> 4
 struct TcMmaOpD {
   uint64_t adesc, bdesc;
-  uint32_t idesc, tmem;           // instruction descriptor; TMEM column (unit ops: + buffer * ubuf)
+  uint32_t idesc, tmem;           // instruction descriptor; TMEM column (low 16 bits; unit ops: + buffer * ubuf)
+                                  // bits 24-31: K=16 steps in the first atom of a two-atom stage (0: one atom)
   uint16_t flags;
   uint8_t unit, nk;
-  uint32_t pad;
+  uint16_t a2, b2;                // descriptor deltas (>> 4) of the stage's second A / B atom
 };
 static_assert(sizeof(TcMmaOpD) == 32, "TcMmaOpD layout");
 
@@ -132,6 +135,7 @@ struct TcChainDesc {
   // ring then carries only A tiles.  Avoids all 148 SMs re-reading the same
   // few weight lines through TMA every stage (L2 same-line contention).
   int32_t resident, wres_bytes;
+  int32_t k2;                            // two K atoms per ring stage (half the stages, twice the MMAs each)
   int32_t bres[kTcMaxLevels], bresm;     // bias boxes: [nchunks] x (Cc x 16), byte offsets
   int32_t fres;                          // F boxes: [Cpad / 64] x (Np x 64)
   int64_t prog_off;                      // tc weight pool offset (elements) of [prod ops][mma ops]

@@ -1,5 +1,5 @@
-TEMCO_WIDE_ASHARE=1 timeout 600 python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1
-for c in resnet50 densenet121; do
-for v in "" "TEMCO_WIDE_ASHARE=1"; do
-  echo "=== $c $v"; env $v timeout 120 python scripts/step_profile.py $c 400 | grep "tc_chain\|total"
-done; done > gpurun_out/exp_ash.log 2>&1
+timeout 600 python -m pytest tests -m gpu -x -q > gpurun_out/gpu_tests.log 2>&1
+for v in "" "TEMCO_WIDE_NOK2=1"; do
+  echo "=== bench $v"; env $v timeout 300 python bench.py --no-cpu-baseline | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print(d['value'], d['ms_per_step'], d['roofline']['frac'], d['fused_group_roofline']['frac'])"
+done > gpurun_out/exp_k2b.log 2>&1
+for c in densenet121 resnet18_cifar vgg16_cp; do echo "=== $c"; timeout 300 python bench.py --config $c --no-cpu-baseline | python -c "import json,sys; d=json.loads(sys.stdin.read().strip().splitlines()[-1]); print(d['value'], d['ms_per_step'])"; done >> gpurun_out/exp_k2b.log 2>&1
