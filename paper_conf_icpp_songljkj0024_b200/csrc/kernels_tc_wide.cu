@@ -156,6 +156,7 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
                 o.bytes = (uint32_t)(n2 * (rows_a + (res ? 0 : Cc)) * t.aw * 2);
                 o.n2 = (uint8_t)n2;
                 o.aw = (uint8_t)t.aw;
+                o.bstep64 = (uint16_t)(Cc * t.aw * 2 / 64);
                 if (!res) {
                   o.kind |= PK_B;
                   o.bmap = moff(t.wmap);
@@ -202,22 +203,31 @@ void build_programs(TcChainDesc& d, std::vector<uint16_t>& tcw) {
         if (!un.last) continue;
         const int pb = un.c & 1;
         const int na = Cc / 64;
-        for (int a = 0; a < na; ++a) {
+        // two F atoms per stage with two-atom stages, when they fit the stage's B region
+        const int fstep = (d.k2 && na == 2 && (res || 2 * d.Np * 128 <= d.slot_b)) ? 2 : 1;
+        for (int a = 0; a < na; a += fstep) {
           if (!res) {
             TcProdOp o{};
             o.kind = PK_B;
             o.bmap = moff(d.fmap);
             o.bx = (int16_t)(un.c * Cc + a * 64);
             o.by = 0;
-            o.bytes = (uint32_t)(d.Np * 128);
-            o.n2 = 1;
+            o.bytes = (uint32_t)(fstep * d.Np * 128);
+            o.n2 = (uint8_t)fstep;
+            o.aw = 64;
+            o.bstep64 = (uint16_t)(d.Np * 128 / 64);
             P.push_back(o);
           }
           TcMmaOp m{};
           m.flags = MF_F | (a == 0 ? MF_P_WAIT : 0) | (a == 0 && un.c == 0 ? MF_OUT_WAIT | MF_ZERO : 0) |
-                    (a == na - 1 ? MF_P_COMMIT : 0) | (res ? MF_BRES : MF_SW | MF_SB | MF_SD);
+                    (a + fstep >= na ? MF_P_COMMIT : 0) | (res ? MF_BRES : MF_SW | MF_SB | MF_SD);
           m.unit = (uint8_t)pb;
-          m.nk = 4;
+          m.nk = (uint8_t)(4 * fstep);
+          if (fstep == 2) {
+            m.nk1 = 4;
+            m.a2 = (uint16_t)(16384 >> 4);
+            m.b2 = (uint16_t)((d.Np * 128) >> 4);
+          }
           m.la = 64;
           m.lb = 64;
           m.aoff = (uint32_t)(pb * pbytes + a * 16384);
@@ -818,7 +828,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           mbar_expect_tx_w(&full[stage], o.bytes);
           uint8_t* sa = ring + stage * slot;
           for (int a = 0; a < (int)o.n2; ++a) {   // one or two K atoms per stage
-            const int aoffb = a * rows_atom * o.aw * 2, boffb = a * Cc * o.aw * 2, ka = a * o.aw;
+            const int aoffb = a * rows_atom * o.aw * 2, boffb = a * o.bstep64 * 64, ka = a * o.aw;
             if (o.kind & PK_A4D)        // (tap-shifted) strided box of the term's input
               tma_load_4d_w(sa + aoffb, dbase + o.amap * 64, &full[stage], o.ac + ka, gg.w0 * o.ts + o.dx,
                             gg.h0 * o.ts + o.dy, gg.n0);

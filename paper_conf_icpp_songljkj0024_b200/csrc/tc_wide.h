@@ -58,7 +58,8 @@ struct TcProdOp {                 // one ring stage
   int16_t bx, by;                 // B coords
   uint32_t bytes;                 // expect_tx
   uint8_t n2, aw;                 // K atoms in the stage (1 or 2), atom width (elements)
-  uint16_t pad[5];
+  uint16_t bstep64;               // byte offset / 64 of the stage's second B atom
+  uint16_t pad[4];
 };
 static_assert(sizeof(TcProdOp) == 32, "TcProdOp layout");
 enum : uint16_t {

@@ -33,3 +33,11 @@ def test_opt_in_concat_kernel_is_selected_by_its_flag():
     m = W.densenet121(batch=2, dtype="bf16", height=64, width=64)
     assert _kernels(m)["mma_cat"] == 0
     assert _kernels(m, FLAG_MMA_CAT)["mma_cat"] > 0
+
+
+def test_bf16_full_configs_never_fall_back_to_the_interpreter():
+    """Every fused group of the bench configs lowers to a tensor-core kernel: a lowering
+    regression would silently route a group to the SIMT interpreter (correct, 100x slower)."""
+    for name in ("resnet18_cifar", "resnet50", "vgg16_cp", "densenet121"):
+        ks = _kernels(W.build_config(name))
+        assert ks["simt_group"] == 0 and ks["simt_group_gap"] == 0, (name, ks)
