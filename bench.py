@@ -178,6 +178,9 @@ def cpu_baseline(config):
             "sample": f"{sample} images of {config} through the oracle's TeMCO executor (fp64 numpy), {dt:.1f} s"}
 
 
+VARIANTS = {"temco": 0, "fusion_only": 2, "skipopt_only": 4, "decomposed": 6}   # TEMCO_FLAG_NO_SKIPOPT=2, NO_FUSION=4
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -187,6 +190,10 @@ def main():
     ap.add_argument("--impl", default="temco", choices=["temco", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--simt-only", action="store_true")
+    # SURVEY 8(f) f3, the paper's ablations (Fig. 10/11) on the GPU:
+    # decomposed = neither rewrite, fusion_only = no skip optimization,
+    # skipopt_only = no fusion.  Not the headline line: same metric, other plan.
+    ap.add_argument("--variant", default="temco", choices=list(VARIANTS))
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -203,7 +210,7 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     B = CONFIG_BATCH[args.config]
     m = W.build_config(args.config, batch=B)
-    flags = FLAG_CUDA_GRAPH | (FLAG_SIMT_ONLY if args.simt_only else 0)
+    flags = FLAG_CUDA_GRAPH | (FLAG_SIMT_ONLY if args.simt_only else 0) | VARIANTS[args.variant]
     plan = Plan(m, flags=flags)
     desc = plan.describe()
     out_shape = plan.output_shape()
@@ -328,7 +335,7 @@ def main():
     # config (scripts/launch_summary.py --json), bytes per step like `achieved`
     traffic = None
     tpath = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
-    if os.path.exists(tpath):
+    if os.path.exists(tpath) and args.variant == "temco":
         traffic = json.load(open(tpath)).get(dom)
 
     if rank == 0:
@@ -342,7 +349,8 @@ def main():
                        "peak_internal_bytes": plan.peak_internal_bytes(0),
                        "peak_internal_bytes_unfused": plan.peak_internal_bytes(1),
                        "internal_memory_reduction": 1 - plan.peak_internal_bytes(0) / plan.peak_internal_bytes(1),
-                       "cuda_graph": True, "kernels": "simt-only" if args.simt_only else "tcgen05+simt"},
+                       "cuda_graph": True, "kernels": "simt-only" if args.simt_only else "tcgen05+simt",
+                       "variant": args.variant},
             "gpu_launches": desc["launches"] * args.steps,
             "e2e": {"value": ws * B / (e2e_ms / 1e3), "unit": "images/s", "api": "temco_run_host_async (pipelined H2D)",
                     "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),

@@ -413,6 +413,34 @@ void lower(temco_plan_s* P) {
         e.stem = !(P->flags & TEMCO_FLAG_SIMT_ONLY) && !dwconv_vec_ok(c) && !conv_rank_ok(c) && conv_stem_ok(c);
         e.kernel = e.stem ? "mma_conv_stem" : v.groups > 1 ? (dwconv_vec_ok(c) ? "simt_dwconv_vec" : "simt_dwconv") : conv_rank_ok(c) ? "simt_conv_rank" : conv_small_ok(c) ? "simt_conv_small" : "simt_conv";
         e.launches = 1;
+        // a standalone 1x1 / stride-1 conv left to the generic SIMT kernel (the unfused restores and
+        // reduces of the ablation plans, Cout > 256) is a plain NHWC GEMM y[NHW, O] = x[NHW, C] W^T:
+        // cuBLAS, bf16 operands, fp32 accumulate; bf16 output written directly when there is no bias
+        if (e.kernel == "simt_conv" && P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && v.w &&
+            v.kh == 1 && v.kw == 1 && v.sh == 1 && v.sw == 1 && v.ph == 0 && v.pw == 0 && v.groups == 1 &&
+            c.x.dtype == DT_BF16 && c.y.dtype == DT_BF16 && x.C % 8 == 0 && v.C % 8 == 0 && !getenv("TEMCO_NO_CONV_BLAS")) {
+          LinearDesc& l = e.lin;
+          l = LinearDesc{};
+          l.x = c.x;
+          l.y = c.y;
+          l.N = N * x.H * x.W; l.K = x.C; l.O = v.C;
+          l.w = -1;
+          l.b = push_params(P, v.b);
+          l.relu = 0;
+          while (P->tcw_h.size() % 512) P->tcw_h.push_back(0);
+          l.wb = (int64_t)P->tcw_h.size();
+          for (float f : *v.w) {            // OIHW with 1x1 taps = [O][C] row-major
+            uint32_t u;
+            memcpy(&u, &f, 4);
+            u += 0x7FFF + ((u >> 16) & 1);
+            P->tcw_h.push_back((uint16_t)(u >> 16));
+          }
+          l.blas = l.b >= 0 ? 1 : 2;
+          // (a nonzero workspace also creates the plan's cuBLAS handle)
+          P->lin_ws_elems = std::max<int64_t>(P->lin_ws_elems, l.blas == 1 ? (int64_t)l.N * l.O : 1);
+          e.kind = K_LINEAR;
+          e.kernel = "blas_conv1x1";
+        }
         break;
       }
       case OP_LINEAR: {
@@ -616,6 +644,15 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
           // y = W x: column-major C[O x N] = W^T[O x K] * x[K x N] (W row-major [O][K], x row-major [N][K])
           const float one = 1.f, zero = 0.f;
           const void* xin = loc_ptr(e.lin.x, rp);
+          if (e.lin.blas == 2) {   // 1x1 conv without bias: bf16 output straight into y
+            if (cublasSetStream(P->blas, st) != CUBLAS_STATUS_SUCCESS ||
+                cublasGemmEx(P->blas, CUBLAS_OP_T, CUBLAS_OP_N, e.lin.O, e.lin.N, e.lin.K, &one, P->tcw_d + e.lin.wb,
+                             CUDA_R_16BF, e.lin.K, xin, CUDA_R_16BF, e.lin.K, &zero,
+                             const_cast<void*>(loc_ptr(e.lin.y, rp)), CUDA_R_16BF, e.lin.O, CUBLAS_COMPUTE_32F,
+                             CUBLAS_GEMM_DEFAULT) != CUBLAS_STATUS_SUCCESS)
+              return set_err(TEMCO_ERR_CUDA, "cublasGemmEx (1x1 conv)");
+            break;
+          }
           if (cublasSetStream(P->blas, st) != CUBLAS_STATUS_SUCCESS ||
               cublasGemmEx(P->blas, CUBLAS_OP_T, CUBLAS_OP_N, e.lin.O, e.lin.N, e.lin.K, &one, P->tcw_d + e.lin.wb,
                            CUDA_R_16BF, e.lin.K, xin, CUDA_R_16BF, e.lin.K, &zero, P->lin_ws_d, CUDA_R_32F, e.lin.O,

@@ -83,3 +83,16 @@ def test_no_device_plan_refuses_to_run():
     with pytest.raises(TemcoError) as e:
         p.run(1, 1, stream=0)
     assert e.value.status == 7
+
+
+@pytest.mark.parametrize("name", ["c1", "t3", "t4"])
+def test_silu_plans(name):
+    """SiLU is fusable like ReLU -- same rewrite, groups and peak bytes."""
+    import copy
+    m = copy.deepcopy(SMALL[name]())
+    for layer in m.layers:
+        if layer.op == "relu":
+            layer.op = "silu"
+    p, o = _compare(m)
+    assert any(s["kind"] == "group" and "silu" in s["op"] for s in p.describe()["steps"]) or \
+        any(st.kind == "group" for st in o.steps)
