@@ -7,6 +7,8 @@
 
 #include <algorithm>
 #include <cfloat>
+#include <cstdint>
+#include <cstdlib>
 
 #include "kernels.h"
 
@@ -542,6 +544,93 @@ __global__ void ew_kernel(EwDesc d, RunPtrs p) {
   }
 }
 
+// bf16 NHWC, C % 8 == 0: the same per-element arithmetic as ew_kernel (same fp32 formula and
+// summation order, same rounding), 8 channels per thread through 16-byte loads / stores -- the
+// standalone BN / ReLU / SiLU / add / concat / pool steps of unfused (ablation) plans are
+// HBM-bound and ew_kernel's 2-byte accesses reach a small fraction of the bandwidth
+__device__ __forceinline__ void unpack8(const uint4& u, float* f) {
+  const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const float2 t = __bfloat1622float2(h[j]);
+    f[2 * j] = t.x;
+    f[2 * j + 1] = t.y;
+  }
+}
+
+__global__ void __launch_bounds__(256) ew_vec_kernel(EwDesc d, RunPtrs p) {
+  uint4* y = reinterpret_cast<uint4*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const int cv = d.C / 8;
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * cv;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(i % cv) * 8;
+    const int64_t pix = i / cv;
+    float v[8], u[8];
+    switch (d.kind) {
+      case EW_BN:
+        unpack8(reinterpret_cast<const uint4*>(loc_ptr(d.x[0], p))[i], u);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = p.params[d.scale + c + j] * u[j] + p.params[d.shift + c + j];
+        break;
+      case EW_RELU:
+        unpack8(reinterpret_cast<const uint4*>(loc_ptr(d.x[0], p))[i], u);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = fmaxf(u[j], 0.f);
+        break;
+      case EW_SILU:
+        unpack8(reinterpret_cast<const uint4*>(loc_ptr(d.x[0], p))[i], u);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = u[j] / (1.f + __expf(-u[j]));
+        break;
+      case EW_ADD:
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = 0.f;
+        for (int k = 0; k < d.n_in; ++k) {
+          unpack8(reinterpret_cast<const uint4*>(loc_ptr(d.x[k], p))[i], u);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[j] += u[j];
+        }
+        break;
+      case EW_CONCAT: {
+        int cc = c, k = 0;
+        while (cc >= d.xc[k]) cc -= d.xc[k++];
+        unpack8(reinterpret_cast<const uint4*>(loc_ptr(d.x[k], p))[(pix * d.xc[k] + cc) / 8], v);
+        break;
+      }
+      case EW_MAXPOOL:
+      case EW_AVGPOOL: {
+        const int wo = (int)(pix % d.Wo);
+        const int64_t t = pix / d.Wo;
+        const int ho = (int)(t % d.Ho);
+        const int n = (int)(t / d.Ho);
+        const uint4* x = reinterpret_cast<const uint4*>(loc_ptr(d.x[0], p));
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[j] = d.kind == EW_MAXPOOL ? -FLT_MAX : 0.f;
+        for (int a = 0; a < d.k; ++a) {
+          const int hi = ho * d.s - d.p + a;
+          if (hi < 0 || hi >= d.H) continue;
+          for (int b = 0; b < d.k; ++b) {
+            const int wi = wo * d.s - d.p + b;
+            if (wi < 0 || wi >= d.W) continue;
+            unpack8(x[((((int64_t)n * d.H + hi) * d.W + wi) * d.C + c) / 8], u);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[j] = d.kind == EW_MAXPOOL ? fmaxf(v[j], u[j]) : v[j] + u[j];
+          }
+        }
+        if (d.kind == EW_AVGPOOL)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[j] = v[j] / (float)(d.k * d.k);
+        break;
+      }
+    }
+    uint4 o;
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) h[j] = __floats2bfloat162_rn(v[2 * j], v[2 * j + 1]);
+    y[i] = o;
+  }
+}
+
 // ---------------------------------------------------------------------------
 // linear: SIMT tiled GEMM, 64x64 tile, 4x4 per thread
 // ---------------------------------------------------------------------------
@@ -820,8 +909,20 @@ void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   conv_small_kernel<<<grid, 256, conv_small_smem(d), s>>>(d, p, tw, th);
 }
 
+static bool ew_vec_ok(const EwDesc& d, const RunPtrs& p) {
+  if (d.kind == EW_GAP || d.C % 8 || d.y.dtype != DT_BF16 || ((uintptr_t)loc_ptr(d.y, p) & 15)) return false;
+  for (int j = 0; j < d.n_in; ++j)
+    if (d.x[j].dtype != DT_BF16 || ((uintptr_t)loc_ptr(d.x[j], p) & 15) || (d.kind == EW_CONCAT && d.xc[j] % 8))
+      return false;
+  return !getenv("TEMCO_NO_EW_VEC");
+}
+
 void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s) {
   const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.C;
+  if (ew_vec_ok(d, p)) {
+    ew_vec_kernel<<<grid_for(total / 8, 256), 256, 0, s>>>(d, p);
+    return;
+  }
   ew_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
 }
 

@@ -100,3 +100,16 @@ def test_silu_activation(name, dt):
         assert np.isfinite(y).all()
         assert _rel(y, ref) <= TOL[dt], (flags, _rel(y, ref))
     assert p.peak_internal_bytes(1) == o.peak_unfused
+
+
+@pytest.mark.parametrize("name", ["t4", "resnet18_s", "densenet121_s"])
+def test_vectorised_elementwise_bit_exact(name, monkeypatch):
+    """The 16-byte elementwise kernel (standalone BN / ReLU / add / concat / pools of
+    unfused plans) does the scalar kernel's arithmetic: identical bits."""
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_NO_FUSION, FLAG_NO_SKIPOPT
+    m = GRAPHS[name]("bf16")
+    x = W.make_input(m)
+    _, y_vec = _run(m, FLAG_NO_FUSION | FLAG_NO_SKIPOPT, x)
+    monkeypatch.setenv("TEMCO_NO_EW_VEC", "1")
+    _, y_ref = _run(m, FLAG_NO_FUSION | FLAG_NO_SKIPOPT, x)
+    assert np.array_equal(y_vec, y_ref)
