@@ -194,6 +194,8 @@ def main():
     # decomposed = neither rewrite, fusion_only = no skip optimization,
     # skipopt_only = no fusion.  Not the headline line: same metric, other plan.
     ap.add_argument("--variant", default="temco", choices=list(VARIANTS))
+    # the same network with every ReLU replaced by SiLU
+    ap.add_argument("--act", default="relu", choices=["relu", "silu"])
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     if args.impl == "reference":
@@ -210,6 +212,10 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     B = CONFIG_BATCH[args.config]
     m = W.build_config(args.config, batch=B)
+    if args.act == "silu":
+        for layer in m.layers:
+            if layer.op == "relu":
+                layer.op = "silu"
     flags = FLAG_CUDA_GRAPH | (FLAG_SIMT_ONLY if args.simt_only else 0) | VARIANTS[args.variant]
     plan = Plan(m, flags=flags)
     desc = plan.describe()
@@ -350,7 +356,7 @@ def main():
                        "peak_internal_bytes_unfused": plan.peak_internal_bytes(1),
                        "internal_memory_reduction": 1 - plan.peak_internal_bytes(0) / plan.peak_internal_bytes(1),
                        "cuda_graph": True, "kernels": "simt-only" if args.simt_only else "tcgen05+simt",
-                       "variant": args.variant},
+                       "variant": args.variant, "activation": args.act},
             "gpu_launches": desc["launches"] * args.steps,
             "e2e": {"value": ws * B / (e2e_ms / 1e3), "unit": "images/s", "api": "temco_run_host_async (pipelined H2D)",
                     "h2d_bytes_per_step": int(xh.numel() * xh.element_size()),

@@ -45,6 +45,7 @@ struct PLevel {
   std::vector<PTerm> terms;
   std::vector<double> bias;
   bool relu = false;
+  bool silu = false;           // SiLU activation of the level, only with allow_silu
   std::vector<PMember> pm;
 };
 
@@ -54,13 +55,15 @@ struct ChainParser {
   int C;
   std::set<int> visited;
   int H, W;
+  bool allow_silu = false;     // set by lowerers whose kernels apply PLevel::silu
 
   bool chain(int v, std::vector<PLevel>& out) {
     if (!members.count(v)) return false;
     visited.insert(v);
-    if (ir.nodes[v].op == OP_RELU) {
+    const int op = ir.nodes[v].op;
+    if (op == OP_RELU || (allow_silu && op == OP_SILU)) {
       if (!pre(ir.oin[v][0], out)) return false;
-      out.back().relu = true;
+      (op == OP_RELU ? out.back().relu : out.back().silu) = true;
       return true;
     }
     return pre(v, out);
@@ -155,6 +158,9 @@ struct ChainParser {
         }
         return true;
       }
+      case OP_SILU:
+        if (!allow_silu) return false;
+        [[fallthrough]];
       case OP_RELU: {
         // a previous chain value t_{l-1}: unit scale, full width, at most one
         if (sc || c0 != 0 || n.C != C || !prev.empty()) return false;

@@ -48,6 +48,7 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
   }
   const Node& cn = ir.nodes[csrc];
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, cn.H, cn.W};
+  P.allow_silu = true;   // act_apply: 1 ReLU, 2 SiLU
   P.members.erase(s.out);
   if (pool) P.members.erase(tsrc);
   std::vector<PLevel> levels;
@@ -90,7 +91,7 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
   int64_t fl_terms = 0, by_terms = 0;
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
-    d.relu[l] = L.relu ? 1 : 0;
+    d.relu[l] = L.relu ? 1 : L.silu ? 2 : 0;
     d.bias[l] = (int32_t)biases.size();
     for (int c = 0; c < d.Cpad; ++c) biases.push_back(c < C ? (float)L.bias[c] : 0.f);
     for (const PTerm& t : L.terms) {
@@ -155,6 +156,11 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
 }
 
 namespace {
+
+// level activation: 1 ReLU, 2 SiLU (x / (1 + e^-x), the SIMT kernels' formula)
+__device__ __forceinline__ float act_apply(float x, int act) {
+  return act == 2 ? x / (1.f + __expf(-x)) : fmaxf(x, 0.f);
+}
 
 __device__ __forceinline__ uint32_t s_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 
@@ -336,7 +342,7 @@ __global__ void __launch_bounds__(32 * kWarps, 1) mma_chain_kernel(const __grid_
 #pragma unroll
           for (int nb = 0; nb < CH / 8; ++nb)
 #pragma unroll
-            for (int i = 0; i < 4; ++i) D[nb][i] = fmaxf(D[nb][i], 0.f);
+            for (int i = 0; i < 4; ++i) D[nb][i] = act_apply(D[nb][i], d.relu[l]);
         }
       }
       if (POOL) {
@@ -508,7 +514,7 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
   const uint32_t* r = reinterpret_cast<const uint32_t*>(p.arena + T.r.off);
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
   const int rs = T.Rp + 8, fs = d.Cpad + 8;
-  const bool relu = d.relu[0] != 0;
+  const int relu = d.relu[0];
   const int taps = d.pool ? d.taps : 1;
   const int nch = d.Cpad / 64;
   // ldmatrix.x4 lane addressing: matrix q = lane / 8 -> (n-tile + q / 2, k half q % 2)
@@ -565,7 +571,7 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
 #pragma unroll
       for (int nt = 0; nt < 8; ++nt)
 #pragma unroll
-        for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+        for (int i = 0; i < 4; ++i) D[nt][i] = act_apply(D[nt][i], relu);
     }
     bool last = true;
     if (d.pool) {
@@ -687,7 +693,7 @@ __global__ void __launch_bounds__(32 * kL64Warps, 1) mma_lean64_kernel(const __g
     bias[nt][0] = b.x;
     bias[nt][1] = b.y;
   }
-  const bool relu = d.relu[0] != 0;
+  const int relu = d.relu[0];
   const int taps = POOL ? d.taps : 1;
   const int64_t nw = (int64_t)gridDim.x * kL64Warps;
   auto advance = [&](LeanCursor& u) {
@@ -719,7 +725,7 @@ __global__ void __launch_bounds__(32 * kL64Warps, 1) mma_lean64_kernel(const __g
 #pragma unroll
       for (int nt = 0; nt < 8; ++nt)
 #pragma unroll
-        for (int i = 0; i < 4; ++i) D[nt][i] = fmaxf(D[nt][i], 0.f);
+        for (int i = 0; i < 4; ++i) D[nt][i] = act_apply(D[nt][i], relu);
     }
     bool last = true;
     if constexpr (POOL) {

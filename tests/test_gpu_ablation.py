@@ -95,6 +95,10 @@ def test_silu_activation(name, dt):
     # SiLU is not ReLU: the plan must not silently compute max(x, 0)
     relu_ref = oracle.run_temco(oracle.plan(GRAPHS[name](dt)), x)
     assert _rel(ref, relu_ref) > 10 * TOL[dt]
+    if dt == "bf16" and name == "resnet18_s":
+        from paper_conf_icpp_songljkj0024_b200 import FLAG_NO_DEVICE, Plan
+        kernels = {s["kernel"] for s in Plan(m, flags=FLAG_NO_DEVICE).describe()["steps"]}
+        assert kernels & {"mma_lean", "mma_chain"}, kernels      # SiLU groups on the mma.sync kernels
     for flags in (0, FLAG_NO_FUSION):
         p, y = _run(m, flags, x)
         assert np.isfinite(y).all()
