@@ -237,6 +237,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   if (gap && tn.H * tn.W > 128) return false;
   if (store && C % kTcCc) return false;
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
+  P.allow_silu = true;   // d.relu[l]: 1 ReLU, 2 SiLU
   if (!store) P.members.erase(s.out);
   std::vector<PLevel> levels;
   if (!P.chain(tsrc, levels)) return false;
@@ -347,7 +348,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   };
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
-    d.relu[l] = L.relu ? 1 : 0;
+    d.relu[l] = L.relu ? 1 : L.silu ? 2 : 0;
     // pooled-member channels take no level bias before the pool: their level
     // bias (the post-BN shift) is added after pooling, in the epilogue
     std::vector<double> lb = L.bias;
@@ -656,6 +657,7 @@ struct Ring {
   }
 };
 
+template <bool SILU>
 __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
@@ -1043,7 +1045,12 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               }
             }
           }
-          const bool relu = d.relu[un.pooled ? 0 : l] != 0;
+          const int act = d.relu[un.pooled ? 0 : l];
+          if (SILU && act == 2) {   // SiLU level: applied in place, then the no-activation path
+#pragma unroll
+            for (int i = 0; i < 32; ++i) t[i] = t[i] / (1.f + __expf(-t[i]));
+          }
+          const bool relu = SILU ? act == 1 : act != 0;
           if (!last) {
             if (relu) {
 #pragma unroll
@@ -1173,7 +1180,7 @@ extern "C" void temco_debug_trace(long long* out) {
 // diagnostics: registers, max threads per block, static / max dynamic SMEM of the chain kernel
 extern "C" int temco_debug_tc_attrs(int* out) {
   cudaFuncAttributes a;
-  const cudaError_t e = cudaFuncGetAttributes(&a, tc_chain_kernel);
+  const cudaError_t e = cudaFuncGetAttributes(&a, tc_chain_kernel<false>);
   out[0] = a.numRegs;
   out[1] = a.maxThreadsPerBlock;
   out[2] = (int)a.sharedSizeBytes;
@@ -1187,7 +1194,8 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   static bool configured = false;
   static int sms = 0;
   if (!configured) {
-    cudaFuncSetAttribute(tc_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tc_chain_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tc_chain_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -1195,7 +1203,9 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   }
   const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
   // >= 114 KB of shared memory keeps one CTA per SM (each owns all 512 TMEM columns)
-  launch_pdl(tc_chain_kernel, dim3(grid), dim3(kThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
+  const bool silu = std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
+  launch_pdl(silu ? tc_chain_kernel<true> : tc_chain_kernel<false>, dim3(grid), dim3(kThreads),
+             std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }
 
 }  // namespace temco

@@ -319,6 +319,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   if (Nout % 8 || Nout > 256) return false;
   if (gap && tn.H * tn.W > 128) return false;
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
+  P.allow_silu = true;
   P.members.erase(s.out);
   std::vector<PLevel> levels;
   if (!P.chain(tsrc, levels)) return false;
@@ -428,7 +429,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   };
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
-    d.relu[l] = L.relu ? 1 : 0;
+    d.relu[l] = L.relu ? 1 : L.silu ? 2 : 0;
     // pooled-member channels take no level bias through the MMA: their level bias
     // (the post-BN shift) is added after pooling, in the epilogue
     std::vector<double> lb = L.bias;
@@ -621,6 +622,14 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
 namespace {
 using namespace ptx;
 
+// level activation: ReLU when a != 0; the SILU instantiation also takes a == 2 -> SiLU (P:L307,
+// the SIMT kernels' formula).  ReLU-only plans launch SILU = false: the epilogue code is unchanged
+template <bool SILU>
+__device__ __forceinline__ float act_w(float x, int a) {
+  if constexpr (SILU) return a == 2 ? x / (1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  else return a ? fmaxf(x, 0.f) : x;
+}
+
 __device__ __forceinline__ bool term_hits(const TcTerm& t, int c, int Cc) {
   return t.c0 < (c + 1) * Cc && t.c0 + t.C > c * Cc;
 }
@@ -715,6 +724,7 @@ __device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
   return g;
 }
 
+template <bool SILU>
 __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
@@ -1019,7 +1029,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
         const int nb = min(2, U - u0);
         for (int l = 0; l < d.n_levels; ++l) {
           const bool last = l == d.n_levels - 1;
-          const bool relu = d.relu[l] != 0;
+          const int relu = d.relu[l];   // 0 none, 1 ReLU, 2 SiLU (SILU instantiation only)
           for (int bi = 0; bi < nb; ++bi) {
             const Unit un = unit_at(d, u0 + bi);
             const int bs = (gu + bi) & 1;
@@ -1093,7 +1103,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 #pragma unroll
                   for (int i = 0; i < 8; ++i) {
                     const float x = cur[8 * qq + i] * sc + pscale * pq[i];
-                    f[i] = relu ? fmaxf(x, 0.f) : x;
+                    f[i] = act_w<SILU>(x, relu);
                   }
                   uint4 pk;
                   pk.x = pack_bf16(f[0], f[1]);
@@ -1114,7 +1124,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
                   const float x = __uint_as_float(a[i]) + bv[i];
-                  a[i] = __float_as_uint(relu ? fmaxf(x, 0.f) : x);
+                  a[i] = __float_as_uint(act_w<SILU>(x, relu));
                 }
                 tmem_st32(ta + g * 32, a);
               }
@@ -1132,7 +1142,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 #pragma unroll
                 for (int i = 0; i < 32; ++i) {
                   const float x0 = __uint_as_float(v[i]) + bv[i];
-                  const float x = relu ? fmaxf(x0, 0.f) : x0;
+                  const float x = act_w<SILU>(x0, relu);
                   red[row * 32 + ((i + row) & 31)] = x;
                 }
                 asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
@@ -1163,7 +1173,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 #pragma unroll
                   for (int i = 0; i < 8; ++i) {
                     const float x = __uint_as_float(v[8 * qq + i]) + bv[8 * qq + i];
-                    f[i] = relu ? fmaxf(x, 0.f) : x;
+                    f[i] = act_w<SILU>(x, relu);
                   }
                   uint4 pk;
                   pk.x = pack_bf16(f[0], f[1]);
@@ -1232,7 +1242,8 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   static bool configured = false;
   static int sms = 0;
   if (!configured) {
-    cudaFuncSetAttribute(tc_chain_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tc_chain_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tc_chain_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -1242,7 +1253,9 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   static const int grid_cap = getenv("TEMCO_TC_GRID") ? atoi(getenv("TEMCO_TC_GRID")) : 0;   // experiments
   if (grid_cap > 0) grid = std::min(grid, grid_cap);
   // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
-  launch_pdl(tc_chain_kernel, dim3(grid), dim3(kThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
+  const bool silu = std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
+  launch_pdl(silu ? tc_chain_kernel<true> : tc_chain_kernel<false>, dim3(grid), dim3(kThreads),
+             std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }
 
 }  // namespace wide

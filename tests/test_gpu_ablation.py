@@ -45,6 +45,7 @@ GRAPHS = {
     "t4": lambda dt: W.t4_mini_densenet(dtype=dt, batch=2),
     "resnet18_s": lambda dt: W.resnet18_cifar(batch=2, dtype=dt, height=16, width=16),
     "densenet121_s": lambda dt: W.densenet121(batch=2, dtype=dt, height=64, width=64),
+    "resnet50_s": lambda dt: W.resnet50(batch=2, dtype=dt, height=64, width=64),
 }
 TOL = {"f32": 1e-4, "bf16": 2e-2}
 
@@ -85,7 +86,7 @@ def _silu(m):
 
 
 @pytest.mark.parametrize("dt", ["f32", "bf16"])
-@pytest.mark.parametrize("name", ["c1", "t3", "t4", "resnet18_s"])
+@pytest.mark.parametrize("name", ["c1", "t3", "t4", "resnet18_s", "resnet50_s", "densenet121_s"])
 def test_silu_activation(name, dt):
     from paper_conf_icpp_songljkj0024_b200 import FLAG_NO_FUSION
     m = _silu(GRAPHS[name](dt))
@@ -95,10 +96,11 @@ def test_silu_activation(name, dt):
     # SiLU is not ReLU: the plan must not silently compute max(x, 0)
     relu_ref = oracle.run_temco(oracle.plan(GRAPHS[name](dt)), x)
     assert _rel(ref, relu_ref) > 10 * TOL[dt]
-    if dt == "bf16" and name == "resnet18_s":
+    if dt == "bf16" and name in ("resnet18_s", "resnet50_s"):
         from paper_conf_icpp_songljkj0024_b200 import FLAG_NO_DEVICE, Plan
         kernels = {s["kernel"] for s in Plan(m, flags=FLAG_NO_DEVICE).describe()["steps"]}
-        assert kernels & {"mma_lean", "mma_chain"}, kernels      # SiLU groups on the mma.sync kernels
+        assert kernels & {"mma_lean", "mma_chain"} and "tc_chain" in kernels, kernels   # SiLU on the tensor-core kernels
+        assert not any(k.startswith("simt_group") for k in kernels), kernels
     for flags in (0, FLAG_NO_FUSION):
         p, y = _run(m, flags, x)
         assert np.isfinite(y).all()
