@@ -39,6 +39,7 @@ struct PMember {               // pooled non-linear member (per-tap epilogue)
   std::vector<PTerm> terms;
   std::vector<double> bias;    // member bias (size C), scaled
   bool relu = false;
+  bool silu = false;           // only with allow_silu
 };
 
 struct PLevel {
@@ -205,10 +206,10 @@ struct ChainParser {
         m.Win = un.W;
         m.bias.assign(n.C, 0.0);
         int lin = u;
-        if (un.op == OP_RELU) {
+        if (un.op == OP_RELU || (allow_silu && un.op == OP_SILU)) {
           if (!members.count(u)) return false;
           visited.insert(u);
-          m.relu = true;
+          (un.op == OP_RELU ? m.relu : m.silu) = true;
           lin = ir.oin[u][0];
         }
         if (!linear(lin, sc, c0, un.H, un.W, m.terms, m.bias, 0)) return false;

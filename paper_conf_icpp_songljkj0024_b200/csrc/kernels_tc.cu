@@ -375,7 +375,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.ms = pm->s;
     d.mp = pm->p;
     d.mtaps = pm->k * pm->k;
-    d.mrelu = pm->relu ? 1 : 0;
+    d.mrelu = pm->relu ? 1 : pm->silu ? 2 : 0;
     d.mHin = pm->Hin;
     d.mWin = pm->Win;
     d.mt0 = j;
@@ -656,6 +656,13 @@ struct Ring {
     if (++s == n) s = 0, ph ^= 1u;
   }
 };
+
+// pooled-member activation: ReLU when a != 0; SILU instantiation: a == 2 -> SiLU
+template <bool SILU>
+__device__ __forceinline__ float act_m(float x, int a) {
+  if constexpr (SILU) return a == 2 ? x / (1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  else return a ? fmaxf(x, 0.f) : x;
+}
 
 template <bool SILU>
 __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
@@ -993,7 +1000,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
 #pragma unroll
                   for (int k = 0; k < 4; ++k) {
                     const float z = __uint_as_float(v[4 * i4 + k]) + bq[k];
-                    t[4 * i4 + k] += d.mrelu ? fmaxf(z, 0.f) : z;
+                    t[4 * i4 + k] += act_m<SILU>(z, d.mrelu);
                   }
                 }
               }
@@ -1016,7 +1023,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 float z = t[i] * sc;
                 if (d.mpool == 1) {
                   z += bq[k];
-                  z = d.mrelu ? fmaxf(z, 0.f) : z;
+                  z = act_m<SILU>(z, d.mrelu);
                 }
                 t[i] = z + pscale * pq[k];
               }
@@ -1203,7 +1210,7 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   }
   const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);
   // >= 114 KB of shared memory keeps one CTA per SM (each owns all 512 TMEM columns)
-  const bool silu = std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
+  const bool silu = d.mrelu == 2 || std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
   launch_pdl(silu ? tc_chain_kernel<true> : tc_chain_kernel<false>, dim3(grid), dim3(kThreads),
              std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }

@@ -457,7 +457,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
     d.ms = pm->s;
     d.mp = pm->p;
     d.mtaps = pm->k * pm->k;
-    d.mrelu = pm->relu ? 1 : 0;
+    d.mrelu = pm->relu ? 1 : pm->silu ? 2 : 0;
     d.mHin = pm->Hin;
     d.mWin = pm->Win;
     d.mt0 = j;
@@ -722,6 +722,13 @@ __device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
     g.w0 = (rem % d.nwb) * d.tw;
   }
   return g;
+}
+
+// pooled-member activation: ReLU when a != 0; SILU instantiation: a == 2 -> SiLU
+template <bool SILU>
+__device__ __forceinline__ float act_m(float x, int a) {
+  if constexpr (SILU) return a == 2 ? x / (1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  else return a ? fmaxf(x, 0.f) : x;
 }
 
 template <bool SILU>
@@ -1078,7 +1085,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   for (int k = 0; k < 4; ++k) {
                     const int i = 4 * i4 + k;
                     float x = __uint_as_float(v[i]) + bq[k];
-                    x = d.mrelu ? fmaxf(x, 0.f) : x;
+                    x = act_m<SILU>(x, d.mrelu);
                     if (d.mpool == 1)
                       cur[i] = valid ? fmaxf(cur[i], x) : cur[i];
                     else
@@ -1253,7 +1260,7 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   static const int grid_cap = getenv("TEMCO_TC_GRID") ? atoi(getenv("TEMCO_TC_GRID")) : 0;   // experiments
   if (grid_cap > 0) grid = std::min(grid, grid_cap);
   // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
-  const bool silu = std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
+  const bool silu = d.mrelu == 2 || std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
   launch_pdl(silu ? tc_chain_kernel<true> : tc_chain_kernel<false>, dim3(grid), dim3(kThreads),
              std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }
