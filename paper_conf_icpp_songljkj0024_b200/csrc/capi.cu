@@ -291,9 +291,7 @@ void lower(temco_plan_s* P) {
       }
       if (mma_ok && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
           mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma) &&
-          ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")) ||
-           std::any_of(e.mma.relu, e.mma.relu + e.mma.n_levels, [](int32_t a) { return a == 2; }))) {
-        // (SiLU levels: the tcgen05 chain kernels apply ReLU only, so mma.sync rather than the interpreter)
+          ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
         e.kind = K_GROUP_MMA;
         e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
         e.launches = 1;

@@ -157,9 +157,9 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
 
 namespace {
 
-// level activation: 1 ReLU, 2 SiLU (x / (1 + e^-x), the SIMT kernels' formula)
+// level activation: 1 ReLU, 2 SiLU (x / (1 + e^-x) with the fast approximate division: bf16 outputs)
 __device__ __forceinline__ float act_apply(float x, int act) {
-  return act == 2 ? x / (1.f + __expf(-x)) : fmaxf(x, 0.f);
+  return act == 2 ? __fdividef(x, 1.f + __expf(-x)) : fmaxf(x, 0.f);
 }
 
 __device__ __forceinline__ uint32_t s_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }

@@ -622,11 +622,11 @@ bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char*
 namespace {
 using namespace ptx;
 
-// level activation: ReLU when a != 0; the SILU instantiation also takes a == 2 -> SiLU (P:L307,
-// the SIMT kernels' formula).  ReLU-only plans launch SILU = false: the epilogue code is unchanged
+// level activation: ReLU when a != 0; the SILU instantiation also takes a == 2 -> SiLU (
+// fast approximate division, bf16 outputs).  ReLU-only plans launch SILU = false: epilogue unchanged
 template <bool SILU>
 __device__ __forceinline__ float act_w(float x, int a) {
-  if constexpr (SILU) return a == 2 ? x / (1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  if constexpr (SILU) return a == 2 ? __fdividef(x, 1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
   else return a ? fmaxf(x, 0.f) : x;
 }
 
@@ -727,7 +727,7 @@ __device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
 // pooled-member activation: ReLU when a != 0; SILU instantiation: a == 2 -> SiLU
 template <bool SILU>
 __device__ __forceinline__ float act_m(float x, int a) {
-  if constexpr (SILU) return a == 2 ? x / (1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  if constexpr (SILU) return a == 2 ? __fdividef(x, 1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
   else return a ? fmaxf(x, 0.f) : x;
 }
 
