@@ -41,3 +41,26 @@ def test_bf16_full_configs_never_fall_back_to_the_interpreter():
     for name in ("resnet18_cifar", "resnet50", "vgg16_cp", "densenet121"):
         ks = _kernels(W.build_config(name))
         assert ks["simt_group"] == 0 and ks["simt_group_gap"] == 0, (name, ks)
+
+
+def _silu(m):
+    for layer in m.layers:
+        if layer.op == "relu":
+            layer.op = "silu"
+    return m
+
+
+def test_silu_full_configs_on_tensor_core_kernels():
+    """SiLU plans of the bench configs (bench.py --act silu) lower every fused group to
+    a tensor-core kernel, like the ReLU plans; the small SiLU parity cases of
+    test_gpu_ablation.py cover the kernel families they launch."""
+    small = collections.Counter()
+    for m in (W.resnet18_cifar(batch=2, dtype="bf16", height=16, width=16),
+              W.resnet50(batch=2, dtype="bf16", height=64, width=64),
+              W.densenet121(batch=2, dtype="bf16", height=64, width=64)):
+        small.update(_kernels(_silu(m)))
+    for name in ("resnet18_cifar", "resnet50", "vgg16_cp", "densenet121"):
+        k = _kernels(_silu(W.build_config(name)))
+        assert not any(x.startswith("simt_group") for x in k), (name, k)
+        if name != "vgg16_cp":
+            assert set(k) <= set(small), (name, set(k) - set(small))
