@@ -17,6 +17,7 @@
 #include "mma_chain.h"
 #include "tc.h"
 #include "tc_wide.h"
+#include "pair.h"
 
 #include <cublas_v2.h>
 
@@ -37,7 +38,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR };
 
 struct StepExec {
   int kind = K_NONE;
@@ -47,6 +48,7 @@ struct StepExec {
   GroupDesc grp{};
   TcChainDesc tc{};
   wide::TcChainDesc tcw{};
+  pair::PairDesc pr{};
   ConvTcDesc ctc{};
   MmaChainDesc mma{};
   RankConvDesc rk{};
@@ -304,6 +306,14 @@ void lower(temco_plan_s* P) {
         e.launches = 1;
         continue;
       }
+      // full-width residual chains with an fconv root: the CTA-pair tcgen05 kernel
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+          pair::pair_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.pr)) {
+        e.kind = K_GROUP_PAIR;
+        e.kernel = "tc_pair";
+        e.launches = 1;
+        continue;
+      }
       if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
           tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tc)) {
         e.kind = K_GROUP_TC;
@@ -551,6 +561,13 @@ std::string make_json(const temco_plan_s* P) {
     o << ",\"inputs\":";
     json_ints(o, s.in);
     o << ",\"bytes\":" << ir.size(s.out);
+    // shapes [C, H, W] of the step's inputs and output (per image)
+    o << ",\"in_chw\":[";
+    for (size_t i = 0; i < s.in.size(); ++i) {
+      const Node& x = ir.nodes[s.in[i]];
+      o << (i ? "," : "") << "[" << x.C << "," << x.H << "," << x.W << "]";
+    }
+    o << "],\"out_chw\":[" << v.C << "," << v.H << "," << v.W << "]";
     if (!P->exec.empty()) {
       const StepExec& e = P->exec[t];
       o << ",\"kernel\":\"" << e.kernel << "\",\"flops\":" << e.flops << ",\"io_bytes\":" << e.io_bytes
@@ -565,6 +582,10 @@ std::string make_json(const temco_plan_s* P) {
           << e.tcw.n_prod << ",\"n_mma\":" << e.tcw.n_mma << ",\"units\":" << e.tcw.units << ",\"stages\":" << e.tcw.stages
           << ",\"resident\":" << e.tcw.resident << ",\"smem\":" << e.tcw.smem_bytes << ",\"tmem\":" << e.tcw.tmem_cols
           << ",\"ntiles\":" << e.tcw.ntiles << ",\"Cc\":" << e.tcw.Cc << ",\"levels\":" << e.tcw.n_levels << "}";
+      if (e.kind == K_GROUP_PAIR)
+        o << ",\"alg_flops\":" << e.pr.alg_flops << ",\"alg_bytes\":" << e.pr.alg_bytes << ",\"tc\":{\"variant\":\"pair\",\"stages\":"
+          << e.pr.stages << ",\"smem\":" << e.pr.smem_bytes << ",\"ntiles\":" << e.pr.ntiles << ",\"units\":" << e.pr.nunits
+          << ",\"levels\":" << e.pr.n_levels << ",\"terms\":" << e.pr.n_terms << "}";
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_CONV_RK) o << ",\"alg_flops\":" << e.rk.alg_flops << ",\"alg_bytes\":" << e.rk.alg_bytes;
       if (e.kind == K_GROUP_CAT) o << ",\"alg_flops\":" << e.cat.alg_flops << ",\"alg_bytes\":" << e.cat.alg_bytes;
@@ -666,6 +687,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
       case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
+      case K_GROUP_PAIR: pair::launch_pair_chain(e.pr, rp, st); break;
       case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
       case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
       case K_GROUP_CAT: launch_mma_cat(e.cat, P->tcw_d, rp, st); break;
@@ -808,6 +830,13 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
     }
     if (!wide::tc_finalize(P->exec.size(), [&](size_t i) -> wide::TcChainDesc* {
           return P->exec[i].kind == K_GROUP_TCW ? &P->exec[i].tcw : nullptr;
+        }, P->arena_d, P->tcw_d, terr)) {
+      free_device(P);
+      delete P;
+      return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
+    }
+    if (!pair::pair_finalize(P->exec.size(), [&](size_t i) -> pair::PairDesc* {
+          return P->exec[i].kind == K_GROUP_PAIR ? &P->exec[i].pr : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {
       free_device(P);
       delete P;

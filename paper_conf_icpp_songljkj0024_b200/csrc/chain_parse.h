@@ -40,6 +40,7 @@ struct PMember {               // pooled non-linear member (per-tap epilogue)
   std::vector<double> bias;    // member bias (size C), scaled
   bool relu = false;
   bool silu = false;           // only with allow_silu
+  std::vector<double> post_scale;   // SiLU member: the post-pool BN scale, applied after the pool
 };
 
 struct PLevel {
@@ -212,7 +213,12 @@ struct ChainParser {
           (un.op == OP_RELU ? m.relu : m.silu) = true;
           lin = ir.oin[u][0];
         }
-        if (!linear(lin, sc, c0, un.H, un.W, m.terms, m.bias, 0)) return false;
+        // a post-pool scale s folds into the member only through a positively
+        // homogeneous activation (relu(s y) = s relu(y), s > 0); SiLU is not, so
+        // its member keeps s aside: s * pool(silu(L r + b)) (+ the level shift)
+        const bool keep_scale = m.silu && sc;
+        if (keep_scale) m.post_scale = *sc;
+        if (!linear(lin, keep_scale ? nullptr : sc, c0, un.H, un.W, m.terms, m.bias, 0)) return false;
         L.pm.push_back(std::move(m));
         return true;
       }

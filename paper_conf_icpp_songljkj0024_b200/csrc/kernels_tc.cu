@@ -289,6 +289,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d.Wo = tn.W;
   d.spatial = mixed ? 1 : 0;
   d.post = -1;
+  d.postsc = -1;
   if (d.spatial) {
     d.tw = std::min(tn.W, 128);
     d.th = std::min(tn.H, 128 / d.tw);
@@ -361,6 +362,13 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
       while (params.size() % 4) params.push_back(0.f);
       d.post = (int64_t)params.size();
       for (double x : post) params.push_back((float)x);
+      if (!pm->post_scale.empty()) {
+        std::vector<double> ps(post.size(), 1.0);
+        for (int c = 0; c < pm->C; ++c) ps[c] = pm->post_scale[c];
+        while (params.size() % 4) params.push_back(0.f);
+        d.postsc = (int64_t)params.size();
+        for (double x : ps) params.push_back((float)x);
+      }
     }
     d.lbias[l] = push_f32(params, lb, d.Cpad);
     for (const PTerm& t : L.terms)
@@ -987,10 +995,23 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
               uint32_t v[32];
               tmem_ld32(ta + r * d.Cc, v);
               tmem_wait_ld();
-              if (d.mpool == 1) {
+              if (d.mpool == 1 && !(SILU && d.mrelu == 2)) {
+                // monotone activation: max of the raw accumulators, bias + act after the pool
                 if (valid) {
 #pragma unroll
                   for (int i = 0; i < 32; ++i) t[i] = fmaxf(t[i], __uint_as_float(v[i]));
+                }
+              } else if (d.mpool == 1) {
+                // SiLU is not monotone (minimum near -1.28): max over act(acc + b) per tap
+                if (valid) {
+#pragma unroll
+                  for (int i4 = 0; i4 < 8; ++i4) {
+                    const float4 bb = __ldg(b4 + i4);
+                    const float bq[4] = {bb.x, bb.y, bb.z, bb.w};
+#pragma unroll
+                    for (int k = 0; k < 4; ++k)
+                      t[4 * i4 + k] = fmaxf(t[4 * i4 + k], act_m<SILU>(__uint_as_float(v[4 * i4 + k]) + bq[k], d.mrelu));
+                  }
                 }
               } else {
 #pragma unroll
@@ -1013,19 +1034,22 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
             const float4* p4 = reinterpret_cast<const float4*>(p.params + (d.post >= 0 ? d.post : d.mbias) + col0);
             const float pscale = d.post >= 0 ? 1.f : 0.f;
             const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
+            const float4* s4 = reinterpret_cast<const float4*>(p.params + (d.postsc >= 0 ? d.postsc : d.mbias) + col0);
 #pragma unroll
             for (int i4 = 0; i4 < 8; ++i4) {
               const float4 bb = __ldg(b4 + i4), pp = __ldg(p4 + i4);
+              const float4 ss = d.postsc >= 0 ? __ldg(s4 + i4) : make_float4(1.f, 1.f, 1.f, 1.f);
               const float bq[4] = {bb.x, bb.y, bb.z, bb.w}, pq[4] = {pp.x, pp.y, pp.z, pp.w};
+              const float sq[4] = {ss.x, ss.y, ss.z, ss.w};
 #pragma unroll
               for (int k = 0; k < 4; ++k) {
                 const int i = 4 * i4 + k;
                 float z = t[i] * sc;
-                if (d.mpool == 1) {
+                if (d.mpool == 1 && !(SILU && d.mrelu == 2)) {
                   z += bq[k];
                   z = act_m<SILU>(z, d.mrelu);
                 }
-                t[i] = z + pscale * pq[k];
+                t[i] = z * sq[k] + pscale * pq[k];
               }
             }
           } else if (d.exp & 1) {

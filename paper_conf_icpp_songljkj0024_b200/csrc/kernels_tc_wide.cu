@@ -370,6 +370,7 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d.Wo = tn.W;
   d.spatial = mixed ? 1 : 0;
   d.post = -1;
+  d.postsc = -1;
   if (d.spatial) {
     d.tw = std::min(tn.W, 128);
     d.th = std::min(tn.H, 128 / d.tw);
@@ -442,6 +443,13 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
       while (params.size() % 4) params.push_back(0.f);
       d.post = (int64_t)params.size();
       for (double x : post) params.push_back((float)x);
+      if (!pm->post_scale.empty()) {
+        std::vector<double> ps(post.size(), 1.0);
+        for (int c = 0; c < pm->C; ++c) ps[c] = pm->post_scale[c];
+        while (params.size() % 4) params.push_back(0.f);
+        d.postsc = (int64_t)params.size();
+        for (double x : ps) params.push_back((float)x);
+      }
     }
     d.boff[l] = push_bias(tcw, lb, 0, d.Cpad);
     d.lbias[l] = push_f32(params, lb, d.Cpad);
@@ -1101,6 +1109,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                 const float sc = d.mpool == 2 ? 1.f / (float)d.mtaps : 1.f;
                 const float4* pv4 = reinterpret_cast<const float4*>(p.params + (d.post >= 0 ? d.post : d.mbias) + un.c * Cc + c_lo);
                 const float pscale = d.post >= 0 ? 1.f : 0.f;
+                const float* psc = p.params + (d.postsc >= 0 ? d.postsc : 0) + un.c * Cc + c_lo;
                 const int ch0 = c_lo / 8;
 #pragma unroll
                 for (int qq = 0; qq < 4; ++qq) {
@@ -1109,7 +1118,8 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
                   const float pq[8] = {pa.x, pa.y, pa.z, pa.w, pb2.x, pb2.y, pb2.z, pb2.w};
 #pragma unroll
                   for (int i = 0; i < 8; ++i) {
-                    const float x = cur[8 * qq + i] * sc + pscale * pq[i];
+                    const float ms = d.postsc >= 0 ? __ldg(psc + 8 * qq + i) : 1.f;
+                    const float x = cur[8 * qq + i] * sc * ms + pscale * pq[i];
                     f[i] = act_w<SILU>(x, relu);
                   }
                   uint4 pk;

@@ -1,0 +1,72 @@
+// tcgen05 CTA-pair fused restore-chain kernel (kernels_pair.cu): lowering + launch interface.
+//
+// One fused group (Listing 1, P:L321-333 add/concat merges; reading R12)
+// whose restored tensor parses into a level chain (chain_parse.h)
+//     t_1 = act_1( sum_{j in 1} Lhat_j r_j + b_1 )
+//     t_l = act_l( sum_{j in l} Lhat_j r_j + b_l + t_{l-1} )      l = 2..D
+//     out = F t_D                                                  (the next fconv)
+// with every term spanning the whole restored width C (the ResNet residual
+// chains: skip restores and the block's own lconv, P:L263 / Fig. 8) and the
+// fconv as root.  A 2-CTA cluster runs cta_group::2 MMAs with M = 256 pixels
+// (128 per CTA): each SM stages its own pixels' reduced inputs and HALF of each
+// 128-channel weight unit.  Every level's product a_l = sum_j Lhat_j r_j goes to
+// a FRESH TMEM accumulator (B rotating buffers), and the epilogue keeps t in
+// registers (t = act(t + a_l + b_l)), so no MMA ever waits for an epilogue
+// result: the tensor pipe only waits for a free buffer, B-1 levels later.
+// After the last level the epilogue writes bf16 P = t_D into shared memory and
+// out += P F_u^T accumulates over the 128-channel units in its own TMEM region.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <functional>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "device.h"
+#include "planner.h"
+
+namespace temco {
+namespace pair {
+
+constexpr int kPairMaxTerms = 16;
+constexpr int kPairMaxLevels = 16;
+constexpr int kPairWu = 128;           // restored channels per unit (MMA N of the restore GEMM)
+
+struct PairTerm {
+  alignas(64) unsigned char amap[128];   // r_j [npix x R] bf16, box {aw, 128}
+  alignas(64) unsigned char wmap[128];   // Lhat_j [Cpad x Rw] bf16, box {aw, 64} (this CTA's half of a unit)
+  Loc r;                                 // reduced input (arena)
+  int32_t R, aw, natoms, Rw;             // rank, K atom width (16/32/64), atoms, packed row length
+  int64_t w;                             // tc weight pool offset (elements)
+};
+
+struct PairDesc {
+  PairTerm term[kPairMaxTerms];
+  alignas(64) unsigned char fmap[128];   // F [Np x Cpad] bf16, box {64, Np/2}
+  int32_t n_terms, n_levels;
+  int32_t lvl_end[kPairMaxLevels];       // terms [lvl_end[l-1], lvl_end[l]) belong to level l
+  int32_t act[kPairMaxLevels];           // 0 none, 1 ReLU, 2 SiLU
+  int64_t lbias;                         // params offset: fp32 [n_levels][Cpad] level biases
+  int32_t C, Cpad, nunits;               // restored width, padded to 128, 128-channel units
+  int32_t nbuf;                          // rotating level accumulators (TMEM columns [0, 128 nbuf))
+  int32_t Nout, Np;                      // fconv outputs, padded to 16
+  int64_t npix;                          // pixels (rows of r_j and y)
+  int32_t ntiles;                        // 256-pixel pair tiles
+  Loc y;                                 // output [npix x Nout] bf16 (arena)
+  int64_t F;                             // tc weight pool offset of F
+  int32_t stages, smem_bytes, bias_bytes;
+  int32_t silu;                          // some level is SiLU: SILU kernel instantiation
+  int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
+};
+
+bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
+                      std::vector<float>& params, PairDesc& d);
+bool pair_finalize(size_t n, const std::function<PairDesc*(size_t)>& get, char* arena, uint16_t* tcw,
+                   std::string& err);
+void launch_pair_chain(const PairDesc& d, const RunPtrs& p, cudaStream_t s);
+
+}  // namespace pair
+}  // namespace temco

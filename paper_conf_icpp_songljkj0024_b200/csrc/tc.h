@@ -115,6 +115,7 @@ struct TcChainDesc {
   int32_t npc, mpool, mk, ms, mp, mtaps, mrelu, mt0, mt1, mHin, mWin;
   int32_t tpu, ntg, ubuf;                // ubuf = TMEM columns of one accumulator slot (tpu * Cc)
   int64_t post;                          // params offset of the post-pool shift, -1 none
+  int64_t postsc;                        // params offset of the post-pool scale (SiLU members), -1 none
   int64_t F;                             // tc weight pool offset of F
   Loc y;                                 // output [npix, Nout] bf16, [N, C] for GAP, [npix, C] for store
   // accumulator slots (TMEM ring, one per unit-level) and output buffers

@@ -129,6 +129,7 @@ struct TcChainDesc {
   int32_t npc, mpool, mk, ms, mp, mtaps, mrelu, mt0, mt1, mHin, mWin;
   int32_t tpu, ntg, ubuf;                // ubuf = TMEM columns of one unit buffer
   int64_t post;                          // params offset of the post-pool shift, -1 none
+  int64_t postsc;                        // params offset of the post-pool scale (SiLU members), -1 none
   int64_t F;                             // tc weight pool offset of F
   int64_t Fb;                            // unused (fconv factors carry no bias)
   Loc y;                                 // output [npix, Nout] bf16, or [N, C] for GAP

@@ -1,0 +1,5 @@
+TEMCO_LIB=build/exp/libtemco_trace.so timeout 120 python scripts/pair_prof.py resnet50 > gpurun_out/r2_pprof.log 2>&1
+cat gpurun_out/r2_pprof.log
+timeout 300 python -m pytest tests/test_gpu_parity.py -x -q -k "bf16_mode or full_config" 2>&1 | tail -2
+timeout 120 python scripts/step_profile.py resnet50 30 > gpurun_out/r2_pair_step_resnet50.log 2>&1
+head -30 gpurun_out/r2_pair_step_resnet50.log
