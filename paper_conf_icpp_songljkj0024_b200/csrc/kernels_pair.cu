@@ -16,8 +16,8 @@
 // and after the last unit out -> bf16 -> global.  The C-wide t never reaches
 // global memory.
 //
-// Warp roles (18 warps): 0 TMA producer (both CTAs), 1 TMEM allocator (both) and
-// MMA issuer (leader CTA), 2-17 epilogue (both).  Barriers the issuer waits on
+// Warp roles (18 warps): 0-15 epilogue (both CTAs), 16 TMA producer (both), 17 TMEM
+// allocator (both) and MMA issuer (leader CTA).  Barriers the issuer waits on
 // live in the leader CTA (peer arrivals through shared::cluster addresses);
 // commits are multicast to both CTAs.
 #include <cuda.h>
@@ -54,10 +54,13 @@ int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
 }
 
 constexpr int kSlotA = 16384;            // 128 rows x 64 bf16 (r atom; or an F atom of Np/2 rows)
-constexpr int kSlotB = 8192;             // 64 rows x 64 bf16 (this CTA's half of a unit's Lhat atom)
-constexpr int kSlot = kSlotA + kSlotB;
-constexpr int kPBytes = 128 * kPairWu * 2;   // P: two SW128 atoms of 128 x 64
+constexpr int kSlotB = 8192;             // 64 rows x 64 bf16: this CTA's half of one unit's Lhat atom
+constexpr int kSlotC = 2048;             // 64 rows x 16 bf16 (bias-MMA groups: this CTA's half of a level bias atom)
+// ring stage: A + B for both units of a pair (+ C for both with bias-MMA): PairDesc::slot bytes
+constexpr int kOnesBytes = 4096;         // 128 rows x 16 bf16 "ones" A tile of the bias MMA
+constexpr int kPBytes = 128 * kPairWu * 2;   // P of one unit: two SW128 atoms of 128 x 64
 constexpr int kBarBytes = 1024;
+constexpr int kChunk = 2;                // ring stages of one level consumed per (u0 pass, u1 pass)
 
 }  // namespace
 
@@ -135,22 +138,69 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     d.lvl_end[l] = j;
   }
   d.n_terms = j;
-  int natoms = 0;
-  for (int i = 0; i < j; ++i) natoms += d.term[i].natoms;
-  if (natoms > 64) return false;   // the kernel's per-unit atom program holds 64 entries
+  // per-pair atom program (identical for every unit pair), in the launch parameters so the
+  // issuer's loop state stays warp-uniform (uniform registers, no per-MMA broadcasts)
+  {
+    int n = 0, jj = 0;
+    for (int l = 0; l < d.n_levels; ++l) {
+      const int n0 = n;
+      for (; jj < d.lvl_end[l]; ++jj) {
+        const PairTerm& T = d.term[jj];
+        for (int a = 0; a < T.natoms; ++a, ++n) {
+          if (n >= kPairMaxAtoms) return false;
+          const int nk = std::min(T.aw / 16, (T.R - a * T.aw + 15) / 16);
+          d.prog[n][0] = (uint32_t)jj | ((uint32_t)T.aw << 8) | ((uint32_t)nk << 16) | ((n == n0 ? 1u : 0u) << 24) |
+                         ((l == 0 ? 4u : 0u) << 24) | ((uint32_t)l << 28);
+          d.prog[n][1] = (uint32_t)(a * T.aw);
+        }
+      }
+      d.prog[n - 1][0] |= 2u << 24;   // last atom of the level
+    }
+    d.prog[n - 1][0] |= 8u << 24;     // last atom of the program
+    d.n_prog = n;
+  }
   std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
   for (int o = 0; o < Nout; ++o)
     for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
   d.F = push_bf16(tcw, f);
   d.alg_flops = flops + d.npix * 2LL * Nout * C;
   d.alg_bytes = bytes + d.npix * 2LL * Nout;
+  // small-rank groups (every level K <= 64: the epilogue, not the tensor core, bounds them)
+  // add the level bias through the tensor core: one K=16 MMA of a constant ones tile times
+  // [hi(b), lo(b)] bf16 columns (error ~2^-16 |b|), so the epilogue does no bias work
+  {
+    int kmax = 0;
+    for (int l = 0, jj = 0; l < d.n_levels; ++l) {
+      int k = 0;
+      for (; jj < d.lvl_end[l]; ++jj) k += d.term[jj].R;
+      kmax = std::max(kmax, k);
+    }
+    d.bias_mma = (kmax <= 64 && !getenv("TEMCO_PAIR_NO_BIASMMA")) ? 1 : 0;
+  }
+  if (d.bias_mma) {
+    std::vector<float> bm((size_t)d.n_levels * d.Cpad * 16, 0.f);
+    for (int l = 0; l < d.n_levels; ++l)
+      for (int c = 0; c < C; ++c) {
+        const float x = (float)levels[l].bias[c];
+        uint32_t u;
+        memcpy(&u, &x, 4);
+        u &= 0xFFFF0000u;   // hi: truncated to bf16 exactly; lo = remainder (rounded to bf16 at upload)
+        float hi;
+        memcpy(&hi, &u, 4);
+        bm[((size_t)l * d.Cpad + c) * 16 + 0] = hi;
+        bm[((size_t)l * d.Cpad + c) * 16 + 1] = x - hi;
+      }
+    d.bmat = push_bf16(tcw, bm);
+  }
   // level biases live in shared memory (fp32 [n_levels][Cpad]): L1 is ~empty next to
   // 200+ KB of shared memory, so per-level global bias loads would each cost an L2 trip
   d.bias_bytes = (d.n_levels * d.Cpad * 4 + 1023) / 1024 * 1024;
-  const int budget = 227 * 1024 - 1024 /*align*/ - kBarBytes - kPBytes - d.bias_bytes;
-  d.stages = std::min(8, budget / kSlot);
-  if (d.stages < 3) return false;
-  d.smem_bytes = 1024 + d.stages * kSlot + kPBytes + d.bias_bytes + kBarBytes;
+  if (d.bias_mma) d.bias_bytes = 0;
+  const int budget = 227 * 1024 - 1024 /*align*/ - kBarBytes - 2 * kPBytes - d.bias_bytes - kOnesBytes;
+  d.slot = kSlotA + 2 * kSlotB + (d.bias_mma ? 2 * kSlotC : 0);
+  d.stages = std::min(8, budget / d.slot);
+  if (d.stages < 2 * kChunk) return false;
+  d.smem_bytes = 1024 + d.stages * d.slot + 2 * kPBytes + d.bias_bytes + kOnesBytes + kBarBytes;
   return true;
 }
 
@@ -193,6 +243,10 @@ bool pair_finalize(size_t n, const std::function<PairDesc*(size_t)>& get, char* 
         return false;
       }
     }
+    if (d->bias_mma && !make(d->bmap, tcw + d->bmat, 16, (uint64_t)d->n_levels * d->Cpad, 64, 16)) {
+      err = "cuTensorMapEncodeTiled failed (pair bias)";
+      return false;
+    }
     if (!make(d->fmap, tcw + d->F, (uint64_t)d->Cpad, (uint64_t)d->Np, (uint32_t)(d->Np / 2), 64)) {
       err = "cuTensorMapEncodeTiled failed (pair F)";
       return false;
@@ -208,44 +262,80 @@ namespace {
 using namespace ptx;
 
 #ifdef TEMCO_TRACE
-// experiment builds only: cycle accounting of pair 0's MMA issuer and of one epilogue warp
-// [launch][0 issuer total, 1 wait full, 2 wait acc_empty, 3 wait p_full, 4 wait out_empty, 5 mma issue,
-//          6 commits, 8 epi total, 9 wait acc_full, 10 wait p_empty, 11 tmem ld+arrive, 12 math,
-//          13 wait out_full, 14 P write, 15 out store]
-__device__ unsigned long long g_pprof[64][16];
-__device__ int g_pprof_n;
-__device__ int g_pdbg;   // 1: producer issues no TMA (stale operands; timing experiment only)
-#define PT0() (_t0 = clock64())
-#define PTADD(i) (_acc[i] += clock64() - _t0)
-#define PTDECL() long long _t0 = 0, _acc[16] = {0}; const long long _start = clock64()
-#define PTSAVE(lo, hi, tot)                                                       \
-  if (blockIdx.x == 0) {                                                          \
-    const int n_ = atomicAdd(&g_pprof_n, 0);                                      \
-    if (n_ < 64) {                                                                \
-      g_pprof[n_][tot] = clock64() - _start;                                      \
-      for (int i_ = lo; i_ < hi; ++i_) g_pprof[n_][i_] = _acc[i_];                \
-    }                                                                             \
-  }
+// experiment builds only: event timeline of CTA 0 (rows: see scripts/pair_timeline.py)
+__device__ long long g_ev[12][512];
+__device__ int g_ev_on, g_launch;
+__device__ int g_pdbg;   // timing experiments: 1 = producer issues no TMA, 2 = epilogue skips TMEM / math
+#define EVDECL() int _evn[12] = {0}; const bool _evon = blockIdx.x == 0 && g_launch == g_ev_on
+#define EV(row)                                                                                   \
+  do {                                                                                            \
+    if (_evon && _evn[row] < 512) g_ev[row][_evn[row]++] = clock64();                             \
+  } while (0)
 #else
-#define PT0() ((void)0)
-#define PTADD(i) ((void)0)
-#define PTDECL() ((void)0)
-#define PTSAVE(lo, hi, tot) ((void)0)
+#define EVDECL() ((void)0)
+#define EV(row) ((void)0)
 #endif
 
 constexpr int kWarps = 18;
 constexpr int kThreads = 32 * kWarps;
-constexpr int kProdWarp = 0, kMmaWarp = 1, kEpiWarp0 = 2;
+// epilogue warps first: the SM sub-partition arbiter favours the highest warp id, so the
+// single-thread producer and MMA issuer (warps 16, 17) win issue slots over the 16
+// epilogue warps sharing their sub-partitions
+constexpr int kEpiWarp0 = 0, kProdWarp = 16, kMmaWarp = 17;
 constexpr int kEpiWarps = 16;
-
-template <bool SILU>
-__device__ __forceinline__ float act_p(float x, int a) {
-  if constexpr (SILU) return a == 2 ? __fdividef(x, 1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
-  else return a ? fmaxf(x, 0.f) : x;
-}
 
 __device__ __forceinline__ int atom_steps(const PairTerm& T, int a) {   // K=16 steps of atom a
   return min(T.aw / 16, (T.R - a * T.aw + 15) / 16);
+}
+
+__device__ __forceinline__ void add2(float& a0, float& a1, float b0, float b1) {   // packed FADD2
+  asm("{\n.reg .b64 x, y;\nmov.b64 x, {%0, %1};\nmov.b64 y, {%2, %3};\nadd.rn.f32x2 x, x, y;\nmov.b64 {%0, %1}, x;\n}\n"
+      : "+f"(a0), "+f"(a1)
+      : "f"(b0), "f"(b1));
+}
+
+__device__ __forceinline__ uint32_t pack_relu(float lo, float hi) {   // bf16x2(max(lo, 0), max(hi, 0))
+  uint32_t r;
+  asm("cvt.rn.relu.bf16x2.f32 %0, %2, %1;" : "=r"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+
+template <bool SILU>
+__device__ __forceinline__ float silu_or(float x, int act) {
+  if constexpr (SILU) return act == 2 ? __fdividef(x, 1.f + __expf(-x)) : x;
+  else return x;
+}
+
+// One level of one unit for this thread's 32 channels: t (bf16x2, 16 words) =
+// act(a (+ bias) (+ t)), a = the level accumulator from TMEM (fp32).  t is held in
+// bf16 between levels -- the precision the unfused bf16 model stores every
+// intermediate tensor in -- and each level rounds once.
+template <bool SILU>
+__device__ __forceinline__ void level_math(uint32_t (&t)[16], const uint32_t (&v)[32], bool first, int act,
+                                           const float* bias) {
+  float z[32];
+#pragma unroll
+  for (int i = 0; i < 32; ++i) z[i] = __uint_as_float(v[i]);
+  if (bias) {
+    const float4* b4 = reinterpret_cast<const float4*>(bias);
+#pragma unroll
+    for (int i4 = 0; i4 < 8; ++i4) {
+      const float4 bb = b4[i4];   // broadcast LDS.128
+      add2(z[4 * i4], z[4 * i4 + 1], bb.x, bb.y);
+      add2(z[4 * i4 + 2], z[4 * i4 + 3], bb.z, bb.w);
+    }
+  }
+  if (!first) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) add2(z[2 * i], z[2 * i + 1], __uint_as_float(t[i] << 16), __uint_as_float(t[i] & 0xFFFF0000u));
+  }
+  if (act == 1) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) t[i] = pack_relu(z[2 * i], z[2 * i + 1]);
+  } else {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) t[i] = pack_bf16(silu_or<SILU>(z[2 * i], act), silu_or<SILU>(z[2 * i + 1], act));
+  }
 }
 
 template <bool SILU>
@@ -253,47 +343,29 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     pair_chain_kernel(const __grid_constant__ PairDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
-  const int S = d.stages, NB = d.nbuf;
+  const int S = d.stages, kSlot = d.slot;
   uint8_t* ring = smem;
-  uint8_t* pbuf = smem + S * kSlot;
-  float* sbias = reinterpret_cast<float*>(pbuf + kPBytes);
-  uint64_t* bars = reinterpret_cast<uint64_t*>(pbuf + kPBytes + d.bias_bytes);
+  uint8_t* pbuf = smem + S * kSlot;                                 // P of unit 0 | unit 1 of a pair
+  uint8_t* ones = pbuf + 2 * kPBytes;                               // bias-MMA A tile (1024-aligned)
+  float* sbias = reinterpret_cast<float*>(ones + kOnesBytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ones + kOnesBytes + d.bias_bytes);
   uint64_t* full = bars;               // [S]  leader: producer expect_tx + both CTAs' TMA bytes
-  uint64_t* empty = bars + S;          // [S]  each CTA: MMA commit (multicast)
-  uint64_t* acc_full = bars + 2 * S;   // [NB] each CTA: level accumulator written (multicast)
-  uint64_t* acc_empty = acc_full + 4;  // [NB] leader: 32 epilogue warps loaded it
-  uint64_t* p_full = acc_empty + 4;    //      leader: 32 warps wrote P
-  uint64_t* p_empty = p_full + 1;      //      each CTA: fconv MMAs read P (multicast)
-  uint64_t* out_full = p_empty + 1;    //      each CTA: out accumulated (multicast)
-  uint64_t* out_empty = out_full + 1;  //      leader: 32 warps drained out
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(out_empty + 1);
-
+  uint64_t* empty = bars + 8;          // [S]  each CTA: MMA commit (multicast)
+  uint64_t* acc_full = bars + 16;      // [2]  each CTA: unit u's level accumulator written (multicast)
+  uint64_t* acc_empty = bars + 18;     // [2]  leader: 32 epilogue warps loaded it
+  uint64_t* p_full = bars + 20;        //      leader: 32 warps wrote P of both units
+  uint64_t* p_empty = bars + 21;       //      each CTA: fconv MMAs read P (multicast)
+  uint64_t* out_full = bars + 22;      //      each CTA: out accumulated (multicast)
+  uint64_t* out_empty = bars + 23;     //      leader: 32 warps drained out
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 24);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t cta = cluster_ctarank();
-  // per-unit atom program (identical for every unit): the producer and the issuer walk it
-  // from shared memory instead of re-reading term fields from the (constant-cached) params
-  uint2* prog = reinterpret_cast<uint2*>(bars) + 64;   // after the barriers, <= 64 entries
-  if (warp == kProdWarp && lane == 0) {
-    int n = 0, j = 0;
-    for (int l = 0; l < d.n_levels; ++l) {
-      const int n0 = n;
-      for (; j < d.lvl_end[l]; ++j) {
-        const PairTerm& T = d.term[j];
-        for (int a = 0; a < T.natoms; ++a, ++n)
-          prog[n] = make_uint2((uint32_t)j | ((uint32_t)T.aw << 8) | ((uint32_t)atom_steps(T, a) << 16) |
-                                   ((n == n0 ? 1u : 0u) << 24) | ((l == 0 ? 4u : 0u) << 24),
-                               (uint32_t)(a * T.aw));
-      }
-      prog[n - 1].x |= 2u << 24;   // last atom of the level
-    }
-    prog[n - 1].x |= 8u << 24;     // last atom of the unit
-  }
   if (warp == kProdWarp && lane == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
       mbar_init(&empty[i], 1);
     }
-    for (int i = 0; i < 4; ++i) {
+    for (int i = 0; i < 2; ++i) {
       mbar_init(&acc_full[i], 1);
       mbar_init(&acc_empty[i], 2 * kEpiWarps);
     }
@@ -302,16 +374,30 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     mbar_init(out_full, 1);
     mbar_init(out_empty, 2 * kEpiWarps);
     fence_mbar_init_cluster();
-    for (int j = 0; j < d.n_terms; ++j) {
-      prefetch_tmap(d.term[j].amap);
-      prefetch_tmap(d.term[j].wmap);
+    for (int jj = 0; jj < d.n_terms; ++jj) {
+      prefetch_tmap(d.term[jj].amap);
+      prefetch_tmap(d.term[jj].wmap);
     }
     prefetch_tmap(d.fmap);
+    if (d.bias_mma) prefetch_tmap(d.bmap);
   }
-  if (warp >= kEpiWarp0) {
-    const float4* src = reinterpret_cast<const float4*>(p.params + d.lbias);
-    float4* dst = reinterpret_cast<float4*>(sbias);
-    for (int i = threadIdx.x - 32 * kEpiWarp0; i < d.n_levels * d.Cpad / 4; i += 32 * kEpiWarps) dst[i] = __ldg(src + i);
+  if (warp < kEpiWarp0 + kEpiWarps) {
+    if (d.bias_mma) {
+      // ones tile, K-major SW32 (32-byte rows; 16-byte chunk c of row r at c ^ ((r >> 2) & 1)):
+      // K columns 0 and 1 = 1.0 (they meet the bias hi / lo columns), the rest 0
+      const int r = threadIdx.x - 32 * kEpiWarp0;
+      if (r < 128) {
+        uint4* rowp = reinterpret_cast<uint4*>(ones + r * 32);
+        const int c0 = (r >> 2) & 1;
+        rowp[c0] = make_uint4(0x3F803F80u, 0u, 0u, 0u);
+        rowp[c0 ^ 1] = make_uint4(0u, 0u, 0u, 0u);
+      }
+      fence_proxy_async();
+    } else {
+      const float4* src = reinterpret_cast<const float4*>(p.params + d.lbias);
+      float4* dst = reinterpret_cast<float4*>(sbias);
+      for (int i = threadIdx.x - 32 * kEpiWarp0; i < d.n_levels * d.Cpad / 4; i += 32 * kEpiWarps) dst[i] = __ldg(src + i);
+    }
   }
   if (warp == kMmaWarp) {
     asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(tslot)));
@@ -320,225 +406,265 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   tc_fence_before();
   cluster_sync_all();
   tc_fence_after();
-  const uint32_t tbase = *tslot;
-  const uint32_t tout = tbase + (uint32_t)(NB * kPairWu);   // out region
+  // the CTA allocates all 512 TMEM columns, so the base address is lane 0 / column 0: a
+  // compile-time constant keeps the issuer's accumulator addresses in uniform registers
+  if (*tslot != 0u) __trap();
+  constexpr uint32_t tbase = 0;
+  constexpr uint32_t tout = tbase + 256u;   // out region [256, 256 + Np)
   pdl_wait();
 
   const int pair_id = blockIdx.x >> 1, npairs = gridDim.x >> 1;
-  const int U = d.nunits, D = d.n_levels;
+  const int U = d.nunits, UP = (U + 1) / 2;   // 128-channel units, unit pairs
 
   if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer (both CTAs)
     if (lane == 0) {
       int stage = 0;
       uint32_t ph = 0;
+// next ring stage (waits until the MMAs freed it); fb = the leader's full barrier of the stage
 #ifdef TEMCO_TRACE
       const bool notma = (g_pdbg & 1) != 0;
 #else
       constexpr bool notma = false;
 #endif
-      auto acquire = [&](uint32_t bytes) -> uint32_t {   // next ring stage; returns the leader's full barrier
-        mbar_wait(&empty[stage], ph ^ 1);
-        if (cta == 0) mbar_expect_tx(&full[stage], notma ? 0u : bytes);
-        return mapa_shared(smem_u32(&full[stage]), 0);
-      };
-      auto next = [&]() {
-        if (++stage == S) stage = 0, ph ^= 1;
-      };
-      auto fconv_atoms = [&](int u) {   // F[:, u*128 + a*64 .. +64], this CTA's Np/2 rows
-        for (int a = 0; a < kPairWu / 64; ++a) {
-          const uint32_t fb = acquire(2u * (uint32_t)(d.Np / 2 * 64 * 2));
-          if (!notma) tma_load_2d_pair(ring + stage * kSlot, d.fmap, fb, u * kPairWu + a * 64, (int)cta * (d.Np / 2));
-          next();
-        }
-      };
-      int pend = -1;   // unit whose fconv follows the next work item's first level
+#define PAIR_ACQUIRE(bytes)                                            \
+  mbar_wait(&empty[stage], ph ^ 1);                                    \
+  if (cta == 0) mbar_expect_tx(&full[stage], notma ? 0u : (bytes));    \
+  const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0)
+#define PAIR_NEXT()           \
+  if (++stage == S) {         \
+    stage = 0;                \
+    ph ^= 1;                  \
+  }
+#define PAIR_FCONV_ATOMS(pp)                                                                                   \
+  for (int u = 2 * (pp); u < min(2 * (pp) + 2, U); ++u)                                                        \
+    for (int a = 0; a < kPairWu / 64; ++a) {                                                                   \
+      PAIR_ACQUIRE(2u * (uint32_t)(d.Np / 2 * 64 * 2));                                                        \
+      if (!notma) tma_load_2d_pair(ring + stage * kSlot, d.fmap, fb, u * kPairWu + a * 64, (int)cta * (d.Np / 2)); \
+      PAIR_NEXT();                                                                                             \
+    }
+      EVDECL();
+      int pend = -1;   // pair whose fconv operands follow the next pair's first level
       const uint8_t* term0 = reinterpret_cast<const uint8_t*>(&d.term[0]);
       for (int tile = pair_id; tile < d.ntiles; tile += npairs) {
         const int row0 = tile * 256 + (int)cta * 128;
-        for (int u = 0; u < U; ++u) {
+        for (int pp = 0; pp < UP; ++pp) {
+          const int u0 = 2 * pp, nu = min(2, U - u0);
           for (int k = 0;; ++k) {
-            const uint2 op = prog[k];
+            const uint2 op = make_uint2(d.prog[k][0], d.prog[k][1]);
             const int j = op.x & 0xFF, aw = (op.x >> 8) & 0xFF;
             const uint32_t fl = op.x >> 24;
             const PairTerm* T = reinterpret_cast<const PairTerm*>(term0 + j * sizeof(PairTerm));
-            const uint32_t fb = acquire(2u * (uint32_t)((128 + 64) * aw * 2));   // both CTAs, A + B
+            const bool bia = d.bias_mma && (fl & 1u);
+            PAIR_ACQUIRE(2u * (uint32_t)((128 + 64 * nu) * aw * 2 + (bia ? nu * 64 * 32 : 0)));
             uint8_t* sa = ring + stage * kSlot;
-            if (!notma) {
-              tma_load_2d_pair(sa, T->amap, fb, (int)op.y, row0);
-              tma_load_2d_pair(sa + kSlotA, T->wmap, fb, (int)op.y, u * kPairWu + (int)cta * 64);
+            EV(0);
+            if (!notma) tma_load_2d_pair(sa, T->amap, fb, (int)op.y, row0);
+            for (int q = 0; q < nu && !notma; ++q) {
+              tma_load_2d_pair(sa + kSlotA + q * kSlotB, T->wmap, fb, (int)op.y, (u0 + q) * kPairWu + (int)cta * 64);
+              if (bia)
+                tma_load_2d_pair(sa + kSlotA + 2 * kSlotB + q * kSlotC, d.bmap, fb, 0,
+                                 (int)(op.x >> 28) * d.Cpad + (u0 + q) * kPairWu + (int)cta * 64);
             }
-            next();
-            if ((fl & 6u) == 6u && pend >= 0) {   // after level 0: the previous unit's fconv operands
-              fconv_atoms(pend);
+            PAIR_NEXT();
+            if ((fl & 6u) == 6u && pend >= 0) {   // after level 0: the previous pair's fconv operands
+              PAIR_FCONV_ATOMS(pend);
               pend = -1;
             }
             if (fl & 8u) break;
           }
-          pend = u;
+          pend = pp;
         }
       }
-      if (pend >= 0) fconv_atoms(pend);
+      if (pend >= 0) {
+        PAIR_FCONV_ATOMS(pend);
+      }
+#undef PAIR_ACQUIRE
+#undef PAIR_NEXT
+#undef PAIR_FCONV_ATOMS
     }
   } else if (warp == kMmaWarp) {
-    // ------------------------------------------------------------ MMA issuer (leader, whole warp)
+    // ------------------------------------------------------------ MMA issuer (leader, whole warp;
+    // one elected lane issues each tcgen05 instruction)
     if (cta == 0) {
-      PTDECL();
       const uint32_t idesc_t = idesc_bf16(256, kPairWu), idesc_f = idesc_bf16(256, d.Np);
       const uint32_t sbase = smem_u32(smem), pbase = smem_u32(pbuf);
+      const uint64_t ones_d = umma_desc_k(smem_u32(ones), 16);
       int stage = 0;
       uint32_t ph = 0;
-      int gl = 0;        // levels issued (accumulator buffer gl % NB, use gl / NB)
-      int nf = 0;        // fconvs issued (P phase)
-      int it = 0;        // tiles whose out region was started
-      auto fconv = [&](int u) {
-        PT0();
-        mbar_wait_cluster(p_full, (uint32_t)nf & 1u);
-        PTADD(3);
-        tc_fence_after();
-        if (u == 0 && it > 0) {   // a new tile's out region: previous tile drained
-          PT0();
-          mbar_wait_cluster(out_empty, (uint32_t)(it - 1) & 1u);
-          PTADD(4);
-          tc_fence_after();
-        }
-        for (int a = 0; a < kPairWu / 64; ++a) {
-          PT0();
-          mbar_wait(&full[stage], ph);
-          PTADD(1);
-          tc_fence_after();
-          const uint64_t fd = umma_desc_k(sbase + stage * kSlot, 64);
-          const uint64_t pd = umma_desc_k(pbase + a * 16384, 64);
-          for (int k = 0; k < 4; ++k)
-            mma2_bf16_w(tout, pd + 2 * k, fd + 2 * k, idesc_f, (u == 0 && a == 0 && k == 0) ? 0u : 1u);
-          mma2_commit_mc_w(&empty[stage], 3);
-          if (++stage == S) stage = 0, ph ^= 1;
-        }
-        mma2_commit_mc_w(p_empty, 3);
-        ++nf;
-        if (u == U - 1) {
-          mma2_commit_mc_w(out_full, 3);
-          ++it;
-        }
-      };
-      int pend = -1;
-      int b = 0, bu = 0;   // accumulator buffer of the current level, its use count
+      int na0 = 0, na1 = 0;   // uses of each unit's accumulator (scalars: no local-memory array)
+      int nf = 0;             // pair fconvs issued
+      int it = 0;             // tiles whose out region was started
+// fconv of unit pair pp: out (+)= P_u F_u^T for its units; the first pair of a tile starts
+// the out region (after the previous tile's out was drained), the last one publishes it
+#define PAIR_FCONV(pp, first_of_tile, last_of_tile)                                                            \
+  {                                                                                                            \
+    mbar_wait_u(p_full, (uint32_t)nf & 1u);                                                              \
+    EV(4);                                                                                                     \
+    tc_fence_after();                                                                                          \
+    if ((first_of_tile) && it > 0) {                                                                           \
+      mbar_wait_u(out_empty, (uint32_t)(it - 1) & 1u);                                                   \
+      tc_fence_after();                                                                                        \
+    }                                                                                                          \
+    for (int q = 0; q < min(2, U - 2 * (pp)); ++q)                                                             \
+      for (int a = 0; a < kPairWu / 64; ++a) {                                                                 \
+        mbar_wait_u(&full[stage], ph);                                                                           \
+        tc_fence_after();                                                                                      \
+        {                                                                                                      \
+          const uint64_t fd = umma_desc_k(sbase + stage * kSlot, 64);                                          \
+          const uint64_t pd = umma_desc_k(pbase + q * kPBytes + a * 16384, 64);                                \
+          for (int k4 = 0; k4 < 4; ++k4)                                                                       \
+            mma2_bf16_w(tout, pd + 2 * k4, fd + 2 * k4, idesc_f, ((first_of_tile) && q == 0 && a == 0 && k4 == 0) ? 0u : 1u); \
+        }                                                                                                      \
+        mma2_commit_mc_w(&empty[stage], 3);                                                                    \
+        if (++stage == S) stage = 0, ph ^= 1;                                                                  \
+      }                                                                                                        \
+    mma2_commit_mc_w(p_empty, 3);                                                                              \
+    ++nf;                                                                                                      \
+    if (last_of_tile) {                                                                                        \
+      mma2_commit_mc_w(out_full, 3);                                                                           \
+      ++it;                                                                                                    \
+    }                                                                                                          \
+  }
+      EVDECL();
+      int pend = -1, pend_tile_first = 0, pend_tile_last = 0;
       for (int tile = pair_id; tile < d.ntiles; tile += npairs) {
-        for (int u = 0; u < U; ++u) {
-          uint32_t dt = 0;
-          for (int k = 0;; ++k) {
-            const uint2 op = prog[k];
-            const int aw = (op.x >> 8) & 0xFF, nk = (op.x >> 16) & 0xFF;
-            const uint32_t fl = op.x >> 24;
-            if (fl & 1u) {   // first atom of a level: its buffer must have been drained
-              if (bu > 0) {
-                PT0();
-                mbar_wait_cluster(&acc_empty[b], (uint32_t)(bu - 1) & 1u);
-                PTADD(2);
-                tc_fence_after();
+        for (int pp = 0; pp < UP; ++pp) {
+          const int nu = min(2, U - 2 * pp);
+          int k = 0;
+          for (;;) {   // one level per iteration, in chunks of <= kChunk ring stages
+            const uint32_t op0x = d.prog[k][0];
+            // atoms of this level
+            int kl = k;
+            while (!((d.prog[kl][0] >> 24) & 2u)) ++kl;
+            const int nat = kl - k + 1;
+            const bool first_level = (op0x >> 24) & 4u;
+            for (int c0 = 0; c0 < nat; c0 += kChunk) {
+              const int cn = min(kChunk, nat - c0);
+              for (int q = 0; q < nu; ++q) {
+                const int na = q ? na1 : na0;
+                if (c0 == 0 && na > 0) {   // the unit's accumulator must have been drained
+                  mbar_wait_u(&acc_empty[q], (uint32_t)(na - 1) & 1u);
+                  tc_fence_after();
+                }
+                const uint32_t dt = tbase + (uint32_t)(q * kPairWu);
+                int st = stage;
+                uint32_t sph = ph;
+                for (int i = 0; i < cn; ++i) {
+                  const uint2 op = make_uint2(d.prog[k + c0 + i][0], d.prog[k + c0 + i][1]);
+                  const int aw = (op.x >> 8) & 0xFF, nk = (op.x >> 16) & 0xFF;
+                  if (q == 0) {
+                    mbar_wait_u(&full[st], sph);
+                    EV(1);
+                    tc_fence_after();
+                  }
+                  const bool lvl0 = c0 == 0 && i == 0;   // first atom of the level
+                  {
+                    const uint32_t sa = sbase + st * kSlot;
+                    const uint64_t ad = umma_desc_k(sa, aw), bd = umma_desc_k(sa + kSlotA + q * kSlotB, aw);
+                    const bool bia = d.bias_mma && lvl0;
+                    if (bia) mma2_bf16_w(dt, ones_d, umma_desc_k(sa + kSlotA + 2 * kSlotB + q * kSlotC, 16), idesc_t, 0u);
+                    for (int kk = 0; kk < nk; ++kk)
+                      mma2_bf16_w(dt, ad + 2 * kk, bd + 2 * kk, idesc_t, (lvl0 && !bia && kk == 0) ? 0u : 1u);
+                  }
+                  EV(2);
+                  if (++st == S) st = 0, sph ^= 1;
+                }
+                if (c0 + cn == nat) {
+                  mma2_commit_mc_w(&acc_full[q], 3);
+                  EV(3);
+                  if (q) ++na1;
+                  else ++na0;
+                }
               }
-              dt = tbase + (uint32_t)(b * kPairWu);
-            }
-            PT0();
-            mbar_wait(&full[stage], ph);
-            PTADD(1);
-            tc_fence_after();
-            const uint32_t sa = sbase + stage * kSlot;
-            const uint64_t ad = umma_desc_k(sa, aw), bd = umma_desc_k(sa + kSlotA, aw);
-            PT0();
-            for (int kk = 0; kk < nk; ++kk)
-              mma2_bf16_w(dt, ad + 2 * kk, bd + 2 * kk, idesc_t, ((fl & 1u) && kk == 0) ? 0u : 1u);
-            PTADD(5);
-            PT0();
-            mma2_commit_mc_w(&empty[stage], 3);
-            PTADD(6);
-            if (++stage == S) stage = 0, ph ^= 1;
-            if (fl & 2u) {   // last atom of the level
-              mma2_commit_mc_w(&acc_full[b], 3);
-              if (++b == NB) b = 0, ++bu;
-              if ((fl & 4u) && pend >= 0) {
-                fconv(pend);
-                pend = -1;
+              for (int i = 0; i < cn; ++i) {
+                mma2_commit_mc_w(&empty[stage], 3);
+                if (++stage == S) stage = 0, ph ^= 1;
               }
             }
-            if (fl & 8u) break;
+            if (first_level && pend >= 0) {
+              PAIR_FCONV(pend, pend_tile_first, pend_tile_last);
+              pend = -1;
+            }
+            const bool last = (d.prog[kl][0] >> 24) & 8u;
+            k = kl + 1;
+            if (last) break;
           }
-          pend = u;
+          pend = pp;
+          pend_tile_first = pp == 0;
+          pend_tile_last = pp == UP - 1;
         }
       }
-      if (pend >= 0) fconv(pend);
-      if (lane == 0) PTSAVE(1, 8, 0);
+      if (pend >= 0) PAIR_FCONV(pend, pend_tile_first, pend_tile_last);
+#undef PAIR_FCONV
     }
   } else {
     // ------------------------------------------------------------ epilogue (16 warps, both CTAs)
-    const int q = warp & 3;                  // TMEM lane quarter of this warp
+    const int q = warp & 3;                  // TMEM lane quarter of this warp (warp % 4)
     const int g = (warp - kEpiWarp0) >> 2;   // 32-column group of a unit
     const int row = q * 32 + lane;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     const uint32_t pfull_c = mapa_shared(smem_u32(p_full), 0);
     const uint32_t oempty_c = mapa_shared(smem_u32(out_empty), 0);
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
-    int b = 0, br = 0, np = 0, it = 0;   // accumulator buffer, its round
-    PTDECL();
+    int nacc[2] = {0, 0}, np = 0, it = 0;
+    EVDECL();
+    const bool ev0 = warp == kEpiWarp0 && lane == 0;
     for (int tile = pair_id; tile < d.ntiles; tile += npairs, ++it) {
       const int64_t prow = (int64_t)tile * 256 + cta * 128 + row;
-      for (int u = 0; u < U; ++u) {
-        float t[32];
-        for (int l = 0; l < D; ++l) {
+      for (int pp = 0; pp < UP; ++pp) {
+        const int nu = min(2, U - 2 * pp);
+        uint32_t t0[16], t1[16];
+        for (int l = 0; l < d.n_levels; ++l) {
           const int act = d.act[l];
-          const float4* b4 = reinterpret_cast<const float4*>(sbias + l * d.Cpad + u * kPairWu + g * 32);
-          PT0();
-          mbar_wait(&acc_full[b], (uint32_t)br & 1u);
-          PTADD(9);
-          tc_fence_after();
-          uint32_t v[32];
-          PT0();
-          tmem_ld32(tbase + lane_off + (uint32_t)(b * kPairWu + g * 32), v);
-          tmem_wait_ld();
-          tc_fence_before();
-          warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[b]), 0));
-          if (++b == NB) b = 0, ++br;
-          PTADD(11);
-          PT0();
 #pragma unroll
-          for (int i4 = 0; i4 < 8; ++i4) {
-            const float4 bb = b4[i4];   // broadcast LDS.128
-            const float bq[4] = {bb.x, bb.y, bb.z, bb.w};
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-              const int i = 4 * i4 + k;
-              const float z = __uint_as_float(v[i]) + bq[k];
-              t[i] = act_p<SILU>(l == 0 ? z : z + t[i], act);
+          for (int qq = 0; qq < 2; ++qq) {
+            if (qq < nu) {
+              const float* bl = d.bias_mma ? nullptr : sbias + l * d.Cpad + (2 * pp + qq) * kPairWu + g * 32;
+              mbar_wait(&acc_full[qq], (uint32_t)nacc[qq] & 1u);
+              if (ev0) EV(qq ? 8 : 5);
+              tc_fence_after();
+              uint32_t v[32];
+#ifdef TEMCO_TRACE
+              if (g_pdbg & 2) {
+                warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[qq]), 0));
+                ++nacc[qq];
+                continue;
+              }
+#endif
+              tmem_ld32(tbase + lane_off + (uint32_t)(qq * kPairWu + g * 32), v);
+              tmem_wait_ld();
+              tc_fence_before();
+              warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[qq]), 0));
+              ++nacc[qq];
+              if (ev0 && !qq) EV(6);
+              level_math<SILU>(qq ? t1 : t0, v, l == 0, act, bl);
+              if (ev0) EV(qq ? 9 : 7);
             }
           }
-          PTADD(12);
         }
-        // P = bf16(t_D) for the unit's fconv
-        PT0();
+        // P = t_D (already bf16x2) of both units for the pair's fconv
         if (np > 0) mbar_wait(p_empty, (uint32_t)(np - 1) & 1u);
-        PTADD(10);
-        PT0();
         ++np;
-        uint8_t* P = pbuf + (g >> 1) * 16384 + row * 128;
 #pragma unroll
-        for (int c4 = 0; c4 < 4; ++c4) {
-          uint4 pk;
-          pk.x = pack_bf16(t[8 * c4 + 0], t[8 * c4 + 1]);
-          pk.y = pack_bf16(t[8 * c4 + 2], t[8 * c4 + 3]);
-          pk.z = pack_bf16(t[8 * c4 + 4], t[8 * c4 + 5]);
-          pk.w = pack_bf16(t[8 * c4 + 6], t[8 * c4 + 7]);
-          const int chunk = (g & 1) * 4 + c4;
-          *reinterpret_cast<uint4*>(P + ((chunk ^ (row & 7)) * 16)) = pk;
+        for (int qq = 0; qq < 2; ++qq) {
+          if (qq < nu) {
+            uint8_t* P = pbuf + qq * kPBytes + (g >> 1) * 16384 + row * 128;
+            const uint32_t* t = qq ? t1 : t0;
+#pragma unroll
+            for (int c4 = 0; c4 < 4; ++c4) {
+              const int chunk = (g & 1) * 4 + c4;
+              *reinterpret_cast<uint4*>(P + ((chunk ^ (row & 7)) * 16)) =
+                  make_uint4(t[4 * c4], t[4 * c4 + 1], t[4 * c4 + 2], t[4 * c4 + 3]);
+            }
+          }
         }
         fence_proxy_async();
         warp_arrive_cluster(pfull_c);
-        PTADD(14);
+        if (ev0) EV(10);
       }
-      // out tile: TMEM columns [128 NB, 128 NB + Np) -> bf16 -> y[prow, :Nout]
-      PT0();
+      // out tile: TMEM columns [256, 256 + Np) -> bf16 -> y[prow, :Nout]
       mbar_wait(out_full, (uint32_t)it & 1u);
-      PTADD(13);
-      PT0();
       tc_fence_after();
       const int nch = d.Np / 8;
       for (int c8 = g; c8 < nch; c8 += 4) {
@@ -556,9 +682,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       }
       tc_fence_before();
       warp_arrive_cluster(oempty_c);
-      PTADD(15);
+      if (ev0) EV(11);
     }
-    if (warp == kEpiWarp0 && lane == 0) PTSAVE(9, 16, 8);
   }
   tc_fence_before();
   cluster_sync_all();
@@ -567,7 +692,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, 512;" ::"r"(tbase));
   }
 #ifdef TEMCO_TRACE
-  if (blockIdx.x == 0 && threadIdx.x == 0) atomicAdd(&g_pprof_n, 1);
+  if (blockIdx.x == 0 && threadIdx.x == 0) g_launch = g_launch + 1;
 #endif
 }
 
@@ -603,14 +728,16 @@ void launch_pair_chain(const PairDesc& d, const RunPtrs& p, cudaStream_t s) {
 }  // namespace temco
 
 
+
 #ifdef TEMCO_TRACE
-extern "C" int temco_debug_pair_prof(unsigned long long* out) {
-  int n = 0;
-  cudaMemcpyFromSymbol(&n, temco::pair::g_pprof_n, sizeof(int));
-  cudaMemcpyFromSymbol(out, temco::pair::g_pprof, sizeof(unsigned long long) * 64 * 16);
+// timeline of CTA 0 for the tc_pair launch with index `launch` (counted from the last reset)
+extern "C" void temco_debug_pair_ev(int launch, long long* out) {
+  if (out) cudaMemcpyFromSymbol(out, temco::pair::g_ev, sizeof(long long) * 12 * 512);
+  cudaMemcpyToSymbol(temco::pair::g_ev_on, &launch, sizeof(int));
   const int z = 0;
-  cudaMemcpyToSymbol(temco::pair::g_pprof_n, &z, sizeof(int));
-  return n;
+  cudaMemcpyToSymbol(temco::pair::g_launch, &z, sizeof(int));
+  static long long zz[12 * 512] = {0};
+  cudaMemcpyToSymbol(temco::pair::g_ev, zz, sizeof(zz));
 }
 extern "C" void temco_debug_pair_dbg(int v) { cudaMemcpyToSymbol(temco::pair::g_pdbg, &v, sizeof(int)); }
 #endif

@@ -33,6 +33,7 @@ namespace pair {
 
 constexpr int kPairMaxTerms = 16;
 constexpr int kPairMaxLevels = 16;
+constexpr int kPairMaxAtoms = 64;       // K atoms of one unit's level chain
 constexpr int kPairWu = 128;           // restored channels per unit (MMA N of the restore GEMM)
 
 struct PairTerm {
@@ -46,10 +47,15 @@ struct PairTerm {
 struct PairDesc {
   PairTerm term[kPairMaxTerms];
   alignas(64) unsigned char fmap[128];   // F [Np x Cpad] bf16, box {64, Np/2}
+  alignas(64) unsigned char bmap[128];   // bias-MMA groups: [n_levels*Cpad x 16] bf16 (hi, lo), box {16, 64}
   int32_t n_terms, n_levels;
+  uint32_t prog[kPairMaxAtoms][2];       // atom program: term | aw << 8 | K16 steps << 16 | flags << 24 | level << 28; x
+  int32_t n_prog;
   int32_t lvl_end[kPairMaxLevels];       // terms [lvl_end[l-1], lvl_end[l]) belong to level l
   int32_t act[kPairMaxLevels];           // 0 none, 1 ReLU, 2 SiLU
   int64_t lbias;                         // params offset: fp32 [n_levels][Cpad] level biases
+  int32_t bias_mma;                      // level biases added by a K=16 MMA (ones x [hi, lo]) instead of the epilogue
+  int64_t bmat;                          // tc weight pool offset of the bias-MMA matrix
   int32_t C, Cpad, nunits;               // restored width, padded to 128, 128-channel units
   int32_t nbuf;                          // rotating level accumulators (TMEM columns [0, 128 nbuf))
   int32_t Nout, Np;                      // fconv outputs, padded to 16
@@ -57,7 +63,7 @@ struct PairDesc {
   int32_t ntiles;                        // 256-pixel pair tiles
   Loc y;                                 // output [npix x Nout] bf16 (arena)
   int64_t F;                             // tc weight pool offset of F
-  int32_t stages, smem_bytes, bias_bytes;
+  int32_t stages, slot, smem_bytes, bias_bytes;   // ring depth, stage bytes
   int32_t silu;                          // some level is SiLU: SILU kernel instantiation
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
 };

@@ -34,7 +34,7 @@ __device__ __forceinline__ void commit(uint64_t* b) {
 }
 
 template <int CG>
-__global__ void __cluster_dims__(CG, 1, 1) k(int iters, int N, int nw, unsigned long long* out) {
+__global__ void __cluster_dims__(CG, 1, 1) k(int iters, int N, int nw, int rot, unsigned long long* out) {
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* base = (uint8_t*)(((uintptr_t)sm + 1023) & ~(uintptr_t)1023);
   __shared__ uint64_t bar[4];
@@ -54,7 +54,7 @@ __global__ void __cluster_dims__(CG, 1, 1) k(int iters, int N, int nw, unsigned 
     for (int i = 0; i < 4; ++i) mbar_init(&bar[i], 1);
     asm volatile("fence.mbarrier_init.release.cluster;");
   }
-  for (int i = threadIdx.x; i < 65536 / 4; i += blockDim.x) ((uint32_t*)base)[i] = 0;
+  for (int i = threadIdx.x; i < 4 * 49152 / 4; i += blockDim.x) ((uint32_t*)base)[i] = 0;
   asm volatile("fence.proxy.async.shared::cta;");
   asm volatile("tcgen05.fence::before_thread_sync;");
   asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
@@ -63,10 +63,12 @@ __global__ void __cluster_dims__(CG, 1, 1) k(int iters, int N, int nw, unsigned 
   const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
   const int w = threadIdx.x >> 5;
   if (rank == 0 && w < nw && (threadIdx.x & 31) == 0) {
-    const uint64_t a = desc(smem_u32(base)), b = desc(smem_u32(base + 32768));
     const uint32_t d = slot + (uint32_t)(w * (512 / nw));
     long long t0 = clock64();
     for (int i = 0; i < iters; ++i) {
+      // rot = 0: one A / B pair; rot > 0: A / B atoms rotate over `rot` distinct 24 KB stages
+      const int st = rot ? (i % rot) : 0;
+      const uint64_t a = desc(smem_u32(base + st * 49152)), b = desc(smem_u32(base + st * 49152 + 16384));
 #pragma unroll
       for (int j = 0; j < 8; ++j) mma<CG>(d, a + 2 * (j & 3), b + 2 * (j & 3), idesc, (i | j) > 0);
     }
@@ -84,28 +86,26 @@ __global__ void __cluster_dims__(CG, 1, 1) k(int iters, int N, int nw, unsigned 
 
 int main() {
   unsigned long long* d;
-  cudaMalloc(&d, 64);
-  cudaFuncSetAttribute(k<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 70000);
-  cudaFuncSetAttribute(k<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 70000);
-  for (int cg : {1, 2})
-    for (int nw : {1, 2, 4})
-      for (int N : {32, 64, 128, 256}) {
-        if (N * nw > 512) continue;
-        const int iters = 500;
-        for (int rep = 0; rep < 2; ++rep) {
-          if (cg == 1) k<1><<<1, 128, 70000>>>(iters, N, nw, d);
-          else k<2><<<2, 128, 70000>>>(iters, N, nw, d);
+  cudaMalloc(&d, 148 * 64);
+  const int smem = 4 * 49152 + 2048;
+  cudaFuncSetAttribute(k<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaFuncSetAttribute(k<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  for (int grid : {2, 148})
+    for (int rot : {0, 4})
+      for (int cg : {1, 2})
+        for (int N : {64, 128, 256}) {
+          const int iters = 500, nw = 1;
+          for (int rep = 0; rep < 2; ++rep) {
+            if (cg == 1) k<1><<<grid, 128, smem>>>(iters, N, nw, rot, d);
+            else k<2><<<grid, 128, smem>>>(iters, N, nw, rot, d);
+          }
+          cudaError_t e = cudaDeviceSynchronize();
+          if (e != cudaSuccess) { printf("err %s\n", cudaGetErrorString(e)); return 1; }
+          unsigned long long c = 0;
+          cudaMemcpy(&c, d, 8, cudaMemcpyDeviceToHost);
+          const double per = (double)c / (iters * 8.0);
+          const double floor_ = (cg == 2 ? 256.0 : 128.0) * N / (256.0 * cg);
+          printf("grid=%3d rot=%d cta_group::%d N=%3d: %6.1f cyc per MMA, floor %5.1f -> %.2f\n", grid, rot, cg, N, per, floor_, floor_ / per);
         }
-        cudaError_t e = cudaDeviceSynchronize();
-        if (e != cudaSuccess) { printf("err %s\n", cudaGetErrorString(e)); return 1; }
-        unsigned long long c[4] = {0, 0, 0, 0};
-        cudaMemcpy(c, d, 8 * nw, cudaMemcpyDeviceToHost);
-        unsigned long long mx = 0;
-        for (int i = 0; i < nw; ++i) mx = c[i] > mx ? c[i] : mx;
-        const double per = (double)mx / (iters * 8.0 * nw);
-        const double floor_ = (cg == 2 ? 256.0 : 128.0) * N / (256.0 * cg);
-        printf("cta_group::%d issuers=%d N=%3d: %6.1f cyc per MMA (all issuers), floor %5.1f -> %.2f of peak\n", cg, nw, N,
-               per, floor_, floor_ / per);
-      }
   return 0;
 }
