@@ -179,6 +179,18 @@ temco_status temco_plan_describe(temco_plan_t plan, char* buf, size_t cap, size_
 temco_status temco_run_profiled(temco_plan_t plan, const void* input, void* output,
                                 temco_stream_t stream, float* step_ms, int32_t n_steps);
 
+/* Verification hook (per-step parity, P:L305 / Fig. 8: every schedule step's tensor
+ * of the TeMCO plan equals the same tensor of the decomposed model): enqueue
+ * steps 0 .. step of one run on `stream` (no CUDA graph), synchronise, and copy
+ * the output tensor of schedule step `step` (a reduced tensor in the arena,
+ * NHWC in the plan dtype; or the graph output) to host_dst.  *bytes = its size;
+ * host_dst = NULL only queries the size.  capacity < size ->
+ * TEMCO_ERR_INVALID_ARGUMENT.  The arena is reused by later steps, so the copy
+ * is taken before any later step runs.  Same device / input / output rules as
+ * temco_run. */
+temco_status temco_debug_step_output(temco_plan_t plan, const void* input, void* output, temco_stream_t stream,
+                                     int32_t step, void* host_dst, int64_t capacity, int64_t* bytes);
+
 temco_status temco_plan_destroy(temco_plan_t plan);
 const char* temco_status_string(temco_status s);
 const char* temco_last_error(void);

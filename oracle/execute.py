@@ -83,8 +83,19 @@ def _eval_group(plan, step, env):
     return value(step.out)
 
 
-def run_temco(plan, x):
-    """Run the TeMCO schedule S (fused groups + remaining ops)."""
+def run_step(plan, t, env):
+    """Output of schedule step t of S given its input tensors env[id] (per-step parity
+    tests feed the GPU's own inputs, so each step is checked in isolation)."""
+    s = plan.steps[t]
+    if s.kind == "group":
+        return _eval_group(plan, s, env)
+    v = plan.onodes[s.out]
+    return apply(v, [env[i] for i in v.inputs])
+
+
+def run_temco(plan, x, on_step=None):
+    """Run the TeMCO schedule S (fused groups + remaining ops).  on_step(t, tensor),
+    if given, sees every step's output as it is produced (per-step parity tests)."""
     g = plan.graph
     steps = plan.steps
     last = {}
@@ -100,6 +111,8 @@ def run_temco(plan, x):
         else:
             v = plan.onodes[s.out]
             env[s.out] = apply(v, [env[i] for i in v.inputs])
+        if on_step is not None:
+            on_step(t, env[s.out])
         for i in s.inputs:
             if last[i] == t and i != g.output:
                 del env[i]

@@ -96,11 +96,16 @@ struct temco_plan_s {
   int max_expr_depth = 0;          // deepest fused-group expression (SIMT interpreter recursion)
   int64_t out_dims[4] = {0, 0, 0, 0};
   int out_ndim = 0;
-  // CUDA graph cache (TEMCO_FLAG_CUDA_GRAPH)
-  cudaGraphExec_t gexec = nullptr;
-  const void* g_in = nullptr;
-  void* g_out = nullptr;
-  cudaStream_t g_stream = nullptr;
+  // CUDA graph cache (TEMCO_FLAG_CUDA_GRAPH): one executable graph per (input, output, stream);
+  // two entries so temco_run_host_async's alternating staging buffers each keep their graph
+  struct GraphEntry {
+    cudaGraphExec_t exec = nullptr;
+    const void* in = nullptr;
+    void* out = nullptr;
+    cudaStream_t stream = nullptr;
+    uint64_t used = 0;
+  } graphs[2];
+  uint64_t graph_clock = 0;
   std::string json;
 };
 
@@ -608,7 +613,8 @@ temco_status upload(T** dst, const std::vector<T>& src) {
 }
 
 void free_device(temco_plan_s* P) {
-  if (P->gexec) cudaGraphExecDestroy(P->gexec);
+  for (auto& g : P->graphs)
+    if (g.exec) cudaGraphExecDestroy(g.exec);
   cudaFree(P->params_d);
   cudaFree(P->gnodes_d);
   cudaFree(P->gchild_d);
@@ -640,9 +646,11 @@ RunPtrs run_ptrs(temco_plan_s* P, const void* in, void* out) {
   return RunPtrs{P->arena_d, in, out, P->params_d};
 }
 
-temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st, cudaEvent_t* ev) {
+temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st, cudaEvent_t* ev,
+                     int64_t last_step = -1) {
   RunPtrs rp = run_ptrs(P, in, out);
-  for (size_t t = 0; t < P->exec.size(); ++t) {
+  const size_t nsteps = last_step >= 0 ? (size_t)last_step + 1 : P->exec.size();
+  for (size_t t = 0; t < nsteps; ++t) {
     const StepExec& e = P->exec[t];
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t], st));
     switch (e.kind) {
@@ -854,23 +862,28 @@ temco_status temco_run(temco_plan_t P, const void* input, void* output, temco_st
   if (!input || !output) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "input / output is NULL");
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   if ((P->flags & TEMCO_FLAG_CUDA_GRAPH) && s != nullptr) {
-    if (!P->gexec || P->g_in != input || P->g_out != output || P->g_stream != s) {
-      if (P->gexec) cudaGraphExecDestroy(P->gexec);
-      P->gexec = nullptr;
+    temco_plan_s::GraphEntry* g = nullptr;
+    for (auto& e : P->graphs)
+      if (e.exec && e.in == input && e.out == output && e.stream == s) g = &e;
+    if (!g) {   // capture into the least recently used entry
+      g = P->graphs[0].used <= P->graphs[1].used ? &P->graphs[0] : &P->graphs[1];
+      if (g->exec) cudaGraphExecDestroy(g->exec);
+      g->exec = nullptr;
       cudaGraph_t graph;
       CUDA_TRY(cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal));
       temco_status e = enqueue(P, input, output, s, nullptr);
       cudaError_t ce = cudaStreamEndCapture(s, &graph);
       if (e != TEMCO_OK) return e;
       if (ce != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string("capture: ") + cudaGetErrorString(ce));
-      ce = cudaGraphInstantiate(&P->gexec, graph, 0);
+      ce = cudaGraphInstantiate(&g->exec, graph, 0);
       cudaGraphDestroy(graph);
       if (ce != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string("instantiate: ") + cudaGetErrorString(ce));
-      P->g_in = input;
-      P->g_out = output;
-      P->g_stream = s;
+      g->in = input;
+      g->out = output;
+      g->stream = s;
     }
-    CUDA_TRY(cudaGraphLaunch(P->gexec, s));
+    g->used = ++P->graph_clock;
+    CUDA_TRY(cudaGraphLaunch(g->exec, s));
     return TEMCO_OK;
   }
   return enqueue(P, input, output, s, nullptr);
@@ -881,9 +894,16 @@ temco_status temco_run_host(temco_plan_t P, const void* host_input, void* host_o
   if (st != TEMCO_OK) return st;
   if (!host_input || !host_output) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "host buffers are NULL");
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  if (!P->host_in_d) {
-    if (cudaMalloc(&P->host_in_d, P->in_bytes) != cudaSuccess || cudaMalloc(&P->host_out_d, P->out_bytes) != cudaSuccess)
+  if (!P->host_in_d || !P->host_out_d) {
+    cudaFree(P->host_in_d);
+    cudaFree(P->host_out_d);
+    P->host_in_d = P->host_out_d = nullptr;
+    if (cudaMalloc(&P->host_in_d, P->in_bytes) != cudaSuccess || cudaMalloc(&P->host_out_d, P->out_bytes) != cudaSuccess) {
+      cudaFree(P->host_in_d);   // all or nothing: a later call retries from scratch
+      P->host_in_d = nullptr;
+      P->host_out_d = nullptr;
       return set_err(TEMCO_ERR_OUT_OF_MEMORY, "staging buffers");
+    }
   }
   CUDA_TRY(cudaMemcpyAsync(P->host_in_d, host_input, P->in_bytes, cudaMemcpyHostToDevice, s));
   st = temco_run(P, P->host_in_d, P->host_out_d, stream);
@@ -900,15 +920,31 @@ temco_status temco_run_host_async(temco_plan_t P, const void* host_input, void* 
   if (!host_input || !host_output) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "host buffers are NULL");
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   if (!P->copy_stream) {
-    for (int b = 0; b < 2; ++b)
-      if (cudaMalloc(&P->async_in_d[b], P->in_bytes) != cudaSuccess ||
-          cudaMalloc(&P->async_out_d[b], P->out_bytes) != cudaSuccess)
-        return set_err(TEMCO_ERR_OUT_OF_MEMORY, "async staging buffers");
-    CUDA_TRY(cudaStreamCreateWithFlags(&P->copy_stream, cudaStreamNonBlocking));
-    for (int b = 0; b < 2; ++b) {
-      CUDA_TRY(cudaEventCreateWithFlags(&P->ev_in_ready[b], cudaEventDisableTiming));
-      CUDA_TRY(cudaEventCreateWithFlags(&P->ev_buf_free[b], cudaEventDisableTiming));
+    // all or nothing: on any failure release what was made, so a later call starts over
+    auto release = [P]() {
+      for (int b = 0; b < 2; ++b) {
+        cudaFree(P->async_in_d[b]);
+        cudaFree(P->async_out_d[b]);
+        P->async_in_d[b] = P->async_out_d[b] = nullptr;
+        if (P->ev_in_ready[b]) cudaEventDestroy(P->ev_in_ready[b]);
+        if (P->ev_buf_free[b]) cudaEventDestroy(P->ev_buf_free[b]);
+        P->ev_in_ready[b] = P->ev_buf_free[b] = nullptr;
+      }
+    };
+    bool ok = true;
+    for (int b = 0; b < 2 && ok; ++b)
+      ok = cudaMalloc(&P->async_in_d[b], P->in_bytes) == cudaSuccess &&
+           cudaMalloc(&P->async_out_d[b], P->out_bytes) == cudaSuccess;
+    for (int b = 0; b < 2 && ok; ++b)
+      ok = cudaEventCreateWithFlags(&P->ev_in_ready[b], cudaEventDisableTiming) == cudaSuccess &&
+           cudaEventCreateWithFlags(&P->ev_buf_free[b], cudaEventDisableTiming) == cudaSuccess;
+    cudaStream_t cs = nullptr;
+    if (ok) ok = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) == cudaSuccess;
+    if (!ok) {
+      release();
+      return set_err(TEMCO_ERR_OUT_OF_MEMORY, "async staging buffers / events / copy stream");
     }
+    P->copy_stream = cs;
   }
   const int b = P->async_flip;
   P->async_flip ^= 1;
@@ -940,6 +976,27 @@ temco_status temco_run_profiled(temco_plan_t P, const void* input, void* output,
   }
   for (auto& e : ev) cudaEventDestroy(e);
   return st;
+}
+
+temco_status temco_debug_step_output(temco_plan_t P, const void* input, void* output, temco_stream_t stream,
+                                     int32_t step, void* host_dst, int64_t capacity, int64_t* bytes) {
+  temco_status st = check_device(P);
+  if (st != TEMCO_OK) return st;
+  if (!input || !output || !bytes || step < 0 || step >= (int32_t)P->exec.size())
+    return set_err(TEMCO_ERR_INVALID_ARGUMENT, "bad step-output arguments");
+  const int id = P->ir.steps[step].out;
+  const Loc l = P->loc.count(id) ? P->loc.at(id) : Loc{W_INPUT, 0, 0};
+  const int64_t need = tensor_bytes(P, id);
+  *bytes = need;
+  if (!host_dst) return TEMCO_OK;   // size query
+  if (capacity < need) return set_err(TEMCO_ERR_INVALID_ARGUMENT, "host buffer too small for the step output");
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  st = enqueue(P, input, output, s, nullptr, step);
+  if (st != TEMCO_OK) return st;
+  const void* src = loc_ptr(l, run_ptrs(P, input, output));
+  CUDA_TRY(cudaMemcpyAsync(host_dst, src, need, cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  return TEMCO_OK;
 }
 
 temco_status temco_peak_internal_bytes(temco_plan_t P, int32_t which, int64_t* bytes) {

@@ -32,8 +32,8 @@ FLAG_MMA_SMALL = 1 << 7
 FLAG_MMA_CAT = 1 << 8
 
 EXPORTS = ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_peak_internal_bytes", "temco_output_shape",
-           "temco_plan_describe", "temco_run_profiled", "temco_plan_destroy", "temco_status_string",
-           "temco_last_error"]
+           "temco_plan_describe", "temco_run_profiled", "temco_debug_step_output", "temco_plan_destroy",
+           "temco_status_string", "temco_last_error"]
 
 _fp = C.POINTER(C.c_float)
 
@@ -66,6 +66,8 @@ _lib.temco_run_host.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
 _lib.temco_run_host_async.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p]
 _lib.temco_run_profiled.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, _fp, C.c_int32]
 _lib.temco_peak_internal_bytes.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_int64)]
+_lib.temco_debug_step_output.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p,
+                                         C.c_int64, C.POINTER(C.c_int64)]
 _lib.temco_output_shape.argtypes = [C.c_void_p, C.POINTER(C.c_int64), C.POINTER(C.c_int32)]
 _lib.temco_plan_describe.argtypes = [C.c_void_p, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]
 _lib.temco_plan_destroy.argtypes = [C.c_void_p]
@@ -73,7 +75,7 @@ _lib.temco_status_string.argtypes = [C.c_int]
 _lib.temco_status_string.restype = C.c_char_p
 _lib.temco_last_error.restype = C.c_char_p
 for _f in ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_run_profiled", "temco_peak_internal_bytes",
-           "temco_output_shape", "temco_plan_describe", "temco_plan_destroy"]:
+           "temco_output_shape", "temco_plan_describe", "temco_debug_step_output", "temco_plan_destroy"]:
     getattr(_lib, _f).restype = C.c_int
 
 
@@ -210,6 +212,19 @@ class Plan:
         _check(_lib.temco_run_profiled(self._h, C.c_void_p(x.data_ptr()), C.c_void_p(y.data_ptr()),
                                        _stream_handle(stream), ms, n), "temco_run_profiled")
         return list(ms)
+
+    def step_output(self, x, y, step, stream=None):
+        """Run schedule steps 0..step and return that step's output tensor as raw
+        bytes (NHWC, plan dtype; fp32 for the graph output) -- a verification hook."""
+        nb = C.c_int64(0)
+        xs, ys = C.c_void_p(x.data_ptr()), C.c_void_p(y.data_ptr())
+        _check(_lib.temco_debug_step_output(self._h, xs, ys, _stream_handle(stream), step, None, 0, C.byref(nb)),
+               "temco_debug_step_output")
+        buf = np.empty(nb.value, np.uint8)
+        _check(_lib.temco_debug_step_output(self._h, xs, ys, _stream_handle(stream), step,
+                                            buf.ctypes.data_as(C.c_void_p), nb.value, C.byref(nb)),
+               "temco_debug_step_output")
+        return buf
 
     def close(self):
         if getattr(self, "_h", None):

@@ -159,3 +159,16 @@ def test_run_host_async_pipeline_matches_device_run():
     s.synchronize()
     for k in range(3):
         assert np.array_equal(yh[k].numpy(), refs[k])
+
+
+def test_fp32_resnet18c_survey_parity_case():
+    """SURVEY 8(d) C2 fp32 parity case: ResNet-18 (CIFAR) at 32x32, batch 8, fp32 mode
+    (SIMT kernels, no TF32) within 1e-4 relative L2 of the fp64 oracle."""
+    m = W.resnet18_cifar(batch=8, dtype="f32", height=32, width=32)
+    x = W.make_input(m)
+    p, y = _plan_and_run(m, x=x)
+    o = oracle.plan(m)
+    ref = oracle.run_temco(o, x)
+    assert np.isfinite(y).all()
+    assert _rel(y, ref) <= 1e-4, _rel(y, ref)
+    assert p.peak_internal_bytes(0) == o.peak_fused

@@ -1,0 +1,83 @@
+"""Per-step GPU parity at full model size: every tensor the TeMCO schedule
+materialises (each fused group's reduced output, each core conv, the logits) is
+compared element by element with the oracle, for one image at the full
+BASELINE.json resolution of every config.
+
+TeMCO rewrites the graph without changing what any schedule step computes
+(the copied restore layers of P:L263 / Fig. 8 recompute exactly the
+tensor the skip used to carry), so each step of S has a well-defined reference
+value.  Comparing every step (not only the GAP'd logits) catches localized spatial
+errors that a global average pool would divide by H*W.
+
+Two comparisons per step (bf16 storage, fp32 accumulation; both sides see the same
+bf16-representable weights and input):
+  * isolated: the oracle's step evaluated on the GPU's own (bf16) input tensors of
+    that step -- only this step's arithmetic differs, so the bar is tight:
+    relative L2 <= 1e-2 and max |err| <= 3e-2 * max |ref|;
+  * chained: the oracle's full fp64 run -- intermediate tensors carry the rounding
+    of every earlier step (a VGG-16-CP layer alone rounds 4 times), so the sanity
+    bar is relative L2 <= 4e-2; the model output keeps the north-star 2e-2
+    (test_gpu_parity.py::test_full_config_sampled).
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from oracle.execute import run_step
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+CONFIGS = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121"]
+
+
+def _to_f64(raw, shape):
+    n = int(np.prod(shape))
+    if raw.size == 4 * n:
+        return raw.view(np.float32).astype(np.float64).reshape(shape)
+    u = raw.view(np.uint16).astype(np.uint32) << 16
+    return u.view(np.float32).astype(np.float64).reshape(shape)
+
+
+def _rel(a, b):
+    return float(np.linalg.norm(a - b) / max(np.linalg.norm(b), 1e-30))
+
+
+@pytest.mark.parametrize("name", CONFIGS)
+def test_every_step_full_size_one_image(name):
+    from paper_conf_icpp_songljkj0024_b200 import Plan
+    m = W.build_config(name, batch=1)
+    x = W.make_input(m)
+    o = oracle.plan(m)
+    chained = {}
+    oracle.run_temco(o, x, on_step=lambda t, v: chained.__setitem__(t, v))
+    p = Plan(m)
+    steps = p.describe()["steps"]
+    assert len(steps) == len(o.steps)
+    xt = torch.from_numpy(x).cuda().to(torch.bfloat16)
+    y = torch.empty(p.output_shape(), dtype=torch.float32, device="cuda")
+    gpu = {o.steps[0].out: np.asarray(x, np.float64)}      # tensors by id, as the GPU holds them
+    worst_iso = worst_chain = (0.0, None)
+    checked = 0
+    for t, s in enumerate(steps):
+        if s["kernel"] == "none":
+            continue
+        ref_chain = chained[t]
+        got = _to_f64(p.step_output(xt, y, t), ref_chain.shape)
+        assert np.isfinite(got).all(), (name, t, s["kernel"])
+        ref_iso = run_step(o, t, gpu)
+        iso = _rel(got, ref_iso)
+        mx = float(np.abs(got - ref_iso).max() / max(np.abs(ref_iso).max(), 1e-30))
+        assert iso <= 1e-2, (name, t, s["kernel"], s["out"], "isolated rel L2", iso)
+        assert mx <= 3e-2, (name, t, s["kernel"], s["out"], "isolated max-abs / max", mx)
+        ch = _rel(got, ref_chain)
+        assert ch <= 4e-2, (name, t, s["kernel"], s["out"], "chained rel L2", ch)
+        worst_iso = max(worst_iso, (iso, (t, s["kernel"])))
+        worst_chain = max(worst_chain, (ch, (t, s["kernel"])))
+        gpu[s["out"]] = got
+        checked += 1
+    assert checked >= 10
+    print(f"{name}: {checked} steps; worst isolated rel L2 {worst_iso[0]:.2e} at {worst_iso[1]}, "
+          f"worst chained {worst_chain[0]:.2e} at {worst_chain[1]}")

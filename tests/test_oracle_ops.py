@@ -73,3 +73,25 @@ def test_pools_bn_linear_match_torch():
     np.testing.assert_allclose(ops.linear(x, wl, bl)[:, 0, 0, :], ref.numpy(), rtol=1e-12, atol=1e-12)
     np.testing.assert_allclose(ops.relu(x), np.where(x > 0, x, 0))
     np.testing.assert_allclose(ops.silu(x), _nhwc(F.silu(_nchw(x))), rtol=1e-12, atol=1e-12)
+
+
+def test_add_and_concat_match_torch_with_channel_order():
+    """ops.add is the elementwise sum of all inputs; ops.concat stacks channels in
+    input order (Fig. 9 concat split: the first input's channels come first)."""
+    rng = np.random.default_rng(3)
+    xs = [rng.standard_normal((2, 5, 4, c)) for c in (3, 5, 2)]
+    got = ops.concat(xs)
+    ref = torch.cat([_nchw(x) for x in xs], dim=1)
+    np.testing.assert_array_equal(got, _nhwc(ref))
+    # channel order pinned by distinct constants per input
+    cs = [np.full((1, 2, 2, c), float(k + 1)) for k, c in enumerate((3, 5, 2))]
+    cat = ops.concat(cs)
+    assert cat.shape == (1, 2, 2, 10)
+    np.testing.assert_array_equal(cat[0, 0, 0], [1, 1, 1, 2, 2, 2, 2, 2, 3, 3])
+    same = [rng.standard_normal((2, 5, 4, 6)) for _ in range(3)]
+    np.testing.assert_allclose(ops.add(same), _nhwc(torch.stack([_nchw(x) for x in same]).sum(0)), rtol=1e-14)
+    np.testing.assert_allclose(ops.add(same[:2]), same[0] + same[1], rtol=0, atol=0)
+    # ops.add does not alias or modify its first input
+    before = same[0].copy()
+    ops.add(same)
+    np.testing.assert_array_equal(same[0], before)

@@ -96,3 +96,23 @@ def test_silu_plans(name):
     p, o = _compare(m)
     assert any(s["kind"] == "group" and "silu" in s["op"] for s in p.describe()["steps"]) or \
         any(st.kind == "group" for st in o.steps)
+
+
+@pytest.mark.parametrize("name", FULL + ["t3", "t4"])
+def test_step_flops_match_oracle(name):
+    """The C++ planner's per-node FLOP counts (node_flops, reading R1) equal the
+    oracle's graph.flops for every node of every schedule step (the numbers
+    Overhead compares; graph.flops itself is pinned by hand counts in
+    test_oracle_flops.py)."""
+    from oracle.graph import flops
+    m = W.build_config(name) if name in FULL else SMALL[name]()
+    p = Plan(m, flags=FLAG_NO_DEVICE)
+    o = oracle.plan(m)
+    g = o.graph
+    nodes = dict(g.nodes_by_id)
+    nodes.update(o.onodes)
+    g2 = type(g)(nodes=g.nodes, output=g.output, batch=g.batch, dtype=g.dtype, orig_flops=g.orig_flops,
+                 nodes_by_id=nodes)
+    for s in p.describe()["steps"]:
+        want = sum(flops(g2, nodes[i]) for i in s["members"] if nodes[i].op != "input")
+        assert s["flops"] == want, (name, s["out"], s["flops"], want)
