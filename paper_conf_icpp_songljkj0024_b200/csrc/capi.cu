@@ -18,8 +18,8 @@
 #include "tc.h"
 #include "tc_wide.h"
 #include "pair.h"
+#include "gemm.h"
 
-#include <cublas_v2.h>
 
 using namespace temco;
 
@@ -38,7 +38,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR };
+enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM };
 
 struct StepExec {
   int kind = K_NONE;
@@ -49,6 +49,7 @@ struct StepExec {
   TcChainDesc tc{};
   wide::TcChainDesc tcw{};
   pair::PairDesc pr{};
+  GemmDesc gm{};
   ConvTcDesc ctc{};
   MmaChainDesc mma{};
   RankConvDesc rk{};
@@ -80,8 +81,7 @@ struct temco_plan_s {
   int32_t* gchild_d = nullptr;
   uint16_t* tcw_d = nullptr;
   char* arena_d = nullptr;
-  cublasHandle_t blas = nullptr;   // plain library GEMMs (the classifier head)
-  float* lin_ws_d = nullptr;       // fp32 GEMM result before the bias / ReLU / cast epilogue
+  float* lin_ws_d = nullptr;       // fp32 split-K partials of the tcgen05 GEMM steps
   int64_t lin_ws_elems = 0;
   int64_t arena_bytes = 0;
   int64_t in_bytes = 0, out_bytes = 0;
@@ -434,27 +434,19 @@ void lower(temco_plan_s* P) {
         if (e.kernel == "simt_conv" && P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && v.w &&
             v.kh == 1 && v.kw == 1 && v.sh == 1 && v.sw == 1 && v.ph == 0 && v.pw == 0 && v.groups == 1 &&
             c.x.dtype == DT_BF16 && c.y.dtype == DT_BF16 && x.C % 8 == 0 && v.C % 8 == 0 && !getenv("TEMCO_NO_CONV_BLAS")) {
-          LinearDesc& l = e.lin;
-          l = LinearDesc{};
-          l.x = c.x;
-          l.y = c.y;
-          l.N = N * x.H * x.W; l.K = x.C; l.O = v.C;
-          l.w = -1;
-          l.b = push_params(P, v.b);
-          l.relu = 0;
-          while (P->tcw_h.size() % 512) P->tcw_h.push_back(0);
-          l.wb = (int64_t)P->tcw_h.size();
-          for (float f : *v.w) {            // OIHW with 1x1 taps = [O][C] row-major
-            uint32_t u;
-            memcpy(&u, &f, 4);
-            u += 0x7FFF + ((u >> 16) & 1);
-            P->tcw_h.push_back((uint16_t)(u >> 16));
+          GemmDesc& g = e.gm;
+          g = GemmDesc{};
+          g.x = c.x;
+          g.y = c.y;
+          g.y2 = Loc{-1, 0, 0};
+          g.M = N * x.H * x.W;
+          g.K = x.C;
+          g.O = v.C;
+          g.relu = 0;
+          if (gemm_lower(g, v.w->data(), v.b ? v.b.get() : nullptr, P->tcw_h, P->params_h, P->lin_ws_elems)) {
+            e.kind = K_GEMM;
+            e.kernel = "tc_gemm_conv1x1";
           }
-          l.blas = l.b >= 0 ? 1 : 2;
-          // (a nonzero workspace also creates the plan's cuBLAS handle)
-          P->lin_ws_elems = std::max<int64_t>(P->lin_ws_elems, l.blas == 1 ? (int64_t)l.N * l.O : 1);
-          e.kind = K_LINEAR;
-          e.kernel = "blas_conv1x1";
         }
         break;
       }
@@ -474,23 +466,24 @@ void lower(temco_plan_s* P) {
         l.w = push_params(P, w);
         l.b = push_params(P, v.b);
         l.relu = 0;
-        l.wb = -1;
-        l.blas = 0;
         e.kind = K_LINEAR;
         e.kernel = "simt_linear";
         if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && l.x.dtype == DT_BF16) {
-          // bf16 plans: the head is a plain GEMM -> cuBLAS (bf16 operands, fp32 accumulate)
-          while (P->tcw_h.size() % 512) P->tcw_h.push_back(0);
-          l.wb = (int64_t)P->tcw_h.size();
-          for (float f : w) {
-            uint32_t u;
-            memcpy(&u, &f, 4);
-            u += 0x7FFF + ((u >> 16) & 1);
-            P->tcw_h.push_back((uint16_t)(u >> 16));
+          // bf16 plans: the head is a GEMM on the tcgen05 kernel (fused bias; a following
+          // standalone ReLU step is produced by the same epilogue as a second output)
+          GemmDesc& g = e.gm;
+          g = GemmDesc{};
+          g.x = l.x;
+          g.y = l.y;
+          g.y2 = Loc{-1, 0, 0};
+          g.M = l.N;
+          g.K = l.K;
+          g.O = l.O;
+          g.relu = 0;
+          if (gemm_lower(g, w.data(), v.b ? v.b.get() : nullptr, P->tcw_h, P->params_h, P->lin_ws_elems)) {
+            e.kind = K_GEMM;
+            e.kernel = "tc_gemm";
           }
-          l.blas = 1;
-          P->lin_ws_elems = std::max<int64_t>(P->lin_ws_elems, (int64_t)l.N * l.O);
-          e.kernel = "blas_linear";
         }
         e.launches = 1;
         break;
@@ -591,6 +584,7 @@ std::string make_json(const temco_plan_s* P) {
         o << ",\"alg_flops\":" << e.pr.alg_flops << ",\"alg_bytes\":" << e.pr.alg_bytes << ",\"tc\":{\"variant\":\"pair\",\"stages\":"
           << e.pr.stages << ",\"smem\":" << e.pr.smem_bytes << ",\"ntiles\":" << e.pr.ntiles << ",\"units\":" << e.pr.nunits
           << ",\"levels\":" << e.pr.n_levels << ",\"terms\":" << e.pr.n_terms << "}";
+      if (e.kind == K_GEMM) o << ",\"alg_flops\":" << e.gm.alg_flops << ",\"alg_bytes\":" << e.gm.alg_bytes << ",\"splits\":" << e.gm.splits;
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_CONV_RK) o << ",\"alg_flops\":" << e.rk.alg_flops << ",\"alg_bytes\":" << e.rk.alg_bytes;
       if (e.kind == K_GROUP_CAT) o << ",\"alg_flops\":" << e.cat.alg_flops << ",\"alg_bytes\":" << e.cat.alg_bytes;
@@ -630,7 +624,6 @@ void free_device(temco_plan_s* P) {
   }
   if (P->copy_stream) cudaStreamDestroy(P->copy_stream);
   cudaFree(P->lin_ws_d);
-  if (P->blas) cublasDestroy(P->blas);
 }
 
 }  // namespace
@@ -668,34 +661,12 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
           launch_conv(e.conv, rp, st);
         break;
       case K_EW: launch_ew(e.ew, rp, st); break;
-      case K_LINEAR:
-        if (e.lin.blas) {
-          // y = W x: column-major C[O x N] = W^T[O x K] * x[K x N] (W row-major [O][K], x row-major [N][K])
-          const float one = 1.f, zero = 0.f;
-          const void* xin = loc_ptr(e.lin.x, rp);
-          if (e.lin.blas == 2) {   // 1x1 conv without bias: bf16 output straight into y
-            if (cublasSetStream(P->blas, st) != CUBLAS_STATUS_SUCCESS ||
-                cublasGemmEx(P->blas, CUBLAS_OP_T, CUBLAS_OP_N, e.lin.O, e.lin.N, e.lin.K, &one, P->tcw_d + e.lin.wb,
-                             CUDA_R_16BF, e.lin.K, xin, CUDA_R_16BF, e.lin.K, &zero,
-                             const_cast<void*>(loc_ptr(e.lin.y, rp)), CUDA_R_16BF, e.lin.O, CUBLAS_COMPUTE_32F,
-                             CUBLAS_GEMM_DEFAULT) != CUBLAS_STATUS_SUCCESS)
-              return set_err(TEMCO_ERR_CUDA, "cublasGemmEx (1x1 conv)");
-            break;
-          }
-          if (cublasSetStream(P->blas, st) != CUBLAS_STATUS_SUCCESS ||
-              cublasGemmEx(P->blas, CUBLAS_OP_T, CUBLAS_OP_N, e.lin.O, e.lin.N, e.lin.K, &one, P->tcw_d + e.lin.wb,
-                           CUDA_R_16BF, e.lin.K, xin, CUDA_R_16BF, e.lin.K, &zero, P->lin_ws_d, CUDA_R_32F, e.lin.O,
-                           CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT) != CUBLAS_STATUS_SUCCESS)
-            return set_err(TEMCO_ERR_CUDA, "cublasGemmEx (classifier head)");
-          launch_linear_epilogue(e.lin, P->lin_ws_d, rp, st);
-        } else {
-          launch_linear(e.lin, rp, st);
-        }
-        break;
+      case K_LINEAR: launch_linear(e.lin, rp, st); break;
       case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
       case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
       case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
       case K_GROUP_PAIR: pair::launch_pair_chain(e.pr, rp, st); break;
+      case K_GEMM: launch_gemm(e.gm, rp, P->lin_ws_d, st); break;
       case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
       case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
       case K_GROUP_CAT: launch_mma_cat(e.cat, P->tcw_d, rp, st); break;
@@ -815,11 +786,6 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
         delete P;
         return set_err(TEMCO_ERR_OUT_OF_MEMORY, "GEMM workspace cudaMalloc");
       }
-      if (cublasCreate(&P->blas) != CUBLAS_STATUS_SUCCESS) {
-        free_device(P);
-        delete P;
-        return set_err(TEMCO_ERR_CUDA, "cublasCreate");
-      }
     }
     std::string terr;
     for (auto& e : P->exec)
@@ -843,6 +809,12 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
       delete P;
       return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
     }
+    for (auto& e : P->exec)
+      if (e.kind == K_GEMM && !gemm_finalize(e.gm, P->arena_d, P->tcw_d, terr)) {
+        free_device(P);
+        delete P;
+        return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
+      }
     if (!pair::pair_finalize(P->exec.size(), [&](size_t i) -> pair::PairDesc* {
           return P->exec[i].kind == K_GROUP_PAIR ? &P->exec[i].pr : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {

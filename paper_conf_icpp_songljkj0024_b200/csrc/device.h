@@ -144,9 +144,7 @@ struct LinearDesc {           // y[n, o] = b[o] + sum_k W[o, k] x[n, k], x flatt
   Loc x, y;
   int32_t N, K, O;
   int64_t w, b;               // params offsets; W already permuted to NHWC order
-  int32_t relu;               // fused ReLU epilogue (a following standalone relu is folded in)
-  int64_t wb;                 // bf16 plans: tc weight pool offset of the bf16 copy of W (cuBLAS GEMM), -1 none
-  int32_t blas;               // 1: y = epilogue(cublasGemmEx(W, x)) (plain library GEMM, fp32 accumulate)
+  int32_t relu;               // fused ReLU epilogue
 };
 
 // ---------------------------------------------------------------------------

@@ -33,7 +33,6 @@ void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_linear(const LinearDesc& d, const RunPtrs& p, cudaStream_t s);
 // bias + ReLU + cast of the fp32 GEMM result ws [N x O] into y
-void launch_linear_epilogue(const LinearDesc& d, const float* ws, const RunPtrs& p, cudaStream_t s);
 void launch_group_simt(const GroupDesc& d, const GNode* nodes, const int32_t* children, const RunPtrs& p,
                        cudaStream_t s);
 

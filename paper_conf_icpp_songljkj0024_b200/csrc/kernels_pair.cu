@@ -196,6 +196,7 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   // 200+ KB of shared memory, so per-level global bias loads would each cost an L2 trip
   d.bias_bytes = (d.n_levels * d.Cpad * 4 + 1023) / 1024 * 1024;
   if (d.bias_mma) d.bias_bytes = 0;
+  d.nbuf = std::min(3, (512 - d.Np) / kPairWu);   // 3 for Np <= 128, 2 for Np <= 256
   const int budget = 227 * 1024 - 1024 /*align*/ - kBarBytes - 2 * kPBytes - d.bias_bytes - kOnesBytes;
   d.slot = kSlotA + 2 * kSlotB + (d.bias_mma ? 2 * kSlotC : 0);
   d.stages = std::min(8, budget / d.slot);
@@ -351,13 +352,14 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   uint64_t* bars = reinterpret_cast<uint64_t*>(ones + kOnesBytes + d.bias_bytes);
   uint64_t* full = bars;               // [S]  leader: producer expect_tx + both CTAs' TMA bytes
   uint64_t* empty = bars + 8;          // [S]  each CTA: MMA commit (multicast)
-  uint64_t* acc_full = bars + 16;      // [2]  each CTA: unit u's level accumulator written (multicast)
-  uint64_t* acc_empty = bars + 18;     // [2]  leader: 32 epilogue warps loaded it
-  uint64_t* p_full = bars + 20;        //      leader: 32 warps wrote P of both units
-  uint64_t* p_empty = bars + 21;       //      each CTA: fconv MMAs read P (multicast)
-  uint64_t* out_full = bars + 22;      //      each CTA: out accumulated (multicast)
-  uint64_t* out_empty = bars + 23;     //      leader: 32 warps drained out
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 24);
+  uint64_t* acc_full = bars + 16;      // [NB] each CTA: a (unit, level) accumulator written (multicast)
+  uint64_t* acc_empty = bars + 20;     // [NB] leader: 32 epilogue warps loaded it
+  uint64_t* p_full = bars + 24;        //      leader: 32 warps wrote P of both units
+  uint64_t* p_empty = bars + 25;       //      each CTA: fconv MMAs read P (multicast)
+  uint64_t* out_full = bars + 26;      //      each CTA: out accumulated (multicast)
+  uint64_t* out_empty = bars + 27;     //      leader: 32 warps drained out
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 28);
+  const int NB = d.nbuf;               // rotating 128-column accumulators: item i -> buffer i % NB
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t cta = cluster_ctarank();
   if (warp == kProdWarp && lane == 0) {
@@ -365,7 +367,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       mbar_init(&full[i], 1);
       mbar_init(&empty[i], 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NB; ++i) {
       mbar_init(&acc_full[i], 1);
       mbar_init(&acc_empty[i], 2 * kEpiWarps);
     }
@@ -410,7 +412,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   // compile-time constant keeps the issuer's accumulator addresses in uniform registers
   if (*tslot != 0u) __trap();
   constexpr uint32_t tbase = 0;
-  constexpr uint32_t tout = tbase + 256u;   // out region [256, 256 + Np)
+  const uint32_t tout = tbase + (uint32_t)(NB * kPairWu);   // out region [128 NB, 128 NB + Np)
   pdl_wait();
 
   const int pair_id = blockIdx.x >> 1, npairs = gridDim.x >> 1;
@@ -492,7 +494,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       const uint64_t ones_d = umma_desc_k(smem_u32(ones), 16);
       int stage = 0;
       uint32_t ph = 0;
-      int na0 = 0, na1 = 0;   // uses of each unit's accumulator (scalars: no local-memory array)
+      int gi = 0;             // (unit, level) accumulator items issued
       int nf = 0;             // pair fconvs issued
       int it = 0;             // tiles whose out region was started
 // fconv of unit pair pp: out (+)= P_u F_u^T for its units; the first pair of a tile starts
@@ -542,12 +544,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             for (int c0 = 0; c0 < nat; c0 += kChunk) {
               const int cn = min(kChunk, nat - c0);
               for (int q = 0; q < nu; ++q) {
-                const int na = q ? na1 : na0;
-                if (c0 == 0 && na > 0) {   // the unit's accumulator must have been drained
-                  mbar_wait_u(&acc_empty[q], (uint32_t)(na - 1) & 1u);
+                const int item = gi + q, b = item % NB, use = item / NB;
+                if (c0 == 0 && use > 0) {   // the buffer's previous item must have been drained
+                  mbar_wait_u(&acc_empty[b], (uint32_t)(use - 1) & 1u);
                   tc_fence_after();
                 }
-                const uint32_t dt = tbase + (uint32_t)(q * kPairWu);
+                const uint32_t dt = tbase + (uint32_t)(b * kPairWu);
                 int st = stage;
                 uint32_t sph = ph;
                 for (int i = 0; i < cn; ++i) {
@@ -571,10 +573,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                   if (++st == S) st = 0, sph ^= 1;
                 }
                 if (c0 + cn == nat) {
-                  mma2_commit_mc_w(&acc_full[q], 3);
+                  mma2_commit_mc_w(&acc_full[b], 3);
                   EV(3);
-                  if (q) ++na1;
-                  else ++na0;
                 }
               }
               for (int i = 0; i < cn; ++i) {
@@ -582,6 +582,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                 if (++stage == S) stage = 0, ph ^= 1;
               }
             }
+            gi += nu;
             if (first_level && pend >= 0) {
               PAIR_FCONV(pend, pend_tile_first, pend_tile_last);
               pend = -1;
@@ -607,7 +608,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     const uint32_t pfull_c = mapa_shared(smem_u32(p_full), 0);
     const uint32_t oempty_c = mapa_shared(smem_u32(out_empty), 0);
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
-    int nacc[2] = {0, 0}, np = 0, it = 0;
+    int gi = 0, np = 0, it = 0;   // gi: (unit, level) accumulator items consumed
     EVDECL();
     const bool ev0 = warp == kEpiWarp0 && lane == 0;
     for (int tile = pair_id; tile < d.ntiles; tile += npairs, ++it) {
@@ -621,27 +622,27 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           for (int qq = 0; qq < 2; ++qq) {
             if (qq < nu) {
               const float* bl = d.bias_mma ? nullptr : sbias + l * d.Cpad + (2 * pp + qq) * kPairWu + g * 32;
-              mbar_wait(&acc_full[qq], (uint32_t)nacc[qq] & 1u);
+              const int item = gi + qq, b = item % NB;
+              mbar_wait(&acc_full[b], (uint32_t)(item / NB) & 1u);
               if (ev0) EV(qq ? 8 : 5);
               tc_fence_after();
               uint32_t v[32];
 #ifdef TEMCO_TRACE
               if (g_pdbg & 2) {
-                warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[qq]), 0));
-                ++nacc[qq];
+                warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[b]), 0));
                 continue;
               }
 #endif
-              tmem_ld32(tbase + lane_off + (uint32_t)(qq * kPairWu + g * 32), v);
+              tmem_ld32(tbase + lane_off + (uint32_t)(b * kPairWu + g * 32), v);
               tmem_wait_ld();
               tc_fence_before();
-              warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[qq]), 0));
-              ++nacc[qq];
+              warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[b]), 0));
               if (ev0 && !qq) EV(6);
               level_math<SILU>(qq ? t1 : t0, v, l == 0, act, bl);
               if (ev0) EV(qq ? 9 : 7);
             }
           }
+          gi += nu;
         }
         // P = t_D (already bf16x2) of both units for the pair's fconv
         if (np > 0) mbar_wait(p_empty, (uint32_t)(np - 1) & 1u);

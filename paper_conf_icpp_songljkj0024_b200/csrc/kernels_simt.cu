@@ -829,22 +829,6 @@ void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   conv_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
 }
 
-__global__ void linear_epilogue_kernel(LinearDesc d, const float* ws, RunPtrs p) {
-  void* y = const_cast<void*>(loc_ptr(d.y, p));
-  const int64_t total = (int64_t)d.N * d.O;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-    const int o = (int)(i % d.O);
-    float v = ws[i] + (d.b >= 0 ? p.params[d.b + o] : 0.f);
-    if (d.relu) v = fmaxf(v, 0.f);
-    stv(y, i, v, d.y.dtype);
-  }
-}
-
-void launch_linear_epilogue(const LinearDesc& d, const float* ws, const RunPtrs& p, cudaStream_t s) {
-  const int64_t total = (int64_t)d.N * d.O;
-  linear_epilogue_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, ws, p);
-}
-
 bool dwconv_vec_ok(const ConvDesc& d) {
   return d.groups == d.C && d.K == d.C && d.C % 8 == 0 && d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.w2 >= 0 &&
          d.kh * d.kw <= 9;

@@ -45,6 +45,7 @@ SMALL = {
     "resnet50_s": lambda dt: W.resnet50(batch=2, dtype=dt, height=64, width=64),
     "vgg16_s": lambda dt: W.vgg16_cp(batch=2, dtype=dt, height=32, width=32),
     "densenet121_s": lambda dt: W.densenet121(batch=2, dtype=dt, height=64, width=64),
+    "alexnet_s": lambda dt: W.alexnet(batch=2, dtype=dt, height=127, width=127),
 }
 
 
@@ -82,7 +83,8 @@ def test_ragged_batch_and_tiles():
     assert _rel(y, ref) <= 2e-2
 
 
-FULL = {"resnet18_cifar": [0, 77, 127], "resnet50": [0, 255], "vgg16_cp": [0, 255], "densenet121": [0, 127]}
+FULL = {"resnet18_cifar": [0, 77, 127], "resnet50": [0, 255], "vgg16_cp": [0, 255], "densenet121": [0, 127],
+        "alexnet": [0, 255]}
 
 
 @pytest.mark.parametrize("name", list(FULL))

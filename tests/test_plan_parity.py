@@ -17,7 +17,7 @@ SMALL = {
     "t2_3": lambda: W.t2_stem_blocks(3), "t3": W.t3_mini_bottleneck, "t4": W.t4_mini_densenet,
     "c1_bf16": lambda: W.c1_basic_block(dtype="bf16", batch=3),
 }
-FULL = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121"]
+FULL = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet"]
 
 
 def _compare(m, flags=0, **okw):
@@ -44,7 +44,9 @@ def test_small_graphs(name):
 def test_full_configs(name):
     m = W.build_config(name)
     p, o = _compare(m)
-    assert 1 - p.peak_internal_bytes(0) / p.peak_internal_bytes(1) >= 0.70
+    # the north-star >= 70 % target is stated for the BASELINE.json configs; AlexNet (f2, no
+    # skip connections: activation-layer fusion only, P:L355 reports 49.4 %) reaches 54.9 %
+    assert 1 - p.peak_internal_bytes(0) / p.peak_internal_bytes(1) >= (0.54 if name == "alexnet" else 0.70)
 
 
 @pytest.mark.parametrize("name", ["t2_3", "t3", "t4"])

@@ -404,12 +404,35 @@ def densenet121(batch=128, dtype=BF16, height=224, width=224, seed=404):
     return g.m
 
 
+def alexnet(batch=256, dtype=BF16, height=224, width=224, seed=505):
+    """AlexNet (torchvision layout: 5 convs with bias, ReLU, three 3x3/s2 max pools,
+    classifier 9216-4096-4096-1000; dropout is the identity at inference), every conv
+    Tucker-2 decomposed with R(c) (the paper applies Tucker decomposition to all
+    models).  No skip connections: TeMCO applies activation-layer fusion only (P:L345,
+    P:L355).  At 224x224 the last pool is 6x6, so torchvision's adaptive average pool
+    is the identity and is omitted."""
+    g = _G("alexnet", batch, height, width, 3, dtype, seed)
+    x = g.relu(g.conv(0, 64, 11, 4, 2, bias=True, name="features.0"), "features.1")
+    x = g.maxpool(x, 3, 2, 0, "features.2")
+    x = g.relu(g.conv(x, 192, 5, 1, 2, bias=True, name="features.3"), "features.4")
+    x = g.maxpool(x, 3, 2, 0, "features.5")
+    x = g.relu(g.conv(x, 384, 3, 1, 1, bias=True, name="features.6"), "features.7")
+    x = g.relu(g.conv(x, 256, 3, 1, 1, bias=True, name="features.8"), "features.9")
+    x = g.relu(g.conv(x, 256, 3, 1, 1, bias=True, name="features.10"), "features.11")
+    x = g.maxpool(x, 3, 2, 0, "features.12")
+    x = g.relu(g.linear(x, 4096, "classifier.1", gain=2.0), "classifier.2")
+    x = g.relu(g.linear(x, 4096, "classifier.4", gain=2.0), "classifier.5")
+    g.linear(x, 1000, "classifier.6")
+    return g.m
+
+
 CONFIGS = {
     "c1": lambda **kw: c1_basic_block(**kw),
     "resnet18_cifar": lambda **kw: resnet18_cifar(**kw),
     "resnet50": lambda **kw: resnet50(**kw),
     "vgg16_cp": lambda **kw: vgg16_cp(**kw),
     "densenet121": lambda **kw: densenet121(**kw),
+    "alexnet": lambda **kw: alexnet(**kw),
 }
 
 
