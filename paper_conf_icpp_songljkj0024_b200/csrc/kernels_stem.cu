@@ -105,7 +105,10 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
 #pragma unroll
     for (int e = 0; e < 2; ++e) bias[nt][e] = d.b >= 0 ? p.params[d.b + nt * 8 + 2 * tq + e] : 0.f;
   // both buffers start zeroed: the pad channels and the slack are never written again
-  for (int i = threadIdx.x; i < g.buf; i += kStThreads) reinterpret_cast<uint32_t*>(xs)[i] = 0u;
+  // (2 buffers x g.buf words); the barrier orders the zeroing before the first footprint
+  // store (compute-sanitizer racecheck: the stores of store() overlapped the zeroing)
+  for (int i = threadIdx.x; i < 2 * g.buf; i += kStThreads) reinterpret_cast<uint32_t*>(xs)[i] = 0u;
+  __syncthreads();
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
   const uint4* x4 = reinterpret_cast<const uint4*>(loc_ptr(d.x, p));
   const int rowC = d.W * d.C;            // image row in elements (% 8 == 0)
