@@ -69,7 +69,11 @@ typedef enum {
   TEMCO_OP_MAXPOOL = 7,        /* kernel, stride, pad (-inf padding)                           */
   TEMCO_OP_AVGPOOL = 8,        /* kernel, stride, no padding                                   */
   TEMCO_OP_GLOBAL_AVGPOOL = 9, /* mean over H, W                                               */
-  TEMCO_OP_LINEAR = 10         /* y = flatten_NCHW(x) W^T + b, W [out_channels, C*H*W]          */
+  TEMCO_OP_LINEAR = 10,        /* y = flatten_NCHW(x) W^T + b, W [out_channels, C*H*W]          */
+  TEMCO_OP_CONV_TRANSPOSE2D = 11 /* transposed conv (UNet up-conv): square kernel,
+                                  * stride, pad; H' = (H-1)*stride - 2*pad + kernel; weight
+                                  * [C_in, C_out, k, k] (PyTorch ConvTranspose2d); Tucker-2 only:
+                                  * first [R_in, C_in], core [R_in, R_out, k, k], last [C_out, R_out] */
 } temco_op;
 
 typedef struct {

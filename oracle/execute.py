@@ -20,6 +20,8 @@ def apply(v: Node, xs):
     """One node of L / O on its input tensors (NHWC fp64)."""
     if v.op == "conv":
         return ops.conv2d(xs[0], v.weight, v.bias, (v.sh, v.sw), (v.ph, v.pw), v.groups)
+    if v.op == "convt":
+        return ops.conv_transpose2d(xs[0], v.weight, v.bias, v.sh, v.ph)
     if v.op == "bn":
         g, b, m, var, eps = v.bn
         return ops.batchnorm(xs[0], g, b, m, var, eps)

@@ -131,6 +131,32 @@ def expand(model) -> Graph:
                          weight=np.asarray(d.last)[:, :, None, None], bias=layer.bias)
             else:
                 raise ValueError(d.kind)
+        elif layer.op == "conv_transpose":
+            # UNet up-conv, Tucker-2 like a conv (fconv -> core ->
+            # lconv); the core is the transposed conv on the reduced channels
+            x = src[0]
+            k, s, p = layer.kernel, layer.stride, layer.pad
+            ho, wo = (x.H - 1) * s - 2 * p + k, (x.W - 1) * s - 2 * p + k
+            orig_flops[li] = 2 * x.C * layer.out_channels * k * k * x.H * x.W * model.batch
+            d = model.decomps.get(li)
+            if d is None:
+                n = push(op="convt", inputs=ins, orig=li, name=layer.name, kh=k, kw=k, sh=s, sw=s, ph=p, pw=p,
+                         C=layer.out_channels, H=ho, W=wo, weight=layer.weight, bias=layer.bias)
+            else:
+                assert d.kind == "tucker2"
+                cur = x
+                if d.first is not None:
+                    cur = push(op="conv", inputs=[cur.id], role="fconv", orig=li, name=layer.name + ".fconv",
+                               C=d.rank_in, H=cur.H, W=cur.W, weight=np.asarray(d.first)[:, :, None, None])
+                has_last = d.last is not None
+                cur = push(op="convt", inputs=[cur.id], role="core", orig=li, name=layer.name + ".core",
+                           kh=k, kw=k, sh=s, sw=s, ph=p, pw=p, C=d.rank_out, H=ho, W=wo,
+                           weight=np.asarray(d.core), bias=None if has_last else layer.bias)
+                if has_last:
+                    cur = push(op="conv", inputs=[cur.id], role="lconv", orig=li, name=layer.name + ".lconv",
+                               C=layer.out_channels, H=ho, W=wo,
+                               weight=np.asarray(d.last)[:, :, None, None], bias=layer.bias)
+                n = cur
         elif layer.op == "bn":
             x = src[0]
             n = push(op="bn", inputs=ins, orig=li, name=layer.name, C=x.C, H=x.H, W=x.W,
@@ -171,7 +197,8 @@ def expand(model) -> Graph:
 
 def flops(g: Graph, v: Node) -> int:
     """FLOPs of one node of L or O at the graph's batch (reading R1): conv
-    2*(C_in/groups)*C_out*kh*kw*H'*W'; bn 2/elt; relu, add 1/elt (per extra
+    2*(C_in/groups)*C_out*kh*kw*H'*W'; transposed conv 2*C_in*C_out*kh*kw*H*W (per input
+    pixel); bn 2/elt; relu, add 1/elt (per extra
     input); silu 4/elt; pools kh*kw per output elt; concat 0; gap 1 per input
     elt; linear 2*in*out."""
     N = g.batch
@@ -179,6 +206,9 @@ def flops(g: Graph, v: Node) -> int:
     if v.op == "conv":
         cin = g.nodes_by_id[v.inputs[0]].C
         return 2 * (cin // v.groups) * v.C * v.kh * v.kw * v.H * v.W * N
+    if v.op == "convt":
+        x = g.nodes_by_id[v.inputs[0]]
+        return 2 * x.C * v.C * v.kh * v.kw * x.H * x.W * N
     if v.op == "bn":
         return 2 * numel
     if v.op == "relu":

@@ -49,6 +49,26 @@ def conv2d(x, w, bias, stride, pad, groups):
     return out
 
 
+def conv_transpose2d(x, w, bias, stride, pad):
+    """Transposed convolution (UNet up-conv): every input pixel scatters through every
+    tap, out[n, ih*s + i - p, iw*s + j - p, o] += sum_c x[n, ih, iw, c] * w[c, o, i, j]
+    (w in PyTorch ConvTranspose2d layout [C_in, C_out, kh, kw]); then the p-border is
+    cropped.  Output size (H - 1) * s - 2p + k."""
+    n, h, wd, c = x.shape
+    ci, o, kh, kw = w.shape
+    assert ci == c
+    s, p = stride, pad
+    full = np.zeros((n, (h - 1) * s + kh, (wd - 1) * s + kw, o), np.float64)
+    w = np.asarray(w, np.float64)
+    for i in range(kh):
+        for j in range(kw):
+            full[:, i:i + s * (h - 1) + 1:s, j:j + s * (wd - 1) + 1:s, :] += x @ w[:, :, i, j]
+    out = full[:, p:full.shape[1] - p, p:full.shape[2] - p, :]
+    if bias is not None:
+        out = out + np.asarray(bias, np.float64)
+    return np.ascontiguousarray(out)
+
+
 def batchnorm(x, gamma, beta, mean, var, eps):
     """y = gamma * (x - mean) / sqrt(var + eps) + beta, per channel."""
     g = np.asarray(gamma, np.float64)

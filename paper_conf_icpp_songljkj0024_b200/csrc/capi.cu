@@ -38,7 +38,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM };
+enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM };
 
 struct StepExec {
   int kind = K_NONE;
@@ -450,6 +450,51 @@ void lower(temco_plan_s* P) {
         }
         break;
       }
+      case OP_CONVT: {
+        const Node& x = ir.nodes[ir.oin[s.out][0]];
+        ConvDesc& c = e.conv;
+        c.x = tensor_loc(P, x.id);
+        c.y = tensor_loc(P, s.out);
+        c.N = N; c.H = x.H; c.W = x.W; c.C = x.C;
+        c.Ho = v.H; c.Wo = v.W; c.K = v.C;
+        c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = 1;
+        // W [C][K][kh][kw] (ConvTranspose2d layout) -> [kh*kw][K][C]
+        std::vector<float> w((size_t)v.kh * v.kw * v.C * x.C);
+        const std::vector<float>& src = *v.w;
+        for (int ci = 0; ci < x.C; ++ci)
+          for (int o = 0; o < v.C; ++o)
+            for (int t = 0; t < v.kh * v.kw; ++t)
+              w[((size_t)t * v.C + o) * x.C + ci] = src[((size_t)ci * v.C + o) * v.kh * v.kw + t];
+        c.w = push_params(P, w);
+        c.b = push_params(P, v.b);
+        c.w2 = -1;
+        e.kind = K_CONVT;
+        e.kernel = "simt_conv_transpose";
+        e.launches = 1;
+        // k x k / stride k, no padding (the UNet up-conv): one GEMM x[NHW, C] W'[k*k*K, C]^T whose
+        // epilogue stores column (i*k + j)*K + o at output pixel (h*k + i, w*k + j)
+        if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && v.kh == v.sh && v.kw == v.sw && v.kh == v.kw &&
+            v.ph == 0 && v.pw == 0 && x.C % 8 == 0 && c.x.dtype == DT_BF16 && c.y.dtype == DT_BF16) {
+          GemmDesc& g = e.gm;
+          g = GemmDesc{};
+          g.x = c.x;
+          g.y = c.y;
+          g.y2 = Loc{-1, 0, 0};
+          g.M = N * x.H * x.W;
+          g.K = x.C;
+          g.O = v.kh * v.kw * v.C;
+          g.shuffle_k = v.kh;
+          g.sh_H = x.H; g.sh_W = x.W; g.sh_Co = v.C;
+          std::vector<float> bias_t;
+          if (v.b)
+            for (int t = 0; t < v.kh * v.kw; ++t) bias_t.insert(bias_t.end(), v.b->begin(), v.b->end());
+          if (gemm_lower(g, w.data(), v.b ? &bias_t : nullptr, P->tcw_h, P->params_h, P->lin_ws_elems)) {
+            e.kind = K_GEMM;
+            e.kernel = "tc_gemm_convt";
+          }
+        }
+        break;
+      }
       case OP_LINEAR: {
         const Node& x = ir.nodes[ir.oin[s.out][0]];
         LinearDesc& l = e.lin;
@@ -648,6 +693,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t], st));
     switch (e.kind) {
       case K_NONE: break;
+      case K_CONVT: launch_conv_transpose(e.conv, rp, st); break;
       case K_CONV:
         if (e.stem)
           launch_conv_stem(e.conv, rp, st);

@@ -49,6 +49,10 @@ struct PLevel {
   bool relu = false;
   bool silu = false;           // SiLU activation of the level, only with allow_silu
   std::vector<PMember> pm;
+  // only with allow_member_act: per-channel activation of activated concat members
+  // (UNet decoder: concat(relu(bn(lconv(skip))), lconv(up-conv))); -1 = the level's own
+  // activation, 1 ReLU, 2 SiLU, 0 none.  Empty: every channel takes the level activation.
+  std::vector<int> act_ch;
 };
 
 struct ChainParser {
@@ -58,6 +62,7 @@ struct ChainParser {
   std::set<int> visited;
   int H, W;
   bool allow_silu = false;     // set by lowerers whose kernels apply PLevel::silu
+  bool allow_member_act = false;   // set by lowerers whose kernels apply PLevel::act_ch
 
   bool chain(int v, std::vector<PLevel>& out) {
     if (!members.count(v)) return false;
@@ -165,8 +170,18 @@ struct ChainParser {
         [[fallthrough]];
       case OP_RELU: {
         // a previous chain value t_{l-1}: unit scale, full width, at most one
-        if (sc || c0 != 0 || n.C != C || !prev.empty()) return false;
-        return chain(v, prev);
+        if (!(sc || c0 != 0 || n.C != C || !prev.empty())) return chain(v, prev);
+        // an activated member of a concat (channels [c0, c0 + n.C)): act(linear), its own
+        // terms and bias inside this level, the activation recorded per channel
+        if (!allow_member_act || sc || (c0 == 0 && n.C == C)) return false;
+        std::vector<PTerm> terms;
+        std::vector<double> b(n.C, 0.0);
+        if (!linear(ir.oin[v][0], nullptr, c0, n.H, n.W, terms, b, 0)) return false;
+        for (PTerm& t : terms) L.terms.push_back(std::move(t));
+        for (int c = 0; c < n.C; ++c) L.bias[c0 + c] += b[c];
+        if (L.act_ch.empty()) L.act_ch.assign(C, -1);
+        for (int c = 0; c < n.C; ++c) L.act_ch[c0 + c] = n.op == OP_RELU ? 1 : 2;
+        return true;
       }
       case OP_MAXPOOL:
       case OP_AVGPOOL: {

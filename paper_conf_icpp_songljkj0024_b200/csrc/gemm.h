@@ -28,6 +28,9 @@ struct GemmDesc {
   int64_t w;                             // tc weight pool offset of W (elements)
   int64_t b;                             // fp32 params offset of the bias, -1 none
   int32_t relu;                          // act on y itself
+  // pixel-shuffle store (a k x k / stride-k transposed conv as one GEMM, UNet up-conv core):
+  // row m = (n, h, w) of an H x W input, column (i*k + j)*Co + o -> y[n, h*k+i, w*k+j, o]
+  int32_t shuffle_k, sh_H, sh_W, sh_Co;
   int32_t splits, kper;                  // split-K: K atoms per split
   int32_t stages, smem_bytes;
   int64_t alg_flops, alg_bytes;

@@ -13,6 +13,8 @@
 namespace temco {
 
 void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
+// transposed conv (UNet up-conv core): d.w = fp32 [kh*kw][K][C] (tap, out, in)
+void launch_conv_transpose(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_small_ok(const ConvDesc& d);   // small-Cin direct conv applies (stem on the image)
 void launch_conv_small(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_stem_ok(const ConvDesc& d);    // bf16 small-Cin conv on tensor cores (mma.sync, kernels_stem.cu)
@@ -32,7 +34,6 @@ bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf
 void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_ew(const EwDesc& d, const RunPtrs& p, cudaStream_t s);
 void launch_linear(const LinearDesc& d, const RunPtrs& p, cudaStream_t s);
-// bias + ReLU + cast of the fp32 GEMM result ws [N x O] into y
 void launch_group_simt(const GroupDesc& d, const GNode* nodes, const int32_t* children, const RunPtrs& p,
                        cudaStream_t s);
 

@@ -96,6 +96,16 @@ bool gemm_finalize(GemmDesc& d, char* arena, uint16_t* tcw, std::string& err) {
 namespace {
 using namespace ptx;
 
+// output element index of GEMM entry (m, o): row-major [M x O], or the pixel-shuffle
+// position of a stride-k transposed conv
+__device__ __forceinline__ int64_t out_index(const GemmDesc& d, int64_t m, int o) {
+  if (!d.shuffle_k) return m * d.O + o;
+  const int k = d.shuffle_k;
+  const int tap = o / d.sh_Co, oc = o - tap * d.sh_Co, i = tap / k, j = tap - i * k;
+  const int64_t w = m % d.sh_W, t = m / d.sh_W, h = t % d.sh_H, n = t / d.sh_H;
+  return (((n * d.sh_H * k + h * k + i) * (int64_t)d.sh_W * k) + w * k + j) * d.sh_Co + oc;
+}
+
 __device__ __forceinline__ void store_out(void* y, int dtype, int64_t i, float v) {
   if (dtype == DT_F32)
     static_cast<float*>(y)[i] = v;
@@ -186,8 +196,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1) gemm_kernel(const __grid_cons
       if (o >= d.O) break;
       float x = __uint_as_float(v[i]) + (d.b >= 0 ? p.params[d.b + o] : 0.f);
       if (d.relu) x = fmaxf(x, 0.f);
-      store_out(y, d.y.dtype, (int64_t)m * d.O + o, x);
-      if (y2) store_out(y2, d.y2.dtype, (int64_t)m * d.O + o, fmaxf(x, 0.f));
+      store_out(y, d.y.dtype, out_index(d, m, o), x);
+      if (y2) store_out(y2, d.y2.dtype, out_index(d, m, o), fmaxf(x, 0.f));
     }
   }
   tc_fence_before();
@@ -210,8 +220,8 @@ __global__ void gemm_reduce_kernel(const __grid_constant__ GemmDesc d, RunPtrs p
     float x = d.b >= 0 ? p.params[d.b + o] : 0.f;
     for (int s = 0; s < d.splits; ++s) x += ws[((int64_t)s * d.M + m) * d.Opad + o];
     if (d.relu) x = fmaxf(x, 0.f);
-    store_out(y, d.y.dtype, i, x);
-    if (y2) store_out(y2, d.y2.dtype, i, fmaxf(x, 0.f));
+    store_out(y, d.y.dtype, out_index(d, m, o), x);
+    if (y2) store_out(y2, d.y2.dtype, out_index(d, m, o), fmaxf(x, 0.f));
   }
 }
 

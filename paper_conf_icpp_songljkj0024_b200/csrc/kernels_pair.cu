@@ -75,6 +75,7 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   if (Nout % 8 || (Nout + 15) / 16 * 16 > 256) return false;
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
   P.allow_silu = true;
+  P.allow_member_act = true;
   P.members.erase(s.out);
   std::vector<PLevel> levels;
   if (!P.chain(tsrc, levels)) return false;
@@ -83,7 +84,7 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   for (auto& L : levels) {
     if (!L.pm.empty()) return false;
     for (auto& t : L.terms) {
-      if (t.tk != 1 || t.c0 != 0 || ir.nodes[t.lconv].C != C) return false;   // full-width plain terms
+      if (t.tk != 1) return false;   // plain terms (a concat member covers its channel range only)
       const int r = ir.oin[t.lconv][0];
       const Loc& l = loc.at(r);
       const Node& rn = ir.nodes[r];
@@ -110,11 +111,26 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   int64_t flops = 0, bytes = 0;
   while (params.size() % 4) params.push_back(0.f);
   d.lbias = (int64_t)params.size();
+  d.ngroups = d.Cpad / 32;
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
     d.act[l] = L.relu ? 1 : L.silu ? 2 : 0;
     d.silu |= L.silu ? 1 : 0;
     for (int c = 0; c < d.Cpad; ++c) params.push_back(c < C ? (float)L.bias[c] : 0.f);
+    if (!L.act_ch.empty()) {   // activated concat members: one activation per 32-channel group
+      if (d.n_levels * d.ngroups > kPairMaxActGroups) return false;
+      d.mixed_act = 1;
+    }
+    for (int gi = 0; gi < d.ngroups; ++gi) {
+      int a = -2;
+      for (int c = gi * 32; c < std::min(C, gi * 32 + 32); ++c) {
+        const int ac = L.act_ch.empty() || L.act_ch[c] < 0 ? d.act[l] : L.act_ch[c];
+        if (a == -2) a = ac;
+        else if (a != ac) return false;   // an activation boundary inside a 32-channel group
+        if (ac == 2) d.silu = 1;
+      }
+      if (l * d.ngroups + gi < kPairMaxActGroups) d.actg[l * d.ngroups + gi] = (uint8_t)(a < 0 ? 0 : a);
+    }
   }
   int j = 0;
   for (int l = 0; l < d.n_levels; ++l) {
@@ -128,11 +144,11 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
       T.aw = R <= 16 ? 16 : R <= 32 ? 32 : 64;
       T.natoms = (R + T.aw - 1) / T.aw;
       T.Rw = (R + 7) / 8 * 8;
-      std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);
-      for (int c = 0; c < C; ++c)
-        for (int k = 0; k < R; ++k) w[(size_t)c * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
+      std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);   // rows outside [c0, c0 + C_term) stay zero
+      for (int c = 0; c < lc.C; ++c)
+        for (int k = 0; k < R; ++k) w[(size_t)(t.c0 + c) * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
       T.w = push_bf16(tcw, w);
-      flops += d.npix * 2LL * C * R;
+      flops += d.npix * 2LL * lc.C * R;
       bytes += d.npix * 2LL * R;
     }
     d.lvl_end[l] = j;
@@ -617,10 +633,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         const int nu = min(2, U - 2 * pp);
         uint32_t t0[16], t1[16];
         for (int l = 0; l < d.n_levels; ++l) {
-          const int act = d.act[l];
 #pragma unroll
           for (int qq = 0; qq < 2; ++qq) {
             if (qq < nu) {
+              const int act = d.mixed_act ? (int)d.actg[l * d.ngroups + (2 * pp + qq) * (kPairWu / 32) + g] : d.act[l];
               const float* bl = d.bias_mma ? nullptr : sbias + l * d.Cpad + (2 * pp + qq) * kPairWu + g * 32;
               const int item = gi + qq, b = item % NB;
               mbar_wait(&acc_full[b], (uint32_t)(item / NB) & 1u);

@@ -829,6 +829,46 @@ void launch_conv(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   conv_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
 }
 
+// transposed convolution: y[n, oh, ow, o] = b[o] + sum over taps (i, j) with oh = ih*sh - ph + i,
+// ow = iw*sw - pw + j of sum_c x[n, ih, iw, c] W[c, o, i, j]; weights packed [i*kw + j][o][c].
+// One thread per output element; the stride-2, 2x2 up-conv cores of UNet meet one tap each.
+__global__ void conv_transpose_kernel(ConvDesc d, RunPtrs p) {
+  const void* x = loc_ptr(d.x, p);
+  void* y = const_cast<void*>(loc_ptr(d.y, p));
+  const float* w = p.params + d.w;
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.K;
+  for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total; idx += (int64_t)gridDim.x * blockDim.x) {
+    const int o = (int)(idx % d.K);
+    int64_t r = idx / d.K;
+    const int ow = (int)(r % d.Wo);
+    r /= d.Wo;
+    const int oh = (int)(r % d.Ho);
+    const int n = (int)(r / d.Ho);
+    float acc = d.b >= 0 ? p.params[d.b + o] : 0.f;
+    for (int i = 0; i < d.kh; ++i) {
+      const int th = oh + d.ph - i;
+      if (th < 0 || th % d.sh) continue;
+      const int ih = th / d.sh;
+      if (ih >= d.H) continue;
+      for (int j = 0; j < d.kw; ++j) {
+        const int tw = ow + d.pw - j;
+        if (tw < 0 || tw % d.sw) continue;
+        const int iw = tw / d.sw;
+        if (iw >= d.W) continue;
+        const int64_t xb = (((int64_t)n * d.H + ih) * d.W + iw) * d.C;
+        const float* wr = w + ((int64_t)(i * d.kw + j) * d.K + o) * d.C;
+        for (int c = 0; c < d.C; ++c) acc += ldv(x, xb + c, d.x.dtype) * wr[c];
+      }
+    }
+    stv(y, idx, acc, d.y.dtype);
+  }
+}
+
+void launch_conv_transpose(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.K;
+  conv_transpose_kernel<<<grid_for(total, 256), 256, 0, s>>>(d, p);
+}
+
 bool dwconv_vec_ok(const ConvDesc& d) {
   return d.groups == d.C && d.K == d.C && d.C % 8 == 0 && d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.w2 >= 0 &&
          d.kh * d.kw <= 9;

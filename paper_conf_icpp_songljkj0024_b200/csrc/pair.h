@@ -34,6 +34,7 @@ namespace pair {
 constexpr int kPairMaxTerms = 16;
 constexpr int kPairMaxLevels = 16;
 constexpr int kPairMaxAtoms = 64;       // K atoms of one unit's level chain
+constexpr int kPairMaxActGroups = 256;  // (level, 32-channel group) activation codes
 constexpr int kPairWu = 128;           // restored channels per unit (MMA N of the restore GEMM)
 
 struct PairTerm {
@@ -53,6 +54,8 @@ struct PairDesc {
   int32_t n_prog;
   int32_t lvl_end[kPairMaxLevels];       // terms [lvl_end[l-1], lvl_end[l]) belong to level l
   int32_t act[kPairMaxLevels];           // 0 none, 1 ReLU, 2 SiLU
+  int32_t mixed_act, ngroups;            // per-channel-group activations (activated concat members)
+  uint8_t actg[kPairMaxActGroups];       // [level][32-channel group] activation code when mixed_act
   int64_t lbias;                         // params offset: fp32 [n_levels][Cpad] level biases
   int32_t bias_mma;                      // level biases added by a K=16 MMA (ones x [hi, lo]) instead of the epilogue
   int64_t bmat;                          // tc weight pool offset of the bias-MMA matrix

@@ -22,6 +22,7 @@ const char* op_name(Op op) {
     case OP_AVGPOOL: return "avgpool";
     case OP_GAP: return "gap";
     case OP_LINEAR: return "linear";
+    case OP_CONVT: return "convt";
   }
   return "?";
 }
@@ -76,7 +77,8 @@ void expand(const temco_layer* layers, int n_layers, const temco_decomp* decomps
   for (int i = 0; i < n_decomps; ++i) {
     const temco_decomp& d = decomps[i];
     if (d.layer <= 0 || d.layer >= n_layers) fail(TEMCO_ERR_INVALID_GRAPH, "decomp refers to a bad layer");
-    if (layers[d.layer].op != TEMCO_OP_CONV2D) fail(TEMCO_ERR_INVALID_GRAPH, "decomp of a non-conv layer");
+    if (layers[d.layer].op != TEMCO_OP_CONV2D && layers[d.layer].op != TEMCO_OP_CONV_TRANSPOSE2D)
+      fail(TEMCO_ERR_INVALID_GRAPH, "decomp of a non-conv layer");
     if (dec[d.layer]) fail(TEMCO_ERR_INVALID_GRAPH, "two decomps for one layer");
     dec[d.layer] = &d;
   }
@@ -199,6 +201,58 @@ void expand(const temco_layer* layers, int n_layers, const temco_decomp* decomps
         } else {
           fail(TEMCO_ERR_INVALID_ARGUMENT, "unknown decomposition kind");
         }
+        break;
+      }
+      case TEMCO_OP_CONV_TRANSPOSE2D: {
+        // transposed conv: out[h*s + i - p, w*s + j - p, o] += x[h, w, c] W[c, o, i, j]
+        need(1);
+        const Node x = ir.nodes[ins[0]];
+        const int k = l.kernel, s = l.stride, p = l.pad;
+        if (k <= 0 || s <= 0 || p < 0 || l.out_channels <= 0 || (l.groups > 1)) fail(TEMCO_ERR_INVALID_GRAPH, "bad conv_transpose params");
+        const int ho = (x.H - 1) * s - 2 * p + k, wo = (x.W - 1) * s - 2 * p + k;
+        if (ho <= 0 || wo <= 0) fail(TEMCO_ERR_INVALID_GRAPH, "conv_transpose output is empty");
+        // original FLOPs (reading R1): every input pixel meets every k x k tap
+        ir.orig_flops[li] = 2LL * x.C * l.out_channels * k * k * (int64_t)x.H * x.W * cfg.batch;
+        const temco_decomp* d = dec[li];
+        if (!d) {
+          if (!l.weight) fail(TEMCO_ERR_INVALID_ARGUMENT, "undecomposed conv_transpose needs a weight");
+          n.op = OP_CONVT; n.kh = n.kw = k; n.sh = n.sw = s; n.ph = n.pw = p;
+          n.C = l.out_channels; n.H = ho; n.W = wo;
+          n.w = copy_buf(l.weight, (size_t)x.C * l.out_channels * k * k);
+          n.b = copy_buf(l.bias, l.out_channels);
+          n.in = ins;
+          out_of[li] = push(n);
+          break;
+        }
+        if (d->kind != TEMCO_DECOMP_TUCKER2) fail(TEMCO_ERR_UNSUPPORTED, "conv_transpose: Tucker-2 decomposition only");
+        const int ri = d->rank_in, ro = d->rank_out;
+        if (ri <= 0 || ro <= 0 || ri > x.C || ro > l.out_channels) fail(TEMCO_ERR_UNSUPPORTED, "bad conv_transpose ranks");
+        if (!d->core || (ri < x.C && !d->first) || (ro < l.out_channels && !d->last))
+          fail(TEMCO_ERR_INVALID_ARGUMENT, "conv_transpose factor is NULL");
+        int cur = ins[0];
+        if (d->first) {
+          Node f; f.op = OP_CONV; f.role = ROLE_FCONV; f.orig = li; f.in = {cur};
+          f.C = ri; f.H = x.H; f.W = x.W;
+          f.w = copy_buf(d->first, (size_t)ri * x.C);
+          cur = push(f);
+        } else if (ri != x.C) {
+          fail(TEMCO_ERR_INVALID_GRAPH, "rank_in != C_in requires a first factor");
+        }
+        Node c; c.op = OP_CONVT; c.role = ROLE_CORE; c.orig = li; c.in = {cur};
+        c.kh = c.kw = k; c.sh = c.sw = s; c.ph = c.pw = p; c.C = ro; c.H = ho; c.W = wo;
+        c.w = copy_buf(d->core, (size_t)ri * ro * k * k);
+        if (!d->last) c.b = copy_buf(l.bias, ro);
+        cur = push(c);
+        if (d->last) {
+          Node q; q.op = OP_CONV; q.role = ROLE_LCONV; q.orig = li; q.in = {cur};
+          q.C = l.out_channels; q.H = ho; q.W = wo;
+          q.w = copy_buf(d->last, (size_t)l.out_channels * ro);
+          q.b = copy_buf(l.bias, l.out_channels);
+          cur = push(q);
+        } else if (ro != l.out_channels) {
+          fail(TEMCO_ERR_INVALID_GRAPH, "rank_out != C_out requires a last factor");
+        }
+        out_of[li] = cur;
         break;
       }
       case TEMCO_OP_BATCHNORM: {
@@ -369,6 +423,10 @@ int64_t node_flops(const IR& ir, int id) {   // reading R1
     case OP_CONV: {
       const Node& x = ir.nodes[v.in[0]];
       return 2LL * (x.C / v.groups) * v.C * v.kh * v.kw * (int64_t)v.H * v.W * N;
+    }
+    case OP_CONVT: {   // per input pixel: C_in x C_out x k x k MACs
+      const Node& x = ir.nodes[v.in[0]];
+      return 2LL * x.C * v.C * v.kh * v.kw * (int64_t)x.H * x.W * N;
     }
     case OP_BN: return 2 * numel;
     case OP_RELU: return numel;

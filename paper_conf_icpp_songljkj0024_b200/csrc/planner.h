@@ -14,7 +14,8 @@
 
 namespace temco {
 
-enum Op { OP_INPUT, OP_CONV, OP_BN, OP_RELU, OP_SILU, OP_ADD, OP_CONCAT, OP_MAXPOOL, OP_AVGPOOL, OP_GAP, OP_LINEAR };
+enum Op { OP_INPUT, OP_CONV, OP_BN, OP_RELU, OP_SILU, OP_ADD, OP_CONCAT, OP_MAXPOOL, OP_AVGPOOL, OP_GAP, OP_LINEAR,
+          OP_CONVT /* transposed conv (UNet up-conv core) */ };
 enum Role { ROLE_NONE, ROLE_FCONV, ROLE_CORE, ROLE_LCONV };
 
 const char* op_name(Op op);

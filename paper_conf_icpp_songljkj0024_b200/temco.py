@@ -19,7 +19,7 @@ if not os.path.exists(_LIB_PATH):
 _lib = C.CDLL(_LIB_PATH)
 
 OPS = {"input": 0, "conv": 1, "bn": 2, "relu": 3, "silu": 4, "add": 5, "concat": 6, "maxpool": 7,
-       "avgpool": 8, "gap": 9, "linear": 10}
+       "avgpool": 8, "gap": 9, "linear": 10, "conv_transpose": 11}
 F32, BF16 = 0, 1
 FLAG_NO_DEVICE = 1 << 0
 FLAG_NO_SKIPOPT = 1 << 1

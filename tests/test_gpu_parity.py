@@ -46,6 +46,7 @@ SMALL = {
     "vgg16_s": lambda dt: W.vgg16_cp(batch=2, dtype=dt, height=32, width=32),
     "densenet121_s": lambda dt: W.densenet121(batch=2, dtype=dt, height=64, width=64),
     "alexnet_s": lambda dt: W.alexnet(batch=2, dtype=dt, height=127, width=127),
+    "unet_s": lambda dt: W.unet(batch=2, dtype=dt, height=32, width=32, base=16),
 }
 
 
@@ -84,7 +85,7 @@ def test_ragged_batch_and_tiles():
 
 
 FULL = {"resnet18_cifar": [0, 77, 127], "resnet50": [0, 255], "vgg16_cp": [0, 255], "densenet121": [0, 127],
-        "alexnet": [0, 255]}
+        "alexnet": [0, 255], "unet": [0, 15]}
 
 
 @pytest.mark.parametrize("name", list(FULL))

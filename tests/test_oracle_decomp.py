@@ -106,3 +106,24 @@ def test_tucker2_omitted_factors_and_bias_placement():
     assert pl.graph.nodes[2].bias is not None
     x = np.random.default_rng(5).standard_normal((2, m.height, m.width, 4))
     np.testing.assert_allclose(oracle.run_unfused(pl, x), _ref(m, W, b, x), rtol=1e-10, atol=1e-10)
+
+
+@pytest.mark.parametrize("cin,cout,k,s,p", [(4, 6, 2, 2, 0), (5, 3, 3, 2, 1)])
+def test_tucker2_full_rank_reconstructs_conv_transpose(cin, cout, k, s, p):
+    """UNet up-conv: the Tucker-2 expansion fconv (V^T) -> transposed core
+    G -> lconv (U) of a ConvTranspose2d weight W [C_in, C_out, k, k], with
+    G[a, b] = sum_{c,o} V[c, a] W[c, o] U[o, b], reproduces torch's conv_transpose2d of W."""
+    rng = np.random.default_rng(9)
+    W = rng.standard_normal((cin, cout, k, k))
+    b = rng.standard_normal(cout)
+    U, V = _orth(rng, cout), _orth(rng, cin)
+    G = np.einsum("ca,cokl,ob->abkl", V, W, U)
+    m = Model("single_t", 2, 5, 4, cin, "f32")
+    m.layers = [Layer("input", [], out_channels=cin),
+                Layer("conv_transpose", [0], out_channels=cout, kernel=k, stride=s, pad=p, weight=W, bias=b)]
+    m.decomps = {1: Decomp(1, "tucker2", cin, cout, V.T.copy(), G, None, U)}
+    x = rng.standard_normal((2, 5, 4, cin))
+    got = oracle.run_unfused(oracle.plan(m), x)
+    t = F.conv_transpose2d(torch.from_numpy(np.transpose(x, (0, 3, 1, 2))), torch.from_numpy(W),
+                           torch.from_numpy(b), stride=s, padding=p)
+    np.testing.assert_allclose(got, np.transpose(t.numpy(), (0, 2, 3, 1)), rtol=1e-10, atol=1e-10)

@@ -95,3 +95,30 @@ def test_add_and_concat_match_torch_with_channel_order():
     before = same[0].copy()
     ops.add(same)
     np.testing.assert_array_equal(same[0], before)
+
+
+@pytest.mark.parametrize("c,o,k,s,p", [(4, 6, 2, 2, 0), (3, 5, 3, 2, 1), (6, 4, 4, 2, 1), (5, 5, 3, 1, 1)])
+def test_conv_transpose2d_matches_torch(c, o, k, s, p):
+    rng = np.random.default_rng(7)
+    x = rng.standard_normal((2, 5, 6, c))
+    w = rng.standard_normal((c, o, k, k))
+    b = rng.standard_normal(o)
+    got = ops.conv_transpose2d(x, w, b, s, p)
+    ref = F.conv_transpose2d(_nchw(x), torch.from_numpy(w), torch.from_numpy(b), stride=s, padding=p)
+    np.testing.assert_allclose(got, _nhwc(ref), rtol=1e-12, atol=1e-12)
+
+
+def test_conv_transpose2d_literal_loop():
+    """The scatter definition written as plain loops on a tiny input."""
+    rng = np.random.default_rng(8)
+    x = rng.standard_normal((1, 2, 3, 2))
+    w = rng.standard_normal((2, 3, 3, 3))
+    s, p = 2, 1
+    got = ops.conv_transpose2d(x, w, None, s, p)
+    ho, wo = (2 - 1) * s - 2 * p + 3, (3 - 1) * s - 2 * p + 3
+    ref = np.zeros((1, ho, wo, 3))
+    for ih, iw, ci, oc, i, j in itertools.product(range(2), range(3), range(2), range(3), range(3), range(3)):
+        oh, ow = ih * s - p + i, iw * s - p + j
+        if 0 <= oh < ho and 0 <= ow < wo:
+            ref[0, oh, ow, oc] += x[0, ih, iw, ci] * w[ci, oc, i, j]
+    np.testing.assert_allclose(got, ref, rtol=1e-12, atol=1e-12)

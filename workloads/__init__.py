@@ -10,5 +10,5 @@ consume what it produces, independently.
 from .models import (  # noqa: F401
     Layer, Decomp, Model, rank_rule, bf16_round, skip_edges, make_input,
     c1_basic_block, t1_chain, t2_stem_blocks, t3_mini_bottleneck, t4_mini_densenet,
-    resnet18_cifar, resnet50, vgg16_cp, densenet121, alexnet, CONFIGS, build_config,
+    resnet18_cifar, resnet50, vgg16_cp, densenet121, alexnet, unet, CONFIGS, build_config,
 )

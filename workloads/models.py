@@ -190,6 +190,23 @@ class _G:
         wo = (w + 2 * p - k) // s + 1
         return self._add(layer, (cout, ho, wo))
 
+    def conv_transpose(self, x, cout, k, s, p=0, bias=False, name=""):
+        """ConvTranspose2d (UNet up-conv), Tucker-2 decomposed with R(c): first [R_in, C_in],
+        core [R_in, R_out, k, k] (transposed-conv layout), last [C_out, R_out]."""
+        cin, h, w = self.shape[x]
+        rng = self.rng()
+        idx = len(self.m.layers)
+        b = self._q(rng.normal(0.0, 0.01, cout).astype(np.float32)) if bias else None
+        layer = Layer("conv_transpose", [x], name=name, out_channels=cout, kernel=k, stride=s, pad=p, bias=b)
+        ri, ro = min(self.rank(cin), cin), min(self.rank(cout), cout)
+        first = self._orth(rng, cin, ri).T if ri < cin else None
+        # each output pixel meets ~ (k/s)^2 taps of R_in channels
+        core = rng.standard_normal((ri, ro, k, k)) / np.sqrt(ri * max(1.0, (k / s) ** 2))
+        last = self._orth(rng, cout, ro) * np.sqrt(cout / ro) if ro < cout else None
+        self.m.decomps[idx] = Decomp(idx, "tucker2", ri, ro, None if first is None else self._q(first),
+                                     self._q(core), None, None if last is None else self._q(last))
+        return self._add(layer, (cout, (h - 1) * s - 2 * p + k, (w - 1) * s - 2 * p + k))
+
     def bn(self, x, name=""):
         c, h, w = self.shape[x]
         rng = self.rng()
@@ -426,6 +443,32 @@ def alexnet(batch=256, dtype=BF16, height=224, width=224, seed=505):
     return g.m
 
 
+def unet(batch=16, dtype=BF16, height=256, width=256, seed=606, base=64, n_classes=2):
+    """UNet (Ronneberger et al. [34], the paper's segmentation model, P:L126 / P:L345 / P:L355):
+    four down blocks (2x2 max pool + DoubleConv), four up blocks (2x2 / stride-2 transposed
+    conv "up-conv" + channel concat with the encoder feature of the same resolution +
+    DoubleConv), DoubleConv = (3x3 conv (no bias) -> BN -> ReLU) x 2, 1x1 output conv to
+    n_classes (Carvana masks).  Every conv and up-conv Tucker-2 decomposed with R(c).  The
+    encoder features x1..x4 are the long-range skips (76.2 % of the decomposed model's peak
+    in the paper's Fig. 4a).  Shape only: the paper's Carvana images are matched in shape."""
+    g = _G("unet", batch, height, width, 3, dtype, seed)
+
+    def dconv(x, c, name):
+        x = g.relu(g.bn(g.conv(x, c, 3, 1, 1, name=f"{name}.conv1"), f"{name}.bn1"), f"{name}.relu1")
+        return g.relu(g.bn(g.conv(x, c, 3, 1, 1, name=f"{name}.conv2"), f"{name}.bn2"), f"{name}.relu2")
+
+    c = [base, base * 2, base * 4, base * 8, base * 16]
+    xs = [dconv(0, c[0], "inc")]
+    for i in range(1, 5):
+        xs.append(dconv(g.maxpool(xs[-1], 2, 2, 0, f"down{i}.pool"), c[i], f"down{i}"))
+    x = xs[4]
+    for i in range(3, -1, -1):
+        u = g.conv_transpose(x, c[i], 2, 2, 0, bias=True, name=f"up{4 - i}.upconv")
+        x = dconv(g.concat([xs[i], u], f"up{4 - i}.cat"), c[i], f"up{4 - i}")
+    g.conv(x, n_classes, 1, 1, 0, bias=True, name="outc")
+    return g.m
+
+
 CONFIGS = {
     "c1": lambda **kw: c1_basic_block(**kw),
     "resnet18_cifar": lambda **kw: resnet18_cifar(**kw),
@@ -433,6 +476,7 @@ CONFIGS = {
     "vgg16_cp": lambda **kw: vgg16_cp(**kw),
     "densenet121": lambda **kw: densenet121(**kw),
     "alexnet": lambda **kw: alexnet(**kw),
+    "unet": lambda **kw: unet(**kw),
 }
 
 
