@@ -317,7 +317,7 @@ def main():
     classes = {}
     for s, t in zip(steps, prof):
         k = s["kernel"]
-        if k == "none":
+        if s["launches"] == 0:      # "none" (the input) and steps produced by another step's epilogue
             continue
         c = classes.setdefault(k, {"ms": 0.0, "flops": 0, "bytes": 0, "launches": 0})
         c["ms"] += float(t)

@@ -569,6 +569,19 @@ void lower(temco_plan_s* P) {
       }
     }
   }
+  // a standalone ReLU right after a GEMM head layer (AlexNet / VGG FC stacks): the GEMM
+  // epilogue writes it as a second output, the ReLU step launches nothing
+  for (size_t t = 0; t + 1 < ir.steps.size(); ++t) {
+    StepExec& e = P->exec[t];
+    StepExec& r = P->exec[t + 1];
+    const Step& s1 = ir.steps[t + 1];
+    if (e.kind != K_GEMM || e.gm.shuffle_k || e.gm.relu || r.kind != K_EW || s1.group) continue;
+    if (ir.nodes[s1.out].op != OP_RELU || ir.oin[s1.out].size() != 1 || ir.oin[s1.out][0] != ir.steps[t].out) continue;
+    e.gm.y2 = tensor_loc(P, s1.out);
+    r.kind = K_NONE;
+    r.kernel = "in_gemm";
+    r.launches = 0;
+  }
 }
 
 void json_ints(std::ostringstream& o, const std::vector<int>& v) {

@@ -18,7 +18,7 @@
 namespace temco {
 
 struct ConvTcDesc {
-  alignas(64) unsigned char wmap[128];   // CUtensorMap of W [Np x Kp], box {64, Np}
+  alignas(64) unsigned char wmap[128];   // CUtensorMap of W [nsl*Np x Kp], box {64, Np}
   alignas(64) unsigned char xmap[128];   // TMA mode: 4D map of x [N, H, W, Cin], box {64, tw*s, th*s, tn}
   // TMA mode (Cin % 8 == 0): output tiles are spatial boxes tn x th x tw (<= 128
   // pixels); tap (a, b) of 64-channel atom kc is one tap-shifted, strided box
@@ -29,6 +29,10 @@ struct ConvTcDesc {
   int32_t N, H, W, Cin;
   int32_t Ho, Wo, kh, kw, sh, sw, ph, pw;
   int32_t Nout, Np;
+  // output-channel slices (blockIdx.y): slice j computes channels [j*Nsl, min(Nout, (j+1)*Nsl))
+  // with its own resident weight block (rows [j*Np, (j+1)*Np) of W), so wide-K cores whose
+  // full weight matrix exceeds the SMEM budget still run on the tensor cores
+  int32_t nsl, Nsl;
   int32_t vec;            // 1: Cin % 8 == 0 (16-byte chunks per tap); 0: element gather
   int32_t K, kchunks;     // GEMM K (kh*kw*Cin) and 16-byte chunks of it
   int32_t katoms;         // 64-wide K atoms

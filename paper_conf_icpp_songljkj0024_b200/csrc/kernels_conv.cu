@@ -38,14 +38,13 @@ bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::ve
   const Loc& xl = loc.at(x.id);
   const Loc& yl = loc.at(out);
   if (xl.dtype != DT_BF16 || yl.dtype != DT_BF16 || yl.where != W_ARENA) return false;
-  if (v.C % 8 || v.C > 256) return false;
+  if (v.C % 8) return false;
   d = ConvTcDesc();
   d.x = xl;
   d.y = yl;
   d.N = ir.batch; d.H = x.H; d.W = x.W; d.Cin = x.C;
   d.Ho = v.H; d.Wo = v.W; d.kh = v.kh; d.kw = v.kw; d.sh = v.sh; d.sw = v.sw; d.ph = v.ph; d.pw = v.pw;
   d.Nout = v.C;
-  d.Np = (v.C + 15) / 16 * 16;
   d.vec = x.C % 8 == 0 ? 1 : 0;
   d.K = v.kh * v.kw * x.C;
   d.kchunks = (d.K + 7) / 8;
@@ -70,10 +69,17 @@ bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::ve
     if (d.tw * d.s > 256 || d.th * d.s > 256) d.tma = 0;
   }
   if (!d.tma) d.katoms = (d.K + 63) / 64;
+  // fewest output-channel slices whose resident weight block fits the SMEM budget
+  for (d.nsl = (v.C + 255) / 256;; ++d.nsl) {
+    d.Nsl = ((v.C + d.nsl - 1) / d.nsl + 7) / 8 * 8;
+    d.Np = (d.Nsl + 15) / 16 * 16;
+    if (d.katoms * d.Np * 128 <= 112 * 1024) break;
+    if (d.Nsl <= 8 || d.nsl >= 16) return false;
+  }
+  d.nsl = (v.C + d.Nsl - 1) / d.Nsl;
   const int wbytes = d.katoms * d.Np * 128;
-  if (wbytes > 112 * 1024) return false;
   const int Kp = d.katoms * 64;
-  std::vector<uint16_t> w((size_t)d.Np * Kp, 0);
+  std::vector<uint16_t> w((size_t)d.nsl * d.Np * Kp, 0);
   const std::vector<float>& src = *v.w;   // OIHW
   for (int o = 0; o < v.C; ++o)
     for (int c = 0; c < x.C; ++c)
@@ -82,7 +88,8 @@ bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::ve
           // TMA mode: k = (tap * kpt + c / 64) * 64 + c % 64; gather mode: k = tap * Cin + c
           const int tap = a * v.kw + b;
           const size_t k = d.tma ? (size_t)(tap * d.kpt) * 64 + c : (size_t)tap * x.C + c;
-          w[(size_t)o * Kp + k] = f2bf(src[(((size_t)o * x.C + c) * v.kh + a) * v.kw + b]);
+          const size_t row = (size_t)(o / d.Nsl) * d.Np + o % d.Nsl;
+          w[row * Kp + k] = f2bf(src[(((size_t)o * x.C + c) * v.kh + a) * v.kw + b]);
         }
   while (tcw.size() % 512) tcw.push_back(0);
   d.w = (int64_t)tcw.size();
@@ -115,7 +122,7 @@ bool conv_tc_finalize(ConvTcDesc& d, uint16_t* tcw, std::string& err) {
     encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
   }
   const uint64_t Kp = (uint64_t)d.katoms * 64;
-  cuuint64_t dims[2] = {Kp, (cuuint64_t)d.Np};
+  cuuint64_t dims[2] = {Kp, (cuuint64_t)d.nsl * d.Np};
   cuuint64_t strides[1] = {Kp * 2};
   cuuint32_t box[2] = {64, (cuuint32_t)d.Np};
   cuuint32_t es[2] = {1, 1};
@@ -292,7 +299,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
     // ------------------------------------------------------------ weights + MMA issuer
     if (lane == 0) {
       mbar_expect_tx(wbar, wbytes);
-      for (int kb = 0; kb < d.katoms; ++kb) tma_load_2d(wres + kb * d.Np * 128, d.wmap, wbar, kb * 64, 0);
+      for (int kb = 0; kb < d.katoms; ++kb) tma_load_2d(wres + kb * d.Np * 128, d.wmap, wbar, kb * 64, blockIdx.y * d.Np);
       mbar_wait(wbar, 0);
       int stage = 0;
       uint32_t phase = 0;
@@ -323,6 +330,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
     const int row = threadIdx.x;
     const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+    const int oc0 = blockIdx.y * d.Nsl;
     int it = 0;
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
       const int buf = it & 1;
@@ -333,11 +341,12 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_tc_kernel(const __grid_c
         uint32_t v[8];
         tmem_ld8(tbase + lane_off + buf * d.Np + g * 8, v);
         tmem_wait_ld();
-        if (m < d.npix && g * 8 < d.Nout) {
+        const int o = oc0 + g * 8;
+        if (m < d.npix && g * 8 < d.Nsl && o < d.Nout) {
           float f[8];
 #pragma unroll
-          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.b >= 0 ? __ldg(p.params + d.b + g * 8 + i) : 0.f);
-          *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) =
+          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.b >= 0 ? __ldg(p.params + d.b + o + i) : 0.f);
+          *reinterpret_cast<uint4*>(y + m * d.Nout + o) =
               make_uint4(pack_bf16(f[0], f[1]), pack_bf16(f[2], f[3]), pack_bf16(f[4], f[5]), pack_bf16(f[6], f[7]));
         }
       }
@@ -401,7 +410,7 @@ __global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __gr
   if (warp == 4) {
     if (lane == 0) {
       mbar_expect_tx(wbar, wbytes);
-      for (int kb = 0; kb < d.katoms; ++kb) tma_load_2d(wres + kb * d.Np * 128, d.wmap, wbar, kb * 64, 0);
+      for (int kb = 0; kb < d.katoms; ++kb) tma_load_2d(wres + kb * d.Np * 128, d.wmap, wbar, kb * 64, blockIdx.y * d.Np);
       int stage = 0;
       uint32_t phase = 0;
       const uint32_t bytes = 128u * d.tw * d.th * d.tn;
@@ -450,6 +459,7 @@ __global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __gr
     const int row = threadIdx.x;
     const uint32_t lane_off = (uint32_t)(warp * 32) << 16;
     __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
+    const int oc0 = blockIdx.y * d.Nsl;
     const int wi = row % d.tw, hi = (row / d.tw) % d.th, ni = row / (d.tw * d.th);
     int it = 0;
     for (int tile = blockIdx.x; tile < d.ntiles; tile += gridDim.x, ++it) {
@@ -464,11 +474,12 @@ __global__ void __launch_bounds__(kConvTmaThreads, 1) conv_tma_kernel(const __gr
         uint32_t v[8];
         tmem_ld8(tbase + lane_off + buf * d.Np + g * 8, v);
         tmem_wait_ld();
-        if (valid && g * 8 < d.Nout) {
+        const int o = oc0 + g * 8;
+        if (valid && g * 8 < d.Nsl && o < d.Nout) {
           float f[8];
 #pragma unroll
-          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.b >= 0 ? __ldg(p.params + d.b + g * 8 + i) : 0.f);
-          *reinterpret_cast<uint4*>(y + m * d.Nout + g * 8) =
+          for (int i = 0; i < 8; ++i) f[i] = __uint_as_float(v[i]) + (d.b >= 0 ? __ldg(p.params + d.b + o + i) : 0.f);
+          *reinterpret_cast<uint4*>(y + m * d.Nout + o) =
               make_uint4(pack_bf16(f[0], f[1]), pack_bf16(f[2], f[3]), pack_bf16(f[4], f[5]), pack_bf16(f[6], f[7]));
         }
       }
@@ -497,11 +508,12 @@ void launch_conv_tc(const ConvTcDesc& d, const RunPtrs& p, cudaStream_t s) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
-  const int grid = std::min(d.ntiles, sms > 0 ? sms : 148);   // persistent, one CTA per SM
+  // persistent, one CTA per SM, output-channel slices along y
+  const int grid = std::min(d.ntiles, std::max(1, (sms > 0 ? sms : 148) / d.nsl));
   if (d.tma)
-    launch_pdl(conv_tma_kernel, dim3(grid), dim3(kConvTmaThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
+    launch_pdl(conv_tma_kernel, dim3(grid, d.nsl), dim3(kConvTmaThreads), std::max(d.smem_bytes, 116 * 1024), s, d, p);
   else
-    conv_tc_kernel<<<grid, kConvThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
+    conv_tc_kernel<<<dim3(grid, d.nsl), kConvThreads, std::max(d.smem_bytes, 116 * 1024), s>>>(d, p);
 }
 
 }  // namespace temco

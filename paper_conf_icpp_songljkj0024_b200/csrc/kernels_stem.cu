@@ -26,12 +26,15 @@ namespace temco {
 
 namespace {
 
-constexpr int kStTH = 16, kStTW = 32;   // output tile (rows x cols); 8 warps x 4 m-tiles of 16 pixels
+// output tile (rows x cols): 16 x 32 (8 warps x 4 m-tiles of 16 pixels); strided stems whose
+// 16 x 32 footprint overflows the stage (AlexNet's 11x11 / s4) take 8 x 16 (one m-tile per warp)
+constexpr int kStTH = 16, kStTW = 32;
 constexpr int kStThreads = 256;
 
 constexpr int kStCPT = 6;   // footprint chunks (16 B of an image row) per thread and tile
 
 struct StemGeo {
+  int TH, TW, MPW;        // output tile, m-tiles (16 pixels) per warp
   int Cp, rowK, KS, NT;   // padded channels, elements per kernel row, k-steps, n-tiles
   int PR, PC, rowlen;     // footprint rows / pixels, elements per footprint row
   int ncr;                // 16-byte image-row chunks covering one footprint row
@@ -40,20 +43,24 @@ struct StemGeo {
   int smem;               // bytes (two buffers)
 };
 
-StemGeo stem_geo(const ConvDesc& d) {
+StemGeo stem_geo(const ConvDesc& d, int TH = kStTH, int TW = kStTW) {
   StemGeo g;
+  g.TH = TH;
+  g.TW = TW;
+  g.MPW = TH * TW / 16 / 8;
   g.Cp = (d.C + 1) / 2 * 2;
   g.rowK = d.kw * g.Cp;
   g.KS = (d.kh * g.rowK + 15) / 16;
   g.NT = d.K / 8;
-  g.PR = (kStTH - 1) * d.sh + d.kh;
-  g.PC = (kStTW - 1) * d.sw + d.kw;
+  g.PR = (TH - 1) * d.sh + d.kh;
+  g.PC = (TW - 1) * d.sw + d.kw;
   g.rowlen = g.PC * g.Cp;
   g.ncr = (g.PC * d.C + 7) / 8 + 1;
   g.cmagic = ((1 << 17) + d.C - 1) / d.C;
   // + slack: padded k columns past the last kernel row read (finite) footprint data
   g.buf = (g.PR * g.rowlen + 64) / 2;
-  g.smem = g.buf * 4 * 2;
+  // + SMEM B fragments and k-offsets (long K)
+  g.smem = g.buf * 4 * 2 + (g.KS > 16 ? g.KS * g.NT * 32 * 8 + g.KS * 8 * 4 : 0);
   return g;
 }
 
@@ -78,15 +85,24 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
   const int gq = lane >> 2, tq = lane & 3;
   // ---- per-thread k-pair offsets into a pixel's footprint window and the B fragments
   const float* wf = p.params + d.w;   // fp32 [K][kh][kw][Cin]
-  int off[KS][2];
-  uint32_t bfr[NT][KS][2];
+  // long K (AlexNet's 11x11 stem, 31 k-steps): the B fragments live in SMEM (one LDS.64 per
+  // k-step) instead of 62 registers per n-tile
+  constexpr bool kBs = KS > 16;
+  uint2* bs = reinterpret_cast<uint2*>(reinterpret_cast<uint32_t*>(xs) + 2 * g.buf);
+  int* os = reinterpret_cast<int*>(bs + KS * NT * 32);   // [ks][h][tq]
+  int off[kBs ? 1 : KS][2];
+  uint32_t bfr[kBs ? 1 : NT][kBs ? 1 : KS][2];
 #pragma unroll
   for (int ks = 0; ks < KS; ++ks)
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
       const int k = ks * 16 + 2 * tq + 8 * h;           // even: the pair (k, k+1) shares its kernel row
       const int kr = k / g.rowK, j = k - kr * g.rowK;
-      off[ks][h] = kr < d.kh ? kr * g.rowlen + j : 0;
+      if constexpr (kBs) {
+        if (gq == 0) os[(ks * 2 + h) * 4 + tq] = kr < d.kh ? kr * g.rowlen + j : 0;
+      } else {
+        off[ks][h] = kr < d.kh ? kr * g.rowlen + j : 0;
+      }
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt) {
         const int o = nt * 8 + gq;
@@ -96,7 +112,10 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
           const int jj = j + e, px = jj / g.Cp, c = jj - px * g.Cp;
           w2[e] = (kr < d.kh && c < d.C) ? wf[(((int64_t)o * d.kh + kr) * d.kw + px) * d.C + c] : 0.f;
         }
-        bfr[nt][ks][h] = pack2(w2[0], w2[1]);
+        if constexpr (kBs)
+          reinterpret_cast<uint32_t*>(&bs[(ks * NT + nt) * 32 + lane])[h] = pack2(w2[0], w2[1]);
+        else
+          bfr[nt][ks][h] = pack2(w2[0], w2[1]);
       }
     }
   float bias[NT][2];
@@ -118,7 +137,7 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
   uint4 v[kStCPT];
   auto load = [&](int tile) {
     const int n = tile / (tiles_w * tiles_h);
-    const int h0 = (tile / tiles_w) % tiles_h * kStTH, w0 = tile % tiles_w * kStTW;
+    const int h0 = (tile / tiles_w) % tiles_h * g.TH, w0 = tile % tiles_w * g.TW;
     const int hi0 = h0 * d.sh - d.ph, e0 = (w0 * d.sw - d.pw) * d.C;
     const int a0 = e0 >= 0 ? e0 / 8 : -((7 - e0) / 8);
 #pragma unroll
@@ -131,8 +150,7 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
     }
   };
   auto store = [&](int tile, __nv_bfloat16* buf) {
-    const int h0 = (tile / tiles_w) % tiles_h * kStTH, w0 = tile % tiles_w * kStTW;
-    (void)h0;
+    const int w0 = tile % tiles_w * g.TW;
     const int e0 = (w0 * d.sw - d.pw) * d.C;
     const int a0 = e0 >= 0 ? e0 / 8 : -((7 - e0) / 8);
 #pragma unroll
@@ -163,13 +181,13 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
     store(tile, buf);
     __syncthreads();
     const int n = tile / (tiles_w * tiles_h);
-    const int h0 = (tile / tiles_w) % tiles_h * kStTH, w0 = tile % tiles_w * kStTW;
+    const int h0 = (tile / tiles_w) % tiles_h * g.TH, w0 = tile % tiles_w * g.TW;
     if (tile + (int)gridDim.x < ntiles) load(tile + gridDim.x);   // in flight during the MMAs
     const uint32_t* xw = reinterpret_cast<const uint32_t*>(buf);
-    // ---- 4 m-tiles per warp: output row (warp * 2 + mt / 2), 16 columns (mt & 1)
+    // ---- MPW m-tiles per warp: m-tile gm covers output row gm / (TW / 16), 16 columns
 #pragma unroll 1
-    for (int mt = 0; mt < 4; ++mt) {
-      const int orow = warp * 2 + (mt >> 1), ocol = (mt & 1) * 16;
+    for (int gm = warp * g.MPW; gm < (warp + 1) * g.MPW; ++gm) {
+      const int orow = gm / (g.TW / 16), ocol = gm % (g.TW / 16) * 16;
       const int b0 = (orow * d.sh) * g.rowlen + ((ocol + gq) * d.sw) * g.Cp;     // pixel rows gq, gq + 8
       const int b1 = b0 + 8 * d.sw * g.Cp;
       float acc[NT][4];
@@ -181,12 +199,27 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
 #pragma unroll
       for (int ks = 0; ks < KS; ++ks) {
         uint32_t a[4];
-        a[0] = xw[(b0 + off[ks][0]) >> 1];
-        a[1] = xw[(b1 + off[ks][0]) >> 1];
-        a[2] = xw[(b0 + off[ks][1]) >> 1];
-        a[3] = xw[(b1 + off[ks][1]) >> 1];
+        int o0, o1;
+        if constexpr (kBs) {
+          o0 = os[ks * 8 + tq];
+          o1 = os[ks * 8 + 4 + tq];
+        } else {
+          o0 = off[ks][0];
+          o1 = off[ks][1];
+        }
+        a[0] = xw[(b0 + o0) >> 1];
+        a[1] = xw[(b1 + o0) >> 1];
+        a[2] = xw[(b0 + o1) >> 1];
+        a[3] = xw[(b1 + o1) >> 1];
 #pragma unroll
-        for (int nt = 0; nt < NT; ++nt) mma_bf16_16816(acc[nt], a, bfr[nt][ks][0], bfr[nt][ks][1]);
+        for (int nt = 0; nt < NT; ++nt) {
+          if constexpr (kBs) {
+            const uint2 bb = bs[(ks * NT + nt) * 32 + lane];
+            mma_bf16_16816(acc[nt], a, bb.x, bb.y);
+          } else {
+            mma_bf16_16816(acc[nt], a, bfr[nt][ks][0], bfr[nt][ks][1]);
+          }
+        }
       }
       const int oy = h0 + orow;
       if (oy >= d.Ho) continue;
@@ -216,7 +249,7 @@ void launch_stem_t(const ConvDesc& d, const StemGeo& g, const RunPtrs& p, cudaSt
   }
   int per_sm = 1;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, conv_stem_kernel<KS, NT>, kStThreads, g.smem);
-  const int tw = (d.Wo + kStTW - 1) / kStTW, th = (d.Ho + kStTH - 1) / kStTH;
+  const int tw = (d.Wo + g.TW - 1) / g.TW, th = (d.Ho + g.TH - 1) / g.TH;
   const int ntiles = d.N * tw * th;
   const int grid = std::min(ntiles, sms * std::max(per_sm, 1));
   launch_pdl(conv_stem_kernel<KS, NT>, dim3((unsigned)grid), dim3(kStThreads), g.smem, s, d, g, p, tw, th);
@@ -254,14 +287,22 @@ __global__ void __launch_bounds__(256) conv_pw_small_kernel(ConvDesc d, RunPtrs 
   }
 }
 
+bool stem_fits(const ConvDesc& d, const StemGeo& g) {
+  return g.smem <= 96 * 1024 && g.PR * g.ncr <= kStCPT * kStThreads && g.PC * d.C < 2048;
+}
+
+StemGeo stem_pick(const ConvDesc& d) {
+  const StemGeo g = stem_geo(d);
+  return stem_fits(d, g) ? g : stem_geo(d, 8, 16);
+}
+
 }  // namespace
 
 bool conv_stem_ok(const ConvDesc& d) {
   if (d.x.dtype != DT_BF16 || d.y.dtype != DT_BF16 || d.groups != 1 || d.C > 8 || d.K % 8 || d.sh != d.sw) return false;
-  const StemGeo g = stem_geo(d);
-  const bool shape = (g.NT == 1 || g.NT == 2) && (g.KS == 1 || g.KS == 3 || g.KS == 13);
-  return shape && g.smem <= 96 * 1024 && (d.W * d.C) % 8 == 0 && g.PR * g.ncr <= kStCPT * kStThreads &&
-         g.PC * d.C < 2048;
+  const StemGeo g = stem_pick(d);
+  const bool shape = (g.NT == 1 || g.NT == 2) && (g.KS == 1 || g.KS == 3 || g.KS == 13 || g.KS == 31);
+  return shape && stem_fits(d, g) && (d.W * d.C) % 8 == 0;
 }
 
 void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
@@ -271,7 +312,7 @@ void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
     launch_pdl(conv_pw_small_kernel<3>, dim3(grid), dim3(256), 0, s, d, p);
     return;
   }
-  const StemGeo g = stem_geo(d);
+  const StemGeo g = stem_pick(d);
 #define TEMCO_STEM_CASE(ks, nt) \
   if (g.KS == ks && g.NT == nt) return launch_stem_t<ks, nt>(d, g, p, s);
   TEMCO_STEM_CASE(1, 1)
@@ -280,6 +321,7 @@ void launch_conv_stem(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   TEMCO_STEM_CASE(1, 2)
   TEMCO_STEM_CASE(3, 2)
   TEMCO_STEM_CASE(13, 2)
+  TEMCO_STEM_CASE(31, 1)
 #undef TEMCO_STEM_CASE
 }
 

@@ -45,8 +45,12 @@ SMALL = {
     "resnet50_s": lambda dt: W.resnet50(batch=2, dtype=dt, height=64, width=64),
     "vgg16_s": lambda dt: W.vgg16_cp(batch=2, dtype=dt, height=32, width=32),
     "densenet121_s": lambda dt: W.densenet121(batch=2, dtype=dt, height=64, width=64),
-    "alexnet_s": lambda dt: W.alexnet(batch=2, dtype=dt, height=127, width=127),
-    "unet_s": lambda dt: W.unet(batch=2, dtype=dt, height=32, width=32, base=16),
+    # batch 60 at 224: the 13x13 pooled group has enough pixels (10140, a ragged 256-pixel
+    # pair tile) for the CTA-pair kernel, as at the full batch
+    "alexnet_s": lambda dt: W.alexnet(batch=60, dtype=dt, height=224, width=224),
+    # full width (base 64): the 3x3 cores of the bottom level exceed one SMEM weight block
+    # (output-channel-sliced tc_conv), as in the full config
+    "unet_s": lambda dt: W.unet(batch=2, dtype=dt, height=32, width=32, base=64),
 }
 
 
