@@ -58,7 +58,7 @@ bool gemm_lower(GemmDesc& d, const float* w, const std::vector<float>* bias, std
   d.kper = (katoms + splits - 1) / splits;
   d.splits = (katoms + d.kper - 1) / d.kper;
   if (d.splits > 1) ws_elems = std::max<int64_t>(ws_elems, (int64_t)d.splits * d.M * d.Opad);
-  d.stages = kGemmStages;
+  d.stages = std::max(2, std::min(kGemmStages, d.kper));   // short K: smaller ring, 2 CTAs per SM
   d.smem_bytes = 1024 + d.stages * kStage + 256;
   d.alg_flops = 2LL * d.M * d.K * d.O;
   d.alg_bytes = 2LL * d.M * d.K + 2LL * d.O * d.K + (int64_t)d.M * d.O * (d.y.dtype == DT_F32 ? 4 : 2);
@@ -177,6 +177,8 @@ __global__ void __launch_bounds__(kGemmThreads, 1) gemm_kernel(const __grid_cons
   const uint32_t trow = tbase + ((uint32_t)(warp * 32) << 16);
   void* y = const_cast<void*>(loc_ptr(d.y, p));
   void* y2 = d.y2.where >= 0 ? const_cast<void*>(loc_ptr(d.y2, p)) : nullptr;
+  const bool vec8 = d.y.dtype == DT_BF16 && (y2 == nullptr || d.y2.dtype == DT_BF16) &&
+                    (d.shuffle_k ? d.sh_Co % 8 == 0 : d.O % 8 == 0);
   for (int c = 0; c < kBN; c += 32) {
     uint32_t v[32];
     tmem_ld32(trow + c, v);
@@ -188,6 +190,27 @@ __global__ void __launch_bounds__(kGemmThreads, 1) gemm_kernel(const __grid_cons
       for (int i = 0; i < 8; ++i)
         dst[i] = make_float4(__uint_as_float(v[4 * i]), __uint_as_float(v[4 * i + 1]), __uint_as_float(v[4 * i + 2]),
                              __uint_as_float(v[4 * i + 3]));
+      continue;
+    }
+    if (vec8) {   // bf16 output, 8 consecutive channels per 16-byte store
+#pragma unroll
+      for (int g8 = 0; g8 < 4; ++g8) {
+        const int o = n0 + c + g8 * 8;
+        if (o >= d.O) break;
+        float f[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          f[i] = __uint_as_float(v[g8 * 8 + i]) + (d.b >= 0 ? p.params[d.b + o + i] : 0.f);
+          if (d.relu) f[i] = fmaxf(f[i], 0.f);
+        }
+        const int64_t oi = out_index(d, m, o);
+        *reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(y) + oi) =
+            make_uint4(pack_bf16(f[0], f[1]), pack_bf16(f[2], f[3]), pack_bf16(f[4], f[5]), pack_bf16(f[6], f[7]));
+        if (y2)
+          *reinterpret_cast<uint4*>(static_cast<__nv_bfloat16*>(y2) + oi) =
+              make_uint4(pack_bf16(fmaxf(f[0], 0.f), fmaxf(f[1], 0.f)), pack_bf16(fmaxf(f[2], 0.f), fmaxf(f[3], 0.f)),
+                         pack_bf16(fmaxf(f[4], 0.f), fmaxf(f[5], 0.f)), pack_bf16(fmaxf(f[6], 0.f), fmaxf(f[7], 0.f)));
+      }
       continue;
     }
 #pragma unroll
