@@ -59,7 +59,9 @@ constexpr int kSlotC = 2048;             // 64 rows x 16 bf16 (bias-MMA groups: 
 // ring stage: A + B for both units of a pair (+ C for both with bias-MMA): PairDesc::slot bytes
 constexpr int kOnesBytes = 4096;         // 128 rows x 16 bf16 "ones" A tile of the bias MMA
 constexpr int kPBytes = 128 * kPairWu * 2;   // P of one unit: two SW128 atoms of 128 x 64
-constexpr int kBarBytes = 1024;
+constexpr int kBarBytes = 2048;   // barriers (first 1 KB) + the issuer's atom table (kTabOff)
+constexpr int kTabOff = 1024;
+constexpr int kPairMaxStages = 16;
 constexpr int kChunk = 2;                // ring stages of one level consumed per (u0 pass, u1 pass)
 
 }  // namespace
@@ -214,10 +216,43 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   if (d.bias_mma) d.bias_bytes = 0;
   d.nbuf = std::min(3, (512 - d.Np) / kPairWu);   // 3 for Np <= 128, 2 for Np <= 256
   const int budget = 227 * 1024 - 1024 /*align*/ - kBarBytes - 2 * kPBytes - d.bias_bytes - kOnesBytes;
-  d.slot = kSlotA + 2 * kSlotB + (d.bias_mma ? 2 * kSlotC : 0);
-  d.stages = std::min(8, budget / d.slot);
+  // resident weights: per unit pair pp and program atom k, this CTA's halves of both units'
+  // Lhat atoms; per (pp, level) the bias-MMA atoms; per (unit, 64-channel atom) F
+  {
+    int awmax = 16;
+    for (int jj = 0; jj < d.n_terms; ++jj) awmax = std::max(awmax, (int)d.term[jj].aw);
+    const int UP = (d.nunits + 1) / 2;
+    d.bsz = 64 * awmax * 2;
+    d.fsz = d.Np / 2 * 128;
+    const int rb = UP * d.n_prog * 2 * d.bsz;
+    const int rc = d.bias_mma ? UP * d.n_levels * 2 * kSlotC : 0;
+    const int rf = d.nunits * 2 * d.fsz;
+    d.res_c = (rb + 1023) / 1024 * 1024;
+    d.res_f = d.res_c + (rc + 1023) / 1024 * 1024;
+    d.res_bytes = d.res_f + (rf + 1023) / 1024 * 1024;
+    int64_t tx = 0;
+    for (int pp = 0; pp < UP; ++pp) {
+      const int nu = std::min(2, d.nunits - 2 * pp);
+      for (int k = 0; k < d.n_prog; ++k) tx += nu * 64 * (int)((d.prog[k][0] >> 8) & 0xFF) * 2;
+      if (d.bias_mma) tx += (int64_t)nu * d.n_levels * 64 * 16 * 2;
+    }
+    tx += (int64_t)d.nunits * 2 * d.fsz;
+    d.res_tx = (int)tx;
+    const int slot_r = 128 * awmax * 2;
+    const int st_r = std::min(kPairMaxStages, (budget - d.res_bytes) / slot_r);
+    d.resident = !getenv("TEMCO_PAIR_NO_RES") && st_r >= std::max(8, d.n_prog + 2) ? 1 : 0;
+    if (d.resident) {
+      d.slot = slot_r;
+      d.stages = st_r;
+    }
+  }
+  if (!d.resident) {
+    d.res_bytes = 0;
+    d.slot = kSlotA + 2 * kSlotB + (d.bias_mma ? 2 * kSlotC : 0);
+    d.stages = std::min(8, budget / d.slot);
+  }
   if (d.stages < 2 * kChunk) return false;
-  d.smem_bytes = 1024 + d.stages * d.slot + 2 * kPBytes + d.bias_bytes + kOnesBytes + kBarBytes;
+  d.smem_bytes = 1024 + d.res_bytes + d.stages * d.slot + 2 * kPBytes + d.bias_bytes + kOnesBytes + kBarBytes;
   return true;
 }
 
@@ -280,10 +315,10 @@ using namespace ptx;
 
 #ifdef TEMCO_TRACE
 // experiment builds only: event timeline of CTA 0 (rows: see scripts/pair_timeline.py)
-__device__ long long g_ev[12][512];
+__device__ long long g_ev[16][512];
 __device__ int g_ev_on, g_launch;
 __device__ int g_pdbg;   // timing experiments: 1 = producer issues no TMA, 2 = epilogue skips TMEM / math
-#define EVDECL() int _evn[12] = {0}; const bool _evon = blockIdx.x == 0 && g_launch == g_ev_on
+#define EVDECL() int _evn[16] = {0}; const bool _evon = blockIdx.x == 0 && g_launch == g_ev_on
 #define EV(row)                                                                                   \
   do {                                                                                            \
     if (_evon && _evn[row] < 512) g_ev[row][_evn[row]++] = clock64();                             \
@@ -291,6 +326,14 @@ __device__ int g_pdbg;   // timing experiments: 1 = producer issues no TMA, 2 = 
 #else
 #define EVDECL() ((void)0)
 #define EV(row) ((void)0)
+#endif
+
+// epilogue waits: sleep on the barrier (suspend-time hint) rather than re-issuing
+// try_wait, so 16 waiting warps do not take issue slots from the producer / issuer
+#ifdef TEMCO_PAIR_SPIN
+#define PAIR_EPI_WAIT(b, p) mbar_wait(b, p)
+#else
+#define PAIR_EPI_WAIT(b, p) mbar_wait_sleep(b, p)
 #endif
 
 constexpr int kWarps = 18;
@@ -361,20 +404,22 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   const int S = d.stages, kSlot = d.slot;
-  uint8_t* ring = smem;
-  uint8_t* pbuf = smem + S * kSlot;                                 // P of unit 0 | unit 1 of a pair
+  uint8_t* res = smem;                                              // resident weights (d.resident)
+  uint8_t* ring = smem + d.res_bytes;
+  uint8_t* pbuf = ring + S * kSlot;                                 // P of unit 0 | unit 1 of a pair
   uint8_t* ones = pbuf + 2 * kPBytes;                               // bias-MMA A tile (1024-aligned)
   float* sbias = reinterpret_cast<float*>(ones + kOnesBytes);
   uint64_t* bars = reinterpret_cast<uint64_t*>(ones + kOnesBytes + d.bias_bytes);
   uint64_t* full = bars;               // [S]  leader: producer expect_tx + both CTAs' TMA bytes
-  uint64_t* empty = bars + 8;          // [S]  each CTA: MMA commit (multicast)
-  uint64_t* acc_full = bars + 16;      // [NB] each CTA: a (unit, level) accumulator written (multicast)
-  uint64_t* acc_empty = bars + 20;     // [NB] leader: 32 epilogue warps loaded it
-  uint64_t* p_full = bars + 24;        //      leader: 32 warps wrote P of both units
-  uint64_t* p_empty = bars + 25;       //      each CTA: fconv MMAs read P (multicast)
-  uint64_t* out_full = bars + 26;      //      each CTA: out accumulated (multicast)
-  uint64_t* out_empty = bars + 27;     //      leader: 32 warps drained out
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 28);
+  uint64_t* empty = bars + 16;         // [S]  each CTA: MMA commit (multicast)
+  uint64_t* acc_full = bars + 32;      // [NB] each CTA: a (unit, level) accumulator written (multicast)
+  uint64_t* acc_empty = bars + 36;     // [NB] leader: 32 epilogue warps loaded it
+  uint64_t* p_full = bars + 40;        //      leader: 32 warps wrote P of both units
+  uint64_t* p_empty = bars + 41;       //      each CTA: fconv MMAs read P (multicast)
+  uint64_t* out_full = bars + 42;      //      each CTA: out accumulated (multicast)
+  uint64_t* out_empty = bars + 43;     //      leader: 32 warps drained out
+  uint64_t* wbar = bars + 44;          //      leader: resident weights landed (both CTAs' bytes)
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(bars + 45);
   const int NB = d.nbuf;               // rotating 128-column accumulators: item i -> buffer i % NB
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t cta = cluster_ctarank();
@@ -391,6 +436,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     mbar_init(p_empty, 1);
     mbar_init(out_full, 1);
     mbar_init(out_empty, 2 * kEpiWarps);
+    mbar_init(wbar, 1);
     fence_mbar_init_cluster();
     for (int jj = 0; jj < d.n_terms; ++jj) {
       prefetch_tmap(d.term[jj].amap);
@@ -464,6 +510,27 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       EVDECL();
       int pend = -1;   // pair whose fconv operands follow the next pair's first level
       const uint8_t* term0 = reinterpret_cast<const uint8_t*>(&d.term[0]);
+      if (d.resident) {   // every weight atom of this CTA's halves, once
+        if (cta == 0) mbar_expect_tx(wbar, 2u * (uint32_t)d.res_tx);
+        const uint32_t wb = mapa_shared(smem_u32(wbar), 0);
+        for (int pp = 0; pp < UP; ++pp) {
+          const int u0 = 2 * pp, nu = min(2, U - u0);
+          for (int k = 0; k < d.n_prog; ++k) {
+            const uint2 op = make_uint2(d.prog[k][0], d.prog[k][1]);
+            const PairTerm* T = reinterpret_cast<const PairTerm*>(term0 + (op.x & 0xFF) * sizeof(PairTerm));
+            for (int q = 0; q < nu; ++q) {
+              tma_load_2d_pair(res + ((pp * d.n_prog + k) * 2 + q) * d.bsz, T->wmap, wb, (int)op.y,
+                               (u0 + q) * kPairWu + (int)cta * 64);
+              if (d.bias_mma && ((op.x >> 24) & 1u))
+                tma_load_2d_pair(res + d.res_c + ((pp * d.n_levels + (int)(op.x >> 28)) * 2 + q) * kSlotC, d.bmap, wb, 0,
+                                 (int)(op.x >> 28) * d.Cpad + (u0 + q) * kPairWu + (int)cta * 64);
+            }
+          }
+        }
+        for (int u = 0; u < U; ++u)
+          for (int a = 0; a < kPairWu / 64; ++a)
+            tma_load_2d_pair(res + d.res_f + (u * 2 + a) * d.fsz, d.fmap, wb, u * kPairWu + a * 64, (int)cta * (d.Np / 2));
+      }
       for (int tile = pair_id; tile < d.ntiles; tile += npairs) {
         const int row0 = tile * 256 + (int)cta * 128;
         for (int pp = 0; pp < UP; ++pp) {
@@ -473,19 +540,19 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             const int j = op.x & 0xFF, aw = (op.x >> 8) & 0xFF;
             const uint32_t fl = op.x >> 24;
             const PairTerm* T = reinterpret_cast<const PairTerm*>(term0 + j * sizeof(PairTerm));
-            const bool bia = d.bias_mma && (fl & 1u);
-            PAIR_ACQUIRE(2u * (uint32_t)((128 + 64 * nu) * aw * 2 + (bia ? nu * 64 * 32 : 0)));
+            const bool bia = d.bias_mma && (fl & 1u) && !d.resident;
+            PAIR_ACQUIRE(2u * (uint32_t)((128 + (d.resident ? 0 : 64 * nu)) * aw * 2 + (bia ? nu * 64 * 32 : 0)));
             uint8_t* sa = ring + stage * kSlot;
             EV(0);
             if (!notma) tma_load_2d_pair(sa, T->amap, fb, (int)op.y, row0);
-            for (int q = 0; q < nu && !notma; ++q) {
+            for (int q = 0; q < nu && !notma && !d.resident; ++q) {
               tma_load_2d_pair(sa + kSlotA + q * kSlotB, T->wmap, fb, (int)op.y, (u0 + q) * kPairWu + (int)cta * 64);
               if (bia)
                 tma_load_2d_pair(sa + kSlotA + 2 * kSlotB + q * kSlotC, d.bmap, fb, 0,
                                  (int)(op.x >> 28) * d.Cpad + (u0 + q) * kPairWu + (int)cta * 64);
             }
             PAIR_NEXT();
-            if ((fl & 6u) == 6u && pend >= 0) {   // after level 0: the previous pair's fconv operands
+            if ((fl & 6u) == 6u && pend >= 0 && !d.resident) {   // after level 0: the previous pair's fconv operands
               PAIR_FCONV_ATOMS(pend);
               pend = -1;
             }
@@ -494,7 +561,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           pend = pp;
         }
       }
-      if (pend >= 0) {
+      if (pend >= 0 && !d.resident) {
         PAIR_FCONV_ATOMS(pend);
       }
 #undef PAIR_ACQUIRE
@@ -506,38 +573,61 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     // one elected lane issues each tcgen05 instruction)
     if (cta == 0) {
       const uint32_t idesc_t = idesc_bf16(256, kPairWu), idesc_f = idesc_bf16(256, d.Np);
-      const uint32_t sbase = smem_u32(smem), pbase = smem_u32(pbuf);
-      const uint64_t ones_d = umma_desc_k(smem_u32(ones), 16);
+      const uint32_t rbase = smem_u32(res), sbase = smem_u32(ring), pbase = smem_u32(pbuf);
+      // per-atom table (shared memory; the param-space program would be a dynamically indexed
+      // constant load per atom): {program word, descriptor hi of its K atom width, resident
+      // Lhat descriptor lo (pair 0, unit 0), resident bias descriptor lo (pair 0, unit 0)}
+      uint4* tab = reinterpret_cast<uint4*>(reinterpret_cast<uint8_t*>(bars) + kTabOff);
+      for (int k = lane; k < d.n_prog; k += 32) {
+        const uint32_t x = d.prog[k][0];
+        const int aw = (x >> 8) & 0xFF;
+        tab[k] = make_uint4(x, udesc_hi(aw), udesc_lo(rbase + (uint32_t)(k * 2 * d.bsz)),
+                            udesc_lo(rbase + (uint32_t)(d.res_c + (int)(x >> 28) * 2 * kSlotC)));
+      }
+      __syncwarp();
+      if (d.resident) {
+        mbar_wait_u(wbar, 0);
+        tc_fence_after();
+      }
+      const uint32_t a_lo0 = udesc_lo(sbase), slot16 = (uint32_t)kSlot >> 4;
+      const uint32_t hi16 = udesc_hi(16), hi64 = udesc_hi(64), ones_lo = udesc_lo(smem_u32(ones));
+      const uint32_t pb_step = (uint32_t)(d.n_prog * 2 * d.bsz) >> 4, bq16 = (uint32_t)d.bsz >> 4;
+      const uint32_t pc_step = (uint32_t)(d.n_levels * 2 * kSlotC) >> 4, cq16 = (uint32_t)kSlotC >> 4;
       int stage = 0;
       uint32_t ph = 0;
-      int gi = 0;             // (unit, level) accumulator items issued
-      int nf = 0;             // pair fconvs issued
-      int it = 0;             // tiles whose out region was started
+      int b = 0;                   // accumulator buffer of the next item (items rotate over NB)
+      uint32_t used = 0, par = 0;  // per buffer: used before / parity of its next acc_empty wait
+      int nf = 0;                  // pair fconvs issued
+      int it = 0;                  // tiles whose out region was started
 // fconv of unit pair pp: out (+)= P_u F_u^T for its units; the first pair of a tile starts
 // the out region (after the previous tile's out was drained), the last one publishes it
 #define PAIR_FCONV(pp, first_of_tile, last_of_tile)                                                            \
   {                                                                                                            \
-    mbar_wait_u(p_full, (uint32_t)nf & 1u);                                                              \
+    EV(14);                                                                                                    \
+    mbar_wait_u(p_full, (uint32_t)nf & 1u);                                                                    \
     EV(4);                                                                                                     \
     tc_fence_after();                                                                                          \
     if ((first_of_tile) && it > 0) {                                                                           \
-      mbar_wait_u(out_empty, (uint32_t)(it - 1) & 1u);                                                   \
+      mbar_wait_u(out_empty, (uint32_t)(it - 1) & 1u);                                                         \
       tc_fence_after();                                                                                        \
     }                                                                                                          \
     for (int q = 0; q < min(2, U - 2 * (pp)); ++q)                                                             \
       for (int a = 0; a < kPairWu / 64; ++a) {                                                                 \
-        mbar_wait_u(&full[stage], ph);                                                                           \
-        tc_fence_after();                                                                                      \
-        {                                                                                                      \
-          const uint64_t fd = umma_desc_k(sbase + stage * kSlot, 64);                                          \
-          const uint64_t pd = umma_desc_k(pbase + q * kPBytes + a * 16384, 64);                                \
-          for (int k4 = 0; k4 < 4; ++k4)                                                                       \
-            mma2_bf16_w(tout, pd + 2 * k4, fd + 2 * k4, idesc_f, ((first_of_tile) && q == 0 && a == 0 && k4 == 0) ? 0u : 1u); \
+        if (!d.resident) {                                                                                     \
+          mbar_wait_u(&full[stage], ph);                                                                       \
+          tc_fence_after();                                                                                    \
         }                                                                                                      \
-        mma2_commit_mc_w(&empty[stage], 3);                                                                    \
-        if (++stage == S) stage = 0, ph ^= 1;                                                                  \
+        const uint32_t f_lo = d.resident ? udesc_lo(rbase + (uint32_t)(d.res_f + ((2 * (pp) + q) * 2 + a) * d.fsz)) \
+                                         : a_lo0 + (uint32_t)stage * slot16;                                   \
+        mma2_k4_w(tout, udesc_lo(pbase + (uint32_t)(q * kPBytes + a * 16384)), hi64, f_lo, hi64, idesc_f,     \
+                  ((first_of_tile) && q == 0 && a == 0) ? 0u : 1u, 4u);                                        \
+        if (!d.resident) {                                                                                     \
+          mma2_commit_mc_w(&empty[stage], 3);                                                                  \
+          if (++stage == S) stage = 0, ph ^= 1;                                                                \
+        }                                                                                                      \
       }                                                                                                        \
     mma2_commit_mc_w(p_empty, 3);                                                                              \
+    EV(15);                                                                                                    \
     ++nf;                                                                                                      \
     if (last_of_tile) {                                                                                        \
       mma2_commit_mc_w(out_full, 3);                                                                           \
@@ -549,47 +639,62 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       for (int tile = pair_id; tile < d.ntiles; tile += npairs) {
         for (int pp = 0; pp < UP; ++pp) {
           const int nu = min(2, U - 2 * pp);
+          const uint32_t pbo = (uint32_t)pp * pb_step, pco = (uint32_t)pp * pc_step;
           int k = 0;
           for (;;) {   // one level per iteration, in chunks of <= kChunk ring stages
-            const uint32_t op0x = d.prog[k][0];
-            // atoms of this level
-            int kl = k;
-            while (!((d.prog[kl][0] >> 24) & 2u)) ++kl;
+            const uint32_t op0x = tab[k].x;
+            int kl = k;   // last atom of this level
+            while (!((tab[kl].x >> 24) & 2u)) ++kl;
             const int nat = kl - k + 1;
             const bool first_level = (op0x >> 24) & 4u;
             for (int c0 = 0; c0 < nat; c0 += kChunk) {
               const int cn = min(kChunk, nat - c0);
               for (int q = 0; q < nu; ++q) {
-                const int item = gi + q, b = item % NB, use = item / NB;
-                if (c0 == 0 && use > 0) {   // the buffer's previous item must have been drained
-                  mbar_wait_u(&acc_empty[b], (uint32_t)(use - 1) & 1u);
-                  tc_fence_after();
+                int bq = b + q;
+                if (bq >= NB) bq -= NB;
+                if (c0 == 0) {   // a new item in buffer bq: its previous item must have been drained
+                  if ((used >> bq) & 1u) {
+#ifdef TEMCO_TRACE
+                    if (!(g_pdbg & 4)) {   // timing experiment 4: no acc_empty waits
+#endif
+                    EV(12);
+                    mbar_wait_u(&acc_empty[bq], (par >> bq) & 1u);
+                    EV(13);
+                    tc_fence_after();
+#ifdef TEMCO_TRACE
+                    }
+#endif
+                    par ^= 1u << bq;
+                  } else {
+                    used |= 1u << bq;
+                  }
                 }
-                const uint32_t dt = tbase + (uint32_t)(b * kPairWu);
+                const uint32_t dt = tbase + (uint32_t)(bq * kPairWu);
                 int st = stage;
                 uint32_t sph = ph;
                 for (int i = 0; i < cn; ++i) {
-                  const uint2 op = make_uint2(d.prog[k + c0 + i][0], d.prog[k + c0 + i][1]);
-                  const int aw = (op.x >> 8) & 0xFF, nk = (op.x >> 16) & 0xFF;
+                  const uint4 tk = tab[k + c0 + i];
                   if (q == 0) {
                     mbar_wait_u(&full[st], sph);
                     EV(1);
                     tc_fence_after();
                   }
                   const bool lvl0 = c0 == 0 && i == 0;   // first atom of the level
-                  {
-                    const uint32_t sa = sbase + st * kSlot;
-                    const uint64_t ad = umma_desc_k(sa, aw), bd = umma_desc_k(sa + kSlotA + q * kSlotB, aw);
-                    const bool bia = d.bias_mma && lvl0;
-                    if (bia) mma2_bf16_w(dt, ones_d, umma_desc_k(sa + kSlotA + 2 * kSlotB + q * kSlotC, 16), idesc_t, 0u);
-                    for (int kk = 0; kk < nk; ++kk)
-                      mma2_bf16_w(dt, ad + 2 * kk, bd + 2 * kk, idesc_t, (lvl0 && !bia && kk == 0) ? 0u : 1u);
+                  const bool bia = d.bias_mma && lvl0;
+                  const uint32_t a_lo = a_lo0 + (uint32_t)st * slot16;
+                  if (bia) {
+                    const uint32_t c_lo = d.resident ? tk.w + pco + (uint32_t)q * cq16
+                                                     : a_lo + ((uint32_t)(kSlotA + 2 * kSlotB + q * kSlotC) >> 4);
+                    mma2_k4_w(dt, ones_lo, hi16, c_lo, hi16, idesc_t, 0u, 1u);
                   }
+                  const uint32_t b_lo = d.resident ? tk.z + pbo + (uint32_t)q * bq16
+                                                   : a_lo + ((uint32_t)(kSlotA + q * kSlotB) >> 4);
+                  mma2_k4_w(dt, a_lo, tk.y, b_lo, tk.y, idesc_t, (lvl0 && !bia) ? 0u : 1u, (tk.x >> 16) & 0xFFu);
                   EV(2);
                   if (++st == S) st = 0, sph ^= 1;
                 }
                 if (c0 + cn == nat) {
-                  mma2_commit_mc_w(&acc_full[b], 3);
+                  mma2_commit_mc_w(&acc_full[bq], 3);
                   EV(3);
                 }
               }
@@ -598,12 +703,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                 if (++stage == S) stage = 0, ph ^= 1;
               }
             }
-            gi += nu;
+            b += nu;
+            if (b >= NB) b -= NB;
             if (first_level && pend >= 0) {
               PAIR_FCONV(pend, pend_tile_first, pend_tile_last);
               pend = -1;
             }
-            const bool last = (d.prog[kl][0] >> 24) & 8u;
+            const bool last = (tab[kl].x >> 24) & 8u;
             k = kl + 1;
             if (last) break;
           }
@@ -627,6 +733,33 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     int gi = 0, np = 0, it = 0;   // gi: (unit, level) accumulator items consumed
     EVDECL();
     const bool ev0 = warp == kEpiWarp0 && lane == 0;
+    // out tile of tile `oit` (pixel row orow): TMEM columns [128 NB, 128 NB + Np) -> bf16 -> y.
+    // The issuer runs a tile's last fconv after the NEXT tile's level 0, so the epilogue
+    // drains that out region after consuming the next tile's level-0 items (not before
+    // them: that would idle the epilogue for a whole fconv round trip per tile)
+    auto drain_out = [&](int oit, int64_t orow) {
+      PAIR_EPI_WAIT(out_full, (uint32_t)oit & 1u);
+      tc_fence_after();
+      const int nch = d.Np / 8;
+      for (int c8 = g; c8 < nch; c8 += 4) {
+        uint32_t v[8];
+        tmem_ld8(tout + lane_off + c8 * 8, v);
+        tmem_wait_ld();
+        if (orow < d.npix && c8 * 8 < d.Nout) {
+          uint4 pk;
+          pk.x = pack_bf16(__uint_as_float(v[0]), __uint_as_float(v[1]));
+          pk.y = pack_bf16(__uint_as_float(v[2]), __uint_as_float(v[3]));
+          pk.z = pack_bf16(__uint_as_float(v[4]), __uint_as_float(v[5]));
+          pk.w = pack_bf16(__uint_as_float(v[6]), __uint_as_float(v[7]));
+          *reinterpret_cast<uint4*>(y + orow * d.Nout + c8 * 8) = pk;
+        }
+      }
+      tc_fence_before();
+      warp_arrive_cluster(oempty_c);
+      if (ev0) EV(11);
+    };
+    int pend_it = -1;
+    int64_t pend_row = 0;
     for (int tile = pair_id; tile < d.ntiles; tile += npairs, ++it) {
       const int64_t prow = (int64_t)tile * 256 + cta * 128 + row;
       for (int pp = 0; pp < UP; ++pp) {
@@ -639,7 +772,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
               const int act = d.mixed_act ? (int)d.actg[l * d.ngroups + (2 * pp + qq) * (kPairWu / 32) + g] : d.act[l];
               const float* bl = d.bias_mma ? nullptr : sbias + l * d.Cpad + (2 * pp + qq) * kPairWu + g * 32;
               const int item = gi + qq, b = item % NB;
-              mbar_wait(&acc_full[b], (uint32_t)(item / NB) & 1u);
+              PAIR_EPI_WAIT(&acc_full[b], (uint32_t)(item / NB) & 1u);
               if (ev0) EV(qq ? 8 : 5);
               tc_fence_after();
               uint32_t v[32];
@@ -659,9 +792,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             }
           }
           gi += nu;
+          if (l == 0 && pp == 0 && pend_it >= 0) {
+            drain_out(pend_it, pend_row);
+            pend_it = -1;
+          }
         }
         // P = t_D (already bf16x2) of both units for the pair's fconv
-        if (np > 0) mbar_wait(p_empty, (uint32_t)(np - 1) & 1u);
+        if (np > 0) PAIR_EPI_WAIT(p_empty, (uint32_t)(np - 1) & 1u);
         ++np;
 #pragma unroll
         for (int qq = 0; qq < 2; ++qq) {
@@ -680,27 +817,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         warp_arrive_cluster(pfull_c);
         if (ev0) EV(10);
       }
-      // out tile: TMEM columns [256, 256 + Np) -> bf16 -> y[prow, :Nout]
-      mbar_wait(out_full, (uint32_t)it & 1u);
-      tc_fence_after();
-      const int nch = d.Np / 8;
-      for (int c8 = g; c8 < nch; c8 += 4) {
-        uint32_t v[8];
-        tmem_ld8(tout + lane_off + c8 * 8, v);
-        tmem_wait_ld();
-        if (prow < d.npix && c8 * 8 < d.Nout) {
-          uint4 pk;
-          pk.x = pack_bf16(__uint_as_float(v[0]), __uint_as_float(v[1]));
-          pk.y = pack_bf16(__uint_as_float(v[2]), __uint_as_float(v[3]));
-          pk.z = pack_bf16(__uint_as_float(v[4]), __uint_as_float(v[5]));
-          pk.w = pack_bf16(__uint_as_float(v[6]), __uint_as_float(v[7]));
-          *reinterpret_cast<uint4*>(y + prow * d.Nout + c8 * 8) = pk;
-        }
-      }
-      tc_fence_before();
-      warp_arrive_cluster(oempty_c);
-      if (ev0) EV(11);
+      pend_it = it;
+      pend_row = prow;
     }
+    if (pend_it >= 0) drain_out(pend_it, pend_row);
   }
   tc_fence_before();
   cluster_sync_all();
@@ -749,11 +869,11 @@ void launch_pair_chain(const PairDesc& d, const RunPtrs& p, cudaStream_t s) {
 #ifdef TEMCO_TRACE
 // timeline of CTA 0 for the tc_pair launch with index `launch` (counted from the last reset)
 extern "C" void temco_debug_pair_ev(int launch, long long* out) {
-  if (out) cudaMemcpyFromSymbol(out, temco::pair::g_ev, sizeof(long long) * 12 * 512);
+  if (out) cudaMemcpyFromSymbol(out, temco::pair::g_ev, sizeof(long long) * 16 * 512);
   cudaMemcpyToSymbol(temco::pair::g_ev_on, &launch, sizeof(int));
   const int z = 0;
   cudaMemcpyToSymbol(temco::pair::g_launch, &z, sizeof(int));
-  static long long zz[12 * 512] = {0};
+  static long long zz[16 * 512] = {0};
   cudaMemcpyToSymbol(temco::pair::g_ev, zz, sizeof(zz));
 }
 extern "C" void temco_debug_pair_dbg(int v) { cudaMemcpyToSymbol(temco::pair::g_pdbg, &v, sizeof(int)); }

@@ -67,6 +67,12 @@ struct PairDesc {
   Loc y;                                 // output [npix x Nout] bf16 (arena)
   int64_t F;                             // tc weight pool offset of F
   int32_t stages, slot, smem_bytes, bias_bytes;   // ring depth, stage bytes
+  // resident-weight mode (every Lhat / bias / F atom of this CTA's halves fits in SMEM next
+  // to a deep ring): the weights are loaded once per CTA and the ring carries only the
+  // reduced-input atoms r_j, so several tiles' loads are in flight (small-C groups)
+  int32_t resident, res_bytes, res_tx;   // resident region bytes, TMA bytes per CTA
+  int32_t bsz, fsz;                      // resident Lhat atom slot (64 x awmax bf16), F atom (Np/2 x 64 bf16)
+  int32_t res_c, res_f;                  // offsets of the bias-MMA and F atoms in the resident region
   int32_t silu;                          // some level is SiLU: SILU kernel instantiation
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
 };

@@ -376,6 +376,49 @@ __device__ __forceinline__ void mma2_bf16_w(uint32_t dtmem, uint64_t adesc, uint
       "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
 }
 
+// UMMA shared-memory descriptor halves (K-major, swizzle by K atom width aw = 64 / 32 / 16
+// elements: SW128 / SW64 / SW32): lo = start address >> 4 | LBO 1, hi = SBO | version | layout.
+// Advancing K by 16 elements adds 2 to lo.
+__host__ __device__ __forceinline__ uint32_t udesc_lo(uint32_t saddr) { return ((saddr & 0x3FFFFu) >> 4) | 0x10000u; }
+__host__ __device__ __forceinline__ uint32_t udesc_hi(int aw) {
+  const uint32_t layout = aw == 64 ? 2u : aw == 32 ? 4u : 6u;
+  return ((uint32_t)(16 * aw) >> 4) | (1u << 14) | (layout << 29);
+}
+
+// warp-wide: one elected lane issues nk (1..4) cta_group::2 MMAs of consecutive K16 steps
+// (A, B descriptors advance by 32 bytes), the first with accumulate = acc0, the rest
+// accumulating -- one asm block, so the descriptors are moved to uniform registers once
+__device__ __forceinline__ void mma2_k4_w(uint32_t dtmem, uint32_t a_lo, uint32_t a_hi, uint32_t b_lo, uint32_t b_hi,
+                                          uint32_t idesc, uint32_t acc0, uint32_t nk) {
+  asm volatile(
+      "{\n"
+      ".reg .pred e, pa, pt, q1, q2, q3;\n"
+      ".reg .b64 da, db;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.ne.b32 pa, %6, 0;\n"
+      "setp.eq.b32 pt, %7, %7;\n"
+      "setp.gt.u32 q1, %7, 1;\n"
+      "setp.gt.u32 q2, %7, 2;\n"
+      "setp.gt.u32 q3, %7, 3;\n"
+      "and.pred q1, q1, e;\n"
+      "and.pred q2, q2, e;\n"
+      "and.pred q3, q3, e;\n"
+      "mov.b64 da, {%1, %2};\n"
+      "mov.b64 db, {%3, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pa;\n"
+      "add.s64 da, da, 2;\n"
+      "add.s64 db, db, 2;\n"
+      "@q1 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pt;\n"
+      "add.s64 da, da, 2;\n"
+      "add.s64 db, db, 2;\n"
+      "@q2 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pt;\n"
+      "add.s64 da, da, 2;\n"
+      "add.s64 db, db, 2;\n"
+      "@q3 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pt;\n"
+      "}\n" ::"r"(dtmem),
+      "r"(a_lo), "r"(a_hi), "r"(b_lo), "r"(b_hi), "r"(idesc), "r"(acc0), "r"(nk));
+}
+
 // warp-wide: the elected lane's prior cta_group::2 MMAs complete -> arrive on the
 // barrier at this shared offset in every CTA of `mask`
 __device__ __forceinline__ void mma2_commit_mc_w(uint64_t* bar, uint16_t mask) {
