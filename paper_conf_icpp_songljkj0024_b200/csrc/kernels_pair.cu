@@ -585,6 +585,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                             udesc_lo(rbase + (uint32_t)(d.res_c + (int)(x >> 28) * 2 * kSlotC)));
       }
       __syncwarp();
+      const uint32_t tab_s = smem_u32(tab);
       if (d.resident) {
         mbar_wait_u(wbar, 0);
         tc_fence_after();
@@ -642,17 +643,19 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           const uint32_t pbo = (uint32_t)pp * pb_step, pco = (uint32_t)pp * pc_step;
           int k = 0;
           for (;;) {   // one level per iteration, in chunks of <= kChunk ring stages
-            const uint32_t op0x = tab[k].x;
+            const uint32_t op0x = lds128(tab_s + 16u * k).x;
             int kl = k;   // last atom of this level
-            while (!((tab[kl].x >> 24) & 2u)) ++kl;
+            while (!((lds128(tab_s + 16u * kl).x >> 24) & 2u)) ++kl;
             const int nat = kl - k + 1;
             const bool first_level = (op0x >> 24) & 4u;
+            int b1 = b + 1;   // buffer of the pair's second unit
+            if (b1 >= NB) b1 -= NB;
+            const uint32_t d0 = tbase + (uint32_t)(b * kPairWu), d1 = tbase + (uint32_t)(b1 * kPairWu);
             for (int c0 = 0; c0 < nat; c0 += kChunk) {
               const int cn = min(kChunk, nat - c0);
-              for (int q = 0; q < nu; ++q) {
-                int bq = b + q;
-                if (bq >= NB) bq -= NB;
-                if (c0 == 0) {   // a new item in buffer bq: its previous item must have been drained
+              if (c0 == 0) {   // new items in buffers b (, b1): their previous items must have been drained
+                for (int q = 0; q < nu; ++q) {
+                  const int bq = q ? b1 : b;
                   if ((used >> bq) & 1u) {
 #ifdef TEMCO_TRACE
                     if (!(g_pdbg & 4)) {   // timing experiment 4: no acc_empty waits
@@ -660,7 +663,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                     EV(12);
                     mbar_wait_u(&acc_empty[bq], (par >> bq) & 1u);
                     EV(13);
-                    tc_fence_after();
 #ifdef TEMCO_TRACE
                     }
 #endif
@@ -669,34 +671,31 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                     used |= 1u << bq;
                   }
                 }
-                const uint32_t dt = tbase + (uint32_t)(bq * kPairWu);
-                int st = stage;
-                uint32_t sph = ph;
-                for (int i = 0; i < cn; ++i) {
-                  const uint4 tk = tab[k + c0 + i];
-                  if (q == 0) {
-                    mbar_wait_u(&full[st], sph);
-                    EV(1);
-                    tc_fence_after();
-                  }
-                  const bool lvl0 = c0 == 0 && i == 0;   // first atom of the level
-                  const bool bia = d.bias_mma && lvl0;
-                  const uint32_t a_lo = a_lo0 + (uint32_t)st * slot16;
-                  if (bia) {
-                    const uint32_t c_lo = d.resident ? tk.w + pco + (uint32_t)q * cq16
-                                                     : a_lo + ((uint32_t)(kSlotA + 2 * kSlotB + q * kSlotC) >> 4);
-                    mma2_k4_w(dt, ones_lo, hi16, c_lo, hi16, idesc_t, 0u, 1u);
-                  }
-                  const uint32_t b_lo = d.resident ? tk.z + pbo + (uint32_t)q * bq16
-                                                   : a_lo + ((uint32_t)(kSlotA + q * kSlotB) >> 4);
-                  mma2_k4_w(dt, a_lo, tk.y, b_lo, tk.y, idesc_t, (lvl0 && !bia) ? 0u : 1u, (tk.x >> 16) & 0xFFu);
-                  EV(2);
-                  if (++st == S) st = 0, sph ^= 1;
-                }
-                if (c0 + cn == nat) {
-                  mma2_commit_mc_w(&acc_full[bq], 3);
-                  EV(3);
-                }
+                tc_fence_after();
+              }
+              int st = stage;
+              uint32_t sph = ph;
+              for (int i = 0; i < cn; ++i) {
+                const uint4 tk = lds128(tab_s + 16u * (k + c0 + i));
+                mbar_wait_u(&full[st], sph);
+                EV(1);
+                tc_fence_after();
+                const bool lvl0 = c0 == 0 && i == 0;   // first atom of the level
+                const bool bia = d.bias_mma && lvl0;
+                const uint32_t a_lo = a_lo0 + (uint32_t)st * slot16;
+                const uint32_t b0_lo = d.resident ? tk.z + pbo : a_lo + ((uint32_t)kSlotA >> 4);
+                const uint32_t b1_lo = b0_lo + (d.resident ? bq16 : ((uint32_t)kSlotB >> 4));
+                const uint32_t c0_lo = d.resident ? tk.w + pco : a_lo + ((uint32_t)(kSlotA + 2 * kSlotB) >> 4);
+                const uint32_t c1_lo = c0_lo + (d.resident ? cq16 : ((uint32_t)kSlotC >> 4));
+                mma2_atom2_w(d0, d1, a_lo, tk.y, b0_lo, b1_lo, c0_lo, c1_lo, ones_lo, hi16, idesc_t, (tk.x >> 16) & 0xFFu,
+                             (uint32_t)nu, bia ? 1u : 0u, (lvl0 && !bia) ? 0u : 1u);
+                EV(2);
+                if (++st == S) st = 0, sph ^= 1;
+              }
+              if (c0 + cn == nat) {
+                mma2_commit_mc_w(&acc_full[b], 3);
+                if (nu > 1) mma2_commit_mc_w(&acc_full[b1], 3);
+                EV(3);
               }
               for (int i = 0; i < cn; ++i) {
                 mma2_commit_mc_w(&empty[stage], 3);
@@ -709,7 +708,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
               PAIR_FCONV(pend, pend_tile_first, pend_tile_last);
               pend = -1;
             }
-            const bool last = (tab[kl].x >> 24) & 8u;
+            const bool last = (lds128(tab_s + 16u * kl).x >> 24) & 8u;
             k = kl + 1;
             if (last) break;
           }

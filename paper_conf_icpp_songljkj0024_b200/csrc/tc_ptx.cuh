@@ -331,6 +331,8 @@ __device__ __forceinline__ void mbar_wait_u(uint64_t* bar, uint32_t parity) {
       "{\n"
       ".reg .pred p, q;\n"
       ".reg .u64 t0, t1;\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@p bra DONE_%=;\n"
       "mov.u64 t0, %%clock64;\n"
       "WAIT_%=:\n"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
@@ -376,6 +378,12 @@ __device__ __forceinline__ void mma2_bf16_w(uint32_t dtmem, uint64_t adesc, uint
       "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
 }
 
+__device__ __forceinline__ uint4 lds128(uint32_t saddr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(saddr));
+  return v;
+}
+
 // UMMA shared-memory descriptor halves (K-major, swizzle by K atom width aw = 64 / 32 / 16
 // elements: SW128 / SW64 / SW32): lo = start address >> 4 | LBO 1, hi = SBO | version | layout.
 // Advancing K by 16 elements adds 2 to lo.
@@ -417,6 +425,63 @@ __device__ __forceinline__ void mma2_k4_w(uint32_t dtmem, uint32_t a_lo, uint32_
       "@q3 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pt;\n"
       "}\n" ::"r"(dtmem),
       "r"(a_lo), "r"(a_hi), "r"(b_lo), "r"(b_hi), "r"(idesc), "r"(acc0), "r"(nk));
+}
+
+// warp-wide: one K atom of a level for both units of a CTA pair in one asm block (one elect):
+// for unit q < nu: [bias MMA ones x C_q into D_q, accumulate off, if bia] then nk K16 MMAs
+// A x B_q into D_q (A, B advance 32 bytes per step; the first accumulates iff acc0)
+__device__ __forceinline__ void mma2_atom2_w(uint32_t d0, uint32_t d1, uint32_t a_lo, uint32_t a_hi, uint32_t b0_lo,
+                                             uint32_t b1_lo, uint32_t c0_lo, uint32_t c1_lo, uint32_t ones_lo,
+                                             uint32_t hi16, uint32_t idesc, uint32_t nk, uint32_t nu, uint32_t bia,
+                                             uint32_t acc0) {
+  asm volatile(
+      "{\n"
+      ".reg .pred e, e1, pb, pb1, pa, pt, pf, q1, q2, q3, r1, r2, r3;\n"
+      ".reg .b64 da, db, dn, dc;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.gt.u32 e1, %12, 1;\n"
+      "and.pred e1, e1, e;\n"
+      "setp.ne.b32 pb, %13, 0;\n"
+      "and.pred pb, pb, e;\n"
+      "and.pred pb1, pb, e1;\n"
+      "setp.ne.b32 pa, %14, 0;\n"
+      "setp.eq.b32 pt, %11, %11;\n"
+      "setp.ne.b32 pf, %11, %11;\n"
+      "setp.gt.u32 q1, %11, 1;\n"
+      "setp.gt.u32 q2, %11, 2;\n"
+      "setp.gt.u32 q3, %11, 3;\n"
+      "and.pred r1, q1, e1;\n"
+      "and.pred r2, q2, e1;\n"
+      "and.pred r3, q3, e1;\n"
+      "and.pred q1, q1, e;\n"
+      "and.pred q2, q2, e;\n"
+      "and.pred q3, q3, e;\n"
+      "mov.b64 dn, {%8, %9};\n"
+      "mov.b64 dc, {%6, %9};\n"
+      "@pb tcgen05.mma.cta_group::2.kind::f16 [%0], dn, dc, %10, pf;\n"
+      "mov.b64 da, {%2, %3};\n"
+      "mov.b64 db, {%4, %3};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %10, pa;\n"
+      "add.s64 da, da, 2;\n add.s64 db, db, 2;\n"
+      "@q1 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %10, pt;\n"
+      "add.s64 da, da, 2;\n add.s64 db, db, 2;\n"
+      "@q2 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %10, pt;\n"
+      "add.s64 da, da, 2;\n add.s64 db, db, 2;\n"
+      "@q3 tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %10, pt;\n"
+      "mov.b64 dc, {%7, %9};\n"
+      "@pb1 tcgen05.mma.cta_group::2.kind::f16 [%1], dn, dc, %10, pf;\n"
+      "mov.b64 da, {%2, %3};\n"
+      "mov.b64 db, {%5, %3};\n"
+      "@e1 tcgen05.mma.cta_group::2.kind::f16 [%1], da, db, %10, pa;\n"
+      "add.s64 da, da, 2;\n add.s64 db, db, 2;\n"
+      "@r1 tcgen05.mma.cta_group::2.kind::f16 [%1], da, db, %10, pt;\n"
+      "add.s64 da, da, 2;\n add.s64 db, db, 2;\n"
+      "@r2 tcgen05.mma.cta_group::2.kind::f16 [%1], da, db, %10, pt;\n"
+      "add.s64 da, da, 2;\n add.s64 db, db, 2;\n"
+      "@r3 tcgen05.mma.cta_group::2.kind::f16 [%1], da, db, %10, pt;\n"
+      "}\n" ::"r"(d0),
+      "r"(d1), "r"(a_lo), "r"(a_hi), "r"(b0_lo), "r"(b1_lo), "r"(c0_lo), "r"(c1_lo), "r"(ones_lo), "r"(hi16),
+      "r"(idesc), "r"(nk), "r"(nu), "r"(bia), "r"(acc0));
 }
 
 // warp-wide: the elected lane's prior cta_group::2 MMAs complete -> arrive on the
