@@ -612,21 +612,23 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       mbar_wait_u(out_empty, (uint32_t)(it - 1) & 1u);                                                         \
       tc_fence_after();                                                                                        \
     }                                                                                                          \
-    for (int q = 0; q < min(2, U - 2 * (pp)); ++q)                                                             \
-      for (int a = 0; a < kPairWu / 64; ++a) {                                                                 \
-        if (!d.resident) {                                                                                     \
+    for (int q = 0; q < min(2, U - 2 * (pp)); ++q) {                                                           \
+      if (d.resident) {   /* both 64-channel F atoms of unit q: one block of 8 MMAs */                         \
+        mma2_k8_w(tout, udesc_lo(pbase + (uint32_t)(q * kPBytes)), hi64,                                       \
+                  udesc_lo(rbase + (uint32_t)(d.res_f + (2 * (pp) + q) * 2 * d.fsz)), hi64, 16384u,             \
+                  (uint32_t)d.fsz, idesc_f, ((first_of_tile) && q == 0) ? 0u : 1u);                            \
+      } else {                                                                                                 \
+        for (int a = 0; a < kPairWu / 64; ++a) {                                                               \
           mbar_wait_u(&full[stage], ph);                                                                       \
           tc_fence_after();                                                                                    \
-        }                                                                                                      \
-        const uint32_t f_lo = d.resident ? udesc_lo(rbase + (uint32_t)(d.res_f + ((2 * (pp) + q) * 2 + a) * d.fsz)) \
-                                         : a_lo0 + (uint32_t)stage * slot16;                                   \
-        mma2_k4_w(tout, udesc_lo(pbase + (uint32_t)(q * kPBytes + a * 16384)), hi64, f_lo, hi64, idesc_f,     \
-                  ((first_of_tile) && q == 0 && a == 0) ? 0u : 1u, 4u);                                        \
-        if (!d.resident) {                                                                                     \
+          mma2_k4_w(tout, udesc_lo(pbase + (uint32_t)(q * kPBytes + a * 16384)), hi64,                         \
+                    a_lo0 + (uint32_t)stage * slot16, hi64, idesc_f,                                           \
+                    ((first_of_tile) && q == 0 && a == 0) ? 0u : 1u, 4u);                                      \
           mma2_commit_mc_w(&empty[stage], 3);                                                                  \
           if (++stage == S) stage = 0, ph ^= 1;                                                                \
         }                                                                                                      \
       }                                                                                                        \
+    }                                                                                                          \
     mma2_commit_mc_w(p_empty, 3);                                                                              \
     EV(15);                                                                                                    \
     ++nf;                                                                                                      \
@@ -693,13 +695,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                 if (++st == S) st = 0, sph ^= 1;
               }
               if (c0 + cn == nat) {
-                mma2_commit_mc_w(&acc_full[b], 3);
-                if (nu > 1) mma2_commit_mc_w(&acc_full[b1], 3);
+                mma2_commit2_mc_w(smem_u32(&acc_full[b]), smem_u32(&acc_full[b1]), (uint32_t)nu);
                 EV(3);
               }
-              for (int i = 0; i < cn; ++i) {
-                mma2_commit_mc_w(&empty[stage], 3);
-                if (++stage == S) stage = 0, ph ^= 1;
+              {   // release the chunk's ring stages (kChunk = 2: one block)
+                int s1 = stage + 1;
+                if (s1 == S) s1 = 0;
+                mma2_commit2_mc_w(smem_u32(&empty[stage]), smem_u32(&empty[s1]), (uint32_t)cn);
+                for (int i = 0; i < cn; ++i)
+                  if (++stage == S) stage = 0, ph ^= 1;
               }
             }
             b += nu;

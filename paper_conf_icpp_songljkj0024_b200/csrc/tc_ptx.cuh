@@ -427,6 +427,54 @@ __device__ __forceinline__ void mma2_k4_w(uint32_t dtmem, uint32_t a_lo, uint32_
       "r"(a_lo), "r"(a_hi), "r"(b_lo), "r"(b_hi), "r"(idesc), "r"(acc0), "r"(nk));
 }
 
+// warp-wide: commit to two barriers (n = 1 or 2) in one asm block (one elect)
+__device__ __forceinline__ void mma2_commit2_mc_w(uint32_t bar0, uint32_t bar1, uint32_t n) {
+  asm volatile(
+      "{\n"
+      ".reg .pred e, e1;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.gt.u32 e1, %2, 1;\n"
+      "and.pred e1, e1, e;\n"
+      "@e tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %3;\n"
+      "@e1 tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%1], %3;\n"
+      "}\n" ::"r"(bar0),
+      "r"(bar1), "r"(n), "h"((uint16_t)3)
+      : "memory");
+}
+
+// warp-wide: 8 K16 MMAs of two consecutive 64-wide K atoms (A atom 2 at +a2 bytes, B atom 2 at
+// +b2 bytes from atom 1), one elect; the first accumulates iff acc0
+__device__ __forceinline__ void mma2_k8_w(uint32_t dtmem, uint32_t a_lo, uint32_t a_hi, uint32_t b_lo, uint32_t b_hi,
+                                          uint32_t a2, uint32_t b2, uint32_t idesc, uint32_t acc0) {
+  asm volatile(
+      "{\n"
+      ".reg .pred e, pa, pt;\n"
+      ".reg .b64 da, db, da2, db2;\n"
+      "elect.sync _|e, 0xffffffff;\n"
+      "setp.ne.b32 pa, %8, 0;\n"
+      "setp.eq.b32 pt, %5, %5;\n"
+      "mov.b64 da, {%1, %2};\n"
+      "mov.b64 db, {%3, %4};\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pa;\n"
+      "add.s64 da2, da, 2;\n add.s64 db2, db, 2;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da2, db2, %5, pt;\n"
+      "add.s64 da2, da, 4;\n add.s64 db2, db, 4;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da2, db2, %5, pt;\n"
+      "add.s64 da2, da, 6;\n add.s64 db2, db, 6;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da2, db2, %5, pt;\n"
+      "cvt.u64.u32 da2, %6;\n cvt.u64.u32 db2, %7;\n"
+      "add.s64 da, da, da2;\n add.s64 db, db, db2;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da, db, %5, pt;\n"
+      "add.s64 da2, da, 2;\n add.s64 db2, db, 2;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da2, db2, %5, pt;\n"
+      "add.s64 da2, da, 4;\n add.s64 db2, db, 4;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da2, db2, %5, pt;\n"
+      "add.s64 da2, da, 6;\n add.s64 db2, db, 6;\n"
+      "@e tcgen05.mma.cta_group::2.kind::f16 [%0], da2, db2, %5, pt;\n"
+      "}\n" ::"r"(dtmem),
+      "r"(a_lo), "r"(a_hi), "r"(b_lo), "r"(b_hi), "r"(idesc), "r"(a2 >> 4), "r"(b2 >> 4), "r"(acc0));
+}
+
 // warp-wide: one K atom of a level for both units of a CTA pair in one asm block (one elect):
 // for unit q < nu: [bias MMA ones x C_q into D_q, accumulate off, if bia] then nk K16 MMAs
 // A x B_q into D_q (A, B advance 32 bytes per step; the first accumulates iff acc0)
