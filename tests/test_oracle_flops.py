@@ -43,6 +43,11 @@ def test_flops_hand_counts_per_operator():
     assert flops(g, cat) == 0
     assert flops(g, gap) == 2 * 16 * 6       # one add per input element: 192
     assert flops(g, lin) == 2 * 16 * 10 * 2  # 640
+    # transposed conv 2x2 / stride 2, 4 -> 6 channels on a 3 x 5 input (output 6 x 10): every
+    # input pixel meets every weight once: 2 img * 15 px * 4 in * 6 out * 4 taps * 2 = 5760
+    xt = Node(12, "input", [], C=4, H=3, W=5)
+    ct = Node(13, "convt", [12], kh=2, kw=2, sh=2, sw=2, ph=0, pw=0, C=6, H=6, W=10)
+    assert flops(_g([xt, ct]), ct) == 5760
 
 
 def test_overhead_uses_the_kernel_window():
