@@ -31,7 +31,8 @@ sys.path.insert(0, ROOT)
 
 import workloads as W  # noqa: E402
 
-CONFIG_BATCH = {"resnet18_cifar": 128, "resnet50": 256, "vgg16_cp": 256, "densenet121": 128, "alexnet": 256, "unet": 16}
+CONFIG_BATCH = {"resnet18_cifar": 128, "resnet50": 256, "vgg16_cp": 256, "densenet121": 128, "alexnet": 256, "unet": 16,
+                "resnet18_tt": 128}
 CONFIG_TEXT = {
     "resnet18_cifar": "ResNet-18 Tucker-2 decomposed, CIFAR-10 shape 32x32, batch 128",
     "resnet50": "ResNet-50 Tucker-2 decomposed, ImageNet shape 224x224, batch 256 per GPU, bf16",
@@ -39,6 +40,7 @@ CONFIG_TEXT = {
     "densenet121": "DenseNet-121 Tucker-2 decomposed (concat skips), 224x224, batch 128 per GPU, 8-GPU batch shard",
     "alexnet": "AlexNet Tucker-2 decomposed (SURVEY 8(f) f2; not a BASELINE.json config), 224x224, batch 256 per GPU",
     "unet": "UNet Tucker-2 decomposed (SURVEY 8(f) f1; Carvana shape 256x256, 2 classes; not a BASELINE.json config), batch 16 per GPU",
+    "resnet18_tt": "ResNet-18 Tensor-Train decomposed K x K convs (SURVEY 8(f) f4; not a BASELINE.json config), CIFAR-10 shape 32x32, batch 128",
 }
 METRIC = "images/sec"
 
@@ -139,7 +141,8 @@ def reference_arm(args):
         return
     from threadpoolctl import threadpool_info
     m = W.build_config(args.config)
-    sample = {"resnet18_cifar": 8, "resnet50": 1, "vgg16_cp": 1, "densenet121": 1, "alexnet": 1, "unet": 1}[args.config]
+    sample = {"resnet18_cifar": 8, "resnet50": 1, "vgg16_cp": 1, "densenet121": 1, "alexnet": 1, "unet": 1,
+              "resnet18_tt": 8}[args.config]
     pl = oracle.plan(m)
     times = []
     for step in range(args.warmup + args.steps):
@@ -169,7 +172,8 @@ def cpu_baseline(config):
     from threadpoolctl import threadpool_info
     m = W.build_config(config)
     pl = oracle.plan(m)
-    sample = {"resnet18_cifar": 256, "resnet50": 24, "vgg16_cp": 24, "densenet121": 24, "alexnet": 24, "unet": 4}[config]
+    sample = {"resnet18_cifar": 256, "resnet50": 24, "vgg16_cp": 24, "densenet121": 24, "alexnet": 24, "unet": 4,
+              "resnet18_tt": 256}[config]
     x = W.make_input(m, start=0, count=sample)
     oracle.run_temco(pl, x[:1])                 # warm-up
     t0 = time.perf_counter()

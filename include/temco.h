@@ -88,7 +88,7 @@ typedef struct {
   float bn_eps;
 } temco_layer;
 
-typedef enum { TEMCO_DECOMP_TUCKER2 = 1, TEMCO_DECOMP_CP = 2 } temco_decomp_kind;
+typedef enum { TEMCO_DECOMP_TUCKER2 = 1, TEMCO_DECOMP_CP = 2, TEMCO_DECOMP_TT = 3 } temco_decomp_kind;
 
 /* decomposition of one conv layer (Eq. (2)); fp32, row-major:
  *   Tucker-2: first [rank_in, C_in] (NULL iff rank_in == C_in: no fconv),
@@ -96,6 +96,11 @@ typedef enum { TEMCO_DECOMP_TUCKER2 = 1, TEMCO_DECOMP_CP = 2 } temco_decomp_kind
  *             last  [C_out, rank_out] (NULL iff rank_out == C_out: no lconv)
  *   CP      : rank_in == rank_out == R; first [R, C_in]; core = Kv [R, K];
  *             core2 = Kh [R, K]; last [C_out, R]   (fconv -> dw Kx1 -> dw 1xK -> lconv)
+ *   TT      : Tensor-Train (P:L73 [28]) of W in mode order (C_in, K, K, C_out) with
+ *             ranks r1 = rank_in, r2 = rank_mid, r3 = rank_out: first [r1, C_in] (NULL iff
+ *             r1 == C_in), core [r2, r1, K] (a K x 1 conv, stride (s, 1), pad (p, 0)),
+ *             core2 [r3, r2, K] (a 1 x K conv, stride (1, s), pad (0, p)), last [C_out, r3]
+ *             (fconv -> Kx1 -> 1xK -> lconv; the lconv carries the bias)
  * Any positive rank is accepted; the tcgen05 kernels (bf16 plans) need reduced
  * ranks that are multiples of 8 (16-byte rows for TMA) and run every other
  * group on the generic SIMT kernels. */
@@ -104,6 +109,7 @@ typedef struct {
   int32_t kind;               /* temco_decomp_kind */
   int32_t rank_in, rank_out;
   const float *first, *core, *core2, *last;
+  int32_t rank_mid;           /* TT only: the rank between the two cores (ignored otherwise) */
 } temco_decomp;
 
 /* declared skip edges: must be EXACTLY the input edges (src -> dst) with

@@ -129,6 +129,28 @@ def expand(model) -> Graph:
                 n = push(op="conv", inputs=[hz.id], role="lconv", orig=li, name=layer.name + ".lconv",
                          C=layer.out_channels, H=ho, W=wo,
                          weight=np.asarray(d.last)[:, :, None, None], bias=layer.bias)
+            elif d.kind == "tt":
+                # Tensor-Train (P:L73 [28]; reading R33): the weight W[o, i, a, b] in mode
+                # order (C_in, K_h, K_w, C_out) as a train of cores G1 [C_in x r1],
+                # G2 [r1 x K x r2], G3 [r2 x K x r3], G4 [r3 x C_out]: fconv 1x1 (C_in -> r1),
+                # core K x 1 (r1 -> r2, stride (s, 1), pad (p, 0)), core 1 x K (r2 -> r3,
+                # stride (1, s), pad (0, p)), lconv 1x1 (r3 -> C_out, bias)
+                # (no fconv when r1 == C_in, as for Tucker-2: a full-rank input mode, R17)
+                r1, r2, r3 = d.rank_in, d.rank_mid, d.rank_out
+                f = x
+                if d.first is not None:
+                    f = push(op="conv", inputs=[x.id], role="fconv", orig=li, name=layer.name + ".fconv",
+                             C=r1, H=x.H, W=x.W, weight=np.asarray(d.first)[:, :, None, None])
+                h1, _ = _out_hw(x.H, x.W, k, 1, s, 1, p, 0)
+                v = push(op="conv", inputs=[f.id], role="core", orig=li, name=layer.name + ".core_v",
+                         kh=k, kw=1, sh=s, sw=1, ph=p, pw=0, C=r2, H=h1, W=x.W,
+                         weight=np.asarray(d.core)[:, :, :, None])
+                hz = push(op="conv", inputs=[v.id], role="core", orig=li, name=layer.name + ".core_h",
+                          kh=1, kw=k, sh=1, sw=s, ph=0, pw=p, C=r3, H=ho, W=wo,
+                          weight=np.asarray(d.core2)[:, :, None, :])
+                n = push(op="conv", inputs=[hz.id], role="lconv", orig=li, name=layer.name + ".lconv",
+                         C=layer.out_channels, H=ho, W=wo,
+                         weight=np.asarray(d.last)[:, :, None, None], bias=layer.bias)
             else:
                 raise ValueError(d.kind)
         elif layer.op == "conv_transpose":

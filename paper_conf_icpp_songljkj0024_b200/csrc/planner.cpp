@@ -198,6 +198,35 @@ void expand(const temco_layer* layers, int n_layers, const temco_decomp* decomps
           q.w = copy_buf(d->last, (size_t)l.out_channels * r);
           q.b = copy_buf(l.bias, l.out_channels);
           out_of[li] = push(q);
+        } else if (d->kind == TEMCO_DECOMP_TT) {
+          // Tensor-Train (P:L73 [28]; reading R33): fconv 1x1 (C_in -> r1, omitted when
+          // r1 == C_in) -> K x 1 conv (r1 -> r2) -> 1 x K conv (r2 -> r3) -> lconv 1x1 (r3 -> C_out)
+          const int r1 = d->rank_in, r2 = d->rank_mid, r3 = d->rank_out;
+          if (r2 <= 0) fail(TEMCO_ERR_UNSUPPORTED, "ranks must be positive");
+          if (!d->core || !d->core2 || !d->last) fail(TEMCO_ERR_INVALID_ARGUMENT, "TT factor is NULL");
+          if (r1 > x.C) fail(TEMCO_ERR_UNSUPPORTED, "TT rank exceeds its mode");
+          int cur = ins[0];
+          if (d->first) {
+            Node f; f.op = OP_CONV; f.role = ROLE_FCONV; f.orig = li; f.in = {cur};
+            f.C = r1; f.H = x.H; f.W = x.W; f.w = copy_buf(d->first, (size_t)r1 * x.C);
+            cur = push(f);
+          } else if (r1 != x.C) {
+            fail(TEMCO_ERR_INVALID_GRAPH, "rank_in != C_in requires a first factor");
+          }
+          const int h1 = (x.H + 2 * p - k) / s + 1;
+          Node v; v.op = OP_CONV; v.role = ROLE_CORE; v.orig = li; v.in = {cur};
+          v.kh = k; v.kw = 1; v.sh = s; v.sw = 1; v.ph = p; v.pw = 0;
+          v.C = r2; v.H = h1; v.W = x.W; v.w = copy_buf(d->core, (size_t)r2 * r1 * k);
+          const int vi = push(v);
+          Node h; h.op = OP_CONV; h.role = ROLE_CORE; h.orig = li; h.in = {vi};
+          h.kh = 1; h.kw = k; h.sh = 1; h.sw = s; h.ph = 0; h.pw = p;
+          h.C = r3; h.H = ho; h.W = wo; h.w = copy_buf(d->core2, (size_t)r3 * r2 * k);
+          const int hi = push(h);
+          Node q; q.op = OP_CONV; q.role = ROLE_LCONV; q.orig = li; q.in = {hi};
+          q.C = l.out_channels; q.H = ho; q.W = wo;
+          q.w = copy_buf(d->last, (size_t)l.out_channels * r3);
+          q.b = copy_buf(l.bias, l.out_channels);
+          out_of[li] = push(q);
         } else {
           fail(TEMCO_ERR_INVALID_ARGUMENT, "unknown decomposition kind");
         }

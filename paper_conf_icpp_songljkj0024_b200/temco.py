@@ -47,7 +47,7 @@ class _Layer(C.Structure):
 
 class _Decomp(C.Structure):
     _fields_ = [("layer", C.c_int32), ("kind", C.c_int32), ("rank_in", C.c_int32), ("rank_out", C.c_int32),
-                ("first", _fp), ("core", _fp), ("core2", _fp), ("last", _fp)]
+                ("first", _fp), ("core", _fp), ("core2", _fp), ("last", _fp), ("rank_mid", C.c_int32)]
 
 
 class _Edge(C.Structure):
@@ -145,8 +145,9 @@ class Plan:
         decs = (_Decomp * max(1, len(model.decomps)))()
         for j, (li, d) in enumerate(sorted(model.decomps.items())):
             D = decs[j]
-            D.layer, D.kind = li, {"tucker2": 1, "cp": 2}[d.kind]
+            D.layer, D.kind = li, {"tucker2": 1, "cp": 2, "tt": 3}[d.kind]
             D.rank_in, D.rank_out = d.rank_in, d.rank_out
+            D.rank_mid = getattr(d, "rank_mid", 0)
             for name in ("first", "core", "core2", "last"):
                 a = _f32(getattr(d, name))
                 keep.append(a)

@@ -51,6 +51,8 @@ SMALL = {
     # full width (base 64): the 3x3 cores of the bottom level exceed one SMEM weight block
     # (output-channel-sliced tc_conv), as in the full config
     "unet_s": lambda dt: W.unet(batch=2, dtype=dt, height=32, width=32, base=64),
+    # Tensor-Train (f4): K x 1 and 1 x K cores on reduced channels
+    "resnet18_tt_s": lambda dt: W.resnet18_cifar(batch=3, dtype=dt, height=16, width=16, tt=True),
 }
 
 
@@ -89,7 +91,7 @@ def test_ragged_batch_and_tiles():
 
 
 FULL = {"resnet18_cifar": [0, 77, 127], "resnet50": [0, 255], "vgg16_cp": [0, 255], "densenet121": [0, 127],
-        "alexnet": [0, 255], "unet": [0, 15]}
+        "alexnet": [0, 255], "unet": [0, 15], "resnet18_tt": [0, 127]}
 
 
 @pytest.mark.parametrize("name", list(FULL))

@@ -30,7 +30,7 @@ pytestmark = pytest.mark.gpu
 
 torch = pytest.importorskip("torch")
 
-CONFIGS = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet", "unet"]
+CONFIGS = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet", "unet", "resnet18_tt"]
 
 
 def _to_f64(raw, shape):

@@ -19,10 +19,11 @@ def test_small_cases_cover_the_full_configs():
               W.vgg16_cp(batch=2, dtype="bf16", height=32, width=32),
               W.densenet121(batch=2, dtype="bf16", height=64, width=64),
               W.alexnet(batch=60, dtype="bf16", height=224, width=224),
-              W.unet(batch=2, dtype="bf16", height=32, width=32, base=64)):
+              W.unet(batch=2, dtype="bf16", height=32, width=32, base=64),
+              W.resnet18_cifar(batch=3, dtype="bf16", height=16, width=16, tt=True)):
         small.update(_kernels(m))
     full = collections.Counter()
-    for name in ("resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet", "unet"):
+    for name in ("resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet", "unet", "resnet18_tt"):
         full.update(_kernels(W.build_config(name)))
     assert set(full) <= set(small), set(full) - set(small)
     # the tensor-core families are all on the bench path

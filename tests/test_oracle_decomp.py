@@ -91,6 +91,60 @@ def test_cp_full_rank_reconstructs_conv(cin, cout, k, s, p):
     np.testing.assert_allclose(got, _ref(m, W, b, x), rtol=1e-10, atol=1e-10)
 
 
+def tt_full(W, rng):
+    """TT-SVD (Oseledets' sequential truncated SVDs, no truncation) of W in mode order
+    (C_in, K_h, K_w, C_out): exact TT ranks r1 = min(C_in, K K C_out),
+    r2 = min(r1 K, K C_out), r3 = min(r2 K, C_out)."""
+    cout, cin, k, _ = W.shape
+    A = np.transpose(W, (1, 2, 3, 0))                               # [C_in, K_h, K_w, C_out]
+    U1, S1, V1 = np.linalg.svd(A.reshape(cin, k * k * cout), full_matrices=False)
+    r1 = len(S1)
+    rest = (S1[:, None] * V1).reshape(r1 * k, k * cout)
+    U2, S2, V2 = np.linalg.svd(rest, full_matrices=False)
+    r2 = len(S2)
+    rest = (S2[:, None] * V2).reshape(r2 * k, cout)
+    U3, S3, V3 = np.linalg.svd(rest, full_matrices=False)
+    r3 = len(S3)
+    G1 = U1                                                         # [C_in, r1]
+    G2 = U2.reshape(r1, k, r2)
+    G3 = U3.reshape(r2, k, r3)
+    G4 = S3[:, None] * V3                                           # [r3, C_out]
+    # conv weights: fconv [r1, C_in]; K x 1 core [r2, r1, K]; 1 x K core [r3, r2, K]; lconv [C_out, r3]
+    return Decomp(1, "tt", r1, r3, G1.T.copy(), np.transpose(G2, (2, 0, 1)).copy(),
+                  np.transpose(G3, (2, 0, 1)).copy(), G4.T.copy(), rank_mid=r2)
+
+
+@pytest.mark.parametrize("cin,cout,k,s,p", [(3, 5, 3, 1, 1), (4, 4, 3, 2, 1), (2, 3, 5, 2, 2), (3, 2, 3, 1, 0)])
+def test_tt_full_rank_reconstructs_conv(cin, cout, k, s, p):
+    """Tensor-Train (reading R33) at the exact TT ranks reproduces the conv, including
+    stride and padding, through fconv -> K x 1 core -> 1 x K core -> lconv."""
+    m, W, b = _single_conv_model(cin, cout, k, s, p, tt_full)
+    x = np.random.default_rng(5).standard_normal((2, m.height, m.width, cin))
+    pl = oracle.plan(m)
+    g = pl.graph
+    assert [n.role for n in g.nodes] == ["", "fconv", "core", "core", "lconv"]
+    assert (g.nodes[2].kh, g.nodes[2].kw, g.nodes[2].sh, g.nodes[2].ph, g.nodes[2].groups) == (k, 1, s, p, 1)
+    assert (g.nodes[3].kh, g.nodes[3].kw, g.nodes[3].sw, g.nodes[3].pw, g.nodes[3].groups) == (1, k, s, p, 1)
+    d = m.decomps[1]
+    assert (g.nodes[1].C, g.nodes[2].C, g.nodes[3].C) == (d.rank_in, d.rank_mid, d.rank_out)
+    got = oracle.run_unfused(pl, x)
+    np.testing.assert_allclose(got, _ref(m, W, b, x), rtol=1e-10, atol=1e-10)
+
+
+def test_tt_truncated_ranks_change_the_output():
+    """A TT train truncated below its exact ranks no longer reproduces the conv (the pin above
+    is not vacuous: every core takes part)."""
+    def tt_cut(W, rng):
+        d = tt_full(W, rng)
+        d.core = d.core.copy()
+        d.core[-1] = 0.0                                            # drop one r2 channel
+        return d
+    m, W, b = _single_conv_model(3, 4, 3, 1, 1, tt_cut)
+    x = np.random.default_rng(6).standard_normal((2, m.height, m.width, 3))
+    got = oracle.run_unfused(oracle.plan(m), x)
+    assert np.abs(got - _ref(m, W, b, x)).max() > 1e-3
+
+
 def test_tucker2_omitted_factors_and_bias_placement():
     """R_in == C_in drops the fconv; R_out == C_out drops the lconv and the
     bias moves onto the core (O1)."""

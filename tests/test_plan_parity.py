@@ -17,7 +17,7 @@ SMALL = {
     "t2_3": lambda: W.t2_stem_blocks(3), "t3": W.t3_mini_bottleneck, "t4": W.t4_mini_densenet,
     "c1_bf16": lambda: W.c1_basic_block(dtype="bf16", batch=3),
 }
-FULL = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet", "unet"]
+FULL = ["resnet18_cifar", "resnet50", "vgg16_cp", "densenet121", "alexnet", "unet", "resnet18_tt"]
 
 
 def _compare(m, flags=0, **okw):

@@ -73,13 +73,14 @@ class Layer:
 @dataclass
 class Decomp:
     layer: int
-    kind: str                    # "tucker2" | "cp"
+    kind: str                    # "tucker2" | "cp" | "tt"
     rank_in: int
     rank_out: int
     first: Optional[np.ndarray]
     core: np.ndarray
     core2: Optional[np.ndarray]
     last: Optional[np.ndarray]
+    rank_mid: int = 0            # Tensor-Train: the rank between the two cores
 
 
 @dataclass
@@ -132,13 +133,14 @@ def make_input(model: Model, start: int = 0, count: Optional[int] = None) -> np.
 class _G:
     """Appends layers, tracks (C, H, W) per layer, draws seeded weights."""
 
-    def __init__(self, name, batch, h, w, c, dtype, seed, rank=rank_rule, cp=False):
+    def __init__(self, name, batch, h, w, c, dtype, seed, rank=rank_rule, cp=False, tt=False):
         self.m = Model(name, batch, h, w, c, dtype)
         self.m.layers.append(Layer("input", [], name="input", out_channels=c))
         self.shape = [(c, h, w)]
         self.seed = seed
         self.rank = rank
         self.cp = cp
+        self.tt = tt
 
     def rng(self):
         return np.random.default_rng(self.seed * 1_000_003 + len(self.m.layers))
@@ -175,6 +177,19 @@ class _G:
             kh = rng.standard_normal((r, k)) / np.sqrt(k)
             last = rng.standard_normal((cout, r)) * np.sqrt(2.0 / r)
             d = Decomp(idx, "cp", r, r, self._q(first), self._q(kv), self._q(kh), self._q(last))
+        elif self.tt and k > 1:
+            # Tensor-Train (reading R33): r1 = R(C_in), r2 = r3 = R(C_out); orthonormal outer
+            # factors as for Tucker-2, Gaussian cores scaled by their fan-in
+            r1 = min(self.rank(cin), cin) if ranks is None else ranks[0]
+            r3 = min(self.rank(cout), cout) if ranks is None else ranks[1]
+            r2 = r3
+            first = self._orth(rng, cin, r1).T if r1 < cin else None       # no fconv on a full-rank mode
+            cv = rng.standard_normal((r2, r1, k)) / np.sqrt(r1 * k)
+            ch = rng.standard_normal((r3, r2, k)) / np.sqrt(r2 * k)
+            last = self._orth(rng, cout, r3) * np.sqrt(cout / r3) if r3 <= cout else \
+                rng.standard_normal((cout, r3)) * np.sqrt(2.0 / r3)
+            d = Decomp(idx, "tt", r1, r3, None if first is None else self._q(first), self._q(cv), self._q(ch),
+                       self._q(last), rank_mid=r2)
         else:
             ri = self.rank(cin) if ranks is None else ranks[0]
             ro = self.rank(cout) if ranks is None else ranks[1]
@@ -339,10 +354,12 @@ def _basic_block(g, x, cout, stride, name):
     return g.relu(g.add([b, sc], f"{name}.add"), f"{name}.relu2")
 
 
-def resnet18_cifar(batch=128, dtype=BF16, height=32, width=32, seed=101):
+def resnet18_cifar(batch=128, dtype=BF16, height=32, width=32, seed=101, tt=False):
     """BASELINE.json configs[1]: ResNet-18, CIFAR-10 shape (kuangliu layout,
-    reading R23): 3x3 s1 stem, no maxpool, widths 64-512, 10 classes."""
-    g = _G("resnet18_cifar", batch, height, width, 3, dtype, seed)
+    reading R23): 3x3 s1 stem, no maxpool, widths 64-512, 10 classes.  tt=True: every
+    K x K conv Tensor-Train decomposed (reading R33), the 1x1
+    shortcut convs Tucker-2."""
+    g = _G("resnet18_tt" if tt else "resnet18_cifar", batch, height, width, 3, dtype, seed, tt=tt)
     x = g.relu(g.bn(g.conv(0, 64, 3, 1, 1, name="conv1"), "bn1"), "relu")
     for si, (c, s) in enumerate([(64, 1), (128, 2), (256, 2), (512, 2)]):
         for bi in range(2):
@@ -472,6 +489,7 @@ def unet(batch=16, dtype=BF16, height=256, width=256, seed=606, base=64, n_class
 CONFIGS = {
     "c1": lambda **kw: c1_basic_block(**kw),
     "resnet18_cifar": lambda **kw: resnet18_cifar(**kw),
+    "resnet18_tt": lambda **kw: resnet18_cifar(tt=True, **kw),
     "resnet50": lambda **kw: resnet50(**kw),
     "vgg16_cp": lambda **kw: vgg16_cp(**kw),
     "densenet121": lambda **kw: densenet121(**kw),
