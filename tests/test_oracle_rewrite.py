@@ -335,3 +335,63 @@ def test_temco_equals_unfused(make):
     x = W.make_input(m)
     a, b = oracle.run_temco(pl, x), oracle.run_unfused(pl, x)
     assert np.linalg.norm(a - b) <= 1e-5 * np.linalg.norm(b)
+
+
+# ----------------------------------------------------------------------------
+# reading R34: the CP depthwise core pair as one step
+# ----------------------------------------------------------------------------
+
+def _cp_single(s=2, R=4):
+    import numpy as np
+    from workloads import Decomp, Layer, Model
+    rng = np.random.default_rng(11)
+    m = Model("cp1", 1, 8, 8, 1, "f32")
+    m.layers = [Layer("input", [], out_channels=1),
+                Layer("conv", [0], out_channels=1, kernel=3, stride=s, pad=1, bias=rng.standard_normal(1))]
+    m.decomps = {1: Decomp(1, "cp", R, R, rng.standard_normal((R, 1)), rng.standard_normal((R, 3)),
+                           rng.standard_normal((R, 3)), rng.standard_normal((1, R)))}
+    return m
+
+
+def test_cp_pair_live_bytes_by_hand():
+    """C = 1 -> R = 4, 3x3 stride 2 on 8 x 8 (fp32): x 256 B, fconv out r 1024 B, K x 1 out
+    (stride (2, 1): 4 x 8) 512 B, 1 x K out (4 x 4) 256 B, lconv out 64 B.  Without the pair
+    rule the K x 1 step holds r + mid = 1536 B (the peak); with it the pair step holds
+    r + h = 1280 B and the intermediate never exists."""
+    m = _cp_single()
+    a = oracle.plan(m, cp_pair=False)
+    b = oracle.plan(m)
+    assert a.live_fused == [256, 1280, 1536, 768, 320] and a.peak_fused == 1536
+    assert b.live_fused == [256, 1280, 1280, 320] and b.peak_fused == 1280
+    pair = [s for s in b.steps if s.kind == "group" and len(s.members) == 2]
+    assert len(pair) == 1
+    v, h = (b.onodes[x] for x in pair[0].members)
+    assert (v.kh, v.kw, h.kh, h.kw) == (3, 1, 1, 3) and pair[0].inputs == v.inputs
+
+
+def test_cp_pair_semantics_and_vgg_pairs():
+    """The paired schedule computes the same tensor as the op-by-op one, and every
+    CP layer of VGG-16-CP pairs its cores (their K x 1 output has no other reader)."""
+    import numpy as np
+    m = _cp_single(s=1)
+    x = W.make_input(m)
+    np.testing.assert_allclose(oracle.run_temco(oracle.plan(m), x), oracle.run_unfused(oracle.plan(m), x),
+                               rtol=1e-12, atol=1e-12)
+    v = W.vgg16_cp(batch=1, dtype="f32", height=32, width=32)
+    p = oracle.plan(v)
+    pairs = [s for s in p.steps if s.kind == "group" and all(p.onodes[x].role == "core" for x in s.members)]
+    assert len(pairs) == 13 and all(len(s.members) == 2 for s in pairs)
+    x = W.make_input(v)
+    np.testing.assert_allclose(oracle.run_temco(p, x), oracle.run_unfused(p, x), rtol=1e-9, atol=1e-9)
+
+
+def test_cp_pair_not_formed_when_the_intermediate_has_another_reader():
+    """A K x 1 core whose output is also read elsewhere keeps its own step (R34)."""
+    from oracle.rewrite import pair_cp_cores
+    m = _cp_single()
+    p = oracle.plan(m, cp_pair=False)
+    v = next(n for n in p.graph.nodes if n.role == "core" and n.kw == 1)
+    O = list(p.O) + [10_000]
+    on = dict(p.onodes)
+    on[10_000] = type(v)(10_000, "relu", [v.id], C=v.C, H=v.H, W=v.W)
+    assert pair_cp_cores(O, on, {}) == {}
