@@ -38,7 +38,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM };
+enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM, K_DWPAIR };
 
 struct StepExec {
   int kind = K_NONE;
@@ -54,6 +54,7 @@ struct StepExec {
   MmaChainDesc mma{};
   RankConvDesc rk{};
   CatDesc cat{};
+  DwPairDesc dwp{};
   std::string kernel;
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
@@ -280,6 +281,29 @@ void lower(temco_plan_s* P) {
     for (int m : s.members) e.flops += node_flops(ir, m);
     for (int x : s.in) e.io_bytes += tensor_bytes(P, x);
     if (v.op != OP_INPUT) e.io_bytes += tensor_bytes(P, s.out);
+    if (s.group && s.members.size() == 2 && ir.nodes[s.members[0]].op == OP_CONV &&
+        ir.nodes[s.members[0]].groups > 1) {
+      // CP depthwise core pair (reading R34): one kernel, the K x 1 output stays in registers
+      const Node& v = ir.nodes[s.members[0]];
+      const Node& h = ir.nodes[s.members[1]];
+      const Node& x = ir.nodes[ir.oin[s.members[0]][0]];
+      DwPairDesc& q = e.dwp;
+      q = DwPairDesc{};
+      q.x = tensor_loc(P, x.id);
+      q.y = tensor_loc(P, s.out);
+      q.N = N; q.H = x.H; q.W = x.W; q.C = x.C;
+      q.H1 = v.H; q.Ho = h.H; q.Wo = h.W; q.K = v.kh;
+      q.sv = v.sh; q.pv = v.ph; q.sh = h.sw; q.ph = h.pw;
+      if (h.kw != v.kh || v.C != x.C) throw std::runtime_error("CP core pair: unexpected shapes");
+      q.wv = push_params(P, v.w);
+      q.wh = push_params(P, h.w);
+      q.bv = push_params(P, v.b);
+      q.bh = push_params(P, h.b);
+      e.kind = K_DWPAIR;
+      e.kernel = dwpair_fast_ok(q) ? "simt_dwpair" : "simt_dwpair_generic";
+      e.launches = 1;
+      continue;
+    }
     if (s.group) {
       // groups with a 3x3/s2 max-pooled 64-channel member (the stem restore copies):
       // restore-once mma.sync kernel; single-input groups: the lean mma.sync kernels;
@@ -707,6 +731,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
     switch (e.kind) {
       case K_NONE: break;
       case K_CONVT: launch_conv_transpose(e.conv, rp, st); break;
+      case K_DWPAIR: launch_dwpair(e.dwp, rp, st); break;
       case K_CONV:
         if (e.stem)
           launch_conv_stem(e.conv, rp, st);

@@ -76,6 +76,18 @@ struct ConvDesc {             // direct NHWC convolution (fconv on full tensors,
   int64_t w2;                 // depthwise: params offset of the weights in [kh][kw][C] order, -1 none
 };
 
+// the two depthwise cores of one CP decomposition as one step (reading R34): K x 1 (vertical
+// stride sv, pad pv) then 1 x K (horizontal stride sh, pad ph) on C channels; the vertical result
+// never leaves registers
+struct DwPairDesc {
+  Loc x, y;
+  int32_t N, H, W, C;         // input
+  int32_t H1, Ho, Wo, K;      // rows after the vertical core, output spatial, taps
+  int32_t sv, pv, sh, ph;
+  int64_t wv, wh;             // params offsets: per-channel taps [C][K] of each core
+  int64_t bv, bh;             // params offsets of the cores' biases, -1 none
+};
+
 struct RankConvDesc {          // reduced-rank conv on tensor cores (kernels_rank.cu), bf16
   Loc x, y;
   int32_t N, H, W, C, Ho, Wo, K;

@@ -29,6 +29,8 @@ void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cud
 bool mma_poolcat_ok(const CatDesc& d);
 bool mma_catp_ok(const CatDesc& d);      // chunk-parallel concat kernel applies (launch_mma_cat dispatches)   // restore-once 3x3/s2 max-pooled member (launch_mma_cat dispatches)
 bool dwconv_vec_ok(const ConvDesc& d);   // depthwise bf16, C % 8 == 0: vectorised kernel
+void launch_dwpair(const DwPairDesc& d, const RunPtrs& p, cudaStream_t s);   // CP core pair (R34)
+bool dwpair_fast_ok(const DwPairDesc& d);
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);
 bool conv_rank_ok(const ConvDesc& d);    // reduced-rank direct conv applies (bf16, Cin, K <= 64, % 8)
 void launch_conv_rank(const ConvDesc& d, const RunPtrs& p, cudaStream_t s);

@@ -874,6 +874,129 @@ bool dwconv_vec_ok(const ConvDesc& d) {
          d.kh * d.kw <= 9;
 }
 
+// ---------------------------------------------------------------------------
+// CP depthwise core pair (reading R34): out(h, w, c) = sum_i Kv[c][i] sum_j Kh[c][j]
+// x(h sv + i - pv, w sh + j - ph, c), zero outside the image -- the separable product of the
+// K x 1 and 1 x K cores, whose intermediate (the K x 1 output) is never stored.
+// ---------------------------------------------------------------------------
+constexpr int kPairRows = 16;   // output rows per thread strip (fast kernel)
+
+// fast path: bf16, C % 8 == 0, K = 3, unit strides, no biases.  A thread owns one (column,
+// 8-channel group) and a strip of kPairRows output rows; per input row it forms the horizontal
+// 1 x 3 combination H(r) of its three 16-byte neighbours (the neighbours' loads hit L1: the
+// adjacent threads read them too), and each output row is the vertical 3 x 1 combination of a
+// sliding window of three H rows -- x is read from HBM once, the output written once.
+__global__ void __launch_bounds__(256) dwpair_kernel(DwPairDesc d, RunPtrs p) {
+  const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
+  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+  const int cg = d.C / 8;
+  const int idx = blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= d.Wo * cg) return;
+  const int wo = idx / cg, g = idx - wo * cg;
+  float kv[3][8], kh[3][8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j)
+#pragma unroll
+    for (int t = 0; t < 3; ++t) {
+      kv[t][j] = __ldg(p.params + d.wv + (int64_t)(g * 8 + j) * 3 + t);
+      kh[t][j] = __ldg(p.params + d.wh + (int64_t)(g * 8 + j) * 3 + t);
+    }
+  pdl_wait();
+  pdl_trigger_early();
+  const int spi = (d.Ho + kPairRows - 1) / kPairRows;
+  auto hrow = [&](int n, int r, float (&hv)[8]) {   // H(r) at this thread's column
+#pragma unroll
+    for (int j = 0; j < 8; ++j) hv[j] = 0.f;
+    if (r < 0 || r >= d.H) return;
+    const uint4* row = reinterpret_cast<const uint4*>(x + ((int64_t)n * d.H + r) * d.W * d.C);
+#pragma unroll
+    for (int t = 0; t < 3; ++t) {
+      const int wi = wo - d.ph + t;
+      if (wi < 0 || wi >= d.W) continue;
+      const uint4 v = __ldg(row + (int64_t)wi * cg + g);
+      const uint32_t uw[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+      for (int j = 0; j < 8; ++j)
+        hv[j] = fmaf(__uint_as_float(j & 1 ? (uw[j / 2] & 0xFFFF0000u) : (uw[j / 2] << 16)), kh[t][j], hv[j]);
+    }
+  };
+  for (int st = blockIdx.y; st < d.N * spi; st += gridDim.y) {
+    const int n = st / spi, h0 = (st - n * spi) * kPairRows;
+    float h_a[8], h_b[8], h_c[8];                 // H rows h - pv, h - pv + 1, h - pv + 2
+    hrow(n, h0 - d.pv, h_a);
+    hrow(n, h0 - d.pv + 1, h_b);
+    for (int r = 0; r < kPairRows; ++r) {
+      const int h = h0 + r;
+      if (h >= d.Ho) break;
+      hrow(n, h - d.pv + 2, h_c);
+      float o[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) o[j] = fmaf(kv[0][j], h_a[j], fmaf(kv[1][j], h_b[j], kv[2][j] * h_c[j]));
+      uint4 pk;
+      __nv_bfloat162 q0 = __floats2bfloat162_rn(o[0], o[1]), q1 = __floats2bfloat162_rn(o[2], o[3]);
+      __nv_bfloat162 q2 = __floats2bfloat162_rn(o[4], o[5]), q3 = __floats2bfloat162_rn(o[6], o[7]);
+      pk.x = *reinterpret_cast<uint32_t*>(&q0);
+      pk.y = *reinterpret_cast<uint32_t*>(&q1);
+      pk.z = *reinterpret_cast<uint32_t*>(&q2);
+      pk.w = *reinterpret_cast<uint32_t*>(&q3);
+      reinterpret_cast<uint4*>(y + (((int64_t)n * d.Ho + h) * d.Wo + wo) * d.C)[g] = pk;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        h_a[j] = h_b[j];
+        h_b[j] = h_c[j];
+      }
+    }
+  }
+}
+
+// any dtype / K / strides / biases: one thread per output element, the vertical core evaluated
+// (with its bias) at each of the K columns the horizontal core reads
+__global__ void __launch_bounds__(256) dwpair_generic_kernel(DwPairDesc d, RunPtrs p) {
+  const void* x = loc_ptr(d.x, p);
+  void* y = const_cast<void*>(loc_ptr(d.y, p));
+  pdl_wait();
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.C;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int c = (int)(i % d.C);
+    int64_t t = i / d.C;
+    const int wo = (int)(t % d.Wo);
+    t /= d.Wo;
+    const int h = (int)(t % d.Ho);
+    const int n = (int)(t / d.Ho);
+    float acc = d.bh >= 0 ? p.params[d.bh + c] : 0.f;
+    for (int j = 0; j < d.K; ++j) {
+      const int w1 = wo * d.sh - d.ph + j;          // column of the vertical core's output
+      if (w1 < 0 || w1 >= d.W) continue;
+      float v = d.bv >= 0 ? p.params[d.bv + c] : 0.f;
+      for (int q = 0; q < d.K; ++q) {
+        const int r = h * d.sv - d.pv + q;
+        if (r < 0 || r >= d.H) continue;
+        v = fmaf(p.params[d.wv + (int64_t)c * d.K + q], ldv(x, (((int64_t)n * d.H + r) * d.W + w1) * d.C + c, d.x.dtype), v);
+      }
+      acc = fmaf(p.params[d.wh + (int64_t)c * d.K + j], v, acc);
+    }
+    stv(y, i, acc, d.y.dtype);
+  }
+}
+
+bool dwpair_fast_ok(const DwPairDesc& d) {
+  return d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.C % 8 == 0 && d.K == 3 && d.sv == 1 && d.sh == 1 &&
+         d.bv < 0 && d.bh < 0 && d.Ho == d.H + 2 * d.pv - 2 && d.Wo == d.W + 2 * d.ph - 2;
+}
+
+void launch_dwpair(const DwPairDesc& d, const RunPtrs& p, cudaStream_t s) {
+  if (dwpair_fast_ok(d)) {
+    const int xb = (d.Wo * (d.C / 8) + 255) / 256;
+    const int strips = d.N * ((d.Ho + kPairRows - 1) / kPairRows);
+    launch_pdl(dwpair_kernel, dim3((unsigned)xb, (unsigned)std::min(strips, std::max(1, 148 * 8 / xb))), dim3(256), 0, s,
+               d, p);
+    return;
+  }
+  const int64_t total = (int64_t)d.N * d.Ho * d.Wo * d.C;
+  const int grid = (int)std::min<int64_t>((total + 255) / 256, 148LL * 16);
+  launch_pdl(dwpair_generic_kernel, dim3(grid), dim3(256), 0, s, d, p);
+}
+
 void launch_dwconv_vec(const ConvDesc& d, const RunPtrs& p, cudaStream_t s) {
   const int per_row = d.Wo * (d.C / 8);
   const int rows = d.N * d.Ho;

@@ -614,6 +614,24 @@ void group_and_schedule(IR& ir, bool fusion) {
       grouped.insert(mem.begin(), mem.end());
     }
   }
+  if (fusion) {
+    // reading R34: the K x 1 and 1 x K depthwise cores of one CP decomposition
+    // form one step when the K x 1 output has no other consumer (oracle: pair_cp_cores)
+    for (int x : ir.O) {
+      const Node& h = ir.nodes[x];
+      if (h.op != OP_CONV || ir.oin[x].size() != 1 || grouped.count(x)) continue;
+      const int vi = ir.oin[x][0];
+      const Node& v = ir.nodes[vi];
+      if (grouped.count(vi) || cons[vi].size() != 1 || cons[vi][0] != x) continue;
+      const bool pair = v.op == OP_CONV && v.role == ROLE_CORE && h.role == ROLE_CORE && v.orig == h.orig &&
+                        v.groups == v.C && h.groups == h.C && v.C == h.C && v.kw == 1 && v.kh > 1 && h.kh == 1 &&
+                        h.kw > 1;
+      if (!pair) continue;
+      ir.groups[x] = {vi, x};
+      grouped.insert(vi);
+      grouped.insert(x);
+    }
+  }
   std::map<int, int> member_of;
   for (auto& kv : ir.groups)
     for (int x : kv.second) member_of[x] = kv.first;
