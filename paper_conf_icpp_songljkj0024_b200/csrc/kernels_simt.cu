@@ -879,20 +879,50 @@ bool dwconv_vec_ok(const ConvDesc& d) {
 // x(h sv + i - pv, w sh + j - ph, c), zero outside the image -- the separable product of the
 // K x 1 and 1 x K cores, whose intermediate (the K x 1 output) is never stored.
 // ---------------------------------------------------------------------------
-constexpr int kPairRows = 16;   // output rows per thread strip (fast kernel)
+constexpr int kPairRows = 8;   // output rows per thread strip (fast kernel)
 
-// fast path: bf16, C % 8 == 0, K = 3, unit strides, no biases.  A thread owns one (column,
-// 8-channel group) and a strip of kPairRows output rows; per input row it forms the horizontal
-// 1 x 3 combination H(r) of its three 16-byte neighbours (the neighbours' loads hit L1: the
-// adjacent threads read them too), and each output row is the vertical 3 x 1 combination of a
-// sliding window of three H rows -- x is read from HBM once, the output written once.
-__global__ void __launch_bounds__(256) dwpair_kernel(DwPairDesc d, RunPtrs p) {
+__device__ __forceinline__ void hcomb(float (&hv)[8], const uint4& l, const uint4& c, const uint4& r,
+                                      const float (&kh)[3][8]) {
+  const uint32_t ul[4] = {l.x, l.y, l.z, l.w}, uc[4] = {c.x, c.y, c.z, c.w}, ur[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    const int q = j / 2;
+    const bool hi = j & 1;
+    const float xl = __uint_as_float(hi ? (ul[q] & 0xFFFF0000u) : (ul[q] << 16));
+    const float xc = __uint_as_float(hi ? (uc[q] & 0xFFFF0000u) : (uc[q] << 16));
+    const float xr = __uint_as_float(hi ? (ur[q] & 0xFFFF0000u) : (ur[q] << 16));
+    hv[j] = fmaf(kh[0][j], xl, fmaf(kh[1][j], xc, kh[2][j] * xr));
+  }
+}
+
+__device__ __forceinline__ uint4 shfl4(unsigned mask, const uint4& v, int delta, bool up) {
+  uint4 o;
+  if (up) {
+    o.x = __shfl_up_sync(mask, v.x, delta); o.y = __shfl_up_sync(mask, v.y, delta);
+    o.z = __shfl_up_sync(mask, v.z, delta); o.w = __shfl_up_sync(mask, v.w, delta);
+  } else {
+    o.x = __shfl_down_sync(mask, v.x, delta); o.y = __shfl_down_sync(mask, v.y, delta);
+    o.z = __shfl_down_sync(mask, v.z, delta); o.w = __shfl_down_sync(mask, v.w, delta);
+  }
+  return o;
+}
+
+// fast path: bf16, C % 8 == 0 (<= 128 channels), K = 3, unit strides, pad 1, no biases.  A
+// thread owns one (column, 8-channel group) and a strip of kPairRows output rows: it loads its
+// own column's kPairRows + 2 input rows (16 bytes each, all in flight), takes the left / right
+// neighbour columns from the lanes cg away (warp shuffles; lanes whose neighbour lies outside
+// the warp load it), forms the horizontal 1 x 3 combination H of every input row and the
+// vertical 3 x 1 combination of three H rows per output row.  x is read from HBM once and the
+// output written once; the K x 1 intermediate never exists.
+__global__ void __launch_bounds__(256, 2) dwpair_kernel(DwPairDesc d, RunPtrs p) {
   const __nv_bfloat16* x = reinterpret_cast<const __nv_bfloat16*>(loc_ptr(d.x, p));
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
   const int cg = d.C / 8;
+  const int per_row = d.W * cg;
   const int idx = blockIdx.x * blockDim.x + threadIdx.x;
-  if (idx >= d.Wo * cg) return;
-  const int wo = idx / cg, g = idx - wo * cg;
+  const bool valid = idx < per_row;                  // idle lanes stay for the shuffles
+  const int wo = valid ? idx / cg : 0, g = valid ? idx - (idx / cg) * cg : 0;
+  const int lane = threadIdx.x & 31;
   float kv[3][8], kh[3][8];
 #pragma unroll
   for (int j = 0; j < 8; ++j)
@@ -904,46 +934,49 @@ __global__ void __launch_bounds__(256) dwpair_kernel(DwPairDesc d, RunPtrs p) {
   pdl_wait();
   pdl_trigger_early();
   const int spi = (d.Ho + kPairRows - 1) / kPairRows;
-  auto hrow = [&](int n, int r, float (&hv)[8]) {   // H(r) at this thread's column
-#pragma unroll
-    for (int j = 0; j < 8; ++j) hv[j] = 0.f;
-    if (r < 0 || r >= d.H) return;
-    const uint4* row = reinterpret_cast<const uint4*>(x + ((int64_t)n * d.H + r) * d.W * d.C);
-#pragma unroll
-    for (int t = 0; t < 3; ++t) {
-      const int wi = wo - d.ph + t;
-      if (wi < 0 || wi >= d.W) continue;
-      const uint4 v = __ldg(row + (int64_t)wi * cg + g);
-      const uint32_t uw[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-      for (int j = 0; j < 8; ++j)
-        hv[j] = fmaf(__uint_as_float(j & 1 ? (uw[j / 2] & 0xFFFF0000u) : (uw[j / 2] << 16)), kh[t][j], hv[j]);
-    }
-  };
+  const bool own_left = lane < cg, own_right = lane + cg >= 32;   // neighbour outside the warp
+  const uint4 z = make_uint4(0, 0, 0, 0);
   for (int st = blockIdx.y; st < d.N * spi; st += gridDim.y) {
     const int n = st / spi, h0 = (st - n * spi) * kPairRows;
-    float h_a[8], h_b[8], h_c[8];                 // H rows h - pv, h - pv + 1, h - pv + 2
-    hrow(n, h0 - d.pv, h_a);
-    hrow(n, h0 - d.pv + 1, h_b);
-    for (int r = 0; r < kPairRows; ++r) {
-      const int h = h0 + r;
-      if (h >= d.Ho) break;
-      hrow(n, h - d.pv + 2, h_c);
-      float o[8];
+    const uint4* img = reinterpret_cast<const uint4*>(x + (int64_t)n * d.H * d.W * d.C);
+    uint4 v[kPairRows + 2];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) o[j] = fmaf(kv[0][j], h_a[j], fmaf(kv[1][j], h_b[j], kv[2][j] * h_c[j]));
-      uint4 pk;
-      __nv_bfloat162 q0 = __floats2bfloat162_rn(o[0], o[1]), q1 = __floats2bfloat162_rn(o[2], o[3]);
-      __nv_bfloat162 q2 = __floats2bfloat162_rn(o[4], o[5]), q3 = __floats2bfloat162_rn(o[6], o[7]);
-      pk.x = *reinterpret_cast<uint32_t*>(&q0);
-      pk.y = *reinterpret_cast<uint32_t*>(&q1);
-      pk.z = *reinterpret_cast<uint32_t*>(&q2);
-      pk.w = *reinterpret_cast<uint32_t*>(&q3);
-      reinterpret_cast<uint4*>(y + (((int64_t)n * d.Ho + h) * d.Wo + wo) * d.C)[g] = pk;
+    for (int r = 0; r < kPairRows + 2; ++r) {
+      const int hi = h0 - 1 + r;
+      v[r] = (valid && hi >= 0 && hi < d.H && h0 + r - 2 < d.Ho) ? __ldg(img + ((int64_t)hi * d.W + wo) * cg + g) : z;
+    }
+    float ha[8], hb[8];
+#pragma unroll
+    for (int r = 0; r < kPairRows + 2; ++r) {
+      const int hi = h0 - 1 + r;
+      uint4 l = shfl4(0xffffffffu, v[r], cg, true), rr = shfl4(0xffffffffu, v[r], cg, false);
+      const bool rowok = valid && hi >= 0 && hi < d.H;
+      if (own_left) l = (rowok && wo > 0) ? __ldg(img + ((int64_t)hi * d.W + wo - 1) * cg + g) : z;
+      if (own_right) rr = (rowok && wo + 1 < d.W) ? __ldg(img + ((int64_t)hi * d.W + wo + 1) * cg + g) : z;
+      if (wo == 0) l = z;
+      if (wo + 1 >= d.W) rr = z;
+      float hc[8];
+      hcomb(hc, l, v[r], rr, kh);
+      if (r >= 2) {
+        const int h = h0 + r - 2;
+        if (valid && h < d.Ho) {
+          float o[8];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) o[j] = fmaf(kv[0][j], ha[j], fmaf(kv[1][j], hb[j], kv[2][j] * hc[j]));
+          uint4 pk;
+          __nv_bfloat162 q0 = __floats2bfloat162_rn(o[0], o[1]), q1 = __floats2bfloat162_rn(o[2], o[3]);
+          __nv_bfloat162 q2 = __floats2bfloat162_rn(o[4], o[5]), q3 = __floats2bfloat162_rn(o[6], o[7]);
+          pk.x = *reinterpret_cast<uint32_t*>(&q0);
+          pk.y = *reinterpret_cast<uint32_t*>(&q1);
+          pk.z = *reinterpret_cast<uint32_t*>(&q2);
+          pk.w = *reinterpret_cast<uint32_t*>(&q3);
+          reinterpret_cast<uint4*>(y + (((int64_t)n * d.Ho + h) * d.Wo + wo) * d.C)[g] = pk;
+        }
+      }
 #pragma unroll
       for (int j = 0; j < 8; ++j) {
-        h_a[j] = h_b[j];
-        h_b[j] = h_c[j];
+        ha[j] = hb[j];
+        hb[j] = hc[j];
       }
     }
   }
@@ -980,13 +1013,13 @@ __global__ void __launch_bounds__(256) dwpair_generic_kernel(DwPairDesc d, RunPt
 }
 
 bool dwpair_fast_ok(const DwPairDesc& d) {
-  return d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.C % 8 == 0 && d.K == 3 && d.sv == 1 && d.sh == 1 &&
-         d.bv < 0 && d.bh < 0 && d.Ho == d.H + 2 * d.pv - 2 && d.Wo == d.W + 2 * d.ph - 2;
+  return d.x.dtype == DT_BF16 && d.y.dtype == DT_BF16 && d.C % 8 == 0 && d.C / 8 <= 16 && d.K == 3 && d.sv == 1 &&
+         d.sh == 1 && d.pv == 1 && d.ph == 1 && d.bv < 0 && d.bh < 0 && d.Ho == d.H && d.Wo == d.W;
 }
 
 void launch_dwpair(const DwPairDesc& d, const RunPtrs& p, cudaStream_t s) {
   if (dwpair_fast_ok(d)) {
-    const int xb = (d.Wo * (d.C / 8) + 255) / 256;
+    const int xb = (d.W * (d.C / 8) + 255) / 256;
     const int strips = d.N * ((d.Ho + kPairRows - 1) / kPairRows);
     launch_pdl(dwpair_kernel, dim3((unsigned)xb, (unsigned)std::min(strips, std::max(1, 148 * 8 / xb))), dim3(256), 0, s,
                d, p);
