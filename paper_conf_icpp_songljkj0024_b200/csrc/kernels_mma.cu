@@ -157,9 +157,15 @@ bool mma_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc,
 
 namespace {
 
-// level activation: 1 ReLU, 2 SiLU (x / (1 + e^-x) with the fast approximate division: bf16 outputs)
+// level activation: 1 ReLU, 2 SiLU (h + h tanh(h), h = x / 2, one tanh.approx: bf16 outputs)
 __device__ __forceinline__ float act_apply(float x, int act) {
-  return act == 2 ? __fdividef(x, 1.f + __expf(-x)) : fmaxf(x, 0.f);
+  if (act == 2) {
+    const float h = 0.5f * x;
+    float t;
+    asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(h));
+    return fmaf(h, t, h);
+  }
+  return fmaxf(x, 0.f);
 }
 
 __device__ __forceinline__ uint32_t s_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }

@@ -362,7 +362,7 @@ __device__ __forceinline__ uint32_t pack_relu(float lo, float hi) {   // bf16x2(
 
 template <bool SILU>
 __device__ __forceinline__ float silu_or(float x, int act) {
-  if constexpr (SILU) return act == 2 ? __fdividef(x, 1.f + __expf(-x)) : x;
+  if constexpr (SILU) return act == 2 ? silu_fast(x) : x;
   else return x;
 }
 
@@ -392,6 +392,9 @@ __device__ __forceinline__ void level_math(uint32_t (&t)[16], const uint32_t (&v
   if (act == 1) {
 #pragma unroll
     for (int i = 0; i < 16; ++i) t[i] = pack_relu(z[2 * i], z[2 * i + 1]);
+  } else if (SILU && act == 2) {
+#pragma unroll
+    for (int i = 0; i < 16; ++i) t[i] = pack_silu_bf16(z[2 * i], z[2 * i + 1]);
   } else {
 #pragma unroll
     for (int i = 0; i < 16; ++i) t[i] = pack_bf16(silu_or<SILU>(z[2 * i], act), silu_or<SILU>(z[2 * i + 1], act));

@@ -668,7 +668,7 @@ struct Ring {
 // pooled-member activation: ReLU when a != 0; SILU instantiation: a == 2 -> SiLU
 template <bool SILU>
 __device__ __forceinline__ float act_m(float x, int a) {
-  if constexpr (SILU) return a == 2 ? __fdividef(x, 1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  if constexpr (SILU) return a == 2 ? silu_fast(x) : (a ? fmaxf(x, 0.f) : x);
   else return a ? fmaxf(x, 0.f) : x;
 }
 
@@ -1079,7 +1079,7 @@ __global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_cons
           const int act = d.relu[un.pooled ? 0 : l];
           if (SILU && act == 2) {   // SiLU level: applied in place, then the no-activation path
 #pragma unroll
-            for (int i = 0; i < 32; ++i) t[i] = __fdividef(t[i], 1.f + __expf(-t[i]));
+            for (int i = 0; i < 32; ++i) t[i] = silu_fast(t[i]);
           }
           const bool relu = SILU ? act == 1 : act != 0;
           if (!last) {

@@ -634,7 +634,7 @@ using namespace ptx;
 // fast approximate division, bf16 outputs).  ReLU-only plans launch SILU = false: epilogue unchanged
 template <bool SILU>
 __device__ __forceinline__ float act_w(float x, int a) {
-  if constexpr (SILU) return a == 2 ? __fdividef(x, 1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  if constexpr (SILU) return a == 2 ? silu_fast(x) : (a ? fmaxf(x, 0.f) : x);
   else return a ? fmaxf(x, 0.f) : x;
 }
 
@@ -735,7 +735,7 @@ __device__ __forceinline__ TileGeo tile_geo(const TcChainDesc& d, int tile) {
 // pooled-member activation: ReLU when a != 0; SILU instantiation: a == 2 -> SiLU
 template <bool SILU>
 __device__ __forceinline__ float act_m(float x, int a) {
-  if constexpr (SILU) return a == 2 ? __fdividef(x, 1.f + __expf(-x)) : (a ? fmaxf(x, 0.f) : x);
+  if constexpr (SILU) return a == 2 ? silu_fast(x) : (a ? fmaxf(x, 0.f) : x);
   else return a ? fmaxf(x, 0.f) : x;
 }
 

@@ -219,6 +219,27 @@ __device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
   return *reinterpret_cast<uint32_t*>(&h);
 }
 
+// silu(x) = h + h tanh(h), h = x / 2, one MUFU operation (tanh.approx.f32, relative error
+// ~2^-11) instead of an exponential and a reciprocal: bf16-output tensor-core epilogues only
+__device__ __forceinline__ float silu_fast(float x) {
+  const float h = 0.5f * x;
+  float t;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(h));
+  return fmaf(h, t, h);
+}
+
+// bf16x2 of (silu(a), silu(b)) for epilogues whose output is bf16: silu(x) = h + h tanh(h),
+// h = x / 2, with one packed bf16x2 tanh (one MUFU operation per two values instead of an
+// exponential and a reciprocal per value); tanh in bf16 adds <= 2^-9 |h| absolute error, below
+// the bf16 rounding of the output itself
+__device__ __forceinline__ uint32_t pack_silu_bf16(float a, float b) {
+  const float ha = 0.5f * a, hb = 0.5f * b;
+  uint32_t hp = pack_bf16(ha, hb), th;
+  asm("tanh.approx.bf16x2 %0, %1;" : "=r"(th) : "r"(hp));
+  const float ta = __uint_as_float(th << 16), tb = __uint_as_float(th & 0xFFFF0000u);
+  return pack_bf16(fmaf(ha, ta, ha), fmaf(hb, tb, hb));
+}
+
 // bf16x2 of (max(a, 0), max(b, 0)) in one instruction
 __device__ __forceinline__ uint32_t pack_bf16_relu(float a, float b) {
   uint32_t r;
