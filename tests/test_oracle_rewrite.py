@@ -395,3 +395,61 @@ def test_cp_pair_not_formed_when_the_intermediate_has_another_reader():
     on = dict(p.onodes)
     on[10_000] = type(v)(10_000, "relu", [v.id], C=v.C, H=v.H, W=v.W)
     assert pair_cp_cores(O, on, {}) == {}
+
+
+# ----------------------------------------------------------------------------
+# reading R35: a 1x1 core folds into the fconv feeding it
+# ----------------------------------------------------------------------------
+
+def _fold_model():
+    from workloads import Decomp, Layer, Model
+    rng = np.random.default_rng(21)
+    m = Model("fold", 1, 5, 5, 4, "f32")
+    m.layers = [Layer("input", [], out_channels=4),
+                Layer("conv", [0], out_channels=6, kernel=1),
+                Layer("relu", [1]),
+                Layer("conv", [2], out_channels=4, kernel=1)]
+    m.decomps = {1: Decomp(1, "tucker2", 2, 3, rng.standard_normal((2, 4)), rng.standard_normal((3, 2, 1, 1)),
+                           None, rng.standard_normal((6, 3))),
+                 3: Decomp(3, "tucker2", 3, 2, rng.standard_normal((3, 6)), rng.standard_normal((2, 3, 1, 1)),
+                           None, rng.standard_normal((4, 2)))}
+    return m
+
+
+def test_fold_1x1_core_by_hand():
+    """fconv 4 -> 2, core 1x1 2 -> 3, lconv 3 -> 6, ReLU, fconv 6 -> 3, core 3 -> 2, lconv 2 -> 4 on
+    5 x 5 (fp32, 100 B per channel).  Folded: node 2 = fconv 4 -> 3 with weight G2 F1, node 6 =
+    fconv 6 -> 2 with G6 F5; steps input, fconv'(2), group {3, 4, 6}, group {7}; live bytes
+    [400, 400 + 300, 300 + 200, 200 + 400].  Unfolded: [400, 600, 500, 600, 500, 600]."""
+    m = _fold_model()
+    a = oracle.plan(m, fold_cores=False)
+    b = oracle.plan(m)
+    assert a.live_fused == [400, 600, 500, 600, 500, 600]
+    assert b.live_fused == [400, 700, 500, 600] and b.peak_fused == 700
+    assert [s.out for s in b.steps] == [0, 2, 6, 7]
+    n2, n6 = b.onodes[2], b.onodes[6]
+    assert (n2.role, n2.inputs, n2.C, n6.role, n6.inputs, n6.C) == ("fconv", [0], 3, "fconv", [4], 2)
+    d1, d3 = m.decomps[1], m.decomps[3]
+    np.testing.assert_allclose(n2.weight[:, :, 0, 0], d1.core[:, :, 0, 0] @ d1.first, rtol=1e-12)
+    np.testing.assert_allclose(n6.weight[:, :, 0, 0], d3.core[:, :, 0, 0] @ d3.first, rtol=1e-12)
+    x = W.make_input(m)
+    np.testing.assert_allclose(oracle.run_temco(b, x), oracle.run_unfused(b, x), rtol=1e-10, atol=1e-12)
+
+
+def test_fold_skips_shared_fconv_outputs_and_kxk_cores():
+    """No fold when the fconv output has another reader or the core is K x K / strided (R35)."""
+    from oracle.rewrite import fold_1x1_cores
+    m = _fold_model()
+    p = oracle.plan(m, fold_cores=False)
+    O = list(p.O) + [10_000]
+    on = dict(p.onodes)
+    on[10_000] = type(on[1])(10_000, "relu", [1], C=2, H=5, W=5)      # a second reader of fconv 1
+    O2, on2 = fold_1x1_cores(O, on, 0)
+    assert 1 in O2 and on2[2].role == "core"
+    r = W.resnet50(batch=1, dtype="f32", height=32, width=32)
+    pr = oracle.plan(r)
+    # every unstrided 1x1 core of ResNet-50 is folded; the stride-2 downsample cores are kept
+    assert all(not (n.role == "core" and n.kh == 1 and n.kw == 1 and n.sh == 1 and pr.onodes[n.inputs[0]].role == "fconv")
+               for n in (pr.onodes[x] for x in pr.O))
+    assert any(pr.onodes[x].role == "core" and pr.onodes[x].kh == 1 and pr.onodes[x].sh == 2 for x in pr.O)
+    assert any(pr.onodes[x].role == "core" and pr.onodes[x].kh == 3 for x in pr.O)
