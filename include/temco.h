@@ -128,6 +128,9 @@ enum {
   TEMCO_FLAG_OVERHEAD_ALWAYS = 1 << 5, /* force Overhead() true  (tests)                 */
   TEMCO_FLAG_OVERHEAD_NEVER = 1 << 6,  /* force Overhead() false (tests)                 */
   TEMCO_FLAG_MMA_SMALL = 1 << 7,       /* run groups with C <= 256 on the mma.sync kernel */
+  TEMCO_FLAG_PAPER_SCHEDULE = 1 << 9,  /* the paper's schedule exactly: without the round-2
+                                          extensions R34 (CP depthwise core pair as one step) and
+                                          R35 (a 1x1 core folded into the fconv feeding it)     */
   TEMCO_FLAG_MMA_CAT = 1 << 8          /* single-level concat groups on the mma.sync concat
                                           kernel (kernels_cat.cu; measured slower than tcgen05) */
 };

@@ -809,6 +809,7 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
   opt.distance_threshold = cfg->distance_threshold > 0 ? cfg->distance_threshold : 1;
   opt.skip_opt = !(cfg->flags & TEMCO_FLAG_NO_SKIPOPT);
   opt.fusion = !(cfg->flags & TEMCO_FLAG_NO_FUSION);
+  opt.extensions = !(cfg->flags & TEMCO_FLAG_PAPER_SCHEDULE);
   opt.overhead_policy = (cfg->flags & TEMCO_FLAG_OVERHEAD_ALWAYS) ? 1 : (cfg->flags & TEMCO_FLAG_OVERHEAD_NEVER) ? 2 : 0;
   opt.bf16 = P->bf16;
   std::string err;

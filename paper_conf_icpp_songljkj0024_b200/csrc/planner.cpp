@@ -560,7 +560,49 @@ void dce(IR& ir) {   // reading R11
   }
 }
 
-void group_and_schedule(IR& ir, bool fusion) {
+// reading R35 (oracle: fold_1x1_cores): an unstrided, unpadded, ungrouped, bias-free 1x1 core
+// whose input is an fconv read by nothing else folds into that fconv (two linear 1x1 maps):
+// the core's node becomes the fconv with weight G F, the fconv leaves O
+void fold_1x1_cores(IR& ir) {
+  std::map<int, std::vector<int>> cons;
+  for (int x : ir.O) {
+    std::vector<int> seen;
+    for (int p : ir.oin[x])
+      if (std::find(seen.begin(), seen.end(), p) == seen.end()) {
+        seen.push_back(p);
+        cons[p].push_back(x);
+      }
+  }
+  std::set<int> drop;
+  for (int x : ir.O) {
+    Node& c = ir.nodes[x];
+    if (!(c.op == OP_CONV && c.role == ROLE_CORE && c.kh == 1 && c.kw == 1 && c.sh == 1 && c.sw == 1 && c.ph == 0 &&
+          c.pw == 0 && c.groups == 1 && !c.b && ir.oin[x].size() == 1))
+      continue;
+    const int fi = ir.oin[x][0];
+    const Node& f = ir.nodes[fi];
+    if (fi == ir.input || f.op != OP_CONV || f.role != ROLE_FCONV || f.kh != 1 || f.kw != 1 || f.b) continue;
+    if (cons[fi].size() != 1 || cons[fi][0] != x) continue;
+    const int R_out = c.C, R_in = f.C, Cin = ir.nodes[ir.oin[fi][0]].C;
+    auto w = std::make_shared<std::vector<float>>((size_t)R_out * Cin, 0.f);
+    for (int o = 0; o < R_out; ++o)
+      for (int k = 0; k < R_in; ++k) {
+        const double g = (*c.w)[(size_t)o * R_in + k];
+        for (int i = 0; i < Cin; ++i) (*w)[(size_t)o * Cin + i] += (float)(g * (*f.w)[(size_t)k * Cin + i]);
+      }
+    c.role = ROLE_FCONV;
+    c.w = w;
+    c.in = f.in;
+    ir.oin[x] = ir.oin[fi];
+    drop.insert(fi);
+  }
+  std::vector<int> O;
+  for (int x : ir.O)
+    if (!drop.count(x)) O.push_back(x);
+  ir.O = O;
+}
+
+void group_and_schedule(IR& ir, bool fusion, bool extensions) {
   std::map<int, int> pos;
   for (size_t i = 0; i < ir.O.size(); ++i) pos[ir.O[i]] = (int)i;
   std::map<int, std::vector<int>> cons;
@@ -614,7 +656,7 @@ void group_and_schedule(IR& ir, bool fusion) {
       grouped.insert(mem.begin(), mem.end());
     }
   }
-  if (fusion) {
+  if (fusion && extensions) {
     // reading R34: the K x 1 and 1 x K depthwise cores of one CP decomposition
     // form one step when the K x 1 output has no other consumer (oracle: pair_cp_cores)
     for (int x : ir.O) {
@@ -686,7 +728,8 @@ temco_status build_ir(const temco_layer* layers, int n_layers, const temco_decom
       skip_opt(ir, opt);
       dce(ir);
     }
-    group_and_schedule(ir, opt.fusion);
+    if (opt.fusion && opt.extensions) fold_1x1_cores(ir);
+    group_and_schedule(ir, opt.fusion, opt.extensions);
     ir.peak_fused = peak_of(ir, ir.steps, ir.live_fused);
     return TEMCO_OK;
   } catch (const Fail& f) {

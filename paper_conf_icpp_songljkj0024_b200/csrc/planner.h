@@ -75,6 +75,7 @@ struct BuildOptions {
   int distance_threshold = 1;
   bool skip_opt = true;
   bool fusion = true;
+  bool extensions = true;        // readings R34 (CP core pair) and R35 (1x1 core folded into its fconv)
   int overhead_policy = 0;       // 0 paper, 1 always, 2 never
   bool bf16 = false;
 };

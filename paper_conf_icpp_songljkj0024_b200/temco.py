@@ -30,6 +30,7 @@ FLAG_OVERHEAD_ALWAYS = 1 << 5
 FLAG_OVERHEAD_NEVER = 1 << 6
 FLAG_MMA_SMALL = 1 << 7
 FLAG_MMA_CAT = 1 << 8
+FLAG_PAPER_SCHEDULE = 1 << 9   # without the round-2 schedule extensions R34 / R35
 
 EXPORTS = ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_peak_internal_bytes", "temco_output_shape",
            "temco_plan_describe", "temco_run_profiled", "temco_debug_step_output", "temco_plan_destroy",

@@ -8,7 +8,7 @@ import pytest
 import oracle
 import workloads as W
 from paper_conf_icpp_songljkj0024_b200 import (FLAG_NO_DEVICE, FLAG_NO_FUSION, FLAG_NO_SKIPOPT,
-                                              FLAG_OVERHEAD_NEVER, Plan, TemcoError)
+                                              FLAG_OVERHEAD_NEVER, FLAG_PAPER_SCHEDULE, Plan, TemcoError)
 
 KEYS = ("kind", "out", "op", "role", "members", "inputs", "bytes")
 
@@ -47,6 +47,14 @@ def test_full_configs(name):
     # the north-star >= 70 % target is stated for the BASELINE.json configs; AlexNet (f2, no
     # skip connections: activation-layer fusion only, P:L355 reports 49.4 %) reaches 54.9 %
     assert 1 - p.peak_internal_bytes(0) / p.peak_internal_bytes(1) >= (0.54 if name == "alexnet" else 0.70)
+
+
+@pytest.mark.parametrize("name", FULL + list(SMALL))
+def test_paper_schedule_mode(name):
+    """TEMCO_FLAG_PAPER_SCHEDULE == the oracle without readings R34 / R35 (the paper's own
+    schedule, whose peaks SURVEY P2 pins)."""
+    m = W.build_config(name) if name in FULL else SMALL[name]()
+    _compare(m, FLAG_PAPER_SCHEDULE, cp_pair=False, fold_cores=False)
 
 
 @pytest.mark.parametrize("name", ["t2_3", "t3", "t4"])
