@@ -74,7 +74,7 @@ def test_eq3_original_peak(case):
 def test_eq4_decomposed_peak_and_fig5_fused_peak(case):
     C, Cp, Cpp, H, Wd, k1, s1, k2, s2, (C1, C2, C3, C4) = case
     m, (hw, hw1, hw2) = fig3_chain(C, Cp, Cpp, H, Wd, k1, s1, k2, s2, (C1, C2, C3, C4))
-    pl = oracle.plan(m, cp_pair=False, fold_cores=False)   # the paper's schedule (Fig. 5)
+    pl = oracle.plan(m, cp_pair=False, fold_cores=False, pool_first=False)   # the paper's schedule (Fig. 5)
     eq4 = max(C * hw + C1 * hw, C1 * hw + C2 * hw1, C2 * hw1 + Cp * hw1, 2 * Cp * hw1,
               Cp * hw1 + C3 * hw1, C3 * hw1 + C4 * hw2, C4 * hw2 + Cpp * hw2)
     assert pl.peak_unfused == eq4 * 4
@@ -295,7 +295,7 @@ def test_full_config_peaks_meet_the_70_percent_target(name, unfused, fused):
     """Values at the configs' batch and bf16 (SURVEY.md table P2 was produced
     by an independent simulation under the same readings; here they are a
     regression pin and the >= 70 % north-star target)."""
-    pl = oracle.plan(W.build_config(name), cp_pair=False, fold_cores=False)   # paper schedule
+    pl = oracle.plan(W.build_config(name), cp_pair=False, fold_cores=False, pool_first=False)   # paper schedule
     assert (pl.peak_unfused, pl.peak_fused) == (unfused, fused)
     assert 1 - pl.peak_fused / pl.peak_unfused >= 0.70
 
@@ -305,7 +305,7 @@ def test_extended_schedule_peaks(name):
     """With readings R34 / R35 (the default plan) the fused peak never exceeds the paper
     schedule's on the four configs and keeps the >= 70 % target."""
     m = W.build_config(name)
-    ext, paper = oracle.plan(m), oracle.plan(m, cp_pair=False, fold_cores=False)
+    ext, paper = oracle.plan(m), oracle.plan(m, cp_pair=False, fold_cores=False, pool_first=False)
     assert ext.peak_unfused == paper.peak_unfused
     assert ext.peak_fused <= paper.peak_fused
     assert 1 - ext.peak_fused / ext.peak_unfused >= 0.70
@@ -464,3 +464,44 @@ def test_fold_skips_shared_fconv_outputs_and_kxk_cores():
                for n in (pr.onodes[x] for x in pr.O))
     assert any(pr.onodes[x].role == "core" and pr.onodes[x].kh == 1 and pr.onodes[x].sh == 2 for x in pr.O)
     assert any(pr.onodes[x].role == "core" and pr.onodes[x].kh == 3 for x in pr.O)
+
+
+# ----------------------------------------------------------------------------
+# reading R36: average pool before the restore, shared by every copy
+# ----------------------------------------------------------------------------
+
+def test_pool_before_restore_densenet_transitions():
+    """DenseNet's transition output reaches every group of the next block as a pooled restore
+    copy avgpool(lconv(r)); R36 turns each copy into lconv(p) with ONE shared p = avgpool(r) on
+    the reduced channels, placed right after r.  Same tensor, no pooled member left,
+    never a higher peak."""
+    m = W.densenet121(batch=1, dtype="f32", height=64, width=64)
+    a = oracle.plan(m, pool_first=False)
+    b = oracle.plan(m)
+    pools = [x for x in b.O if b.onodes[x].op == "avgpool"]
+    assert len(pools) == 3                                   # one per transition
+    for x in pools:
+        p = b.onodes[x]
+        r = b.onodes[p.inputs[0]]
+        assert b.O[b.O.index(r.id) + 1] == x                 # right after r
+        assert (p.C, p.H, p.W) == (r.C, r.H // 2, r.W // 2) and r.role == "fconv"
+        users = [y for y in b.O if x in b.onodes[y].inputs]
+        assert len(users) > 5 and all(b.onodes[y].role == "lconv" for y in users)
+    assert not any(b.onodes[x].op == "avgpool" and b.onodes[b.onodes[x].inputs[0]].role == "lconv" for x in b.O)
+    assert b.peak_fused <= a.peak_fused
+    x = W.make_input(m)
+    np.testing.assert_allclose(oracle.run_temco(b, x), oracle.run_unfused(b, x), rtol=1e-9, atol=1e-12)
+    np.testing.assert_allclose(oracle.run_temco(b, x), oracle.run_temco(a, x), rtol=1e-9, atol=1e-12)
+
+
+def test_pool_before_restore_commutes_by_hand():
+    """avgpool_2x2(L r + b) == L avgpool_2x2(r) + b on a literal 2 x 2 window (the identity R36
+    rests on): r = [[1, 2], [3, 4]] (one channel), L = [2, -1], b = [0.5, 0]."""
+    from oracle.ops import avgpool, conv2d
+    r = np.array([1.0, 2.0, 3.0, 4.0]).reshape(1, 2, 2, 1)
+    Lw = np.array([[2.0], [-1.0]])[:, :, None, None]
+    b = np.array([0.5, 0.0])
+    restore_then_pool = avgpool(conv2d(r, Lw, b, (1, 1), (0, 0), 1), 2, 2)
+    pool_then_restore = conv2d(avgpool(r, 2, 2), Lw, b, (1, 1), (0, 0), 1)
+    np.testing.assert_allclose(restore_then_pool.ravel(), [5.5, -2.5])
+    np.testing.assert_allclose(pool_then_restore.ravel(), [5.5, -2.5])
