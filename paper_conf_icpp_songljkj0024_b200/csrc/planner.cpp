@@ -5,6 +5,7 @@
 #include <algorithm>
 #include <numeric>
 #include <set>
+#include <tuple>
 #include <sstream>
 
 namespace temco {
@@ -602,6 +603,69 @@ void fold_1x1_cores(IR& ir) {
   ir.O = O;
 }
 
+// reading R36 (oracle: pool_before_restore): avgpool(lconv(r)) = lconv(avgpool(r)); each pooled
+// restore copy becomes a plain restore of ONE shared pooled reduced tensor placed right after r
+void pool_before_restore(IR& ir) {
+  std::map<int, std::vector<int>> cons;
+  for (int x : ir.O) {
+    std::vector<int> seen;
+    for (int p : ir.oin[x])
+      if (std::find(seen.begin(), seen.end(), p) == seen.end()) {
+        seen.push_back(p);
+        cons[p].push_back(x);
+      }
+  }
+  std::map<std::tuple<int, int, int, int, int>, int> shared;
+  std::map<int, std::vector<int>> placed;   // r -> pooled nodes to insert after it
+  std::set<int> drop;
+  for (int x : ir.O) {
+    const Node a = ir.nodes[x];
+    if (a.op != OP_AVGPOOL || ir.oin[x].size() != 1) continue;
+    const int li = ir.oin[x][0];
+    const Node l = ir.nodes[li];
+    if (!(l.op == OP_CONV && l.role == ROLE_LCONV && l.kh == 1 && l.kw == 1 && l.sh == 1 && l.sw == 1 &&
+          l.groups == 1 && cons[li].size() == 1 && cons[li][0] == x))
+      continue;
+    const int ri = ir.oin[li][0];
+    const Node& r = ir.nodes[ri];
+    const auto key = std::make_tuple(ri, a.kh, a.kw, a.sh, a.sw);
+    auto it = shared.find(key);
+    int pid;
+    if (it == shared.end()) {
+      Node p;
+      p.op = OP_AVGPOOL; p.orig = a.orig; p.in = {ri};
+      p.kh = a.kh; p.kw = a.kw; p.sh = a.sh; p.sw = a.sw; p.ph = a.ph; p.pw = a.pw;
+      p.C = r.C; p.H = a.H; p.W = a.W;
+      pid = (int)ir.nodes.size();
+      p.id = pid;
+      ir.oin.push_back({ri});
+      ir.nodes.push_back(std::move(p));
+      shared[key] = pid;
+      placed[ri].push_back(pid);
+    } else {
+      pid = it->second;
+    }
+    Node q = l;          // the pooled node becomes the restore of the pooled reduced tensor
+    q.id = x;
+    q.in = {pid};
+    q.H = a.H;
+    q.W = a.W;
+    q.copy_of = l.copy_of;
+    ir.nodes[x] = q;
+    ir.oin[x] = {pid};
+    drop.insert(li);
+  }
+  if (shared.empty()) return;
+  std::vector<int> O;
+  for (int x : ir.O) {
+    if (drop.count(x)) continue;
+    O.push_back(x);
+    auto pl = placed.find(x);
+    if (pl != placed.end()) O.insert(O.end(), pl->second.begin(), pl->second.end());
+  }
+  ir.O = O;
+}
+
 void group_and_schedule(IR& ir, bool fusion, bool extensions) {
   std::map<int, int> pos;
   for (size_t i = 0; i < ir.O.size(); ++i) pos[ir.O[i]] = (int)i;
@@ -728,7 +792,10 @@ temco_status build_ir(const temco_layer* layers, int n_layers, const temco_decom
       skip_opt(ir, opt);
       dce(ir);
     }
-    if (opt.fusion && opt.extensions) fold_1x1_cores(ir);
+    if (opt.fusion && opt.extensions) {
+      fold_1x1_cores(ir);
+      pool_before_restore(ir);
+    }
     group_and_schedule(ir, opt.fusion, opt.extensions);
     ir.peak_fused = peak_of(ir, ir.steps, ir.live_fused);
     return TEMCO_OK;
