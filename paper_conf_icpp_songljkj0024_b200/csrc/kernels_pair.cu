@@ -59,7 +59,7 @@ constexpr int kSlotC = 2048;             // 64 rows x 16 bf16 (bias-MMA groups: 
 // ring stage: A + B for both units of a pair (+ C for both with bias-MMA): PairDesc::slot bytes
 constexpr int kOnesBytes = 4096;         // 128 rows x 16 bf16 "ones" A tile of the bias MMA
 constexpr int kPBytes = 128 * kPairWu * 2;   // P of one unit: two SW128 atoms of 128 x 64
-constexpr int kBarBytes = 2048;   // barriers (first 1 KB) + the issuer's atom table (kTabOff)
+constexpr int kBarBytes = 1024 + 16 * kPairMaxAtoms;   // barriers (first 1 KB) + the issuer's atom table (kTabOff)
 constexpr int kTabOff = 1024;
 constexpr int kPairMaxStages = 16;
 constexpr int kChunk = 2;                // ring stages of one level consumed per (u0 pass, u1 pass)
@@ -135,6 +135,7 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     }
   }
   int j = 0;
+  std::vector<int> term_c0, term_c1;   // restored channel range of each term
   for (int l = 0; l < d.n_levels; ++l) {
     for (const PTerm& t : levels[l].terms) {
       const Node& lc = ir.nodes[t.lconv];
@@ -150,31 +151,42 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
       for (int c = 0; c < lc.C; ++c)
         for (int k = 0; k < R; ++k) w[(size_t)(t.c0 + c) * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
       T.w = push_bf16(tcw, w);
+      term_c0.push_back(t.c0);
+      term_c1.push_back(t.c0 + lc.C);
       flops += d.npix * 2LL * lc.C * R;
       bytes += d.npix * 2LL * R;
     }
     d.lvl_end[l] = j;
   }
   d.n_terms = j;
-  // per-pair atom program (identical for every unit pair), in the launch parameters so the
-  // issuer's loop state stays warp-uniform (uniform registers, no per-MMA broadcasts)
+  // per-unit-pair atom programs, in the launch parameters: pair pp runs the atoms of the terms
+  // whose restored channel range meets its 256 channels (every term of a residual chain; a
+  // concat member only in the pair(s) holding its channels -- DenseNet's 32-channel members)
   {
-    int n = 0, jj = 0;
-    for (int l = 0; l < d.n_levels; ++l) {
-      const int n0 = n;
-      for (; jj < d.lvl_end[l]; ++jj) {
-        const PairTerm& T = d.term[jj];
-        for (int a = 0; a < T.natoms; ++a, ++n) {
-          if (n >= kPairMaxAtoms) return false;
-          const int nk = std::min(T.aw / 16, (T.R - a * T.aw + 15) / 16);
-          d.prog[n][0] = (uint32_t)jj | ((uint32_t)T.aw << 8) | ((uint32_t)nk << 16) | ((n == n0 ? 1u : 0u) << 24) |
-                         ((l == 0 ? 4u : 0u) << 24) | ((uint32_t)l << 28);
-          d.prog[n][1] = (uint32_t)(a * T.aw);
+    const int UPn = (d.nunits + 1) / 2;
+    if (UPn > kPairMaxUnitPairs) return false;
+    int n = 0;
+    for (int pp = 0; pp < UPn; ++pp) {
+      d.pstart[pp] = (int16_t)n;
+      const int ch0 = pp * 2 * kPairWu, ch1 = std::min(C, ch0 + 2 * kPairWu);
+      for (int l = 0, jj = 0; l < d.n_levels; ++l) {
+        const int n0 = n;
+        for (; jj < d.lvl_end[l]; ++jj) {
+          if (term_c1[jj] <= ch0 || term_c0[jj] >= ch1) continue;
+          const PairTerm& T = d.term[jj];
+          for (int a = 0; a < T.natoms; ++a, ++n) {
+            if (n >= kPairMaxAtoms) return false;
+            const int nk = std::min(T.aw / 16, (T.R - a * T.aw + 15) / 16);
+            d.prog[n][0] = (uint32_t)jj | ((uint32_t)T.aw << 8) | ((uint32_t)nk << 16) | ((n == n0 ? 1u : 0u) << 24) |
+                           ((l == 0 ? 4u : 0u) << 24) | ((uint32_t)l << 28);
+            d.prog[n][1] = (uint32_t)(a * T.aw);
+          }
         }
+        if (n == n0) return false;      // a level with nothing in this pair (not produced by the parser)
+        d.prog[n - 1][0] |= 2u << 24;   // last atom of the level
       }
-      d.prog[n - 1][0] |= 2u << 24;   // last atom of the level
+      d.prog[n - 1][0] |= 8u << 24;     // last atom of the pair's program
     }
-    d.prog[n - 1][0] |= 8u << 24;     // last atom of the program
     d.n_prog = n;
   }
   std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
@@ -224,7 +236,7 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     const int UP = (d.nunits + 1) / 2;
     d.bsz = 64 * awmax * 2;
     d.fsz = d.Np / 2 * 128;
-    const int rb = UP * d.n_prog * 2 * d.bsz;
+    const int rb = d.n_prog * 2 * d.bsz;
     const int rc = d.bias_mma ? UP * d.n_levels * 2 * kSlotC : 0;
     const int rf = d.nunits * 2 * d.fsz;
     d.res_c = (rb + 1023) / 1024 * 1024;
@@ -233,14 +245,17 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     int64_t tx = 0;
     for (int pp = 0; pp < UP; ++pp) {
       const int nu = std::min(2, d.nunits - 2 * pp);
-      for (int k = 0; k < d.n_prog; ++k) tx += nu * 64 * (int)((d.prog[k][0] >> 8) & 0xFF) * 2;
+      const int pend = pp + 1 < UP ? d.pstart[pp + 1] : d.n_prog;
+      for (int k = d.pstart[pp]; k < pend; ++k) tx += nu * 64 * (int)((d.prog[k][0] >> 8) & 0xFF) * 2;
       if (d.bias_mma) tx += (int64_t)nu * d.n_levels * 64 * 16 * 2;
     }
     tx += (int64_t)d.nunits * 2 * d.fsz;
     d.res_tx = (int)tx;
     const int slot_r = 128 * awmax * 2;
     const int st_r = std::min(kPairMaxStages, (budget - d.res_bytes) / slot_r);
-    d.resident = !getenv("TEMCO_PAIR_NO_RES") && st_r >= std::max(8, d.n_prog + 2) ? 1 : 0;
+    int maxp = 0;   // longest unit-pair program
+    for (int pp = 0; pp < UP; ++pp) maxp = std::max(maxp, (pp + 1 < UP ? d.pstart[pp + 1] : d.n_prog) - d.pstart[pp]);
+    d.resident = !getenv("TEMCO_PAIR_NO_RES") && st_r >= std::max(8, maxp + 2) ? 1 : 0;
     if (d.resident) {
       d.slot = slot_r;
       d.stages = st_r;
@@ -518,11 +533,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         const uint32_t wb = mapa_shared(smem_u32(wbar), 0);
         for (int pp = 0; pp < UP; ++pp) {
           const int u0 = 2 * pp, nu = min(2, U - u0);
-          for (int k = 0; k < d.n_prog; ++k) {
+          const int pend = pp + 1 < UP ? d.pstart[pp + 1] : d.n_prog;
+          for (int k = d.pstart[pp]; k < pend; ++k) {
             const uint2 op = make_uint2(d.prog[k][0], d.prog[k][1]);
             const PairTerm* T = reinterpret_cast<const PairTerm*>(term0 + (op.x & 0xFF) * sizeof(PairTerm));
             for (int q = 0; q < nu; ++q) {
-              tma_load_2d_pair(res + ((pp * d.n_prog + k) * 2 + q) * d.bsz, T->wmap, wb, (int)op.y,
+              tma_load_2d_pair(res + (k * 2 + q) * d.bsz, T->wmap, wb, (int)op.y,
                                (u0 + q) * kPairWu + (int)cta * 64);
               if (d.bias_mma && ((op.x >> 24) & 1u))
                 tma_load_2d_pair(res + d.res_c + ((pp * d.n_levels + (int)(op.x >> 28)) * 2 + q) * kSlotC, d.bmap, wb, 0,
@@ -538,7 +554,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         const int row0 = tile * 256 + (int)cta * 128;
         for (int pp = 0; pp < UP; ++pp) {
           const int u0 = 2 * pp, nu = min(2, U - u0);
-          for (int k = 0;; ++k) {
+          for (int k = d.pstart[pp];; ++k) {
             const uint2 op = make_uint2(d.prog[k][0], d.prog[k][1]);
             const int j = op.x & 0xFF, aw = (op.x >> 8) & 0xFF;
             const uint32_t fl = op.x >> 24;
@@ -595,7 +611,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       }
       const uint32_t a_lo0 = udesc_lo(sbase), slot16 = (uint32_t)kSlot >> 4;
       const uint32_t hi16 = udesc_hi(16), hi64 = udesc_hi(64), ones_lo = udesc_lo(smem_u32(ones));
-      const uint32_t pb_step = (uint32_t)(d.n_prog * 2 * d.bsz) >> 4, bq16 = (uint32_t)d.bsz >> 4;
+      const uint32_t bq16 = (uint32_t)d.bsz >> 4;
       const uint32_t pc_step = (uint32_t)(d.n_levels * 2 * kSlotC) >> 4, cq16 = (uint32_t)kSlotC >> 4;
       int stage = 0;
       uint32_t ph = 0;
@@ -645,8 +661,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       for (int tile = pair_id; tile < d.ntiles; tile += npairs) {
         for (int pp = 0; pp < UP; ++pp) {
           const int nu = min(2, U - 2 * pp);
-          const uint32_t pbo = (uint32_t)pp * pb_step, pco = (uint32_t)pp * pc_step;
-          int k = 0;
+          const uint32_t pco = (uint32_t)pp * pc_step;
+          int k = d.pstart[pp];
           for (;;) {   // one level per iteration, in chunks of <= kChunk ring stages
             const uint32_t op0x = lds128(tab_s + 16u * k).x;
             int kl = k;   // last atom of this level
@@ -688,7 +704,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                 const bool lvl0 = c0 == 0 && i == 0;   // first atom of the level
                 const bool bia = d.bias_mma && lvl0;
                 const uint32_t a_lo = a_lo0 + (uint32_t)st * slot16;
-                const uint32_t b0_lo = d.resident ? tk.z + pbo : a_lo + ((uint32_t)kSlotA >> 4);
+                const uint32_t b0_lo = d.resident ? tk.z : a_lo + ((uint32_t)kSlotA >> 4);
                 const uint32_t b1_lo = b0_lo + (d.resident ? bq16 : ((uint32_t)kSlotB >> 4));
                 const uint32_t c0_lo = d.resident ? tk.w + pco : a_lo + ((uint32_t)(kSlotA + 2 * kSlotB) >> 4);
                 const uint32_t c1_lo = c0_lo + (d.resident ? cq16 : ((uint32_t)kSlotC >> 4));

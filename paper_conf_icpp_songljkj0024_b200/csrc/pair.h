@@ -31,9 +31,10 @@
 namespace temco {
 namespace pair {
 
-constexpr int kPairMaxTerms = 16;
+constexpr int kPairMaxTerms = 32;
+constexpr int kPairMaxUnitPairs = 16;    // C <= 4096
 constexpr int kPairMaxLevels = 16;
-constexpr int kPairMaxAtoms = 64;       // K atoms of one unit's level chain
+constexpr int kPairMaxAtoms = 256;      // K atoms of all unit pairs' programs
 constexpr int kPairMaxActGroups = 256;  // (level, 32-channel group) activation codes
 constexpr int kPairWu = 128;           // restored channels per unit (MMA N of the restore GEMM)
 
@@ -50,8 +51,10 @@ struct PairDesc {
   alignas(64) unsigned char fmap[128];   // F [Np x Cpad] bf16, box {64, Np/2}
   alignas(64) unsigned char bmap[128];   // bias-MMA groups: [n_levels*Cpad x 16] bf16 (hi, lo), box {16, 64}
   int32_t n_terms, n_levels;
-  uint32_t prog[kPairMaxAtoms][2];       // atom program: term | aw << 8 | K16 steps << 16 | flags << 24 | level << 28; x
-  int32_t n_prog;
+  uint32_t prog[kPairMaxAtoms][2];       // atom programs: term | aw << 8 | K16 steps << 16 | flags << 24 | level << 28; x
+  int32_t n_prog;                        // atoms of all programs
+  int16_t pstart[kPairMaxUnitPairs];     // unit pair pp's program: atoms [pstart[pp], next 'last' flag]; a
+                                         // concat term only appears in the pairs whose channels it covers
   int32_t lvl_end[kPairMaxLevels];       // terms [lvl_end[l-1], lvl_end[l]) belong to level l
   int32_t act[kPairMaxLevels];           // 0 none, 1 ReLU, 2 SiLU
   int32_t mixed_act, ngroups;            // per-channel-group activations (activated concat members)
