@@ -10,6 +10,8 @@ computes (PAPER.md = /root/reference/PAPER.md, cited as P:L<line>):
                   Overhead (P:L176, P:L188, P:L219), COPY + InsertBefore
                   (P:L213-214), DCE, activation-layer fusion grouping
                    with the layer transformations,
+                  the merged-fconv CSE (reading R37) and the memory-optimal
+                  re-scheduling of S (reading R38),
                   and the peak internal-tensor accounting (Eq. (3)/(4),
                   P:L109-120),
   * ops.py     -- fp64 direct-loop convolution / BN / ReLU / pools / linear,

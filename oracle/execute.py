@@ -68,6 +68,8 @@ def run_unfused(plan, x):
 
 
 def _eval_group(plan, step, env):
+    """Every output of a fused group (its root; a merged group's further reduce outputs,
+    reading R37, share the one evaluation of the restored tensor)."""
     members = set(step.members)
     memo = {}
 
@@ -82,15 +84,16 @@ def _eval_group(plan, step, env):
         memo[nid] = apply(v, [value(i) for i in v.inputs])
         return memo[nid]
 
-    return value(step.out)
+    return {o: value(o) for o in step.outs}
 
 
-def run_step(plan, t, env):
-    """Output of schedule step t of S given its input tensors env[id] (per-step parity
-    tests feed the GPU's own inputs, so each step is checked in isolation)."""
+def run_step(plan, t, env, which=None):
+    """Output `which` (default: the step's root) of schedule step t of S given its input
+    tensors env[id] (per-step parity tests feed the GPU's own inputs, so each step is
+    checked in isolation)."""
     s = plan.steps[t]
     if s.kind == "group":
-        return _eval_group(plan, s, env)
+        return _eval_group(plan, s, env)[s.out if which is None else which]
     v = plan.onodes[s.out]
     return apply(v, [env[i] for i in v.inputs])
 
@@ -109,7 +112,7 @@ def run_temco(plan, x, on_step=None):
         if t == 0:
             env[s.out] = np.asarray(x, np.float64)
         elif s.kind == "group":
-            env[s.out] = _eval_group(plan, s, env)
+            env.update(_eval_group(plan, s, env))
         else:
             v = plan.onodes[s.out]
             env[s.out] = apply(v, [env[i] for i in v.inputs])

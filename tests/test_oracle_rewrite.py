@@ -74,7 +74,7 @@ def test_eq3_original_peak(case):
 def test_eq4_decomposed_peak_and_fig5_fused_peak(case):
     C, Cp, Cpp, H, Wd, k1, s1, k2, s2, (C1, C2, C3, C4) = case
     m, (hw, hw1, hw2) = fig3_chain(C, Cp, Cpp, H, Wd, k1, s1, k2, s2, (C1, C2, C3, C4))
-    pl = oracle.plan(m, cp_pair=False, fold_cores=False, pool_first=False)   # the paper's schedule (Fig. 5)
+    pl = oracle.plan(m, cp_pair=False, fold_cores=False, pool_first=False, cse=False, reorder=False)   # the paper's schedule (Fig. 5)
     eq4 = max(C * hw + C1 * hw, C1 * hw + C2 * hw1, C2 * hw1 + Cp * hw1, 2 * Cp * hw1,
               Cp * hw1 + C3 * hw1, C3 * hw1 + C4 * hw2, C4 * hw2 + Cpp * hw2)
     assert pl.peak_unfused == eq4 * 4
@@ -240,9 +240,10 @@ def _simulated_peak(pl, steps):
     cur = peak = 0
     live = {}
     for t, s in enumerate(steps):
-        sz = g.size(pl.onodes.get(s.out, g.nodes_by_id[s.out]))
-        live[s.out] = sz
-        cur += sz
+        for o in s.outs:                     # a merged group (R37) allocates every reduce output
+            sz = g.size(pl.onodes.get(o, g.nodes_by_id[o]))
+            live[o] = sz
+            cur += sz
         peak = max(peak, cur)
         for x in list(live):
             if last.get(x, t) <= t and x != g.output:
@@ -296,7 +297,7 @@ def test_full_config_peaks_meet_the_70_percent_target(name, unfused, fused):
     """Values at the configs' batch and bf16 (SURVEY.md table P2 was produced
     by an independent simulation under the same readings; here they are a
     regression pin and the >= 70 % north-star target)."""
-    pl = oracle.plan(W.build_config(name), cp_pair=False, fold_cores=False, pool_first=False)   # paper schedule
+    pl = oracle.plan(W.build_config(name), cp_pair=False, fold_cores=False, pool_first=False, cse=False, reorder=False)   # paper schedule
     assert (pl.peak_unfused, pl.peak_fused) == (unfused, fused)
     assert 1 - pl.peak_fused / pl.peak_unfused >= 0.70
 
@@ -306,7 +307,7 @@ def test_extended_schedule_peaks(name):
     """With readings R34 / R35 (the default plan) the fused peak never exceeds the paper
     schedule's on the four configs and keeps the >= 70 % target."""
     m = W.build_config(name)
-    ext, paper = oracle.plan(m), oracle.plan(m, cp_pair=False, fold_cores=False, pool_first=False)
+    ext, paper = oracle.plan(m), oracle.plan(m, cp_pair=False, fold_cores=False, pool_first=False, cse=False, reorder=False)
     assert ext.peak_unfused == paper.peak_unfused
     assert ext.peak_fused <= paper.peak_fused
     assert 1 - ext.peak_fused / ext.peak_unfused >= 0.70
@@ -506,3 +507,184 @@ def test_pool_before_restore_commutes_by_hand():
     pool_then_restore = conv2d(avgpool(r, 2, 2), Lw, b, (1, 1), (0, 0), 1)
     np.testing.assert_allclose(restore_then_pool.ravel(), [5.5, -2.5])
     np.testing.assert_allclose(pool_then_restore.ravel(), [5.5, -2.5])
+
+
+# ----------------------------------------------------------------------------
+# reading R37: merged-fconv CSE (one restore feeding several fconvs)
+# ----------------------------------------------------------------------------
+
+def test_merged_fconv_t3_by_hand():
+    """t3 (fp32, batch 1): the stem restore t = maxpool(relu(bn(lconv(r1)))) (r1: 2 x 16 x 16,
+    2048 B) feeds block 0's conv1 fconv (node 7, 2 x 8 x 8 = 512 B) and, after Alg. 1's COPY,
+    its downsample fconv (node 21, 4 x 8 x 8 = 1024 B).  R37 runs both reduces in one step:
+    live = r1 + out7 + out21 = 2048 + 512 + 1024 = 3584 B; at the next step r1 is gone:
+    out7 + out21 + out11 = 512 + 1024 + 512 = 2048 B.  The unmerged schedule restores t twice
+    (steps 7 and 21).  Same tensors."""
+    m = W.t3_mini_bottleneck()
+    a = oracle.plan(m, cse=False)
+    b = oracle.plan(m)
+    assert [(s.out, s.extra) for s in b.steps if s.extra] == [(7, [21])]
+    assert [s.out for s in b.steps] == [0, 1, 7, 11, 12, 17, 27, 31, 32, 37, 41]
+    assert b.live_fused[2:4] == [2048 + 512 + 1024, 512 + 1024 + 512]
+    assert b.peak_fused == a.peak_fused == 11264
+    assert 21 not in [s.out for s in b.steps] and b.onodes[21].inputs == b.onodes[7].inputs
+    s7 = b.steps[2]
+    assert set(s7.members) > set(a.steps[2].members) and s7.members[-2:] == [7, 21]
+    # the dropped copy of the restore list is gone from O, b's reduce right after a's
+    assert b.O[b.O.index(7) + 1] == 21 and len(b.O) == len(a.O) - (len(a.steps[6].members) - 1)
+    x = W.make_input(m)
+    np.testing.assert_allclose(oracle.run_temco(b, x), oracle.run_unfused(b, x), rtol=1e-10, atol=1e-12)
+    got = {}
+    oracle.run_temco(b, x, on_step=lambda t, y: got.setdefault(b.steps[t].out, y))
+    ref = {}
+    oracle.run_temco(a, x, on_step=lambda t, y: ref.setdefault(a.steps[t].out, y))
+    np.testing.assert_allclose(got[7], ref[7], rtol=1e-12)
+
+
+def test_merged_fconv_memory_rule_resnet50():
+    """ResNet-50 (b256 bf16): the restore of each stage's first-block input feeds conv1's and the
+    downsample's fconvs.  Stage 2's merge would define both reduces (16 and 32 channels at 56 x 56)
+    while the four 32-channel reduced inputs of that restore are live:
+    4 x 51,380,224 + 25,690,112 + 51,380,224 = 282,591,232 B > the unmerged peak 279,379,968 B, so
+    "nogrow" (memory first) keeps two groups there and merges stages 1, 3 and 4; "bound" (peak <= m,
+    the unfused peak, Overhead's memory test) merges all four."""
+    m = W.resnet50()
+    a = oracle.plan(m, cse=False, reorder=False)
+    b = oracle.plan(m, reorder=False)
+    c = oracle.plan(m, reorder=False, cse_policy="bound")
+    assert a.peak_fused == b.peak_fused == 279_379_968
+    assert [(s.out, s.extra) for s in b.steps if s.extra] == [(7, [21]), (127, [140]), (227, [240])]
+    assert [(s.out, s.extra) for s in c.steps if s.extra] == [(7, [21]), (59, [72]), (127, [140]), (227, [240])]
+    assert c.peak_fused == 4 * 51_380_224 + 25_690_112 + 51_380_224 == 282_591_232 <= c.peak_unfused
+    # no other pair of groups restores the same tensor in any config
+    for name in ("densenet121", "vgg16_cp", "unet", "alexnet"):
+        assert not any(s.extra for s in oracle.plan(W.build_config(name)).steps)
+
+
+def test_restore_key_separates_different_restores():
+    """Two groups with the same ops but different reduced inputs, or a copy with a different
+    attribute, are not merged (reading R37 compares structure AND inputs)."""
+    from oracle.rewrite import restore_key
+    from dataclasses import replace
+    p = oracle.plan(W.t3_mini_bottleneck(), cse=False)
+    g7 = next(s for s in p.steps if s.out == 7)
+    g21 = next(s for s in p.steps if s.out == 21)
+    t7, t21 = p.onodes[7].inputs[0], p.onodes[21].inputs[0]
+    k7 = restore_key(p.onodes, set(g7.members), t7)
+    assert k7 == restore_key(p.onodes, set(g21.members), t21)
+    on = dict(p.onodes)
+    pool = next(x for x in g21.members if on[x].op == "maxpool")
+    on[pool] = replace(on[pool], sh=1)
+    assert restore_key(on, set(g21.members), t21) != k7
+    on = dict(p.onodes)
+    lc = next(x for x in g21.members if on[x].role == "lconv")
+    on[lc] = replace(on[lc], inputs=[12])
+    assert restore_key(on, set(g21.members), t21) != k7
+
+
+# ----------------------------------------------------------------------------
+# reading R38: memory-optimal re-scheduling of S
+# ----------------------------------------------------------------------------
+
+class _Sizes:
+    """A stand-in graph for abstract step DAGs: tensor id -> bytes."""
+
+    def __init__(self, sizes):
+        self.nodes_by_id = {k: k for k in sizes}
+        self._s = sizes
+
+    def size(self, v):
+        return self._s[v]
+
+
+def _topo_orders(steps):
+    prod = {o: i for i, s in enumerate(steps) for o in s.outs}
+    deps = [{prod[x] for x in s.inputs} for s in steps]
+    n = len(steps)
+
+    def rec(done, order):
+        if len(order) == n:
+            yield list(order)
+            return
+        for v in range(n):
+            if v not in done and deps[v] <= done:
+                done.add(v)
+                order.append(v)
+                yield from rec(done, order)
+                order.pop()
+                done.remove(v)
+
+    yield from rec({0}, [0])
+
+
+def _random_dag(rng, n):
+    from oracle.rewrite import Step
+    steps = [Step(out=0, inputs=[], members=[0])]
+    sizes = {0: int(rng.integers(1, 50))}
+    nid = 1
+    for i in range(1, n):
+        k = int(rng.integers(1, min(3, i) + 1))
+        ins = sorted({int(x) for x in rng.choice([o for s in steps for o in s.outs], size=k)})
+        outs = [nid] + ([nid + 1] if rng.random() < 0.2 else [])
+        nid += len(outs)
+        for o in outs:
+            sizes[o] = int(rng.integers(1, 50))
+        steps.append(Step(out=outs[0], inputs=ins, members=[outs[0]], kind="group", extra=outs[1:]))
+    return steps, sizes
+
+
+def test_reschedule_is_the_brute_force_optimum():
+    """On random step DAGs (<= 8 steps, some with two outputs) the DP's order has the least O10
+    peak over EVERY topological order (brute-force enumeration, peaks by oracle.peak_bytes -- not
+    the DP's own live-set arithmetic), and it is the lexicographically first optimal order (S kept
+    wherever it is optimal)."""
+    from oracle.rewrite import reschedule
+    rng = np.random.default_rng(7)
+    for trial in range(150):
+        steps, sizes = _random_dag(rng, int(rng.integers(2, 9)))
+        g = _Sizes(sizes)
+        gout = steps[-1].out
+        res = reschedule(g, steps, 0, gout)
+        idx = [steps.index(s) for s in res]
+        peaks = {tuple(o): oracle.peak_bytes(g, [steps[i] for i in o], 0, gout)[0] for o in _topo_orders(steps)}
+        best = min(peaks.values())
+        assert tuple(idx) in peaks
+        assert peaks[tuple(idx)] == best
+        assert tuple(idx) == min(o for o, v in peaks.items() if v == best)
+
+
+def test_reschedule_by_hand():
+    """Input 0 (1 B) read by a (-> 1, 50 B) and b (-> 2, 50 B); c reads 1 (-> 3, 1 B), e reads 2
+    (-> 4, 1 B), f reads 3, 4 (-> 5, the output, 1 B).  S = [0, a, b, c, e, f] holds both 50 B
+    branches at once: live 1, 51, 1 + 50 + 50 = 101 at b, 50 + 50 + 1 = 101 at c, 52, 3.  Finishing
+    branch a first, [0, a, c, b, e, f]: 1, 51, 1 + 50 + 1 = 52 at c, 1 + 1 + 50 = 52 at b, 52, 3,
+    the optimum (b's 50 B output always meets two other tensors).  With a's output at 1 B instead,
+    S peaks at 52 = the optimum and is kept unchanged."""
+    from oracle.rewrite import Step, reschedule
+    st = [Step(0, [], [0]), Step(1, [0], [1]), Step(2, [0], [2]), Step(3, [1], [3]), Step(4, [2], [4]),
+          Step(5, [3, 4], [5])]
+    g = _Sizes({0: 1, 1: 50, 2: 50, 3: 1, 4: 1, 5: 1})
+    assert oracle.peak_bytes(g, st, 0, 5)[1] == [1, 51, 101, 101, 52, 3]
+    r = reschedule(g, st, 0, 5)
+    assert [s.out for s in r] == [0, 1, 3, 2, 4, 5]
+    assert oracle.peak_bytes(g, r, 0, 5)[1] == [1, 51, 52, 52, 52, 3]
+    g = _Sizes({0: 1, 1: 1, 2: 50, 3: 1, 4: 1, 5: 1})
+    assert oracle.peak_bytes(g, st, 0, 5)[1] == [1, 2, 52, 52, 52, 3]
+    assert [s.out for s in reschedule(g, st, 0, 5)] == [0, 1, 2, 3, 4, 5]
+
+
+def test_reschedule_configs_semantics_and_peaks():
+    """R38 never raises a peak; it lowers ResNet-50's (b256 bf16) from 279,379,968 B to
+    263,323,648 B and keeps every other config's S; the re-scheduled plans compute the same
+    tensors (small shapes, fp64)."""
+    for name in ("resnet50", "resnet18_cifar", "densenet121", "vgg16_cp", "unet", "alexnet", "resnet18_tt"):
+        m = W.build_config(name)
+        a, b = oracle.plan(m, reorder=False), oracle.plan(m)
+        assert b.peak_fused <= a.peak_fused
+        assert sorted(s.out for s in a.steps) == sorted(s.out for s in b.steps)
+        if name == "resnet50":
+            assert (a.peak_fused, b.peak_fused) == (279_379_968, 263_323_648)
+    m = W.resnet50(batch=1, dtype="f32", height=32, width=32)
+    p = oracle.plan(m)
+    x = W.make_input(m)
+    np.testing.assert_allclose(oracle.run_temco(p, x), oracle.run_unfused(p, x), rtol=1e-9, atol=1e-12)

@@ -54,7 +54,7 @@ def test_paper_schedule_mode(name):
     """TEMCO_FLAG_PAPER_SCHEDULE == the oracle without readings R34 / R35 (the paper's own
     schedule, whose peaks SURVEY P2 pins)."""
     m = W.build_config(name) if name in FULL else SMALL[name]()
-    _compare(m, FLAG_PAPER_SCHEDULE, cp_pair=False, fold_cores=False, pool_first=False)
+    _compare(m, FLAG_PAPER_SCHEDULE, cp_pair=False, fold_cores=False, pool_first=False, cse=False, reorder=False)
 
 
 @pytest.mark.parametrize("name", ["t2_3", "t3", "t4"])
