@@ -129,10 +129,17 @@ enum {
   TEMCO_FLAG_OVERHEAD_NEVER = 1 << 6,  /* force Overhead() false (tests)                 */
   TEMCO_FLAG_MMA_SMALL = 1 << 7,       /* run groups with C <= 256 on the mma.sync kernel */
   TEMCO_FLAG_PAPER_SCHEDULE = 1 << 9,  /* the paper's schedule exactly: without the round-2
-                                          extensions R34 (CP depthwise core pair as one step) and
-                                          R35 (a 1x1 core folded into the fconv feeding it)     */
-  TEMCO_FLAG_MMA_CAT = 1 << 8          /* single-level concat groups on the mma.sync concat
+                                          extensions R34 (CP depthwise core pair as one step),
+                                          R35 (a 1x1 core folded into the fconv feeding it), R36
+                                          (pool before the restore), R37 (merged fconvs) and R38
+                                          (memory-optimal re-scheduling of S)                  */
+  TEMCO_FLAG_MMA_CAT = 1 << 8,         /* single-level concat groups on the mma.sync concat
                                           kernel (kernels_cat.cu; measured slower than tcgen05) */
+  TEMCO_FLAG_NO_CSE = 1 << 10,         /* no merged-fconv CSE (reading R37)         */
+  TEMCO_FLAG_NO_RESCHEDULE = 1 << 11,  /* keep S's order (no reading R38 re-scheduling)        */
+  TEMCO_FLAG_CSE_BOUND = 1 << 12       /* R37 keeps a merge iff the fused peak stays <= the
+                                          unfused peak (Overhead's memory test) instead
+                                          of iff it does not grow                              */
 };
 
 typedef struct {
@@ -203,6 +210,13 @@ temco_status temco_run_profiled(temco_plan_t plan, const void* input, void* outp
  * temco_run. */
 temco_status temco_debug_step_output(temco_plan_t plan, const void* input, void* output, temco_stream_t stream,
                                      int32_t step, void* host_dst, int64_t capacity, int64_t* bytes);
+
+/* The same for output `which` of step `step`: 0 = the step's tensor above, 1 .. = the further
+ * reduce outputs of a merged group (reading R37; temco_plan_describe lists them as the
+ * step's "extra"), in that order.  which out of range -> TEMCO_ERR_INVALID_ARGUMENT. */
+temco_status temco_debug_step_tensor(temco_plan_t plan, const void* input, void* output, temco_stream_t stream,
+                                     int32_t step, int32_t which, void* host_dst, int64_t capacity,
+                                     int64_t* bytes);
 
 temco_status temco_plan_destroy(temco_plan_t plan);
 const char* temco_status_string(temco_status s);

@@ -98,9 +98,10 @@ def run_step(plan, t, env, which=None):
     return apply(v, [env[i] for i in v.inputs])
 
 
-def run_temco(plan, x, on_step=None):
+def run_temco(plan, x, on_step=None, on_tensor=None):
     """Run the TeMCO schedule S (fused groups + remaining ops).  on_step(t, tensor),
-    if given, sees every step's output as it is produced (per-step parity tests)."""
+    if given, sees every step's output as it is produced, on_tensor(id, tensor) every
+    tensor a step defines (a merged group defines several; per-step parity tests)."""
     g = plan.graph
     steps = plan.steps
     last = {}
@@ -118,6 +119,9 @@ def run_temco(plan, x, on_step=None):
             env[s.out] = apply(v, [env[i] for i in v.inputs])
         if on_step is not None:
             on_step(t, env[s.out])
+        if on_tensor is not None:
+            for o in s.outs:
+                on_tensor(o, env[o])
         for i in s.inputs:
             if last[i] == t and i != g.output:
                 del env[i]

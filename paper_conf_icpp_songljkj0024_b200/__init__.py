@@ -8,7 +8,8 @@ lazy import only lets `build` run before the library exists.
 """
 _BINDING = {"Plan", "TemcoError", "library_path", "exported_symbols", "EXPORTS", "F32", "BF16", "FLAG_NO_DEVICE",
             "FLAG_NO_SKIPOPT", "FLAG_NO_FUSION", "FLAG_CUDA_GRAPH", "FLAG_SIMT_ONLY", "FLAG_OVERHEAD_ALWAYS",
-            "FLAG_OVERHEAD_NEVER", "FLAG_MMA_SMALL", "FLAG_MMA_CAT", "FLAG_PAPER_SCHEDULE"}
+            "FLAG_OVERHEAD_NEVER", "FLAG_MMA_SMALL", "FLAG_MMA_CAT", "FLAG_PAPER_SCHEDULE", "FLAG_NO_CSE",
+            "FLAG_NO_RESCHEDULE", "FLAG_CSE_BOUND"}
 
 
 def __getattr__(name):

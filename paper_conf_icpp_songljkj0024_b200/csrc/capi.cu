@@ -38,7 +38,8 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM, K_DWPAIR };
+enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM, K_DWPAIR,
+                K_MULTI /* a merged group replayed once per output: the launches of sub_exec[sub] */ };
 
 struct StepExec {
   int kind = K_NONE;
@@ -59,6 +60,7 @@ struct StepExec {
   int64_t flops = 0, io_bytes = 0;
   int launches = 0;
   bool stem = false;   // K_CONV on the tensor-core small-Cin kernel (kernels_stem.cu)
+  std::vector<int> sub;   // K_MULTI: indices into temco_plan_s::sub_exec
 };
 
 }  // namespace
@@ -72,6 +74,7 @@ struct temco_plan_s {
   bool has_device = false;
 
   std::vector<StepExec> exec;
+  std::vector<StepExec> sub_exec;  // launches of merged groups replayed per output (K_MULTI)
   std::map<int, Loc> loc;
   std::vector<float> params_h;
   std::vector<GNode> gnodes_h;
@@ -223,8 +226,12 @@ int64_t plan_arena(temco_plan_s* P) {
   const int T = (int)ir.steps.size();
   std::map<int, int> def, last;
   for (int t = 0; t < T; ++t) {
-    def[ir.steps[t].out] = t;
-    if (!last.count(ir.steps[t].out)) last[ir.steps[t].out] = t;
+    std::vector<int> outs = {ir.steps[t].out};
+    outs.insert(outs.end(), ir.steps[t].extra.begin(), ir.steps[t].extra.end());
+    for (int o : outs) {
+      def[o] = t;
+      if (!last.count(o)) last[o] = t;
+    }
     for (int x : ir.steps[t].in) last[x] = t;
   }
   struct Item { int id; int64_t bytes; int a, b; int64_t off; };
@@ -270,6 +277,93 @@ int64_t tensor_bytes(const temco_plan_s* P, int id) {
   return el * (id == P->ir.output ? 4 : (P->bf16 ? 2 : 4));
 }
 
+// lowering of one fused-group step (one output) onto the fastest kernel that takes its shape
+void lower_group(temco_plan_s* P, const Step& s, StepExec& e) {
+  IR& ir = P->ir;
+  const int N = ir.batch;
+  const Node& v = ir.nodes[s.out];
+  // groups with a 3x3/s2 max-pooled 64-channel member (the stem restore copies):
+  // restore-once mma.sync kernel; single-input groups: the lean mma.sync kernels;
+  // opt-in (TEMCO_FLAG_MMA_CAT, measured slower than tcgen05): the generic mma.sync
+  // concat kernel; else tcgen05, else the interpreter
+  const bool mma_ok = P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY);
+  std::vector<uint16_t> scratch;
+  CatDesc cd;
+  const bool cat_form = mma_ok && mma_cat_lower(ir, s, P->loc, scratch, cd);
+  if (cat_form && mma_poolcat_ok(cd) && !getenv("TEMCO_NO_POOLCAT") &&
+      mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+    e.kind = K_GROUP_CAT;
+    e.kernel = "mma_poolcat";
+    e.launches = 1;
+    return;
+  }
+  if (mma_ok && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
+      mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma) &&
+      ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
+    e.kind = K_GROUP_MMA;
+    e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
+    e.launches = 1;
+    return;
+  }
+  if (cat_form && ((mma_catp_ok(cd) && !getenv("TEMCO_NO_CATP")) || (P->flags & TEMCO_FLAG_MMA_CAT)) &&
+      mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+    e.kind = K_GROUP_CAT;
+    e.kernel = mma_catp_ok(e.cat) ? "mma_catp" : "mma_cat";
+    e.launches = 1;
+    return;
+  }
+  // full-width residual chains with an fconv root: the CTA-pair tcgen05 kernel
+  if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+      pair::pair_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.pr)) {
+    e.kind = K_GROUP_PAIR;
+    e.kernel = "tc_pair";
+    e.launches = 1;
+    return;
+  }
+  if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+      tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tc)) {
+    e.kind = K_GROUP_TC;
+    e.kernel = "tc_chain";
+    e.launches = 1;
+    return;
+  }
+  // groups whose per-tile reduced inputs exceed shared memory: TMEM-resident levels
+  if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
+      wide::tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tcw)) {
+    e.kind = K_GROUP_TCW;
+    e.kernel = "tc_chain";
+    e.launches = 1;
+    return;
+  }
+  GroupLowering gl{P, std::set<int>(s.members.begin(), s.members.end()), {}};
+  GroupDesc& g = e.grp;
+  int tsrc;
+  if (v.role == ROLE_FCONV) {
+    g.root = ROOT_FCONV;
+    tsrc = ir.oin[s.out][0];
+    g.Nout = v.C;
+    if (v.C > 256) throw std::runtime_error("fused fconv with more than 256 outputs");
+    g.F = push_params(P, v.w);
+    g.Fb = push_params(P, v.b);
+    gl.members.erase(s.out);
+  } else if (v.op == OP_GAP) {
+    g.root = ROOT_GAP;
+    tsrc = ir.oin[s.out][0];
+    gl.members.erase(s.out);
+  } else {
+    g.root = ROOT_STORE;
+    tsrc = s.out;
+  }
+  const Node& tn = ir.nodes[tsrc];
+  g.tnode = gl.node(tsrc);
+  g.N = N; g.H = tn.H; g.W = tn.W; g.C = tn.C;
+  g.y = tensor_loc(P, s.out);
+  e.kind = K_GROUP_SIMT;
+  e.kernel = g.root == ROOT_GAP ? "simt_group_gap" : "simt_group";
+  e.launches = 1;
+  return;
+}
+
 void lower(temco_plan_s* P) {
   IR& ir = P->ir;
   const int N = ir.batch;
@@ -281,6 +375,7 @@ void lower(temco_plan_s* P) {
     for (int m : s.members) e.flops += node_flops(ir, m);
     for (int x : s.in) e.io_bytes += tensor_bytes(P, x);
     if (v.op != OP_INPUT) e.io_bytes += tensor_bytes(P, s.out);
+    for (int x : s.extra) e.io_bytes += tensor_bytes(P, x);
     if (s.group && s.members.size() == 2 && ir.nodes[s.members[0]].op == OP_CONV &&
         ir.nodes[s.members[0]].groups > 1) {
       // CP depthwise core pair (reading R34): one kernel, the K x 1 output stays in registers
@@ -304,38 +399,19 @@ void lower(temco_plan_s* P) {
       e.launches = 1;
       continue;
     }
-    if (s.group) {
-      // groups with a 3x3/s2 max-pooled 64-channel member (the stem restore copies):
-      // restore-once mma.sync kernel; single-input groups: the lean mma.sync kernels;
-      // opt-in (TEMCO_FLAG_MMA_CAT, measured slower than tcgen05): the generic mma.sync
-      // concat kernel; else tcgen05, else the interpreter
-      const bool mma_ok = P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY);
+    if (s.group && !s.extra.empty()) {
+      // merged group (reading R37): one CTA-pair launch computing every reduce output from one
+      // restore when its kernel takes the shape; else the group replayed once per output
       std::vector<uint16_t> scratch;
       CatDesc cd;
-      const bool cat_form = mma_ok && mma_cat_lower(ir, s, P->loc, scratch, cd);
-      if (cat_form && mma_poolcat_ok(cd) && !getenv("TEMCO_NO_POOLCAT") &&
-          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
+      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) && !getenv("TEMCO_NO_POOLCAT") &&
+          mma_cat_lower(ir, s, P->loc, scratch, cd) && mma_poolcat_ok(cd) &&
+          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {   // the restore-once pooled kernel, stacked F
         e.kind = K_GROUP_CAT;
         e.kernel = "mma_poolcat";
         e.launches = 1;
         continue;
       }
-      if (mma_ok && ir.nodes[ir.oin[s.out][0]].C <= 256 &&
-          mma_lower_chain(ir, s, P->loc, P->tcw_h, e.mma) &&
-          ((P->flags & TEMCO_FLAG_MMA_SMALL) || (mma_lean_ok(e.mma) && !getenv("TEMCO_NO_LEAN")))) {
-        e.kind = K_GROUP_MMA;
-        e.kernel = mma_lean_ok(e.mma) ? "mma_lean" : "mma_chain";
-        e.launches = 1;
-        continue;
-      }
-      if (cat_form && ((mma_catp_ok(cd) && !getenv("TEMCO_NO_CATP")) || (P->flags & TEMCO_FLAG_MMA_CAT)) &&
-          mma_cat_lower(ir, s, P->loc, P->tcw_h, e.cat)) {
-        e.kind = K_GROUP_CAT;
-        e.kernel = mma_catp_ok(e.cat) ? "mma_catp" : "mma_cat";
-        e.launches = 1;
-        continue;
-      }
-      // full-width residual chains with an fconv root: the CTA-pair tcgen05 kernel
       if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
           pair::pair_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.pr)) {
         e.kind = K_GROUP_PAIR;
@@ -343,47 +419,29 @@ void lower(temco_plan_s* P) {
         e.launches = 1;
         continue;
       }
-      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
-          tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tc)) {
-        e.kind = K_GROUP_TC;
-        e.kernel = "tc_chain";
-        e.launches = 1;
-        continue;
+      e.kind = K_MULTI;
+      e.launches = 0;
+      std::vector<int> outs = {s.out};
+      outs.insert(outs.end(), s.extra.begin(), s.extra.end());
+      for (int o : outs) {
+        Step sub;
+        sub.out = o;
+        sub.in = s.in;
+        sub.group = true;
+        for (int m : s.members)
+          if (m == o || std::find(outs.begin(), outs.end(), m) == outs.end()) sub.members.push_back(m);
+        StepExec se;
+        lower_group(P, sub, se);
+        if (e.kernel.empty() || e.kernel == se.kernel) e.kernel = se.kernel;
+        else e.kernel = "multi";
+        e.launches += se.launches;
+        e.sub.push_back((int)P->sub_exec.size());
+        P->sub_exec.push_back(std::move(se));
       }
-      // groups whose per-tile reduced inputs exceed shared memory: TMEM-resident levels
-      if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
-          wide::tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tcw)) {
-        e.kind = K_GROUP_TCW;
-        e.kernel = "tc_chain";
-        e.launches = 1;
-        continue;
-      }
-      GroupLowering gl{P, std::set<int>(s.members.begin(), s.members.end()), {}};
-      GroupDesc& g = e.grp;
-      int tsrc;
-      if (v.role == ROLE_FCONV) {
-        g.root = ROOT_FCONV;
-        tsrc = ir.oin[s.out][0];
-        g.Nout = v.C;
-        if (v.C > 256) throw std::runtime_error("fused fconv with more than 256 outputs");
-        g.F = push_params(P, v.w);
-        g.Fb = push_params(P, v.b);
-        gl.members.erase(s.out);
-      } else if (v.op == OP_GAP) {
-        g.root = ROOT_GAP;
-        tsrc = ir.oin[s.out][0];
-        gl.members.erase(s.out);
-      } else {
-        g.root = ROOT_STORE;
-        tsrc = s.out;
-      }
-      const Node& tn = ir.nodes[tsrc];
-      g.tnode = gl.node(tsrc);
-      g.N = N; g.H = tn.H; g.W = tn.W; g.C = tn.C;
-      g.y = tensor_loc(P, s.out);
-      e.kind = K_GROUP_SIMT;
-      e.kernel = g.root == ROOT_GAP ? "simt_group_gap" : "simt_group";
-      e.launches = 1;
+      continue;
+    }
+    if (s.group) {
+      lower_group(P, s, e);
       continue;
     }
     switch (v.op) {
@@ -640,7 +698,8 @@ std::string make_json(const temco_plan_s* P) {
     json_ints(o, s.members);
     o << ",\"inputs\":";
     json_ints(o, s.in);
-    o << ",\"bytes\":" << ir.size(s.out);
+    o << ",\"bytes\":" << ir.size(s.out) << ",\"extra\":";
+    json_ints(o, s.extra);
     // shapes [C, H, W] of the step's inputs and output (per image)
     o << ",\"in_chw\":[";
     for (size_t i = 0; i < s.in.size(); ++i) {
@@ -721,6 +780,40 @@ RunPtrs run_ptrs(temco_plan_s* P, const void* in, void* out) {
   return RunPtrs{P->arena_d, in, out, P->params_d};
 }
 
+void launch_exec(temco_plan_s* P, const StepExec& e, const RunPtrs& rp, cudaStream_t st) {
+  switch (e.kind) {
+    case K_NONE: break;
+    case K_CONVT: launch_conv_transpose(e.conv, rp, st); break;
+    case K_DWPAIR: launch_dwpair(e.dwp, rp, st); break;
+    case K_CONV:
+      if (e.stem)
+        launch_conv_stem(e.conv, rp, st);
+      else if (dwconv_vec_ok(e.conv))
+        launch_dwconv_vec(e.conv, rp, st);
+      else if (conv_rank_ok(e.conv))
+        launch_conv_rank(e.conv, rp, st);
+      else if (conv_small_ok(e.conv))
+        launch_conv_small(e.conv, rp, st);
+      else
+        launch_conv(e.conv, rp, st);
+      break;
+    case K_EW: launch_ew(e.ew, rp, st); break;
+    case K_LINEAR: launch_linear(e.lin, rp, st); break;
+    case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
+    case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
+    case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
+    case K_GROUP_PAIR: pair::launch_pair_chain(e.pr, rp, st); break;
+    case K_GEMM: launch_gemm(e.gm, rp, P->lin_ws_d, st); break;
+    case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
+    case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
+    case K_GROUP_CAT: launch_mma_cat(e.cat, P->tcw_d, rp, st); break;
+    case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
+    case K_MULTI:
+      for (int k : e.sub) launch_exec(P, P->sub_exec[k], rp, st);
+      break;
+  }
+}
+
 temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st, cudaEvent_t* ev,
                      int64_t last_step = -1) {
   RunPtrs rp = run_ptrs(P, in, out);
@@ -728,34 +821,7 @@ temco_status enqueue(temco_plan_s* P, const void* in, void* out, cudaStream_t st
   for (size_t t = 0; t < nsteps; ++t) {
     const StepExec& e = P->exec[t];
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t], st));
-    switch (e.kind) {
-      case K_NONE: break;
-      case K_CONVT: launch_conv_transpose(e.conv, rp, st); break;
-      case K_DWPAIR: launch_dwpair(e.dwp, rp, st); break;
-      case K_CONV:
-        if (e.stem)
-          launch_conv_stem(e.conv, rp, st);
-        else if (dwconv_vec_ok(e.conv))
-          launch_dwconv_vec(e.conv, rp, st);
-        else if (conv_rank_ok(e.conv))
-          launch_conv_rank(e.conv, rp, st);
-        else if (conv_small_ok(e.conv))
-          launch_conv_small(e.conv, rp, st);
-        else
-          launch_conv(e.conv, rp, st);
-        break;
-      case K_EW: launch_ew(e.ew, rp, st); break;
-      case K_LINEAR: launch_linear(e.lin, rp, st); break;
-      case K_GROUP_SIMT: launch_group_simt(e.grp, P->gnodes_d, P->gchild_d, rp, st); break;
-      case K_GROUP_TC: launch_tc_chain(e.tc, P->tcw_d, rp, st); break;
-      case K_GROUP_TCW: wide::launch_tc_chain(e.tcw, P->tcw_d, rp, st); break;
-      case K_GROUP_PAIR: pair::launch_pair_chain(e.pr, rp, st); break;
-      case K_GEMM: launch_gemm(e.gm, rp, P->lin_ws_d, st); break;
-      case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
-      case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
-      case K_GROUP_CAT: launch_mma_cat(e.cat, P->tcw_d, rp, st); break;
-      case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
-    }
+    launch_exec(P, e, rp, st);
     if (ev) CUDA_TRY(cudaEventRecord(ev[2 * t + 1], st));
   }
   cudaError_t err = cudaGetLastError();
@@ -810,6 +876,9 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
   opt.skip_opt = !(cfg->flags & TEMCO_FLAG_NO_SKIPOPT);
   opt.fusion = !(cfg->flags & TEMCO_FLAG_NO_FUSION);
   opt.extensions = !(cfg->flags & TEMCO_FLAG_PAPER_SCHEDULE);
+  opt.cse = !(cfg->flags & TEMCO_FLAG_NO_CSE);
+  opt.cse_policy = (cfg->flags & TEMCO_FLAG_CSE_BOUND) ? 1 : 0;
+  opt.reorder = !(cfg->flags & TEMCO_FLAG_NO_RESCHEDULE);
   opt.overhead_policy = (cfg->flags & TEMCO_FLAG_OVERHEAD_ALWAYS) ? 1 : (cfg->flags & TEMCO_FLAG_OVERHEAD_NEVER) ? 2 : 0;
   opt.bf16 = P->bf16;
   std::string err;
@@ -873,35 +942,38 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
       }
     }
     std::string terr;
-    for (auto& e : P->exec)
-      if (e.kind == K_CONV_TC && (!conv_tc_finalize(e.ctc, P->tcw_d, terr) ||
-                                   !conv_tc_finalize_x(e.ctc, P->arena_d + e.ctc.x.off, terr))) {
+    std::vector<StepExec*> ex;   // every launch: the steps' and the replayed merged groups'
+    for (auto& e : P->exec) ex.push_back(&e);
+    for (auto& e : P->sub_exec) ex.push_back(&e);
+    for (StepExec* e : ex)
+      if (e->kind == K_CONV_TC && (!conv_tc_finalize(e->ctc, P->tcw_d, terr) ||
+                                    !conv_tc_finalize_x(e->ctc, P->arena_d + e->ctc.x.off, terr))) {
         free_device(P);
         delete P;
         return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
       }
-    if (!tc_finalize(P->exec.size(), [&](size_t i) -> TcChainDesc* {
-          return P->exec[i].kind == K_GROUP_TC ? &P->exec[i].tc : nullptr;
+    if (!tc_finalize(ex.size(), [&](size_t i) -> TcChainDesc* {
+          return ex[i]->kind == K_GROUP_TC ? &ex[i]->tc : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {
       free_device(P);
       delete P;
       return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
     }
-    if (!wide::tc_finalize(P->exec.size(), [&](size_t i) -> wide::TcChainDesc* {
-          return P->exec[i].kind == K_GROUP_TCW ? &P->exec[i].tcw : nullptr;
+    if (!wide::tc_finalize(ex.size(), [&](size_t i) -> wide::TcChainDesc* {
+          return ex[i]->kind == K_GROUP_TCW ? &ex[i]->tcw : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {
       free_device(P);
       delete P;
       return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
     }
-    for (auto& e : P->exec)
-      if (e.kind == K_GEMM && !gemm_finalize(e.gm, P->arena_d, P->tcw_d, terr)) {
+    for (StepExec* e : ex)
+      if (e->kind == K_GEMM && !gemm_finalize(e->gm, P->arena_d, P->tcw_d, terr)) {
         free_device(P);
         delete P;
         return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
       }
-    if (!pair::pair_finalize(P->exec.size(), [&](size_t i) -> pair::PairDesc* {
-          return P->exec[i].kind == K_GROUP_PAIR ? &P->exec[i].pr : nullptr;
+    if (!pair::pair_finalize(ex.size(), [&](size_t i) -> pair::PairDesc* {
+          return ex[i]->kind == K_GROUP_PAIR ? &ex[i]->pr : nullptr;
         }, P->arena_d, P->tcw_d, terr)) {
       free_device(P);
       delete P;
@@ -1035,13 +1107,14 @@ temco_status temco_run_profiled(temco_plan_t P, const void* input, void* output,
   return st;
 }
 
-temco_status temco_debug_step_output(temco_plan_t P, const void* input, void* output, temco_stream_t stream,
-                                     int32_t step, void* host_dst, int64_t capacity, int64_t* bytes) {
+temco_status temco_debug_step_tensor(temco_plan_t P, const void* input, void* output, temco_stream_t stream,
+                                     int32_t step, int32_t which, void* host_dst, int64_t capacity, int64_t* bytes) {
   temco_status st = check_device(P);
   if (st != TEMCO_OK) return st;
-  if (!input || !output || !bytes || step < 0 || step >= (int32_t)P->exec.size())
+  if (!input || !output || !bytes || step < 0 || step >= (int32_t)P->exec.size() || which < 0 ||
+      which > (int32_t)P->ir.steps[step].extra.size())
     return set_err(TEMCO_ERR_INVALID_ARGUMENT, "bad step-output arguments");
-  const int id = P->ir.steps[step].out;
+  const int id = which == 0 ? P->ir.steps[step].out : P->ir.steps[step].extra[which - 1];
   const Loc l = P->loc.count(id) ? P->loc.at(id) : Loc{W_INPUT, 0, 0};
   const int64_t need = tensor_bytes(P, id);
   *bytes = need;
@@ -1054,6 +1127,11 @@ temco_status temco_debug_step_output(temco_plan_t P, const void* input, void* ou
   CUDA_TRY(cudaMemcpyAsync(host_dst, src, need, cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaStreamSynchronize(s));
   return TEMCO_OK;
+}
+
+temco_status temco_debug_step_output(temco_plan_t P, const void* input, void* output, temco_stream_t stream,
+                                     int32_t step, void* host_dst, int64_t capacity, int64_t* bytes) {
+  return temco_debug_step_tensor(P, input, output, stream, step, 0, host_dst, capacity, bytes);
 }
 
 temco_status temco_peak_internal_bytes(temco_plan_t P, int32_t which, int64_t* bytes) {

@@ -133,7 +133,10 @@ struct CatDesc {
   int32_t lbias, mbias;       // fp32 offsets (floats) after the bf16 part
   int32_t blob_bf16, blob_bytes;
   int64_t blob;               // tc weight pool offset
-  Loc y;
+  Loc y;                      // = ys[0]
+  int32_t n_out;              // reduce outputs (a merged group, reading R37: its fconvs; mma_poolcat only)
+  Loc ys[4];                  // output k: columns [ycol[k], ycol[k + 1]) of the stacked F
+  int32_t ycol[5];
   int64_t alg_flops, alg_bytes;
 };
 

@@ -43,15 +43,23 @@ uint16_t f2bf(float f) {
 
 bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                    CatDesc& d) {
-  const Node& root = ir.nodes[s.out];
-  if (root.role != ROLE_FCONV || root.b) return false;
+  // roots: the fconv, or the fconvs of a merged group (reading R37) reading the same t
+  std::vector<int> roots = {s.out};
+  roots.insert(roots.end(), s.extra.begin(), s.extra.end());
+  if (roots.size() > 4) return false;
   const int tsrc = ir.oin[s.out][0];
+  int Nout = 0;
+  for (int r : roots) {
+    const Node& rn = ir.nodes[r];
+    if (rn.role != ROLE_FCONV || rn.b || ir.oin[r].size() != 1 || ir.oin[r][0] != tsrc || rn.C % 8) return false;
+    Nout += rn.C;
+  }
   const Node& tn = ir.nodes[tsrc];
-  const int C = tn.C, Nout = root.C;
+  const int C = tn.C;
   if (Nout % 8 || Nout > 64 || C % 8 || C > 64 * kCatMaxChunks) return false;
   const int Cpad = (C + 63) / 64 * 64;   // a short last chunk: zero weights / bias / F columns
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
-  P.members.erase(s.out);
+  for (int r : roots) P.members.erase(r);
   std::vector<PLevel> levels;
   if (!P.chain(tsrc, levels)) return false;
   if (P.visited != P.members || levels.size() != 1) return false;
@@ -71,9 +79,15 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
   if ((int64_t)ir.batch * tn.H * tn.W >= (1LL << 31) - 16) return false;
   d.nblocks = (d.npix + 15) / 16;
   d.relu = L.relu ? 1 : 0;
-  const Loc& yl = loc.at(s.out);
-  if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
-  d.y = yl;
+  d.n_out = (int)roots.size();
+  d.ycol[0] = 0;
+  for (int k = 0; k < d.n_out; ++k) {
+    const Loc& yl = loc.at(roots[k]);
+    if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
+    d.ys[k] = yl;
+    d.ycol[k + 1] = d.ycol[k] + ir.nodes[roots[k]].C;
+  }
+  d.y = d.ys[0];
 
   std::vector<uint16_t> blob;
   std::vector<float> fbias;
@@ -127,8 +141,11 @@ bool mma_cat_lower(const IR& ir, const Step& s, const std::map<int, Loc>& loc, s
   d.f = (int32_t)blob.size();
   d.fs = Cpad + 8;
   blob.resize(blob.size() + (size_t)Nout * d.fs, 0);
-  for (int o = 0; o < Nout; ++o)
-    for (int c = 0; c < C; ++c) blob[d.f + (size_t)o * d.fs + c] = f2bf((*root.w)[(size_t)o * C + c]);
+  for (int k = 0; k < d.n_out; ++k) {   // the roots' F stacked row-wise
+    const Node& rn = ir.nodes[roots[k]];
+    for (int o = 0; o < rn.C; ++o)
+      for (int c = 0; c < C; ++c) blob[d.f + (size_t)(d.ycol[k] + o) * d.fs + c] = f2bf((*rn.w)[(size_t)o * C + c]);
+  }
   while (blob.size() % 8) blob.push_back(0);
   d.blob_bf16 = (int32_t)blob.size();
   // fp32: level bias [C] (pooled channels: the post-pool shift), member bias [C] (0 elsewhere)
@@ -522,7 +539,6 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
   const __nv_bfloat16* blob = reinterpret_cast<const __nv_bfloat16*>(smem);
   const float* fb = reinterpret_cast<const float*>(smem + (size_t)d.blob_bf16 * 2);
   uint32_t* fp = reinterpret_cast<uint32_t*>(smem + (d.blob_bytes + 15) / 16 * 16);   // footprint [PR*PC][kPcStride]
-  __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(p.arena + d.y.off);
   const int lq = lane >> 3, lr = lane & 7;
   const uint32_t sbase = s_u32(blob);
   const CatTerm& M = d.term[d.n_plain];                 // the pooled member's (single) term
@@ -702,7 +718,11 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
 #pragma unroll
         for (int nb = 0; nb < NO; ++nb) {
           if (nb >= d.NO) break;
-          *reinterpret_cast<uint32_t*>(y + m * d.Nout + nb * 8 + 2 * t4) = pk2(O[nb][2 * h], O[nb][2 * h + 1]);
+          int k = 0;   // output holding n-tile nb (a merged group's fconvs, reading R37)
+          while (k + 1 < d.n_out && nb * 8 >= d.ycol[k + 1]) ++k;
+          __nv_bfloat16* yk = reinterpret_cast<__nv_bfloat16*>(p.arena + d.ys[k].off);
+          *reinterpret_cast<uint32_t*>(yk + m * (d.ycol[k + 1] - d.ycol[k]) + (nb * 8 - d.ycol[k]) + 2 * t4) =
+              pk2(O[nb][2 * h], O[nb][2 * h + 1]);
         }
       }
     }
@@ -908,7 +928,7 @@ void launch_cat_no(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cuda
 bool mma_catp_ok(const CatDesc& d) {
   // measured (B200): wins only where the tcgen05 kernel's 128-pixel tiles leave most SMs idle
   // (ResNet-18c stages 3-4: 16-64 tiles); 1.5-2x slower than tcgen05 on DenseNet's blocks 2-4
-  if (d.pool != 0 || d.nchunks > 8 || d.npix >= 74 * 128) return false;
+  if (d.pool != 0 || d.nchunks > 8 || d.npix >= 74 * 128 || d.n_out > 1) return false;
   for (int j = 0; j < d.n_terms; ++j)
     if (d.term[j].ks > 4) return false;
   return (d.blob_bytes + 15) / 16 * 16 + kCpWarps * 16 * d.Nout * 4 <= 227 * 1024;
@@ -916,7 +936,7 @@ bool mma_catp_ok(const CatDesc& d) {
 
 bool mma_poolcat_ok(const CatDesc& d) {
   const bool win = (d.pk == 3 && d.ps == 2 && d.pp == 1) || (d.pk == 2 && d.ps == 2 && d.pp == 0);
-  if (d.pool != 1 || !win || d.pc0 != 0 || d.pc1 != 1 || d.NO > 4) return false;
+  if (d.pool != 1 || !win || d.pc0 != 0 || d.pc1 != 1 || d.NO > 6) return false;
   if (d.n_terms != d.n_plain + 1 || d.term[d.n_plain].R > 16) return false;
   for (int j = 0; j < d.n_plain; ++j)
     if (d.term[j].tk != 1 || d.term[j].R > 16) return false;
@@ -938,11 +958,13 @@ void launch_mma_cat(const CatDesc& d, const uint16_t* tcw, const RunPtrs& p, cud
     if (d.pk == 2) {   // VGG's 2x2 / stride-2 pools
       if (d.NO == 1) return launch_poolcat_t<1, 2, 2, 0>(d, tcw, p, s);
       if (d.NO == 2) return launch_poolcat_t<2, 2, 2, 0>(d, tcw, p, s);
-      return launch_poolcat_t<4, 2, 2, 0>(d, tcw, p, s);
+      if (d.NO <= 4) return launch_poolcat_t<4, 2, 2, 0>(d, tcw, p, s);
+      return launch_poolcat_t<6, 2, 2, 0>(d, tcw, p, s);
     }
     if (d.NO == 1) return launch_poolcat_t<1, 3, 2, 1>(d, tcw, p, s);
     if (d.NO == 2) return launch_poolcat_t<2, 3, 2, 1>(d, tcw, p, s);
-    return launch_poolcat_t<4, 3, 2, 1>(d, tcw, p, s);   // 3 or 4 n-tiles (bounded by d.NO inside)
+    if (d.NO <= 4) return launch_poolcat_t<4, 3, 2, 1>(d, tcw, p, s);   // 3 or 4 n-tiles (bounded by d.NO inside)
+    return launch_poolcat_t<6, 3, 2, 1>(d, tcw, p, s);   // a merged group's stacked F (R37): 5 or 6 n-tiles
   }
   int ksm = 1;
   for (int j = 0; j < d.n_terms; ++j) ksm = std::max(ksm, d.term[j].ks);

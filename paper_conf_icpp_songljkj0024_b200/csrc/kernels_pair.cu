@@ -69,16 +69,25 @@ constexpr int kChunk = 2;                // ring stages of one level consumed pe
 bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, std::vector<uint16_t>& tcw,
                       std::vector<float>& params, PairDesc& d) {
   if (getenv("TEMCO_NO_PAIR")) return false;
-  const Node& root = ir.nodes[s.out];
-  if (root.role != ROLE_FCONV || root.b) return false;   // fconv factors carry no bias (O1)
+  // roots: the fconv, or every fconv of a merged group (reading R37), all reading the same t
+  std::vector<int> roots = {s.out};
+  roots.insert(roots.end(), s.extra.begin(), s.extra.end());
+  if ((int)roots.size() > kPairMaxOuts) return false;
   const int tsrc = ir.oin[s.out][0];
+  int Nout = 0;
+  for (int r : roots) {
+    const Node& rn = ir.nodes[r];
+    if (rn.role != ROLE_FCONV || rn.b || ir.oin[r].size() != 1 || ir.oin[r][0] != tsrc) return false;   // no bias (O1)
+    if (rn.C % 8) return false;
+    Nout += rn.C;
+  }
   const Node& tn = ir.nodes[tsrc];
-  const int C = tn.C, Nout = root.C;
+  const int C = tn.C;
   if (Nout % 8 || (Nout + 15) / 16 * 16 > 256) return false;
   ChainParser P{ir, std::set<int>(s.members.begin(), s.members.end()), C, {}, tn.H, tn.W};
   P.allow_silu = true;
   P.allow_member_act = true;
-  P.members.erase(s.out);
+  for (int r : roots) P.members.erase(r);
   std::vector<PLevel> levels;
   if (!P.chain(tsrc, levels)) return false;
   if (P.visited != P.members) return false;
@@ -95,8 +104,10 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     }
   }
   if ((int)levels.size() > kPairMaxLevels || nterms > kPairMaxTerms || nterms == 0) return false;
-  const Loc& yl = loc.at(s.out);
-  if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
+  for (int r : roots) {
+    const Loc& yl = loc.at(r);
+    if (yl.where != W_ARENA || yl.dtype != DT_BF16) return false;
+  }
 
   d = PairDesc();
   d.C = C;
@@ -108,7 +119,12 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   if (d.nbuf < 2) return false;
   d.npix = (int64_t)ir.batch * tn.H * tn.W;
   d.ntiles = (int)((d.npix + 255) / 256);
-  d.y = yl;
+  d.n_out = (int)roots.size();
+  d.ycol[0] = 0;
+  for (int k = 0; k < d.n_out; ++k) {
+    d.ys[k] = loc.at(roots[k]);
+    d.ycol[k + 1] = d.ycol[k] + ir.nodes[roots[k]].C;
+  }
   d.n_levels = (int)levels.size();
   int64_t flops = 0, bytes = 0;
   while (params.size() % 4) params.push_back(0.f);
@@ -189,9 +205,12 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     }
     d.n_prog = n;
   }
-  std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);
-  for (int o = 0; o < Nout; ++o)
-    for (int c = 0; c < C; ++c) f[(size_t)o * d.Cpad + c] = (*root.w)[(size_t)o * C + c];
+  std::vector<float> f((size_t)d.Np * d.Cpad, 0.f);   // the roots' F stacked row-wise
+  for (int k = 0; k < d.n_out; ++k) {
+    const Node& rn = ir.nodes[roots[k]];
+    for (int o = 0; o < rn.C; ++o)
+      for (int c = 0; c < C; ++c) f[(size_t)(d.ycol[k] + o) * d.Cpad + c] = (*rn.w)[(size_t)o * C + c];
+  }
   d.F = push_bf16(tcw, f);
   d.alg_flops = flops + d.npix * 2LL * Nout * C;
   d.alg_bytes = bytes + d.npix * 2LL * Nout;
@@ -751,7 +770,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     const uint32_t pfull_c = mapa_shared(smem_u32(p_full), 0);
     const uint32_t oempty_c = mapa_shared(smem_u32(out_empty), 0);
-    __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
+    __nv_bfloat16* yk[kPairMaxOuts];
+    for (int k = 0; k < kPairMaxOuts; ++k)
+      yk[k] = k < d.n_out ? reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.ys[k], p))) : nullptr;
     int gi = 0, np = 0, it = 0;   // gi: (unit, level) accumulator items consumed
     EVDECL();
     const bool ev0 = warp == kEpiWarp0 && lane == 0;
@@ -773,7 +794,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           pk.y = pack_bf16(__uint_as_float(v[2]), __uint_as_float(v[3]));
           pk.z = pack_bf16(__uint_as_float(v[4]), __uint_as_float(v[5]));
           pk.w = pack_bf16(__uint_as_float(v[6]), __uint_as_float(v[7]));
-          *reinterpret_cast<uint4*>(y + orow * d.Nout + c8 * 8) = pk;
+          int k = 0;   // output holding column c8 * 8 (a merged group's fconvs, reading R37)
+          while (k + 1 < d.n_out && c8 * 8 >= d.ycol[k + 1]) ++k;
+          *reinterpret_cast<uint4*>(yk[k] + orow * (d.ycol[k + 1] - d.ycol[k]) + (c8 * 8 - d.ycol[k])) = pk;
         }
       }
       tc_fence_before();

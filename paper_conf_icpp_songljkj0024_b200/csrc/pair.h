@@ -37,6 +37,7 @@ constexpr int kPairMaxLevels = 16;
 constexpr int kPairMaxAtoms = 256;      // K atoms of all unit pairs' programs
 constexpr int kPairMaxActGroups = 256;  // (level, 32-channel group) activation codes
 constexpr int kPairWu = 128;           // restored channels per unit (MMA N of the restore GEMM)
+constexpr int kPairMaxOuts = 4;        // reduce outputs of a merged group (reading R37)
 
 struct PairTerm {
   alignas(64) unsigned char amap[128];   // r_j [npix x R] bf16, box {aw, 128}
@@ -67,7 +68,9 @@ struct PairDesc {
   int32_t Nout, Np;                      // fconv outputs, padded to 16
   int64_t npix;                          // pixels (rows of r_j and y)
   int32_t ntiles;                        // 256-pixel pair tiles
-  Loc y;                                 // output [npix x Nout] bf16 (arena)
+  int32_t n_out;                         // reduce outputs (1; a merged group, reading R37: its fconvs)
+  Loc ys[kPairMaxOuts];                  // output k: [npix x (ycol[k+1] - ycol[k])] bf16 (arena) = out
+  int32_t ycol[kPairMaxOuts + 1];        //   columns [ycol[k], ycol[k+1]) of the concatenated F
   int64_t F;                             // tc weight pool offset of F
   int32_t stages, slot, smem_bytes, bias_bytes;   // ring depth, stage bytes
   // resident-weight mode (every Lhat / bias / F atom of this CTA's halves fits in SMEM next

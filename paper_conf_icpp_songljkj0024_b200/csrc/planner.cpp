@@ -373,8 +373,12 @@ int64_t peak_of(const IR& ir, const std::vector<Step>& steps, std::vector<int64_
   const int T = (int)steps.size();
   std::map<int, int> def, last;
   for (int t = 0; t < T; ++t) {
-    def[steps[t].out] = t;
-    if (!last.count(steps[t].out)) last[steps[t].out] = t;
+    std::vector<int> outs = {steps[t].out};
+    outs.insert(outs.end(), steps[t].extra.begin(), steps[t].extra.end());
+    for (int o : outs) {
+      def[o] = t;
+      if (!last.count(o)) last[o] = t;
+    }
     for (int x : steps[t].in) last[x] = t;
   }
   last[ir.output] = T - 1;
@@ -764,6 +768,188 @@ void group_and_schedule(IR& ir, bool fusion, bool extensions) {
   }
 }
 
+// reading R37 (oracle: restore_key / merge_fconvs): merged-fconv CSE.  A member's identity is the
+// node of L it was COPY'd from (Alg. 1 line 23; the root of a copy chain) with its attributes and
+// the identities of its inputs; a tensor from outside the group is identified by its id.
+int copy_root(const IR& ir, int x) {
+  const int c = ir.nodes[x].copy_of;
+  if (c < 0) return x;
+  int b = c;
+  while (ir.nodes[b].copy_of >= 0) b = ir.nodes[b].copy_of;
+  return b;
+}
+
+void restore_key(const IR& ir, const std::set<int>& mem, int x, std::vector<int64_t>& k) {
+  if (!mem.count(x)) {
+    k.push_back(-1);
+    k.push_back(x);
+    return;
+  }
+  const Node& v = ir.nodes[x];
+  const int64_t a[] = {-2, copy_root(ir, x), v.op, v.role, v.kh, v.kw, v.sh, v.sw, v.ph, v.pw, v.groups, v.C, v.H,
+                       v.W, (int64_t)ir.oin[x].size()};
+  k.insert(k.end(), a, a + sizeof(a) / sizeof(a[0]));
+  for (int i : ir.oin[x]) restore_key(ir, mem, i, k);
+  k.push_back(-3);
+}
+
+// taking the fused groups in S order, a later group whose fconv root reads a tensor with the same
+// key as an earlier group's root runs its reduce in the earlier group's step (its other members
+// leave O); kept iff the fused peak does not grow (policy 1: iff it stays <= the unfused peak m)
+void merge_fconvs(IR& ir, int policy) {
+  std::vector<int64_t> scratch;
+  int64_t cur = peak_of(ir, ir.steps, scratch);
+  auto fconv_group = [&](const Step& s) { return s.group && ir.nodes[s.out].role == ROLE_FCONV; };
+  auto key_of = [&](const Step& s) {
+    std::vector<int64_t> k;
+    restore_key(ir, std::set<int>(s.members.begin(), s.members.end()), ir.oin[s.out][0], k);
+    return k;
+  };
+  for (size_t i = 0; i < ir.steps.size(); ++i) {
+    if (!fconv_group(ir.steps[i])) continue;
+    const int ta = ir.oin[ir.steps[i].out][0];
+    const std::vector<int64_t> ka = key_of(ir.steps[i]);
+    size_t j = i + 1;
+    while (j < ir.steps.size()) {
+      const Step b = ir.steps[j];
+      if (!fconv_group(b) || key_of(b) != ka) {
+        ++j;
+        continue;
+      }
+      Step merged = ir.steps[i];
+      merged.members.push_back(b.out);
+      merged.extra.push_back(b.out);
+      std::vector<Step> trial = ir.steps;
+      trial[i] = merged;
+      trial.erase(trial.begin() + (long)j);
+      const int64_t np = peak_of(ir, trial, scratch);
+      if (np > (policy == 1 ? ir.peak_unfused : cur)) {
+        ++j;
+        continue;
+      }
+      cur = np;
+      ir.steps.swap(trial);
+      ir.oin[b.out] = {ta};   // b's reduce reads a's restored tensor
+      std::set<int> dropped(b.members.begin(), b.members.end());
+      std::vector<int> O;
+      for (int x : ir.O)
+        if (!dropped.count(x)) O.push_back(x);
+      auto at = std::find(O.begin(), O.end(), merged.out);
+      O.insert(at + (long)merged.extra.size(), b.out);   // right after a's outputs
+      ir.O.swap(O);
+      ir.groups[merged.out] = merged.members;
+      ir.groups.erase(b.out);
+    }
+  }
+}
+
+// reading R38 (oracle: reschedule): the order of S with the least peak (O10), exactly, by dynamic
+// programming over the sets of executed steps; among the optimal orders the lexicographically first
+// (at every point the earliest step of S whose choice keeps the optimum reachable).  More than
+// kMaxStates reachable sets: S is kept.
+constexpr size_t kRescheduleMaxStates = 100000;
+
+struct Rescheduler {
+  const IR& ir;
+  int n = 0, words = 0;
+  std::vector<std::vector<int>> outs, deps;          // per step
+  std::map<int, std::vector<int>> readers;           // tensor -> reading steps
+  std::vector<int64_t> osz;
+  std::map<std::vector<uint64_t>, int64_t> memo;
+  struct TooMany {};
+
+  static bool has(const std::vector<uint64_t>& X, int v) { return (X[v >> 6] >> (v & 63)) & 1u; }
+  static std::vector<uint64_t> with(std::vector<uint64_t> X, int v) {
+    X[v >> 6] |= 1ull << (v & 63);
+    return X;
+  }
+  int count(const std::vector<uint64_t>& X) const {
+    int c = 0;
+    for (uint64_t w : X) c += __builtin_popcountll(w);
+    return c;
+  }
+  bool ready(const std::vector<uint64_t>& X, int v) const {
+    if (has(X, v)) return false;
+    for (int d : deps[v])
+      if (!has(X, d)) return false;
+    return true;
+  }
+  int64_t live(const std::vector<uint64_t>& X) const {
+    int64_t tot = 0;
+    for (int i = 0; i < n; ++i) {
+      if (!has(X, i)) continue;
+      for (int o : outs[i]) {
+        bool keep = o == ir.output;
+        auto it = readers.find(o);
+        if (!keep && it != readers.end())
+          for (int r : it->second)
+            if (!has(X, r)) keep = true;
+        if (keep) tot += ir.size(o);
+      }
+    }
+    return tot;
+  }
+  int64_t best(const std::vector<uint64_t>& X) {
+    if (count(X) == n) return 0;
+    auto it = memo.find(X);
+    if (it != memo.end()) return it->second;
+    if (memo.size() >= kRescheduleMaxStates) throw TooMany{};
+    const int64_t L = live(X);
+    int64_t b = -1;
+    for (int v = 0; v < n; ++v) {
+      if (!ready(X, v)) continue;
+      const int64_t r = std::max(L + osz[v], best(with(X, v)));
+      if (b < 0 || r < b) b = r;
+    }
+    memo[X] = b;
+    return b;
+  }
+};
+
+void reschedule(IR& ir) {
+  Rescheduler R{ir};
+  const auto& S = ir.steps;
+  R.n = (int)S.size();
+  R.words = (R.n + 63) / 64;
+  std::map<int, int> prod;
+  R.outs.resize(R.n);
+  R.deps.resize(R.n);
+  R.osz.assign(R.n, 0);
+  for (int i = 0; i < R.n; ++i) {
+    R.outs[i] = {S[i].out};
+    R.outs[i].insert(R.outs[i].end(), S[i].extra.begin(), S[i].extra.end());
+    for (int o : R.outs[i]) {
+      prod[o] = i;
+      R.osz[i] += ir.size(o);
+    }
+  }
+  for (int i = 0; i < R.n; ++i)
+    for (int x : S[i].in) {
+      R.deps[i].push_back(prod.at(x));
+      auto& rd = R.readers[x];
+      if (std::find(rd.begin(), rd.end(), i) == rd.end()) rd.push_back(i);
+    }
+  std::vector<uint64_t> X(R.words, 0);
+  X = Rescheduler::with(X, 0);
+  int64_t opt;
+  try {
+    opt = std::max(R.osz[0], R.best(X));
+  } catch (const Rescheduler::TooMany&) {
+    return;
+  }
+  std::vector<Step> order = {S[0]};
+  for (int k = 1; k < R.n; ++k) {
+    const int64_t L = R.live(X);
+    int pick = -1;
+    for (int v = 0; v < R.n && pick < 0; ++v)
+      if (R.ready(X, v) && std::max(L + R.osz[v], R.best(Rescheduler::with(X, v))) <= opt) pick = v;
+    if (pick < 0) throw std::runtime_error("reschedule: no step keeps the optimum");
+    order.push_back(S[pick]);
+    X = Rescheduler::with(X, pick);
+  }
+  ir.steps.swap(order);
+}
+
 }  // namespace
 
 temco_status build_ir(const temco_layer* layers, int n_layers, const temco_decomp* decomps, int n_decomps,
@@ -797,6 +983,8 @@ temco_status build_ir(const temco_layer* layers, int n_layers, const temco_decom
       pool_before_restore(ir);
     }
     group_and_schedule(ir, opt.fusion, opt.extensions);
+    if (opt.fusion && opt.extensions && opt.cse) merge_fconvs(ir, opt.cse_policy);
+    if (opt.fusion && opt.extensions && opt.reorder) reschedule(ir);
     ir.peak_fused = peak_of(ir, ir.steps, ir.live_fused);
     return TEMCO_OK;
   } catch (const Fail& f) {

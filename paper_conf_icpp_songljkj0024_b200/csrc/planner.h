@@ -42,6 +42,7 @@ struct Step {
   std::vector<int> in;           // tensors read from outside the step
   std::vector<int> members;      // executed nodes in O order (1 for a plain op)
   bool group = false;
+  std::vector<int> extra;        // further reduce outputs of a merged group (reading R37)
 };
 
 struct SkipDecision {
@@ -75,7 +76,11 @@ struct BuildOptions {
   int distance_threshold = 1;
   bool skip_opt = true;
   bool fusion = true;
-  bool extensions = true;        // readings R34 (CP core pair) and R35 (1x1 core folded into its fconv)
+  bool extensions = true;        // readings R34 (CP core pair), R35 (1x1 core folded into its fconv),
+                                 // R36 (pool before the restore), R37 (merged fconvs), R38 (re-scheduling)
+  bool cse = true;               // reading R37 (with extensions)
+  int cse_policy = 0;            // 0: keep a merge iff the fused peak does not grow; 1: iff <= unfused peak
+  bool reorder = true;           // reading R38 (with extensions)
   int overhead_policy = 0;       // 0 paper, 1 always, 2 never
   bool bf16 = false;
 };

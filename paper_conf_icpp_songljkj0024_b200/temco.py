@@ -30,10 +30,14 @@ FLAG_OVERHEAD_ALWAYS = 1 << 5
 FLAG_OVERHEAD_NEVER = 1 << 6
 FLAG_MMA_SMALL = 1 << 7
 FLAG_MMA_CAT = 1 << 8
-FLAG_PAPER_SCHEDULE = 1 << 9   # without the round-2 schedule extensions R34 / R35
+FLAG_PAPER_SCHEDULE = 1 << 9   # without the round-2 schedule extensions R34-R38
+FLAG_NO_CSE = 1 << 10          # no merged-fconv CSE (R37)
+FLAG_NO_RESCHEDULE = 1 << 11   # keep S's order (no R38)
+FLAG_CSE_BOUND = 1 << 12       # R37 keeps merges with peak <= the unfused peak
 
 EXPORTS = ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_peak_internal_bytes", "temco_output_shape",
-           "temco_plan_describe", "temco_run_profiled", "temco_debug_step_output", "temco_plan_destroy",
+           "temco_plan_describe", "temco_run_profiled", "temco_debug_step_output", "temco_debug_step_tensor",
+           "temco_plan_destroy",
            "temco_status_string", "temco_last_error"]
 
 _fp = C.POINTER(C.c_float)
@@ -69,6 +73,8 @@ _lib.temco_run_profiled.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void
 _lib.temco_peak_internal_bytes.argtypes = [C.c_void_p, C.c_int32, C.POINTER(C.c_int64)]
 _lib.temco_debug_step_output.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_void_p,
                                          C.c_int64, C.POINTER(C.c_int64)]
+_lib.temco_debug_step_tensor.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_int32, C.c_int32,
+                                         C.c_void_p, C.c_int64, C.POINTER(C.c_int64)]
 _lib.temco_output_shape.argtypes = [C.c_void_p, C.POINTER(C.c_int64), C.POINTER(C.c_int32)]
 _lib.temco_plan_describe.argtypes = [C.c_void_p, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]
 _lib.temco_plan_destroy.argtypes = [C.c_void_p]
@@ -76,7 +82,8 @@ _lib.temco_status_string.argtypes = [C.c_int]
 _lib.temco_status_string.restype = C.c_char_p
 _lib.temco_last_error.restype = C.c_char_p
 for _f in ["temco_plan_create", "temco_run", "temco_run_host", "temco_run_host_async", "temco_run_profiled", "temco_peak_internal_bytes",
-           "temco_output_shape", "temco_plan_describe", "temco_debug_step_output", "temco_plan_destroy"]:
+           "temco_output_shape", "temco_plan_describe", "temco_debug_step_output", "temco_debug_step_tensor",
+           "temco_plan_destroy"]:
     getattr(_lib, _f).restype = C.c_int
 
 
@@ -215,17 +222,18 @@ class Plan:
                                        _stream_handle(stream), ms, n), "temco_run_profiled")
         return list(ms)
 
-    def step_output(self, x, y, step, stream=None):
-        """Run schedule steps 0..step and return that step's output tensor as raw
-        bytes (NHWC, plan dtype; fp32 for the graph output) -- a verification hook."""
+    def step_output(self, x, y, step, stream=None, which=0):
+        """Run schedule steps 0..step and return that step's output tensor `which` (0: the
+        step's tensor; 1..: a merged group's further reduce outputs) as raw bytes (NHWC,
+        plan dtype; fp32 for the graph output) -- a verification hook."""
         nb = C.c_int64(0)
         xs, ys = C.c_void_p(x.data_ptr()), C.c_void_p(y.data_ptr())
-        _check(_lib.temco_debug_step_output(self._h, xs, ys, _stream_handle(stream), step, None, 0, C.byref(nb)),
-               "temco_debug_step_output")
+        _check(_lib.temco_debug_step_tensor(self._h, xs, ys, _stream_handle(stream), step, which, None, 0,
+                                            C.byref(nb)), "temco_debug_step_tensor")
         buf = np.empty(nb.value, np.uint8)
-        _check(_lib.temco_debug_step_output(self._h, xs, ys, _stream_handle(stream), step,
+        _check(_lib.temco_debug_step_tensor(self._h, xs, ys, _stream_handle(stream), step, which,
                                             buf.ctypes.data_as(C.c_void_p), nb.value, C.byref(nb)),
-               "temco_debug_step_output")
+               "temco_debug_step_tensor")
         return buf
 
     def close(self):

@@ -181,3 +181,25 @@ def test_fp32_resnet18c_survey_parity_case():
     assert np.isfinite(y).all()
     assert _rel(y, ref) <= 1e-4, _rel(y, ref)
     assert p.peak_internal_bytes(0) == o.peak_fused
+
+
+@pytest.mark.parametrize("name", ["t3", "resnet18_s", "resnet50_s", "resnet18_tt_s"])
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+def test_merge_and_reschedule_variants(name, dt):
+    """Readings R37 (merged fconvs) and R38 (re-scheduling) under each policy: the default, the
+    "bound" merge policy (every candidate merged: ResNet-50's stage-2 group on the CTA-pair kernel
+    with two reduce outputs), and neither.  Output vs the oracle's plan with the same options, peak
+    bytes exact; a merged group's outputs are checked step by step in test_gpu_steps.py."""
+    from paper_conf_icpp_songljkj0024_b200 import FLAG_CSE_BOUND, FLAG_NO_CSE, FLAG_NO_RESCHEDULE
+    m = SMALL[name](dt)
+    x = W.make_input(m)
+    tol = 1e-4 if dt == "f32" else 2e-2
+    for flags, kw in ((0, {}), (FLAG_CSE_BOUND, {"cse_policy": "bound"}),
+                      (FLAG_NO_CSE | FLAG_NO_RESCHEDULE, {"cse": False, "reorder": False})):
+        o = oracle.plan(m, **kw)
+        ref = oracle.run_temco(o, x)
+        p, y = _plan_and_run(m, flags=flags, x=x)
+        assert np.isfinite(y).all()
+        assert _rel(y, ref) <= tol, (flags, _rel(y, ref))
+        assert p.peak_internal_bytes(0) == o.peak_fused
+        assert [s["extra"] for s in p.describe()["steps"]] == [s.extra for s in o.steps]

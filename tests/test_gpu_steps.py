@@ -51,8 +51,8 @@ def test_every_step_full_size_one_image(name):
     m = W.build_config(name, batch=1)
     x = W.make_input(m)
     o = oracle.plan(m)
-    chained = {}
-    oracle.run_temco(o, x, on_step=lambda t, v: chained.__setitem__(t, v))
+    chained = {}                                           # every tensor S defines, by id
+    oracle.run_temco(o, x, on_tensor=lambda i, v: chained.__setitem__(i, v))
     p = Plan(m)
     steps = p.describe()["steps"]
     assert len(steps) == len(o.steps)
@@ -64,20 +64,24 @@ def test_every_step_full_size_one_image(name):
     for t, s in enumerate(steps):
         if s["kernel"] == "none":
             continue
-        ref_chain = chained[t]
-        got = _to_f64(p.step_output(xt, y, t), ref_chain.shape)
-        assert np.isfinite(got).all(), (name, t, s["kernel"])
-        ref_iso = run_step(o, t, gpu)
-        iso = _rel(got, ref_iso)
-        mx = float(np.abs(got - ref_iso).max() / max(np.abs(ref_iso).max(), 1e-30))
-        assert iso <= 1e-2, (name, t, s["kernel"], s["out"], "isolated rel L2", iso)
-        assert mx <= 3e-2, (name, t, s["kernel"], s["out"], "isolated max-abs / max", mx)
-        ch = _rel(got, ref_chain)
-        assert ch <= 4e-2, (name, t, s["kernel"], s["out"], "chained rel L2", ch)
-        worst_iso = max(worst_iso, (iso, (t, s["kernel"])))
-        worst_chain = max(worst_chain, (ch, (t, s["kernel"])))
-        gpu[s["out"]] = got
-        checked += 1
+        # every tensor the step defines: its root and a merged group's further reduces (R37)
+        got_all = {}
+        for which, tid in enumerate([s["out"]] + s["extra"]):
+            ref_chain = chained[tid]
+            got = _to_f64(p.step_output(xt, y, t, which=which), ref_chain.shape)
+            assert np.isfinite(got).all(), (name, t, s["kernel"])
+            ref_iso = run_step(o, t, gpu, which=tid)
+            iso = _rel(got, ref_iso)
+            mx = float(np.abs(got - ref_iso).max() / max(np.abs(ref_iso).max(), 1e-30))
+            assert iso <= 1e-2, (name, t, s["kernel"], tid, "isolated rel L2", iso)
+            assert mx <= 3e-2, (name, t, s["kernel"], tid, "isolated max-abs / max", mx)
+            ch = _rel(got, ref_chain)
+            assert ch <= 4e-2, (name, t, s["kernel"], tid, "chained rel L2", ch)
+            worst_iso = max(worst_iso, (iso, (t, s["kernel"])))
+            worst_chain = max(worst_chain, (ch, (t, s["kernel"])))
+            got_all[tid] = got
+            checked += 1
+        gpu.update(got_all)
     assert checked >= 10
     print(f"{name}: {checked} steps; worst isolated rel L2 {worst_iso[0]:.2e} at {worst_iso[1]}, "
           f"worst chained {worst_chain[0]:.2e} at {worst_chain[1]}")

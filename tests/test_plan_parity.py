@@ -10,7 +10,7 @@ import workloads as W
 from paper_conf_icpp_songljkj0024_b200 import (FLAG_NO_DEVICE, FLAG_NO_FUSION, FLAG_NO_SKIPOPT,
                                               FLAG_OVERHEAD_NEVER, FLAG_PAPER_SCHEDULE, Plan, TemcoError)
 
-KEYS = ("kind", "out", "op", "role", "members", "inputs", "bytes")
+KEYS = ("kind", "out", "op", "role", "members", "inputs", "bytes", "extra")
 
 SMALL = {
     "c1": W.c1_basic_block, "t1": W.t1_chain, "t2_1": lambda: W.t2_stem_blocks(1),
