@@ -17,7 +17,7 @@ BUILD = os.path.join(ROOT, "build", "temco" + ("_" + VARIANT if VARIANT else "")
 LIB = os.path.join(ROOT, "build", "exp", f"libtemco_{VARIANT}.so") if VARIANT else os.path.join(PKG, "libtemco.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
-SOURCES = ["planner.cpp", "capi.cu", "kernels_simt.cu", "kernels_tc.cu", "kernels_tc_wide.cu", "kernels_conv.cu", "kernels_mma.cu", "kernels_stem.cu", "kernels_rank.cu", "kernels_cat.cu", "kernels_pair.cu", "kernels_gemm.cu"]
+SOURCES = ["planner.cpp", "capi.cu", "kernels_simt.cu", "kernels_tc.cu", "kernels_tc_wide.cu", "kernels_conv.cu", "kernels_mma.cu", "kernels_stem.cu", "kernels_rank.cu", "kernels_cat.cu", "kernels_pair.cu", "kernels_gemm.cu", "kernels_tile.cu"]
 GENCODE = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
           "--expt-relaxed-constexpr", "-I" + os.path.join(ROOT, "include")]

@@ -19,6 +19,7 @@
 #include "tc_wide.h"
 #include "pair.h"
 #include "gemm.h"
+#include "tile.h"
 
 
 using namespace temco;
@@ -38,7 +39,7 @@ temco_status set_err(temco_status s, const std::string& m) {
     if (e_ != cudaSuccess) return set_err(TEMCO_ERR_CUDA, std::string(#expr ": ") + cudaGetErrorString(e_)); \
   } while (0)
 
-enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM, K_DWPAIR,
+enum StepKind { K_NONE, K_CONVT, K_CONV, K_EW, K_LINEAR, K_GROUP_SIMT, K_GROUP_TC, K_CONV_TC, K_GROUP_MMA, K_GROUP_TCW, K_CONV_RK, K_GROUP_CAT, K_GROUP_PAIR, K_GEMM, K_DWPAIR, K_CONV_TILE,
                 K_MULTI /* a merged group replayed once per output: the launches of sub_exec[sub] */ };
 
 struct StepExec {
@@ -54,6 +55,7 @@ struct StepExec {
   ConvTcDesc ctc{};
   MmaChainDesc mma{};
   RankConvDesc rk{};
+  TileConvDesc tile{};
   CatDesc cat{};
   DwPairDesc dwp{};
   std::string kernel;
@@ -459,6 +461,15 @@ void lower(temco_plan_s* P) {
           c.Ho = v.H; c.Wo = v.W; c.K = v.C;
           c.kh = v.kh; c.kw = v.kw; c.sh = v.sh; c.sw = v.sw; c.ph = v.ph; c.pw = v.pw; c.groups = v.groups;
           c.b = v.b ? push_params(P, v.b) : -1;
+          {   // reduced-rank cores: TMA-staged footprints, ldmatrix A / B, mma.sync (kernels_tile.cu)
+            const std::vector<float> w = repack_conv(v, x.C);
+            if (tile_conv_lower(c, w.data(), P->tcw_h, e.tile)) {
+              e.kind = K_CONV_TILE;
+              e.kernel = "mma_conv_tile";
+              e.launches = 1;
+              break;
+            }
+          }
           // 3x3 cores on 8 channels: the direct SIMT kernel measured faster (kernels_simt.cu)
           // (wider outputs stay on the tcgen05 implicit GEMM: measured faster for K > 64)
           if (c.C <= 256 && c.K <= 64 && !(c.C == 8 && c.K == 8 && c.kh * c.kw > 1)) {
@@ -728,6 +739,7 @@ std::string make_json(const temco_plan_s* P) {
       if (e.kind == K_GEMM) o << ",\"alg_flops\":" << e.gm.alg_flops << ",\"alg_bytes\":" << e.gm.alg_bytes << ",\"splits\":" << e.gm.splits;
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;
       if (e.kind == K_CONV_RK) o << ",\"alg_flops\":" << e.rk.alg_flops << ",\"alg_bytes\":" << e.rk.alg_bytes;
+      if (e.kind == K_CONV_TILE) o << ",\"alg_flops\":" << e.tile.alg_flops << ",\"alg_bytes\":" << e.tile.alg_bytes;
       if (e.kind == K_GROUP_CAT) o << ",\"alg_flops\":" << e.cat.alg_flops << ",\"alg_bytes\":" << e.cat.alg_bytes;
       if (e.kind == K_GROUP_MMA) o << ",\"alg_flops\":" << e.mma.alg_flops << ",\"alg_bytes\":" << e.mma.alg_bytes;
     }
@@ -806,6 +818,7 @@ void launch_exec(temco_plan_s* P, const StepExec& e, const RunPtrs& rp, cudaStre
     case K_GEMM: launch_gemm(e.gm, rp, P->lin_ws_d, st); break;
     case K_CONV_TC: launch_conv_tc(e.ctc, rp, st); break;
     case K_CONV_RK: launch_conv_rank_mma(e.rk, P->tcw_d, rp, st); break;
+    case K_CONV_TILE: launch_tile_conv(e.tile, P->tcw_d, rp, st); break;
     case K_GROUP_CAT: launch_mma_cat(e.cat, P->tcw_d, rp, st); break;
     case K_GROUP_MMA: launch_mma_chain(e.mma, P->tcw_d, rp, st); break;
     case K_MULTI:
@@ -966,6 +979,12 @@ temco_status temco_plan_create(const temco_layer* layers, int32_t n_layers, cons
       delete P;
       return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
     }
+    for (StepExec* e : ex)
+      if (e->kind == K_CONV_TILE && !tile_conv_finalize(e->tile, P->arena_d, terr)) {
+        free_device(P);
+        delete P;
+        return set_err(TEMCO_ERR_CUDA, "tensor maps: " + terr);
+      }
     for (StepExec* e : ex)
       if (e->kind == K_GEMM && !gemm_finalize(e->gm, P->arena_d, P->tcw_d, terr)) {
         free_device(P);
