@@ -49,23 +49,31 @@ bool tile_conv_lower(const ConvDesc& c, const float* w, std::vector<uint16_t>& t
   d.Ho = c.Ho; d.Wo = c.Wo; d.K = c.K;
   d.kh = c.kh; d.kw = c.kw; d.sh = c.sh; d.sw = c.sw; d.ph = c.ph; d.pw = c.pw;
   d.b = c.b;
+  d.dbg = getenv("TEMCO_TILE_DBG") ? atoi(getenv("TEMCO_TILE_DBG")) : 0;
   const int taps = c.kh * c.kw;
   d.pair = (c.C == 8 && taps > 1) ? 1 : 0;
   d.ksc = (c.C + 15) / 16;
   d.nks = d.pair ? (taps + 1) / 2 : taps * d.ksc;
   const int cb = c.C * 2;
-  d.swz = cb == 32 ? 1 : cb == 64 ? 2 : cb == 128 ? 3 : 0;
   // 1x1 strided cores (the downsample cores): the TMA box takes every sh-th row / sw-th column
   const bool sub = c.kh == 1 && c.kw == 1;
+  // TMA view: cw pixels per inner row (up to 128 bytes) so that narrow pixels (C = 8 .. 32) are not
+  // fetched 16 / 32 / 64 bytes per TMA row; the inner row is the swizzle span
+  d.cw = 1;
+  if (!sub)
+    while (d.cw * 2 * cb <= 128 && c.W % (d.cw * 2) == 0) d.cw *= 2;
+  const int ib = d.cw * cb;
+  d.swz = ib == 32 ? 1 : ib == 64 ? 2 : ib == 128 ? 3 : 0;
   // tile: columns split into <= 32-wide equal parts; whole small images grouped
   const int ntw = (c.Wo + 31) / 32;
   d.TW = (c.Wo + ntw - 1) / ntw;
   d.TN = 1;
   if (c.Ho * d.TW < 128) d.TN = std::max(1, std::min({c.N, 256 / (c.Ho * d.TW), 256}));
   d.TH = d.TN > 1 ? c.Ho : std::min(c.Ho, (256 + d.TW - 1) / d.TW);
-  auto foot = [&](int TH, int TN) {
+  auto foot = [&](int TH, int TN) {   // TMA bytes of a footprint: FH rows of G inner rows
     const int FH = sub ? TH : (TH - 1) * c.sh + c.kh, FW = sub ? d.TW : (d.TW - 1) * c.sw + c.kw;
-    return (int64_t)FH * FW * TN * cb;
+    const int G = (FW + d.cw - 1 + d.cw - 1) / d.cw;   // any start offset within an inner row
+    return (int64_t)FH * (sub ? FW : G * d.cw) * TN * cb;
   };
   while (d.TN > 1 && foot(d.TH, d.TN) > kTcFootBudget) --d.TN;
   while (d.TH > 1 && foot(d.TH, d.TN) > kTcFootBudget) --d.TH;
@@ -81,6 +89,9 @@ bool tile_conv_lower(const ConvDesc& c, const float* w, std::vector<uint16_t>& t
   while (d.TN == 1 && d.TH * d.TW > 64 && d.TH > 1 && count(d.TH, 1) < 296) d.TH = (d.TH + 1) / 2;
   d.FH = sub ? d.TH : (d.TH - 1) * c.sh + c.kh;
   d.FW = sub ? d.TW : (d.TW - 1) * c.sw + c.kw;
+  d.G = sub ? d.FW : (d.FW + 2 * d.cw - 2) / d.cw;
+  d.RP = sub ? d.FW : d.G * d.cw;
+  if (d.G > 256) return false;
   d.tiles_w = (c.Wo + d.TW - 1) / d.TW;
   d.tiles_h = (c.Ho + d.TH - 1) / d.TH;
   d.tiles_n = (c.N + d.TN - 1) / d.TN;
@@ -138,10 +149,11 @@ bool tile_conv_finalize(TileConvDesc& d, const char* arena, std::string& err) {
     encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
   }
   const bool sub = d.kh == 1 && d.kw == 1;
-  cuuint64_t dims[4] = {(cuuint64_t)d.C, (cuuint64_t)d.W, (cuuint64_t)d.H, (cuuint64_t)d.N};
-  cuuint64_t strides[3] = {(cuuint64_t)d.C * 2, (cuuint64_t)d.W * d.C * 2, (cuuint64_t)d.H * d.W * d.C * 2};
-  cuuint32_t box[4] = {(cuuint32_t)d.C, (cuuint32_t)(sub ? d.TW * d.sw : d.FW), (cuuint32_t)(sub ? d.TH * d.sh : d.FH),
-                       (cuuint32_t)d.TN};
+  // view (cw * C, W / cw, H, N): an inner row = cw consecutive pixels of an image row
+  cuuint64_t dims[4] = {(cuuint64_t)d.cw * d.C, (cuuint64_t)(d.W / d.cw), (cuuint64_t)d.H, (cuuint64_t)d.N};
+  cuuint64_t strides[3] = {(cuuint64_t)d.cw * d.C * 2, (cuuint64_t)d.W * d.C * 2, (cuuint64_t)d.H * d.W * d.C * 2};
+  cuuint32_t box[4] = {(cuuint32_t)(d.cw * d.C), (cuuint32_t)(sub ? d.TW * d.sw : d.G),
+                       (cuuint32_t)(sub ? d.TH * d.sh : d.FH), (cuuint32_t)d.TN};
   cuuint32_t es[4] = {1, (cuuint32_t)(sub ? d.sw : 1), (cuuint32_t)(sub ? d.sh : 1), 1};
   const CUtensorMapSwizzle sw = d.swz == 1   ? CU_TENSOR_MAP_SWIZZLE_32B
                                 : d.swz == 2 ? CU_TENSOR_MAP_SWIZZLE_64B
@@ -221,7 +233,7 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
         boff = (ks % d.ksc) * 32 + h * 16;
       }
       const int ty = tap / d.kw, tx = tap - ty * d.kw;
-      ktab[i] = make_int2(ty * d.FW + tx, boff);
+      ktab[i] = make_int2(ty * d.RP + tx, boff);
     }
     // slack after each footprint: the upper half of the last k-step of C % 16 == 8 reads 16 bytes
     // past the last pixel (zero weights; the data must only be finite)
@@ -231,6 +243,7 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
   }
   __syncthreads();
   pdl_wait();
+  if (d.dbg & 4) return;
   const int G = gridDim.x;
   const int tpi = d.tiles_w * d.tiles_h;
   if (warp == kTcWarps) {
@@ -242,9 +255,14 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
         const int b = it % kTcBufs;
         if (it >= kTcBufs) mbar_wait(&empty[b], (uint32_t)(it / kTcBufs - 1) & 1u);
         const int tn = tile / tpi, th = (tile / d.tiles_w) % d.tiles_h, tw = tile % d.tiles_w;
+        if (d.dbg & 2) {
+          mbar_arrive(&full[b]);
+          continue;
+        }
         mbar_expect_tx(&full[b], (uint32_t)d.box_bytes);
-        tma_load_4d(smem + b * d.buf_bytes, d.xmap, &full[b], 0, tw * d.TW * d.sw - d.pw, th * d.TH * d.sh - d.ph,
-                    tn * d.TN);
+        const int x0 = tw * d.TW * d.sw - d.pw;   // first footprint column; its inner row (floor)
+        const int xg = x0 >= 0 ? x0 / d.cw : -((d.cw - 1 - x0) / d.cw);
+        tma_load_4d(smem + b * d.buf_bytes, d.xmap, &full[b], 0, xg, th * d.TH * d.sh - d.ph, tn * d.TN);
       }
     }
     return;
@@ -272,8 +290,10 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
     const uint32_t fbase = smem_u32(smem + b * d.buf_bytes);
     const int tn = tile / tpi, th = (tile / d.tiles_w) % d.tiles_h, tw = tile % d.tiles_w;
     const int n0 = tn * d.TN, oh0 = th * d.TH, ow0 = tw * d.TW;
+    const int x0 = ow0 * d.sw - d.pw, xr = x0 - (x0 >= 0 ? x0 / d.cw : -((d.cw - 1 - x0) / d.cw)) * d.cw;
     int pr = warp - pstart % kTcWarps;
     if (pr < 0) pr += kTcWarps;
+    if (d.dbg & 1) pr = npair;
     for (; pr < npair; pr += kTcWarps) {
       const int mt0 = 2 * pr;
       int pbase[2];
@@ -282,7 +302,7 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
         int q = (mt0 + j) * 16 + ar;
         if (q >= npx) q = 0;
         const int pn = fdiv(q, d.mpx, d.spx), rem = q - pn * pxt, py = fdiv(rem, d.mtw, d.stw), px = rem - py * d.TW;
-        pbase[j] = (pn * d.FH + py * she) * d.FW + px * swe;
+        pbase[j] = (pn * d.FH + py * she) * d.RP + px * swe + xr;   // + the box's start offset
       }
       float acc[2][2 * NT2][4];
 #pragma unroll

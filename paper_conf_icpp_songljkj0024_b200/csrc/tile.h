@@ -25,6 +25,8 @@ struct TileConvDesc {
   int32_t kh, kw, sh, sw, ph, pw;
   int32_t TH, TW, TN;            // output tile: rows, columns, images
   int32_t FH, FW;                // input footprint rows / columns of one image
+  int32_t cw, G, RP;             // TMA view: cw pixels per inner row (cw*C*2 bytes, the swizzle span),
+                                 // G inner rows per footprint row, RP = G*cw pixels per SMEM footprint row
   int32_t tiles_w, tiles_h, tiles_n, ntiles;
   int32_t pair;                  // C == 8: one k-step of 16 covers two taps
   int32_t ksc;                   // k-steps per tap (C > 8): ceil(C / 16)
@@ -39,6 +41,7 @@ struct TileConvDesc {
   int32_t smem_bytes;
   int64_t b;                     // params offset of an fp32 bias, or -1
   int64_t alg_flops, alg_bytes;
+  int32_t dbg;                   // timing experiments (TEMCO_TILE_DBG): 1 no compute, 2 no TMA
 };
 
 // w = fp32 [K][kh][kw][C]; false if the conv is outside the kernel's shapes (bf16, C % 8 == 0,

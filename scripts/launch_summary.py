@@ -13,7 +13,7 @@ CLASS = {"tc_chain_kernel": "tc_chain", "conv_tc_kernel": "tc_conv", "conv_tma_k
          "conv_small_kernel": "simt_conv_small", "conv_stem_kernel": "mma_conv_stem", "linear_kernel": "simt_linear", "conv_kernel": "simt_conv",
          "ew_kernel": "simt_ew", "group_simt_kernel": "simt_group", "group_gap_kernel": "simt_group_gap",
          "mma_chain_kernel": "mma_chain", "mma_lean_kernel": "mma_lean", "conv_rank_mma_kernel": "mma_conv_rank", "mma_catp_kernel": "mma_catp",
-         "conv_rank_kernel": "simt_conv_rank", "dwconv_vec_kernel": "simt_dwconv_vec", "gemm_kernel": "tc_gemm", "gemm_reduce_kernel": "tc_gemm", "pair_chain_kernel": "tc_pair",
+         "conv_rank_kernel": "simt_conv_rank", "dwconv_vec_kernel": "simt_dwconv_vec", "gemm_kernel": "tc_gemm", "tile_conv_kernel": "mma_conv_tile", "dwpair_kernel": "simt_dwpair", "dwpair_generic_kernel": "simt_dwpair", "gemm_reduce_kernel": "tc_gemm", "pair_chain_kernel": "tc_pair",
          "mma_lean64_kernel": "mma_lean", "mma_poolcat_kernel": "mma_poolcat", "mma_cat_kernel": "mma_cat",
          "dwconv_col_kernel": "simt_dwconv_vec", "dwconv_row_kernel": "simt_dwconv_vec"}
 
