@@ -126,6 +126,10 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
     d.ycol[k + 1] = d.ycol[k] + ir.nodes[roots[k]].C;
   }
   d.n_levels = (int)levels.size();
+  {
+    const char* e = getenv("TEMCO_PAIR_FCONV_LAG");
+    d.flag = std::min(d.n_levels - 1, e ? atoi(e) : 0);
+  }
   int64_t flops = 0, bytes = 0;
   while (params.size() % 4) params.push_back(0.f);
   d.lbias = (int64_t)params.size();
@@ -224,7 +228,7 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
       for (; jj < d.lvl_end[l]; ++jj) k += d.term[jj].R;
       kmax = std::max(kmax, k);
     }
-    d.bias_mma = (kmax <= 64 && !getenv("TEMCO_PAIR_NO_BIASMMA")) ? 1 : 0;
+    d.bias_mma = getenv("TEMCO_PAIR_NO_BIASMMA") ? 0 : 1;
   }
   if (d.bias_mma) {
     std::vector<float> bm((size_t)d.n_levels * d.Cpad * 16, 0.f);
@@ -407,6 +411,31 @@ __device__ __forceinline__ float silu_or(float x, int act) {
 template <bool SILU>
 __device__ __forceinline__ void level_math(uint32_t (&t)[16], const uint32_t (&v)[32], bool first, int act,
                                            const float* bias) {
+  if (!bias && act != 2) {
+    // bias added by the tensor core (bias MMA): t = act(a + t) in packed bf16x2 -- the level
+    // accumulator a rounded to bf16 (cvt, one instruction per two channels), then one fused
+    // a * 1 + t with the ReLU (fma.rn.relu.bf16x2) rounding once: two instructions per two
+    // channels instead of unpacking t to fp32 (reading R29: t lives in bf16 between levels)
+    if (first) {
+#pragma unroll
+      for (int i = 0; i < 16; ++i)
+        t[i] = act == 1 ? pack_relu(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]))
+                        : pack_bf16(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+    } else if (act == 1) {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        const uint32_t a2 = pack_bf16(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+        asm("fma.rn.relu.bf16x2 %0, %1, %2, %0;" : "+r"(t[i]) : "r"(a2), "r"(0x3F803F80u));
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        const uint32_t a2 = pack_bf16(__uint_as_float(v[2 * i]), __uint_as_float(v[2 * i + 1]));
+        asm("fma.rn.bf16x2 %0, %1, %2, %0;" : "+r"(t[i]) : "r"(a2), "r"(0x3F803F80u));
+      }
+    }
+    return;
+  }
   float z[32];
 #pragma unroll
   for (int i = 0; i < 32; ++i) z[i] = __uint_as_float(v[i]);
@@ -590,7 +619,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                                  (int)(op.x >> 28) * d.Cpad + (u0 + q) * kPairWu + (int)cta * 64);
             }
             PAIR_NEXT();
-            if ((fl & 6u) == 6u && pend >= 0 && !d.resident) {   // after level 0: the previous pair's fconv operands
+            if ((fl & 2u) && (int)(op.x >> 28) == d.flag && pend >= 0 && !d.resident) {   // after level flag: the previous pair's fconv operands
               PAIR_FCONV_ATOMS(pend);
               pend = -1;
             }
@@ -687,7 +716,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             int kl = k;   // last atom of this level
             while (!((lds128(tab_s + 16u * kl).x >> 24) & 2u)) ++kl;
             const int nat = kl - k + 1;
-            const bool first_level = (op0x >> 24) & 4u;
             int b1 = b + 1;   // buffer of the pair's second unit
             if (b1 >= NB) b1 -= NB;
             const uint32_t d0 = tbase + (uint32_t)(b * kPairWu), d1 = tbase + (uint32_t)(b1 * kPairWu);
@@ -746,7 +774,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             }
             b += nu;
             if (b >= NB) b -= NB;
-            if (first_level && pend >= 0) {
+            if ((int)(op0x >> 28) == d.flag && pend >= 0) {   // the previous pair's fconv, d.flag levels late
               PAIR_FCONV(pend, pend_tile_first, pend_tile_last);
               pend = -1;
             }
@@ -770,9 +798,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     const uint32_t pfull_c = mapa_shared(smem_u32(p_full), 0);
     const uint32_t oempty_c = mapa_shared(smem_u32(out_empty), 0);
-    __nv_bfloat16* yk[kPairMaxOuts];
-    for (int k = 0; k < kPairMaxOuts; ++k)
-      yk[k] = k < d.n_out ? reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.ys[k], p))) : nullptr;
+
     int gi = 0, np = 0, it = 0;   // gi: (unit, level) accumulator items consumed
     EVDECL();
     const bool ev0 = warp == kEpiWarp0 && lane == 0;
@@ -796,7 +822,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           pk.w = pack_bf16(__uint_as_float(v[6]), __uint_as_float(v[7]));
           int k = 0;   // output holding column c8 * 8 (a merged group's fconvs, reading R37)
           while (k + 1 < d.n_out && c8 * 8 >= d.ycol[k + 1]) ++k;
-          *reinterpret_cast<uint4*>(yk[k] + orow * (d.ycol[k + 1] - d.ycol[k]) + (c8 * 8 - d.ycol[k])) = pk;
+          __nv_bfloat16* yk = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.ys[k], p)));
+          *reinterpret_cast<uint4*>(yk + orow * (d.ycol[k + 1] - d.ycol[k]) + (c8 * 8 - d.ycol[k])) = pk;
         }
       }
       tc_fence_before();
@@ -837,7 +864,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             }
           }
           gi += nu;
-          if (l == 0 && pp == 0 && pend_it >= 0) {
+          if (l == d.flag && pp == 0 && pend_it >= 0) {
             drain_out(pend_it, pend_row);
             pend_it = -1;
           }

@@ -80,6 +80,9 @@ struct PairDesc {
   int32_t bsz, fsz;                      // resident Lhat atom slot (64 x awmax bf16), F atom (Np/2 x 64 bf16)
   int32_t res_c, res_f;                  // offsets of the bias-MMA and F atoms in the resident region
   int32_t silu;                          // some level is SiLU: SILU kernel instantiation
+  int32_t flag;                          // the previous unit pair's fconv is issued after this level of the
+                                         // next pair (and the out tile drained after it): the epilogue's P
+                                         // writes have that many levels of slack before the issuer waits
   int64_t alg_flops, alg_bytes;          // algorithmic work (unpadded ranks), for the roofline
 };
 

@@ -1,0 +1,7 @@
+timeout 900 python -m pytest tests -m gpu -q -x -k "every_step or full_config or bf16_mode or merge" > gpurun_out/r2b_pair_tests.log 2>&1; tail -2 gpurun_out/r2b_pair_tests.log
+TEMCO_PAIR_BIASMMA_ALL=1 timeout 900 python -m pytest tests -m gpu -q -x -k "every_step or full_config or bf16_mode" > gpurun_out/r2b_pair_tests2.log 2>&1; tail -2 gpurun_out/r2b_pair_tests2.log
+for v in "" "TEMCO_PAIR_BIASMMA_ALL=1"; do
+  for c in resnet50 densenet121 resnet18_cifar unet vgg16_cp; do
+    echo "=== $c $v $(env $v timeout 300 python bench.py --config $c --no-cpu-baseline 2>/dev/null | tail -1 | python -c 'import json,sys; d=json.loads(sys.stdin.read()); print(round(d["value"]), round(d["ms_per_step"],4), round(d["roofline"]["frac"],3))')"
+  done
+done
