@@ -184,7 +184,9 @@ def cpu_baseline(config):
             "sample": f"{sample} images of {config} through the oracle's TeMCO executor (fp64 numpy), {dt:.1f} s"}
 
 
-VARIANTS = {"temco": 0, "fusion_only": 2, "skipopt_only": 4, "decomposed": 6}   # TEMCO_FLAG_NO_SKIPOPT=2, NO_FUSION=4
+VARIANTS = {"temco": 0, "fusion_only": 2, "skipopt_only": 4, "decomposed": 6,   # TEMCO_FLAG_NO_SKIPOPT=2, NO_FUSION=4
+            "paper_schedule": 1 << 9,   # the paper's schedule: no readings R34-R38 (TEMCO_FLAG_PAPER_SCHEDULE)
+            "cse_bound": 1 << 12}       # reading R37 merges kept while the peak stays <= the unfused peak
 
 
 def main():

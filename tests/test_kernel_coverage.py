@@ -27,7 +27,7 @@ def test_small_cases_cover_the_full_configs():
         full.update(_kernels(W.build_config(name)))
     assert set(full) <= set(small), set(full) - set(small)
     # the tensor-core families are all on the bench path
-    for k in ("tc_chain", "tc_pair", "mma_lean", "mma_conv_rank", "mma_conv_stem", "tc_conv", "tc_gemm",
+    for k in ("tc_chain", "tc_pair", "mma_lean", "mma_conv_tile", "mma_conv_stem", "tc_conv", "tc_gemm",
               "tc_gemm_convt"):
         assert full[k] > 0, k
 
