@@ -653,12 +653,21 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
           const float2 b = *reinterpret_cast<const float2*>(fb + d.lbias + ch * 64 + nt * 8 + 2 * t4);
           D[nt][0] = b.x; D[nt][1] = b.y; D[nt][2] = b.x; D[nt][3] = b.y;
         }
-        for (int ui = 0; ui < d.n_units; ++ui) {
-          const CatUnit u = d.unit[ui];
-          if (u.chunk != ch || u.term < 0) continue;
-          uint32_t a[1][4];
+        // this chunk's units only, their A loads issued together (in flight at once)
+        const int cu0 = d.chunk_u0[ch], cu1 = d.chunk_u0[ch + 1];
+        for (int ub = cu0; ub < cu1; ub += 4) {
+        uint32_t aq[4][1][4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
           bool va[2];
-          cat_load<1>(a, va, d, p, u, rw, t4);
+          if (ub + q < cu1) cat_load<1>(aq[q], va, d, p, d.unit[ub + q], rw, t4);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          if (ub + q >= cu1) break;
+          const CatUnit u = d.unit[ub + q];
+          if (u.term < 0) continue;
+          uint32_t (&a)[1][4] = aq[q];
           const int rs = d.term[u.term].rs;
           const uint32_t wb = sbase + (uint32_t)((u.woff + ((lq >> 1) * 8 + lr) * rs + (lq & 1) * 8) * 2);
           const uint32_t wb2 = sbase + (uint32_t)((u.woff + lr * rs + (lq & 1) * 8) * 2);
@@ -682,6 +691,7 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
               mma16816(D[nt + 1], a[0], b0, b1);
             }
           }
+        }
         }
         if (d.relu) {
 #pragma unroll

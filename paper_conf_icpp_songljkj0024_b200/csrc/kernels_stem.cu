@@ -135,7 +135,7 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
   const int ntiles = d.N * tiles_w * tiles_h;
   // footprint of a tile as 16-byte chunks of image rows, kStCPT chunks per thread in registers
   uint4 v[kStCPT];
-  auto load = [&](int tile) {
+  auto load_any = [&](int tile) {
     const int n = tile / (tiles_w * tiles_h);
     const int h0 = (tile / tiles_w) % tiles_h * g.TH, w0 = tile % tiles_w * g.TW;
     const int hi0 = h0 * d.sh - d.ph, e0 = (w0 * d.sw - d.pw) * d.C;
@@ -149,7 +149,7 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
       v[q] = ok ? __ldg(x4 + (((int64_t)n * d.H + hi) * rowC) / 8 + ch) : make_uint4(0, 0, 0, 0);
     }
   };
-  auto store = [&](int tile, __nv_bfloat16* buf) {
+  auto store_any = [&](int tile, __nv_bfloat16* buf) {
     const int w0 = tile % tiles_w * g.TW;
     const int e0 = (w0 * d.sw - d.pw) * d.C;
     const int a0 = e0 >= 0 ? e0 / 8 : -((7 - e0) / 8);
@@ -170,6 +170,69 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
         }
       }
     }
+  };
+  // 3-channel images (every stem here): 8-pixel groups -- 3 chunks of 16 bytes = 24 elements = 8 whole
+  // pixels -- so each pixel goes to SMEM as one 8-byte (c0, c1, c2, 0) store with compile-time element
+  // extraction, instead of 8 scalar stores per chunk with per-element index arithmetic
+  const bool g3 = d.C == 3 && g.Cp == 4;
+  auto grp = [&](int tile, int& gA, int& ng, int& fx0) {
+    const int w0 = tile % tiles_w * g.TW;
+    fx0 = w0 * d.sw - d.pw;
+    gA = fx0 >= 0 ? fx0 / 8 : -((7 - fx0) / 8);
+    const int e = fx0 + g.PC;   // one past the last footprint column
+    ng = (e >= 0 ? (e + 7) / 8 : -((-e) / 8)) - gA;
+  };
+  auto load3 = [&](int tile) {
+    const int n = tile / (tiles_w * tiles_h);
+    const int h0 = (tile / tiles_w) % tiles_h * g.TH;
+    const int hi0 = h0 * d.sh - d.ph;
+    int gA, ng, fx0;
+    grp(tile, gA, ng, fx0);
+#pragma unroll
+    for (int q = 0; q < kStCPT / 3; ++q) {
+      const int i = threadIdx.x + q * kStThreads;
+      const int r = i / ng, gg = i - r * ng, hi = hi0 + r;
+      const bool rok = i < g.PR * ng && hi >= 0 && hi < d.H;
+      const int64_t rowb = (((int64_t)n * d.H + hi) * rowC) / 8;
+#pragma unroll
+      for (int c3 = 0; c3 < 3; ++c3) {
+        const int ch = (gA + gg) * 3 + c3;
+        v[q * 3 + c3] = (rok && ch >= 0 && ch * 8 < rowC) ? __ldg(x4 + rowb + ch) : make_uint4(0, 0, 0, 0);
+      }
+    }
+  };
+  auto store3 = [&](int tile, __nv_bfloat16* buf) {
+    int gA, ng, fx0;
+    grp(tile, gA, ng, fx0);
+#pragma unroll
+    for (int q = 0; q < kStCPT / 3; ++q) {
+      const int i = threadIdx.x + q * kStThreads;
+      if (i >= g.PR * ng) break;
+      const int r = i / ng, gg = i - r * ng;
+      const uint32_t w[12] = {v[3 * q].x, v[3 * q].y, v[3 * q].z, v[3 * q].w, v[3 * q + 1].x, v[3 * q + 1].y,
+                              v[3 * q + 1].z, v[3 * q + 1].w, v[3 * q + 2].x, v[3 * q + 2].y, v[3 * q + 2].z,
+                              v[3 * q + 2].w};
+      const int fc0 = (gA + gg) * 8 - fx0;
+#pragma unroll
+      for (int pp = 0; pp < 8; ++pp) {
+        const int fc = fc0 + pp;
+        if (fc < 0 || fc >= g.PC) continue;
+        const int e = 3 * pp;   // compile-time element positions of this pixel's three channels
+        const uint32_t c0 = (w[e >> 1] >> ((e & 1) * 16)) & 0xFFFFu;
+        const uint32_t c1 = (w[(e + 1) >> 1] >> (((e + 1) & 1) * 16)) & 0xFFFFu;
+        const uint32_t c2 = (w[(e + 2) >> 1] >> (((e + 2) & 1) * 16)) & 0xFFFFu;
+        *reinterpret_cast<uint2*>(reinterpret_cast<unsigned short*>(buf) + r * g.rowlen + fc * 4) =
+            make_uint2(c0 | (c1 << 16), c2);
+      }
+    }
+  };
+  auto load = [&](int tile) {
+    if (g3) load3(tile);
+    else load_any(tile);
+  };
+  auto store = [&](int tile, __nv_bfloat16* buf) {
+    if (g3) store3(tile, buf);
+    else store_any(tile, buf);
   };
   int tile = blockIdx.x;
   pdl_wait();
@@ -288,7 +351,8 @@ __global__ void __launch_bounds__(256) conv_pw_small_kernel(ConvDesc d, RunPtrs 
 }
 
 bool stem_fits(const ConvDesc& d, const StemGeo& g) {
-  return g.smem <= 96 * 1024 && g.PR * g.ncr <= kStCPT * kStThreads && g.PC * d.C < 2048;
+  const bool g3_fits = d.C != 3 || g.PR * ((g.PC + 7) / 8 + 1) <= kStCPT / 3 * kStThreads;   // 8-pixel groups
+  return g.smem <= 96 * 1024 && g.PR * g.ncr <= kStCPT * kStThreads && g.PC * d.C < 2048 && g3_fits;
 }
 
 StemGeo stem_pick(const ConvDesc& d) {
