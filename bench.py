@@ -361,7 +361,7 @@ def main():
         by_class[k] = {"bound": "tensor" if tb else "hbm", "achieved": round(ach, 1),
                        "unit": "TFLOP/s" if tb else "GB/s", "frac": round(ach / (tf_peak if tb else hbm), 4),
                        "ms": round(v["ms"], 4)}
-    fused_k = ("tc_pair", "tc_chain", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat", "mma_catp")
+    fused_k = ("tc_pair", "tc_chain", "tc_chain_wide", "mma_lean", "mma_chain", "mma_poolcat", "mma_cat", "mma_catp")
     ideal = actual = 0.0
     for s, t in zip(steps, prof):
         if s["kernel"] in fused_k and t > 0:

@@ -333,7 +333,7 @@ void lower_group(temco_plan_s* P, const Step& s, StepExec& e) {
   if (P->bf16 && !(P->flags & TEMCO_FLAG_SIMT_ONLY) &&
       wide::tc_lower_chain(ir, s, P->loc, P->tcw_h, P->params_h, e.tcw)) {
     e.kind = K_GROUP_TCW;
-    e.kernel = "tc_chain";
+    e.kernel = "tc_chain_wide";
     e.launches = 1;
     return;
   }

@@ -740,7 +740,7 @@ __device__ __forceinline__ float act_m(float x, int a) {
 }
 
 template <bool SILU>
-__global__ void __launch_bounds__(kThreads, 1) tc_chain_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
+__global__ void __launch_bounds__(kThreads, 1) tc_wide_kernel(const __grid_constant__ TcChainDesc d, RunPtrs p) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
   const int S = d.stages;
@@ -1259,8 +1259,8 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   static bool configured = false;
   static int sms = 0;
   if (!configured) {
-    cudaFuncSetAttribute(tc_chain_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
-    cudaFuncSetAttribute(tc_chain_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tc_wide_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tc_wide_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -1271,7 +1271,7 @@ void launch_tc_chain(const TcChainDesc& d, const uint16_t* tcw, const RunPtrs& p
   if (grid_cap > 0) grid = std::min(grid, grid_cap);
   // >= 114 KB of shared memory keeps one CTA per SM (each may own all 512 TMEM columns)
   const bool silu = d.mrelu == 2 || std::any_of(d.relu, d.relu + d.n_levels, [](int32_t a) { return a == 2; });
-  launch_pdl(silu ? tc_chain_kernel<true> : tc_chain_kernel<false>, dim3(grid), dim3(kThreads),
+  launch_pdl(silu ? tc_wide_kernel<true> : tc_wide_kernel<false>, dim3(grid), dim3(kThreads),
              std::max(d.smem_bytes, 116 * 1024), s, d, p);
 }
 

@@ -9,7 +9,7 @@ per-class times, not absolute values.
 """
 import collections, csv, io, json, sys
 
-CLASS = {"tc_chain_kernel": "tc_chain", "conv_tc_kernel": "tc_conv", "conv_tma_kernel": "tc_conv",
+CLASS = {"tc_chain_kernel": "tc_chain", "tc_wide_kernel": "tc_chain_wide", "conv_tc_kernel": "tc_conv", "conv_tma_kernel": "tc_conv",
          "conv_small_kernel": "simt_conv_small", "conv_stem_kernel": "mma_conv_stem", "linear_kernel": "simt_linear", "conv_kernel": "simt_conv",
          "ew_kernel": "simt_ew", "group_simt_kernel": "simt_group", "group_gap_kernel": "simt_group_gap",
          "mma_chain_kernel": "mma_chain", "mma_lean_kernel": "mma_lean", "conv_rank_mma_kernel": "mma_conv_rank", "mma_catp_kernel": "mma_catp",

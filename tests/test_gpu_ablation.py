@@ -99,7 +99,7 @@ def test_silu_activation(name, dt):
     if dt == "bf16" and name in ("resnet18_s", "resnet50_s", "densenet121_s"):
         from paper_conf_icpp_songljkj0024_b200 import FLAG_NO_DEVICE, Plan
         kernels = {s["kernel"] for s in Plan(m, flags=FLAG_NO_DEVICE).describe()["steps"]}
-        assert kernels & {"mma_lean", "mma_chain"} and "tc_chain" in kernels, kernels   # SiLU on the tensor-core kernels
+        assert kernels & {"mma_lean", "mma_chain"} and kernels & {"tc_chain", "tc_chain_wide"}, kernels   # SiLU on the tensor-core kernels
         assert not any(k.startswith("simt_group") for k in kernels), kernels            # incl. pooled members
     for flags in (0, FLAG_NO_FUSION):
         p, y = _run(m, flags, x)
