@@ -734,7 +734,7 @@ std::string make_json(const temco_plan_s* P) {
           << ",\"ntiles\":" << e.tcw.ntiles << ",\"Cc\":" << e.tcw.Cc << ",\"levels\":" << e.tcw.n_levels << "}";
       if (e.kind == K_GROUP_PAIR)
         o << ",\"alg_flops\":" << e.pr.alg_flops << ",\"alg_bytes\":" << e.pr.alg_bytes << ",\"tc\":{\"variant\":\"pair\",\"stages\":"
-          << e.pr.stages << ",\"smem\":" << e.pr.smem_bytes << ",\"ntiles\":" << e.pr.ntiles << ",\"units\":" << e.pr.nunits
+          << e.pr.stages << ",\"slot\":" << e.pr.slot << ",\"resident\":" << e.pr.resident << ",\"smem\":" << e.pr.smem_bytes << ",\"ntiles\":" << e.pr.ntiles << ",\"units\":" << e.pr.nunits
           << ",\"levels\":" << e.pr.n_levels << ",\"terms\":" << e.pr.n_terms << "}";
       if (e.kind == K_GEMM) o << ",\"alg_flops\":" << e.gm.alg_flops << ",\"alg_bytes\":" << e.gm.alg_bytes << ",\"splits\":" << e.gm.splits;
       if (e.kind == K_CONV_TC) o << ",\"alg_flops\":" << e.ctc.alg_flops << ",\"alg_bytes\":" << e.ctc.alg_bytes;

@@ -286,8 +286,22 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
   }
   if (!d.resident) {
     d.res_bytes = 0;
-    d.slot = kSlotA + 2 * kSlotB + (d.bias_mma ? 2 * kSlotC : 0);
-    d.stages = std::min(8, budget / d.slot);
+    // ring stages sized by the widest K atom of the group (an r atom of 128 rows, both units' Lhat
+    // halves of 64 rows, the bias atoms) and by one fconv F atom (Np/2 rows of 64 columns): rank-8
+    // concat members (DenseNet) take 12 KB stages, so 16 of them are in flight instead of 4 x 36 KB
+    int awmax = 16;
+    for (int jj = 0; jj < d.n_terms; ++jj) awmax = std::max(awmax, (int)d.term[jj].aw);
+    d.sa = 128 * awmax * 2;
+    d.sb = 64 * awmax * 2;
+    d.slot = std::max(d.sa + 2 * d.sb + (d.bias_mma ? 2 * kSlotC : 0), d.Np / 2 * 128);
+    d.slot = (d.slot + 1023) / 1024 * 1024;
+    const char* e = getenv("TEMCO_PAIR_FIXED_SLOTS");
+    if (e && atoi(e)) {
+      d.sa = kSlotA;
+      d.sb = kSlotB;
+      d.slot = kSlotA + 2 * kSlotB + (d.bias_mma ? 2 * kSlotC : 0);
+    }
+    d.stages = std::min(e && atoi(e) ? 8 : kPairMaxStages, budget / d.slot);
   }
   if (d.stages < 2 * kChunk) return false;
   d.smem_bytes = 1024 + d.res_bytes + d.stages * d.slot + 2 * kPBytes + d.bias_bytes + kOnesBytes + kBarBytes;
@@ -613,9 +627,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             EV(0);
             if (!notma) tma_load_2d_pair(sa, T->amap, fb, (int)op.y, row0);
             for (int q = 0; q < nu && !notma && !d.resident; ++q) {
-              tma_load_2d_pair(sa + kSlotA + q * kSlotB, T->wmap, fb, (int)op.y, (u0 + q) * kPairWu + (int)cta * 64);
+              tma_load_2d_pair(sa + d.sa + q * d.sb, T->wmap, fb, (int)op.y, (u0 + q) * kPairWu + (int)cta * 64);
               if (bia)
-                tma_load_2d_pair(sa + kSlotA + 2 * kSlotB + q * kSlotC, d.bmap, fb, 0,
+                tma_load_2d_pair(sa + d.sa + 2 * d.sb + q * kSlotC, d.bmap, fb, 0,
                                  (int)(op.x >> 28) * d.Cpad + (u0 + q) * kPairWu + (int)cta * 64);
             }
             PAIR_NEXT();
@@ -751,9 +765,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
                 const bool lvl0 = c0 == 0 && i == 0;   // first atom of the level
                 const bool bia = d.bias_mma && lvl0;
                 const uint32_t a_lo = a_lo0 + (uint32_t)st * slot16;
-                const uint32_t b0_lo = d.resident ? tk.z : a_lo + ((uint32_t)kSlotA >> 4);
-                const uint32_t b1_lo = b0_lo + (d.resident ? bq16 : ((uint32_t)kSlotB >> 4));
-                const uint32_t c0_lo = d.resident ? tk.w + pco : a_lo + ((uint32_t)(kSlotA + 2 * kSlotB) >> 4);
+                const uint32_t b0_lo = d.resident ? tk.z : a_lo + ((uint32_t)d.sa >> 4);
+                const uint32_t b1_lo = b0_lo + (d.resident ? bq16 : ((uint32_t)d.sb >> 4));
+                const uint32_t c0_lo = d.resident ? tk.w + pco : a_lo + ((uint32_t)(d.sa + 2 * d.sb) >> 4);
                 const uint32_t c1_lo = c0_lo + (d.resident ? cq16 : ((uint32_t)kSlotC >> 4));
                 mma2_atom2_w(d0, d1, a_lo, tk.y, b0_lo, b1_lo, c0_lo, c1_lo, ones_lo, hi16, idesc_t, (tk.x >> 16) & 0xFFu,
                              (uint32_t)nu, bia ? 1u : 0u, (lvl0 && !bia) ? 0u : 1u);

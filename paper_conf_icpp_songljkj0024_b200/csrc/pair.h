@@ -73,6 +73,7 @@ struct PairDesc {
   int32_t ycol[kPairMaxOuts + 1];        //   columns [ycol[k], ycol[k+1]) of the concatenated F
   int64_t F;                             // tc weight pool offset of F
   int32_t stages, slot, smem_bytes, bias_bytes;   // ring depth, stage bytes
+  int32_t sa, sb;                        // ring stage: r atom bytes, one unit's Lhat-half bytes (then bias atoms)
   // resident-weight mode (every Lhat / bias / F atom of this CTA's halves fits in SMEM next
   // to a deep ring): the weights are loaded once per CTA and the ring carries only the
   // reduced-input atoms r_j, so several tiles' loads are in flight (small-C groups)
