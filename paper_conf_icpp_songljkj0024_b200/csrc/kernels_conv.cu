@@ -14,6 +14,7 @@
 
 #include <algorithm>
 
+#include "tmap.h"
 #include "conv_tc.h"
 #include "tc_ptx.cuh"
 
@@ -111,16 +112,8 @@ bool conv_tc_lower(const IR& ir, int out, const std::map<int, Loc>& loc, std::ve
 }
 
 bool conv_tc_finalize(ConvTcDesc& d, uint16_t* tcw, std::string& err) {
-  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
-  if (!encode) {
-    cudaDriverEntryPointQueryResult q;
-    void* fn = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-      err = "cuTensorMapEncodeTiled unavailable";
-      return false;
-    }
-    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  }
+  const auto encode = tmap_encoder(err);
+  if (!encode) return false;
   const uint64_t Kp = (uint64_t)d.katoms * 64;
   cuuint64_t dims[2] = {Kp, (cuuint64_t)d.nsl * d.Np};
   cuuint64_t strides[1] = {Kp * 2};
@@ -138,13 +131,8 @@ bool conv_tc_finalize(ConvTcDesc& d, uint16_t* tcw, std::string& err) {
 
 bool conv_tc_finalize_x(ConvTcDesc& d, const void* x, std::string& err) {
   if (!d.tma) return true;
-  void* fn = nullptr;
-  cudaDriverEntryPointQueryResult q;
-  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-    err = "cuTensorMapEncodeTiled unavailable";
-    return false;
-  }
-  auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  const auto encode = tmap_encoder(err);
+  if (!encode) return false;
   cuuint64_t dims[4] = {(cuuint64_t)d.Cin, (cuuint64_t)d.W, (cuuint64_t)d.H, (cuuint64_t)d.N};
   cuuint64_t strides[3] = {(cuuint64_t)d.Cin * 2, (cuuint64_t)d.W * d.Cin * 2, (cuuint64_t)d.H * d.W * d.Cin * 2};
   cuuint32_t box[4] = {64, (cuuint32_t)(d.tw * d.s), (cuuint32_t)(d.th * d.s), (cuuint32_t)d.tn};

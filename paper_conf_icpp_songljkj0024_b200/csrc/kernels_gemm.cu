@@ -15,6 +15,7 @@
 #include <algorithm>
 #include <cstring>
 
+#include "tmap.h"
 #include "gemm.h"
 #include "tc_ptx.cuh"
 
@@ -66,16 +67,8 @@ bool gemm_lower(GemmDesc& d, const float* w, const std::vector<float>* bias, std
 }
 
 bool gemm_finalize(GemmDesc& d, char* arena, uint16_t* tcw, std::string& err) {
-  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
-  if (!encode) {
-    cudaDriverEntryPointQueryResult q;
-    void* fn = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-      err = "cuTensorMapEncodeTiled unavailable";
-      return false;
-    }
-    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  }
+  const auto encode = tmap_encoder(err);
+  if (!encode) return false;
   auto make = [&](unsigned char* dst, void* base, uint64_t inner, uint64_t outer, uint32_t box_outer) {
     cuuint64_t dims[2] = {inner, outer};
     cuuint64_t strides[1] = {inner * 2};

@@ -29,6 +29,7 @@
 #include <cstring>
 #include <set>
 
+#include "tmap.h"
 #include "chain_parse.h"
 #include "pair.h"
 #include "tc_ptx.cuh"
@@ -310,30 +311,13 @@ bool pair_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc
 
 bool pair_finalize(size_t n, const std::function<PairDesc*(size_t)>& get, char* arena, uint16_t* tcw,
                    std::string& err) {
-  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   bool any = false;
   for (size_t i = 0; i < n; ++i) any |= get(i) != nullptr;
   if (!any) return true;
-  if (!encode) {
-    cudaDriverEntryPointQueryResult q;
-    void* fn = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-      err = "cuTensorMapEncodeTiled unavailable";
-      return false;
-    }
-    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  }
+  const auto encode = tmap_encoder(err);
+  if (!encode) return false;
   auto make = [&](unsigned char* dst, void* base, uint64_t inner, uint64_t outer, uint32_t box_outer, int aw) {
-    cuuint64_t dims[2] = {inner, outer};
-    cuuint64_t strides[1] = {inner * 2};
-    cuuint32_t box[2] = {(cuuint32_t)aw, box_outer};
-    cuuint32_t es[2] = {1, 1};
-    const CUtensorMapSwizzle sw = aw == 64 ? CU_TENSOR_MAP_SWIZZLE_128B
-                                  : aw == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
-                                             : CU_TENSOR_MAP_SWIZZLE_32B;
-    return encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, base, dims, strides, box,
-                  es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    return tmap_2d_bf16(encode, dst, base, inner, outer, (uint32_t)aw, box_outer, tmap_swizzle_bf16(aw));
   };
   for (size_t i = 0; i < n; ++i) {
     PairDesc* d = get(i);

@@ -29,6 +29,8 @@
 #include <cmath>
 #include <set>
 
+#include "tmap.h"
+#include "chain_lower.h"
 #include "chain_parse.h"
 #include "tc.h"
 #include "tc_ptx.cuh"
@@ -40,28 +42,12 @@ namespace temco {
 // ===========================================================================
 namespace {
 using namespace chainp;
+using chainl::push_bf16;
+using chainl::push_f32;
+using chainl::to_bf16;
 
-uint16_t to_bf16(float f) {
-  uint32_t u;
-  memcpy(&u, &f, 4);
-  u += 0x7FFF + ((u >> 16) & 1);
-  return (uint16_t)(u >> 16);
-}
 
-int64_t push_bf16(std::vector<uint16_t>& pool, const std::vector<float>& v) {
-  while (pool.size() % 512) pool.push_back(0);   // 1024-byte aligned blocks (TMA base alignment)
-  int64_t off = (int64_t)pool.size();
-  for (float f : v) pool.push_back(to_bf16(f));
-  return off;
-}
 
-// fp32 vector padded with zeros to n entries, 16-byte aligned in the params pool
-int64_t push_f32(std::vector<float>& params, const std::vector<double>& v, int n) {
-  while (params.size() % 4) params.push_back(0.f);
-  const int64_t off = (int64_t)params.size();
-  for (int i = 0; i < n; ++i) params.push_back(i < (int)v.size() ? (float)v[i] : 0.f);
-  return off;
-}
 
 struct HUnit {
   int c, tg, nt;
@@ -277,76 +263,10 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
   d = TcChainDesc();
   d.C = C;
   d.Cc = kTcCc;
-  d.Cpad = (C + d.Cc - 1) / d.Cc * d.Cc;
-  d.nchunks = d.Cpad / d.Cc;
-  d.Nout = Nout;
-  d.Np = (Nout + 15) / 16 * 16;
-  d.npix = (int64_t)ir.batch * tn.H * tn.W;
-  d.nimg = ir.batch;
-  d.gap = gap ? 1 : 0;
-  d.hw = tn.H * tn.W;
-  d.Ho = tn.H;
-  d.Wo = tn.W;
-  d.spatial = mixed ? 1 : 0;
-  d.post = -1;
-  d.postsc = -1;
-  if (d.spatial) {
-    d.tw = std::min(tn.W, 128);
-    d.th = std::min(tn.H, 128 / d.tw);
-    d.tn = (d.th == tn.H && d.tw == tn.W) ? std::max(1, std::min(ir.batch, 128 / (tn.H * tn.W))) : 1;
-    d.nwb = (tn.W + d.tw - 1) / d.tw;
-    d.nhb = (tn.H + d.th - 1) / d.th;
-    d.nnb = (ir.batch + d.tn - 1) / d.tn;
-    d.mused = d.tw * d.th * d.tn;
-    d.ntiles = d.nnb * d.nhb * d.nwb;
-    d.rows_per_tile = 128;
-    if (gap) {
-      if (d.th != tn.H || d.tw != tn.W) return false;    // GAP needs whole images per tile
-      d.ipt = d.tn;
-    }
-  } else if (gap) {
-    d.ipt = 128 / d.hw;
-    d.rows_per_tile = d.ipt * d.hw;
-    d.ntiles = (ir.batch + d.ipt - 1) / d.ipt;
-  } else {
-    d.rows_per_tile = 128;
-    d.ntiles = (int)((d.npix + 127) / 128);
-  }
-  d.y = yl;
-  d.n_levels = (int)levels.size();
+  if (!chainl::tile_geometry(d, ir, tn, Nout, gap, mixed, yl, (int)levels.size())) return false;
   int64_t flops = 0, bytes = 0;
   int j = 0;
-  auto add_term = [&](const PTerm& t) -> bool {
-    const Node& lc = ir.nodes[t.lconv];
-    const int r = ir.oin[t.lconv][0];
-    const Node& rn = ir.nodes[r];
-    const int R = rn.C;
-    TcTerm& T = d.term[j++];
-    T.r = loc.at(r);
-    T.R = R;
-    T.aw = R <= 16 ? 16 : R <= 32 ? 32 : 64;      // box width ~ rank: no mostly-OOB boxes
-    T.Rp = (R + T.aw - 1) / T.aw * T.aw;
-    T.Rw = (R + 7) / 8 * 8;
-    T.c0 = t.c0;
-    T.C = lc.C;
-    T.Hin = rn.H;
-    T.Win = rn.W;
-    T.tk = t.tk;
-    T.ts = t.ts;
-    T.tp = t.tp;
-    T.cfirst = t.c0 / d.Cc;
-    T.nhit = (t.c0 + lc.C - 1) / d.Cc - T.cfirst + 1;
-    std::vector<float> w((size_t)d.Cpad * T.Rw, 0.f);
-    for (int c = 0; c < lc.C; ++c)
-      for (int k = 0; k < R; ++k)
-        w[(size_t)(t.c0 + c) * T.Rw + k] = (float)(t.scale[c] * (*lc.w)[(size_t)c * R + k]);
-    T.w = push_bf16(tcw, w);
-    const int64_t in_pix = (int64_t)ir.batch * rn.H * rn.W;
-    flops += in_pix * 2LL * lc.C * R;
-    bytes += in_pix * 2LL * R;
-    if (d.spatial && (d.tw * T.ts > 256 || d.th * T.ts > 256)) return false;
-    return true;
-  };
+  auto add_term = [&](const PTerm& t) -> bool { return chainl::add_term(d, d.term[j++], ir, loc, tcw, t, flops, bytes); };
   for (int l = 0; l < d.n_levels; ++l) {
     const PLevel& L = levels[l];
     d.relu[l] = L.relu ? 1 : L.silu ? 2 : 0;
@@ -522,31 +442,14 @@ bool tc_lower_chain(const IR& ir, const Step& s, const std::map<int, Loc>& loc, 
 
 bool tc_finalize(size_t n, const std::function<TcChainDesc*(size_t)>& get, char* arena, uint16_t* tcw,
                  std::string& err) {
-  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   bool any = false;
   for (size_t i = 0; i < n; ++i) any |= get(i) != nullptr;
   if (!any) return true;
-  if (!encode) {
-    cudaDriverEntryPointQueryResult q;
-    void* fn = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-      err = "cuTensorMapEncodeTiled unavailable";
-      return false;
-    }
-    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  }
-  auto swz = [](int aw) {
-    return aw == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : aw == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
-  };
+  const auto encode = tmap_encoder(err);
+  if (!encode) return false;
+  auto swz = [](int aw) { return tmap_swizzle_bf16(aw); };
   auto make = [&](unsigned char* dst, void* base, uint64_t inner, uint64_t outer, uint32_t box_outer, int aw = 64) {
-    cuuint64_t dims[2] = {inner, outer};
-    cuuint64_t strides[1] = {inner * 2};
-    cuuint32_t box[2] = {(cuuint32_t)aw, box_outer};
-    cuuint32_t es[2] = {1, 1};
-    CUresult r = encode(reinterpret_cast<CUtensorMap*>(dst), CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, base, dims, strides,
-                        box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz(aw),
-                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    return r == CUDA_SUCCESS;
+    return tmap_2d_bf16(encode, dst, base, inner, outer, (uint32_t)aw, box_outer, swz(aw));
   };
   auto make4 = [&](unsigned char* dst, void* base, const TcChainDesc* d, const TcTerm& t) {
     cuuint64_t dims[4] = {(cuuint64_t)t.R, (cuuint64_t)t.Win, (cuuint64_t)t.Hin, (cuuint64_t)d->nimg};

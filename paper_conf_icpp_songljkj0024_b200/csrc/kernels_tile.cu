@@ -18,6 +18,7 @@
 
 #include <algorithm>
 
+#include "tmap.h"
 #include "tc_ptx.cuh"
 #include "tile.h"
 
@@ -138,16 +139,8 @@ bool tile_conv_lower(const ConvDesc& c, const float* w, std::vector<uint16_t>& t
 }
 
 bool tile_conv_finalize(TileConvDesc& d, const char* arena, std::string& err) {
-  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
-  if (!encode) {
-    void* fn = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess || !fn) {
-      err = "cuTensorMapEncodeTiled unavailable";
-      return false;
-    }
-    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  }
+  const auto encode = tmap_encoder(err);
+  if (!encode) return false;
   const bool sub = d.kh == 1 && d.kw == 1;
   // view (cw * C, W / cw, H, N): an inner row = cw consecutive pixels of an image row
   cuuint64_t dims[4] = {(cuuint64_t)d.cw * d.C, (cuuint64_t)(d.W / d.cw), (cuuint64_t)d.H, (cuuint64_t)d.N};

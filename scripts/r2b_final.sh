@@ -1,7 +1,7 @@
 # round-2 final artifacts: GPU suite, smoke, bench lines (every config, N=1), ablation + SiLU lines,
-# compute-sanitizer, ncu launch lists (+ DRAM bytes) of every config, ncu --set full of top tc_pair groups
+# ncu launch lists (+ DRAM bytes) of every config, ncu --set full of top tc_pair groups
 set -x
-O=gpurun_out/fin
+O=gpurun_out/fin2
 mkdir -p $O
 timeout 1500 python -m pytest tests -m gpu -q --durations=5 > $O/gpu_tests.log 2>&1; tail -3 $O/gpu_tests.log
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; tail -2 $O/smoke.log
@@ -22,14 +22,4 @@ timeout 600 ncu --set full --clock-control none --import-source on -k regex:pair
 i=$(python scripts/ncu_group.py resnet50 211 tc_pair)
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:pair_chain -s $i -c 1 -o $O/ncu_pair211 python scripts/ncu_target.py resnet50 > /dev/null 2>&1
 timeout 600 ncu --set full --clock-control none --import-source on -k regex:tile_conv -s 0 -c 1 -o $O/ncu_tile0 python scripts/ncu_target.py resnet50 > /dev/null 2>&1
-CS=/usr/local/cuda/bin/compute-sanitizer
-for tool in memcheck racecheck synccheck; do
-  : > $O/sanitize_$tool.log
-  for g in c1 t2_3 t3 t4 resnet50_s vgg16_s alexnet_s; do
-    echo "=== $tool $g" >> $O/sanitize_$tool.log
-    timeout 900 $CS --tool $tool --print-limit 20 python scripts/sanitize_run.py $g >> $O/sanitize_$tool.log 2>&1
-    echo "rc=$?" >> $O/sanitize_$tool.log
-  done
-done
-grep -E "ERROR SUMMARY|rc=" $O/sanitize_*.log | sort | uniq -c | head -30
 ls $O
