@@ -99,9 +99,9 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
       const int k = ks * 16 + 2 * tq + 8 * h;           // even: the pair (k, k+1) shares its kernel row
       const int kr = k / g.rowK, j = k - kr * g.rowK;
       if constexpr (kBs) {
-        if (gq == 0) os[(ks * 2 + h) * 4 + tq] = kr < d.kh ? kr * g.rowlen + j : 0;
+        if (gq == 0) os[(ks * 2 + h) * 4 + tq] = kr < d.kh ? 2 * (kr * g.rowlen + j) : 0;   // bytes
       } else {
-        off[ks][h] = kr < d.kh ? kr * g.rowlen + j : 0;
+        off[ks][h] = kr < d.kh ? 2 * (kr * g.rowlen + j) : 0;   // bytes (even element offsets)
       }
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt) {
@@ -246,13 +246,14 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
     const int n = tile / (tiles_w * tiles_h);
     const int h0 = (tile / tiles_w) % tiles_h * g.TH, w0 = tile % tiles_w * g.TW;
     if (tile + (int)gridDim.x < ntiles) load(tile + gridDim.x);   // in flight during the MMAs
-    const uint32_t* xw = reinterpret_cast<const uint32_t*>(buf);
     // ---- MPW m-tiles per warp: m-tile gm covers output row gm / (TW / 16), 16 columns
 #pragma unroll 1
     for (int gm = warp * g.MPW; gm < (warp + 1) * g.MPW; ++gm) {
-      const int orow = gm / (g.TW / 16), ocol = gm % (g.TW / 16) * 16;
-      const int b0 = (orow * d.sh) * g.rowlen + ((ocol + gq) * d.sw) * g.Cp;     // pixel rows gq, gq + 8
-      const int b1 = b0 + 8 * d.sw * g.Cp;
+      // m-tile gm: output row gm / (TW / 16), columns 16 (gm % (TW / 16)) .. (TW is 16 or 32)
+      const int orow = g.TW == 32 ? gm >> 1 : gm, ocol = g.TW == 32 ? (gm & 1) * 16 : 0;
+      // byte addresses of the fragment rows gq, gq + 8 (element offsets are even: 4-byte aligned words)
+      const uint8_t* xb0 = reinterpret_cast<const uint8_t*>(buf) + 2 * ((orow * d.sh) * g.rowlen + ((ocol + gq) * d.sw) * g.Cp);
+      const uint8_t* xb1 = xb0 + 2 * 8 * d.sw * g.Cp;
       float acc[NT][4];
 #pragma unroll
       for (int nt = 0; nt < NT; ++nt) {
@@ -270,10 +271,10 @@ __global__ void __launch_bounds__(kStThreads, 2) conv_stem_kernel(ConvDesc d, St
           o0 = off[ks][0];
           o1 = off[ks][1];
         }
-        a[0] = xw[(b0 + o0) >> 1];
-        a[1] = xw[(b1 + o0) >> 1];
-        a[2] = xw[(b0 + o1) >> 1];
-        a[3] = xw[(b1 + o1) >> 1];
+        a[0] = *reinterpret_cast<const uint32_t*>(xb0 + o0);
+        a[1] = *reinterpret_cast<const uint32_t*>(xb1 + o0);
+        a[2] = *reinterpret_cast<const uint32_t*>(xb0 + o1);
+        a[3] = *reinterpret_cast<const uint32_t*>(xb1 + o1);
 #pragma unroll
         for (int nt = 0; nt < NT; ++nt) {
           if constexpr (kBs) {
