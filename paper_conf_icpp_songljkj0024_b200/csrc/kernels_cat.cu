@@ -544,12 +544,18 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
   const CatTerm& M = d.term[d.n_plain];                 // the pooled member's (single) term
   const int PR = (kPcTH - 1) * PS + PK, PC = (kPcTW - 1) * PS + PK;
   // member restore fragments and bias (registers for the whole kernel)
-  uint32_t wm[8][2];
-  float mb[8][2];
+  // 3x3 windows: the member's restore weights are ldmatrix'd from SMEM per use (holding them in 16
+  // registers for the whole kernel spilled: local-memory loads and ~200 register moves per tile);
+  // 2x2 windows (VGG) keep them in registers (measured faster there)
+  constexpr bool kWmReg = PK == 2;
+  uint32_t wm[kWmReg ? 8 : 1][2];
+  if constexpr (kWmReg) {
 #pragma unroll
-  for (int np = 0; np < 4; ++np)
-    ldsm_x4(sbase + (uint32_t)((M.w + (np * 16 + (lq >> 1) * 8 + lr) * M.rs + (lq & 1) * 8) * 2), wm[2 * np][0],
-            wm[2 * np][1], wm[2 * np + 1][0], wm[2 * np + 1][1]);
+    for (int np = 0; np < 4; ++np)
+      ldsm_x4(sbase + (uint32_t)((M.w + (np * 16 + (lq >> 1) * 8 + lr) * M.rs + (lq & 1) * 8) * 2), wm[2 * np][0],
+              wm[2 * np][1], wm[2 * np + 1][0], wm[2 * np + 1][1]);
+  }
+  float mb[8][2];
 #pragma unroll
   for (int nt = 0; nt < 8; ++nt) {
     const float2 b = *reinterpret_cast<const float2*>(fb + d.mbias + nt * 8 + 2 * t4);
@@ -587,7 +593,14 @@ __global__ void __launch_bounds__(32 * kPcWarps, 2) mma_poolcat_kernel(const __g
 #pragma unroll
       for (int nt = 0; nt < 8; ++nt) {
         float D[4] = {mb[nt][0], mb[nt][1], mb[nt][0], mb[nt][1]};
-        mma16816(D, a[q], wm[nt][0], wm[nt][1]);
+        uint32_t w0, w1;   // n-tile nt: rows 8 nt .. of the member's Lhat, k halves 0 / 1
+        if constexpr (kWmReg) {
+          w0 = wm[nt][0];
+          w1 = wm[nt][1];
+        } else {
+          ldsm_x2(sbase + (uint32_t)((M.w + (nt * 8 + lr) * M.rs + (lq & 1) * 8) * 2), w0, w1);
+        }
+        mma16816(D, a[q], w0, w1);
         if (d.mrelu) {
 #pragma unroll
           for (int i = 0; i < 4; ++i) D[i] = fmaxf(D[i], 0.f);
