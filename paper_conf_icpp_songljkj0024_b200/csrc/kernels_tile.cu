@@ -189,7 +189,7 @@ __device__ __forceinline__ int fdiv(int q, uint32_t m, uint32_t sh) {
   return (int)((__umulhi((uint32_t)q, m) + (uint32_t)q) >> sh);
 }
 
-template <int NT2>   // pairs of n-tiles (output channels / 16, rounded up)
+template <int NT2, int NTU>   // pairs of n-tiles (Kp / 16); n-tiles used (K / 8: 1 for the 8-channel cores)
 __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel(const __grid_constant__ TileConvDesc d, RunPtrs p,
                                                                   const uint16_t* __restrict__ tcw) {
   extern __shared__ uint8_t smem_raw[];
@@ -265,9 +265,9 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
   const uint32_t smask = d.swz == 0 ? 0u : (1u << d.swz) - 1u;
   const int pxt = d.TH * d.TW, npx = d.TN * pxt, nmt = (npx + 15) / 16, npair = (nmt + 1) / 2;
   __nv_bfloat16* y = reinterpret_cast<__nv_bfloat16*>(const_cast<void*>(loc_ptr(d.y, p)));
-  float bias[2 * NT2][2];
+  float bias[NTU][2];
 #pragma unroll
-  for (int nt = 0; nt < 2 * NT2; ++nt)
+  for (int nt = 0; nt < NTU; ++nt)
 #pragma unroll
     for (int e = 0; e < 2; ++e) {
       const int col = nt * 8 + 2 * t4 + e;
@@ -297,11 +297,11 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
         const int pn = fdiv(q, d.mpx, d.spx), rem = q - pn * pxt, py = fdiv(rem, d.mtw, d.stw), px = rem - py * d.TW;
         pbase[j] = (pn * d.FH + py * she) * d.RP + px * swe + xr;   // + the box's start offset
       }
-      float acc[2][2 * NT2][4];
+      float acc[2][NTU][4];
 #pragma unroll
       for (int j = 0; j < 2; ++j)
 #pragma unroll
-        for (int nt = 0; nt < 2 * NT2; ++nt) {
+        for (int nt = 0; nt < NTU; ++nt) {
           acc[j][nt][0] = acc[j][nt][2] = bias[nt][0];
           acc[j][nt][1] = acc[j][nt][3] = bias[nt][1];
         }
@@ -315,14 +315,23 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
           off ^= ((off >> 7) & smask) << 4;   // the TMA swizzle of 32 / 64 / 128-byte rows
           ldsm4(fbase + off, a[j]);
         }
+        if constexpr (NTU == 1) {   // one n-tile (K = 8): its two k halves only
+          uint32_t b0, b1;
+          asm volatile("ldmatrix.sync.aligned.m8n8.x2.shared.b16 {%0, %1}, [%2];"
+                       : "=r"(b0), "=r"(b1)
+                       : "r"(wbase + (uint32_t)(ks * 2 * d.Kp * 16) + boff_lane));
 #pragma unroll
-        for (int np = 0; np < NT2; ++np) {
-          uint32_t bb[4];
-          ldsm4(wbase + (uint32_t)((ks * 2 * d.Kp + np * 16) * 16) + boff_lane, bb);
+          for (int j = 0; j < 2; ++j) mma16816(acc[j][0], a[j], b0, b1);
+        } else {
 #pragma unroll
-          for (int j = 0; j < 2; ++j) {
-            mma16816(acc[j][2 * np], a[j], bb[0], bb[1]);
-            mma16816(acc[j][2 * np + 1], a[j], bb[2], bb[3]);
+          for (int np = 0; np < NT2; ++np) {
+            uint32_t bb[4];
+            ldsm4(wbase + (uint32_t)((ks * 2 * d.Kp + np * 16) * 16) + boff_lane, bb);
+#pragma unroll
+            for (int j = 0; j < 2; ++j) {
+              mma16816(acc[j][2 * np], a[j], bb[0], bb[1]);
+              mma16816(acc[j][2 * np + 1], a[j], bb[2], bb[3]);
+            }
           }
         }
       }
@@ -337,7 +346,7 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
           if (on >= d.N || oh >= d.Ho || ow >= d.Wo) continue;
           __nv_bfloat16* yp = y + (((int64_t)on * d.Ho + oh) * d.Wo + ow) * d.K + 2 * t4;
 #pragma unroll
-          for (int nt = 0; nt < 2 * NT2; ++nt)
+          for (int nt = 0; nt < NTU; ++nt)
             if (nt * 8 < d.K)
               *reinterpret_cast<uint32_t*>(yp + nt * 8) = pk2(acc[j][nt][2 * hf], acc[j][nt][2 * hf + 1]);
         }
@@ -346,31 +355,32 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
   }
 }
 
-template <int NT2>
+template <int NT2, int NTU>
 void launch_t(const TileConvDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
   static bool configured = false;
   static int sms = 148;
   if (!configured) {
-    cudaFuncSetAttribute(tile_conv_kernel<NT2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(tile_conv_kernel<NT2, NTU>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     configured = true;
   }
   int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tile_conv_kernel<NT2>, kTcThreads, d.smem_bytes);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, tile_conv_kernel<NT2, NTU>, kTcThreads, d.smem_bytes);
   const int grid = std::min(d.ntiles, sms * std::max(per_sm, 1));
-  launch_pdl(tile_conv_kernel<NT2>, dim3((unsigned)grid), dim3(kTcThreads), (size_t)d.smem_bytes, s, d, p, tcw);
+  launch_pdl(tile_conv_kernel<NT2, NTU>, dim3((unsigned)grid), dim3(kTcThreads), (size_t)d.smem_bytes, s, d, p, tcw);
 }
 
 }  // namespace
 
 void launch_tile_conv(const TileConvDesc& d, const uint16_t* tcw, const RunPtrs& p, cudaStream_t s) {
+  if (d.K == 8) return launch_t<1, 1>(d, tcw, p, s);
   switch (d.Kp / 16) {
-    case 1: launch_t<1>(d, tcw, p, s); break;
-    case 2: launch_t<2>(d, tcw, p, s); break;
-    case 3: launch_t<3>(d, tcw, p, s); break;
-    default: launch_t<4>(d, tcw, p, s); break;
+    case 1: launch_t<1, 2>(d, tcw, p, s); break;
+    case 2: launch_t<2, 4>(d, tcw, p, s); break;
+    case 3: launch_t<3, 6>(d, tcw, p, s); break;
+    default: launch_t<4, 8>(d, tcw, p, s); break;
   }
 }
 
