@@ -103,7 +103,7 @@ bool tile_conv_lower(const ConvDesc& c, const float* w, std::vector<uint16_t>& t
   d.buf_bytes = (d.box_bytes + 64 + 1023) / 1024 * 1024;   // + zeroed slack: the half k-step past C
   d.Kp = (c.K + 15) / 16 * 16;
   d.w_bytes = d.nks * 2 * d.Kp * 16;
-  d.smem_bytes = 1024 + kTcBufs * d.buf_bytes + d.w_bytes + 64 + d.nks * 2 * 8;
+  d.smem_bytes = 1024 + kTcBufs * d.buf_bytes + d.w_bytes + 64 + d.nks * 2 * 8 + kTcBufs * 16;
   auto magic = [](int dv, uint32_t& m, uint32_t& sh) {   // q / dv = (umulhi(q, m) + q) >> sh
     sh = 0;
     while ((1u << sh) < (uint32_t)dv) ++sh;
@@ -198,6 +198,7 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
   uint64_t* full = reinterpret_cast<uint64_t*>(wsm + d.w_bytes);   // [kTcBufs] TMA bytes landed
   uint64_t* empty = full + kTcBufs;                                // [kTcBufs] the compute warps are done
   int2* ktab = reinterpret_cast<int2*>(full + 8);   // per (k-step, k half): footprint pixel offset, byte offset
+  int4* tinfo = reinterpret_cast<int4*>(ktab + 2 * d.nks);   // per buffer: its tile's n0, oh0, ow0, column shift
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int g = lane >> 2, t4 = lane & 3;
   const bool sub = d.kh == 1 && d.kw == 1;
@@ -249,12 +250,16 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
         if (it >= kTcBufs) mbar_wait(&empty[b], (uint32_t)(it / kTcBufs - 1) & 1u);
         const int tn = tile / tpi, th = (tile / d.tiles_w) % d.tiles_h, tw = tile % d.tiles_w;
         if (d.dbg & 2) {
+          const int x0 = tw * d.TW * d.sw - d.pw;
+          tinfo[b] = make_int4(tn * d.TN, th * d.TH, tw * d.TW, x0 - (x0 >= 0 ? x0 / d.cw : -((d.cw - 1 - x0) / d.cw)) * d.cw);
           mbar_arrive(&full[b]);
           continue;
         }
-        mbar_expect_tx(&full[b], (uint32_t)d.box_bytes);
         const int x0 = tw * d.TW * d.sw - d.pw;   // first footprint column; its inner row (floor)
         const int xg = x0 >= 0 ? x0 / d.cw : -((d.cw - 1 - x0) / d.cw);
+        // the tile's coordinates for the compute warps (published by the barrier's arrive: release)
+        tinfo[b] = make_int4(tn * d.TN, th * d.TH, tw * d.TW, x0 - xg * d.cw);
+        mbar_expect_tx(&full[b], (uint32_t)d.box_bytes);
         tma_load_4d(smem + b * d.buf_bytes, d.xmap, &full[b], 0, xg, th * d.TH * d.sh - d.ph, tn * d.TN);
       }
     }
@@ -281,9 +286,8 @@ __global__ void __launch_bounds__(kTcThreads, NT2 >= 3 ? 1 : 2) tile_conv_kernel
     const int b = it % kTcBufs;
     mbar_wait(&full[b], (uint32_t)(it / kTcBufs) & 1u);
     const uint32_t fbase = smem_u32(smem + b * d.buf_bytes);
-    const int tn = tile / tpi, th = (tile / d.tiles_w) % d.tiles_h, tw = tile % d.tiles_w;
-    const int n0 = tn * d.TN, oh0 = th * d.TH, ow0 = tw * d.TW;
-    const int x0 = ow0 * d.sw - d.pw, xr = x0 - (x0 >= 0 ? x0 / d.cw : -((d.cw - 1 - x0) / d.cw)) * d.cw;
+    const int4 ti = tinfo[b];   // written by the producer before the barrier's arrive
+    const int n0 = ti.x, oh0 = ti.y, ow0 = ti.z, xr = ti.w;
     int pr = warp - pstart % kTcWarps;
     if (pr < 0) pr += kTcWarps;
     if (d.dbg & 1) pr = npair;
