@@ -380,10 +380,6 @@ constexpr int kThreads = 32 * kWarps;
 constexpr int kEpiWarp0 = 0, kProdWarp = 16, kMmaWarp = 17;
 constexpr int kEpiWarps = 16;
 
-__device__ __forceinline__ int atom_steps(const PairTerm& T, int a) {   // K=16 steps of atom a
-  return min(T.aw / 16, (T.R - a * T.aw + 15) / 16);
-}
-
 __device__ __forceinline__ void add2(float& a0, float& a1, float b0, float b1) {   // packed FADD2
   asm("{\n.reg .b64 x, y;\nmov.b64 x, {%0, %1};\nmov.b64 y, {%2, %3};\nadd.rn.f32x2 x, x, y;\nmov.b64 {%0, %1}, x;\n}\n"
       : "+f"(a0), "+f"(a1)
@@ -798,6 +794,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     const uint32_t oempty_c = mapa_shared(smem_u32(out_empty), 0);
 
     int gi = 0, np = 0, it = 0;   // gi: (unit, level) accumulator items consumed
+    int eb = 0;                   // buffer of item gi (gi mod NB)
+    uint32_t ephase = 0;          // per buffer: parity of its next acc_full phase
+    const uint32_t aempty_c = mapa_shared(smem_u32(&acc_empty[0]), 0);   // leader's acc_empty[0]
     EVDECL();
     const bool ev0 = warp == kEpiWarp0 && lane == 0;
     // out tile of tile `oit` (pixel row orow): TMEM columns [128 NB, 128 NB + Np) -> bf16 -> y.
@@ -841,8 +840,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             if (qq < nu) {
               const int act = d.mixed_act ? (int)d.actg[l * d.ngroups + (2 * pp + qq) * (kPairWu / 32) + g] : d.act[l];
               const float* bl = d.bias_mma ? nullptr : sbias + l * d.Cpad + (2 * pp + qq) * kPairWu + g * 32;
-              const int item = gi + qq, b = item % NB;
-              PAIR_EPI_WAIT(&acc_full[b], (uint32_t)(item / NB) & 1u);
+              // item gi + qq: buffer (gi + qq) mod NB and its use parity, kept incrementally (no division)
+              int b = eb + qq;
+              if (b >= NB) b -= NB;
+              PAIR_EPI_WAIT(&acc_full[b], (ephase >> b) & 1u);
+              ephase ^= 1u << b;
               if (ev0) EV(qq ? 8 : 5);
               tc_fence_after();
               uint32_t v[32];
@@ -855,13 +857,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
               tmem_ld32(tbase + lane_off + (uint32_t)(b * kPairWu + g * 32), v);
               tmem_wait_ld();
               tc_fence_before();
-              warp_arrive_cluster(mapa_shared(smem_u32(&acc_empty[b]), 0));
+              warp_arrive_cluster(aempty_c + 8u * (uint32_t)b);
               if (ev0 && !qq) EV(6);
               level_math<SILU>(qq ? t1 : t0, v, l == 0, act, bl);
               if (ev0) EV(qq ? 9 : 7);
             }
           }
           gi += nu;
+          eb += nu;
+          if (eb >= NB) eb -= NB;
           if (l == d.flag && pp == 0 && pend_it >= 0) {
             drain_out(pend_it, pend_row);
             pend_it = -1;
