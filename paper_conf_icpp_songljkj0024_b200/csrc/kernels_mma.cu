@@ -543,15 +543,31 @@ __global__ void __launch_bounds__(32 * kLeanWarps, 1) mma_lean_kernel(const __gr
   if (cur.blk < d.nblocks) lean_set_block(d, cur, g);
   LeanCursor pf = cur;
   uint32_t a[KS][4], an[KS][4], ann[KS][4];
+  // unpooled groups: a block's later 64-channel chunks read the same A rows -- reuse the
+  // fragments of the unit before instead of reloading them
   if (pf.blk < d.nblocks) lean_load_a<KS>(a, d, r, pf, T.R, g, t4);
   advance(pf);
-  if (pf.blk < d.nblocks) lean_load_a<KS>(an, d, r, pf, T.R, g, t4);
+  if (!d.pool && pf.ch > 0) {
+#pragma unroll
+    for (int ks = 0; ks < KS; ++ks)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) an[ks][i] = a[ks][i];
+  } else if (pf.blk < d.nblocks) {
+    lean_load_a<KS>(an, d, r, pf, T.R, g, t4);
+  }
   advance(pf);
   float O[NO][4];
   float run[8][4];
   const float sc = d.pool == 2 ? 1.f / (float)d.taps : 1.f;
   for (; cur.blk < d.nblocks; advance(cur)) {
-    if (pf.blk < d.nblocks) lean_load_a<KS>(ann, d, r, pf, T.R, g, t4);
+    if (!d.pool && pf.ch > 0) {
+#pragma unroll
+      for (int ks = 0; ks < KS; ++ks)
+#pragma unroll
+        for (int i = 0; i < 4; ++i) ann[ks][i] = an[ks][i];
+    } else if (pf.blk < d.nblocks) {
+      lean_load_a<KS>(ann, d, r, pf, T.R, g, t4);
+    }
     advance(pf);
     const int c0 = cur.ch * 64;
     if (cur.ch == 0 && cur.tap == 0) {
