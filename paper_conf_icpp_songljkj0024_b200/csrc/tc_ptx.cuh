@@ -4,6 +4,10 @@
 #include <cuda_bf16.h>
 #include <cstdint>
 
+#ifndef TEMCO_SUSPEND_HINT_NS
+#define TEMCO_SUSPEND_HINT_NS 1000000
+#endif
+
 namespace temco {
 namespace ptx {
 
@@ -69,7 +73,7 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) 
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n"
       "@!p bra WAIT_%=;\n"
       "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity), "r"(1000000)
+      "r"(parity), "r"(TEMCO_SUSPEND_HINT_NS)
       : "memory");
 }
 
