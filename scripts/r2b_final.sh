@@ -1,7 +1,7 @@
 # round-2 final artifacts: GPU suite, smoke, bench lines (every config, N=1), ablation + SiLU lines,
 # ncu launch lists (+ DRAM bytes) of every config, ncu --set full of top tc_pair groups
 set -x
-O=gpurun_out/fin4
+O=gpurun_out/fin5
 mkdir -p $O
 timeout 1500 python -m pytest tests -m gpu -q --durations=5 > $O/gpu_tests.log 2>&1; tail -3 $O/gpu_tests.log
 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; tail -2 $O/smoke.log
